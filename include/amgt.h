@@ -1,0 +1,269 @@
+/*
+ * amgt.h — C ABI of libamgt.so, the B200 (sm_100a) implementation of AmgT's hot path
+ * (Lu et al., "AmgT: Algebraic Multigrid Solver on Tensor Cores", SC'24).
+ * Citations "Lnnn" are /root/reference/PAPER.md line numbers; "Rnn" are the readings
+ * of ambiguous passages listed in DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *   - Array pointers are DEVICE pointers unless the name ends in _host.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     Calls are stream-ordered; only functions documented as "syncs" block the host.
+ *   - Inputs are never modified.  No exception crosses the ABI: every call returns an
+ *     amgt_status; amgt_last_error() gives a thread-local message for the last failure.
+ *     On error, outputs are left unallocated (or freed) and the status is returned.
+ *   - Memory the library returns in an amgt_mbsr is obtained from the caller's
+ *     amgt_allocator (NULL allocator = cudaMallocAsync/cudaFreeAsync on `stream`) and is
+ *     released with amgt_mbsr_free using the same allocator.
+ *   - Indices: column indices int32, pointers/counters int64 (R26).
+ *   - Determinism: structure is always identical for identical inputs; values are
+ *     deterministic except where a function says otherwise.
+ */
+#ifndef AMGT_H
+#define AMGT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#pragma GCC visibility push(default)
+#endif
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define AMGT_VERSION_MAJOR 0
+#define AMGT_VERSION_MINOR 1
+
+typedef enum {
+    AMGT_OK = 0,
+    AMGT_ERR_ARG = 1,         /* bad argument: NULL, negative size, A.n != B.m, precision mismatch */
+    AMGT_ERR_FORMAT = 2,      /* CSR input with unsorted/duplicate/out-of-range columns or bad row_ptr */
+    AMGT_ERR_ALLOC = 3,       /* the allocator returned NULL */
+    AMGT_ERR_CUDA = 4,        /* a CUDA runtime call or kernel launch failed */
+    AMGT_ERR_NCCL = 5,        /* reserved for the distributed path */
+    AMGT_ERR_RANGE = 6,       /* a value does not fit the target precision (FP16 overflow, R18) */
+    AMGT_ERR_UNSUPPORTED = 7  /* valid request this build does not implement */
+} amgt_status;
+
+typedef enum { AMGT_FP64 = 0, AMGT_FP32 = 1, AMGT_FP16 = 2 } amgt_prec;
+
+/* Stream-ordered allocator supplied by the caller (e.g. the torch caching allocator). */
+typedef struct {
+    void* (*alloc)(size_t bytes, void* stream, void* ctx);
+    void (*free)(void* p, size_t bytes, void* stream, void* ctx);
+    void* ctx;
+} amgt_allocator;
+
+/*
+ * mBSR matrix (§IV.B; Fig. 3 caption L120).  A two-level structure:
+ *   blc_ptr[blc_row+1]   offset of the first tile of each block row (int64, non-decreasing)
+ *   blc_idx[blc_num]     tile column of each tile, strictly increasing within a block row
+ *                        (the paper's blcIdx / BlcCid)
+ *   blc_map[blc_num]     16-bit bitmap, one unsigned short per tile (L122): bit 4*r+c set
+ *                        <=> entry (4I+r, 4J+c) structurally present (R1); never 0 (R5)
+ *   blc_val[16*blc_num]  dense 4x4 values, row-major within a tile (index 4r+c), exactly
+ *                        +0.0 where the bit is clear (R2); element type given by `prec`
+ * Tiles are 4x4 because tensor-core shapes are multiples of 4 (L116).
+ * blc_row = ceil(m/4), blc_col = ceil(n/4); bits outside m x n are never set (R25).
+ * `own` and `aux` are library-managed (zero-initialise the struct before first use).
+ */
+typedef struct {
+    int64_t m, n;
+    int64_t blc_row, blc_col, blc_num;
+    int64_t* blc_ptr;
+    int32_t* blc_idx;
+    uint16_t* blc_map;
+    void* blc_val;
+    amgt_prec prec;
+    uint32_t own;      /* bit0: structure arrays owned, bit1: values owned */
+    void* aux;         /* library-owned analysis (SpMV plan); NULL until amgt_spmv_analyze */
+} amgt_mbsr;
+
+const char* amgt_last_error(void);
+const char* amgt_version(void);
+
+/*
+ * CSR -> mBSR conversion (CSR2MBSR, L234, L262; Fig. 6 step 4).  For each block row I
+ * the tile columns are the sorted union of col/4 over CSR rows 4I..4I+3; each entry
+ * sets bit 4*(r%4)+(c%4) and stores its value at 16*t + bit; explicit zeros keep their
+ * bit (R3).  Values are rounded once, directly from FP64, to `prec` (R18).
+ *   row_ptr[m+1] int64, col_idx[nnz] int32 (sorted, unique per row, in [0, n)),
+ *   val[nnz] float64.   out: filled, structure+values allocated with `al`.
+ * Errors: AMGT_ERR_FORMAT for unsorted/duplicate/out-of-range columns or a row_ptr that
+ * is not non-decreasing from 0 to nnz; AMGT_ERR_RANGE if prec = FP16 and |v| > 65504.
+ * Syncs once (to size the tile arrays).
+ */
+amgt_status amgt_csr_to_mbsr(int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr, const int32_t* col_idx,
+                             const double* val, amgt_prec prec, amgt_mbsr* out, const amgt_allocator* al,
+                             void* stream);
+
+/* Number of structural nonzeros (sum of popcounts of blc_map, P5).  Syncs. */
+amgt_status amgt_mbsr_nnz(const amgt_mbsr* A, int64_t* nnz_host, void* stream);
+
+/*
+ * mBSR -> CSR (MBSR2CSR, L234, L262; Fig. 6 step 5).  Per scalar row, tiles in column
+ * order, set bits of the row's nibble in column order.  Caller allocates row_ptr[m+1],
+ * col_idx[nnz], val[nnz] (float64) with nnz from amgt_mbsr_nnz.  Values widen exactly.
+ */
+amgt_status amgt_mbsr_to_csr(const amgt_mbsr* A, int64_t* row_ptr, int32_t* col_idx, double* val, void* stream);
+
+/*
+ * Per-level precision cast (L266: "data precision conversions ... completed before
+ * calling the kernels").  out shares in's structure arrays (not owned) and gets new
+ * values of precision `to`, rounded to nearest even directly from the source (R18).
+ * Errors: AMGT_ERR_RANGE if to = FP16 and a value overflows (detected on device; the
+ * call then syncs to report it), AMGT_ERR_ARG if `to` is wider than in->prec.
+ */
+amgt_status amgt_mbsr_cast(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, const amgt_allocator* al,
+                           void* stream);
+
+/* Release whatever A owns (structure, values, aux) and zero the struct. */
+amgt_status amgt_mbsr_free(amgt_mbsr* A, const amgt_allocator* al, void* stream);
+
+/*
+ * Tile-level transpose out = in^T (R = P^T of Alg. 1 line 4, L54): tile (I,J) becomes
+ * (J,I) with its 4x4 values and bitmap transposed; block rows of out sorted by column.
+ * Same precision as in.  Syncs once (to size nothing — tile count is unchanged — but to
+ * read back a format flag).
+ */
+amgt_status amgt_mbsr_transpose(const amgt_mbsr* in, amgt_mbsr* out, const amgt_allocator* al, void* stream);
+
+/* Build an mBSR from device arrays the caller owns (no copy; own = 0). */
+amgt_status amgt_mbsr_wrap(int64_t m, int64_t n, int64_t blc_num, int64_t* blc_ptr, int32_t* blc_idx,
+                           uint16_t* blc_map, void* blc_val, amgt_prec prec, amgt_mbsr* out);
+
+/* ------------------------------------------------------------------ SpGEMM (§IV.C) */
+
+typedef struct {
+    int64_t bin_rows[8];     /* block rows of C per bin (L151; edges 128*2^b, R7)          */
+    int64_t cub_total;       /* sum over rows of Cub_per_row (intermediate tile products)  */
+    int64_t pairs_nonzero;   /* tile pairs with BITMAPMULTIPLY(mapA, mapB) != 0 (L165)     */
+    int64_t pairs_tc;        /* of those, pairs whose A tile takes the tensor-core route   */
+    int64_t scalar_products; /* sum over nonzero pairs of scalar multiply-adds (FLOP = 2x)  */
+    int64_t numeric_rows[3]; /* C block rows per numeric path (warp/smem, warp/global, empty) */
+} amgt_spgemm_info;
+
+/*
+ * Symbolic SpGEMM C = A*B (§IV.C.1-2; Alg. 3).  Data analysis
+ * (Cub_per_row), binning into 8 bins (<128, [128,256), ..., >=8192), two-step hash
+ * symbolic (step 1 counts distinct C tiles with BITMAPMULTIPLY != 0, prefix sum to
+ * blc_ptrC, allocation, step 2 re-inserts, compresses and sorts -> blc_idxC) and, in
+ * this build, the OR of BITMAPMULTIPLY results into blc_mapC (R15).
+ * A, B: same precision, A.n == B.m.  C: output; structure allocated and filled, values
+ * allocated (not computed).  info may be NULL.  Syncs once (the C tile count, L153)
+ * plus once more if info != NULL.
+ */
+amgt_status amgt_spgemm_symbolic(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, amgt_spgemm_info* info,
+                                 const amgt_allocator* al, void* stream);
+
+/*
+ * Numeric SpGEMM (§IV.C.3; Alg. 4).  One warp per C block row.
+ * Per A tile: POPCOUNT(mapA) >= tc_threshold -> warp-level tensor-core route (FP64:
+ * DMMA m8n8k4 with fragA = [A;A], fragB = [B_j | B_j'], keeping the two diagonal 4x4
+ * quadrants, L157-171; FP16: HMMA m16n8k16 with FP32 accumulation, 8 tile products per
+ * instruction); otherwise the thread-level CUDA-core route.  FP32 always takes the
+ * CUDA-core route (no TF32, R17).  C must come from amgt_spgemm_symbolic(A, B).
+ * Values: deterministic.
+ */
+amgt_status amgt_spgemm_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, void* stream);
+
+/* Tensor-core routing threshold on POPCOUNT(mapA) (paper: 10, L157).  17 disables the
+ * tensor-core route, 0 forces it.  Applies to SpGEMM numeric and SpMV. Process-global. */
+amgt_status amgt_set_tc_threshold(int spgemm_threshold, int spmv_threshold);
+
+/* Galerkin product Ac = R*(A*P) via two SpGEMM calls (Alg. 1 line 5, L54; R20). */
+amgt_status amgt_rap(const amgt_mbsr* R, const amgt_mbsr* A, const amgt_mbsr* P, amgt_mbsr* Ac,
+                     const amgt_allocator* al, void* stream);
+
+/* -------------------------------------------------------------------- SpMV (§IV.D) */
+
+/*
+ * Optional SpMV preprocessing (L220 "data preprocessing"): computes avg_nnz_blc, the
+ * variation (coefficient of variation of tiles per block row, R11) and the
+ * load-balancing work list (block rows longer than 64 tiles are split into chunks of
+ * WARP_CAPACITY = 64 tiles, Alg. 5, R12).  Stored in A->aux (freed by amgt_mbsr_free).
+ * Without it amgt_spmv still works (no row splitting).  Syncs once.
+ */
+amgt_status amgt_spmv_analyze(amgt_mbsr* A, const amgt_allocator* al, void* stream);
+
+typedef struct {
+    double avg_nnz_blc;      /* nnz / blc_num (L220)                          */
+    double variation;        /* CV of tiles per block row (R11)               */
+    int64_t long_rows;       /* block rows split over several warps           */
+    int64_t chunks;          /* warp work items for the long rows             */
+    int64_t tc_tiles;        /* tiles with popcount >= the SpMV TC threshold  */
+} amgt_spmv_stats;
+amgt_status amgt_spmv_get_stats(const amgt_mbsr* A, amgt_spmv_stats* st_host);
+
+/*
+ * y = A*x (§IV.D; Alg. 5).  x has 4*blc_col elements and y has
+ * 4*blc_row elements (zero padding beyond n / m is read as zero / written as zero).
+ * x and y precisions FP64 or FP32 independently of A's (FP64/FP32/FP16).  Arithmetic:
+ * FP64 when A is FP64, else FP32 (FP16 values widened in registers).  Tiles with
+ * popcount >= the SpMV TC threshold go through DMMA (FP64) two tiles per instruction,
+ * y taken from the diagonal blocks of fragY (L222-228, R14); others use CUDA cores with
+ * 4 lanes per tile, one tile row per lane (L230).  Values: deterministic.
+ */
+amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec,
+                      void* stream);
+
+/* ------------------------------------------------------ hierarchy + V-cycle (§II) */
+
+typedef struct {
+    int max_levels;          /* <= 8 (paper: <= 7, L302) */
+    int nu1, nu2;            /* pre/post smoothing sweeps (paper num_sweep = 1, L300) */
+    double omega;            /* weighted-Jacobi weight (R21; default 2/3) */
+    amgt_prec level_prec[8]; /* matrix precision per level (L266: FP64, FP32, FP16...) */
+} amgt_vcycle_opts;
+
+typedef struct amgt_hierarchy amgt_hierarchy;
+
+/*
+ * Setup (Alg. 1, L52-58) with fixed interpolation: A (FP64 mBSR, level 1) and P[k]
+ * (FP64 mBSR, n_k x n_{k+1}), k = 0..nlev-2.  For each level: R_k = P_k^T is built on
+ * the device, A_{k+1} = R_k A_k P_k (two SpGEMM calls, run in level k's precision),
+ * then cast to level k+1's precision (L266).  The coarsest level is converted back to
+ * CSR (MBSR2CSR, L262) and factorised (dense Cholesky, FP64, R22).  Syncs.
+ */
+amgt_status amgt_hierarchy_create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nlev,
+                                  const amgt_vcycle_opts* o, const amgt_allocator* al, void* stream,
+                                  amgt_hierarchy** H);
+
+/* Level-k operators (borrowed pointers valid until destroy); k = 0 .. nlev-1. */
+amgt_status amgt_hierarchy_level(const amgt_hierarchy* H, int k, const amgt_mbsr** A, const amgt_mbsr** P,
+                                 const amgt_mbsr** R);
+int amgt_hierarchy_nlev(const amgt_hierarchy* H);
+
+/*
+ * Solve phase (Alg. 2, L68-82): ncycles V-cycles on A x = b, weighted Jacobi smoothing,
+ * direct coarsest solve; after each cycle the level-1 residual and its 2-norm (L308).
+ * b, x: FP64 device vectors of length 4*blc_row(A_1); x = initial guess in, result out.
+ * res_norms_host[ncycles+1] (||b - A x0|| first) and *spmv_calls_host (may be NULL).
+ * Syncs once at the end (norms are accumulated on the device).
+ */
+amgt_status amgt_vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_norms_host,
+                        int64_t* spmv_calls_host, void* stream);
+
+amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H);
+
+/* ------------------------------------------------------------- instrumentation */
+
+/* Per-kernel-class device timing with CUDA events recorded on the launching stream.
+ * Classes: 0 SpMV level-1, 1 SpMV other levels, 2 SpGEMM symbolic, 3 SpGEMM numeric,
+ * 4 CSR->mBSR, 5 mBSR->CSR, 6 cast, 7 vector ops. */
+#define AMGT_TIMER_CLASSES 8
+amgt_status amgt_timing_enable(int on);
+amgt_status amgt_timing_reset(void);
+/* Syncs the recorded events; fills ms_total[8], launches[8] and bytes[8] (algorithmic
+ * bytes of SURVEY §8(d) per class) on the host. */
+amgt_status amgt_timing_read(double* ms_total_host, int64_t* launches_host, double* bytes_host);
+/* Number of kernel launches issued by the library since the last reset. */
+int64_t amgt_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#if defined(__GNUC__)
+#pragma GCC visibility pop
+#endif
+#endif /* AMGT_H */

@@ -1,0 +1,397 @@
+"""ctypes binding of libamgt.so (include/amgt.h) — argument marshalling only.
+
+Every computation runs in the library's CUDA kernels.  torch supplies device memory
+(the caching allocator is handed to the library as its amgt_allocator), the current
+stream, and tensor views of library-owned arrays.  There is no CPU fallback: if
+libamgt.so is missing this module raises on import.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libamgt.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} not built — run `python __graft_entry__.py build` "
+                      "(there is no CPU fallback for the AmgT kernels)")
+_L = ctypes.CDLL(LIB_PATH)
+
+FP64, FP32, FP16 = 0, 1, 2
+PREC = {"f64": FP64, "f32": FP32, "f16": FP16, FP64: FP64, FP32: FP32, FP16: FP16}
+PREC_DTYPE = {FP64: torch.float64, FP32: torch.float32, FP16: torch.float16}
+PREC_NAME = {FP64: "f64", FP32: "f32", FP16: "f16"}
+STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_FORMAT", 3: "ERR_ALLOC", 4: "ERR_CUDA", 5: "ERR_NCCL", 6: "ERR_RANGE",
+          7: "ERR_UNSUPPORTED"}
+
+
+class AmgtError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class c_mbsr(ctypes.Structure):
+    _fields_ = [("m", ctypes.c_int64), ("n", ctypes.c_int64), ("blc_row", ctypes.c_int64),
+                ("blc_col", ctypes.c_int64), ("blc_num", ctypes.c_int64), ("blc_ptr", ctypes.c_void_p),
+                ("blc_idx", ctypes.c_void_p), ("blc_map", ctypes.c_void_p), ("blc_val", ctypes.c_void_p),
+                ("prec", ctypes.c_int), ("own", ctypes.c_uint32), ("aux", ctypes.c_void_p)]
+
+
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+
+
+class c_allocator(ctypes.Structure):
+    _fields_ = [("alloc", _ALLOC_FN), ("free", _FREE_FN), ("ctx", ctypes.c_void_p)]
+
+
+class c_spgemm_info(ctypes.Structure):
+    _fields_ = [("bin_rows", ctypes.c_int64 * 8), ("cub_total", ctypes.c_int64), ("pairs_nonzero", ctypes.c_int64),
+                ("pairs_tc", ctypes.c_int64), ("scalar_products", ctypes.c_int64),
+                ("numeric_rows", ctypes.c_int64 * 3)]
+
+    def as_dict(self):
+        return {"bin_rows": list(self.bin_rows), "cub_total": self.cub_total, "pairs_nonzero": self.pairs_nonzero,
+                "pairs_tc": self.pairs_tc, "scalar_products": self.scalar_products,
+                "numeric_rows": list(self.numeric_rows)}
+
+
+class c_spmv_stats(ctypes.Structure):
+    _fields_ = [("avg_nnz_blc", ctypes.c_double), ("variation", ctypes.c_double), ("long_rows", ctypes.c_int64),
+                ("chunks", ctypes.c_int64), ("tc_tiles", ctypes.c_int64)]
+
+
+class c_vcycle_opts(ctypes.Structure):
+    _fields_ = [("max_levels", ctypes.c_int), ("nu1", ctypes.c_int), ("nu2", ctypes.c_int), ("omega", ctypes.c_double),
+                ("level_prec", ctypes.c_int * 8)]
+
+
+_vp, _i64, _i32, _int = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_int
+_P = ctypes.POINTER
+_sigs = {
+    "amgt_last_error": (ctypes.c_char_p, []),
+    "amgt_version": (ctypes.c_char_p, []),
+    "amgt_csr_to_mbsr": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _int, _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_mbsr_nnz": (_int, [_P(c_mbsr), _P(_i64), _vp]),
+    "amgt_mbsr_to_csr": (_int, [_P(c_mbsr), _vp, _vp, _vp, _vp]),
+    "amgt_mbsr_cast": (_int, [_P(c_mbsr), _int, _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_mbsr_free": (_int, [_P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_mbsr_transpose": (_int, [_P(c_mbsr), _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_mbsr_wrap": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _int, _P(c_mbsr)]),
+    "amgt_spgemm_symbolic": (_int, [_P(c_mbsr), _P(c_mbsr), _P(c_mbsr), _P(c_spgemm_info), _P(c_allocator), _vp]),
+    "amgt_spgemm_numeric": (_int, [_P(c_mbsr), _P(c_mbsr), _P(c_mbsr), _vp]),
+    "amgt_set_tc_threshold": (_int, [_int, _int]),
+    "amgt_rap": (_int, [_P(c_mbsr), _P(c_mbsr), _P(c_mbsr), _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_spmv_analyze": (_int, [_P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_spmv_get_stats": (_int, [_P(c_mbsr), _P(c_spmv_stats)]),
+    "amgt_spmv": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _vp]),
+    "amgt_hierarchy_create": (_int, [_P(c_mbsr), _P(_P(c_mbsr)), _int, _P(c_vcycle_opts), _P(c_allocator), _vp,
+                                     _P(_vp)]),
+    "amgt_hierarchy_level": (_int, [_vp, _int, _P(_P(c_mbsr)), _P(_P(c_mbsr)), _P(_P(c_mbsr))]),
+    "amgt_hierarchy_nlev": (_int, [_vp]),
+    "amgt_vcycle": (_int, [_vp, _vp, _vp, _int, _P(ctypes.c_double), _P(_i64), _vp]),
+    "amgt_hierarchy_destroy": (_int, [_vp]),
+    "amgt_timing_enable": (_int, [_int]),
+    "amgt_timing_reset": (_int, []),
+    "amgt_timing_read": (_int, [_P(ctypes.c_double), _P(_i64), _P(ctypes.c_double)]),
+    "amgt_launch_count": (_i64, []),
+}
+for _name, (_res, _args) in _sigs.items():
+    _f = getattr(_L, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+EXPORTED = tuple(_sigs)
+
+
+def _check(st: int):
+    if st != 0:
+        raise AmgtError(st, _L.amgt_last_error().decode(errors="replace"))
+
+
+def version() -> str:
+    return _L.amgt_version().decode()
+
+
+def _stream(stream=None) -> int:
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+
+
+# ------------------------------------------------------------------ allocator (torch caching allocator)
+_live: dict[int, int] = {}
+
+
+@_ALLOC_FN
+def _torch_alloc(nbytes, stream, ctx):
+    try:
+        p = torch.cuda.caching_allocator_alloc(int(nbytes), torch.cuda.current_device(),
+                                               torch.cuda.ExternalStream(stream) if stream else None)
+        _live[p] = int(nbytes)
+        return p
+    except Exception:  # allocation failure is reported by the library as AMGT_ERR_ALLOC
+        return None
+
+
+@_FREE_FN
+def _torch_free(p, nbytes, stream, ctx):
+    if p:
+        _live.pop(p, None)
+        torch.cuda.caching_allocator_delete(p)
+
+
+ALLOCATOR = c_allocator(_torch_alloc, _torch_free, None)
+_AL = ctypes.byref(ALLOCATOR)
+
+
+class _DevView:
+    """__cuda_array_interface__ for a library-owned device array (keeps its owner alive)."""
+
+    def __init__(self, owner, ptr: int, n: int, typestr: str):
+        self.owner = owner
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": typestr, "data": (int(ptr or 0), False),
+                                         "version": 3, "strides": None, "stream": None}
+
+
+def _view(owner, ptr, n, dtype) -> torch.Tensor:
+    if n == 0 or not ptr:
+        return torch.empty(0, dtype=dtype, device="cuda")
+    ts = {torch.int64: "<i8", torch.int32: "<i4", torch.int16: "<i2", torch.float64: "<f8", torch.float32: "<f4",
+          torch.float16: "<f2"}[dtype]
+    return torch.as_tensor(_DevView(owner, ptr, n, ts), device="cuda")
+
+
+# ------------------------------------------------------------------ mBSR handle
+class Mbsr:
+    """An mBSR matrix in device memory (library-owned arrays, torch-allocated)."""
+
+    def __init__(self, c: c_mbsr | None = None, keep=()):
+        self.c = c if c is not None else c_mbsr()
+        self._keep = list(keep)  # tensors this matrix borrows from
+
+    # -- properties
+    m = property(lambda s: s.c.m)
+    n = property(lambda s: s.c.n)
+    blc_row = property(lambda s: s.c.blc_row)
+    blc_col = property(lambda s: s.c.blc_col)
+    blc_num = property(lambda s: s.c.blc_num)
+    prec = property(lambda s: s.c.prec)
+
+    @property
+    def blc_ptr(self):
+        return _view(self, self.c.blc_ptr, self.c.blc_row + 1, torch.int64)
+
+    @property
+    def blc_idx(self):
+        return _view(self, self.c.blc_idx, self.c.blc_num, torch.int32)
+
+    @property
+    def blc_map(self):
+        """uint16 bitmaps (returned as int16 storage; use .to(torch.int32) & 0xFFFF)."""
+        return _view(self, self.c.blc_map, self.c.blc_num, torch.int16)
+
+    @property
+    def blc_val(self):
+        return _view(self, self.c.blc_val, 16 * self.c.blc_num, PREC_DTYPE[self.c.prec])
+
+    def map_u16(self) -> torch.Tensor:
+        return self.blc_map.to(torch.int32) & 0xFFFF
+
+    def free(self):
+        if self.c.own or self.c.aux:
+            _check(_L.amgt_mbsr_free(ctypes.byref(self.c), _AL, _stream()))
+        self.c = c_mbsr()
+
+    def __del__(self):
+        try:
+            if self.c.own or self.c.aux:
+                torch.cuda.synchronize()
+                _L.amgt_mbsr_free(ctypes.byref(self.c), _AL, _stream())
+        except Exception:
+            pass
+
+    # -- operations
+    def nnz(self, stream=None) -> int:
+        v = ctypes.c_int64(0)
+        _check(_L.amgt_mbsr_nnz(ctypes.byref(self.c), ctypes.byref(v), _stream(stream)))
+        return int(v.value)
+
+    def to_csr(self, stream=None):
+        nnz = self.nnz(stream)
+        rp = torch.empty(self.m + 1, dtype=torch.int64, device="cuda")
+        ci = torch.empty(max(nnz, 1), dtype=torch.int32, device="cuda")
+        v = torch.empty(max(nnz, 1), dtype=torch.float64, device="cuda")
+        _check(_L.amgt_mbsr_to_csr(ctypes.byref(self.c), rp.data_ptr(), ci.data_ptr(), v.data_ptr(), _stream(stream)))
+        return rp, ci[:nnz], v[:nnz]
+
+    def cast(self, prec, stream=None) -> "Mbsr":
+        out = Mbsr(keep=[self])
+        _check(_L.amgt_mbsr_cast(ctypes.byref(self.c), PREC[prec], ctypes.byref(out.c), _AL, _stream(stream)))
+        return out
+
+    def transpose(self, stream=None) -> "Mbsr":
+        out = Mbsr()
+        _check(_L.amgt_mbsr_transpose(ctypes.byref(self.c), ctypes.byref(out.c), _AL, _stream(stream)))
+        return out
+
+    def analyze(self, stream=None) -> "Mbsr":
+        _check(_L.amgt_spmv_analyze(ctypes.byref(self.c), _AL, _stream(stream)))
+        return self
+
+    def spmv_stats(self) -> dict:
+        st = c_spmv_stats()
+        _check(_L.amgt_spmv_get_stats(ctypes.byref(self.c), ctypes.byref(st)))
+        return {k: getattr(st, k) for k, _ in c_spmv_stats._fields_}
+
+
+def csr_to_mbsr(m, n, row_ptr: torch.Tensor, col: torch.Tensor, val: torch.Tensor, prec="f64", stream=None) -> Mbsr:
+    """amgt_csr_to_mbsr on device CSR arrays (int64 / int32 / float64, CUDA tensors)."""
+    for t, dt in ((row_ptr, torch.int64), (col, torch.int32), (val, torch.float64)):
+        if not t.is_cuda or t.dtype != dt or not t.is_contiguous():
+            raise TypeError(f"expected contiguous CUDA {dt}, got {t.dtype} on {t.device}")
+    out = Mbsr()
+    _check(_L.amgt_csr_to_mbsr(int(m), int(n), int(col.numel()), row_ptr.data_ptr(), col.data_ptr(), val.data_ptr(),
+                               PREC[prec], ctypes.byref(out.c), _AL, _stream(stream)))
+    return out
+
+
+def from_csr(A, prec="f64", stream=None) -> Mbsr:
+    """gen.CSR (any device) -> Mbsr via amgt_csr_to_mbsr."""
+    d = A.to("cuda")
+    return csr_to_mbsr(d.m, d.n, d.row_ptr.contiguous(), d.col.contiguous(), d.val.contiguous(), prec, stream)
+
+
+def spgemm_symbolic(A: Mbsr, B: Mbsr, stream=None, info: bool = False):
+    C = Mbsr()
+    inf = c_spgemm_info() if info else None
+    _check(_L.amgt_spgemm_symbolic(ctypes.byref(A.c), ctypes.byref(B.c), ctypes.byref(C.c),
+                                   ctypes.byref(inf) if info else None, _AL, _stream(stream)))
+    return (C, inf.as_dict()) if info else C
+
+
+def spgemm_numeric(A: Mbsr, B: Mbsr, C: Mbsr, stream=None) -> Mbsr:
+    _check(_L.amgt_spgemm_numeric(ctypes.byref(A.c), ctypes.byref(B.c), ctypes.byref(C.c), _stream(stream)))
+    return C
+
+
+def spgemm(A: Mbsr, B: Mbsr, stream=None, info: bool = False):
+    r = spgemm_symbolic(A, B, stream, info)
+    C = r[0] if info else r
+    spgemm_numeric(A, B, C, stream)
+    return r
+
+
+def rap(R: Mbsr, A: Mbsr, P: Mbsr, stream=None) -> Mbsr:
+    C = Mbsr()
+    _check(_L.amgt_rap(ctypes.byref(R.c), ctypes.byref(A.c), ctypes.byref(P.c), ctypes.byref(C.c), _AL,
+                       _stream(stream)))
+    return C
+
+
+def set_tc_threshold(spgemm: int = 10, spmv: int = 17):
+    _check(_L.amgt_set_tc_threshold(int(spgemm), int(spmv)))
+
+
+def spmv(A: Mbsr, x: torch.Tensor, y: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """y = A x.  x: CUDA float64/float32 of length >= 4*blc_col (padding read as given);
+    y: float64/float32 of length 4*blc_row (allocated as float64 if None)."""
+    xp = {torch.float64: FP64, torch.float32: FP32}[x.dtype]
+    if x.numel() < 4 * A.blc_col:
+        xx = torch.zeros(4 * A.blc_col, dtype=x.dtype, device=x.device)
+        xx[:x.numel()] = x
+        x = xx
+    if y is None:
+        y = torch.empty(4 * A.blc_row, dtype=torch.float64, device="cuda")
+    yp = {torch.float64: FP64, torch.float32: FP32}[y.dtype]
+    assert y.numel() >= 4 * A.blc_row and x.is_contiguous() and y.is_contiguous()
+    _check(_L.amgt_spmv(ctypes.byref(A.c), x.data_ptr(), xp, y.data_ptr(), yp, _stream(stream)))
+    return y
+
+
+def wrap(m, n, blc_ptr, blc_idx, blc_map, blc_val, prec) -> Mbsr:
+    out = Mbsr(keep=[blc_ptr, blc_idx, blc_map, blc_val])
+    _check(_L.amgt_mbsr_wrap(int(m), int(n), int(blc_idx.numel()), blc_ptr.data_ptr(), blc_idx.data_ptr(),
+                             blc_map.data_ptr(), blc_val.data_ptr(), PREC[prec], ctypes.byref(out.c)))
+    return out
+
+
+# ------------------------------------------------------------------ hierarchy / V-cycle
+class Hierarchy:
+    """amgt_hierarchy_create / amgt_vcycle / amgt_hierarchy_destroy."""
+
+    def __init__(self, A: Mbsr, Ps: list, level_prec=("f64", "f32", "f16", "f16", "f16", "f16", "f16", "f16"),
+                 nu1=1, nu2=1, omega=2.0 / 3.0, stream=None):
+        self.nlev = len(Ps) + 1
+        o = c_vcycle_opts()
+        o.max_levels = self.nlev
+        o.nu1, o.nu2, o.omega = int(nu1), int(nu2), float(omega)
+        lp = list(level_prec) + ["f16"] * 8
+        for k in range(8):
+            o.level_prec[k] = PREC[lp[k]]
+        self._keep = [A, *Ps]
+        arr = (_P(c_mbsr) * max(len(Ps), 1))(*[ctypes.pointer(p.c) for p in Ps])
+        h = ctypes.c_void_p()
+        _check(_L.amgt_hierarchy_create(ctypes.byref(A.c), arr, self.nlev, ctypes.byref(o), _AL, _stream(stream),
+                                        ctypes.byref(h)))
+        self.h = h
+
+    def level(self, k: int):
+        a, p, r = _P(c_mbsr)(), _P(c_mbsr)(), _P(c_mbsr)()
+        _check(_L.amgt_hierarchy_level(self.h, k, ctypes.byref(a), ctypes.byref(p), ctypes.byref(r)))
+
+        def mk(ptr):
+            if not ptr:
+                return None
+            M = Mbsr(c_mbsr.from_buffer_copy(ptr.contents), keep=[self])
+            M.c.own = 0
+            M.c.aux = None
+            return M
+        return mk(a), mk(p), mk(r)
+
+    def vcycle(self, b: torch.Tensor, x: torch.Tensor, ncycles: int, stream=None):
+        assert b.dtype == torch.float64 and x.dtype == torch.float64 and b.is_cuda and x.is_cuda
+        res = (ctypes.c_double * (ncycles + 1))()
+        calls = ctypes.c_int64(0)
+        _check(_L.amgt_vcycle(self.h, b.data_ptr(), x.data_ptr(), int(ncycles), res, ctypes.byref(calls),
+                              _stream(stream)))
+        return list(res), int(calls.value)
+
+    def close(self):
+        if self.h:
+            _L.amgt_hierarchy_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# ------------------------------------------------------------------ instrumentation
+TIMER_CLASSES = ("spmv_l1", "spmv", "spgemm_symbolic", "spgemm_numeric", "csr2mbsr", "mbsr2csr", "cast", "vector")
+
+
+def timing_enable(on: bool = True):
+    _check(_L.amgt_timing_enable(1 if on else 0))
+
+
+def timing_reset():
+    _check(_L.amgt_timing_reset())
+
+
+def timing_read() -> dict:
+    ms = (ctypes.c_double * 8)()
+    n = (ctypes.c_int64 * 8)()
+    by = (ctypes.c_double * 8)()
+    _check(_L.amgt_timing_read(ms, n, by))
+    return {TIMER_CLASSES[i]: {"ms": ms[i], "launches": n[i], "bytes": by[i]} for i in range(8)}
+
+
+def launch_count() -> int:
+    return int(_L.amgt_launch_count())

@@ -1,0 +1,148 @@
+// common.cuh — internal helpers of libamgt (never installed; not part of the ABI).
+#pragma once
+
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <string>
+
+#include "amgt.h"
+
+namespace amgt {
+
+// ------------------------------------------------------------------ errors
+void set_error(const char* fmt, ...);
+amgt_status fail(amgt_status st, const char* fmt, ...);
+
+#define AMGT_CUDA(call)                                                                    \
+    do {                                                                                   \
+        cudaError_t e_ = (call);                                                           \
+        if (e_ != cudaSuccess)                                                             \
+            return ::amgt::fail(AMGT_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call, \
+                                cudaGetErrorString(e_));                                   \
+    } while (0)
+
+#define AMGT_LAUNCHED()                                                                          \
+    do {                                                                                         \
+        ::amgt::count_launch();                                                                  \
+        cudaError_t e_ = cudaGetLastError();                                                     \
+        if (e_ != cudaSuccess)                                                                   \
+            return ::amgt::fail(AMGT_ERR_CUDA, "%s:%d launch: %s", __FILE__, __LINE__,           \
+                                cudaGetErrorString(e_));                                         \
+    } while (0)
+
+#define AMGT_TRY(expr)                       \
+    do {                                     \
+        amgt_status s_ = (expr);             \
+        if (s_ != AMGT_OK) return s_;        \
+    } while (0)
+
+// ------------------------------------------------------------------ allocator
+struct Alloc {
+    const amgt_allocator* al;
+    cudaStream_t s;
+    void* get(size_t bytes);
+    void put(void* p, size_t bytes);
+};
+
+// RAII scratch buffer from the caller's allocator (stream-ordered).
+template <typename T>
+struct Scratch {
+    Alloc* a = nullptr;
+    T* p = nullptr;
+    size_t n = 0;
+    Scratch() = default;
+    Scratch(const Scratch&) = delete;
+    Scratch& operator=(const Scratch&) = delete;
+    amgt_status init(Alloc& al, size_t count) {
+        a = &al;
+        n = count;
+        if (count == 0) return AMGT_OK;
+        p = static_cast<T*>(al.get(count * sizeof(T)));
+        if (!p) return fail(AMGT_ERR_ALLOC, "scratch allocation of %zu bytes failed", count * sizeof(T));
+        return AMGT_OK;
+    }
+    ~Scratch() {
+        if (a && p) a->put(p, n * sizeof(T));
+    }
+};
+
+// ------------------------------------------------------------------ types
+size_t prec_bytes(amgt_prec p);
+inline bool prec_valid(int p) { return p == AMGT_FP64 || p == AMGT_FP32 || p == AMGT_FP16; }
+
+template <typename T> struct AccOf { using type = float; };
+template <> struct AccOf<double> { using type = double; };
+
+__device__ __forceinline__ double to_f64(double v) { return v; }
+__device__ __forceinline__ double to_f64(float v) { return (double)v; }
+__device__ __forceinline__ double to_f64(__half v) { return (double)__half2float(v); }
+__device__ __forceinline__ float to_f32(double v) { return (float)v; }
+__device__ __forceinline__ float to_f32(float v) { return v; }
+__device__ __forceinline__ float to_f32(__half v) { return __half2float(v); }
+
+template <typename T> __device__ __forceinline__ T from_f64(double v);
+template <> __device__ __forceinline__ double from_f64<double>(double v) { return v; }
+template <> __device__ __forceinline__ float from_f64<float>(double v) { return __double2float_rn(v); }
+template <> __device__ __forceinline__ __half from_f64<__half>(double v) { return __double2half(v); }  // RN, direct
+
+template <typename T> __device__ __forceinline__ T from_acc(double v) { return from_f64<T>(v); }
+template <typename T> __device__ __forceinline__ T from_acc(float v);
+template <> __device__ __forceinline__ double from_acc<double>(float v) { return (double)v; }
+template <> __device__ __forceinline__ float from_acc<float>(float v) { return v; }
+template <> __device__ __forceinline__ __half from_acc<__half>(float v) { return __float2half_rn(v); }
+
+template <typename A> __device__ __forceinline__ A acc_from(double v);
+template <> __device__ __forceinline__ double acc_from<double>(double v) { return v; }
+template <> __device__ __forceinline__ float acc_from<float>(double v) { return (float)v; }
+template <typename A> __device__ __forceinline__ A acc_of(double v) { return (A)v; }
+template <typename A> __device__ __forceinline__ A acc_of(float v) { return (A)v; }
+template <typename A> __device__ __forceinline__ A acc_of(__half v) { return (A)__half2float(v); }
+
+// ------------------------------------------------------------------ bitmaps
+// BITMAPMULTIPLY (Alg. 3 line 7, Alg. 4 lines 8/22; reading R4): boolean 4x4 product.
+// (mapA >> k) & 0x1111 marks rows r with A(r,k) != 0 at bit 4r; multiplying by B's
+// row-k nibble places that nibble at 4r for each such r (no carries: nibbles disjoint).
+__device__ __forceinline__ uint32_t bitmap_multiply(uint32_t a, uint32_t b) {
+    return (((a >> 0) & 0x1111u) * ((b >> 0) & 0xFu)) | (((a >> 1) & 0x1111u) * ((b >> 4) & 0xFu)) |
+           (((a >> 2) & 0x1111u) * ((b >> 8) & 0xFu)) | (((a >> 3) & 0x1111u) * ((b >> 12) & 0xFu));
+}
+
+// ------------------------------------------------------------------ device flags
+// Bits of the per-call device error word.
+enum : uint32_t { FLAG_FORMAT = 1u, FLAG_RANGE = 2u };
+
+// ------------------------------------------------------------------ scan
+// out[0] = 0, out[i+1] = in[0] + ... + in[i]  (int64, n >= 0).  `in` may alias `out+1`? no.
+amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a, cudaStream_t s);
+
+// ------------------------------------------------------------------ instrumentation
+enum TimerClass : int {
+    TC_SPMV_L1 = 0,
+    TC_SPMV = 1,
+    TC_SPGEMM_SYM = 2,
+    TC_SPGEMM_NUM = 3,
+    TC_CSR2MBSR = 4,
+    TC_MBSR2CSR = 5,
+    TC_CAST = 6,
+    TC_VEC = 7
+};
+void count_launch();
+struct TimerScope {  // records start/end events on `s` when timing is enabled
+    int cls;
+    double bytes;
+    cudaStream_t s;
+    int slot;
+    TimerScope(int cls, double bytes, cudaStream_t s);
+    ~TimerScope();
+};
+
+extern int g_tc_thr_spgemm;
+extern int g_tc_thr_spmv;
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+int num_sms();
+
+}  // namespace amgt

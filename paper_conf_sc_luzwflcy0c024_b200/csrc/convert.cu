@@ -1,0 +1,548 @@
+// convert.cu — CSR <-> mBSR conversion, per-level precision cast, tile transpose.
+//
+// CSR2MBSR (L234, L262; Fig. 6 step 4) on B200: a 4-lane group owns one block row and
+// lane r owns CSR row 4I+r.  The group walks the four sorted column lists in lockstep
+// (a 4-way merge on tile column col>>2, two shuffles per step); each lane writes its own
+// tile row (one 16 B / 32 B vector store) and the group ORs its four nibbles into the
+// 16-bit bitmap (bit 4r+c, R1).  Eight block rows per warp, all reads of a lane
+// sequential in its row.  Two passes (count, fill) around a device prefix sum; one
+// host sync to size the tile arrays.
+#include <climits>
+
+#include "common.cuh"
+
+namespace amgt {
+
+static __device__ __forceinline__ void store_row(double* p, const double (&v)[4]) {
+    reinterpret_cast<double2*>(p)[0] = make_double2(v[0], v[1]);
+    reinterpret_cast<double2*>(p)[1] = make_double2(v[2], v[3]);
+}
+static __device__ __forceinline__ void store_row(float* p, const double (&v)[4]) {
+    *reinterpret_cast<float4*>(p) =
+        make_float4(__double2float_rn(v[0]), __double2float_rn(v[1]), __double2float_rn(v[2]), __double2float_rn(v[3]));
+}
+static __device__ __forceinline__ void store_row(__half* p, const double (&v)[4]) {
+    __half2 a = __halves2half2(__double2half(v[0]), __double2half(v[1]));
+    __half2 b = __halves2half2(__double2half(v[2]), __double2half(v[3]));
+    uint2 u;
+    u.x = *reinterpret_cast<uint32_t*>(&a);
+    u.y = *reinterpret_cast<uint32_t*>(&b);
+    *reinterpret_cast<uint2*>(p) = u;
+}
+
+template <typename T> __device__ __forceinline__ bool overflows(double v) { return false; }
+template <> __device__ __forceinline__ bool overflows<__half>(double v) {
+    return fabs(v) > 65504.0 && fabs(v) < INFINITY && __hisinf(__double2half(v));
+}
+
+// FILL = false: count tiles per block row into cnt[I] and validate the CSR.
+// FILL = true : write blc_idx / blc_map / blc_val at offsets bptr[I].
+template <bool FILL, typename T>
+__global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t nnz, int64_t BR,
+                                                  const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                                                  const double* __restrict__ v, int64_t* __restrict__ cnt,
+                                                  const int64_t* __restrict__ bptr, int32_t* __restrict__ bidx,
+                                                  uint16_t* __restrict__ bmap, T* __restrict__ bval,
+                                                  uint32_t* __restrict__ flag) {
+    const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
+    const int64_t I = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 8 + g;
+    if ((((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 8 >= BR) return;  // whole warp idle
+    const bool active = I < BR;
+    const int64_t row = 4 * I + r;
+    int64_t p = 0, e = 0;
+    uint32_t bad = 0, range = 0;
+    if (active && row < m) {
+        p = rp[row];
+        e = rp[row + 1];
+        if (!FILL) {
+            if (p > e || p < 0 || e > nnz) { bad = 1; e = p; }
+            if (row == 0 && p != 0) bad = 1;
+            if (row == m - 1 && e != nnz) bad = 1;
+        }
+    }
+    int64_t t = (FILL && active) ? bptr[I] : 0;
+    int64_t c = 0;
+    int32_t prev = -1;
+    for (;;) {
+        const int32_t J = (p < e) ? (__ldg(ci + p) >> 2) : INT_MAX;
+        int32_t Jm = min(J, __shfl_xor_sync(0xffffffffu, J, 1));
+        Jm = min(Jm, __shfl_xor_sync(0xffffffffu, Jm, 2));
+        if (!__any_sync(0xffffffffu, Jm != INT_MAX)) break;
+        double rv[4] = {0.0, 0.0, 0.0, 0.0};
+        uint32_t nib = 0;
+        if (Jm != INT_MAX) {
+            while (p < e) {
+                const int32_t col = __ldg(ci + p);
+                if ((col >> 2) != Jm) break;
+                if (!FILL) {
+                    if (col <= prev || col >= n) bad = 1;
+                    prev = col;
+                } else {
+                    const int cc = col & 3;
+                    const double x = __ldg(v + p);
+                    rv[0] = cc == 0 ? x : rv[0];
+                    rv[1] = cc == 1 ? x : rv[1];
+                    rv[2] = cc == 2 ? x : rv[2];
+                    rv[3] = cc == 3 ? x : rv[3];
+                    if (overflows<T>(x)) range = 1;
+                }
+                nib |= 1u << (col & 3);
+                ++p;
+            }
+        }
+        uint32_t mp = nib << (4 * r);
+        mp |= __shfl_xor_sync(0xffffffffu, mp, 1);
+        mp |= __shfl_xor_sync(0xffffffffu, mp, 2);
+        if (Jm != INT_MAX) {
+            if (FILL) {
+                store_row(bval + 16 * t + 4 * r, rv);
+                if (r == 0) {
+                    bidx[t] = Jm;
+                    bmap[t] = (uint16_t)mp;
+                }
+            }
+            ++c;
+            ++t;
+        }
+    }
+    if (!FILL && active && r == 0) cnt[I] = c;
+    if (bad) atomicOr(flag, FLAG_FORMAT);
+    if (range) atomicOr(flag, FLAG_RANGE);
+}
+
+// Row nnz from bitmaps: lane r counts the set bits of nibble r over the block row.
+__global__ void __launch_bounds__(256) k_mbsr2csr_count(int64_t m, int64_t BR, const int64_t* __restrict__ bptr,
+                                                        const uint16_t* __restrict__ bmap, int64_t* __restrict__ rn) {
+    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t I = gt >> 2;
+    const int r = (int)(gt & 3);
+    if (I >= BR) return;
+    const int64_t row = 4 * I + r;
+    if (row >= m) return;
+    int64_t c = 0;
+    for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t) c += __popc((bmap[t] >> (4 * r)) & 0xFu);
+    rn[row] = c;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_mbsr2csr_fill(int64_t m, int64_t BR, const int64_t* __restrict__ bptr,
+                                                       const int32_t* __restrict__ bidx,
+                                                       const uint16_t* __restrict__ bmap, const T* __restrict__ bval,
+                                                       const int64_t* __restrict__ rp, int32_t* __restrict__ ci,
+                                                       double* __restrict__ v) {
+    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t I = gt >> 2;
+    const int r = (int)(gt & 3);
+    if (I >= BR) return;
+    const int64_t row = 4 * I + r;
+    if (row >= m) return;
+    int64_t d = rp[row];
+    for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t) {
+        const uint32_t nib = (bmap[t] >> (4 * r)) & 0xFu;
+        if (!nib) continue;
+        const int32_t J = bidx[t];
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+            if (nib & (1u << c)) {
+                ci[d] = 4 * J + c;
+                v[d] = to_f64(bval[16 * t + 4 * r + c]);
+                ++d;
+            }
+    }
+}
+
+__global__ void k_popc_sum(int64_t T, const uint16_t* __restrict__ bmap, unsigned long long* __restrict__ out) {
+    int64_t s = 0;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < T; t += (int64_t)gridDim.x * blockDim.x)
+        s += __popc(bmap[t]);
+    for (int d = 16; d; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
+    if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, (unsigned long long)s);
+}
+
+template <typename Ti, typename To>
+__global__ void k_cast(int64_t n, const Ti* __restrict__ in, To* __restrict__ out, uint32_t* __restrict__ flag) {
+    uint32_t bad = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double x = to_f64(in[i]);
+        To y;
+        if constexpr (sizeof(Ti) == 4 && sizeof(To) == 2) {
+            y = __float2half_rn((float)x);  // FP32 -> FP16 (single rounding from FP32)
+        } else {
+            y = from_f64<To>(x);  // direct from FP64 (R18)
+        }
+        if (overflows<To>(x)) bad = 1;
+        out[i] = y;
+    }
+    if (bad) atomicOr(flag, FLAG_RANGE);
+}
+
+// ---- transpose: (1) count per destination row, (2) scan, (3) scatter (idx, perm),
+// (4) per-row sort by column, (5) gather transposed tiles.
+__global__ void k_tr_count(int64_t T, const int32_t* __restrict__ bidx, unsigned long long* __restrict__ cnt) {
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < T; t += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(cnt + bidx[t], 1ull);
+}
+
+__global__ void k_tr_scatter(int64_t BR, const int64_t* __restrict__ bptr, const int32_t* __restrict__ bidx,
+                             const int64_t* __restrict__ optr, unsigned long long* __restrict__ fill,
+                             int32_t* __restrict__ oidx, int64_t* __restrict__ perm) {
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t) {
+            const int32_t J = bidx[t];
+            const int64_t d = optr[J] + (int64_t)atomicAdd(fill + J, 1ull);
+            oidx[d] = (int32_t)I;
+            perm[d] = t;
+        }
+}
+
+__global__ void k_tr_sort(int64_t BRo, const int64_t* __restrict__ optr, int32_t* __restrict__ oidx,
+                          int64_t* __restrict__ perm) {
+    for (int64_t J = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; J < BRo; J += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t a = optr[J], b = optr[J + 1];
+        for (int64_t i = a + 1; i < b; ++i) {  // insertion sort (rows of P^T are short)
+            const int32_t k = oidx[i];
+            const int64_t pv = perm[i];
+            int64_t j = i - 1;
+            while (j >= a && oidx[j] > k) {
+                oidx[j + 1] = oidx[j];
+                perm[j + 1] = perm[j];
+                --j;
+            }
+            oidx[j + 1] = k;
+            perm[j + 1] = pv;
+        }
+    }
+}
+
+template <typename T>
+__global__ void k_tr_gather(int64_t T_, const int64_t* __restrict__ perm, const uint16_t* __restrict__ bmap,
+                            const T* __restrict__ bval, uint16_t* __restrict__ omap, T* __restrict__ oval) {
+    for (int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; d < T_; d += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t s = perm[d];
+        const uint32_t mp = bmap[s];
+        uint32_t tm = 0;
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                if (mp & (1u << (4 * r + c))) tm |= 1u << (4 * c + r);
+        omap[d] = (uint16_t)tm;
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) oval[16 * d + 4 * c + r] = bval[16 * s + 4 * r + c];
+    }
+}
+
+static unsigned grid_for(int64_t work, int threads) {
+    int64_t b = ceil_div(work, threads);
+    int64_t cap = (int64_t)num_sms() * 16;
+    if (b > cap) b = cap;
+    if (b < 1) b = 1;
+    return (unsigned)b;
+}
+
+amgt_status mbsr_alloc(amgt_mbsr* M, int64_t m, int64_t n, int64_t T, amgt_prec prec, Alloc& a, bool structure,
+                       bool values, int64_t* existing_ptr) {
+    M->m = m;
+    M->n = n;
+    M->blc_row = ceil_div(m, 4);
+    M->blc_col = ceil_div(n, 4);
+    M->blc_num = T;
+    M->prec = prec;
+    M->aux = nullptr;
+    M->own = 0;
+    if (structure) {
+        M->blc_ptr = existing_ptr ? existing_ptr : (int64_t*)a.get((M->blc_row + 1) * sizeof(int64_t));
+        M->blc_idx = (int32_t*)a.get(T * sizeof(int32_t));
+        M->blc_map = (uint16_t*)a.get(((T + 1) & ~int64_t(1)) * sizeof(uint16_t));  // even count: u32 atomics
+        M->own |= 1u;
+        if (!M->blc_ptr || !M->blc_idx || !M->blc_map) return fail(AMGT_ERR_ALLOC, "mBSR structure allocation failed");
+    }
+    if (values) {
+        M->blc_val = a.get(16 * T * prec_bytes(prec));
+        M->own |= 2u;
+        if (!M->blc_val) return fail(AMGT_ERR_ALLOC, "mBSR value allocation failed (%lld tiles)", (long long)T);
+    }
+    return AMGT_OK;
+}
+
+void spmv_plan_free(void* aux, Alloc& a);
+
+amgt_status mbsr_release(amgt_mbsr* M, Alloc& a) {
+    if (!M) return AMGT_OK;
+    if (M->aux) spmv_plan_free(M->aux, a);
+    if (M->own & 1u) {
+        a.put(M->blc_ptr, (M->blc_row + 1) * sizeof(int64_t));
+        a.put(M->blc_idx, M->blc_num * sizeof(int32_t));
+        a.put(M->blc_map, ((M->blc_num + 1) & ~int64_t(1)) * sizeof(uint16_t));
+    }
+    if (M->own & 2u) a.put(M->blc_val, 16 * M->blc_num * prec_bytes(M->prec));
+    *M = amgt_mbsr{};
+    return AMGT_OK;
+}
+
+static amgt_status read_flag(uint32_t* dflag, cudaStream_t s, uint32_t* out) {
+    AMGT_CUDA(cudaMemcpyAsync(out, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    return AMGT_OK;
+}
+
+amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* rp, const int32_t* ci,
+                             const double* v, amgt_prec prec, amgt_mbsr* out, Alloc& a) {
+    cudaStream_t s = a.s;
+    const int64_t BR = ceil_div(m, 4);
+    Scratch<int64_t> cnt;
+    Scratch<uint32_t> flag;
+    AMGT_TRY(cnt.init(a, BR + 1));
+    AMGT_TRY(flag.init(a, 1));
+    AMGT_CUDA(cudaMemsetAsync(flag.p, 0, sizeof(uint32_t), s));
+    amgt_mbsr M{};
+    const double bytes_in = nnz * 12.0 + (m + 1) * 8.0;
+    const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 256);
+    {
+        TimerScope ts(TC_CSR2MBSR, bytes_in, s);
+        if (BR > 0) {
+            k_csr2mbsr<false, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, cnt.p, nullptr, nullptr,
+                                                             nullptr, nullptr, flag.p);
+            AMGT_LAUNCHED();
+        }
+    }
+    // blc_ptr lives in the output; scan the counts into it.
+    M.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
+    if (!M.blc_ptr) return fail(AMGT_ERR_ALLOC, "blc_ptr allocation failed");
+    AMGT_TRY(scan_exclusive(cnt.p, M.blc_ptr, BR, a, s));
+    int64_t hT[1] = {0};
+    uint32_t hflag = 0;
+    AMGT_CUDA(cudaMemcpyAsync(hT, M.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaMemcpyAsync(&hflag, flag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    if (hflag & FLAG_FORMAT) {
+        a.put(M.blc_ptr, (BR + 1) * sizeof(int64_t));
+        return fail(AMGT_ERR_FORMAT, "CSR input: row_ptr not monotone from 0 to nnz, or columns unsorted/duplicate/out of range");
+    }
+    const int64_t T = hT[0];
+    amgt_status st = mbsr_alloc(&M, m, n, T, prec, a, true, true, M.blc_ptr);
+    if (st != AMGT_OK) { mbsr_release(&M, a); return st; }
+    {
+        const double bytes = bytes_in + T * (16.0 * prec_bytes(prec) + 6.0) + (BR + 1) * 8.0;
+        TimerScope ts(TC_CSR2MBSR, bytes, s);
+        if (BR > 0) {
+            switch (prec) {
+                case AMGT_FP64:
+                    k_csr2mbsr<true, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, nullptr, M.blc_ptr,
+                                                                    M.blc_idx, M.blc_map, (double*)M.blc_val, flag.p);
+                    break;
+                case AMGT_FP32:
+                    k_csr2mbsr<true, float><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, nullptr, M.blc_ptr,
+                                                                   M.blc_idx, M.blc_map, (float*)M.blc_val, flag.p);
+                    break;
+                default:
+                    k_csr2mbsr<true, __half><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, nullptr, M.blc_ptr,
+                                                                    M.blc_idx, M.blc_map, (__half*)M.blc_val, flag.p);
+            }
+            AMGT_LAUNCHED();
+        }
+    }
+    if (prec == AMGT_FP16) {
+        AMGT_TRY(read_flag(flag.p, s, &hflag));
+        if (hflag & FLAG_RANGE) {
+            mbsr_release(&M, a);
+            return fail(AMGT_ERR_RANGE, "value exceeds the FP16 range (65504)");
+        }
+    }
+    *out = M;
+    return AMGT_OK;
+}
+
+template <typename T>
+static void launch_m2c_fill(const amgt_mbsr* A, const int64_t* rp, int32_t* ci, double* v, cudaStream_t s) {
+    const unsigned blocks = (unsigned)ceil_div(A->blc_row * 4, 256);
+    k_mbsr2csr_fill<T><<<blocks, 256, 0, s>>>(A->m, A->blc_row, A->blc_ptr, A->blc_idx, A->blc_map,
+                                              (const T*)A->blc_val, rp, ci, v);
+}
+
+amgt_status mbsr_to_csr_impl(const amgt_mbsr* A, int64_t* rp, int32_t* ci, double* v, Alloc& a) {
+    cudaStream_t s = a.s;
+    Scratch<int64_t> rn;
+    AMGT_TRY(rn.init(a, A->m + 1));
+    const int64_t nnz_est = A->blc_num * 16;
+    TimerScope ts(TC_MBSR2CSR, A->blc_num * (16.0 * prec_bytes(A->prec) + 6.0) + (A->m + 1) * 8.0, s);
+    if (A->blc_row > 0) {
+        k_mbsr2csr_count<<<(unsigned)ceil_div(A->blc_row * 4, 256), 256, 0, s>>>(A->m, A->blc_row, A->blc_ptr,
+                                                                                  A->blc_map, rn.p);
+        AMGT_LAUNCHED();
+    }
+    AMGT_TRY(scan_exclusive(rn.p, rp, A->m, a, s));
+    (void)nnz_est;
+    if (A->blc_row > 0) {
+        switch (A->prec) {
+            case AMGT_FP64: launch_m2c_fill<double>(A, rp, ci, v, s); break;
+            case AMGT_FP32: launch_m2c_fill<float>(A, rp, ci, v, s); break;
+            default: launch_m2c_fill<__half>(A, rp, ci, v, s);
+        }
+        AMGT_LAUNCHED();
+    }
+    return AMGT_OK;
+}
+
+amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& a) {
+    cudaStream_t s = a.s;
+    if (prec_bytes(to) > prec_bytes(in->prec)) return fail(AMGT_ERR_ARG, "cast must not widen (from %d to %d)", in->prec, to);
+    amgt_mbsr M = *in;
+    M.own = 0;
+    M.aux = nullptr;
+    M.prec = to;
+    const int64_t n = 16 * in->blc_num;
+    M.blc_val = a.get(n * prec_bytes(to));
+    if (!M.blc_val) return fail(AMGT_ERR_ALLOC, "cast value allocation failed");
+    M.own = 2u;
+    Scratch<uint32_t> flag;
+    AMGT_TRY(flag.init(a, 1));
+    AMGT_CUDA(cudaMemsetAsync(flag.p, 0, sizeof(uint32_t), s));
+    {
+        TimerScope ts(TC_CAST, (double)n * (prec_bytes(in->prec) + prec_bytes(to)), s);
+        if (n > 0) {
+            const unsigned g = grid_for(n, 256);
+            if (in->prec == to) {
+                AMGT_CUDA(cudaMemcpyAsync(M.blc_val, in->blc_val, n * prec_bytes(to), cudaMemcpyDeviceToDevice, s));
+            } else if (in->prec == AMGT_FP64 && to == AMGT_FP32) {
+                k_cast<double, float><<<g, 256, 0, s>>>(n, (const double*)in->blc_val, (float*)M.blc_val, flag.p);
+                AMGT_LAUNCHED();
+            } else if (in->prec == AMGT_FP64 && to == AMGT_FP16) {
+                k_cast<double, __half><<<g, 256, 0, s>>>(n, (const double*)in->blc_val, (__half*)M.blc_val, flag.p);
+                AMGT_LAUNCHED();
+            } else {
+                k_cast<float, __half><<<g, 256, 0, s>>>(n, (const float*)in->blc_val, (__half*)M.blc_val, flag.p);
+                AMGT_LAUNCHED();
+            }
+        }
+    }
+    if (to == AMGT_FP16 && in->prec != AMGT_FP16) {
+        uint32_t hflag = 0;
+        AMGT_TRY(read_flag(flag.p, s, &hflag));
+        if (hflag & FLAG_RANGE) {
+            a.put(M.blc_val, n * prec_bytes(to));
+            return fail(AMGT_ERR_RANGE, "value exceeds the FP16 range (65504)");
+        }
+    }
+    *out = M;
+    return AMGT_OK;
+}
+
+template <typename T>
+static void launch_tr_gather(const amgt_mbsr* in, const int64_t* perm, amgt_mbsr* o, cudaStream_t s) {
+    k_tr_gather<T><<<grid_for(in->blc_num, 256), 256, 0, s>>>(in->blc_num, perm, in->blc_map, (const T*)in->blc_val,
+                                                             o->blc_map, (T*)o->blc_val);
+}
+
+amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a) {
+    cudaStream_t s = a.s;
+    amgt_mbsr M{};
+    AMGT_TRY(mbsr_alloc(&M, in->n, in->m, in->blc_num, in->prec, a, true, true, nullptr));
+    const int64_t BRo = M.blc_row, T = in->blc_num;
+    Scratch<unsigned long long> cnt;
+    Scratch<int64_t> perm;
+    amgt_status st = cnt.init(a, BRo + 1);
+    if (st == AMGT_OK) st = perm.init(a, T);
+    if (st != AMGT_OK) { mbsr_release(&M, a); return st; }
+    AMGT_CUDA(cudaMemsetAsync(cnt.p, 0, (BRo + 1) * sizeof(unsigned long long), s));
+    if (T > 0) {
+        k_tr_count<<<grid_for(T, 256), 256, 0, s>>>(T, in->blc_idx, cnt.p);
+        AMGT_LAUNCHED();
+    }
+    AMGT_TRY(scan_exclusive((const int64_t*)cnt.p, M.blc_ptr, BRo, a, s));
+    AMGT_CUDA(cudaMemsetAsync(cnt.p, 0, (BRo + 1) * sizeof(unsigned long long), s));
+    if (T > 0) {
+        k_tr_scatter<<<grid_for(in->blc_row, 128), 128, 0, s>>>(in->blc_row, in->blc_ptr, in->blc_idx, M.blc_ptr, cnt.p,
+                                                                M.blc_idx, perm.p);
+        AMGT_LAUNCHED();
+        k_tr_sort<<<grid_for(BRo, 128), 128, 0, s>>>(BRo, M.blc_ptr, M.blc_idx, perm.p);
+        AMGT_LAUNCHED();
+        switch (in->prec) {
+            case AMGT_FP64: launch_tr_gather<double>(in, perm.p, &M, s); break;
+            case AMGT_FP32: launch_tr_gather<float>(in, perm.p, &M, s); break;
+            default: launch_tr_gather<__half>(in, perm.p, &M, s);
+        }
+        AMGT_LAUNCHED();
+    }
+    *out = M;
+    return AMGT_OK;
+}
+
+}  // namespace amgt
+
+using namespace amgt;
+
+extern "C" {
+
+amgt_status amgt_csr_to_mbsr(int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr, const int32_t* col_idx,
+                             const double* val, amgt_prec prec, amgt_mbsr* out, const amgt_allocator* al,
+                             void* stream) {
+    if (!out || m < 0 || n < 0 || nnz < 0 || !prec_valid(prec)) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: bad argument");
+    if (m > 0 && !row_ptr) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: row_ptr is NULL");
+    if (nnz > 0 && (!col_idx || !val)) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: col/val NULL");
+    if (ceil_div(n, 4) > INT32_MAX) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: too many columns for int32 tile indices");
+    Alloc a{al, (cudaStream_t)stream};
+    return csr_to_mbsr_impl(m, n, nnz, row_ptr, col_idx, val, prec, out, a);
+}
+
+amgt_status amgt_mbsr_nnz(const amgt_mbsr* A, int64_t* nnz_host, void* stream) {
+    if (!A || !nnz_host) return fail(AMGT_ERR_ARG, "amgt_mbsr_nnz: NULL argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    Alloc a{nullptr, s};
+    Scratch<unsigned long long> d;
+    AMGT_TRY(d.init(a, 1));
+    AMGT_CUDA(cudaMemsetAsync(d.p, 0, sizeof(unsigned long long), s));
+    if (A->blc_num > 0) {
+        k_popc_sum<<<grid_for(A->blc_num, 256), 256, 0, s>>>(A->blc_num, A->blc_map, d.p);
+        AMGT_LAUNCHED();
+    }
+    unsigned long long h = 0;
+    AMGT_CUDA(cudaMemcpyAsync(&h, d.p, sizeof(h), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    *nnz_host = (int64_t)h;
+    return AMGT_OK;
+}
+
+amgt_status amgt_mbsr_to_csr(const amgt_mbsr* A, int64_t* row_ptr, int32_t* col_idx, double* val, void* stream) {
+    if (!A || !row_ptr) return fail(AMGT_ERR_ARG, "amgt_mbsr_to_csr: NULL argument");
+    Alloc a{nullptr, (cudaStream_t)stream};
+    return mbsr_to_csr_impl(A, row_ptr, col_idx, val, a);
+}
+
+amgt_status amgt_mbsr_cast(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, const amgt_allocator* al, void* stream) {
+    if (!in || !out || !prec_valid(to)) return fail(AMGT_ERR_ARG, "amgt_mbsr_cast: bad argument");
+    Alloc a{al, (cudaStream_t)stream};
+    return cast_impl(in, to, out, a);
+}
+
+amgt_status amgt_mbsr_free(amgt_mbsr* A, const amgt_allocator* al, void* stream) {
+    Alloc a{al, (cudaStream_t)stream};
+    return mbsr_release(A, a);
+}
+
+amgt_status amgt_mbsr_transpose(const amgt_mbsr* in, amgt_mbsr* out, const amgt_allocator* al, void* stream) {
+    if (!in || !out) return fail(AMGT_ERR_ARG, "amgt_mbsr_transpose: NULL argument");
+    Alloc a{al, (cudaStream_t)stream};
+    return transpose_impl(in, out, a);
+}
+
+amgt_status amgt_mbsr_wrap(int64_t m, int64_t n, int64_t blc_num, int64_t* blc_ptr, int32_t* blc_idx,
+                           uint16_t* blc_map, void* blc_val, amgt_prec prec, amgt_mbsr* out) {
+    if (!out || m < 0 || n < 0 || blc_num < 0 || !prec_valid(prec)) return fail(AMGT_ERR_ARG, "amgt_mbsr_wrap: bad argument");
+    *out = amgt_mbsr{};
+    out->m = m;
+    out->n = n;
+    out->blc_row = ceil_div(m, 4);
+    out->blc_col = ceil_div(n, 4);
+    out->blc_num = blc_num;
+    out->blc_ptr = blc_ptr;
+    out->blc_idx = blc_idx;
+    out->blc_map = blc_map;
+    out->blc_val = blc_val;
+    out->prec = prec;
+    return AMGT_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,245 @@
+// runtime.cu — error reporting, allocator glue, device prefix sum, timing/launch counters.
+#include <atomic>
+#include <cstdarg>
+#include <mutex>
+#include <vector>
+
+#include "common.cuh"
+
+namespace amgt {
+
+static thread_local char g_err[1024] = "";
+
+void set_error(const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+amgt_status fail(amgt_status st, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return st;
+}
+
+void* Alloc::get(size_t bytes) {
+    if (bytes == 0) bytes = 16;
+    if (al && al->alloc) return al->alloc(bytes, (void*)s, al->ctx);
+    void* p = nullptr;
+    if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return p;
+}
+
+void Alloc::put(void* p, size_t bytes) {
+    if (!p) return;
+    if (bytes == 0) bytes = 16;
+    if (al && al->free) {
+        al->free(p, bytes, (void*)s, al->ctx);
+        return;
+    }
+    cudaFreeAsync(p, s);
+}
+
+size_t prec_bytes(amgt_prec p) { return p == AMGT_FP64 ? 8 : (p == AMGT_FP32 ? 4 : 2); }
+
+int num_sms() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+int g_tc_thr_spgemm = 10;  // paper: POPCOUNT(mapA) >= 10 (L157)
+int g_tc_thr_spmv = 17;    // see DESIGN.md: TC SpMV route off by default on B200 (DMMA = DFMA rate)
+
+// ------------------------------------------------------------------ scan
+// Block-wide exclusive scan: 1024 threads x 8 items = 8192 items per block.
+constexpr int SCAN_T = 1024, SCAN_I = 8, SCAN_TILE = SCAN_T * SCAN_I;
+
+__device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t* sh_warp, int64_t* total) {
+    int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int64_t x = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        int64_t y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= d) x += y;
+    }
+    if (lane == 31) sh_warp[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        int64_t s = (lane < (int)(blockDim.x >> 5)) ? sh_warp[lane] : 0;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            int64_t y = __shfl_up_sync(0xffffffffu, s, d);
+            if (lane >= d) s += y;
+        }
+        sh_warp[lane] = s;  // inclusive warp-sum prefix
+    }
+    __syncthreads();
+    int64_t base = (w > 0) ? sh_warp[w - 1] : 0;
+    if (total) *total = sh_warp[(blockDim.x >> 5) - 1];
+    int64_t r = base + x - v;
+    __syncthreads();
+    return r;
+}
+
+__global__ void k_scan_reduce(const int64_t* __restrict__ in, int64_t n, int64_t* __restrict__ bsum) {
+    __shared__ int64_t sh[32];
+    int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_I;
+    int64_t s = 0;
+#pragma unroll
+    for (int i = 0; i < SCAN_I; ++i)
+        if (base + i < n) s += in[base + i];
+    int64_t tot;
+    block_excl_scan(s, sh, &tot);
+    if (threadIdx.x == 0) bsum[blockIdx.x] = tot;
+}
+
+// Scan of `in` (n items) into out (out[0]=0 ... out[n]) adding boff[blockIdx] (exclusive
+// block offsets, or nullptr).
+__global__ void k_scan_tile(const int64_t* __restrict__ in, int64_t n, const int64_t* __restrict__ boff,
+                            int64_t* __restrict__ out) {
+    __shared__ int64_t sh[32];
+    int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_I;
+    int64_t v[SCAN_I];
+    int64_t s = 0;
+#pragma unroll
+    for (int i = 0; i < SCAN_I; ++i) {
+        v[i] = (base + i < n) ? in[base + i] : 0;
+        s += v[i];
+    }
+    int64_t tot;
+    int64_t off = block_excl_scan(s, sh, &tot) + (boff ? boff[blockIdx.x] : 0);
+    if (blockIdx.x == 0 && threadIdx.x == 0) out[0] = 0;
+#pragma unroll
+    for (int i = 0; i < SCAN_I; ++i) {
+        off += v[i];
+        if (base + i < n) out[base + i + 1] = off;
+    }
+}
+
+amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a, cudaStream_t s) {
+    if (n <= 0) {
+        AMGT_CUDA(cudaMemsetAsync(out, 0, sizeof(int64_t), s));
+        return AMGT_OK;
+    }
+    int64_t nb = ceil_div(n, SCAN_TILE);
+    if (nb == 1) {
+        k_scan_tile<<<1, SCAN_T, 0, s>>>(in, n, nullptr, out);
+        AMGT_LAUNCHED();
+        return AMGT_OK;
+    }
+    Scratch<int64_t> bsum, boff;
+    AMGT_TRY(bsum.init(a, nb));
+    AMGT_TRY(boff.init(a, nb + 1));
+    k_scan_reduce<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, bsum.p);
+    AMGT_LAUNCHED();
+    AMGT_TRY(scan_exclusive(bsum.p, boff.p, nb, a, s));
+    k_scan_tile<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, boff.p, out);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+// ------------------------------------------------------------------ instrumentation
+static std::atomic<int64_t> g_launches{0};
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+struct TimerRec {
+    int cls;
+    double bytes;
+    cudaEvent_t e0, e1;
+};
+static std::mutex g_tmu;
+static bool g_timing = false;
+static std::vector<TimerRec> g_recs;
+static std::vector<cudaEvent_t> g_pool;
+static size_t g_used = 0;
+
+static cudaEvent_t pool_event() {
+    if (g_used < g_pool.size()) return g_pool[g_used++];
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    g_pool.push_back(e);
+    ++g_used;
+    return e;
+}
+
+TimerScope::TimerScope(int c, double b, cudaStream_t st) : cls(c), bytes(b), s(st), slot(-1) {
+    if (!g_timing) return;
+    std::lock_guard<std::mutex> lk(g_tmu);
+    TimerRec r{c, b, pool_event(), pool_event()};
+    cudaEventRecord(r.e0, s);
+    g_recs.push_back(r);
+    slot = (int)g_recs.size() - 1;
+}
+
+TimerScope::~TimerScope() {
+    if (slot < 0) return;
+    std::lock_guard<std::mutex> lk(g_tmu);
+    g_recs[slot].bytes = bytes;
+    cudaEventRecord(g_recs[slot].e1, s);
+}
+
+}  // namespace amgt
+
+using namespace amgt;
+
+extern "C" {
+
+const char* amgt_last_error(void) { return amgt::g_err; }
+
+const char* amgt_version(void) { return "amgt-b200 0.1 (sm_100a)"; }
+
+amgt_status amgt_set_tc_threshold(int spgemm_threshold, int spmv_threshold) {
+    if (spgemm_threshold < 0 || spgemm_threshold > 17 || spmv_threshold < 0 || spmv_threshold > 17)
+        return fail(AMGT_ERR_ARG, "thresholds must be in [0, 17]");
+    g_tc_thr_spgemm = spgemm_threshold;
+    g_tc_thr_spmv = spmv_threshold;
+    return AMGT_OK;
+}
+
+amgt_status amgt_timing_enable(int on) {
+    std::lock_guard<std::mutex> lk(g_tmu);
+    g_timing = on != 0;
+    return AMGT_OK;
+}
+
+amgt_status amgt_timing_reset(void) {
+    std::lock_guard<std::mutex> lk(g_tmu);
+    g_recs.clear();
+    g_used = 0;
+    g_launches.store(0);
+    return AMGT_OK;
+}
+
+amgt_status amgt_timing_read(double* ms_total_host, int64_t* launches_host, double* bytes_host) {
+    std::lock_guard<std::mutex> lk(g_tmu);
+    for (int c = 0; c < AMGT_TIMER_CLASSES; ++c) {
+        if (ms_total_host) ms_total_host[c] = 0;
+        if (launches_host) launches_host[c] = 0;
+        if (bytes_host) bytes_host[c] = 0;
+    }
+    for (auto& r : g_recs) {
+        if (cudaEventSynchronize(r.e1) != cudaSuccess) return fail(AMGT_ERR_CUDA, "event sync failed");
+        float ms = 0;
+        cudaEventElapsedTime(&ms, r.e0, r.e1);
+        if (ms_total_host) ms_total_host[r.cls] += ms;
+        if (launches_host) launches_host[r.cls] += 1;
+        if (bytes_host) bytes_host[r.cls] += r.bytes;
+    }
+    return AMGT_OK;
+}
+
+int64_t amgt_launch_count(void) { return g_launches.load(); }
+
+}  // extern "C"

@@ -1,0 +1,913 @@
+// spgemm.cu — C = A*B over mBSR (§IV.C; Alg. 3; Alg. 4).
+//
+// Pipeline (all on the device; host syncs: bin sizes, then the C tile count, L153):
+//   k_analyze     Cub_per_row(I) = sum_{K in A(I,:)} #tiles(B(K,:)) and bin(I) (L149-151;
+//                 8 bins, edges 128*2^b, reading R7); also the pair statistics.
+//   k_bin_*       row lists per bin (stable order irrelevant: rows are independent).
+//   step 1        per bin: distinct tile columns J with BITMAPMULTIPLY(mapA, mapB) != 0
+//                 (Alg. 3 lines 1-13) -> nnzC_row; prefix sum -> blc_ptrC; allocation.
+//   step 2        per bin: insert again, OR the bitmaps (R15), compress, sort ascending
+//                 (Alg. 3 lines 13-14) -> blc_idxC, blc_mapC.
+//   numeric       one warp per C block row (L155).  A tiles with POPCOUNT >= threshold go
+//                 to the tensor-core route (DMMA m8n8k4: fragA = [A;A], fragB = [Bj|Bj'],
+//                 keep the two diagonal quadrants, L157-171); the others to CUDA cores,
+//                 one lane per (A tile, B tile) pair (L173).  Accumulation in shared
+//                 memory for rows with <= 32 C tiles, in global memory (conflict-free, one
+//                 A tile at a time) for longer rows.  Deterministic.
+//
+// Hash tables (R8): power-of-two, >= 2x the bin's Cub upper bound, multiplicative hash,
+// linear probing.  Bins 0-1: one warp per row, table per warp; bins 2-6: one block per
+// row, table per block; bin 7 (Cub >= 8192): dense bitmap over B's tile columns
+// (shared memory when it fits, else a per-block global slice) — sorted by construction.
+#include <algorithm>
+#include <climits>
+
+#include "common.cuh"
+
+namespace amgt {
+
+amgt_status mbsr_alloc(amgt_mbsr* M, int64_t m, int64_t n, int64_t T, amgt_prec prec, Alloc& a, bool structure,
+                       bool values, int64_t* existing_ptr);
+amgt_status mbsr_release(amgt_mbsr* M, Alloc& a);
+
+constexpr int NBINS = 8;
+constexpr int EMPTY_KEY = -1;
+
+struct SymCtx {  // device pointers shared by the symbolic kernels
+    const int64_t* aptr;
+    const int32_t* aidx;
+    const uint16_t* amap;
+    const int64_t* bptr;
+    const int32_t* bidx;
+    const uint16_t* bmap;
+};
+
+// ---------------------------------------------------------------- analysis + binning
+__global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, unsigned long long* __restrict__ stats,
+                          int tc_thr) {
+    // stats: [0..7] bin counts, [8] cub_total, [9] pairs_nonzero, [10] pairs_tc, [11] scalar products
+    __shared__ unsigned long long sh[12];
+    if (threadIdx.x < 12) sh[threadIdx.x] = 0;
+    __syncthreads();
+    unsigned long long cubs = 0, pnz = 0, ptc = 0, sp = 0;
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+        int64_t cub = 0;
+        for (int64_t t = c.aptr[I]; t < c.aptr[I + 1]; ++t) {
+            const int32_t K = c.aidx[t];
+            const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
+            cub += b1 - b0;
+            const uint32_t ma = c.amap[t];
+            const bool tc = __popc(ma) >= tc_thr;
+            for (int64_t j = b0; j < b1; ++j) {  // pair statistics (info only)
+                const uint32_t mb = c.bmap[j];
+                if (bitmap_multiply(ma, mb)) {
+                    ++pnz;
+                    ptc += tc;
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) sp += __popc((ma >> k) & 0x1111u) * __popc((mb >> (4 * k)) & 0xFu);
+                }
+            }
+        }
+        int b = 0;
+        while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
+        bin_of[I] = b;
+        atomicAdd(&sh[b], 1ull);
+        cubs += cub;
+    }
+    atomicAdd(&sh[8], cubs);
+    atomicAdd(&sh[9], pnz);
+    atomicAdd(&sh[10], ptc);
+    atomicAdd(&sh[11], sp);
+    __syncthreads();
+    if (threadIdx.x < 12 && sh[threadIdx.x]) atomicAdd(&stats[threadIdx.x], sh[threadIdx.x]);
+}
+
+__global__ void k_bin_scatter(int64_t BR, const int64_t* __restrict__ bin_of, const unsigned long long* __restrict__ stats,
+                              unsigned long long* __restrict__ cursor, int32_t* __restrict__ rows) {
+    __shared__ unsigned long long off[NBINS];
+    if (threadIdx.x == 0) {
+        unsigned long long s = 0;
+        for (int b = 0; b < NBINS; ++b) { off[b] = s; s += stats[b]; }
+    }
+    __syncthreads();
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+        const int b = (int)bin_of[I];
+        rows[off[b] + atomicAdd(&cursor[b], 1ull)] = (int32_t)I;
+    }
+}
+
+// ---------------------------------------------------------------- hashing
+__device__ __forceinline__ uint32_t hash_slot(int32_t J, int logS) {
+    return ((uint32_t)J * 0x9E3779B1u) >> (32 - logS);
+}
+
+// Returns true when J was newly inserted.
+__device__ __forceinline__ bool hash_insert(int* keys, uint32_t* maps, int logS, int32_t J, uint32_t mapC, bool or_map) {
+    const uint32_t mask = (1u << logS) - 1u;
+    uint32_t h = hash_slot(J, logS);
+    for (;;) {
+        const int k = ((volatile int*)keys)[h];
+        if (k == J) {
+            if (or_map) atomicOr(maps + h, mapC);
+            return false;
+        }
+        if (k == EMPTY_KEY) {
+            const int old = atomicCAS(keys + h, EMPTY_KEY, J);
+            if (old == EMPTY_KEY || old == J) {
+                if (or_map) atomicOr(maps + h, mapC);
+                return old == EMPTY_KEY;
+            }
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+// Warp-cooperative enumeration of the (A tile, B tile) pairs of block row I: lanes take
+// up to 32 A tiles, warp-scan their B-row lengths, then spread the pairs over lanes.
+// fn(J, mapC) is called for every pair with mapC != 0.
+template <typename F>
+__device__ __forceinline__ void warp_pairs(const SymCtx& c, int64_t I, int lane, F&& fn) {
+    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+    for (int64_t base = a0; base < a1; base += 32) {
+        const int64_t t = base + lane;
+        const bool v = t < a1;
+        const int32_t K = v ? c.aidx[t] : 0;
+        const uint32_t ma = v ? c.amap[t] : 0u;
+        const int64_t b0 = v ? c.bptr[K] : 0;
+        const int64_t len = v ? c.bptr[K + 1] - b0 : 0;
+        int64_t incl = len;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        const int64_t excl = incl - len;
+        const int64_t total = __shfl_sync(0xffffffffu, incl, 31);
+        for (int64_t p0 = 0; p0 < total; p0 += 32) {
+            const int64_t p = p0 + lane;
+            int lo = 0;
+#pragma unroll
+            for (int step = 16; step; step >>= 1) {
+                const int cand = lo + step;
+                const int64_t e = __shfl_sync(0xffffffffu, excl, cand & 31);
+                if (cand < 32 && e <= p) lo = cand;
+            }
+            const int64_t ob0 = __shfl_sync(0xffffffffu, b0, lo);
+            const int64_t oex = __shfl_sync(0xffffffffu, excl, lo);
+            const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
+            if (p < total) {
+                const int64_t j = ob0 + (p - oex);
+                const uint32_t mc = bitmap_multiply(oma, c.bmap[j]);
+                if (mc) fn(c.bidx[j], mc);
+            }
+        }
+    }
+}
+
+// Block-cooperative version: chunks of blockDim A tiles, owner search in shared memory.
+template <typename F>
+__device__ __forceinline__ void block_pairs(const SymCtx& c, int64_t I, int64_t* sh_excl, int64_t* sh_b0,
+                                            uint32_t* sh_ma, int64_t* sh_tot, F&& fn) {
+    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+    const int nt = blockDim.x, tid = threadIdx.x;
+    const int lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    for (int64_t base = a0; base < a1; base += nt) {
+        const int64_t t = base + tid;
+        const bool v = t < a1;
+        const int32_t K = v ? c.aidx[t] : 0;
+        const uint32_t ma = v ? c.amap[t] : 0u;
+        const int64_t b0 = v ? c.bptr[K] : 0;
+        const int64_t len = v ? c.bptr[K + 1] - b0 : 0;
+        // block exclusive scan of len (warp scans + warp totals in sh_tot)
+        int64_t incl = len;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        if (lane == 31) sh_tot[w] = incl;
+        __syncthreads();
+        if (tid == 0) {
+            int64_t s = 0;
+            for (int k = 0; k < nw; ++k) { const int64_t x = sh_tot[k]; sh_tot[k] = s; s += x; }
+            sh_tot[nw] = s;
+        }
+        __syncthreads();
+        const int64_t excl = sh_tot[w] + incl - len;
+        sh_excl[tid] = excl;
+        sh_b0[tid] = b0;
+        sh_ma[tid] = ma;
+        const int64_t total = sh_tot[nw];
+        __syncthreads();
+        const int nvalid = (int)min((int64_t)nt, a1 - base);
+        for (int64_t p = tid; p < total; p += nt) {
+            int lo = 0, hi = nvalid - 1;  // largest o with excl[o] <= p
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (sh_excl[mid] <= p) lo = mid; else hi = mid - 1;
+            }
+            const int64_t j = sh_b0[lo] + (p - sh_excl[lo]);
+            const uint32_t mc = bitmap_multiply(sh_ma[lo], c.bmap[j]);
+            if (mc) fn(c.bidx[j], mc);
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------- step kernels: warp bins
+// LOGS = log2(table slots per warp).  STEP 1: count -> nnz_row[I].  STEP 2: write sorted
+// idx/map at ptrC[I].
+template <int LOGS, int STEP>
+__global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
+                                                  int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
+                                                  int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
+    constexpr int S = 1 << LOGS;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int* keys = reinterpret_cast<int*>(smem_raw) + w * 2 * S;
+    uint32_t* maps = reinterpret_cast<uint32_t*>(keys + S);
+    const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (wg >= nrows) return;
+    const int64_t I = rows[wg];
+    for (int i = lane; i < S; i += 32) {
+        keys[i] = EMPTY_KEY;
+        maps[i] = 0;
+    }
+    __syncwarp();
+    int cnt = 0;
+    warp_pairs(c, I, lane, [&](int32_t J, uint32_t mc) { cnt += hash_insert(keys, maps, LOGS, J, mc, STEP == 2); });
+    __syncwarp();
+    if (STEP == 1) {
+#pragma unroll
+        for (int d = 16; d; d >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, d);
+        if (lane == 0) nnz_row[I] = cnt;
+        return;
+    }
+    // compress in place (rounds of 32 slots; all reads of a round precede its writes)
+    int n = 0;
+    for (int base = 0; base < S; base += 32) {
+        const int k = keys[base + lane];
+        const uint32_t mp = maps[base + lane];
+        const bool v = k != EMPTY_KEY;
+        const uint32_t bal = __ballot_sync(0xffffffffu, v);
+        __syncwarp();
+        if (v) {
+            const int pos = n + __popc(bal & ((1u << lane) - 1u));
+            keys[pos] = k;
+            maps[pos] = mp;
+        }
+        n += __popc(bal);
+        __syncwarp();
+    }
+    // rank sort (n <= S/2 distinct keys)
+    const int64_t out = cptr[I];
+    for (int i = lane; i < n; i += 32) {
+        const int k = keys[i];
+        int rank = 0;
+        for (int j = 0; j < n; ++j) rank += keys[j] < k;
+        cidx[out + rank] = k;
+        cmap[out + rank] = (uint16_t)maps[i];
+    }
+}
+
+// ---------------------------------------------------------------- step kernels: block bins
+template <int LOGS, int STEP>
+__global__ void k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c, int64_t* __restrict__ nnz_row,
+                            const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
+    constexpr int S = 1 << LOGS;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    // layout: keys[S] | maps[S] | list u64[S/2] (step 2) ; pair-search scratch in static smem
+    int* keys = reinterpret_cast<int*>(smem_raw);
+    uint32_t* maps = reinterpret_cast<uint32_t*>(keys + S);
+    unsigned long long* list = reinterpret_cast<unsigned long long*>(maps + S);
+    __shared__ int64_t sh_excl[512], sh_b0[512], sh_tot[17];
+    __shared__ uint32_t sh_ma[512];
+    __shared__ int sh_cnt[17];
+    const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    for (int64_t rr = blockIdx.x; rr < nrows; rr += gridDim.x) {
+        const int64_t I = rows[rr];
+        for (int i = tid; i < S; i += nt) {
+            keys[i] = EMPTY_KEY;
+            maps[i] = 0;
+        }
+        __syncthreads();
+        int cnt = 0;
+        block_pairs(c, I, sh_excl, sh_b0, sh_ma, sh_tot,
+                    [&](int32_t J, uint32_t mc) { cnt += hash_insert(keys, maps, LOGS, J, mc, STEP == 2); });
+        __syncthreads();
+        if (STEP == 1) {
+#pragma unroll
+            for (int d = 16; d; d >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, d);
+            if (lane == 0) sh_cnt[w] = cnt;
+            __syncthreads();
+            if (tid == 0) {
+                int s = 0;
+                for (int k = 0; k < nw; ++k) s += sh_cnt[k];
+                nnz_row[I] = s;
+            }
+            __syncthreads();
+            continue;
+        }
+        // compress into list (packed key<<16 | map), block-wide ballot prefix per round
+        int n = 0;
+        for (int base = 0; base < S; base += nt) {
+            const int k = keys[base + tid];
+            const bool v = k != EMPTY_KEY;
+            const uint32_t bal = __ballot_sync(0xffffffffu, v);
+            if (lane == 0) sh_cnt[w] = __popc(bal);
+            __syncthreads();
+            if (tid == 0) {
+                int s = 0;
+                for (int q = 0; q < nw; ++q) { const int x = sh_cnt[q]; sh_cnt[q] = s; s += x; }
+                sh_cnt[nw] = s;
+            }
+            __syncthreads();
+            if (v) {
+                const int pos = n + sh_cnt[w] + __popc(bal & ((1u << lane) - 1u));
+                list[pos] = ((unsigned long long)(uint32_t)k << 16) | (maps[base + tid] & 0xFFFFu);
+            }
+            n += sh_cnt[nw];
+            __syncthreads();
+        }
+        int N = 1;
+        while (N < n) N <<= 1;
+        for (int i = n + tid; i < N; i += nt) list[i] = ~0ull;
+        __syncthreads();
+        for (int k = 2; k <= N; k <<= 1)  // bitonic sort, ascending
+            for (int j = k >> 1; j > 0; j >>= 1) {
+                for (int i = tid; i < N; i += nt) {
+                    const int ixj = i ^ j;
+                    if (ixj > i) {
+                        const unsigned long long a = list[i], b = list[ixj];
+                        const bool up = (i & k) == 0;
+                        if ((a > b) == up) { list[i] = b; list[ixj] = a; }
+                    }
+                }
+                __syncthreads();
+            }
+        const int64_t out = cptr[I];
+        for (int i = tid; i < n; i += nt) {
+            const unsigned long long e = list[i];
+            cidx[out + i] = (int32_t)(e >> 16);
+            cmap[out + i] = (uint16_t)(e & 0xFFFFu);
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------- step kernels: bin 7 (dense bitmap)
+template <int STEP>
+__global__ void __launch_bounds__(512) k_sym_dense(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
+                                                   int64_t W, uint32_t* __restrict__ gws, int64_t* __restrict__ nnz_row,
+                                                   const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx,
+                                                   uint16_t* __restrict__ cmap) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ int64_t sh_excl[512], sh_b0[512], sh_tot[17];
+    __shared__ uint32_t sh_ma[512];
+    __shared__ long long sh_sum[17];
+    uint32_t* bm;
+    uint32_t* pre;
+    if (gws) {
+        bm = gws + (int64_t)blockIdx.x * 2 * W;
+        pre = bm + W;
+    } else {
+        bm = reinterpret_cast<uint32_t*>(smem_raw);
+        pre = bm + W;
+    }
+    const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    for (int64_t rr = blockIdx.x; rr < nrows; rr += gridDim.x) {
+        const int64_t I = rows[rr];
+        for (int64_t i = tid; i < W; i += nt) bm[i] = 0;
+        __syncthreads();
+        block_pairs(c, I, sh_excl, sh_b0, sh_ma, sh_tot,
+                    [&](int32_t J, uint32_t) { atomicOr(bm + (J >> 5), 1u << (J & 31)); });
+        __syncthreads();
+        // per-thread contiguous word ranges -> block scan of popcounts
+        const int64_t per = (W + nt - 1) / nt;
+        const int64_t w0 = min(W, per * (int64_t)tid), w1 = min(W, w0 + per);
+        long long s = 0;
+        for (int64_t i = w0; i < w1; ++i) s += __popc(bm[i]);
+        long long incl = s;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const long long y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        if (lane == 31) sh_sum[w] = incl;
+        __syncthreads();
+        if (tid == 0) {
+            long long a = 0;
+            for (int k = 0; k < nw; ++k) { const long long x = sh_sum[k]; sh_sum[k] = a; a += x; }
+            sh_sum[nw] = a;
+        }
+        __syncthreads();
+        if (STEP == 1) {
+            if (tid == 0) nnz_row[I] = sh_sum[nw];
+            __syncthreads();
+            continue;
+        }
+        long long run = sh_sum[w] + incl - s;
+        const int64_t out = cptr[I];
+        for (int64_t i = w0; i < w1; ++i) {
+            pre[i] = (uint32_t)run;
+            uint32_t bits = bm[i];
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                bits &= bits - 1;
+                cidx[out + run] = (int32_t)(32 * i + b);
+                ++run;
+            }
+        }
+        __syncthreads();
+        block_pairs(c, I, sh_excl, sh_b0, sh_ma, sh_tot, [&](int32_t J, uint32_t mc) {
+            const int64_t q = out + pre[J >> 5] + __popc(bm[J >> 5] & ((1u << (J & 31)) - 1u));
+            atomicOr(reinterpret_cast<unsigned int*>(cmap) + (q >> 1), mc << (16 * (q & 1)));
+        });
+        __syncthreads();
+    }
+}
+
+__global__ void k_numeric_rows_stats(int64_t BR, const int64_t* __restrict__ cptr, unsigned long long* __restrict__ out) {
+    unsigned long long a = 0, b = 0, e = 0;
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t n = cptr[I + 1] - cptr[I];
+        if (n == 0) ++e; else if (n <= 32) ++a; else ++b;
+    }
+    atomicAdd(out, a);
+    atomicAdd(out + 1, b);
+    atomicAdd(out + 2, e);
+}
+
+// ---------------------------------------------------------------- numeric
+template <typename T> struct TileIO;
+template <> struct TileIO<double> {
+    static __device__ __forceinline__ void load(const double* p, double (&v)[16]) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const double2 d = __ldg(reinterpret_cast<const double2*>(p) + i);
+            v[2 * i] = d.x;
+            v[2 * i + 1] = d.y;
+        }
+    }
+};
+template <> struct TileIO<float> {
+    static __device__ __forceinline__ void load(const float* p, float (&v)[16]) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const float4 d = __ldg(reinterpret_cast<const float4*>(p) + i);
+            v[4 * i] = d.x; v[4 * i + 1] = d.y; v[4 * i + 2] = d.z; v[4 * i + 3] = d.w;
+        }
+    }
+};
+template <> struct TileIO<__half> {
+    static __device__ __forceinline__ void load(const __half* p, float (&v)[16]) {
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+            const uint4 u = __ldg(reinterpret_cast<const uint4*>(p) + i);
+            const uint32_t w[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w[k]));
+                v[8 * i + 2 * k] = f.x;
+                v[8 * i + 2 * k + 1] = f.y;
+            }
+        }
+    }
+};
+
+// C tile += A tile * B tile on CUDA cores (64 FMAs, fixed order k = 0..3).
+template <typename Acc>
+__device__ __forceinline__ void tile_mma(const Acc (&a)[16], const Acc (&b)[16], Acc (&c)[16]) {
+#pragma unroll
+    for (int r = 0; r < 4; ++r)
+#pragma unroll
+        for (int col = 0; col < 4; ++col) {
+            Acc s = a[4 * r] * b[col];
+            s = fma(a[4 * r + 1], b[4 + col], s);
+            s = fma(a[4 * r + 2], b[8 + col], s);
+            s = fma(a[4 * r + 3], b[12 + col], s);
+            c[4 * r + col] = s;
+        }
+}
+
+__device__ __forceinline__ int bsearch_row(const int32_t* idx, int n, int32_t J) {
+    int lo = 0, hi = n - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (idx[mid] < J) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+constexpr int NUM_WARPS = 4;
+constexpr int CAP = 32;  // C tiles per row accumulated in shared memory
+
+template <typename Acc> struct NumSmem {
+    Acc acc[CAP][16];
+    Acc stage[32][16];
+    int32_t cidx[CAP];
+};
+
+// DMMA m8n8k4 FP64 (sm_80+ DMMA; native DMMA.8x8x4 on sm_100a).
+__device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                 : "+d"(c0), "+d"(c1)
+                 : "d"(a), "d"(b));
+}
+
+// T = storage type, Acc = accumulation type (double for FP64, float otherwise).
+// gacc: FP32 accumulation workspace for FP16 global-path rows (indexed like C values).
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(int64_t BR, SymCtx c, const T* __restrict__ aval,
+                                                            const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                            const int32_t* __restrict__ cidx_g,
+                                                            const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+                                                            Acc* __restrict__ gacc, int tc_thr) {
+    __shared__ NumSmem<Acc> sm[NUM_WARPS];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t I = (int64_t)blockIdx.x * NUM_WARPS + w;
+    if (I >= BR) return;
+    NumSmem<Acc>& S = sm[w];
+    const int64_t c0 = cptr[I];
+    const int nC = (int)(cptr[I + 1] - c0);
+    if (nC == 0) return;
+    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+    const bool small = nC <= CAP;
+    // accumulator access: smem for small rows, global (C values or FP32 workspace) otherwise
+    Acc* gbase = nullptr;
+    if (small) {
+        if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
+        for (int e = lane; e < CAP * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
+    } else {
+        gbase = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
+        for (int64_t e = lane; e < 16 * (int64_t)nC; e += 32) gbase[e] = Acc(0);
+    }
+    __syncwarp();
+    const int32_t* rowidx = small ? S.cidx : cidx_g + c0;
+    auto accp = [&](int q) -> Acc* { return small ? S.acc[q] : gbase + 16 * (int64_t)q; };
+
+    // ---- tensor-core route (FP64 only): A tiles with POPCOUNT >= tc_thr, one at a time.
+    if constexpr (sizeof(T) == 8) {
+        for (int64_t base = a0; base < a1; base += 32) {
+            const int64_t t = base + lane;
+            const uint32_t ma = t < a1 ? c.amap[t] : 0u;
+            uint32_t dense = __ballot_sync(0xffffffffu, t < a1 && __popc(ma) >= tc_thr);
+            while (dense) {
+                const int src = __ffs(dense) - 1;
+                dense &= dense - 1;
+                const int64_t ta = base + src;
+                const uint32_t mA = __shfl_sync(0xffffffffu, ma, src);
+                const int32_t K = c.aidx[ta];
+                // fragA[row][k] = A[row & 3][k]: lane l -> element (l>>2 & 3, l&3)
+                const double fa = (double)aval[16 * ta + 4 * ((lane >> 2) & 3) + (lane & 3)];
+                const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
+                for (int64_t jb = b0; jb < b1; jb += 32) {
+                    const int64_t j = jb + lane;
+                    const uint32_t mb = j < b1 ? c.bmap[j] : 0u;
+                    const uint32_t mc = j < b1 ? bitmap_multiply(mA, mb) : 0u;
+                    const int q = mc ? bsearch_row(rowidx, nC, c.bidx[j]) : -1;
+                    uint32_t valid = __ballot_sync(0xffffffffu, mc != 0);
+                    while (valid) {
+                        const int l1 = __ffs(valid) - 1;
+                        valid &= valid - 1;
+                        int l2 = -1;
+                        if (valid) { l2 = __ffs(valid) - 1; valid &= valid - 1; }
+                        const int q1 = __shfl_sync(0xffffffffu, q, l1);
+                        const int q2 = __shfl_sync(0xffffffffu, q, l2 < 0 ? l1 : l2);
+                        // fragB[k][n]: lane l -> (k = l&3, n = l>>2); n<4 -> B_j1[k][n], else B_j2[k][n-4]
+                        const int n8 = lane >> 2, k4 = lane & 3;
+                        double fb = 0.0;
+                        if (n8 < 4) fb = (double)bval[16 * (jb + l1) + 4 * k4 + n8];
+                        else if (l2 >= 0) fb = (double)bval[16 * (jb + l2) + 4 * k4 + (n8 - 4)];
+                        double d0 = 0.0, d1 = 0.0;
+                        dmma(d0, d1, fa, fb);
+                        // C[g][2t..2t+1] in lane 4g+t; quadrant (0:4,0:4) -> tile q1, (4:8,4:8) -> q2
+                        if (n8 < 4 && k4 < 2) {
+                            Acc* p = accp(q1) + 4 * n8 + 2 * k4;
+                            p[0] += d0;
+                            p[1] += d1;
+                        } else if (n8 >= 4 && k4 >= 2 && l2 >= 0) {
+                            Acc* p = accp(q2) + 4 * (n8 - 4) + 2 * (k4 - 2);
+                            p[0] += d0;
+                            p[1] += d1;
+                        }
+                        __syncwarp();
+                    }
+                }
+            }
+        }
+    }
+
+    // ---- CUDA-core route: pairs of the remaining A tiles.
+    const int thr = (sizeof(T) == 8) ? tc_thr : 17;
+    if (small) {
+        // flattened pairs, conflicts resolved per round by match_any (deterministic)
+        for (int64_t base = a0; base < a1; base += 32) {
+            const int64_t t = base + lane;
+            const bool v = t < a1;
+            const uint32_t ma = v ? c.amap[t] : 0u;
+            const bool sp = v && __popc(ma) < thr;
+            const int32_t K = sp ? c.aidx[t] : 0;
+            const int64_t b0 = sp ? c.bptr[K] : 0;
+            const int64_t len = sp ? c.bptr[K + 1] - b0 : 0;
+            int64_t incl = len;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                if (lane >= d) incl += y;
+            }
+            const int64_t excl = incl - len;
+            const int64_t total = __shfl_sync(0xffffffffu, incl, 31);
+            for (int64_t p0 = 0; p0 < total; p0 += 32) {
+                const int64_t p = p0 + lane;
+                int lo = 0;
+#pragma unroll
+                for (int step = 16; step; step >>= 1) {
+                    const int cand = lo + step;
+                    const int64_t e = __shfl_sync(0xffffffffu, excl, cand & 31);
+                    if (cand < 32 && e <= p) lo = cand;
+                }
+                const int64_t ob0 = __shfl_sync(0xffffffffu, b0, lo);
+                const int64_t oex = __shfl_sync(0xffffffffu, excl, lo);
+                const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
+                const int64_t ot = base + lo;
+                int q = -1;
+                Acc prod[16];
+                if (p < total) {
+                    const int64_t j = ob0 + (p - oex);
+                    const uint32_t mc = bitmap_multiply(oma, c.bmap[j]);
+                    if (mc) {
+                        q = bsearch_row(rowidx, nC, c.bidx[j]);
+                        Acc av[16], bv[16];
+                        TileIO<T>::load(aval + 16 * ot, av);
+                        TileIO<T>::load(bval + 16 * j, bv);
+                        tile_mma(av, bv, prod);
+                    }
+                }
+                const uint32_t peers = __match_any_sync(0xffffffffu, q);
+                const bool alone = __popc(peers) == 1;
+                if (q >= 0 && alone) {
+#pragma unroll
+                    for (int e = 0; e < 16; ++e) S.acc[q][e] += prod[e];
+                }
+                const bool shared = q >= 0 && !alone;
+                if (__any_sync(0xffffffffu, shared)) {
+                    if (shared) {
+#pragma unroll
+                        for (int e = 0; e < 16; ++e) S.stage[lane][e] = prod[e];
+                    }
+                    __syncwarp();
+                    if (shared && (__ffs(peers) - 1) == lane) {  // leader: add peers in lane order
+                        uint32_t pm = peers;
+                        while (pm) {
+                            const int src = __ffs(pm) - 1;
+                            pm &= pm - 1;
+#pragma unroll
+                            for (int e = 0; e < 16; ++e) S.acc[q][e] += S.stage[src][e];
+                        }
+                    }
+                }
+                __syncwarp();
+            }
+        }
+    } else {
+        // global accumulation: one sparse A tile at a time, lanes over its B row (distinct C tiles)
+        for (int64_t t = a0; t < a1; ++t) {
+            const uint32_t ma = c.amap[t];
+            if (__popc(ma) >= thr) continue;
+            const int32_t K = c.aidx[t];
+            Acc av[16];
+            TileIO<T>::load(aval + 16 * t, av);
+            const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
+            for (int64_t j = b0 + lane; j < b1; j += 32) {
+                const uint32_t mc = bitmap_multiply(ma, c.bmap[j]);
+                if (!mc) continue;
+                const int q = bsearch_row(rowidx, nC, c.bidx[j]);
+                Acc bv[16], prod[16];
+                TileIO<T>::load(bval + 16 * j, bv);
+                tile_mma(av, bv, prod);
+                Acc* p = gbase + 16 * (int64_t)q;
+#pragma unroll
+                for (int e = 0; e < 16; ++e) p[e] += prod[e];
+            }
+            __syncwarp();
+        }
+    }
+    __syncwarp();
+    // ---- write out, +0.0 where the bitmap bit is clear (R2)
+    for (int64_t e = lane; e < 16 * (int64_t)nC; e += 32) {
+        const int q = (int)(e >> 4), b = (int)(e & 15);
+        const bool bit = (cmap_g[c0 + q] >> b) & 1u;
+        const Acc v = small ? S.acc[q][b] : gbase[e];
+        cval[16 * c0 + e] = bit ? from_acc<T>(v) : from_acc<T>(Acc(0));
+    }
+}
+
+static unsigned capped(int64_t blocks) {
+    const int64_t cap = (int64_t)num_sms() * 32;
+    return (unsigned)(blocks < 1 ? 1 : (blocks > cap ? cap : blocks));
+}
+
+template <int LOGS, int STEP>
+static amgt_status launch_warp_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t* nnz_row, const int64_t* cptr,
+                                   int32_t* cidx, uint16_t* cmap, cudaStream_t s) {
+    if (n == 0) return AMGT_OK;
+    const size_t sm = (size_t)8 * 2 * (1 << LOGS) * sizeof(int);
+    auto kern = k_sym_warp<LOGS, STEP>;
+    if (sm > 48 * 1024) AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    kern<<<(unsigned)ceil_div(n * 32, 256), 256, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+template <int LOGS, int STEP>
+static amgt_status launch_block_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t* nnz_row,
+                                    const int64_t* cptr, int32_t* cidx, uint16_t* cmap, cudaStream_t s) {
+    if (n == 0) return AMGT_OK;
+    constexpr int S = 1 << LOGS;
+    const size_t sm = (size_t)S * 4 * 2 + (STEP == 2 ? (size_t)S / 2 * 8 : 0);
+    const int threads = LOGS >= 12 ? 512 : 256;
+    auto kern = k_sym_block<LOGS, STEP>;
+    AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    kern<<<capped(n), threads, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+template <int STEP>
+static amgt_status launch_dense_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t BCB, Alloc& a,
+                                    int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
+                                    cudaStream_t s) {
+    if (n == 0) return AMGT_OK;
+    const int64_t W = ceil_div(BCB, 32);
+    const size_t need = (size_t)W * 2 * sizeof(uint32_t);
+    auto kern = k_sym_dense<STEP>;
+    const size_t max_dyn = 160 * 1024;
+    if (need <= max_dyn) {
+        AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)need));
+        kern<<<capped(n), 512, need, s>>>(n, rows, c, W, nullptr, nnz_row, cptr, cidx, cmap);
+        AMGT_LAUNCHED();
+    } else {
+        const int64_t G = std::min<int64_t>(n, (int64_t)num_sms());
+        Scratch<uint32_t> ws;
+        AMGT_TRY(ws.init(a, (size_t)G * 2 * W));
+        kern<<<(unsigned)G, 512, 0, s>>>(n, rows, c, W, ws.p, nnz_row, cptr, cidx, cmap);
+        AMGT_LAUNCHED();
+    }
+    return AMGT_OK;
+}
+
+template <int STEP>
+static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_t* rows, const SymCtx& c, int64_t BCB,
+                            Alloc& a, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
+                            cudaStream_t s) {
+    AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY((launch_dense_bin<STEP>(cnt[7], rows + off[7], c, BCB, a, nnz_row, cptr, cidx, cmap, s)));
+    return AMGT_OK;
+}
+
+static double spgemm_bytes(const amgt_mbsr* A, const amgt_mbsr* B, const amgt_mbsr* C, bool values) {
+    const double s = values ? 16.0 * prec_bytes(A->prec) : 0.0;
+    return (A->blc_num + B->blc_num + C->blc_num) * (s + 6.0) + (A->blc_row + B->blc_row + C->blc_row + 3) * 8.0;
+}
+
+amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* Cout, amgt_spgemm_info* info,
+                                 Alloc& a) {
+    cudaStream_t s = a.s;
+    if (A->n != B->m) return fail(AMGT_ERR_ARG, "SpGEMM: A.n (%lld) != B.m (%lld)", (long long)A->n, (long long)B->m);
+    if (A->prec != B->prec) return fail(AMGT_ERR_ARG, "SpGEMM: A and B precisions differ");
+    const int64_t BR = A->blc_row;
+    SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
+    Scratch<int64_t> bin_of, nnz_row;
+    Scratch<unsigned long long> stats, cursor;
+    Scratch<int32_t> rows;
+    AMGT_TRY(bin_of.init(a, BR + 1));
+    AMGT_TRY(nnz_row.init(a, BR + 1));
+    AMGT_TRY(stats.init(a, 16));
+    AMGT_TRY(cursor.init(a, NBINS));
+    AMGT_TRY(rows.init(a, BR + 1));
+    AMGT_CUDA(cudaMemsetAsync(stats.p, 0, 16 * sizeof(unsigned long long), s));
+    AMGT_CUDA(cudaMemsetAsync(cursor.p, 0, NBINS * sizeof(unsigned long long), s));
+    amgt_mbsr C{};
+    C.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
+    if (!C.blc_ptr) return fail(AMGT_ERR_ALLOC, "SpGEMM: blc_ptr allocation failed");
+    unsigned long long hs[16];
+    {
+        TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
+        if (BR > 0) {
+            k_analyze<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+            AMGT_LAUNCHED();
+            k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats.p, cursor.p, rows.p);
+            AMGT_LAUNCHED();
+        }
+        AMGT_CUDA(cudaMemcpyAsync(hs, stats.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));  // sync 1: bin sizes
+        int64_t cnt[NBINS], off[NBINS], acc = 0;
+        for (int b = 0; b < NBINS; ++b) { cnt[b] = (int64_t)hs[b]; off[b] = acc; acc += cnt[b]; }
+        if (BR > 0) {
+            amgt_status st = run_bins<1>(cnt, off, rows.p, c, B->blc_col, a, nnz_row.p, nullptr, nullptr, nullptr, s);
+            if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
+        }
+        AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s));
+        int64_t TC = 0;
+        AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));  // sync 2: C tile count (L153)
+        amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
+        if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+        if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
+        if (BR > 0) {
+            st = run_bins<2>(cnt, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
+            if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+        }
+        ts.bytes = (A->blc_num + B->blc_num) * 6.0 * 2 + (A->blc_row + B->blc_row) * 8.0 + TC * 6.0 + (BR + 1) * 8.0;
+    }
+    if (info) {
+        for (int b = 0; b < NBINS; ++b) info->bin_rows[b] = (int64_t)hs[b];
+        info->cub_total = (int64_t)hs[8];
+        info->pairs_nonzero = (int64_t)hs[9];
+        info->pairs_tc = (int64_t)hs[10];
+        info->scalar_products = (int64_t)hs[11];
+        Scratch<unsigned long long> nr;
+        AMGT_TRY(nr.init(a, 3));
+        AMGT_CUDA(cudaMemsetAsync(nr.p, 0, 3 * sizeof(unsigned long long), s));
+        if (BR > 0) {
+            k_numeric_rows_stats<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, C.blc_ptr, nr.p);
+            AMGT_LAUNCHED();
+        }
+        unsigned long long h3[3];
+        AMGT_CUDA(cudaMemcpyAsync(h3, nr.p, sizeof(h3), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+        for (int k = 0; k < 3; ++k) info->numeric_rows[k] = (int64_t)h3[k];
+    }
+    *Cout = C;
+    return AMGT_OK;
+}
+
+template <typename T, typename Acc>
+static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a) {
+    cudaStream_t s = a.s;
+    const int64_t BR = A->blc_row;
+    if (BR == 0 || C->blc_num == 0) return AMGT_OK;
+    SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
+    Scratch<Acc> gacc;
+    if (sizeof(T) < sizeof(Acc)) AMGT_TRY(gacc.init(a, 16 * (size_t)C->blc_num));
+    k_numeric<T, Acc><<<(unsigned)ceil_div(BR, NUM_WARPS), NUM_WARPS * 32, 0, s>>>(
+        BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
+        sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+amgt_status spgemm_numeric_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a) {
+    if (A->n != B->m || C->m != A->m || C->n != B->n) return fail(AMGT_ERR_ARG, "SpGEMM numeric: dimension mismatch");
+    if (A->prec != B->prec || C->prec != A->prec) return fail(AMGT_ERR_ARG, "SpGEMM numeric: precision mismatch");
+    TimerScope ts(TC_SPGEMM_NUM, spgemm_bytes(A, B, C, true), a.s);
+    switch (A->prec) {
+        case AMGT_FP64: return launch_numeric<double, double>(A, B, C, a);
+        case AMGT_FP32: return launch_numeric<float, float>(A, B, C, a);
+        default: return launch_numeric<__half, float>(A, B, C, a);
+    }
+}
+
+}  // namespace amgt
+
+using namespace amgt;
+
+extern "C" {
+
+amgt_status amgt_spgemm_symbolic(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, amgt_spgemm_info* info,
+                                 const amgt_allocator* al, void* stream) {
+    if (!A || !B || !C) return fail(AMGT_ERR_ARG, "amgt_spgemm_symbolic: NULL argument");
+    Alloc a{al, (cudaStream_t)stream};
+    return spgemm_symbolic_impl(A, B, C, info, a);
+}
+
+amgt_status amgt_spgemm_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, void* stream) {
+    if (!A || !B || !C) return fail(AMGT_ERR_ARG, "amgt_spgemm_numeric: NULL argument");
+    Alloc a{nullptr, (cudaStream_t)stream};
+    return spgemm_numeric_impl(A, B, C, a);
+}
+
+amgt_status amgt_rap(const amgt_mbsr* R, const amgt_mbsr* A, const amgt_mbsr* P, amgt_mbsr* Ac,
+                     const amgt_allocator* al, void* stream) {
+    if (!R || !A || !P || !Ac) return fail(AMGT_ERR_ARG, "amgt_rap: NULL argument");
+    Alloc a{al, (cudaStream_t)stream};
+    amgt_mbsr AP{};
+    AMGT_TRY(spgemm_symbolic_impl(A, P, &AP, nullptr, a));
+    amgt_status st = spgemm_numeric_impl(A, P, &AP, a);
+    if (st == AMGT_OK) st = spgemm_symbolic_impl(R, &AP, Ac, nullptr, a);
+    if (st == AMGT_OK) {
+        st = spgemm_numeric_impl(R, &AP, Ac, a);
+        if (st != AMGT_OK) mbsr_release(Ac, a);
+    }
+    mbsr_release(&AP, a);
+    return st;
+}
+
+}  // extern "C"

@@ -1,0 +1,508 @@
+// spmv.cu — y = A x over mBSR (§IV.D; Alg. 5; Fig. 5).
+//
+// B200 design (HBM-bound: 134 B per FP64 tile, <=1 flop/B):
+//  * Row kernel: a 4-lane group owns one block row, 8 block rows per warp (no cross-group
+//    reduction).  Per tile, each lane issues 128-bit loads only: FP64 lane q loads the
+//    16-B halves {16q, 64+16q} of the 128-B tile (so every load instruction of the
+//    group covers one contiguous 64-B span) plus one 16-B x segment; FP32 lane q loads
+//    its row (16 B); FP16 lane q loads its row (8 B).  Each lane multiplies only the
+//    entries whose bitmap bit is set (Alg. 5 lines 9-11, GETBIT).  Two tiles in flight
+//    per lane per iteration.
+//  * Load balancing (L220, Fig. 5): with a plan (amgt_spmv_analyze), block rows longer
+//    than WARP_CAPACITY = 64 tiles are split into 64-tile warp chunks (8 groups x 8
+//    tiles, Alg. 5 lines 4-6 with reading R12); each chunk reduces its 8 groups with
+//    shuffles and writes a partial; a combine kernel sums the partials of a row in chunk
+//    order (deterministic, no atomics).
+//  * Tensor-core route (L222-228, R14): tiles with popcount >= the SpMV threshold are
+//    multiplied with DMMA m8n8k4 two at a time inside the row kernel (FP64 only).  Off by
+//    default on B200 (DMMA rate == DFMA rate), enabled by
+//    amgt_set_tc_threshold.
+#include <climits>
+
+#include "common.cuh"
+
+namespace amgt {
+
+constexpr int WARP_CAPACITY = 64;  // tiles per warp chunk (L220)
+
+struct SpmvPlan {
+    int64_t nlong = 0, nchunks = 0;
+    int32_t* long_rows = nullptr;  // [nlong]
+    int64_t* chunk_ptr = nullptr;  // [nlong+1]
+    int32_t* chunk_lr = nullptr;   // [nchunks] -> index into long_rows
+    double* partial = nullptr;     // [nchunks*4] (double or float accumulators)
+    amgt_spmv_stats st{};
+};
+
+void spmv_plan_free(void* aux, Alloc& a) {
+    SpmvPlan* p = (SpmvPlan*)aux;
+    if (!p) return;
+    a.put(p->long_rows, p->nlong * sizeof(int32_t));
+    a.put(p->chunk_ptr, (p->nlong + 1) * sizeof(int64_t));
+    a.put(p->chunk_lr, p->nchunks * sizeof(int32_t));
+    a.put(p->partial, p->nchunks * 4 * sizeof(double));
+    delete p;
+}
+
+// ---------------------------------------------------------------- loads
+__device__ __forceinline__ double2 ldg_stream(const double2* p) {
+    double2 r;
+    asm volatile("ld.global.nc.v2.f64 {%0, %1}, [%2];" : "=d"(r.x), "=d"(r.y) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ float4 ldg_stream(const float4* p) {
+    float4 r;
+    asm volatile("ld.global.nc.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint2 ldg_stream(const uint2* p) {
+    uint2 r;
+    asm volatile("ld.global.nc.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    return r;
+}
+
+// x pair (elements 2h, 2h+1 of the 4-segment at 4J) as doubles.
+__device__ __forceinline__ double2 x_pair(const double* x, int64_t J, int h) {
+    return __ldg(reinterpret_cast<const double2*>(x + 4 * J + 2 * h));
+}
+__device__ __forceinline__ double2 x_pair(const float* x, int64_t J, int h) {
+    float2 f = __ldg(reinterpret_cast<const float2*>(x + 4 * J + 2 * h));
+    return make_double2(f.x, f.y);
+}
+// x quad as floats.
+__device__ __forceinline__ float4 x_quad(const float* x, int64_t J) { return __ldg(reinterpret_cast<const float4*>(x + 4 * J)); }
+__device__ __forceinline__ float4 x_quad(const double* x, int64_t J) {
+    double2 a = __ldg(reinterpret_cast<const double2*>(x + 4 * J));
+    double2 b = __ldg(reinterpret_cast<const double2*>(x + 4 * J + 2));
+    return make_float4((float)a.x, (float)a.y, (float)b.x, (float)b.y);
+}
+
+template <typename Y> __device__ __forceinline__ void store_y(Y* y, int64_t i, double v) { y[i] = (Y)v; }
+template <typename Y> __device__ __forceinline__ void store_y(Y* y, int64_t i, float v) { y[i] = (Y)v; }
+
+// ---------------------------------------------------------------- FP64 tile step
+// Lane q of the group: elements e0 = 2q, 2q+1 (row q>>1) and e1 = 8+2q, 9+2q (row 2+(q>>1)),
+// columns 2(q&1), 2(q&1)+1.
+struct F64Lane {
+    double acc0 = 0.0, acc1 = 0.0;
+    __device__ __forceinline__ void step(const double* tile, uint32_t mp, double2 xv, int q) {
+        const double2 a = ldg_stream(reinterpret_cast<const double2*>(tile) + q);
+        const double2 b = ldg_stream(reinterpret_cast<const double2*>(tile) + 4 + q);
+        const uint32_t s0 = mp >> (2 * q), s1 = mp >> (8 + 2 * q);
+        acc0 = (s0 & 1u) ? fma(a.x, xv.x, acc0) : acc0;
+        acc0 = (s0 & 2u) ? fma(a.y, xv.y, acc0) : acc0;
+        acc1 = (s1 & 1u) ? fma(b.x, xv.x, acc1) : acc1;
+        acc1 = (s1 & 2u) ? fma(b.y, xv.y, acc1) : acc1;
+    }
+};
+
+// DMMA m8n8k4 (FP64 tensor core) on two tiles: fragA rows 0-3 = tile a, rows 4-7 = tile b;
+// fragB cols 0-3 = x_a (every column), cols 4-7 = x_b.  fragC[g][*] for g<4 = (A_a x_a)[g],
+// g>=4 = (A_b x_b)[g-4]  ("diagonal of fragY", L228).
+__device__ __forceinline__ void dmma_884(double& c0, double& c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                 : "+d"(c0), "+d"(c1)
+                 : "d"(a), "d"(b));
+}
+
+// ---------------------------------------------------------------- row kernel
+// MatT = double / float / __half; XT, YT = double / float.
+template <typename MatT, typename XT, typename YT>
+__global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __restrict__ bptr,
+                                                   const int32_t* __restrict__ bidx,
+                                                   const uint16_t* __restrict__ bmap, const MatT* __restrict__ bval,
+                                                   const XT* __restrict__ x, YT* __restrict__ y, int64_t long_thr,
+                                                   int tc_thr) {
+    const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
+    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t I = wid * 8 + g;
+    if (wid * 8 >= BR) return;
+    int64_t t0 = 0, t1 = 0;
+    bool write = false;
+    if (I < BR) {
+        t0 = __ldg(bptr + I);
+        t1 = __ldg(bptr + I + 1);
+        write = t1 - t0 <= long_thr;
+        if (!write) t1 = t0;  // long row: handled by the chunk kernel
+    }
+    if constexpr (sizeof(MatT) == 8) {
+        F64Lane L;
+        const bool use_tc = tc_thr <= 16;
+        if (!use_tc) {
+            int64_t t = t0;
+            for (; t + 1 < t1; t += 2) {
+                const int32_t J0 = __ldg(bidx + t), J1 = __ldg(bidx + t + 1);
+                const uint32_t m0 = __ldg(bmap + t), m1 = __ldg(bmap + t + 1);
+                const double2 x0 = x_pair(x, J0, q & 1), x1 = x_pair(x, J1, q & 1);
+                L.step((const double*)bval + 16 * t, m0, x0, q);
+                L.step((const double*)bval + 16 * (t + 1), m1, x1, q);
+            }
+            if (t < t1) {
+                const int32_t J0 = __ldg(bidx + t);
+                const uint32_t m0 = __ldg(bmap + t);
+                L.step((const double*)bval + 16 * t, m0, x_pair(x, J0, q & 1), q);
+            }
+        } else {
+            // Per-tile routing: each iteration the 8 groups hold one tile each; tiles with
+            // popcount >= tc_thr are paired and multiplied with DMMA, the rest use CUDA cores.
+            const int64_t len = t1 - t0;
+            int64_t maxlen = len;
+#pragma unroll
+            for (int d = 4; d < 32; d <<= 1) maxlen = max(maxlen, __shfl_xor_sync(0xffffffffu, maxlen, d));
+            double tcacc = 0.0;  // lane q of group g: row q contribution from the TC route
+            for (int64_t k = 0; k < maxlen; ++k) {
+                const bool have = k < len;
+                const int64_t t = t0 + k;
+                const uint32_t mp = have ? __ldg(bmap + t) : 0u;
+                const int32_t J = have ? __ldg(bidx + t) : 0;
+                const bool dense = have && __popc(mp) >= tc_thr;
+                if (have && !dense) L.step((const double*)bval + 16 * t, mp, x_pair(x, J, q & 1), q);
+                uint32_t dm = __ballot_sync(0xffffffffu, dense && q == 0);  // bit 4g per dense group
+                while (dm) {
+                    const int ga = __ffs(dm) - 1;
+                    dm &= dm - 1;
+                    int gb = -1;
+                    if (dm) { gb = __ffs(dm) - 1; dm &= dm - 1; }
+                    const int gA = ga >> 2, gB = gb >= 0 ? (gb >> 2) : -1;
+                    // fragment coordinates: lane = 4*row8 + k4 for A (row row8, col k4);
+                    // B: row k4, col row8.
+                    const int row8 = lane >> 2, k4 = lane & 3;
+                    const int src = row8 < 4 ? gA : gB;  // tile owner for this lane's A element
+                    const int64_t ta = __shfl_sync(0xffffffffu, t, 4 * gA);
+                    const int64_t tb = gB >= 0 ? __shfl_sync(0xffffffffu, t, 4 * gB) : ta;
+                    const int32_t Ja = __shfl_sync(0xffffffffu, J, 4 * gA);
+                    const int32_t Jb = gB >= 0 ? __shfl_sync(0xffffffffu, J, 4 * gB) : Ja;
+                    const uint32_t ma = __shfl_sync(0xffffffffu, mp, 4 * gA);
+                    const uint32_t mb = gB >= 0 ? __shfl_sync(0xffffffffu, mp, 4 * gB) : 0u;
+                    double av = 0.0, bv = 0.0;
+                    if (src >= 0) {
+                        const int64_t tt = row8 < 4 ? ta : tb;
+                        const uint32_t mm = row8 < 4 ? ma : mb;
+                        const int e = 4 * (row8 & 3) + k4;
+                        av = ((mm >> e) & 1u) ? ((const double*)bval)[16 * tt + e] : 0.0;
+                    }
+                    {
+                        const bool first = row8 < 4;
+                        const int32_t JJ = first ? Ja : Jb;
+                        if (first || gB >= 0) bv = (double)x[4 * (int64_t)JJ + k4];
+                    }
+                    double c0 = 0.0, c1 = 0.0;
+                    dmma_884(c0, c1, av, bv);
+                    // C[row8][2*k4'] lives in lane 4*row8 + k4'; column 0 of rows 0-3 -> tile a,
+                    // column 4 of rows 4-7 -> tile b.  Lane (gA, q) takes row q of tile a.
+                    const double ya = __shfl_sync(0xffffffffu, c0, 4 * q + 0);
+                    const double yb = __shfl_sync(0xffffffffu, c0, 4 * (4 + q) + 2);
+                    if (g == gA) tcacc += ya;
+                    if (gB >= 0 && g == gB) tcacc += yb;
+                }
+            }
+            // fold the TC contribution (row q) into the FP64 lane layout: lane q adds it to
+            // the row it will write (rowmap below) — gather via shuffles inside the group.
+            const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
+            const double tcmine = __shfl_sync(0xffffffffu, tcacc, 4 * g + myrow);
+            const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
+            const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
+            if (write) store_y(y, 4 * I + myrow, ((q & 1) ? s1 : s0) + tcmine);
+            return;
+        }
+        const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
+        const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
+        const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
+        if (write) store_y(y, 4 * I + myrow, (q & 1) ? s1 : s0);
+    } else {
+        float acc = 0.f;
+        for (int64_t t = t0; t < t1; ++t) {
+            const int32_t J = __ldg(bidx + t);
+            const uint32_t nib = (__ldg(bmap + t) >> (4 * q)) & 0xFu;
+            const float4 xv = x_quad(x, J);
+            float a0, a1, a2, a3;
+            if constexpr (sizeof(MatT) == 4) {
+                const float4 a = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * t) + q);
+                a0 = a.x; a1 = a.y; a2 = a.z; a3 = a.w;
+            } else {
+                const uint2 u = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * t) + q);
+                const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
+                const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
+                a0 = lo.x; a1 = lo.y; a2 = hi.x; a3 = hi.y;
+            }
+            acc = (nib & 1u) ? fmaf(a0, xv.x, acc) : acc;
+            acc = (nib & 2u) ? fmaf(a1, xv.y, acc) : acc;
+            acc = (nib & 4u) ? fmaf(a2, xv.z, acc) : acc;
+            acc = (nib & 8u) ? fmaf(a3, xv.w, acc) : acc;
+        }
+        if (write) store_y(y, 4 * I + q, acc);
+    }
+}
+
+// ---------------------------------------------------------------- chunk kernel (long rows)
+template <typename MatT, typename XT>
+__global__ void __launch_bounds__(256) k_spmv_chunks(int64_t nchunks, const int64_t* __restrict__ bptr,
+                                                     const int32_t* __restrict__ bidx,
+                                                     const uint16_t* __restrict__ bmap,
+                                                     const MatT* __restrict__ bval, const XT* __restrict__ x,
+                                                     const int32_t* __restrict__ long_rows,
+                                                     const int64_t* __restrict__ chunk_ptr,
+                                                     const int32_t* __restrict__ chunk_lr,
+                                                     typename AccOf<MatT>::type* __restrict__ partial) {
+    using Acc = typename AccOf<MatT>::type;
+    const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const int32_t lr = chunk_lr[c];
+    const int64_t row = long_rows[lr];
+    const int64_t k = c - chunk_ptr[lr];
+    const int64_t a = bptr[row] + k * WARP_CAPACITY;
+    const int64_t b = min(a + WARP_CAPACITY, bptr[row + 1]);
+    Acc out;
+    if constexpr (sizeof(MatT) == 8) {
+        F64Lane L;
+        for (int64_t t = a + g; t < b; t += 8) {
+            const int32_t J = __ldg(bidx + t);
+            L.step((const double*)bval + 16 * t, __ldg(bmap + t), x_pair(x, J, q & 1), q);
+        }
+        double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
+        double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
+        double v = (q & 1) ? s1 : s0;  // row rowmap(q)
+        v += __shfl_xor_sync(0xffffffffu, v, 4);
+        v += __shfl_xor_sync(0xffffffffu, v, 8);
+        v += __shfl_xor_sync(0xffffffffu, v, 16);
+        const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
+        if (g == 0) partial[4 * c + myrow] = v;
+        (void)out;
+    } else {
+        float acc = 0.f;
+        for (int64_t t = a + g; t < b; t += 8) {
+            const int32_t J = __ldg(bidx + t);
+            const uint32_t nib = (__ldg(bmap + t) >> (4 * q)) & 0xFu;
+            const float4 xv = x_quad(x, J);
+            float a0, a1, a2, a3;
+            if constexpr (sizeof(MatT) == 4) {
+                const float4 av = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * t) + q);
+                a0 = av.x; a1 = av.y; a2 = av.z; a3 = av.w;
+            } else {
+                const uint2 u = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * t) + q);
+                const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
+                const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
+                a0 = lo.x; a1 = lo.y; a2 = hi.x; a3 = hi.y;
+            }
+            acc = (nib & 1u) ? fmaf(a0, xv.x, acc) : acc;
+            acc = (nib & 2u) ? fmaf(a1, xv.y, acc) : acc;
+            acc = (nib & 4u) ? fmaf(a2, xv.z, acc) : acc;
+            acc = (nib & 8u) ? fmaf(a3, xv.w, acc) : acc;
+        }
+        acc += __shfl_xor_sync(0xffffffffu, acc, 4);
+        acc += __shfl_xor_sync(0xffffffffu, acc, 8);
+        acc += __shfl_xor_sync(0xffffffffu, acc, 16);
+        if (g == 0) partial[4 * c + q] = acc;
+    }
+}
+
+template <typename Acc, typename YT>
+__global__ void k_spmv_combine(int64_t nlong, const int32_t* __restrict__ long_rows,
+                               const int64_t* __restrict__ chunk_ptr, const Acc* __restrict__ partial,
+                               YT* __restrict__ y) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= 4 * nlong) return;
+    const int64_t lr = i >> 2;
+    const int r = (int)(i & 3);
+    Acc s = 0;
+    for (int64_t c = chunk_ptr[lr]; c < chunk_ptr[lr + 1]; ++c) s += partial[4 * c + r];
+    store_y(y, 4 * (int64_t)long_rows[lr] + r, s);
+}
+
+// ---------------------------------------------------------------- analysis kernels
+__global__ void k_plan_rows(int64_t BR, const int64_t* __restrict__ bptr, int64_t* __restrict__ islong,
+                            int64_t* __restrict__ nch, double* __restrict__ sums /*[2]: sum len, sum len^2*/) {
+    double s1 = 0, s2 = 0;
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t len = bptr[I + 1] - bptr[I];
+        const bool lg = len > WARP_CAPACITY;
+        islong[I] = lg;
+        nch[I] = lg ? (len + WARP_CAPACITY - 1) / WARP_CAPACITY : 0;
+        s1 += (double)len;
+        s2 += (double)len * (double)len;
+    }
+    for (int d = 16; d; d >>= 1) {
+        s1 += __shfl_xor_sync(0xffffffffu, s1, d);
+        s2 += __shfl_xor_sync(0xffffffffu, s2, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(sums, s1);
+        atomicAdd(sums + 1, s2);
+    }
+}
+
+__global__ void k_plan_fill(int64_t BR, const int64_t* __restrict__ bptr, const int64_t* __restrict__ lpos,
+                            const int64_t* __restrict__ cpos, int32_t* __restrict__ long_rows,
+                            int64_t* __restrict__ chunk_ptr, int32_t* __restrict__ chunk_lr) {
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+        if (lpos[I + 1] == lpos[I]) continue;
+        const int64_t lr = lpos[I];
+        long_rows[lr] = (int32_t)I;
+        chunk_ptr[lr] = cpos[I];
+        for (int64_t c = cpos[I]; c < cpos[I + 1]; ++c) chunk_lr[c] = (int32_t)lr;
+    }
+}
+
+__global__ void k_count_tc(int64_t T, const uint16_t* __restrict__ bmap, int thr, unsigned long long* __restrict__ out) {
+    int64_t s = 0, nz = 0;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < T; t += (int64_t)gridDim.x * blockDim.x) {
+        const int p = __popc(bmap[t]);
+        s += p >= thr;
+        nz += p;
+    }
+    for (int d = 16; d; d >>= 1) {
+        s += __shfl_xor_sync(0xffffffffu, s, d);
+        nz += __shfl_xor_sync(0xffffffffu, nz, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(out, (unsigned long long)s);
+        atomicAdd(out + 1, (unsigned long long)nz);
+    }
+}
+
+static unsigned grid_cap(int64_t work, int threads) {
+    int64_t b = ceil_div(work, threads);
+    int64_t cap = (int64_t)num_sms() * 16;
+    return (unsigned)(b < 1 ? 1 : (b > cap ? cap : b));
+}
+
+amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
+    cudaStream_t s = a.s;
+    if (A->aux) { spmv_plan_free(A->aux, a); A->aux = nullptr; }
+    const int64_t BR = A->blc_row;
+    Scratch<int64_t> islong, nch, lpos, cpos;
+    Scratch<double> sums;
+    Scratch<unsigned long long> tcc;
+    AMGT_TRY(islong.init(a, BR + 1));
+    AMGT_TRY(nch.init(a, BR + 1));
+    AMGT_TRY(lpos.init(a, BR + 1));
+    AMGT_TRY(cpos.init(a, BR + 1));
+    AMGT_TRY(sums.init(a, 2));
+    AMGT_TRY(tcc.init(a, 2));
+    AMGT_CUDA(cudaMemsetAsync(sums.p, 0, 2 * sizeof(double), s));
+    AMGT_CUDA(cudaMemsetAsync(tcc.p, 0, 2 * sizeof(unsigned long long), s));
+    if (BR > 0) {
+        k_plan_rows<<<grid_cap(BR, 256), 256, 0, s>>>(BR, A->blc_ptr, islong.p, nch.p, sums.p);
+        AMGT_LAUNCHED();
+    }
+    if (A->blc_num > 0) {
+        k_count_tc<<<grid_cap(A->blc_num, 256), 256, 0, s>>>(A->blc_num, A->blc_map, g_tc_thr_spmv, tcc.p);
+        AMGT_LAUNCHED();
+    }
+    AMGT_TRY(scan_exclusive(islong.p, lpos.p, BR, a, s));
+    AMGT_TRY(scan_exclusive(nch.p, cpos.p, BR, a, s));
+    int64_t nl = 0, ncx = 0;
+    double hs[2];
+    unsigned long long ht[2];
+    AMGT_CUDA(cudaMemcpyAsync(&nl, lpos.p + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaMemcpyAsync(&ncx, cpos.p + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaMemcpyAsync(hs, sums.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaMemcpyAsync(ht, tcc.p, sizeof(ht), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    SpmvPlan* P = new SpmvPlan();
+    P->nlong = nl;
+    P->nchunks = ncx;
+    if (nl > 0) {
+        P->long_rows = (int32_t*)a.get(nl * sizeof(int32_t));
+        P->chunk_ptr = (int64_t*)a.get((nl + 1) * sizeof(int64_t));
+        P->chunk_lr = (int32_t*)a.get(ncx * sizeof(int32_t));
+        P->partial = (double*)a.get(ncx * 4 * sizeof(double));
+        if (!P->long_rows || !P->chunk_ptr || !P->chunk_lr || !P->partial) {
+            spmv_plan_free(P, a);
+            return fail(AMGT_ERR_ALLOC, "SpMV plan allocation failed");
+        }
+        k_plan_fill<<<grid_cap(BR, 256), 256, 0, s>>>(BR, A->blc_ptr, lpos.p, cpos.p, P->long_rows, P->chunk_ptr,
+                                                     P->chunk_lr);
+        AMGT_LAUNCHED();
+        AMGT_CUDA(cudaMemcpyAsync(P->chunk_ptr + nl, &ncx, sizeof(int64_t), cudaMemcpyHostToDevice, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));  // ncx is a host stack value
+    }
+    const double mean = BR ? hs[0] / BR : 0.0;
+    const double var = BR ? hs[1] / BR - mean * mean : 0.0;
+    P->st.avg_nnz_blc = A->blc_num ? (double)ht[1] / (double)A->blc_num : 0.0;
+    P->st.variation = mean > 0 ? sqrt(var > 0 ? var : 0) / mean : 0.0;
+    P->st.long_rows = nl;
+    P->st.chunks = ncx;
+    P->st.tc_tiles = (int64_t)ht[0];
+    A->aux = P;
+    return AMGT_OK;
+}
+
+template <typename MatT, typename XT, typename YT>
+static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, cudaStream_t s) {
+    const SpmvPlan* P = (const SpmvPlan*)A->aux;
+    const int64_t long_thr = (P && P->nlong > 0) ? WARP_CAPACITY : INT64_MAX;
+    const int64_t BR = A->blc_row;
+    if (BR > 0) {
+        const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 256);
+        k_spmv_rows<MatT, XT, YT><<<blocks, 256, 0, s>>>(BR, A->blc_ptr, A->blc_idx, A->blc_map,
+                                                         (const MatT*)A->blc_val, (const XT*)x, (YT*)y, long_thr,
+                                                         sizeof(MatT) == 8 ? g_tc_thr_spmv : 17);
+        AMGT_LAUNCHED();
+    }
+    if (P && P->nlong > 0) {
+        using Acc = typename AccOf<MatT>::type;
+        k_spmv_chunks<MatT, XT><<<(unsigned)ceil_div(P->nchunks * 32, 256), 256, 0, s>>>(
+            P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, P->long_rows,
+            P->chunk_ptr, P->chunk_lr, (Acc*)P->partial);
+        AMGT_LAUNCHED();
+        k_spmv_combine<Acc, YT><<<(unsigned)ceil_div(4 * P->nlong, 256), 256, 0, s>>>(
+            P->nlong, P->long_rows, P->chunk_ptr, (const Acc*)P->partial, (YT*)y);
+        AMGT_LAUNCHED();
+    }
+    return AMGT_OK;
+}
+
+template <typename MatT>
+static amgt_status dispatch_xy(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s) {
+    if (xp == AMGT_FP64 && yp == AMGT_FP64) return launch_spmv<MatT, double, double>(A, x, y, s);
+    if (xp == AMGT_FP64 && yp == AMGT_FP32) return launch_spmv<MatT, double, float>(A, x, y, s);
+    if (xp == AMGT_FP32 && yp == AMGT_FP64) return launch_spmv<MatT, float, double>(A, x, y, s);
+    return launch_spmv<MatT, float, float>(A, x, y, s);
+}
+
+double spmv_bytes(const amgt_mbsr* A, amgt_prec xp, amgt_prec yp) {
+    // T(16s + 4 + 2) + (BR+1) 8 + 4 BC s_x + 4 BR s_y
+    return A->blc_num * (16.0 * prec_bytes(A->prec) + 6.0) + (A->blc_row + 1) * 8.0 +
+           4.0 * A->blc_col * prec_bytes(xp) + 4.0 * A->blc_row * prec_bytes(yp);
+}
+
+amgt_status spmv_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s,
+                      int timer_class) {
+    TimerScope ts(timer_class, spmv_bytes(A, xp, yp), s);
+    switch (A->prec) {
+        case AMGT_FP64: return dispatch_xy<double>(A, x, xp, y, yp, s);
+        case AMGT_FP32: return dispatch_xy<float>(A, x, xp, y, yp, s);
+        default: return dispatch_xy<__half>(A, x, xp, y, yp, s);
+    }
+}
+
+}  // namespace amgt
+
+using namespace amgt;
+
+extern "C" {
+
+amgt_status amgt_spmv_analyze(amgt_mbsr* A, const amgt_allocator* al, void* stream) {
+    if (!A) return fail(AMGT_ERR_ARG, "amgt_spmv_analyze: NULL matrix");
+    Alloc a{al, (cudaStream_t)stream};
+    return spmv_analyze_impl(A, a);
+}
+
+amgt_status amgt_spmv_get_stats(const amgt_mbsr* A, amgt_spmv_stats* st) {
+    if (!A || !st) return fail(AMGT_ERR_ARG, "amgt_spmv_get_stats: NULL argument");
+    if (!A->aux) return fail(AMGT_ERR_ARG, "amgt_spmv_get_stats: matrix not analysed");
+    *st = ((const SpmvPlan*)A->aux)->st;
+    return AMGT_OK;
+}
+
+amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec, void* stream) {
+    if (!A || (!x && A->blc_col > 0) || (!y && A->blc_row > 0)) return fail(AMGT_ERR_ARG, "amgt_spmv: NULL argument");
+    if ((xprec != AMGT_FP64 && xprec != AMGT_FP32) || (yprec != AMGT_FP64 && yprec != AMGT_FP32))
+        return fail(AMGT_ERR_ARG, "amgt_spmv: x/y precision must be FP64 or FP32");
+    if (!prec_valid(A->prec)) return fail(AMGT_ERR_ARG, "amgt_spmv: bad matrix precision");
+    return spmv_impl(A, x, xprec, y, yprec, (cudaStream_t)stream, TC_SPMV);
+}
+
+}  // extern "C"

@@ -1,0 +1,490 @@
+// vcycle.cu — AMG setup with fixed interpolation (Alg. 1, L52-58) and the V-cycle solve
+// (Alg. 2, L68-82) driving the mBSR SpGEMM/SpMV kernels, with per-level precision
+// (L266: level 1 FP64, level 2 FP32, levels >= 3 FP16; vectors FP64 at level 1, FP32
+// below, reading R16).  Smoother: weighted Jacobi x += w D^-1 (b - A x) (R21).
+// Coarsest level: MBSR2CSR (L262), dense Cholesky-based inverse in FP64 on the host,
+// applied on the device as a dense FP64 matvec (R22).
+#include <cmath>
+#include <vector>
+
+#include "common.cuh"
+
+namespace amgt {
+
+amgt_status mbsr_release(amgt_mbsr* M, Alloc& a);
+amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& a);
+amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a);
+amgt_status mbsr_to_csr_impl(const amgt_mbsr* A, int64_t* rp, int32_t* ci, double* v, Alloc& a);
+amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a);
+amgt_status spmv_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s,
+                      int timer_class);
+amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* Cout, amgt_spgemm_info* info,
+                                 Alloc& a);
+amgt_status spgemm_numeric_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a);
+
+}  // namespace amgt
+
+using namespace amgt;
+
+struct amgt_level {
+    amgt_mbsr A{}, P{}, R{};  // A_k at level precision; P_k, R_k at level k precision
+    bool ownA = false;
+    int64_t npad = 0;         // 4 * blc_row
+    amgt_prec vprec = AMGT_FP64;
+    void *b = nullptr, *x = nullptr, *r = nullptr, *t = nullptr, *dinv = nullptr;
+};
+
+struct amgt_hierarchy {
+    int nlev = 0;
+    amgt_vcycle_opts o{};
+    amgt_allocator al{};
+    bool has_al = false;
+    cudaStream_t s = nullptr;
+    amgt_level L[8];
+    int64_t nM = 0;
+    double* Ainv = nullptr;     // dense inverse of the coarsest operator (FP64, nM x nM)
+    double* partial = nullptr;  // norm partial sums
+    double* norms = nullptr;    // per-cycle squared residual norms (device)
+    int norms_cap = 0;
+    int64_t spmv_calls = 0;
+    Alloc alloc() { return Alloc{has_al ? &al : nullptr, s}; }
+};
+
+namespace amgt {
+
+constexpr int NORM_BLOCKS = 256;
+
+template <typename V, typename M>
+__global__ void k_dinv(int64_t BR, int64_t m, const int64_t* __restrict__ bptr, const int32_t* __restrict__ bidx,
+                       const M* __restrict__ bval, V* __restrict__ dinv) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= 4 * BR) return;
+    const int64_t I = i >> 2;
+    const int r = (int)(i & 3);
+    double d = 0.0;
+    if (i < m)
+        for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t)
+            if (bidx[t] == (int32_t)I) { d = to_f64(bval[16 * t + 5 * r]); break; }
+    dinv[i] = (V)(d != 0.0 ? 1.0 / d : 0.0);
+}
+
+template <typename V>
+__global__ void k_jacobi(int64_t n, V* __restrict__ x, const V* __restrict__ b, const V* __restrict__ t,
+                         const V* __restrict__ dinv, V omega) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] = x[i] + omega * dinv[i] * (b[i] - t[i]);
+}
+
+template <typename V>
+__global__ void k_residual(int64_t n, V* __restrict__ r, const V* __restrict__ b, const V* __restrict__ t) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        r[i] = b[i] - t[i];
+}
+
+template <typename V>
+__global__ void k_axpy(int64_t n, V* __restrict__ x, const V* __restrict__ e) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] += e[i];
+}
+
+// Deterministic ||b - t||^2: fixed grid of NORM_BLOCKS, per-block partials, then one block.
+__global__ void k_resnorm_partial(int64_t n, const double* __restrict__ b, const double* __restrict__ t,
+                                  double* __restrict__ partial) {
+    __shared__ double sh[32];
+    double s = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double d = b[i] - t[i];
+        s = fma(d, d, s);
+    }
+    for (int d = 16; d; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double a = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) a += sh[w];
+        partial[blockIdx.x] = a;
+    }
+}
+
+__global__ void k_resnorm_final(const double* __restrict__ partial, double* __restrict__ out) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) {
+        double a = 0.0;
+        for (int i = 0; i < NORM_BLOCKS; ++i) a += partial[i];
+        *out = a;
+    }
+}
+
+// x = Ainv * b (dense FP64), one warp per row.
+template <typename V>
+__global__ void k_dense_solve(int64_t n, int64_t npad, const double* __restrict__ Ainv, const V* __restrict__ b,
+                              V* __restrict__ x) {
+    const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (row >= npad) return;
+    double s = 0.0;
+    if (row < n)
+        for (int64_t j = lane; j < n; j += 32) s = fma(Ainv[row * n + j], (double)b[j], s);
+    for (int d = 16; d; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
+    if (lane == 0) x[row] = (V)s;
+}
+
+static unsigned vgrid(int64_t n) {
+    int64_t b = ceil_div(n, 256);
+    const int64_t cap = (int64_t)num_sms() * 8;
+    return (unsigned)(b < 1 ? 1 : (b > cap ? cap : b));
+}
+
+static size_t vbytes(amgt_prec p) { return p == AMGT_FP64 ? 8 : 4; }
+
+template <typename V>
+static amgt_status vec_jacobi(amgt_level& L, cudaStream_t s, double omega) {
+    TimerScope ts(TC_VEC, 5.0 * L.npad * sizeof(V), s);
+    k_jacobi<V><<<vgrid(L.npad), 256, 0, s>>>(L.npad, (V*)L.x, (const V*)L.b, (const V*)L.t, (const V*)L.dinv, (V)omega);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+template <typename V>
+static amgt_status vec_residual(amgt_level& L, cudaStream_t s) {
+    TimerScope ts(TC_VEC, 3.0 * L.npad * sizeof(V), s);
+    k_residual<V><<<vgrid(L.npad), 256, 0, s>>>(L.npad, (V*)L.r, (const V*)L.b, (const V*)L.t);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+template <typename V>
+static amgt_status vec_axpy(amgt_level& L, cudaStream_t s) {
+    TimerScope ts(TC_VEC, 3.0 * L.npad * sizeof(V), s);
+    k_axpy<V><<<vgrid(L.npad), 256, 0, s>>>(L.npad, (V*)L.x, (const V*)L.t);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+static amgt_status jacobi(amgt_level& L, cudaStream_t s, double w) {
+    return L.vprec == AMGT_FP64 ? vec_jacobi<double>(L, s, w) : vec_jacobi<float>(L, s, w);
+}
+static amgt_status residual(amgt_level& L, cudaStream_t s) {
+    return L.vprec == AMGT_FP64 ? vec_residual<double>(L, s) : vec_residual<float>(L, s);
+}
+static amgt_status axpy(amgt_level& L, cudaStream_t s) {
+    return L.vprec == AMGT_FP64 ? vec_axpy<double>(L, s) : vec_axpy<float>(L, s);
+}
+
+template <typename V, typename M>
+static void launch_dinv(amgt_level& L, cudaStream_t s) {
+    k_dinv<V, M><<<(unsigned)ceil_div(L.npad, 256), 256, 0, s>>>(L.A.blc_row, L.A.m, L.A.blc_ptr, L.A.blc_idx,
+                                                                (const M*)L.A.blc_val, (V*)L.dinv);
+}
+
+static amgt_status build_dinv(amgt_level& L, cudaStream_t s) {
+    if (L.npad == 0) return AMGT_OK;
+    const bool v64 = L.vprec == AMGT_FP64;
+    switch (L.A.prec) {
+        case AMGT_FP64: v64 ? launch_dinv<double, double>(L, s) : launch_dinv<float, double>(L, s); break;
+        case AMGT_FP32: v64 ? launch_dinv<double, float>(L, s) : launch_dinv<float, float>(L, s); break;
+        default: v64 ? launch_dinv<double, __half>(L, s) : launch_dinv<float, __half>(L, s);
+    }
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+// Host dense Cholesky + inverse of the (SPD) coarsest operator.
+static bool dense_inverse(int64_t n, std::vector<double>& a, std::vector<double>& inv) {
+    std::vector<double> L(a);
+    for (int64_t j = 0; j < n; ++j) {
+        double s = L[j * n + j];
+        for (int64_t k = 0; k < j; ++k) s -= L[j * n + k] * L[j * n + k];
+        if (!(s > 0.0)) return false;
+        const double d = std::sqrt(s);
+        L[j * n + j] = d;
+        for (int64_t i = j + 1; i < n; ++i) {
+            double t = L[i * n + j];
+            for (int64_t k = 0; k < j; ++k) t -= L[i * n + k] * L[j * n + k];
+            L[i * n + j] = t / d;
+        }
+    }
+    inv.assign(n * n, 0.0);
+    std::vector<double> y(n);
+    for (int64_t c = 0; c < n; ++c) {  // solve L L^T x = e_c
+        for (int64_t i = 0; i < n; ++i) {
+            double s = (i == c) ? 1.0 : 0.0;
+            for (int64_t k = 0; k < i; ++k) s -= L[i * n + k] * y[k];
+            y[i] = s / L[i * n + i];
+        }
+        for (int64_t i = n - 1; i >= 0; --i) {
+            double s = y[i];
+            for (int64_t k = i + 1; k < n; ++k) s -= L[k * n + i] * inv[k * n + c];
+            inv[i * n + c] = s / L[i * n + i];
+        }
+    }
+    return true;
+}
+
+static void free_level_vectors(amgt_level& L, Alloc& a) {
+    const size_t vb = vbytes(L.vprec) * (size_t)L.npad;
+    for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv}) {
+        a.put(*p, vb);
+        *p = nullptr;
+    }
+}
+
+static void destroy(amgt_hierarchy* H) {
+    if (!H) return;
+    Alloc a = H->alloc();
+    for (int k = 0; k < H->nlev; ++k) {
+        amgt_level& L = H->L[k];
+        if (L.ownA) mbsr_release(&L.A, a);
+        else if (L.A.aux) { amgt_mbsr tmp{}; tmp.aux = L.A.aux; mbsr_release(&tmp, a); }
+        mbsr_release(&L.P, a);
+        mbsr_release(&L.R, a);
+        free_level_vectors(L, a);
+    }
+    a.put(H->Ainv, (size_t)H->nM * H->nM * sizeof(double));
+    a.put(H->partial, NORM_BLOCKS * sizeof(double));
+    a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
+    cudaStreamSynchronize(H->s);
+    delete H;
+}
+
+static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nlev, const amgt_vcycle_opts* o,
+                          amgt_hierarchy* H) {
+    cudaStream_t s = H->s;
+    Alloc a = H->alloc();
+    H->nlev = nlev;
+    for (int k = 0; k < nlev; ++k) {
+        amgt_level& L = H->L[k];
+        const amgt_prec pk = o->level_prec[k];
+        L.vprec = (k == 0) ? AMGT_FP64 : AMGT_FP32;
+        if (k == 0) {
+            if (pk == A->prec) {
+                L.A = *A;  // borrowed
+                L.A.own = 0;
+                L.A.aux = nullptr;
+                L.ownA = false;
+            } else {
+                AMGT_TRY(cast_impl(A, pk, &L.A, a));
+                L.ownA = true;
+            }
+        }
+        L.npad = 4 * L.A.blc_row;
+        AMGT_TRY(spmv_analyze_impl(&L.A, a));
+        const size_t vb = vbytes(L.vprec) * (size_t)L.npad;
+        for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv}) {
+            *p = a.get(vb);
+            if (!*p) return fail(AMGT_ERR_ALLOC, "hierarchy vector allocation failed");
+            AMGT_CUDA(cudaMemsetAsync(*p, 0, vb, s));
+        }
+        AMGT_TRY(build_dinv(L, s));
+        if (k + 1 < nlev) {
+            const amgt_mbsr* Pk = P[k];
+            if (Pk->m != L.A.m) return fail(AMGT_ERR_ARG, "P[%d] has %lld rows, level has %lld", k, (long long)Pk->m, (long long)L.A.m);
+            AMGT_TRY(cast_impl(Pk, pk, &L.P, a));  // P_k in level k precision (copy when equal)
+            AMGT_TRY(transpose_impl(&L.P, &L.R, a));  // R_k = P_k^T (Alg. 1 line 4)
+            // A_{k+1} = R_k (A_k P_k): two SpGEMM calls in level k precision (Alg. 1 line 5)
+            amgt_mbsr AP{}, Ac{};
+            AMGT_TRY(spgemm_symbolic_impl(&L.A, &L.P, &AP, nullptr, a));
+            amgt_status st = spgemm_numeric_impl(&L.A, &L.P, &AP, a);
+            if (st == AMGT_OK) st = spgemm_symbolic_impl(&L.R, &AP, &Ac, nullptr, a);
+            if (st == AMGT_OK) st = spgemm_numeric_impl(&L.R, &AP, &Ac, a);
+            mbsr_release(&AP, a);
+            if (st != AMGT_OK) { mbsr_release(&Ac, a); return st; }
+            amgt_level& N = H->L[k + 1];
+            const amgt_prec pn = o->level_prec[k + 1];
+            if (pn != Ac.prec) {
+                st = cast_impl(&Ac, pn, &N.A, a);
+                mbsr_release(&Ac, a);
+                if (st != AMGT_OK) return st;
+                N.A.own |= 1u;  // the cast shares Ac's structure: take ownership of it
+            } else {
+                N.A = Ac;
+            }
+            N.ownA = true;
+            AMGT_TRY(spmv_analyze_impl(&L.P, a));
+            AMGT_TRY(spmv_analyze_impl(&L.R, a));
+        }
+    }
+    // coarsest level: MBSR2CSR, dense inverse on the host (FP64)
+    amgt_level& C = H->L[nlev - 1];
+    const int64_t n = C.A.m;
+    if (n > 4096) return fail(AMGT_ERR_UNSUPPORTED, "coarsest level has %lld rows (dense solve limit 4096)", (long long)n);
+    int64_t* rp = (int64_t*)a.get((n + 1) * sizeof(int64_t));
+    int32_t* ci = (int32_t*)a.get(16 * C.A.blc_num * sizeof(int32_t) + 4);
+    double* v = (double*)a.get(16 * C.A.blc_num * sizeof(double) + 8);
+    if (!rp || !ci || !v) return fail(AMGT_ERR_ALLOC, "coarse CSR allocation failed");
+    AMGT_TRY(mbsr_to_csr_impl(&C.A, rp, ci, v, a));
+    std::vector<int64_t> hrp(n + 1);
+    AMGT_CUDA(cudaMemcpyAsync(hrp.data(), rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    const int64_t nnz = hrp[n];
+    std::vector<int32_t> hci(nnz);
+    std::vector<double> hv(nnz);
+    if (nnz) {
+        AMGT_CUDA(cudaMemcpyAsync(hci.data(), ci, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(hv.data(), v, nnz * sizeof(double), cudaMemcpyDeviceToHost, s));
+    }
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    a.put(rp, (n + 1) * sizeof(int64_t));
+    a.put(ci, 16 * C.A.blc_num * sizeof(int32_t) + 4);
+    a.put(v, 16 * C.A.blc_num * sizeof(double) + 8);
+    std::vector<double> dense(n * n, 0.0), inv;
+    for (int64_t i = 0; i < n; ++i)
+        for (int64_t p = hrp[i]; p < hrp[i + 1]; ++p) dense[i * n + hci[p]] = hv[p];
+    if (!dense_inverse(n, dense, inv)) return fail(AMGT_ERR_ARG, "coarsest operator is not SPD (Cholesky failed)");
+    H->nM = n;
+    H->Ainv = (double*)a.get(n * n * sizeof(double) + 8);
+    H->partial = (double*)a.get(NORM_BLOCKS * sizeof(double));
+    if (!H->Ainv || !H->partial) return fail(AMGT_ERR_ALLOC, "coarse inverse allocation failed");
+    AMGT_CUDA(cudaMemcpyAsync(H->Ainv, inv.data(), n * n * sizeof(double), cudaMemcpyHostToDevice, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    return AMGT_OK;
+}
+
+static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const void* x, amgt_prec xp, void* y,
+                                amgt_prec yp, int level) {
+    ++H->spmv_calls;
+    return spmv_impl(M, x, xp, y, yp, H->s, level == 0 ? TC_SPMV_L1 : TC_SPMV);
+}
+
+static amgt_status norm_into(amgt_hierarchy* H, const double* b, const double* t, int64_t n, double* out) {
+    TimerScope ts(TC_VEC, 2.0 * n * 8, H->s);
+    k_resnorm_partial<<<NORM_BLOCKS, 256, 0, H->s>>>(n, b, t, H->partial);
+    AMGT_LAUNCHED();
+    k_resnorm_final<<<1, 32, 0, H->s>>>(H->partial, out);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+template <typename V>
+static amgt_status dense_solve(amgt_hierarchy* H, amgt_level& L) {
+    TimerScope ts(TC_VEC, (double)H->nM * H->nM * 8, H->s);
+    k_dense_solve<V><<<(unsigned)ceil_div(L.npad * 32, 256), 256, 0, H->s>>>(H->nM, L.npad, H->Ainv, (const V*)L.b,
+                                                                           (V*)L.x);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_host,
+                          int64_t* calls_host) {
+    cudaStream_t s = H->s;
+    Alloc a = H->alloc();
+    if (ncycles + 1 > H->norms_cap) {
+        a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
+        H->norms_cap = ncycles + 1;
+        H->norms = (double*)a.get((size_t)H->norms_cap * sizeof(double));
+        if (!H->norms) return fail(AMGT_ERR_ALLOC, "norm buffer allocation failed");
+    }
+    const int M = H->nlev - 1;
+    amgt_level& L0 = H->L[0];
+    const double w = H->o.omega;
+    H->spmv_calls = 0;
+    AMGT_TRY(counted_spmv(H, &L0.A, x, AMGT_FP64, L0.t, AMGT_FP64, 0));
+    AMGT_TRY(norm_into(H, b, (const double*)L0.t, L0.npad, H->norms));
+    for (int c = 1; c <= ncycles; ++c) {
+        for (int k = 0; k < M; ++k) {  // Alg. 2 lines 1-5
+            amgt_level& L = H->L[k];
+            void* bk = k == 0 ? (void*)b : L.b;
+            void* xk = k == 0 ? (void*)x : L.x;
+            void* sb = L.b;
+            void* sx = L.x;
+            L.b = bk;
+            L.x = xk;
+            if (k > 0) AMGT_CUDA(cudaMemsetAsync(L.x, 0, vbytes(L.vprec) * L.npad, s));
+            for (int i = 0; i < H->o.nu1; ++i) {  // line 2
+                AMGT_TRY(counted_spmv(H, &L.A, L.x, L.vprec, L.t, L.vprec, k));
+                AMGT_TRY(jacobi(L, s, w));
+            }
+            AMGT_TRY(counted_spmv(H, &L.A, L.x, L.vprec, L.t, L.vprec, k));  // line 3
+            AMGT_TRY(residual(L, s));
+            amgt_level& N = H->L[k + 1];
+            AMGT_TRY(counted_spmv(H, &L.R, L.r, L.vprec, N.b, N.vprec, k));  // line 4
+            L.b = sb;
+            L.x = sx;
+        }
+        {  // line 6
+            amgt_level& C = H->L[M];
+            if (M == 0) {
+                amgt_level tmp = C;
+                tmp.b = (void*)b;
+                tmp.x = x;
+                AMGT_TRY(dense_solve<double>(H, tmp));
+            } else {
+                AMGT_TRY(C.vprec == AMGT_FP64 ? dense_solve<double>(H, C) : dense_solve<float>(H, C));
+            }
+        }
+        for (int k = M - 1; k >= 0; --k) {  // lines 7-11
+            amgt_level& L = H->L[k];
+            amgt_level& N = H->L[k + 1];
+            void* sb = L.b;
+            void* sx = L.x;
+            if (k == 0) { L.b = (void*)b; L.x = x; }
+            AMGT_TRY(counted_spmv(H, &L.P, N.x, N.vprec, L.t, L.vprec, k));  // line 8
+            AMGT_TRY(axpy(L, s));                                           // line 9
+            for (int i = 0; i < H->o.nu2; ++i) {                            // line 10
+                AMGT_TRY(counted_spmv(H, &L.A, L.x, L.vprec, L.t, L.vprec, k));
+                AMGT_TRY(jacobi(L, s, w));
+            }
+            L.b = sb;
+            L.x = sx;
+        }
+        AMGT_TRY(counted_spmv(H, &L0.A, x, AMGT_FP64, L0.t, AMGT_FP64, 0));  // residual (L308)
+        AMGT_TRY(norm_into(H, b, (const double*)L0.t, L0.npad, H->norms + c));
+    }
+    std::vector<double> hn(ncycles + 1);
+    AMGT_CUDA(cudaMemcpyAsync(hn.data(), H->norms, (ncycles + 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    if (res_host)
+        for (int c = 0; c <= ncycles; ++c) res_host[c] = std::sqrt(hn[c]);
+    if (calls_host) *calls_host = H->spmv_calls;
+    return AMGT_OK;
+}
+
+}  // namespace amgt
+
+extern "C" {
+
+amgt_status amgt_hierarchy_create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nlev, const amgt_vcycle_opts* o,
+                                  const amgt_allocator* al, void* stream, amgt_hierarchy** Hout) {
+    if (!A || !o || !Hout || nlev < 1 || nlev > 8 || (nlev > 1 && !P))
+        return fail(AMGT_ERR_ARG, "amgt_hierarchy_create: bad argument");
+    if (A->prec != AMGT_FP64) return fail(AMGT_ERR_ARG, "amgt_hierarchy_create: A must be FP64");
+    if (A->m != A->n) return fail(AMGT_ERR_ARG, "amgt_hierarchy_create: A must be square");
+    for (int k = 0; k < nlev; ++k)
+        if (!prec_valid(o->level_prec[k])) return fail(AMGT_ERR_ARG, "bad level precision %d", k);
+    for (int k = 0; k + 1 < nlev; ++k)
+        if (!P[k] || P[k]->prec != AMGT_FP64) return fail(AMGT_ERR_ARG, "P[%d] missing or not FP64", k);
+    if (o->nu1 < 0 || o->nu2 < 0) return fail(AMGT_ERR_ARG, "negative sweep count");
+    amgt_hierarchy* H = new amgt_hierarchy();
+    H->o = *o;
+    H->s = (cudaStream_t)stream;
+    if (al) { H->al = *al; H->has_al = true; }
+    amgt_status st = create(A, P, nlev, o, H);
+    if (st != AMGT_OK) {
+        destroy(H);
+        return st;
+    }
+    *Hout = H;
+    return AMGT_OK;
+}
+
+int amgt_hierarchy_nlev(const amgt_hierarchy* H) { return H ? H->nlev : 0; }
+
+amgt_status amgt_hierarchy_level(const amgt_hierarchy* H, int k, const amgt_mbsr** A, const amgt_mbsr** P,
+                                 const amgt_mbsr** R) {
+    if (!H || k < 0 || k >= H->nlev) return fail(AMGT_ERR_ARG, "amgt_hierarchy_level: bad level");
+    if (A) *A = &H->L[k].A;
+    if (P) *P = k + 1 < H->nlev ? &H->L[k].P : nullptr;
+    if (R) *R = k + 1 < H->nlev ? &H->L[k].R : nullptr;
+    return AMGT_OK;
+}
+
+amgt_status amgt_vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_norms_host,
+                        int64_t* spmv_calls_host, void* stream) {
+    if (!H || !b || !x || ncycles < 0) return fail(AMGT_ERR_ARG, "amgt_vcycle: bad argument");
+    H->s = (cudaStream_t)stream;
+    return vcycle(H, b, x, ncycles, res_norms_host, spmv_calls_host);
+}
+
+amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H) {
+    destroy(H);
+    return AMGT_OK;
+}
+
+}  // extern "C"

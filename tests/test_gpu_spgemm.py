@@ -1,0 +1,155 @@
+"""GPU parity: SpGEMM (a3-a6) and RAP (a7) vs the oracle (O1, O2, O5).
+Structure bit-exact against O2(O1(A, B)); FP64 values |g - o| <= 1e-12 (|A||B|)_ij and
+exact on integer/dyadic data; FP32 1e-5 (inf-norm), FP16 5e-3 (2-norm) against the
+oracle's FP64 product of the unrounded inputs."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gpu_helpers import assert_structure_equal, check_fp64_entrywise, rel_2, rel_inf, tile_values_to_csr_order
+
+pytestmark = pytest.mark.gpu
+
+
+def _amgt():
+    import paper_conf_sc_luzwflcy0c024_b200 as amgt
+    return amgt
+
+
+def _check_product(C, Co_csr, Cabs=None, exact=False):
+    Co = oracle.csr_to_mbsr(Co_csr)
+    assert_structure_equal(C, Co)
+    rp, ci, v = tile_values_to_csr_order(C)
+    assert np.array_equal(rp, Co_csr.row_ptr) and np.array_equal(ci, Co_csr.col)
+    if exact:
+        assert np.array_equal(v, Co_csr.val)
+    else:
+        check_fp64_entrywise(v, Co_csr.val, Cabs)
+    # +0.0 wherever the bitmap bit is clear (R2)
+    val = C.blc_val.cpu().numpy().reshape(-1, 16)
+    bits = ((C.map_u16().cpu().numpy()[:, None] >> np.arange(16)) & 1).astype(bool)
+    assert np.all(val[~bits] == 0) and not np.signbit(val[~bits]).any()
+
+
+PAIRS = [
+    ("rand_small", lambda: (gen.random_csr(37, 29, 0.2, 1, zero_frac=0.1, empty_rows=3), gen.random_csr(29, 43, 0.2, 2))),
+    ("rand_cancel_int", lambda: (gen.random_csr(64, 64, 0.15, 3, integer=True), gen.random_csr(64, 64, 0.15, 4, integer=True))),
+    ("cfg1_AA", lambda: (gen.laplacian_5pt(64), gen.laplacian_5pt(64))),
+    ("27pt_AA", lambda: (gen.laplacian_27pt(8), gen.laplacian_27pt(8))),
+    ("dense_tiles", lambda: (gen.random_csr(96, 96, 0.8, 5), gen.random_csr(96, 80, 0.7, 6))),
+    ("wide_rows", lambda: (gen.random_csr(16, 3000, 0.3, 7), gen.random_csr(3000, 900, 0.01, 8))),
+]
+
+
+@pytest.mark.parametrize("thr", [10, 0, 17])
+@pytest.mark.parametrize("name,mk", PAIRS, ids=[p[0] for p in PAIRS])
+def test_spgemm_fp64(name, mk, thr):
+    amgt = _amgt()
+    A, B = mk()
+    Ao, Bo = oracle.as_csr(A), oracle.as_csr(B)
+    Co, Cabs = oracle.spgemm(Ao, Bo, with_abs=True)
+    amgt.set_tc_threshold(thr, 17)
+    try:
+        C, info = amgt.spgemm(amgt.from_csr(A), amgt.from_csr(B), info=True)
+    finally:
+        amgt.set_tc_threshold(10, 17)
+    integer = name.endswith("_int") or name.startswith("cfg1") or name.startswith("27pt")
+    _check_product(C, Co, Cabs, exact=integer)
+    deg = np.diff(Bo.row_ptr)
+    assert info["scalar_products"] == int(deg[Ao.col].sum())  # every scalar pair has mapC != 0 here
+
+
+def test_spgemm_info_bins_and_long_rows():
+    """Irregular power-law matrix: exercises several bins incl. bin 7 (dense bitmap) and the
+    global-accumulation numeric path; structure bit-exact, values within 1e-12."""
+    amgt = _amgt()
+    A = gen.irregular_block_sparse(1 << 11, seed=5)
+    Ao = oracle.as_csr(A)
+    Co, Cabs = oracle.spgemm(Ao, Ao, with_abs=True)
+    M = amgt.from_csr(A)
+    C, info = amgt.spgemm(M, M, info=True)
+    _check_product(C, Co, Cabs)
+    # the analysis matches a direct count of Cub per block row
+    Mo = oracle.csr_to_mbsr(Ao)
+    lens = np.diff(Mo.blc_ptr)
+    cub = np.array([lens[Mo.blc_idx[Mo.blc_ptr[I]:Mo.blc_ptr[I + 1]]].sum() for I in range(Mo.blc_row)])
+    edges = 128 * 2 ** np.arange(7)
+    bins = np.searchsorted(edges, cub, side="right")
+    assert info["bin_rows"] == list(np.bincount(bins, minlength=8))
+    assert info["cub_total"] == int(cub.sum())
+    assert sum(info["bin_rows"][2:]) > 0 and info["numeric_rows"][1] > 0
+
+
+@pytest.mark.parametrize("prec", ["f32", "f16"])
+def test_spgemm_low_precision(prec):
+    amgt = _amgt()
+    A = gen.laplacian_7pt(16, spd_seed=2)
+    P = gen.aggregation_P((16, 16, 16), 0.5)
+    for X, Y in ((A, P), (A, A)):
+        Xo, Yo = oracle.as_csr(X), oracle.as_csr(Y)
+        Co = oracle.spgemm(Xo, Yo)
+        C = amgt.spgemm(amgt.from_csr(X, prec=prec), amgt.from_csr(Y, prec=prec))
+        assert_structure_equal(C, oracle.csr_to_mbsr(Co))
+        _, _, v = tile_values_to_csr_order(C)
+        if prec == "f32":
+            assert rel_inf(v, Co.val) <= 1e-5
+        else:
+            assert rel_2(v, Co.val) <= 5e-3
+
+
+@pytest.mark.parametrize("kind,N,alpha", [("7pt", 24, 0.5), ("27pt", 16, 0.5), ("7pt", 16, 1.0)])
+def test_rap_closed_form_and_oracle(kind, N, alpha):
+    amgt = _amgt()
+    A = {"7pt": gen.laplacian_7pt, "27pt": gen.laplacian_27pt}[kind](N)
+    P = gen.aggregation_P((N, N, N), alpha)
+    R = gen.aggregation_R((N, N, N), alpha)
+    Co = oracle.rap(R, A, P)
+    Ac = amgt.rap(amgt.from_csr(R), amgt.from_csr(A), amgt.from_csr(P))
+    _check_product(Ac, Co, exact=True)  # dyadic data: exact
+    if kind == "7pt":
+        ref = oracle.as_csr(gen.laplacian_7pt(N // 2))
+        _, _, v = tile_values_to_csr_order(Ac)
+        assert np.array_equal(v, ref.val * 4 * alpha * alpha)
+
+
+def test_rap_random_spd_tolerance():
+    amgt = _amgt()
+    N = 20
+    A = gen.laplacian_7pt(N, spd_seed=2)
+    P = gen.aggregation_P((N, N, N), 0.5)
+    R = gen.aggregation_R((N, N, N), 0.5)
+    Co, Cabs = oracle.rap(R, A, P, with_abs=True)
+    Ac = amgt.rap(amgt.from_csr(R), amgt.from_csr(A), amgt.from_csr(P))
+    _check_product(Ac, Co, Cabs)
+
+
+@pytest.mark.slow
+def test_rap_cfg2_full():
+    """Config 2 at full size (7-point 128^3): A*P and R*(AP) structure bit-exact, values exact."""
+    amgt = _amgt()
+    N = 128
+    A = gen.laplacian_7pt(N)
+    P = gen.aggregation_P((N, N, N), 0.5)
+    R = gen.aggregation_R((N, N, N), 0.5)
+    Mo_AP = oracle.spgemm(A, P)
+    MA, MP, MR = amgt.from_csr(A), amgt.from_csr(P), amgt.from_csr(R)
+    AP, info = amgt.spgemm(MA, MP, info=True)
+    assert AP.blc_num == 2_048_000
+    _check_product(AP, Mo_AP, exact=True)
+    Ac = amgt.spgemm(MR, AP)
+    assert Ac.blc_num == 446_464
+    _check_product(Ac, oracle.spgemm(R, Mo_AP), exact=True)
+
+
+@pytest.mark.slow
+def test_spgemm_cfg4_full():
+    """Config 4 at full size: A*A structure bit-exact, values within 1e-12 (|A||A|)."""
+    amgt = _amgt()
+    A = gen.configs.build_matrix(gen.configs.CONFIGS["cfg4"])
+    Ao = oracle.as_csr(A)
+    Co, Cabs = oracle.spgemm(Ao, Ao, with_abs=True)
+    M = amgt.from_csr(A)
+    C, info = amgt.spgemm(M, M, info=True)
+    _check_product(C, Co, Cabs)

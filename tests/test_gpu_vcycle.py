@@ -1,0 +1,68 @@
+"""GPU parity: hierarchy setup (Alg. 1 with fixed P) + V-cycle (a10, Alg. 2) vs oracle O6.
+FP64 everywhere: residual history matches the oracle to 1e-9 relative.  Mixed precision
+(L266): residual reduction per cycle within 1% of the oracle's (north_star), checked
+while ||r_k|| / ||r_0|| > 1e-10 (reading R24).  SpMV call count = 1 + ncycles(5(L-1)+1)."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gpu_helpers import assert_structure_equal
+
+pytestmark = pytest.mark.gpu
+
+
+def _amgt():
+    import paper_conf_sc_luzwflcy0c024_b200 as amgt
+    return amgt
+
+
+def _run(kind, N, nlev, prec, ncycles):
+    amgt = _amgt()
+    A = {"7pt": gen.laplacian_7pt, "27pt": gen.laplacian_27pt, "5pt": gen.laplacian_5pt}[kind](N)
+    dims = (N, N) if kind == "5pt" else (N, N, N)
+    PR = gen.aggregation_hierarchy(dims, nlev)
+    b = gen.uniform_vector(A.m, 3)
+    H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=prec)
+    x = torch.zeros(A.m, dtype=torch.float64, device="cuda")
+    res, calls = H.vcycle(b.cuda(), x, ncycles)
+    As = oracle.build_hierarchy(A, PR)
+    xo, res_o, calls_o = oracle.vcycle(As, PR, b.numpy(), ncycles=ncycles)
+    return H, As, np.array(res), np.array(res_o), calls, calls_o, x.cpu().numpy(), xo
+
+
+@pytest.mark.parametrize("kind,N,nlev", [("7pt", 16, 3), ("27pt", 16, 4), ("5pt", 64, 5), ("7pt", 32, 5)])
+def test_vcycle_fp64_matches_oracle(kind, N, nlev):
+    H, As, res, res_o, calls, calls_o, x, xo = _run(kind, N, nlev, ("f64",) * 8, 8)
+    assert calls == calls_o == 1 + 8 * (5 * (nlev - 1) + 1)
+    np.testing.assert_allclose(res, res_o, rtol=1e-9)
+    np.testing.assert_allclose(x, xo, rtol=0, atol=1e-10 * np.abs(xo).max())
+    # the hierarchy's coarse operators equal the oracle's RAP, bit for bit
+    for k in range(1, H.nlev):
+        Ak, _, _ = H.level(k)
+        assert_structure_equal(Ak, oracle.csr_to_mbsr(As[k]))
+        rp, ci, v = Ak.to_csr()
+        assert np.array_equal(v.cpu().numpy(), As[k].val)
+    H.close()
+
+
+@pytest.mark.parametrize("kind,N,nlev", [("27pt", 32, 4), ("7pt", 32, 5)])
+def test_vcycle_mixed_precision_rho_within_1pct(kind, N, nlev):
+    H, As, res, res_o, calls, calls_o, x, xo = _run(kind, N, nlev, ("f64", "f32", "f16", "f16", "f16"), 12)
+    assert calls == calls_o
+    rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
+    live = res_o[1:] / res_o[0] > 1e-10
+    assert live.sum() >= 3
+    assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
+    H.close()
+
+
+@pytest.mark.slow
+def test_vcycle_cfg3_shape_mixed():
+    """Config 3 shape at 64^3 (27-point, 5 levels, mixed precision, 10 cycles)."""
+    H, As, res, res_o, calls, calls_o, x, xo = _run("27pt", 64, 5, ("f64", "f32", "f16", "f16", "f16"), 10)
+    rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
+    live = res_o[1:] / res_o[0] > 1e-10
+    assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
+    H.close()
