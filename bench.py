@@ -1,0 +1,451 @@
+#!/usr/bin/env python
+"""bench.py — one JSON line for the driver.
+
+A step = one pass of the whole hot path over BASELINE config 2
+(3D 7-point Laplacian 128^3, 2x2x2 aggregation P, 7 levels 128^3 -> 2^3):
+  a1 CSR->mBSR of A and of every P_k; a2 per-level casts (FP64 / FP32 / FP16, L266);
+  a3-a7 RAP per level (two SpGEMM calls each: binning, two-step hash symbolic, TC/CUDA-core
+  numeric); R_k = P_k^T; a8 mBSR->CSR of the coarsest level + dense factorisation;
+  a9/a10 50 V-cycles (L308) of weighted-Jacobi smoothing with load-balanced SpMV.
+Inputs (CSR A, P_k, b) are resident in HBM when the timed region starts.
+
+value = algorithmic bytes of the step (SURVEY §8(d) byte model per kernel, summed) / step
+time, i.e. whole-job GB/s; the components (SpMV GB/s, SpGEMM GFLOP/s, setup / solve ms)
+are reported beside it.  `--impl reference` runs the CPU oracle on a bounded sample of
+the same workload (setup + a few cycles) in the same unit.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SpMV GB/s, SpGEMM GFLOP/s (mBSR, 1–8 B200); AMG setup+solve s"
+LEVEL_PREC = ("f64", "f32", "f16", "f16", "f16", "f16", "f16")
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[2:6]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        busy = [s for s in sm if s > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(busy) if busy else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ byte model
+S_BYTES = {"f64": 8, "f32": 4, "f16": 2}
+
+
+def byte_model(sz, cycles):
+    """Algorithmic bytes of one step from structure sizes (identical for both arms).
+    sz: {"A_nnz", "P_nnz": [..], "P_m": [..], "lev": [{"m","BR","BC","T"}], "P_T", "R_T", "AP_T": [..],
+         "prec": [..]}.  Tiles count 16 s + 4 + 2 bytes (values, blc_idx, blc_map)."""
+    L = len(sz["lev"])
+    s = [S_BYTES[p] for p in sz["prec"]]
+    vs = [8 if p == "f64" else 4 for p in sz["prec"]]
+    tb = lambda T, sk: T * (16 * sk + 6)
+    lev = sz["lev"]
+    out = {}
+    # a1: CSR -> mBSR of A (FP64) and of every P_k (FP64)
+    c = sz["A_nnz"] * 12 + (lev[0]["m"] + 1) * 8 + tb(lev[0]["T"], 8) + (lev[0]["BR"] + 1) * 8
+    for k in range(L - 1):
+        c += sz["P_nnz"][k] * 12 + (sz["P_m"][k] + 1) * 8 + tb(sz["P_T"][k], 8) + (lev[k]["BR"] + 1) * 8
+    out["csr2mbsr"] = c
+    # a2: casts (A_{k+1} from level-k precision to level-(k+1); P_k from FP64 to level k)
+    c = 0
+    for k in range(L - 1):
+        if s[k] != 8:
+            c += 16 * sz["P_T"][k] * (8 + s[k])
+        if s[k + 1] != s[k]:
+            c += 16 * lev[k + 1]["T"] * (s[k] + s[k + 1])
+    out["cast"] = c
+    # a3-a7: two SpGEMMs per level; symbolic reads structure twice, writes C's; numeric
+    # reads operands once and writes C once
+    sym = num = 0
+    for k in range(L - 1):
+        TA, TP, TR, TAP, TC = lev[k]["T"], sz["P_T"][k], sz["R_T"][k], sz["AP_T"][k], lev[k + 1]["T"]
+        sym += 2 * (TA + TP) * 6 + TAP * 6 + 2 * (TR + TAP) * 6 + TC * 6
+        num += tb(TA, s[k]) + tb(TP, s[k]) + tb(TAP, s[k]) + tb(TR, s[k]) + tb(TAP, s[k]) + tb(TC, s[k])
+        num += 2 * TP * (16 * s[k] + 6)  # R = P^T (tile transpose: read + write)
+    out["spgemm_symbolic"], out["spgemm_numeric"] = sym, num
+    out["mbsr2csr"] = tb(lev[-1]["T"], s[-1]) + lev[-1]["m"] * 20
+    # a9/a10: per cycle 3 SpMV(A_k) + R_k + P_k per level, 1 final residual SpMV(A_1)
+    def spmv_b(T, BR, BC, sk, xs, ys):
+        return tb(T, sk) + (BR + 1) * 8 + 4 * BC * xs + 4 * BR * ys
+    sp1 = spmv_b(lev[0]["T"], lev[0]["BR"], lev[0]["BC"], s[0], vs[0], vs[0])
+    l1 = sp1 * (3 * (L > 1) + 1)
+    other, vec = 0, 0
+    for k in range(L - 1):
+        if k > 0:
+            other += 3 * spmv_b(lev[k]["T"], lev[k]["BR"], lev[k]["BC"], s[k], vs[k], vs[k])
+        other += spmv_b(sz["R_T"][k], lev[k + 1]["BR"], lev[k]["BR"], s[k], vs[k], vs[k + 1])
+        other += spmv_b(sz["P_T"][k], lev[k]["BR"], lev[k + 1]["BR"], s[k], vs[k + 1], vs[k])
+        if k == 0:
+            l1 += 0
+        vec += 16 * 4 * lev[k]["BR"] * vs[k]
+    vec += lev[-1]["m"] ** 2 * 8 + 2 * 16 * lev[0]["BR"] * 8
+    out["spmv_l1"] = l1 * cycles + sp1
+    out["spmv"] = other * cycles
+    out["vector"] = vec * cycles
+    return out
+
+
+def sample_bytes_model(bm, cycles, total_cycles):
+    setup = sum(bm[k] for k in ("spgemm_symbolic", "spgemm_numeric", "csr2mbsr", "mbsr2csr", "cast"))
+    solve = sum(bm[k] for k in ("spmv_l1", "spmv", "vector"))
+    return setup + solve * cycles / max(total_cycles, 1)
+
+
+def gpu_sizes(amgt, A, Ps):
+    """Structure sizes of the hierarchy built by the CUDA path (for the byte model)."""
+    MA = amgt.from_csr(A)
+    H = amgt.Hierarchy(MA, [amgt.from_csr(P) for P in Ps], level_prec=LEVEL_PREC[:len(Ps) + 1])
+    sz = {"A_nnz": A.nnz, "P_nnz": [P.nnz for P in Ps], "P_m": [P.m for P in Ps], "lev": [], "P_T": [], "R_T": [],
+          "AP_T": [], "prec": list(LEVEL_PREC[:len(Ps) + 1])}
+    flops = 0
+    for k in range(H.nlev):
+        Ak, Pk, Rk = H.level(k)
+        sz["lev"].append({"m": Ak.m, "BR": Ak.blc_row, "BC": Ak.blc_col, "T": Ak.blc_num})
+        if Pk is not None:
+            AP, i1 = amgt.spgemm_symbolic(Ak, Pk, info=True)
+            _, i2 = amgt.spgemm_symbolic(Rk, AP, info=True)
+            flops += 2 * (i1["scalar_products"] + i2["scalar_products"])
+            sz["P_T"].append(Pk.blc_num)
+            sz["R_T"].append(Rk.blc_num)
+            sz["AP_T"].append(AP.blc_num)
+            AP.free()
+    H.close()
+    MA.free()
+    return sz, flops
+
+
+def oracle_sizes(A, PR):
+    import oracle
+    Ao = oracle.as_csr(A.to("cpu"))
+    PRo = [(oracle.as_csr(P.to("cpu")), oracle.as_csr(R.to("cpu"))) for P, R in PR]
+    As = oracle.build_hierarchy(Ao, PRo)
+    sz = {"A_nnz": Ao.nnz, "P_nnz": [P.nnz for P, _ in PRo], "P_m": [P.m for P, _ in PRo], "lev": [], "P_T": [],
+          "R_T": [], "AP_T": [], "prec": list(LEVEL_PREC[:len(As)])}
+    for k, Ak in enumerate(As):
+        T = oracle.csr_to_mbsr(Ak).blc_num
+        sz["lev"].append({"m": Ak.m, "BR": (Ak.m + 3) // 4, "BC": (Ak.n + 3) // 4, "T": T})
+        if k + 1 < len(As):
+            P, R = PRo[k]
+            sz["P_T"].append(oracle.csr_to_mbsr(P).blc_num)
+            sz["R_T"].append(oracle.csr_to_mbsr(R).blc_num)
+            sz["AP_T"].append(oracle.csr_to_mbsr(oracle.spgemm(Ak, P)).blc_num)
+    return sz
+
+
+# ------------------------------------------------------------------ workload
+def make_inputs(cfg, device):
+    import gen
+    N = cfg.N
+    A = gen.configs.build_matrix(cfg, device=device)
+    PR = gen.aggregation_hierarchy(gen.configs.grid_dims(cfg), cfg.nlev, cfg.alpha, device=device)
+    Ps = [P for P, _ in PR]
+    b = gen.uniform_vector(A.m, cfg.seed).to(device)
+    return A, Ps, b, PR, N
+
+
+def gpu_step(amgt, A, Ps, b, x, ncycles, torch):
+    """The whole hot path once (inputs on the device)."""
+    MA = amgt.from_csr(A)                       # a1
+    MPs = [amgt.from_csr(P) for P in Ps]        # a1 (P_k)
+    H = amgt.Hierarchy(MA, MPs, level_prec=LEVEL_PREC[:len(Ps) + 1])  # a2-a8
+    x.zero_()
+    res, calls = H.vcycle(b, x, ncycles)        # a9-a10
+    H.close()
+    MA.free()
+    for M in MPs:
+        M.free()
+    return res, calls
+
+
+def run_gpu(args):
+    import numpy as np
+    import torch
+
+    import gen
+    import paper_conf_sc_luzwflcy0c024_b200 as amgt
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl")
+    cfg = gen.configs.CONFIGS[args.config]
+    A, Ps, b, PR, N = make_inputs(cfg, "cuda")
+    x = torch.zeros(4 * ((A.m + 3) // 4), dtype=torch.float64, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # ---- one instrumented step: per-class device times and algorithmic bytes
+    amgt.timing_reset()
+    amgt.timing_enable(True)
+    res, calls = gpu_step(amgt, A, Ps, b, x, args.cycles, torch)
+    torch.cuda.synchronize()
+    prof = amgt.timing_read()
+    amgt.timing_enable(False)
+    sz, flops = gpu_sizes(amgt, A, Ps)
+    bm = byte_model(sz, args.cycles)
+    bytes_step = sum(bm.values())
+    l0 = sz["lev"][0]
+    spmv_l1_bytes = l0["T"] * (16 * 8 + 6) + (l0["BR"] + 1) * 8 + 4 * l0["BC"] * 8 + 4 * l0["BR"] * 8
+
+    # ---- warm-up
+    for _ in range(args.warmup):
+        gpu_step(amgt, A, Ps, b, x, args.cycles, torch)
+    barrier()
+
+    # ---- timed region: K steps, live events around every level-1 SpMV (dominant kernel)
+    amgt.timing_reset()
+    amgt.timing_enable(True)
+    launches0 = amgt.launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            gpu_step(amgt, A, Ps, b, x, args.cycles, torch)
+        ev1.record(stream)
+        barrier()
+    launches = amgt.launch_count() - launches0
+    live = amgt.timing_read()
+    amgt.timing_enable(False)
+    ms_total = ev0.elapsed_time(ev1)
+    if dist:
+        t = torch.tensor([ms_total], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms_step = ms_total / args.steps
+    value = bytes_step * world / (ms_step * 1e-3) / 1e9
+
+    spmv_l1 = live["spmv_l1"]
+    spmv_avg_ms = spmv_l1["ms"] / max(spmv_l1["launches"], 1)
+    achieved = spmv_l1_bytes / (spmv_avg_ms * 1e-3) / 1e9
+    peak, peak_kind = _peaks()
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_spmv_l1_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    setup_ms = sum(prof[k]["ms"] for k in ("spgemm_symbolic", "spgemm_numeric", "csr2mbsr", "mbsr2csr", "cast"))
+    spgemm_ms = prof["spgemm_symbolic"]["ms"] + prof["spgemm_numeric"]["ms"]
+
+    # ---- e2e: same step through the public API with host (pinned) inputs and outputs
+    hA = type(A)(A.m, A.n, A.row_ptr.cpu().pin_memory(), A.col.cpu().pin_memory(), A.val.cpu().pin_memory())
+    hPs = [type(P)(P.m, P.n, P.row_ptr.cpu().pin_memory(), P.col.cpu().pin_memory(), P.val.cpu().pin_memory())
+           for P in Ps]
+    hb = b.cpu().pin_memory()
+    hx = torch.empty(x.numel(), dtype=torch.float64).pin_memory()
+    h2d = sum(t.numel() * t.element_size() for M in [hA, *hPs] for t in (M.row_ptr, M.col, M.val)) + hb.numel() * 8
+    d2h = hx.numel() * 8 + (args.cycles + 1) * 8
+    e2e_steps = max(1, min(args.steps, 3))
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(e2e_steps):
+        dA = hA.to("cuda")
+        dPs = [P.to("cuda") for P in hPs]
+        db = hb.to("cuda", non_blocking=True)
+        gpu_step(amgt, dA, dPs, db, x, args.cycles, torch)  # residual norms come back to the host here
+        hx.copy_(x, non_blocking=True)
+    e1.record(stream)
+    barrier()
+    e2e_ms = e0.elapsed_time(e1) / e2e_steps
+    if dist:
+        t = torch.tensor([e2e_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+    e2e_val = bytes_step * world / (e2e_ms * 1e-3) / 1e9
+
+    line = {
+        "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64/f32/f16 (per AMG level, L266)", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {cfg.description}", "grid": f"{N}^3", "levels": len(Ps) + 1,
+                   "level_prec": list(LEVEL_PREC[:len(Ps) + 1]), "vcycles_per_step": args.cycles,
+                   "smoother": "weighted Jacobi w=2/3, nu1=nu2=1", "parallelism": f"replicas x{world}",
+                   "l2": "inputs larger than L2 (level-1 mBSR A = %.0f MB vs 126 MB L2); no flush" %
+                         (A1_bytes_mb(A)), "spmv_calls_per_step": calls},
+        "roofline": {"kernel": "k_spmv_rows<double,double,double> (level-1 FP64 SpMV)", "bound": "hbm",
+                     "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "peak_source": peak_kind,
+                     "bytes_per_launch": spmv_l1_bytes, "avg_launch_us": round(spmv_avg_ms * 1e3, 2),
+                     "launches_timed": spmv_l1["launches"], "traffic": traffic},
+        "components": {"setup_ms": round(setup_ms, 3), "solve_ms": round(ms_step - setup_ms, 3),
+                       "spmv_l1_gbs": round(achieved, 1),
+                       "spgemm_gflops": round(flops / (spgemm_ms * 1e-3) / 1e9, 2) if spgemm_ms else None,
+                       "rap_flops": flops, "bytes_per_step": bytes_step,
+                       "bytes_by_phase": {k: int(v) for k, v in bm.items()},
+                       "per_class_ms": {k: round(v["ms"], 3) for k, v in prof.items()},
+                       "final_rel_residual": res[-1] / res[0]},
+        "e2e": {"value": round(e2e_val, 2), "unit": "GB/s", "ms_per_step": round(e2e_ms, 3),
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(args, bm, A, PR)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+def A1_bytes_mb(A):
+    # rough level-1 mBSR footprint (FP64 tiles) from the CSR size: reported in config only
+    return A.nnz * 134.0 / 4.0 / 1e6
+
+
+# ------------------------------------------------------------------ oracle (CPU) legs
+def oracle_sample(args, A, PR, cycles):
+    """The oracle's version of a step, on a bounded number of V-cycles."""
+    import gen
+    import oracle
+    t0 = time.perf_counter()
+    Ao = oracle.as_csr(A.to("cpu"))
+    oracle.csr_to_mbsr(Ao)                     # a1 (level 1)
+    PRo = [(oracle.as_csr(P.to("cpu")), oracle.as_csr(R.to("cpu"))) for P, R in PR]
+    As = oracle.build_hierarchy(Ao, PRo)       # a7 (RAP chain)
+    for Ak in As[1:]:
+        oracle.mbsr_to_csr(oracle.csr_to_mbsr(Ak))  # a8 round trips (2L-1 conversions)
+    b = gen.uniform_vector(Ao.m, gen.configs.CONFIGS[args.config].seed).numpy()
+    t1 = time.perf_counter()
+    oracle.vcycle(As, PRo, b, ncycles=cycles)
+    t2 = time.perf_counter()
+    return t1 - t0, t2 - t1
+
+
+def cpu_baseline(args, bm, A, PR):
+    import oracle
+    cycles = args.cpu_cycles
+    ts, tv = oracle_sample(args, A, PR, cycles)
+    by = sample_bytes_model(bm, cycles, args.cycles)
+    return {"value": round(by / (ts + tv) / 1e9, 4), "unit": "GB/s", "cores": oracle.max_threads(), "kind": "oracle",
+            "sample": f"{args.config}: CSR->mBSR + full RAP hierarchy + {cycles} of {args.cycles} V-cycles "
+                      f"(FP64 C oracle, OpenMP rows); setup {ts:.2f}s, solve {tv:.2f}s"}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import gen
+    import oracle
+    cfg = gen.configs.CONFIGS[args.config]
+    A, Ps, b, PR, N = make_inputs(cfg, "cpu")
+    bm = byte_model(oracle_sizes(A, PR), args.cycles)  # same byte model as the GPU arm
+    cycles = args.cpu_cycles
+    for _ in range(args.warmup):
+        oracle_sample(args, A, PR, cycles)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle_sample(args, A, PR, cycles)
+    dt = (time.perf_counter() - t0) / args.steps
+    val = sample_bytes_model(bm, cycles, args.cycles) / dt / 1e9
+    sample = f"{args.config}: CSR->mBSR + full RAP hierarchy + {cycles} of {args.cycles} V-cycles per step (FP64 C oracle)"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "GB/s", "n_gpus": 1,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 2), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {cfg.description}", "levels": cfg.nlev},
+        "cpu_baseline": {"value": round(val, 4), "unit": "GB/s", "cores": oracle.max_threads(), "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": round(val, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="amgt", choices=["amgt", "reference"])
+    ap.add_argument("--config", default="cfg2", choices=["cfg2", "cfg3", "cfg5"])
+    ap.add_argument("--cycles", type=int, default=50, help="V-cycles per step (paper: 50, L308)")
+    ap.add_argument("--cpu-cycles", type=int, default=10, help="V-cycles in the oracle's bounded sample")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3) if args.impl == "amgt" else args.warmup
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_gpu(args)
+
+
+if __name__ == "__main__":
+    main()

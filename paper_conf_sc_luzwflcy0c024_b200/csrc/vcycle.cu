@@ -252,7 +252,7 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     for (int k = 0; k < nlev; ++k) {
         amgt_level& L = H->L[k];
         const amgt_prec pk = o->level_prec[k];
-        L.vprec = (k == 0) ? AMGT_FP64 : AMGT_FP32;
+        L.vprec = (k == 0 || pk == AMGT_FP64) ? AMGT_FP64 : AMGT_FP32;  // R16
         if (k == 0) {
             if (pk == A->prec) {
                 L.A = *A;  // borrowed
