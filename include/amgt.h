@@ -252,6 +252,7 @@ amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H);
  * Classes: 0 SpMV level-1, 1 SpMV other levels, 2 SpGEMM symbolic, 3 SpGEMM numeric,
  * 4 CSR->mBSR, 5 mBSR->CSR, 6 cast, 7 vector ops. */
 #define AMGT_TIMER_CLASSES 8
+/* on: 0 = off, -1 = all classes, otherwise a bitmask (bit c enables class c). */
 amgt_status amgt_timing_enable(int on);
 amgt_status amgt_timing_reset(void);
 /* Syncs the recorded events; fills ms_total[8], launches[8] and bytes[8] (algorithmic

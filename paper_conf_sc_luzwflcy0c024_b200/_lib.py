@@ -377,8 +377,9 @@ class Hierarchy:
 TIMER_CLASSES = ("spmv_l1", "spmv", "spgemm_symbolic", "spgemm_numeric", "csr2mbsr", "mbsr2csr", "cast", "vector")
 
 
-def timing_enable(on: bool = True):
-    _check(_L.amgt_timing_enable(1 if on else 0))
+def timing_enable(on=True):
+    """True = all classes, False = off, or an int bitmask over TIMER_CLASSES."""
+    _check(_L.amgt_timing_enable(-1 if on is True else (0 if on is False else int(on))))
 
 
 def timing_reset():

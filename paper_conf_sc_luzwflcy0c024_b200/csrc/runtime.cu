@@ -160,7 +160,7 @@ struct TimerRec {
     cudaEvent_t e0, e1;
 };
 static std::mutex g_tmu;
-static bool g_timing = false;
+static unsigned g_timing = 0;  // bitmask of enabled timer classes
 static std::vector<TimerRec> g_recs;
 static std::vector<cudaEvent_t> g_pool;
 static size_t g_used = 0;
@@ -175,7 +175,7 @@ static cudaEvent_t pool_event() {
 }
 
 TimerScope::TimerScope(int c, double b, cudaStream_t st) : cls(c), bytes(b), s(st), slot(-1) {
-    if (!g_timing) return;
+    if (!(g_timing & (1u << c))) return;
     std::lock_guard<std::mutex> lk(g_tmu);
     TimerRec r{c, b, pool_event(), pool_event()};
     cudaEventRecord(r.e0, s);
@@ -210,7 +210,7 @@ amgt_status amgt_set_tc_threshold(int spgemm_threshold, int spmv_threshold) {
 
 amgt_status amgt_timing_enable(int on) {
     std::lock_guard<std::mutex> lk(g_tmu);
-    g_timing = on != 0;
+    g_timing = on < 0 ? 0xFFu : (unsigned)on & 0xFFu;
     return AMGT_OK;
 }
 

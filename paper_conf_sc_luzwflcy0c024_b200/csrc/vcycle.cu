@@ -290,9 +290,10 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             const amgt_prec pn = o->level_prec[k + 1];
             if (pn != Ac.prec) {
                 st = cast_impl(&Ac, pn, &N.A, a);
-                mbsr_release(&Ac, a);
-                if (st != AMGT_OK) return st;
-                N.A.own |= 1u;  // the cast shares Ac's structure: take ownership of it
+                if (st != AMGT_OK) { mbsr_release(&Ac, a); return st; }
+                Ac.own &= ~1u;  // the cast shares Ac's structure: move its ownership to N.A
+                mbsr_release(&Ac, a);  // frees Ac's values only
+                N.A.own |= 1u;
             } else {
                 N.A = Ac;
             }
