@@ -207,6 +207,23 @@ amgt_status amgt_spmv_get_stats(const amgt_mbsr* A, amgt_spmv_stats* st_host);
 amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec,
                       void* stream);
 
+/*
+ * SpMV with a fused Alg. 2 vector epilogue (NEXT-1 of SURVEY §8(f)), element-wise on
+ * t = (A x)_i, in y's precision:
+ *   AMGT_EPI_Y        y = t
+ *   AMGT_EPI_JACOBI   y = x + omega * dinv .* (b - t)   (weighted Jacobi sweep, Alg. 2 lines 2/10,
+ *                                                       out of place: y != x, A square)
+ *   AMGT_EPI_RESIDUAL y = b - t                          (Alg. 2 line 3)
+ *   AMGT_EPI_ACCUM    y = y + t                          (interpolation + correction, lines 8-9)
+ * b and dinv have y's precision and length 4*blc_row.
+ */
+#define AMGT_EPI_Y 0
+#define AMGT_EPI_JACOBI 1
+#define AMGT_EPI_RESIDUAL 2
+#define AMGT_EPI_ACCUM 3
+amgt_status amgt_spmv_fused(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec, int mode,
+                            const void* b, const void* dinv, double omega, void* stream);
+
 /* ------------------------------------------------------ hierarchy + V-cycle (§II) */
 
 typedef struct {

@@ -89,6 +89,7 @@ _sigs = {
     "amgt_spmv_analyze": (_int, [_P(c_mbsr), _P(c_allocator), _vp]),
     "amgt_spmv_get_stats": (_int, [_P(c_mbsr), _P(c_spmv_stats)]),
     "amgt_spmv": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _vp]),
+    "amgt_spmv_fused": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _int, _vp, _vp, ctypes.c_double, _vp]),
     "amgt_hierarchy_create": (_int, [_P(c_mbsr), _P(_P(c_mbsr)), _int, _P(c_vcycle_opts), _P(c_allocator), _vp,
                                      _P(_vp)]),
     "amgt_hierarchy_level": (_int, [_vp, _int, _P(_P(c_mbsr)), _P(_P(c_mbsr)), _P(_P(c_mbsr))]),
@@ -310,6 +311,20 @@ def spmv(A: Mbsr, x: torch.Tensor, y: torch.Tensor | None = None, stream=None) -
     yp = {torch.float64: FP64, torch.float32: FP32}[y.dtype]
     assert y.numel() >= 4 * A.blc_row and x.is_contiguous() and y.is_contiguous()
     _check(_L.amgt_spmv(ctypes.byref(A.c), x.data_ptr(), xp, y.data_ptr(), yp, _stream(stream)))
+    return y
+
+
+EPI = {"y": 0, "jacobi": 1, "residual": 2, "accum": 3}
+
+
+def spmv_fused(A: Mbsr, x: torch.Tensor, y: torch.Tensor, mode: str, b: torch.Tensor | None = None,
+               dinv: torch.Tensor | None = None, omega: float = 2.0 / 3.0, stream=None) -> torch.Tensor:
+    """amgt_spmv_fused: y = epilogue((A x)_i) — see include/amgt.h (AMGT_EPI_*)."""
+    xp = {torch.float64: FP64, torch.float32: FP32}[x.dtype]
+    yp = {torch.float64: FP64, torch.float32: FP32}[y.dtype]
+    _check(_L.amgt_spmv_fused(ctypes.byref(A.c), x.data_ptr(), xp, y.data_ptr(), yp, EPI[mode],
+                              b.data_ptr() if b is not None else None, dinv.data_ptr() if dinv is not None else None,
+                              float(omega), _stream(stream)))
     return y
 
 

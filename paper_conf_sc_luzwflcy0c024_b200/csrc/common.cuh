@@ -139,6 +139,15 @@ struct TimerScope {  // records start/end events on `s` when timing is enabled
     ~TimerScope();
 };
 
+// SpMV epilogue selection (AMGT_EPI_* in amgt.h) and its operands.
+struct EpiArgs {
+    int mode;
+    const void* b;
+    const void* dinv;
+    const void* xs;
+    double omega;
+};
+
 extern int g_tc_thr_spgemm;
 extern int g_tc_thr_spmv;
 

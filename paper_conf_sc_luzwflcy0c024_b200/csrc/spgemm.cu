@@ -43,6 +43,7 @@ struct SymCtx {  // device pointers shared by the symbolic kernels
 };
 
 // ---------------------------------------------------------------- analysis + binning
+template <bool STATS>
 __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, unsigned long long* __restrict__ stats,
                           int tc_thr) {
     // stats: [0..7] bin counts, [8] cub_total, [9] pairs_nonzero, [10] pairs_tc, [11] scalar products
@@ -56,6 +57,7 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
             const int32_t K = c.aidx[t];
             const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
             cub += b1 - b0;
+            if (!STATS) continue;
             const uint32_t ma = c.amap[t];
             const bool tc = __popc(ma) >= tc_thr;
             for (int64_t j = b0; j < b1; ++j) {  // pair statistics (info only)
@@ -90,9 +92,16 @@ __global__ void k_bin_scatter(int64_t BR, const int64_t* __restrict__ bin_of, co
         for (int b = 0; b < NBINS; ++b) { off[b] = s; s += stats[b]; }
     }
     __syncthreads();
-    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
-        const int b = (int)bin_of[I];
-        rows[off[b] + atomicAdd(&cursor[b], 1ull)] = (int32_t)I;
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < BR; base += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t I = base + threadIdx.x;
+        const int b = I < BR ? (int)bin_of[I] : -1;
+        const uint32_t peers = __match_any_sync(0xffffffffu, b);  // warp-aggregated atomics
+        const int leader = __ffs(peers) - 1;
+        unsigned long long pos = 0;
+        if (lane == leader && b >= 0) pos = atomicAdd(&cursor[b], (unsigned long long)__popc(peers));
+        pos = __shfl_sync(0xffffffffu, pos, leader);
+        if (b >= 0) rows[off[b] + pos + __popc(peers & ((1u << lane) - 1u))] = (int32_t)I;
     }
 }
 
@@ -518,16 +527,11 @@ __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b)
 // T = storage type, Acc = accumulation type (double for FP64, float otherwise).
 // gacc: FP32 accumulation workspace for FP16 global-path rows (indexed like C values).
 template <typename T, typename Acc>
-__global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(int64_t BR, SymCtx c, const T* __restrict__ aval,
-                                                            const T* __restrict__ bval, const int64_t* __restrict__ cptr,
-                                                            const int32_t* __restrict__ cidx_g,
-                                                            const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
-                                                            Acc* __restrict__ gacc, int tc_thr) {
-    __shared__ NumSmem<Acc> sm[NUM_WARPS];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t I = (int64_t)blockIdx.x * NUM_WARPS + w;
-    if (I >= BR) return;
-    NumSmem<Acc>& S = sm[w];
+__device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, const T* __restrict__ aval,
+                                                 const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                 const int32_t* __restrict__ cidx_g,
+                                                 const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+                                                 Acc* __restrict__ gacc, int tc_thr, NumSmem<Acc>& S, int lane) {
     const int64_t c0 = cptr[I];
     const int nC = (int)(cptr[I + 1] - c0);
     if (nC == 0) return;
@@ -537,7 +541,7 @@ __global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(int64_t BR, SymCtx c
     Acc* gbase = nullptr;
     if (small) {
         if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
-        for (int e = lane; e < CAP * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
+        for (int e = lane; e < nC * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
     } else {
         gbase = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
         for (int64_t e = lane; e < 16 * (int64_t)nC; e += 32) gbase[e] = Acc(0);
@@ -703,6 +707,219 @@ __global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(int64_t BR, SymCtx c
     }
 }
 
+// Warp per C block row for the rows in `rows` (count read from the device: the rows the
+// group kernel could not take, nC > GROUP_NC).  Persistent grid-stride over the list.
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(const int32_t* __restrict__ rows,
+                                                            const unsigned long long* __restrict__ nrows_dev, SymCtx c,
+                                                            const T* __restrict__ aval, const T* __restrict__ bval,
+                                                            const int64_t* __restrict__ cptr,
+                                                            const int32_t* __restrict__ cidx_g,
+                                                            const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+                                                            Acc* __restrict__ gacc, int tc_thr) {
+    __shared__ NumSmem<Acc> sm[NUM_WARPS];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t nrows = (int64_t)*nrows_dev;
+    for (int64_t wi = (int64_t)blockIdx.x * NUM_WARPS + w; wi < nrows; wi += (int64_t)gridDim.x * NUM_WARPS) {
+        numeric_warp_row<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, gacc, tc_thr, sm[w], lane);
+        __syncwarp();
+    }
+}
+
+// ---------------------------------------------------------------- numeric: group kernel
+// One 4-lane group per C block row with <= GROUP_NC tiles, 8 rows per warp.  Lane r owns
+// row r of every C tile of its row (accumulators in registers).  The group walks its
+// (A tile, B tile) pairs in order (A tiles ascending, B tiles ascending): deterministic,
+// no conflicts.  Warp-synchronous rounds (one pair per group per round) let the groups
+// whose pair has a dense A tile (POPCOUNT >= tc_thr, FP64) share DMMA m8n8k4 instructions
+// two at a time: fragA = [A_a; A_b], fragB = [B_a | B_b], and the diagonal quadrants of
+// fragC are A_a B_a and A_b B_b (L157-171; the paper pairs two B tiles of one A tile, we
+// pair two groups' tile products — same instruction, same "keep half" extraction).
+// Rows with more tiles are appended to `big` for k_numeric.
+constexpr int GROUP_NC = 8;
+
+template <typename T> struct RowIO;
+template <> struct RowIO<double> {
+    static __device__ __forceinline__ void load(const double* p, double (&v)[4]) {
+        const double2 a = __ldg(reinterpret_cast<const double2*>(p));
+        const double2 b = __ldg(reinterpret_cast<const double2*>(p) + 1);
+        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+    }
+    static __device__ __forceinline__ void store(double* p, const double (&v)[4]) {
+        reinterpret_cast<double2*>(p)[0] = make_double2(v[0], v[1]);
+        reinterpret_cast<double2*>(p)[1] = make_double2(v[2], v[3]);
+    }
+};
+template <> struct RowIO<float> {
+    static __device__ __forceinline__ void load(const float* p, float (&v)[4]) {
+        const float4 a = __ldg(reinterpret_cast<const float4*>(p));
+        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+    }
+    static __device__ __forceinline__ void store(float* p, const float (&v)[4]) {
+        *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    }
+};
+template <> struct RowIO<__half> {
+    static __device__ __forceinline__ void load(const __half* p, float (&v)[4]) {
+        const uint2 u = __ldg(reinterpret_cast<const uint2*>(p));
+        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
+        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
+        v[0] = lo.x; v[1] = lo.y; v[2] = hi.x; v[3] = hi.y;
+    }
+    static __device__ __forceinline__ void store(__half* p, const float (&v)[4]) {
+        __half2 a = __floats2half2_rn(v[0], v[1]), b = __floats2half2_rn(v[2], v[3]);
+        uint2 u;
+        u.x = *reinterpret_cast<uint32_t*>(&a);
+        u.y = *reinterpret_cast<uint32_t*>(&b);
+        *reinterpret_cast<uint2*>(p) = u;
+    }
+};
+
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, const T* __restrict__ aval,
+                                                       const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                       const int32_t* __restrict__ cidx_g,
+                                                       const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+                                                       int32_t* __restrict__ big, unsigned long long* __restrict__ nbig,
+                                                       int tc_thr) {
+    const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
+    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (wid * 8 >= BR) return;
+    const int64_t I = wid * 8 + g;
+    int64_t c0 = 0;
+    int nC = 0;
+    if (I < BR) {
+        c0 = cptr[I];
+        nC = (int)(cptr[I + 1] - c0);
+        if (nC > GROUP_NC) {
+            if (r == 0) big[atomicAdd(nbig, 1ull)] = (int32_t)I;
+            nC = 0;
+        }
+    }
+    int32_t cid[GROUP_NC];
+#pragma unroll
+    for (int k = 0; k < GROUP_NC; ++k) cid[k] = k < nC ? cidx_g[c0 + k] : INT_MAX;
+    Acc acc[GROUP_NC][4];
+#pragma unroll
+    for (int k = 0; k < GROUP_NC; ++k)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) acc[k][e] = Acc(0);
+    // pair cursor
+    int64_t t = 0, a1 = 0, j = 0, jend = 0;
+    uint32_t mA = 0;
+    Acc arow[4] = {Acc(0), Acc(0), Acc(0), Acc(0)};
+    if (nC > 0) {
+        t = c.aptr[I];
+        a1 = c.aptr[I + 1];
+    }
+    auto next_a = [&]() {  // move to the next A tile with a non-empty B row
+        while (t < a1) {
+            const int32_t K = c.aidx[t];
+            j = c.bptr[K];
+            jend = c.bptr[K + 1];
+            if (j < jend) {
+                mA = c.amap[t];
+                RowIO<T>::load(aval + 16 * t + 4 * r, arow);
+                return;
+            }
+            ++t;
+        }
+    };
+    next_a();
+    for (;;) {
+        const bool has = t < a1;
+        if (!__any_sync(0xffffffffu, has)) break;
+        uint32_t mC = 0;
+        int q = 0;
+        if (has) {
+            mC = bitmap_multiply(mA, c.bmap[j]);
+            if (mC) {
+                const int32_t J = c.bidx[j];
+#pragma unroll
+                for (int k = 0; k < GROUP_NC; ++k) q = (cid[k] == J) ? k : q;
+            }
+        }
+        bool dense = false;
+        if constexpr (sizeof(T) == 8) dense = mC != 0 && __popc(mA) >= tc_thr;
+        if (mC && !dense) {  // CUDA-core route: lane r computes row r of A_t * B_j
+            Acc b0[4], b1[4], b2[4], b3[4], v[4];
+            const T* bp = bval + 16 * j;
+            RowIO<T>::load(bp, b0);
+            RowIO<T>::load(bp + 4, b1);
+            RowIO<T>::load(bp + 8, b2);
+            RowIO<T>::load(bp + 12, b3);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                Acc s_ = arow[0] * b0[e];
+                s_ = fma(arow[1], b1[e], s_);
+                s_ = fma(arow[2], b2[e], s_);
+                s_ = fma(arow[3], b3[e], s_);
+                v[e] = s_;
+            }
+#pragma unroll
+            for (int k = 0; k < GROUP_NC; ++k)
+                if (k == q)
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) acc[k][e] += v[e];
+        }
+        if constexpr (sizeof(T) == 8) {
+            uint32_t dm = __ballot_sync(0xffffffffu, dense && r == 0);
+            while (dm) {  // tensor-core route, two groups per DMMA
+                const int ga = (__ffs(dm) - 1) >> 2;
+                dm &= dm - 1;
+                int gb = -1;
+                if (dm) { gb = (__ffs(dm) - 1) >> 2; dm &= dm - 1; }
+                const int row8 = lane >> 2, k4 = lane & 3;
+                const int64_t ta = __shfl_sync(0xffffffffu, t, 4 * ga);
+                const int64_t ja = __shfl_sync(0xffffffffu, j, 4 * ga);
+                const int64_t tb = __shfl_sync(0xffffffffu, t, 4 * (gb < 0 ? ga : gb));
+                const int64_t jb = __shfl_sync(0xffffffffu, j, 4 * (gb < 0 ? ga : gb));
+                double fa = 0.0, fb = 0.0;
+                if (row8 < 4) {
+                    fa = (double)aval[16 * ta + 4 * row8 + k4];
+                    fb = (double)bval[16 * ja + 4 * k4 + row8];
+                } else if (gb >= 0) {
+                    fa = (double)aval[16 * tb + 4 * (row8 - 4) + k4];
+                    fb = (double)bval[16 * jb + 4 * k4 + (row8 - 4)];
+                }
+                double d0 = 0.0, d1 = 0.0;
+                dmma(d0, d1, fa, fb);
+                // C_a row r: lanes (r, 0) and (r, 1); C_b row r: lanes (4+r, 2) and (4+r, 3)
+                const bool isb = (g == gb);
+                const int s0 = isb ? 4 * (4 + r) + 2 : 4 * r;
+                const double x0 = __shfl_sync(0xffffffffu, d0, s0), x1 = __shfl_sync(0xffffffffu, d1, s0);
+                const double x2 = __shfl_sync(0xffffffffu, d0, s0 + 1), x3 = __shfl_sync(0xffffffffu, d1, s0 + 1);
+                if (g == ga || isb) {
+#pragma unroll
+                    for (int k = 0; k < GROUP_NC; ++k)
+                        if (k == q) {
+                            acc[k][0] += x0; acc[k][1] += x1; acc[k][2] += x2; acc[k][3] += x3;
+                        }
+                }
+            }
+        }
+        if (has) {  // advance the cursor
+            if (++j == jend) {
+                ++t;
+                next_a();
+            }
+        }
+    }
+    // write out: lane r writes row r of each tile, +0.0 where the bit is clear (R2)
+#pragma unroll
+    for (int k = 0; k < GROUP_NC; ++k) {
+        if (k < nC) {
+            const uint32_t nib = (cmap_g[c0 + k] >> (4 * r)) & 0xFu;
+            Acc o[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? acc[k][e] : Acc(0);
+            T* dst = cval + 16 * (c0 + k) + 4 * r;
+            if constexpr (sizeof(T) == 2) RowIO<T>::store(dst, o);
+            else RowIO<T>::store(dst, o);
+        }
+    }
+}
+
 static unsigned capped(int64_t blocks) {
     const int64_t cap = (int64_t)num_sms() * 32;
     return (unsigned)(blocks < 1 ? 1 : (blocks > cap ? cap : blocks));
@@ -801,7 +1018,10 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     {
         TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
         if (BR > 0) {
-            k_analyze<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+            if (info)
+                k_analyze<true><<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+            else
+                k_analyze<false><<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
             AMGT_LAUNCHED();
             k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats.p, cursor.p, rows.p);
             AMGT_LAUNCHED();
@@ -855,11 +1075,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     const int64_t BR = A->blc_row;
     if (BR == 0 || C->blc_num == 0) return AMGT_OK;
     SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
+    Scratch<int32_t> big;
+    Scratch<unsigned long long> nbig;
+    AMGT_TRY(big.init(a, BR));
+    AMGT_TRY(nbig.init(a, 1));
+    AMGT_CUDA(cudaMemsetAsync(nbig.p, 0, sizeof(unsigned long long), s));
+    k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
+        BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val, big.p,
+        nbig.p, g_tc_thr_spgemm);
+    AMGT_LAUNCHED();
     Scratch<Acc> gacc;
     if (sizeof(T) < sizeof(Acc)) AMGT_TRY(gacc.init(a, 16 * (size_t)C->blc_num));
-    k_numeric<T, Acc><<<(unsigned)ceil_div(BR, NUM_WARPS), NUM_WARPS * 32, 0, s>>>(
-        BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
-        sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
+    k_numeric<T, Acc><<<(unsigned)num_sms() * 4, NUM_WARPS * 32, 0, s>>>(
+        big.p, nbig.p, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map,
+        (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }

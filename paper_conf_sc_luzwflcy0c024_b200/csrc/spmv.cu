@@ -77,8 +77,31 @@ __device__ __forceinline__ float4 x_quad(const double* x, int64_t J) {
     return make_float4((float)a.x, (float)a.y, (float)b.x, (float)b.y);
 }
 
-template <typename Y> __device__ __forceinline__ void store_y(Y* y, int64_t i, double v) { y[i] = (Y)v; }
-template <typename Y> __device__ __forceinline__ void store_y(Y* y, int64_t i, float v) { y[i] = (Y)v; }
+// Epilogue applied to each (A x)_i (the Alg. 2 vector steps fused into the SpMV, NEXT-1):
+//   EPI_Y        y_i = (A x)_i
+//   EPI_JACOBI   y_i = xs_i + w dinv_i (b_i - (A x)_i)       (out-of-place weighted Jacobi, R21)
+//   EPI_RESIDUAL y_i = b_i - (A x)_i                          (Alg. 2 line 3)
+//   EPI_ACCUM    y_i = y_i + (A x)_i                          (interpolation + correction, lines 8-9)
+// Vector arithmetic is done in the y precision, as the separate vector kernels did.
+template <typename XT, typename YT>
+struct Epi {
+    YT* y;
+    const YT* b;
+    const YT* dinv;
+    const XT* xs;
+    YT omega;
+    int mode;
+    __device__ __forceinline__ void apply(int64_t i, double v) const { put(i, (YT)v); }
+    __device__ __forceinline__ void apply(int64_t i, float v) const { put(i, (YT)v); }
+    __device__ __forceinline__ void put(int64_t i, YT t) const {
+        switch (mode) {
+            case AMGT_EPI_JACOBI: y[i] = (YT)xs[i] + omega * dinv[i] * (b[i] - t); break;
+            case AMGT_EPI_RESIDUAL: y[i] = b[i] - t; break;
+            case AMGT_EPI_ACCUM: y[i] = y[i] + t; break;
+            default: y[i] = t;
+        }
+    }
+};
 
 // ---------------------------------------------------------------- FP64 tile step
 // Lane q of the group: elements e0 = 2q, 2q+1 (row q>>1) and e1 = 8+2q, 9+2q (row 2+(q>>1)),
@@ -111,8 +134,8 @@ template <typename MatT, typename XT, typename YT>
 __global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __restrict__ bptr,
                                                    const int32_t* __restrict__ bidx,
                                                    const uint16_t* __restrict__ bmap, const MatT* __restrict__ bval,
-                                                   const XT* __restrict__ x, YT* __restrict__ y, int64_t long_thr,
-                                                   int tc_thr) {
+                                                   const XT* __restrict__ x, const Epi<XT, YT> epi,
+                                                   int64_t long_thr, int tc_thr) {
     const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t I = wid * 8 + g;
@@ -202,13 +225,13 @@ __global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __
             const double tcmine = __shfl_sync(0xffffffffu, tcacc, 4 * g + myrow);
             const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
             const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
-            if (write) store_y(y, 4 * I + myrow, ((q & 1) ? s1 : s0) + tcmine);
+            if (write) epi.apply(4 * I + myrow, ((q & 1) ? s1 : s0) + tcmine);
             return;
         }
         const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
         const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
         const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
-        if (write) store_y(y, 4 * I + myrow, (q & 1) ? s1 : s0);
+        if (write) epi.apply(4 * I + myrow, (q & 1) ? s1 : s0);
     } else {
         float acc = 0.f;
         for (int64_t t = t0; t < t1; ++t) {
@@ -230,7 +253,7 @@ __global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __
             acc = (nib & 4u) ? fmaf(a2, xv.z, acc) : acc;
             acc = (nib & 8u) ? fmaf(a3, xv.w, acc) : acc;
         }
-        if (write) store_y(y, 4 * I + q, acc);
+        if (write) epi.apply(4 * I + q, acc);
     }
 }
 
@@ -297,17 +320,17 @@ __global__ void __launch_bounds__(256) k_spmv_chunks(int64_t nchunks, const int6
     }
 }
 
-template <typename Acc, typename YT>
+template <typename Acc, typename XT, typename YT>
 __global__ void k_spmv_combine(int64_t nlong, const int32_t* __restrict__ long_rows,
                                const int64_t* __restrict__ chunk_ptr, const Acc* __restrict__ partial,
-                               YT* __restrict__ y) {
+                               const Epi<XT, YT> epi) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= 4 * nlong) return;
     const int64_t lr = i >> 2;
     const int r = (int)(i & 3);
     Acc s = 0;
     for (int64_t c = chunk_ptr[lr]; c < chunk_ptr[lr + 1]; ++c) s += partial[4 * c + r];
-    store_y(y, 4 * (int64_t)long_rows[lr] + r, s);
+    epi.apply(4 * (int64_t)long_rows[lr] + r, s);
 }
 
 // ---------------------------------------------------------------- analysis kernels
@@ -430,14 +453,15 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
 }
 
 template <typename MatT, typename XT, typename YT>
-static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, cudaStream_t s) {
+static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, cudaStream_t s) {
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
     const int64_t long_thr = (P && P->nlong > 0) ? WARP_CAPACITY : INT64_MAX;
     const int64_t BR = A->blc_row;
+    const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode};
     if (BR > 0) {
         const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 256);
         k_spmv_rows<MatT, XT, YT><<<blocks, 256, 0, s>>>(BR, A->blc_ptr, A->blc_idx, A->blc_map,
-                                                         (const MatT*)A->blc_val, (const XT*)x, (YT*)y, long_thr,
+                                                         (const MatT*)A->blc_val, (const XT*)x, epi, long_thr,
                                                          sizeof(MatT) == 8 ? g_tc_thr_spmv : 17);
         AMGT_LAUNCHED();
     }
@@ -447,19 +471,20 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, cudaS
             P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, P->long_rows,
             P->chunk_ptr, P->chunk_lr, (Acc*)P->partial);
         AMGT_LAUNCHED();
-        k_spmv_combine<Acc, YT><<<(unsigned)ceil_div(4 * P->nlong, 256), 256, 0, s>>>(
-            P->nlong, P->long_rows, P->chunk_ptr, (const Acc*)P->partial, (YT*)y);
+        k_spmv_combine<Acc, XT, YT><<<(unsigned)ceil_div(4 * P->nlong, 256), 256, 0, s>>>(
+            P->nlong, P->long_rows, P->chunk_ptr, (const Acc*)P->partial, epi);
         AMGT_LAUNCHED();
     }
     return AMGT_OK;
 }
 
 template <typename MatT>
-static amgt_status dispatch_xy(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s) {
-    if (xp == AMGT_FP64 && yp == AMGT_FP64) return launch_spmv<MatT, double, double>(A, x, y, s);
-    if (xp == AMGT_FP64 && yp == AMGT_FP32) return launch_spmv<MatT, double, float>(A, x, y, s);
-    if (xp == AMGT_FP32 && yp == AMGT_FP64) return launch_spmv<MatT, float, double>(A, x, y, s);
-    return launch_spmv<MatT, float, float>(A, x, y, s);
+static amgt_status dispatch_xy(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp,
+                               const EpiArgs& ea, cudaStream_t s) {
+    if (xp == AMGT_FP64 && yp == AMGT_FP64) return launch_spmv<MatT, double, double>(A, x, y, ea, s);
+    if (xp == AMGT_FP64 && yp == AMGT_FP32) return launch_spmv<MatT, double, float>(A, x, y, ea, s);
+    if (xp == AMGT_FP32 && yp == AMGT_FP64) return launch_spmv<MatT, float, double>(A, x, y, ea, s);
+    return launch_spmv<MatT, float, float>(A, x, y, ea, s);
 }
 
 double spmv_bytes(const amgt_mbsr* A, amgt_prec xp, amgt_prec yp) {
@@ -468,14 +493,21 @@ double spmv_bytes(const amgt_mbsr* A, amgt_prec xp, amgt_prec yp) {
            4.0 * A->blc_col * prec_bytes(xp) + 4.0 * A->blc_row * prec_bytes(yp);
 }
 
+amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, const EpiArgs& ea,
+                         cudaStream_t s, int timer_class) {
+    const double vec = 4.0 * A->blc_row * prec_bytes(yp);
+    const double extra = ea.mode == AMGT_EPI_JACOBI ? 3 * vec : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
+    TimerScope ts(timer_class, spmv_bytes(A, xp, yp) + extra, s);
+    switch (A->prec) {
+        case AMGT_FP64: return dispatch_xy<double>(A, x, xp, y, yp, ea, s);
+        case AMGT_FP32: return dispatch_xy<float>(A, x, xp, y, yp, ea, s);
+        default: return dispatch_xy<__half>(A, x, xp, y, yp, ea, s);
+    }
+}
+
 amgt_status spmv_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s,
                       int timer_class) {
-    TimerScope ts(timer_class, spmv_bytes(A, xp, yp), s);
-    switch (A->prec) {
-        case AMGT_FP64: return dispatch_xy<double>(A, x, xp, y, yp, s);
-        case AMGT_FP32: return dispatch_xy<float>(A, x, xp, y, yp, s);
-        default: return dispatch_xy<__half>(A, x, xp, y, yp, s);
-    }
+    return spmv_ex_impl(A, x, xp, y, yp, EpiArgs{AMGT_EPI_Y, nullptr, nullptr, nullptr, 0.0}, s, timer_class);
 }
 
 }  // namespace amgt
@@ -503,6 +535,18 @@ amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* 
         return fail(AMGT_ERR_ARG, "amgt_spmv: x/y precision must be FP64 or FP32");
     if (!prec_valid(A->prec)) return fail(AMGT_ERR_ARG, "amgt_spmv: bad matrix precision");
     return spmv_impl(A, x, xprec, y, yprec, (cudaStream_t)stream, TC_SPMV);
+}
+
+amgt_status amgt_spmv_fused(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec, int mode,
+                            const void* b, const void* dinv, double omega, void* stream) {
+    if (!A || (!x && A->blc_col > 0) || (!y && A->blc_row > 0)) return fail(AMGT_ERR_ARG, "amgt_spmv_fused: NULL argument");
+    if ((xprec != AMGT_FP64 && xprec != AMGT_FP32) || (yprec != AMGT_FP64 && yprec != AMGT_FP32))
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused: x/y precision must be FP64 or FP32");
+    if (mode < AMGT_EPI_Y || mode > AMGT_EPI_ACCUM) return fail(AMGT_ERR_ARG, "amgt_spmv_fused: bad mode");
+    if ((mode == AMGT_EPI_JACOBI || mode == AMGT_EPI_RESIDUAL) && !b) return fail(AMGT_ERR_ARG, "amgt_spmv_fused: b is NULL");
+    if (mode == AMGT_EPI_JACOBI && (!dinv || xprec != yprec || A->m != A->n || x == y))
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused: Jacobi needs dinv, a square A, x/y of one precision, x != y");
+    return spmv_ex_impl(A, x, xprec, y, yprec, EpiArgs{mode, b, dinv, x, omega}, (cudaStream_t)stream, TC_SPMV);
 }
 
 }  // extern "C"

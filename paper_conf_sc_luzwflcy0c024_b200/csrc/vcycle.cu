@@ -4,6 +4,7 @@
 // below, reading R16).  Smoother: weighted Jacobi x += w D^-1 (b - A x) (R21).
 // Coarsest level: MBSR2CSR (L262), dense Cholesky-based inverse in FP64 on the host,
 // applied on the device as a dense FP64 matvec (R22).
+#include <algorithm>
 #include <cmath>
 #include <vector>
 
@@ -18,6 +19,8 @@ amgt_status mbsr_to_csr_impl(const amgt_mbsr* A, int64_t* rp, int32_t* ci, doubl
 amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a);
 amgt_status spmv_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s,
                       int timer_class);
+amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, const EpiArgs& ea,
+                         cudaStream_t s, int timer_class);
 amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* Cout, amgt_spgemm_info* info,
                                  Alloc& a);
 amgt_status spgemm_numeric_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a);
@@ -31,7 +34,7 @@ struct amgt_level {
     bool ownA = false;
     int64_t npad = 0;         // 4 * blc_row
     amgt_prec vprec = AMGT_FP64;
-    void *b = nullptr, *x = nullptr, *r = nullptr, *t = nullptr, *dinv = nullptr;
+    void *b = nullptr, *x = nullptr, *r = nullptr, *t = nullptr, *dinv = nullptr;  // t: ping-pong partner of x
 };
 
 struct amgt_hierarchy {
@@ -68,32 +71,12 @@ __global__ void k_dinv(int64_t BR, int64_t m, const int64_t* __restrict__ bptr, 
     dinv[i] = (V)(d != 0.0 ? 1.0 / d : 0.0);
 }
 
-template <typename V>
-__global__ void k_jacobi(int64_t n, V* __restrict__ x, const V* __restrict__ b, const V* __restrict__ t,
-                         const V* __restrict__ dinv, V omega) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        x[i] = x[i] + omega * dinv[i] * (b[i] - t[i]);
-}
-
-template <typename V>
-__global__ void k_residual(int64_t n, V* __restrict__ r, const V* __restrict__ b, const V* __restrict__ t) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        r[i] = b[i] - t[i];
-}
-
-template <typename V>
-__global__ void k_axpy(int64_t n, V* __restrict__ x, const V* __restrict__ e) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        x[i] += e[i];
-}
-
-// Deterministic ||b - t||^2: fixed grid of NORM_BLOCKS, per-block partials, then one block.
-__global__ void k_resnorm_partial(int64_t n, const double* __restrict__ b, const double* __restrict__ t,
-                                  double* __restrict__ partial) {
+// Deterministic ||r||^2: fixed grid of NORM_BLOCKS, per-block partials, then one block.
+__global__ void k_resnorm_partial(int64_t n, const double* __restrict__ r, double* __restrict__ partial) {
     __shared__ double sh[32];
     double s = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double d = b[i] - t[i];
+        const double d = r[i];
         s = fma(d, d, s);
     }
     for (int d = 16; d; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
@@ -135,38 +118,6 @@ static unsigned vgrid(int64_t n) {
 }
 
 static size_t vbytes(amgt_prec p) { return p == AMGT_FP64 ? 8 : 4; }
-
-template <typename V>
-static amgt_status vec_jacobi(amgt_level& L, cudaStream_t s, double omega) {
-    TimerScope ts(TC_VEC, 5.0 * L.npad * sizeof(V), s);
-    k_jacobi<V><<<vgrid(L.npad), 256, 0, s>>>(L.npad, (V*)L.x, (const V*)L.b, (const V*)L.t, (const V*)L.dinv, (V)omega);
-    AMGT_LAUNCHED();
-    return AMGT_OK;
-}
-template <typename V>
-static amgt_status vec_residual(amgt_level& L, cudaStream_t s) {
-    TimerScope ts(TC_VEC, 3.0 * L.npad * sizeof(V), s);
-    k_residual<V><<<vgrid(L.npad), 256, 0, s>>>(L.npad, (V*)L.r, (const V*)L.b, (const V*)L.t);
-    AMGT_LAUNCHED();
-    return AMGT_OK;
-}
-template <typename V>
-static amgt_status vec_axpy(amgt_level& L, cudaStream_t s) {
-    TimerScope ts(TC_VEC, 3.0 * L.npad * sizeof(V), s);
-    k_axpy<V><<<vgrid(L.npad), 256, 0, s>>>(L.npad, (V*)L.x, (const V*)L.t);
-    AMGT_LAUNCHED();
-    return AMGT_OK;
-}
-
-static amgt_status jacobi(amgt_level& L, cudaStream_t s, double w) {
-    return L.vprec == AMGT_FP64 ? vec_jacobi<double>(L, s, w) : vec_jacobi<float>(L, s, w);
-}
-static amgt_status residual(amgt_level& L, cudaStream_t s) {
-    return L.vprec == AMGT_FP64 ? vec_residual<double>(L, s) : vec_residual<float>(L, s);
-}
-static amgt_status axpy(amgt_level& L, cudaStream_t s) {
-    return L.vprec == AMGT_FP64 ? vec_axpy<double>(L, s) : vec_axpy<float>(L, s);
-}
 
 template <typename V, typename M>
 static void launch_dinv(amgt_level& L, cudaStream_t s) {
@@ -339,14 +290,16 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
 }
 
 static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const void* x, amgt_prec xp, void* y,
-                                amgt_prec yp, int level) {
+                                amgt_prec yp, int level, int mode = 0, const void* b = nullptr,
+                                const void* dinv = nullptr) {
     ++H->spmv_calls;
-    return spmv_impl(M, x, xp, y, yp, H->s, level == 0 ? TC_SPMV_L1 : TC_SPMV);
+    return spmv_ex_impl(M, x, xp, y, yp, EpiArgs{mode, b, dinv, x, H->o.omega}, H->s,
+                        level == 0 ? TC_SPMV_L1 : TC_SPMV);
 }
 
-static amgt_status norm_into(amgt_hierarchy* H, const double* b, const double* t, int64_t n, double* out) {
-    TimerScope ts(TC_VEC, 2.0 * n * 8, H->s);
-    k_resnorm_partial<<<NORM_BLOCKS, 256, 0, H->s>>>(n, b, t, H->partial);
+static amgt_status norm_into(amgt_hierarchy* H, const double* r, int64_t n, double* out) {
+    TimerScope ts(TC_VEC, 1.0 * n * 8, H->s);
+    k_resnorm_partial<<<NORM_BLOCKS, 256, 0, H->s>>>(n, r, H->partial);
     AMGT_LAUNCHED();
     k_resnorm_final<<<1, 32, 0, H->s>>>(H->partial, out);
     AMGT_LAUNCHED();
@@ -362,8 +315,12 @@ static amgt_status dense_solve(amgt_hierarchy* H, amgt_level& L) {
     return AMGT_OK;
 }
 
+// Alg. 2 with the vector steps fused into the SpMV epilogues: each smoothing sweep is one
+// kernel (out of place, ping-pong between x and t), the residual one kernel, the
+// interpolation + correction one kernel.  SpMV calls are counted exactly as in Alg. 2.
 static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_host,
                           int64_t* calls_host) {
+    constexpr int JAC = 1, RES = 2, ACC = 3;
     cudaStream_t s = H->s;
     Alloc a = H->alloc();
     if (ncycles + 1 > H->norms_cap) {
@@ -374,60 +331,57 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
     }
     const int M = H->nlev - 1;
     amgt_level& L0 = H->L[0];
-    const double w = H->o.omega;
     H->spmv_calls = 0;
-    AMGT_TRY(counted_spmv(H, &L0.A, x, AMGT_FP64, L0.t, AMGT_FP64, 0));
-    AMGT_TRY(norm_into(H, b, (const double*)L0.t, L0.npad, H->norms));
-    for (int c = 1; c <= ncycles; ++c) {
+    void* xc[8];   // buffer currently holding x_k
+    void* xa[8];   // its ping-pong partner
+    xc[0] = x;
+    xa[0] = L0.t;
+    for (int k = 1; k <= M; ++k) { xc[k] = H->L[k].x; xa[k] = H->L[k].t; }
+    AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));
+    AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms));
+    if (M == 0) {
+        for (int c = 1; c <= ncycles; ++c) {
+            amgt_level tmp = L0;
+            tmp.b = (void*)b;
+            tmp.x = xc[0];
+            AMGT_TRY(dense_solve<double>(H, tmp));
+            AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));
+            AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms + c));
+        }
+    }
+    for (int c = 1; c <= ncycles && M > 0; ++c) {
         for (int k = 0; k < M; ++k) {  // Alg. 2 lines 1-5
             amgt_level& L = H->L[k];
-            void* bk = k == 0 ? (void*)b : L.b;
-            void* xk = k == 0 ? (void*)x : L.x;
-            void* sb = L.b;
-            void* sx = L.x;
-            L.b = bk;
-            L.x = xk;
-            if (k > 0) AMGT_CUDA(cudaMemsetAsync(L.x, 0, vbytes(L.vprec) * L.npad, s));
-            for (int i = 0; i < H->o.nu1; ++i) {  // line 2
-                AMGT_TRY(counted_spmv(H, &L.A, L.x, L.vprec, L.t, L.vprec, k));
-                AMGT_TRY(jacobi(L, s, w));
+            const void* bk = k == 0 ? (const void*)b : L.b;
+            if (k > 0) AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, s));
+            for (int i = 0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
+                AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
+                std::swap(xc[k], xa[k]);
             }
-            AMGT_TRY(counted_spmv(H, &L.A, L.x, L.vprec, L.t, L.vprec, k));  // line 3
-            AMGT_TRY(residual(L, s));
+            AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, L.r, L.vprec, k, RES, bk));  // line 3
             amgt_level& N = H->L[k + 1];
-            AMGT_TRY(counted_spmv(H, &L.R, L.r, L.vprec, N.b, N.vprec, k));  // line 4
-            L.b = sb;
-            L.x = sx;
+            AMGT_TRY(counted_spmv(H, &L.R, L.r, L.vprec, N.b, N.vprec, k));  // line 4: restriction
         }
-        {  // line 6
-            amgt_level& C = H->L[M];
-            if (M == 0) {
-                amgt_level tmp = C;
-                tmp.b = (void*)b;
-                tmp.x = x;
-                AMGT_TRY(dense_solve<double>(H, tmp));
-            } else {
-                AMGT_TRY(C.vprec == AMGT_FP64 ? dense_solve<double>(H, C) : dense_solve<float>(H, C));
-            }
+        {  // line 6: coarsest level
+            amgt_level C = H->L[M];
+            C.x = xc[M];
+            AMGT_TRY(C.vprec == AMGT_FP64 ? dense_solve<double>(H, C) : dense_solve<float>(H, C));
         }
         for (int k = M - 1; k >= 0; --k) {  // lines 7-11
             amgt_level& L = H->L[k];
             amgt_level& N = H->L[k + 1];
-            void* sb = L.b;
-            void* sx = L.x;
-            if (k == 0) { L.b = (void*)b; L.x = x; }
-            AMGT_TRY(counted_spmv(H, &L.P, N.x, N.vprec, L.t, L.vprec, k));  // line 8
-            AMGT_TRY(axpy(L, s));                                           // line 9
-            for (int i = 0; i < H->o.nu2; ++i) {                            // line 10
-                AMGT_TRY(counted_spmv(H, &L.A, L.x, L.vprec, L.t, L.vprec, k));
-                AMGT_TRY(jacobi(L, s, w));
+            const void* bk = k == 0 ? (const void*)b : L.b;
+            AMGT_TRY(counted_spmv(H, &L.P, xc[k + 1], N.vprec, xc[k], L.vprec, k, ACC));  // lines 8-9
+            for (int i = 0; i < H->o.nu2; ++i) {  // line 10: post-smoothing
+                AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
+                std::swap(xc[k], xa[k]);
             }
-            L.b = sb;
-            L.x = sx;
         }
-        AMGT_TRY(counted_spmv(H, &L0.A, x, AMGT_FP64, L0.t, AMGT_FP64, 0));  // residual (L308)
-        AMGT_TRY(norm_into(H, b, (const double*)L0.t, L0.npad, H->norms + c));
+        AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));  // residual (L308)
+        AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms + c));
     }
+    if (xc[0] != (void*)x)
+        AMGT_CUDA(cudaMemcpyAsync(x, xc[0], L0.npad * sizeof(double), cudaMemcpyDeviceToDevice, s));
     std::vector<double> hn(ncycles + 1);
     AMGT_CUDA(cudaMemcpyAsync(hn.data(), H->norms, (ncycles + 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
     AMGT_CUDA(cudaStreamSynchronize(s));

@@ -119,3 +119,31 @@ def test_spmv_full_size(cfg):
     x = gen.uniform_vector(A.n, 21).numpy()
     y = amgt.spmv(M, torch.from_numpy(x).cuda()).cpu().numpy()
     check_fp64_entrywise(y[:A.m], oracle.spmv(Ao, x), oracle.spmv_abs(Ao, x))
+
+
+@pytest.mark.parametrize("dt", [torch.float64, torch.float32])
+def test_spmv_fused_epilogues(dt):
+    """amgt_spmv_fused: Jacobi / residual / accumulate epilogues vs oracle SpMV + the
+    Alg. 2 vector formulas (FP64: 1e-12 scaled; FP32 vectors: 1e-5 inf-norm)."""
+    amgt = _amgt()
+    A = gen.laplacian_7pt(20, spd_seed=2)
+    Ao = oracle.as_csr(A)
+    M = amgt.from_csr(A, prec="f64" if dt == torch.float64 else "f32")
+    x = gen.uniform_vector(A.n, 1).numpy()
+    b = gen.uniform_vector(A.n, 2).numpy()
+    y0 = gen.uniform_vector(A.n, 3).numpy()
+    d = 1.0 / Ao.dense().diagonal()
+    w = 2.0 / 3.0
+    Ax = oracle.spmv(Ao, x)
+    scale = oracle.spmv_abs(Ao, x)
+    T = lambda v: torch.from_numpy(np.ascontiguousarray(v)).to(dt).cuda()
+    cases = {"jacobi": x + w * d * (b - Ax), "residual": b - Ax, "accum": y0 + Ax, "y": Ax}
+    for mode, expect in cases.items():
+        y = T(y0) if mode == "accum" else torch.empty(A.m, dtype=dt, device="cuda")
+        amgt.spmv_fused(M, T(x), y, mode, b=T(b), dinv=T(d), omega=w)
+        g = y.double().cpu().numpy()
+        if dt == torch.float64:
+            tol = 1e-12 * (scale * (w * np.abs(d) if mode == "jacobi" else 1.0)) + 1e-15 * (np.abs(expect) + 1)
+            assert np.all(np.abs(g - expect) <= tol), mode
+        else:
+            assert rel_inf(g, expect) <= 1e-5, (mode, rel_inf(g, expect))
