@@ -496,7 +496,8 @@ double spmv_bytes(const amgt_mbsr* A, amgt_prec xp, amgt_prec yp) {
 amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, const EpiArgs& ea,
                          cudaStream_t s, int timer_class) {
     const double vec = 4.0 * A->blc_row * prec_bytes(yp);
-    const double extra = ea.mode == AMGT_EPI_JACOBI ? 3 * vec : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
+    // epilogue operands read once each: Jacobi b, dinv; residual b; accumulate y
+    const double extra = ea.mode == AMGT_EPI_JACOBI ? 2 * vec : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
     TimerScope ts(timer_class, spmv_bytes(A, xp, yp) + extra, s);
     switch (A->prec) {
         case AMGT_FP64: return dispatch_xy<double>(A, x, xp, y, yp, ea, s);

@@ -293,8 +293,9 @@ static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const voi
                                 amgt_prec yp, int level, int mode = 0, const void* b = nullptr,
                                 const void* dinv = nullptr) {
     ++H->spmv_calls;
+    // timer class 0 = the dominant kernel: SpMV with the level-1 operator A_1 (any epilogue)
     return spmv_ex_impl(M, x, xp, y, yp, EpiArgs{mode, b, dinv, x, H->o.omega}, H->s,
-                        level == 0 ? TC_SPMV_L1 : TC_SPMV);
+                        (level == 0 && M == &H->L[0].A) ? TC_SPMV_L1 : TC_SPMV);
 }
 
 static amgt_status norm_into(amgt_hierarchy* H, const double* r, int64_t n, double* out) {
