@@ -840,7 +840,7 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
             }
         }
         bool dense = false;
-        if constexpr (sizeof(T) == 8) dense = mC != 0 && __popc(mA) >= tc_thr;
+        if constexpr (sizeof(T) == 8 || sizeof(T) == 2) dense = mC != 0 && __popc(mA) >= tc_thr;
         if (mC && !dense) {  // CUDA-core route: lane r computes row r of A_t * B_j
             Acc b0[4], b1[4], b2[4], b3[4], v[4];
             const T* bp = bval + 16 * j;
@@ -896,6 +896,76 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
                             acc[k][0] += x0; acc[k][1] += x1; acc[k][2] += x2; acc[k][3] += x3;
                         }
                 }
+            }
+        }
+        if constexpr (sizeof(T) == 2) {
+            // tensor-core route for FP16 (FP32 accumulation): HMMA m16n8k8 with
+            //   A16x8 = rows 0-3 [A0|0], 4-7 [0|A1], 8-11 [A2|0], 12-15 [0|A3]
+            //   B8x8  = [[B0|B2],[B1|B3]]
+            // gives A0B0 (rows 0-3, cols 0-3), A1B1 (4-7, 0-3), A2B2 (8-11, 4-7), A3B3 (12-15, 4-7):
+            // four groups' tile products per instruction.
+            uint32_t dm = __ballot_sync(0xffffffffu, mC != 0 && __popc(mA) >= tc_thr && r == 0);
+            // groups that took this route must skip the CUDA-core update above: handled by
+            // `hdense` below (the CUDA-core block ran only for !hdense groups).
+            while (dm) {
+                int gs[4];
+                int ns = 0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    gs[k] = -1;
+                    if (dm) { gs[k] = (__ffs(dm) - 1) >> 2; dm &= dm - 1; ++ns; }
+                }
+                const int gid = lane >> 2, tid = lane & 3;
+                int64_t ts[4], js[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int src = 4 * (gs[k] < 0 ? gs[0] : gs[k]);
+                    ts[k] = __shfl_sync(0xffffffffu, t, src);
+                    js[k] = __shfl_sync(0xffffffffu, j, src);
+                }
+                const __half* ah = reinterpret_cast<const __half*>(aval);
+                const __half* bh = reinterpret_cast<const __half*>(bval);
+                uint32_t a01 = 0u, a23 = 0u, b01 = 0u;
+                // a0,a1: row gid (slot 0 if gid<4 with tid<2; slot 1 if gid>=4 with tid>=2)
+                const int sA = gid < 4 ? 0 : 1;
+                const bool onA = (gid < 4) == (tid < 2);
+                if (onA && gs[sA] >= 0)
+                    a01 = __ldg(reinterpret_cast<const unsigned int*>(ah + 16 * ts[sA] + 4 * (gid & 3) + 2 * (tid & 1)));
+                const int sA2 = gid < 4 ? 2 : 3;
+                if (onA && gs[sA2] >= 0)
+                    a23 = __ldg(reinterpret_cast<const unsigned int*>(ah + 16 * ts[sA2] + 4 * (gid & 3) + 2 * (tid & 1)));
+                // b0,b1: rows 2tid, 2tid+1 of B8, column gid
+                const int sB = (tid < 2 ? 0 : 1) + (gid < 4 ? 0 : 2);
+                if (gs[sB] >= 0) {
+                    const __half* bp = bh + 16 * js[sB] + 4 * (2 * (tid & 1)) + (gid & 3);
+                    const __half2 bb = __halves2half2(bp[0], bp[4]);
+                    b01 = *reinterpret_cast<const uint32_t*>(&bb);
+                }
+                float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+                asm volatile(
+                    "mma.sync.aligned.m16n8k8.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5}, {%6}, {%0,%1,%2,%3};"
+                    : "+f"(d0), "+f"(d1), "+f"(d2), "+f"(d3)
+                    : "r"(a01), "r"(a23), "r"(b01));
+                // my slot (if my group took part) and the lanes holding row r of its product
+                int slot = -1;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) slot = (gs[k] == g) ? k : slot;
+                const int base = ((slot & 1) ? 16 : 0) + 4 * r + ((slot & 2) ? 2 : 0);
+                const int src = slot < 0 ? lane : base;
+                const float u0 = __shfl_sync(0xffffffffu, d0, src), u1 = __shfl_sync(0xffffffffu, d1, src);
+                const float u2 = __shfl_sync(0xffffffffu, d2, src), u3 = __shfl_sync(0xffffffffu, d3, src);
+                const float w0 = __shfl_sync(0xffffffffu, d0, src + 1), w1 = __shfl_sync(0xffffffffu, d1, src + 1);
+                const float w2 = __shfl_sync(0xffffffffu, d2, src + 1), w3 = __shfl_sync(0xffffffffu, d3, src + 1);
+                if (slot >= 0) {
+                    const bool hi = (slot & 2) != 0;
+                    const float x0 = hi ? u2 : u0, x1 = hi ? u3 : u1, x2 = hi ? w2 : w0, x3 = hi ? w3 : w1;
+#pragma unroll
+                    for (int k = 0; k < GROUP_NC; ++k)
+                        if (k == q) {
+                            acc[k][0] += x0; acc[k][1] += x1; acc[k][2] += x2; acc[k][3] += x3;
+                        }
+                }
+                (void)ns;
             }
         }
         if (has) {  // advance the cursor

@@ -153,3 +153,41 @@ def test_spgemm_cfg4_full():
     M = amgt.from_csr(A)
     C, info = amgt.spgemm(M, M, info=True)
     _check_product(C, Co, Cabs)
+
+
+@pytest.mark.parametrize("thr", [0, 10, 17])
+@pytest.mark.parametrize("prec", ["f16", "f64", "f32"])
+def test_spgemm_tc_routes_integer_exact(prec, thr):
+    """Tensor-core routes (FP64 DMMA m8n8k4, FP16 HMMA m16n8k8 with FP32 accumulation) and the
+    CUDA-core route give the exact product on small-integer data (exact in every precision)."""
+    amgt = _amgt()
+    A = gen.random_csr(96, 88, 0.35, 21, integer=True)
+    B = gen.random_csr(88, 72, 0.35, 22, integer=True)
+    Co = oracle.spgemm(A, B)
+    assert np.abs(Co.val).max() < 2048
+    amgt.set_tc_threshold(thr, 17)
+    try:
+        C, info = amgt.spgemm(amgt.from_csr(A, prec=prec), amgt.from_csr(B, prec=prec), info=True)
+    finally:
+        amgt.set_tc_threshold(10, 17)
+    if thr == 0:
+        assert info["pairs_tc"] == info["pairs_nonzero"]
+    assert_structure_equal(C, oracle.csr_to_mbsr(Co))
+    _, _, v = tile_values_to_csr_order(C)
+    assert np.array_equal(v, Co.val)
+
+
+@pytest.mark.parametrize("thr", [0, 17])
+def test_spgemm_fp16_tc_tolerance(thr):
+    amgt = _amgt()
+    A = gen.random_csr(128, 128, 0.6, 23)
+    Ao = oracle.as_csr(A)
+    Co = oracle.spgemm(Ao, Ao)
+    amgt.set_tc_threshold(thr, 17)
+    try:
+        M = amgt.from_csr(A, prec="f16")
+        C = amgt.spgemm(M, M)
+    finally:
+        amgt.set_tc_threshold(10, 17)
+    _, _, v = tile_values_to_csr_order(C)
+    assert rel_2(v, Co.val) <= 5e-3
