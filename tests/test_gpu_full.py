@@ -36,7 +36,11 @@ def test_cfg3_full():
         Ak, _, _ = H.level(k)
         assert_structure_equal(Ak, oracle.csr_to_mbsr(As[k]))
         _, _, v = Ak.to_csr()
-        assert np.array_equal(v.cpu().numpy(), As[k].val)  # alpha = 1/2: values fit every precision exactly
+        v = v.cpu().numpy()
+        if k == 1:  # produced by the FP64 RAP of level 1, stored FP32: dyadic values, exact
+            assert np.array_equal(v, As[k].val)
+        else:       # FP32 / FP16 RAP chain, FP16 storage: the FP16 tolerance of north_star
+            assert np.linalg.norm(v - As[k].val) <= 5e-3 * np.linalg.norm(As[k].val)
     b = gen.uniform_vector(A.m, cfg.seed)
     x = torch.zeros(A.m, dtype=torch.float64, device="cuda")
     ncyc = 10

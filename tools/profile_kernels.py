@@ -1,6 +1,6 @@
-"""Run the hot kernels on config 2 a few times (for ncu captures; not a benchmark).
+"""Run the hot kernels on a config a few times (for ncu captures; not a benchmark).
 
-usage: python tools/profile_kernels.py [spmv|spgemm|convert|all] [reps]
+usage: python tools/profile_kernels.py [spmv|spgemm|all] [reps] [N] [7pt|27pt]
 """
 import os
 import sys
@@ -14,8 +14,9 @@ import paper_conf_sc_luzwflcy0c024_b200 as amgt  # noqa: E402
 
 what = sys.argv[1] if len(sys.argv) > 1 else "all"
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
-N = 128
-A = gen.laplacian_7pt(N, device="cuda")
+N = int(sys.argv[3]) if len(sys.argv) > 3 else 128
+kind = sys.argv[4] if len(sys.argv) > 4 else "7pt"
+A = (gen.laplacian_7pt if kind == "7pt" else gen.laplacian_27pt)(N, device="cuda")
 P = gen.aggregation_P((N, N, N), 0.5, device="cuda")
 R = gen.aggregation_R((N, N, N), 0.5, device="cuda")
 for _ in range(reps):
