@@ -110,6 +110,21 @@ __device__ __forceinline__ uint32_t bitmap_multiply(uint32_t a, uint32_t b) {
            (((a >> 2) & 0x1111u) * ((b >> 8) & 0xFu)) | (((a >> 3) & 0x1111u) * ((b >> 12) & 0xFu));
 }
 
+// A 4-lane group (lanes gbase..gbase+3, mask gm) holds the four rows of an FP64 4x4 tile,
+// lane r owning row r.  Store the 128-B tile with two instructions that each write 64
+// contiguous bytes (full 32-B sectors: no partial-sector read-for-write in L2): lane q
+// writes elements {2q, 2q+1} (row q>>1) and {8+2q, 9+2q} (row 2+(q>>1)).
+__device__ __forceinline__ void group_store_tile_f64(double* tile, const double (&v)[4], int q, unsigned gm,
+                                                     int gbase) {
+    const int s1 = gbase + (q >> 1), s2 = gbase + 2 + (q >> 1);
+    const double a0 = __shfl_sync(gm, v[0], s1), a1 = __shfl_sync(gm, v[1], s1);
+    const double a2 = __shfl_sync(gm, v[2], s1), a3 = __shfl_sync(gm, v[3], s1);
+    const double b0 = __shfl_sync(gm, v[0], s2), b1 = __shfl_sync(gm, v[1], s2);
+    const double b2 = __shfl_sync(gm, v[2], s2), b3 = __shfl_sync(gm, v[3], s2);
+    reinterpret_cast<double2*>(tile)[q] = (q & 1) ? make_double2(a2, a3) : make_double2(a0, a1);
+    reinterpret_cast<double2*>(tile)[4 + q] = (q & 1) ? make_double2(b2, b3) : make_double2(b0, b1);
+}
+
 // ------------------------------------------------------------------ device flags
 // Bits of the per-call device error word.
 enum : uint32_t { FLAG_FORMAT = 1u, FLAG_RANGE = 2u };

@@ -95,7 +95,10 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
         mp |= __shfl_xor_sync(0xffffffffu, mp, 2);
         if (Jm != INT_MAX) {
             if (FILL) {
-                store_row(bval + 16 * t + 4 * r, rv);
+                if constexpr (sizeof(T) == 8)
+                    group_store_tile_f64((double*)(bval + 16 * t), rv, r, 0xFu << (lane & ~3), lane & ~3);
+                else
+                    store_row(bval + 16 * t + 4 * r, rv);
                 if (r == 0) {
                     bidx[t] = Jm;
                     bmap[t] = (uint16_t)mp;

@@ -983,9 +983,10 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
             Acc o[4];
 #pragma unroll
             for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? acc[k][e] : Acc(0);
-            T* dst = cval + 16 * (c0 + k) + 4 * r;
-            if constexpr (sizeof(T) == 2) RowIO<T>::store(dst, o);
-            else RowIO<T>::store(dst, o);
+            if constexpr (sizeof(T) == 8)
+                group_store_tile_f64((double*)(cval + 16 * (c0 + k)), o, r, 0xFu << (lane & ~3), lane & ~3);
+            else
+                RowIO<T>::store(cval + 16 * (c0 + k) + 4 * r, o);
         }
     }
 }
