@@ -91,6 +91,30 @@ struct Epi {
     const XT* xs;
     YT omega;
     int mode;
+    // operands of row i, loaded before the tile loop so their latency overlaps it
+    struct Pre {
+        YT a = YT(0), c = YT(0), d = YT(0);
+    };
+    __device__ __forceinline__ Pre prefetch(int64_t i) const {
+        Pre p;
+        switch (mode) {
+            case AMGT_EPI_JACOBI: p.a = b[i]; p.c = dinv[i]; p.d = (YT)xs[i]; break;
+            case AMGT_EPI_RESIDUAL: p.a = b[i]; break;
+            case AMGT_EPI_ACCUM: p.a = y[i]; break;
+            default: break;
+        }
+        return p;
+    }
+    template <typename V>
+    __device__ __forceinline__ void finish(int64_t i, V v, const Pre& p) const {
+        const YT t = (YT)v;
+        switch (mode) {
+            case AMGT_EPI_JACOBI: y[i] = p.d + omega * p.c * (p.a - t); break;
+            case AMGT_EPI_RESIDUAL: y[i] = p.a - t; break;
+            case AMGT_EPI_ACCUM: y[i] = p.a + t; break;
+            default: y[i] = t;
+        }
+    }
     __device__ __forceinline__ void apply(int64_t i, double v) const { put(i, (YT)v); }
     __device__ __forceinline__ void apply(int64_t i, float v) const { put(i, (YT)v); }
     __device__ __forceinline__ void put(int64_t i, YT t) const {
@@ -148,6 +172,10 @@ __global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __
         write = t1 - t0 <= long_thr;
         if (!write) t1 = t0;  // long row: handled by the chunk kernel
     }
+    // output element of this lane (FP64 layout: rows {0,2,1,3} for q = 0..3)
+    const int64_t out_i = 4 * I + (sizeof(MatT) == 8 ? ((q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3) : q);
+    typename Epi<XT, YT>::Pre pre;
+    if (write) pre = epi.prefetch(out_i);
     if constexpr (sizeof(MatT) == 8) {
         F64Lane L;
         const bool use_tc = tc_thr <= 16;
@@ -225,13 +253,13 @@ __global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __
             const double tcmine = __shfl_sync(0xffffffffu, tcacc, 4 * g + myrow);
             const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
             const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
-            if (write) epi.apply(4 * I + myrow, ((q & 1) ? s1 : s0) + tcmine);
+            if (write) epi.finish(out_i, ((q & 1) ? s1 : s0) + tcmine, pre);
             return;
         }
         const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
         const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
         const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
-        if (write) epi.apply(4 * I + myrow, (q & 1) ? s1 : s0);
+        if (write) epi.finish(out_i, (q & 1) ? s1 : s0, pre);
     } else {
         float acc = 0.f;
         for (int64_t t = t0; t < t1; ++t) {
@@ -253,7 +281,7 @@ __global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __
             acc = (nib & 4u) ? fmaf(a2, xv.z, acc) : acc;
             acc = (nib & 8u) ? fmaf(a3, xv.w, acc) : acc;
         }
-        if (write) epi.apply(4 * I + q, acc);
+        if (write) epi.finish(out_i, acc, pre);
     }
 }
 
