@@ -24,4 +24,4 @@ from .aggregation import aggregation_P, aggregation_R, aggregation_hierarchy  # 
 from .irregular import irregular_block_sparse  # noqa: F401
 from .vectors import uniform_vector, integer_vector  # noqa: F401
 from .random_csr import random_csr  # noqa: F401
-from . import configs  # noqa: F401
+from . import configs, partition  # noqa: F401

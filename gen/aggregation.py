@@ -32,7 +32,8 @@ def default_alpha(dims) -> float:
     return 0.5 if len(dims) == 3 else 1.0
 
 
-def aggregation_P(dims, alpha: float | None = None, device="cpu") -> CSR:
+def aggregation_P(dims, alpha: float | None = None, device="cpu", rows=None) -> CSR:
+    """rows=(r0, r1): only fine rows r0..r1-1 (global coarse column indices)."""
     dims = tuple(int(d) for d in dims)
     if alpha is None:
         alpha = default_alpha(dims)
@@ -43,14 +44,16 @@ def aggregation_P(dims, alpha: float | None = None, device="cpu") -> CSR:
     nc = 1
     for d in cd:
         nc *= d
-    idx = torch.arange(n, dtype=torch.int64, device=device)
+    r0, r1 = (0, n) if rows is None else (int(rows[0]), int(rows[1]))
+    idx = torch.arange(r0, r1, dtype=torch.int64, device=device)
     coords, rem = [], idx
     for d in dims:
         coords.append(rem % d)
         rem = rem // d
     ccol = _lin([c // 2 for c in coords], cd)
-    row_ptr = torch.arange(n + 1, dtype=torch.int64, device=device)
-    return CSR(n, nc, row_ptr, ccol.to(torch.int32), torch.full((n,), float(alpha), dtype=torch.float64, device=device))
+    m = r1 - r0
+    row_ptr = torch.arange(m + 1, dtype=torch.int64, device=device)
+    return CSR(m, nc, row_ptr, ccol.to(torch.int32), torch.full((m,), float(alpha), dtype=torch.float64, device=device))
 
 
 def aggregation_R(dims, alpha: float | None = None, device="cpu") -> CSR:

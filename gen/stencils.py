@@ -44,8 +44,10 @@ def pair_uniform(i: torch.Tensor, j: torch.Tensor, seed: int) -> torch.Tensor:
     return _lsr(h, 11).to(torch.float64) * (2.0 ** -53)
 
 
-def stencil(dims, offsets, center: float, off: float, device="cpu", spd_seed: int | None = None) -> CSR:
-    """Generic constant-coefficient stencil matrix on a grid of `dims` (x fastest)."""
+def stencil(dims, offsets, center: float, off: float, device="cpu", spd_seed: int | None = None,
+            rows=None) -> CSR:
+    """Generic constant-coefficient stencil matrix on a grid of `dims` (x fastest).
+    rows=(r0, r1): generate only rows r0..r1-1 (global column indices kept)."""
     dims = tuple(int(d) for d in dims)
     nd = len(dims)
     strides = [1]
@@ -56,23 +58,25 @@ def stencil(dims, offsets, center: float, off: float, device="cpu", spd_seed: in
         n *= d
     # sort offsets by linear offset -> ascending column order within a row
     offs = sorted(offsets, key=lambda o: sum(o[k] * strides[k] for k in range(nd)))
-    idx = torch.arange(n, dtype=torch.int64, device=device)
+    r0, r1 = (0, n) if rows is None else (int(rows[0]), int(rows[1]))
+    idx = torch.arange(r0, r1, dtype=torch.int64, device=device)
+    m = r1 - r0
     coords = []
     rem = idx
     for k in range(nd):
         coords.append(rem % dims[k])
         rem = rem // dims[k]
     valids = []
-    count = torch.zeros(n, dtype=torch.int64, device=device)
+    count = torch.zeros(m, dtype=torch.int64, device=device)
     for o in offs:
-        v = torch.ones(n, dtype=torch.bool, device=device)
+        v = torch.ones(m, dtype=torch.bool, device=device)
         for k in range(nd):
             if o[k] != 0:
                 c = coords[k] + o[k]
                 v &= (c >= 0) & (c < dims[k])
         valids.append(v)
         count += v
-    row_ptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    row_ptr = torch.zeros(m + 1, dtype=torch.int64, device=device)
     row_ptr[1:] = torch.cumsum(count, 0)
     nnz = int(row_ptr[-1])
     col = torch.empty(nnz, dtype=torch.int32, device=device)
@@ -97,21 +101,24 @@ def stencil(dims, offsets, center: float, off: float, device="cpu", spd_seed: in
         rows_all = torch.repeat_interleave(idx, count)
         is_diag = col.long() == rows_all
         absoff = torch.where(is_diag, torch.zeros_like(val), val.abs())
-        rowsum = torch.zeros(n, dtype=torch.float64, device=device).index_add_(0, rows_all, absoff)
+        rowsum = torch.zeros(m, dtype=torch.float64, device=device).index_add_(0, rows_all - r0, absoff)
         val[is_diag] = rowsum + 1.0
-    return CSR(n, n, row_ptr, col, val)
+    return CSR(m, n, row_ptr, col, val)
 
 
-def laplacian_5pt(N: int, device="cpu", spd_seed=None) -> CSR:
-    offs = [(0, 0), (1, 0), (-1, 0), (0, 1), (0, -1)]
-    return stencil((N, N), offs, 4.0, -1.0, device, spd_seed)
+OFFS_5PT = [(0, 0), (1, 0), (-1, 0), (0, 1), (0, -1)]
+OFFS_7PT = [(0, 0, 0), (1, 0, 0), (-1, 0, 0), (0, 1, 0), (0, -1, 0), (0, 0, 1), (0, 0, -1)]
+OFFS_27PT = list(itertools.product((-1, 0, 1), repeat=3))
 
 
-def laplacian_7pt(N: int, device="cpu", spd_seed=None) -> CSR:
-    offs = [(0, 0, 0), (1, 0, 0), (-1, 0, 0), (0, 1, 0), (0, -1, 0), (0, 0, 1), (0, 0, -1)]
-    return stencil((N, N, N), offs, 6.0, -1.0, device, spd_seed)
+def laplacian_5pt(N: int, device="cpu", spd_seed=None, rows=None) -> CSR:
+    return stencil((N, N), OFFS_5PT, 4.0, -1.0, device, spd_seed, rows)
 
 
-def laplacian_27pt(N: int, device="cpu", spd_seed=None) -> CSR:
-    offs = list(itertools.product((-1, 0, 1), repeat=3))
-    return stencil((N, N, N), offs, 26.0, -1.0, device, spd_seed)
+def laplacian_7pt(N: int, device="cpu", spd_seed=None, rows=None, dims=None) -> CSR:
+    """7-point Laplacian on N^3 (or on `dims` = (Nx, Ny, Nz))."""
+    return stencil(dims or (N, N, N), OFFS_7PT, 6.0, -1.0, device, spd_seed, rows)
+
+
+def laplacian_27pt(N: int, device="cpu", spd_seed=None, rows=None, dims=None) -> CSR:
+    return stencil(dims or (N, N, N), OFFS_27PT, 26.0, -1.0, device, spd_seed, rows)

@@ -224,6 +224,38 @@ amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* 
 amgt_status amgt_spmv_fused(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec, int mode,
                             const void* b, const void* dinv, double omega, void* stream);
 
+/* Row-range variant used by the distributed SpMV to overlap the halo exchange: only
+ * block rows [blk_begin, blk_end) are computed; y indexed by local row; for Jacobi, x_i is
+ * read from xs (the own segment of x when x is an extended [halo|own|halo] buffer).
+ * Not available for matrices whose SpMV plan splits long rows (AMGT_ERR_UNSUPPORTED). */
+amgt_status amgt_spmv_fused_range(const amgt_mbsr* A, int64_t blk_begin, int64_t blk_end, const void* x,
+                                  amgt_prec xprec, void* y, amgt_prec yprec, int mode, const void* b, const void* dinv,
+                                  const void* xs, double omega, void* stream);
+
+/* ------------------------------------------------ distributed-path helpers (§8(e)) */
+
+/* CSR -> mBSR with column offset: column c becomes c - col_offset, which must lie in
+ * [0, n) (a rank's rows with global columns, remapped to its extended range). */
+amgt_status amgt_csr_to_mbsr_ex(int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr, const int32_t* col_idx,
+                                const double* val, int64_t col_offset, amgt_prec prec, amgt_mbsr* out,
+                                const amgt_allocator* al, void* stream);
+/* In place: blc_idx += delta_tiles; A->n = new_n (remap global -> extended-local columns). */
+amgt_status amgt_mbsr_shift_cols(amgt_mbsr* A, int64_t delta_tiles, int64_t new_n, void* stream);
+/* out3_host = {min column, max column, max |column - (row + row_offset)|} (syncs).  CSR: scalar
+ * units; mBSR: tile units with block-row offset. */
+amgt_status amgt_csr_col_range(int64_t m, const int64_t* row_ptr, const int32_t* col_idx, int64_t row_offset,
+                               int64_t* out3_host, void* stream);
+amgt_status amgt_mbsr_col_range(const amgt_mbsr* A, int64_t blk_row_offset, int64_t* out3_host, void* stream);
+/* dinv[i] = 1 / A(i, i) with the diagonal tile of block row I at column I + diag_tile_offset. */
+amgt_status amgt_dinv(const amgt_mbsr* A, int64_t diag_tile_offset, void* dinv, amgt_prec vprec, void* stream);
+/* Host: inverse of an SPD n x n row-major matrix via Cholesky (coarsest level, R22). */
+amgt_status amgt_dense_spd_inverse(int64_t n, const double* a_host, double* inv_host);
+/* x[0:npad] = Ainv (n x n, FP64, device) * b[0:n], zero-padded to npad. */
+amgt_status amgt_dense_matvec(int64_t n, int64_t npad, const double* Ainv, const void* b, void* x, amgt_prec vprec,
+                              void* stream);
+/* *out_dev = sum r_i^2 (deterministic two-pass reduction, FP64). */
+amgt_status amgt_norm2sq(int64_t n, const double* r, double* out_dev, void* stream);
+
 /* ------------------------------------------------------ hierarchy + V-cycle (§II) */
 
 typedef struct {

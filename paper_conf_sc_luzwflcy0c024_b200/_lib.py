@@ -100,6 +100,16 @@ _sigs = {
     "amgt_timing_reset": (_int, []),
     "amgt_timing_read": (_int, [_P(ctypes.c_double), _P(_i64), _P(ctypes.c_double)]),
     "amgt_launch_count": (_i64, []),
+    "amgt_spmv_fused_range": (_int, [_P(c_mbsr), _i64, _i64, _vp, _int, _vp, _int, _int, _vp, _vp, _vp, ctypes.c_double,
+                                     _vp]),
+    "amgt_csr_to_mbsr_ex": (_int, [_i64, _i64, _i64, _vp, _vp, _vp, _i64, _int, _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_mbsr_shift_cols": (_int, [_P(c_mbsr), _i64, _i64, _vp]),
+    "amgt_csr_col_range": (_int, [_i64, _vp, _vp, _i64, _P(_i64), _vp]),
+    "amgt_mbsr_col_range": (_int, [_P(c_mbsr), _i64, _P(_i64), _vp]),
+    "amgt_dinv": (_int, [_P(c_mbsr), _i64, _vp, _int, _vp]),
+    "amgt_dense_spd_inverse": (_int, [_i64, _vp, _vp]),
+    "amgt_dense_matvec": (_int, [_i64, _i64, _vp, _vp, _vp, _int, _vp]),
+    "amgt_norm2sq": (_int, [_i64, _vp, _vp, _vp]),
 }
 for _name, (_res, _args) in _sigs.items():
     _f = getattr(_L, _name)
@@ -326,6 +336,72 @@ def spmv_fused(A: Mbsr, x: torch.Tensor, y: torch.Tensor, mode: str, b: torch.Te
                               b.data_ptr() if b is not None else None, dinv.data_ptr() if dinv is not None else None,
                               float(omega), _stream(stream)))
     return y
+
+
+def spmv_range(A: Mbsr, blk_begin: int, blk_end: int, x: torch.Tensor, y: torch.Tensor, mode: str = "y",
+               b: torch.Tensor | None = None, dinv: torch.Tensor | None = None, xs: torch.Tensor | None = None,
+               omega: float = 2.0 / 3.0, stream=None) -> torch.Tensor:
+    """amgt_spmv_fused_range: block rows [blk_begin, blk_end) only."""
+    xp = {torch.float64: FP64, torch.float32: FP32}[x.dtype]
+    yp = {torch.float64: FP64, torch.float32: FP32}[y.dtype]
+    ptr = lambda t: t.data_ptr() if t is not None else None
+    _check(_L.amgt_spmv_fused_range(ctypes.byref(A.c), int(blk_begin), int(blk_end), x.data_ptr(), xp, y.data_ptr(), yp,
+                                    EPI[mode], ptr(b), ptr(dinv), ptr(xs), float(omega), _stream(stream)))
+    return y
+
+
+def csr_to_mbsr_ex(m, n, row_ptr, col, val, col_offset: int, prec="f64", stream=None) -> Mbsr:
+    out = Mbsr()
+    _check(_L.amgt_csr_to_mbsr_ex(int(m), int(n), int(col.numel()), row_ptr.data_ptr(), col.data_ptr(), val.data_ptr(),
+                                  int(col_offset), PREC[prec], ctypes.byref(out.c), _AL, _stream(stream)))
+    return out
+
+
+def shift_cols(A: Mbsr, delta_tiles: int, new_n: int, stream=None) -> Mbsr:
+    _check(_L.amgt_mbsr_shift_cols(ctypes.byref(A.c), int(delta_tiles), int(new_n), _stream(stream)))
+    return A
+
+
+def csr_col_range(m, row_ptr, col, row_offset: int, stream=None):
+    out = (ctypes.c_int64 * 3)()
+    _check(_L.amgt_csr_col_range(int(m), row_ptr.data_ptr(), col.data_ptr() if col.numel() else None, int(row_offset),
+                                 out, _stream(stream)))
+    return tuple(out)
+
+
+def mbsr_col_range(A: Mbsr, blk_row_offset: int, stream=None):
+    out = (ctypes.c_int64 * 3)()
+    _check(_L.amgt_mbsr_col_range(ctypes.byref(A.c), int(blk_row_offset), out, _stream(stream)))
+    return tuple(out)
+
+
+def dinv(A: Mbsr, diag_tile_offset: int, dtype=torch.float64, stream=None) -> torch.Tensor:
+    d = torch.zeros(4 * A.blc_row, dtype=dtype, device="cuda")
+    _check(_L.amgt_dinv(ctypes.byref(A.c), int(diag_tile_offset), d.data_ptr(), {torch.float64: FP64, torch.float32: FP32}[dtype],
+                        _stream(stream)))
+    return d
+
+
+def dense_spd_inverse(a):
+    """Host Cholesky-based inverse (numpy float64 n x n -> numpy)."""
+    import numpy as np
+    a = np.ascontiguousarray(a, dtype=np.float64)
+    inv = np.empty_like(a)
+    _check(_L.amgt_dense_spd_inverse(a.shape[0], a.ctypes.data, inv.ctypes.data))
+    return inv
+
+
+def dense_matvec(n: int, Ainv: torch.Tensor, b: torch.Tensor, x: torch.Tensor, stream=None) -> torch.Tensor:
+    _check(_L.amgt_dense_matvec(int(n), int(x.numel()), Ainv.data_ptr(), b.data_ptr(), x.data_ptr(),
+                                {torch.float64: FP64, torch.float32: FP32}[x.dtype], _stream(stream)))
+    return x
+
+
+def norm2sq(r: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    if out is None:
+        out = torch.empty(1, dtype=torch.float64, device="cuda")
+    _check(_L.amgt_norm2sq(int(r.numel()), r.data_ptr(), out.data_ptr(), _stream(stream)))
+    return out
 
 
 def wrap(m, n, blc_ptr, blc_idx, blc_map, blc_val, prec) -> Mbsr:

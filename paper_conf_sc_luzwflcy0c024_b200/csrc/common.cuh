@@ -161,6 +161,7 @@ struct EpiArgs {
     const void* dinv;
     const void* xs;
     double omega;
+    int64_t I0, I1;  // block-row range [I0, I1); I1 < 0 = all rows
 };
 
 extern int g_tc_thr_spgemm;

@@ -38,7 +38,7 @@ template <> __device__ __forceinline__ bool overflows<__half>(double v) {
 // FILL = false: count tiles per block row into cnt[I] and validate the CSR.
 // FILL = true : write blc_idx / blc_map / blc_val at offsets bptr[I].
 template <bool FILL, typename T>
-__global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t nnz, int64_t BR,
+__global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t nnz, int64_t BR, int64_t coff,
                                                   const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
                                                   const double* __restrict__ v, int64_t* __restrict__ cnt,
                                                   const int64_t* __restrict__ bptr, int32_t* __restrict__ bidx,
@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
     int64_t c = 0;
     int32_t prev = -1;
     for (;;) {
-        const int32_t J = (p < e) ? (__ldg(ci + p) >> 2) : INT_MAX;
+        const int32_t J = (p < e) ? (int32_t)((__ldg(ci + p) - coff) >> 2) : INT_MAX;
         int32_t Jm = min(J, __shfl_xor_sync(0xffffffffu, J, 1));
         Jm = min(Jm, __shfl_xor_sync(0xffffffffu, Jm, 2));
         if (!__any_sync(0xffffffffu, Jm != INT_MAX)) break;
@@ -72,10 +72,10 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
         uint32_t nib = 0;
         if (Jm != INT_MAX) {
             while (p < e) {
-                const int32_t col = __ldg(ci + p);
+                const int32_t col = (int32_t)(__ldg(ci + p) - coff);
                 if ((col >> 2) != Jm) break;
                 if (!FILL) {
-                    if (col <= prev || col >= n) bad = 1;
+                    if (col <= prev || col >= n || col < 0) bad = 1;
                     prev = col;
                 } else {
                     const int cc = col & 3;
@@ -292,7 +292,7 @@ static amgt_status read_flag(uint32_t* dflag, cudaStream_t s, uint32_t* out) {
 }
 
 amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* rp, const int32_t* ci,
-                             const double* v, amgt_prec prec, amgt_mbsr* out, Alloc& a) {
+                             const double* v, amgt_prec prec, amgt_mbsr* out, Alloc& a, int64_t coff) {
     cudaStream_t s = a.s;
     const int64_t BR = ceil_div(m, 4);
     Scratch<int64_t> cnt;
@@ -306,7 +306,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     {
         TimerScope ts(TC_CSR2MBSR, bytes_in, s);
         if (BR > 0) {
-            k_csr2mbsr<false, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, cnt.p, nullptr, nullptr,
+            k_csr2mbsr<false, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, cnt.p, nullptr, nullptr,
                                                              nullptr, nullptr, flag.p);
             AMGT_LAUNCHED();
         }
@@ -333,15 +333,15 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
         if (BR > 0) {
             switch (prec) {
                 case AMGT_FP64:
-                    k_csr2mbsr<true, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, nullptr, M.blc_ptr,
+                    k_csr2mbsr<true, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                     M.blc_idx, M.blc_map, (double*)M.blc_val, flag.p);
                     break;
                 case AMGT_FP32:
-                    k_csr2mbsr<true, float><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, nullptr, M.blc_ptr,
+                    k_csr2mbsr<true, float><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                    M.blc_idx, M.blc_map, (float*)M.blc_val, flag.p);
                     break;
                 default:
-                    k_csr2mbsr<true, __half><<<blocks, 256, 0, s>>>(m, n, nnz, BR, rp, ci, v, nullptr, M.blc_ptr,
+                    k_csr2mbsr<true, __half><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                     M.blc_idx, M.blc_map, (__half*)M.blc_val, flag.p);
             }
             AMGT_LAUNCHED();
@@ -473,6 +473,57 @@ amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a) {
     return AMGT_OK;
 }
 
+// ---- distributed-path helpers: tile-column shift and column-range statistics
+__global__ void k_shift_cols(int64_t T, int32_t* __restrict__ idx, int64_t delta) {
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < T; t += (int64_t)gridDim.x * blockDim.x)
+        idx[t] = (int32_t)(idx[t] + delta);
+}
+
+// out[0] = min column, out[1] = max column, out[2] = max |col - (row + row_offset)|;
+// TILES: over mBSR tiles (tile units), else over CSR entries (scalar units).
+template <bool TILES>
+__global__ void k_col_range(int64_t rows, const int64_t* __restrict__ ptr, const int32_t* __restrict__ idx,
+                            int64_t row_offset, unsigned long long* __restrict__ out) {
+    long long mn = LLONG_MAX, mx = LLONG_MIN, bw = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < rows; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t a = ptr[i], b = ptr[i + 1];
+        if (a == b) continue;
+        const long long lo = idx[a], hi = idx[b - 1], g = i + row_offset;
+        mn = min(mn, lo);
+        mx = max(mx, hi);
+        bw = max(bw, max(g - lo, hi - g));
+    }
+    for (int d = 16; d; d >>= 1) {
+        mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, d));
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, d));
+        bw = max(bw, __shfl_xor_sync(0xffffffffu, bw, d));
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicMin(reinterpret_cast<long long*>(out), mn);
+        atomicMax(reinterpret_cast<long long*>(out) + 1, mx);
+        atomicMax(reinterpret_cast<long long*>(out) + 2, bw);
+    }
+}
+
+static amgt_status col_range(bool tiles, int64_t rows, const int64_t* ptr, const int32_t* idx, int64_t row_offset,
+                             int64_t* out_host, cudaStream_t s) {
+    Alloc a{nullptr, s};
+    Scratch<unsigned long long> d;
+    AMGT_TRY(d.init(a, 3));
+    const long long init[3] = {LLONG_MAX, LLONG_MIN, 0};
+    AMGT_CUDA(cudaMemcpyAsync(d.p, init, sizeof(init), cudaMemcpyHostToDevice, s));
+    if (rows > 0) {
+        if (tiles) k_col_range<true><<<grid_for(rows, 256), 256, 0, s>>>(rows, ptr, idx, row_offset, d.p);
+        else k_col_range<false><<<grid_for(rows, 256), 256, 0, s>>>(rows, ptr, idx, row_offset, d.p);
+        AMGT_LAUNCHED();
+    }
+    long long h[3];
+    AMGT_CUDA(cudaMemcpyAsync(h, d.p, sizeof(h), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    for (int k = 0; k < 3; ++k) out_host[k] = h[k];
+    return AMGT_OK;
+}
+
 }  // namespace amgt
 
 using namespace amgt;
@@ -487,7 +538,18 @@ amgt_status amgt_csr_to_mbsr(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     if (nnz > 0 && (!col_idx || !val)) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: col/val NULL");
     if (ceil_div(n, 4) > INT32_MAX) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: too many columns for int32 tile indices");
     Alloc a{al, (cudaStream_t)stream};
-    return csr_to_mbsr_impl(m, n, nnz, row_ptr, col_idx, val, prec, out, a);
+    return csr_to_mbsr_impl(m, n, nnz, row_ptr, col_idx, val, prec, out, a, 0);
+}
+
+amgt_status amgt_csr_to_mbsr_ex(int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr, const int32_t* col_idx,
+                                const double* val, int64_t col_offset, amgt_prec prec, amgt_mbsr* out,
+                                const amgt_allocator* al, void* stream) {
+    if (!out || m < 0 || n < 0 || nnz < 0 || !prec_valid(prec) || col_offset < 0)
+        return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr_ex: bad argument");
+    if (m > 0 && !row_ptr) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr_ex: row_ptr is NULL");
+    if (nnz > 0 && (!col_idx || !val)) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr_ex: col/val NULL");
+    Alloc a{al, (cudaStream_t)stream};
+    return csr_to_mbsr_impl(m, n, nnz, row_ptr, col_idx, val, prec, out, a, col_offset);
 }
 
 amgt_status amgt_mbsr_nnz(const amgt_mbsr* A, int64_t* nnz_host, void* stream) {
@@ -529,6 +591,29 @@ amgt_status amgt_mbsr_transpose(const amgt_mbsr* in, amgt_mbsr* out, const amgt_
     if (!in || !out) return fail(AMGT_ERR_ARG, "amgt_mbsr_transpose: NULL argument");
     Alloc a{al, (cudaStream_t)stream};
     return transpose_impl(in, out, a);
+}
+
+amgt_status amgt_mbsr_shift_cols(amgt_mbsr* A, int64_t delta_tiles, int64_t new_n, void* stream) {
+    if (!A || new_n < 0) return fail(AMGT_ERR_ARG, "amgt_mbsr_shift_cols: bad argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (A->blc_num > 0 && delta_tiles != 0) {
+        k_shift_cols<<<grid_for(A->blc_num, 256), 256, 0, s>>>(A->blc_num, A->blc_idx, delta_tiles);
+        AMGT_LAUNCHED();
+    }
+    A->n = new_n;
+    A->blc_col = ceil_div(new_n, 4);
+    return AMGT_OK;
+}
+
+amgt_status amgt_csr_col_range(int64_t m, const int64_t* row_ptr, const int32_t* col_idx, int64_t row_offset,
+                               int64_t* out3_host, void* stream) {
+    if (!out3_host || m < 0) return fail(AMGT_ERR_ARG, "amgt_csr_col_range: bad argument");
+    return col_range(false, m, row_ptr, col_idx, row_offset, out3_host, (cudaStream_t)stream);
+}
+
+amgt_status amgt_mbsr_col_range(const amgt_mbsr* A, int64_t blk_row_offset, int64_t* out3_host, void* stream) {
+    if (!A || !out3_host) return fail(AMGT_ERR_ARG, "amgt_mbsr_col_range: bad argument");
+    return col_range(true, A->blc_row, A->blc_ptr, A->blc_idx, blk_row_offset, out3_host, (cudaStream_t)stream);
 }
 
 amgt_status amgt_mbsr_wrap(int64_t m, int64_t n, int64_t blc_num, int64_t* blc_ptr, int32_t* blc_idx,

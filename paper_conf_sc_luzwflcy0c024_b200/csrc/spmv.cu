@@ -155,15 +155,15 @@ __device__ __forceinline__ void dmma_884(double& c0, double& c1, double a, doubl
 // ---------------------------------------------------------------- row kernel
 // MatT = double / float / __half; XT, YT = double / float.
 template <typename MatT, typename XT, typename YT>
-__global__ void __launch_bounds__(256) k_spmv_rows(int64_t BR, const int64_t* __restrict__ bptr,
+__global__ void __launch_bounds__(256) k_spmv_rows(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
                                                    const int32_t* __restrict__ bidx,
                                                    const uint16_t* __restrict__ bmap, const MatT* __restrict__ bval,
                                                    const XT* __restrict__ x, const Epi<XT, YT> epi,
                                                    int64_t long_thr, int tc_thr) {
     const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t I = wid * 8 + g;
-    if (wid * 8 >= BR) return;
+    const int64_t I = I0 + wid * 8 + g;  // block rows [I0, BR)
+    if (I0 + wid * 8 >= BR) return;
     int64_t t0 = 0, t1 = 0;
     bool write = false;
     if (I < BR) {
@@ -483,17 +483,19 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
 template <typename MatT, typename XT, typename YT>
 static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, cudaStream_t s) {
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
+    const bool ranged = ea.I1 >= 0;
+    if (ranged && P && P->nlong > 0) return fail(AMGT_ERR_UNSUPPORTED, "row-range SpMV on a matrix with split long rows");
     const int64_t long_thr = (P && P->nlong > 0) ? WARP_CAPACITY : INT64_MAX;
-    const int64_t BR = A->blc_row;
+    const int64_t I0 = ranged ? ea.I0 : 0, BR = ranged ? ea.I1 : A->blc_row;
     const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode};
-    if (BR > 0) {
-        const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 256);
-        k_spmv_rows<MatT, XT, YT><<<blocks, 256, 0, s>>>(BR, A->blc_ptr, A->blc_idx, A->blc_map,
+    if (BR > I0) {
+        const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
+        k_spmv_rows<MatT, XT, YT><<<blocks, 256, 0, s>>>(I0, BR, A->blc_ptr, A->blc_idx, A->blc_map,
                                                          (const MatT*)A->blc_val, (const XT*)x, epi, long_thr,
                                                          sizeof(MatT) == 8 ? g_tc_thr_spmv : 17);
         AMGT_LAUNCHED();
     }
-    if (P && P->nlong > 0) {
+    if (!ranged && P && P->nlong > 0) {
         using Acc = typename AccOf<MatT>::type;
         k_spmv_chunks<MatT, XT><<<(unsigned)ceil_div(P->nchunks * 32, 256), 256, 0, s>>>(
             P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, P->long_rows,
@@ -536,7 +538,7 @@ amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* 
 
 amgt_status spmv_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s,
                       int timer_class) {
-    return spmv_ex_impl(A, x, xp, y, yp, EpiArgs{AMGT_EPI_Y, nullptr, nullptr, nullptr, 0.0}, s, timer_class);
+    return spmv_ex_impl(A, x, xp, y, yp, EpiArgs{AMGT_EPI_Y, nullptr, nullptr, nullptr, 0.0, 0, -1}, s, timer_class);
 }
 
 }  // namespace amgt
@@ -575,7 +577,24 @@ amgt_status amgt_spmv_fused(const amgt_mbsr* A, const void* x, amgt_prec xprec, 
     if ((mode == AMGT_EPI_JACOBI || mode == AMGT_EPI_RESIDUAL) && !b) return fail(AMGT_ERR_ARG, "amgt_spmv_fused: b is NULL");
     if (mode == AMGT_EPI_JACOBI && (!dinv || xprec != yprec || A->m != A->n || x == y))
         return fail(AMGT_ERR_ARG, "amgt_spmv_fused: Jacobi needs dinv, a square A, x/y of one precision, x != y");
-    return spmv_ex_impl(A, x, xprec, y, yprec, EpiArgs{mode, b, dinv, x, omega}, (cudaStream_t)stream, TC_SPMV);
+    return spmv_ex_impl(A, x, xprec, y, yprec, EpiArgs{mode, b, dinv, x, omega, 0, -1}, (cudaStream_t)stream, TC_SPMV);
+}
+
+amgt_status amgt_spmv_fused_range(const amgt_mbsr* A, int64_t blk_begin, int64_t blk_end, const void* x,
+                                  amgt_prec xprec, void* y, amgt_prec yprec, int mode, const void* b, const void* dinv,
+                                  const void* xs, double omega, void* stream) {
+    if (!A || blk_begin < 0 || blk_end < blk_begin || blk_end > A->blc_row)
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_range: bad block-row range");
+    if ((xprec != AMGT_FP64 && xprec != AMGT_FP32) || (yprec != AMGT_FP64 && yprec != AMGT_FP32))
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_range: x/y precision must be FP64 or FP32");
+    if (mode < AMGT_EPI_Y || mode > AMGT_EPI_ACCUM) return fail(AMGT_ERR_ARG, "amgt_spmv_fused_range: bad mode");
+    if ((mode == AMGT_EPI_JACOBI || mode == AMGT_EPI_RESIDUAL) && !b)
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_range: b is NULL");
+    if (mode == AMGT_EPI_JACOBI && (!dinv || !xs || xprec != yprec))
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_range: Jacobi needs dinv, xs and x/y of one precision");
+    if (blk_end == blk_begin) return AMGT_OK;
+    return spmv_ex_impl(A, x, xprec, y, yprec, EpiArgs{mode, b, dinv, xs, omega, blk_begin, blk_end},
+                        (cudaStream_t)stream, TC_SPMV);
 }
 
 }  // extern "C"

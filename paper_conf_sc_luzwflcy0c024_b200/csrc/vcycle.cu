@@ -58,8 +58,8 @@ namespace amgt {
 constexpr int NORM_BLOCKS = 256;
 
 template <typename V, typename M>
-__global__ void k_dinv(int64_t BR, int64_t m, const int64_t* __restrict__ bptr, const int32_t* __restrict__ bidx,
-                       const M* __restrict__ bval, V* __restrict__ dinv) {
+__global__ void k_dinv(int64_t BR, int64_t m, int64_t off, const int64_t* __restrict__ bptr,
+                       const int32_t* __restrict__ bidx, const M* __restrict__ bval, V* __restrict__ dinv) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= 4 * BR) return;
     const int64_t I = i >> 2;
@@ -67,7 +67,7 @@ __global__ void k_dinv(int64_t BR, int64_t m, const int64_t* __restrict__ bptr, 
     double d = 0.0;
     if (i < m)
         for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t)
-            if (bidx[t] == (int32_t)I) { d = to_f64(bval[16 * t + 5 * r]); break; }
+            if (bidx[t] == (int32_t)(I + off)) { d = to_f64(bval[16 * t + 5 * r]); break; }
     dinv[i] = (V)(d != 0.0 ? 1.0 / d : 0.0);
 }
 
@@ -120,22 +120,24 @@ static unsigned vgrid(int64_t n) {
 static size_t vbytes(amgt_prec p) { return p == AMGT_FP64 ? 8 : 4; }
 
 template <typename V, typename M>
-static void launch_dinv(amgt_level& L, cudaStream_t s) {
-    k_dinv<V, M><<<(unsigned)ceil_div(L.npad, 256), 256, 0, s>>>(L.A.blc_row, L.A.m, L.A.blc_ptr, L.A.blc_idx,
-                                                                (const M*)L.A.blc_val, (V*)L.dinv);
+static void launch_dinv(const amgt_mbsr& A, int64_t off, void* dinv, cudaStream_t s) {
+    k_dinv<V, M><<<(unsigned)ceil_div(4 * A.blc_row, 256), 256, 0, s>>>(A.blc_row, A.m, off, A.blc_ptr, A.blc_idx,
+                                                                       (const M*)A.blc_val, (V*)dinv);
 }
 
-static amgt_status build_dinv(amgt_level& L, cudaStream_t s) {
-    if (L.npad == 0) return AMGT_OK;
-    const bool v64 = L.vprec == AMGT_FP64;
-    switch (L.A.prec) {
-        case AMGT_FP64: v64 ? launch_dinv<double, double>(L, s) : launch_dinv<float, double>(L, s); break;
-        case AMGT_FP32: v64 ? launch_dinv<double, float>(L, s) : launch_dinv<float, float>(L, s); break;
-        default: v64 ? launch_dinv<double, __half>(L, s) : launch_dinv<float, __half>(L, s);
+static amgt_status dinv_impl(const amgt_mbsr& A, int64_t off, void* dinv, amgt_prec vprec, cudaStream_t s) {
+    if (A.blc_row == 0) return AMGT_OK;
+    const bool v64 = vprec == AMGT_FP64;
+    switch (A.prec) {
+        case AMGT_FP64: v64 ? launch_dinv<double, double>(A, off, dinv, s) : launch_dinv<float, double>(A, off, dinv, s); break;
+        case AMGT_FP32: v64 ? launch_dinv<double, float>(A, off, dinv, s) : launch_dinv<float, float>(A, off, dinv, s); break;
+        default: v64 ? launch_dinv<double, __half>(A, off, dinv, s) : launch_dinv<float, __half>(A, off, dinv, s);
     }
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
+
+static amgt_status build_dinv(amgt_level& L, cudaStream_t s) { return dinv_impl(L.A, 0, L.dinv, L.vprec, s); }
 
 // Host dense Cholesky + inverse of the (SPD) coarsest operator.
 static bool dense_inverse(int64_t n, std::vector<double>& a, std::vector<double>& inv) {
@@ -294,7 +296,7 @@ static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const voi
                                 const void* dinv = nullptr) {
     ++H->spmv_calls;
     // timer class 0 = the dominant kernel: SpMV with the level-1 operator A_1 (any epilogue)
-    return spmv_ex_impl(M, x, xp, y, yp, EpiArgs{mode, b, dinv, x, H->o.omega}, H->s,
+    return spmv_ex_impl(M, x, xp, y, yp, EpiArgs{mode, b, dinv, x, H->o.omega, 0, -1}, H->s,
                         (level == 0 && M == &H->L[0].A) ? TC_SPMV_L1 : TC_SPMV);
 }
 
@@ -436,6 +438,45 @@ amgt_status amgt_vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycl
     if (!H || !b || !x || ncycles < 0) return fail(AMGT_ERR_ARG, "amgt_vcycle: bad argument");
     H->s = (cudaStream_t)stream;
     return vcycle(H, b, x, ncycles, res_norms_host, spmv_calls_host);
+}
+
+amgt_status amgt_dinv(const amgt_mbsr* A, int64_t diag_tile_offset, void* dinv, amgt_prec vprec, void* stream) {
+    if (!A || !dinv || (vprec != AMGT_FP64 && vprec != AMGT_FP32)) return fail(AMGT_ERR_ARG, "amgt_dinv: bad argument");
+    return dinv_impl(*A, diag_tile_offset, dinv, vprec, (cudaStream_t)stream);
+}
+
+amgt_status amgt_dense_spd_inverse(int64_t n, const double* a_host, double* inv_host) {
+    if (n < 0 || (n > 0 && (!a_host || !inv_host))) return fail(AMGT_ERR_ARG, "amgt_dense_spd_inverse: bad argument");
+    std::vector<double> a(a_host, a_host + n * n), inv;
+    if (!dense_inverse(n, a, inv)) return fail(AMGT_ERR_ARG, "matrix is not SPD (Cholesky failed)");
+    std::copy(inv.begin(), inv.end(), inv_host);
+    return AMGT_OK;
+}
+
+amgt_status amgt_dense_matvec(int64_t n, int64_t npad, const double* Ainv, const void* b, void* x, amgt_prec vprec,
+                              void* stream) {
+    if (n < 0 || npad < n || (vprec != AMGT_FP64 && vprec != AMGT_FP32)) return fail(AMGT_ERR_ARG, "amgt_dense_matvec: bad argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (npad == 0) return AMGT_OK;
+    if (vprec == AMGT_FP64)
+        k_dense_solve<double><<<(unsigned)ceil_div(npad * 32, 256), 256, 0, s>>>(n, npad, Ainv, (const double*)b, (double*)x);
+    else
+        k_dense_solve<float><<<(unsigned)ceil_div(npad * 32, 256), 256, 0, s>>>(n, npad, Ainv, (const float*)b, (float*)x);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
+}
+
+amgt_status amgt_norm2sq(int64_t n, const double* r, double* out_dev, void* stream) {
+    if (n < 0 || !out_dev || (n > 0 && !r)) return fail(AMGT_ERR_ARG, "amgt_norm2sq: bad argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    Alloc a{nullptr, s};
+    Scratch<double> part;
+    AMGT_TRY(part.init(a, NORM_BLOCKS));
+    k_resnorm_partial<<<NORM_BLOCKS, 256, 0, s>>>(n, r, part.p);
+    AMGT_LAUNCHED();
+    k_resnorm_final<<<1, 32, 0, s>>>(part.p, out_dev);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
 }
 
 amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H) {
