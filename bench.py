@@ -226,6 +226,91 @@ def gpu_step(amgt, A, Ps, b, x, ncycles, torch):
     return res, calls
 
 
+def run_dist(args, rank, world, local):
+    """N > 1: the row-slab partitioned path, weak scaling — every rank owns a
+    128^3 slab of a 128 x 128 x (128 N) 7-point grid (N = 1 would be config 2 exactly);
+    halo exchanges over NCCL, all-reduced norms, all-gathered coarsest RHS."""
+    import torch
+    import torch.distributed as dist
+
+    import gen
+    import paper_conf_sc_luzwflcy0c024_b200 as amgt
+    from paper_conf_sc_luzwflcy0c024_b200.dist import Comm, DistHierarchy
+
+    dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    comm = Comm()
+    cfg = gen.configs.CONFIGS["cfg2"]
+    dims = (cfg.N, cfg.N, cfg.N * world)
+    nlev = cfg.nlev
+    A, rows, n, Ps = gen.partition.slab_inputs("7pt", dims, nlev, rank, world, alpha=cfg.alpha, device="cuda")
+    m = rows[1] - rows[0]
+    b = gen.uniform_vector(n, cfg.seed)[rows[0]:rows[1]].cuda()
+    x = torch.zeros(m, dtype=torch.float64, device="cuda")
+    # per-rank algorithmic bytes: the config-2 byte model (each rank's slab is a 128^3 block)
+    A2, Ps2, _, _, _ = make_inputs(cfg, "cuda")
+    sz, flops = gpu_sizes(amgt, A2, Ps2)
+    bm = byte_model(sz, args.cycles)
+    bytes_rank = sum(bm.values())
+    del A2, Ps2
+
+    def step():
+        H = DistHierarchy(comm, A, rows, n, Ps, level_prec=LEVEL_PREC[:nlev])
+        x.zero_()
+        res, calls = H.vcycle(b, x, args.cycles)
+        return H, res, calls
+
+    for _ in range(args.warmup):
+        step()
+    stream = torch.cuda.current_stream()
+    dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = amgt.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            H, res, calls = step()
+        e1.record(stream)
+        dist.barrier()
+        torch.cuda.synchronize()
+    ms = torch.tensor([e0.elapsed_time(e1) / args.steps], dtype=torch.float64, device="cuda")
+    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms_step = float(ms.item())
+    launches = amgt.launch_count() - launches0
+    # distributed level-1 SpMV (halo exchange + interior/boundary kernels), timed with events
+    L0 = H.levels[0]
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(20)]
+    y = torch.empty_like(L0.r)
+    for a_, b_ in ev:
+        a_.record(stream)
+        L0.spmv(L0.cur, y, "y")
+        b_.record(stream)
+    torch.cuda.synchronize()
+    spmv_ms = sum(a_.elapsed_time(b_) for a_, b_ in ev) / len(ev)
+    l0 = sz["lev"][0]
+    sp_bytes = l0["T"] * (16 * 8 + 6) + (l0["BR"] + 1) * 8 + 8 * 4 * l0["BC"] + 8 * 4 * l0["BR"]
+    peak, peak_kind = _peaks()
+    achieved = sp_bytes / (spmv_ms * 1e-3) / 1e9
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": round(bytes_rank * world / (ms_step * 1e-3) / 1e9, 2), "unit": "GB/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64/f32/f16 (per AMG level, L266)",
+            "data": "synthetic",
+            "config": {"workload": f"7-point Laplacian {dims[0]}x{dims[1]}x{dims[2]} row-slab partitioned over {world} GPUs "
+                                   f"(128^3 per rank; N=1 is config 2)", "levels": nlev, "vcycles_per_step": args.cycles,
+                       "parallelism": f"row-slab x{world} (NCCL halo exchange, all-reduce, all-gather)",
+                       "l2": "inputs larger than L2; no flush", "spmv_calls_per_step": calls},
+            "roofline": {"kernel": "distributed level-1 FP64 SpMV (halo exchange + k_spmv_rows interior/boundary)",
+                         "bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "peak_source": peak_kind, "bytes_per_launch": sp_bytes,
+                         "avg_launch_us": round(spmv_ms * 1e3, 2), "traffic": None},
+            "components": {"final_rel_residual": res[-1] / res[0], "bytes_per_rank_step": bytes_rank},
+            "e2e": None, "gpu_launches": launches, "clocks": clk.summary(),
+        }), flush=True)
+    dist.destroy_process_group()
+
+
 def run_gpu(args):
     import numpy as np
     import torch
@@ -238,9 +323,12 @@ def run_gpu(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
     dist = None
-    if world > 1:
-        import torch.distributed as dist
-        dist.init_process_group("nccl")
+    if world > 1 or args.force_dist:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
+        return run_dist(args, rank, world, local)
     cfg = gen.configs.CONFIGS[args.config]
     A, Ps, b, PR, N = make_inputs(cfg, "cuda")
     x = torch.zeros(4 * ((A.m + 3) // 4), dtype=torch.float64, device="cuda")
@@ -445,6 +533,7 @@ def main():
     ap.add_argument("--cycles", type=int, default=50, help="V-cycles per step (paper: 50, L308)")
     ap.add_argument("--cpu-cycles", type=int, default=10, help="V-cycles in the oracle's bounded sample")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--force-dist", action="store_true", help="use the partitioned path even at N = 1 (testing)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "amgt" else args.warmup
     if args.impl == "reference":
