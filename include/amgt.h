@@ -256,6 +256,59 @@ amgt_status amgt_dense_matvec(int64_t n, int64_t npad, const double* Ainv, const
 /* *out_dev = sum r_i^2 (deterministic two-pass reduction, FP64). */
 amgt_status amgt_norm2sq(int64_t n, const double* r, double* out_dev, void* stream);
 
+/* ------------------------------------------- native distributed V-cycle (§8(e)) */
+
+/* Communicator for the row-slab path: NCCL, loaded at run time (libnccl.so.2). */
+typedef struct amgt_dist amgt_dist;
+amgt_status amgt_dist_unique_id(void* id128_host);               /* on one rank; broadcast the 128 bytes */
+amgt_status amgt_dist_create(const void* id128_host, int rank, int size, amgt_dist** D);
+amgt_status amgt_dist_destroy(amgt_dist* D);
+amgt_status amgt_dist_allreduce_sum(amgt_dist* D, double* buf, int64_t count, void* stream);
+
+/* One level of a rank's distributed hierarchy (built by the host-side setup).
+ *   A: own rows, columns in the extended range [eb, ee) (eb 4-aligned) ; P, R: rank-local.
+ *   xe[2]: extended vectors (ping-pong), own rows at element offset `off`; b, r, dinv: own.
+ *   Halo plan: send own elements [send_off, +send_cnt) of xe to send_peer; receive halo
+ *   elements into [recv_off, +recv_cnt) from recv_peer (offsets in elements of xe; host
+ *   arrays).  Block rows [int0, int1) touch no halo (computed while the halo is in flight). */
+typedef struct {
+    const amgt_mbsr* A;
+    const amgt_mbsr* P;
+    const amgt_mbsr* R;
+    int64_t m, off, int0, int1;
+    void* xe[2];
+    void* b;
+    void* r;
+    void* dinv;
+    amgt_prec vprec;
+    int nsend, nrecv;
+    const int32_t* send_peer;
+    const int64_t* send_off;
+    const int64_t* send_cnt;
+    const int32_t* recv_peer;
+    const int64_t* recv_off;
+    const int64_t* recv_cnt;
+} amgt_dist_level;
+
+/* Coarsest level: n global rows, dense FP64 inverse (device), per-rank counts/displacements of
+ * its rows (host arrays of `size` entries), device buffers bfull/xfull of n elements. */
+typedef struct {
+    int64_t n;
+    const double* Ainv;
+    const int64_t* counts;
+    const int64_t* displs;
+    void* bfull;
+    void* xfull;
+} amgt_dist_coarse;
+
+/* Alg. 2 (L68-82) on a row-slab hierarchy: every A_k SpMV exchanges its halo (ncclSend/Recv on
+ * a side stream, overlapped with the interior block rows); residual norms are all-reduced; the
+ * coarsest right-hand side is all-gathered and solved redundantly.  b, x: own rows of level 1
+ * (FP64).  res_norms_host[ncycles+1] (global), spmv_calls_host (this rank).  Syncs at the end. */
+amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* levels, const amgt_dist_coarse* coarse,
+                             double omega, int nu1, int nu2, const double* b, double* x, int ncycles,
+                             double* res_norms_host, int64_t* spmv_calls_host, void* stream);
+
 /* ------------------------------------------------------ hierarchy + V-cycle (§II) */
 
 typedef struct {

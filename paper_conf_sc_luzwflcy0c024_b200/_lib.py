@@ -70,6 +70,20 @@ class c_vcycle_opts(ctypes.Structure):
                 ("level_prec", ctypes.c_int * 8)]
 
 
+class c_dist_level(ctypes.Structure):
+    _fields_ = [("A", ctypes.c_void_p), ("P", ctypes.c_void_p), ("R", ctypes.c_void_p), ("m", ctypes.c_int64),
+                ("off", ctypes.c_int64), ("int0", ctypes.c_int64), ("int1", ctypes.c_int64), ("xe", ctypes.c_void_p * 2),
+                ("b", ctypes.c_void_p), ("r", ctypes.c_void_p), ("dinv", ctypes.c_void_p), ("vprec", ctypes.c_int),
+                ("nsend", ctypes.c_int), ("nrecv", ctypes.c_int), ("send_peer", ctypes.c_void_p),
+                ("send_off", ctypes.c_void_p), ("send_cnt", ctypes.c_void_p), ("recv_peer", ctypes.c_void_p),
+                ("recv_off", ctypes.c_void_p), ("recv_cnt", ctypes.c_void_p)]
+
+
+class c_dist_coarse(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("Ainv", ctypes.c_void_p), ("counts", ctypes.c_void_p),
+                ("displs", ctypes.c_void_p), ("bfull", ctypes.c_void_p), ("xfull", ctypes.c_void_p)]
+
+
 _vp, _i64, _i32, _int = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_int
 _P = ctypes.POINTER
 _sigs = {
@@ -110,6 +124,12 @@ _sigs = {
     "amgt_dense_spd_inverse": (_int, [_i64, _vp, _vp]),
     "amgt_dense_matvec": (_int, [_i64, _i64, _vp, _vp, _vp, _int, _vp]),
     "amgt_norm2sq": (_int, [_i64, _vp, _vp, _vp]),
+    "amgt_dist_unique_id": (_int, [_vp]),
+    "amgt_dist_create": (_int, [_vp, _int, _int, _P(_vp)]),
+    "amgt_dist_destroy": (_int, [_vp]),
+    "amgt_dist_allreduce_sum": (_int, [_vp, _vp, _i64, _vp]),
+    "amgt_dist_vcycle": (_int, [_vp, _int, _P(c_dist_level), _P(c_dist_coarse), ctypes.c_double, _int, _int, _vp, _vp,
+                                _int, _P(ctypes.c_double), _P(_i64), _vp]),
 }
 for _name, (_res, _args) in _sigs.items():
     _f = getattr(_L, _name)

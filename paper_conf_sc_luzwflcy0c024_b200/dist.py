@@ -471,3 +471,80 @@ class DistHierarchy:
         x_own.copy_(L0.own(L0.cur))
         res = torch.stack([n.reshape(()) for n in norms]).double().sqrt().cpu().tolist()
         return res, sum(L.spmv_calls for L in Ls)
+
+
+# ------------------------------------------------------------------ native V-cycle (libamgt + NCCL)
+class NativeComm:
+    """libamgt-owned NCCL communicator (amgt_dist_create); unique id shared over `comm`."""
+
+    def __init__(self, comm: Comm):
+        import ctypes
+        from . import _lib
+        self.L = _lib
+        uid = ctypes.create_string_buffer(128)
+        if comm.rank == 0:
+            _lib._check(_lib._L.amgt_dist_unique_id(uid))
+        raw = comm.allgather_obj(bytes(uid.raw) if comm.rank == 0 else None)[0]
+        uid = ctypes.create_string_buffer(raw, 128)
+        h = ctypes.c_void_p()
+        _lib._check(_lib._L.amgt_dist_create(uid, comm.rank, comm.size, ctypes.byref(h)))
+        self.h = h
+        self.rank, self.size = comm.rank, comm.size
+
+    def close(self):
+        if self.h:
+            self.L._L.amgt_dist_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _native_vcycle(self, native: NativeComm, b_own: torch.Tensor, x_own: torch.Tensor, ncycles: int):
+    """Alg. 2 over the slabs inside libamgt (amgt_dist_vcycle): halo exchanges with NCCL on a
+    side stream overlapped with the interior rows, device-side norms and coarse gather."""
+    import ctypes
+    from . import _lib
+    keep = []
+    levels = (_lib.c_dist_level * self.nlev)()
+    for k, L in enumerate(self.levels):
+        d = levels[k]
+        d.A = ctypes.addressof(L.A.c)
+        d.P = ctypes.addressof(L.P.c) if L.P is not None else None
+        d.R = ctypes.addressof(L.R.c) if L.R is not None else None
+        d.m, d.off, d.int0, d.int1 = L.m, L.off, L.int0, L.int1
+        d.xe[0], d.xe[1] = L.xe[0].data_ptr(), L.xe[1].data_ptr()
+        d.b, d.r = L.b.data_ptr(), L.r.data_ptr()
+        d.dinv = L.dinv.data_ptr() if L.dinv.numel() else None
+        d.vprec = 0 if L.vdt == torch.float64 else 1
+        sp = np.array([q for q, _, _ in L.plan.sends], dtype=np.int32)
+        so = np.array([g0 - L.eb for _, g0, _ in L.plan.sends], dtype=np.int64)
+        sc = np.array([g1 - g0 for _, g0, g1 in L.plan.sends], dtype=np.int64)
+        rp = np.array([q for q, _, _ in L.plan.recvs], dtype=np.int32)
+        ro = np.array([g0 - L.eb for _, g0, _ in L.plan.recvs], dtype=np.int64)
+        rc = np.array([g1 - g0 for _, g0, g1 in L.plan.recvs], dtype=np.int64)
+        keep += [sp, so, sc, rp, ro, rc]
+        d.nsend, d.nrecv = len(sp), len(rp)
+        d.send_peer, d.send_off, d.send_cnt = sp.ctypes.data, so.ctypes.data, sc.ctypes.data
+        d.recv_peer, d.recv_off, d.recv_cnt = rp.ctypes.data, ro.ctypes.data, rc.ctypes.data
+    C = self.levels[-1]
+    counts = np.array([e - b for b, e in self.coarse_ranges], dtype=np.int64)
+    displs = np.array([b for b, _ in self.coarse_ranges], dtype=np.int64)
+    bfull = torch.zeros(self.nM, dtype=C.vdt, device=self.ops.device)
+    xfull = torch.zeros(self.nM, dtype=C.vdt, device=self.ops.device)
+    keep += [counts, displs, bfull, xfull]
+    co = _lib.c_dist_coarse(self.nM, self.Ainv.data_ptr(), counts.ctypes.data, displs.ctypes.data, bfull.data_ptr(),
+                            xfull.data_ptr())
+    res = (ctypes.c_double * (ncycles + 1))()
+    calls = ctypes.c_int64(0)
+    _lib._check(_lib._L.amgt_dist_vcycle(native.h, self.nlev, levels, ctypes.byref(co), float(self.omega), int(self.nu1),
+                                         int(self.nu2), b_own.data_ptr(), x_own.data_ptr(), int(ncycles), res,
+                                         ctypes.byref(calls), _lib._stream()))
+    del keep
+    return list(res), int(calls.value)
+
+
+DistHierarchy.native_vcycle = _native_vcycle

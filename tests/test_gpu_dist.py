@@ -104,3 +104,52 @@ def test_dist_gpu_mixed_precision_rho():
         res = np.array(res)
         rho = res[1:] / res[:-1]
         assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
+
+
+def _native_worker(port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        import paper_conf_sc_luzwflcy0c024_b200 as amgt
+        from paper_conf_sc_luzwflcy0c024_b200.dist import Comm, DistHierarchy, NativeComm
+        comm = Comm()
+        dims, nlev, prec = (32, 32, 32), 5, ("f64", "f32", "f16", "f16", "f16")
+        A, rows, n, Ps = gen.partition.slab_inputs("7pt", dims, nlev, 0, 1, device="cuda")
+        H = DistHierarchy(comm, A, rows, n, Ps, level_prec=prec)
+        nat = NativeComm(comm)
+        b = gen.uniform_vector(n, 3).cuda()
+        x1 = torch.zeros(n, dtype=torch.float64, device="cuda")
+        res_nat, calls_nat = H.native_vcycle(nat, b, x1, 6)
+        x2 = torch.zeros(n, dtype=torch.float64, device="cuda")
+        res_py, calls_py = H.vcycle(b, x2, 6)
+        # the single-GPU library V-cycle on the same problem
+        PR = gen.aggregation_hierarchy(dims, nlev)
+        Hs = amgt.Hierarchy(amgt.from_csr(gen.laplacian_7pt(32, device="cuda")), [amgt.from_csr(P) for P, _ in PR],
+                            level_prec=prec)
+        x3 = torch.zeros(n, dtype=torch.float64, device="cuda")
+        res_s, calls_s = Hs.vcycle(b, x3, 6)
+        nat.close()
+        q.put((res_nat, calls_nat, res_py, calls_py, res_s, calls_s, float((x1 - x3).abs().max()),
+               float((x1 - x2).abs().max())))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_dist_native_single_rank_matches_single_gpu():
+    """amgt_dist_vcycle (NCCL communicator, 1 rank) == the Python distributed driver == the
+    single-GPU amgt_vcycle (same kernels, same per-row order)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_native_worker, args=(_free_port(), q))
+    p.start()
+    try:
+        out = q.get(timeout=600)
+    finally:
+        p.join(timeout=60)
+    res_nat, calls_nat, res_py, calls_py, res_s, calls_s, dx_s, dx_py = out
+    assert calls_nat == calls_py == calls_s
+    np.testing.assert_allclose(res_nat, res_s, rtol=1e-12)
+    np.testing.assert_allclose(res_nat, res_py, rtol=1e-12)
+    assert dx_s <= 1e-12 and dx_py <= 1e-12
