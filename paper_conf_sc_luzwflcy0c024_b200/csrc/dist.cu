@@ -161,7 +161,7 @@ amgt_status dspmv(Ctx& c, const amgt_dist_level& L, int k, void* xe, void* y, in
         if (i1 <= i0) return AMGT_OK;
         return spmv_ex_impl(L.A, xe, L.vprec, y, L.vprec, EpiArgs{mode, b, L.dinv, xs, c.omega, i0, i1}, c.s, tcls);
     };
-    const bool has_int = L.int1 > L.int0;
+    const bool has_int = L.int1 > L.int0 && (L.nsend + L.nrecv) > 0;  // no halo: one launch
     if (has_int) AMGT_TRY(run(L.int0, L.int1));
     if (L.nsend + L.nrecv) AMGT_CUDA(cudaStreamWaitEvent(c.s, c.D->done, 0));
     if (has_int) {
