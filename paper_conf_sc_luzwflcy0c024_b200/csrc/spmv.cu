@@ -18,6 +18,7 @@
 //    default on B200 (DMMA rate == DFMA rate), enabled by
 //    amgt_set_tc_threshold.
 #include <climits>
+#include <cstdlib>
 
 #include "common.cuh"
 
@@ -154,8 +155,44 @@ __device__ __forceinline__ void dmma_884(double& c0, double& c1, double a, doubl
 
 // ---------------------------------------------------------------- row kernel
 // MatT = double / float / __half; XT, YT = double / float.
-template <typename MatT, typename XT, typename YT>
-__global__ void __launch_bounds__(256) k_spmv_rows(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
+// FP64 CUDA-core tile loop, U tiles per iteration: all U tiles' column indices, bitmaps and
+// values are requested before any x segment (one dependent round trip per U tiles).
+template <int U, typename XT>
+__device__ __forceinline__ void f64_tile_loop(F64Lane& L, int64_t t0, int64_t t1, const int32_t* __restrict__ bidx,
+                                              const uint16_t* __restrict__ bmap, const double* __restrict__ bval,
+                                              const XT* __restrict__ x, int q) {
+    for (int64_t t = t0; t < t1; t += U) {
+        int32_t J[U];
+        uint32_t mp[U];
+        double2 a[U], b[U], xv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const bool v = t + u < t1;
+            J[u] = v ? __ldg(bidx + t + u) : 0;
+            mp[u] = v ? __ldg(bmap + t + u) : 0u;
+            if (v) {
+                a[u] = ldg_stream(reinterpret_cast<const double2*>(bval + 16 * (t + u)) + q);
+                b[u] = ldg_stream(reinterpret_cast<const double2*>(bval + 16 * (t + u)) + 4 + q);
+            } else {
+                a[u] = make_double2(0.0, 0.0);
+                b[u] = a[u];
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) xv[u] = mp[u] ? x_pair(x, J[u], q & 1) : make_double2(0.0, 0.0);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t s0 = mp[u] >> (2 * q), s1 = mp[u] >> (8 + 2 * q);
+            L.acc0 = (s0 & 1u) ? fma(a[u].x, xv[u].x, L.acc0) : L.acc0;
+            L.acc0 = (s0 & 2u) ? fma(a[u].y, xv[u].y, L.acc0) : L.acc0;
+            L.acc1 = (s1 & 1u) ? fma(b[u].x, xv[u].x, L.acc1) : L.acc1;
+            L.acc1 = (s1 & 2u) ? fma(b[u].y, xv[u].y, L.acc1) : L.acc1;
+        }
+    }
+}
+
+template <typename MatT, typename XT, typename YT, int U = 2, int MINB = 1, bool TC = false>
+__global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
                                                    const int32_t* __restrict__ bidx,
                                                    const uint16_t* __restrict__ bmap, const MatT* __restrict__ bval,
                                                    const XT* __restrict__ x, const Epi<XT, YT> epi,
@@ -178,21 +215,8 @@ __global__ void __launch_bounds__(256) k_spmv_rows(int64_t I0, int64_t BR, const
     if (write) pre = epi.prefetch(out_i);
     if constexpr (sizeof(MatT) == 8) {
         F64Lane L;
-        const bool use_tc = tc_thr <= 16;
-        if (!use_tc) {
-            int64_t t = t0;
-            for (; t + 1 < t1; t += 2) {
-                const int32_t J0 = __ldg(bidx + t), J1 = __ldg(bidx + t + 1);
-                const uint32_t m0 = __ldg(bmap + t), m1 = __ldg(bmap + t + 1);
-                const double2 x0 = x_pair(x, J0, q & 1), x1 = x_pair(x, J1, q & 1);
-                L.step((const double*)bval + 16 * t, m0, x0, q);
-                L.step((const double*)bval + 16 * (t + 1), m1, x1, q);
-            }
-            if (t < t1) {
-                const int32_t J0 = __ldg(bidx + t);
-                const uint32_t m0 = __ldg(bmap + t);
-                L.step((const double*)bval + 16 * t, m0, x_pair(x, J0, q & 1), q);
-            }
+        if constexpr (!TC) {
+            f64_tile_loop<U>(L, t0, t1, bidx, bmap, (const double*)bval, x, q);
         } else {
             // Per-tile routing: each iteration the 8 groups hold one tile each; tiles with
             // popcount >= tc_thr are paired and multiplied with DMMA, the rest use CUDA cores.
@@ -480,6 +504,18 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
     return AMGT_OK;
 }
 
+// SpMV kernel variant (FP64): 0 = 2 tiles/iteration, 1 = 4 tiles/iteration, 2 = 4 tiles +
+// >= 5 blocks/SM, 3 = 2 tiles + >= 6 blocks/SM.  Environment AMGT_SPMV_VARIANT overrides.
+static int spmv_variant() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_SPMV_VARIANT");
+        v = e ? atoi(e) : 0;
+        if (v < 0 || v > 3) v = 0;
+    }
+    return v;
+}
+
 template <typename MatT, typename XT, typename YT>
 static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, cudaStream_t s) {
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
@@ -490,9 +526,21 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
     const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode};
     if (BR > I0) {
         const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
-        k_spmv_rows<MatT, XT, YT><<<blocks, 256, 0, s>>>(I0, BR, A->blc_ptr, A->blc_idx, A->blc_map,
-                                                         (const MatT*)A->blc_val, (const XT*)x, epi, long_thr,
-                                                         sizeof(MatT) == 8 ? g_tc_thr_spmv : 17);
+        const int tc = sizeof(MatT) == 8 ? g_tc_thr_spmv : 17;
+        auto args = [&](auto kern) {
+            kern<<<blocks, 256, 0, s>>>(I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val,
+                                        (const XT*)x, epi, long_thr, tc);
+        };
+        if (sizeof(MatT) == 8 && tc <= 16) {  // per-tile tensor-core route (separate instantiation)
+            args(k_spmv_rows<MatT, XT, YT, 2, 1, true>);
+        } else {
+            switch (sizeof(MatT) == 8 ? spmv_variant() : 0) {  // tuning knob AMGT_SPMV_VARIANT (FP64)
+                case 1: args(k_spmv_rows<MatT, XT, YT, 4, 1>); break;
+                case 2: args(k_spmv_rows<MatT, XT, YT, 4, 5>); break;
+                case 3: args(k_spmv_rows<MatT, XT, YT, 2, 6>); break;
+                default: args(k_spmv_rows<MatT, XT, YT, 2, 1>);
+            }
+        }
         AMGT_LAUNCHED();
     }
     if (!ranged && P && P->nlong > 0) {
