@@ -215,7 +215,17 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
     if (write) pre = epi.prefetch(out_i);
     if constexpr (sizeof(MatT) == 8) {
         F64Lane L;
-        if constexpr (!TC) {
+        if constexpr (!TC && U == 0) {  // round-1 loop: two tiles per iteration, loads inside step()
+            int64_t t = t0;
+            for (; t + 1 < t1; t += 2) {
+                const int32_t J0 = __ldg(bidx + t), J1 = __ldg(bidx + t + 1);
+                const uint32_t m0 = __ldg(bmap + t), m1 = __ldg(bmap + t + 1);
+                const double2 x0 = x_pair(x, J0, q & 1), x1 = x_pair(x, J1, q & 1);
+                L.step((const double*)bval + 16 * t, m0, x0, q);
+                L.step((const double*)bval + 16 * (t + 1), m1, x1, q);
+            }
+            if (t < t1) L.step((const double*)bval + 16 * t, __ldg(bmap + t), x_pair(x, __ldg(bidx + t), q & 1), q);
+        } else if constexpr (!TC) {
             f64_tile_loop<U>(L, t0, t1, bidx, bmap, (const double*)bval, x, q);
         } else {
             // Per-tile routing: each iteration the 8 groups hold one tile each; tiles with
@@ -511,7 +521,7 @@ static int spmv_variant() {
     if (v < 0) {
         const char* e = getenv("AMGT_SPMV_VARIANT");
         v = e ? atoi(e) : 0;
-        if (v < 0 || v > 3) v = 0;
+        if (v < 0 || v > 6) v = 0;
     }
     return v;
 }
@@ -538,6 +548,9 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
                 case 1: args(k_spmv_rows<MatT, XT, YT, 4, 1>); break;
                 case 2: args(k_spmv_rows<MatT, XT, YT, 4, 5>); break;
                 case 3: args(k_spmv_rows<MatT, XT, YT, 2, 6>); break;
+                case 4: args(k_spmv_rows<MatT, XT, YT, 0, 1>); break;
+                case 5: args(k_spmv_rows<MatT, XT, YT, 0, 5>); break;
+                case 6: args(k_spmv_rows<MatT, XT, YT, 8, 4>); break;
                 default: args(k_spmv_rows<MatT, XT, YT, 2, 1>);
             }
         }
