@@ -84,7 +84,8 @@ __device__ __forceinline__ float4 x_quad(const double* x, int64_t J) {
 //   EPI_RESIDUAL y_i = b_i - (A x)_i                          (Alg. 2 line 3)
 //   EPI_ACCUM    y_i = y_i + (A x)_i                          (interpolation + correction, lines 8-9)
 // Vector arithmetic is done in the y precision, as the separate vector kernels did.
-template <typename XT, typename YT>
+// MODE >= 0 fixes the epilogue at compile time (the row kernels); -1 reads `mode` at run time.
+template <typename XT, typename YT, int MODE = -1>
 struct Epi {
     YT* y;
     const YT* b;
@@ -92,13 +93,14 @@ struct Epi {
     const XT* xs;
     YT omega;
     int mode;
+    __device__ __forceinline__ int md() const { return MODE >= 0 ? MODE : mode; }
     // operands of row i, loaded before the tile loop so their latency overlaps it
     struct Pre {
         YT a = YT(0), c = YT(0), d = YT(0);
     };
     __device__ __forceinline__ Pre prefetch(int64_t i) const {
         Pre p;
-        switch (mode) {
+        switch (md()) {
             case AMGT_EPI_JACOBI: p.a = b[i]; p.c = dinv[i]; p.d = (YT)xs[i]; break;
             case AMGT_EPI_RESIDUAL: p.a = b[i]; break;
             case AMGT_EPI_ACCUM: p.a = y[i]; break;
@@ -109,7 +111,7 @@ struct Epi {
     template <typename V>
     __device__ __forceinline__ void finish(int64_t i, V v, const Pre& p) const {
         const YT t = (YT)v;
-        switch (mode) {
+        switch (md()) {
             case AMGT_EPI_JACOBI: y[i] = p.d + omega * p.c * (p.a - t); break;
             case AMGT_EPI_RESIDUAL: y[i] = p.a - t; break;
             case AMGT_EPI_ACCUM: y[i] = p.a + t; break;
@@ -119,7 +121,7 @@ struct Epi {
     __device__ __forceinline__ void apply(int64_t i, double v) const { put(i, (YT)v); }
     __device__ __forceinline__ void apply(int64_t i, float v) const { put(i, (YT)v); }
     __device__ __forceinline__ void put(int64_t i, YT t) const {
-        switch (mode) {
+        switch (md()) {
             case AMGT_EPI_JACOBI: y[i] = (YT)xs[i] + omega * dinv[i] * (b[i] - t); break;
             case AMGT_EPI_RESIDUAL: y[i] = b[i] - t; break;
             case AMGT_EPI_ACCUM: y[i] = y[i] + t; break;
@@ -191,11 +193,11 @@ __device__ __forceinline__ void f64_tile_loop(F64Lane& L, int64_t t0, int64_t t1
     }
 }
 
-template <typename MatT, typename XT, typename YT, int U = 2, int MINB = 1, bool TC = false>
+template <typename MatT, typename XT, typename YT, int MODE, int U = 2, int MINB = 1, bool TC = false>
 __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
                                                    const int32_t* __restrict__ bidx,
                                                    const uint16_t* __restrict__ bmap, const MatT* __restrict__ bval,
-                                                   const XT* __restrict__ x, const Epi<XT, YT> epi,
+                                                   const XT* __restrict__ x, const Epi<XT, YT, MODE> epi,
                                                    int64_t long_thr, int tc_thr) {
     const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -211,21 +213,11 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
     }
     // output element of this lane (FP64 layout: rows {0,2,1,3} for q = 0..3)
     const int64_t out_i = 4 * I + (sizeof(MatT) == 8 ? ((q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3) : q);
-    typename Epi<XT, YT>::Pre pre;
+    typename Epi<XT, YT, MODE>::Pre pre;
     if (write) pre = epi.prefetch(out_i);
     if constexpr (sizeof(MatT) == 8) {
         F64Lane L;
-        if constexpr (!TC && U == 0) {  // round-1 loop: two tiles per iteration, loads inside step()
-            int64_t t = t0;
-            for (; t + 1 < t1; t += 2) {
-                const int32_t J0 = __ldg(bidx + t), J1 = __ldg(bidx + t + 1);
-                const uint32_t m0 = __ldg(bmap + t), m1 = __ldg(bmap + t + 1);
-                const double2 x0 = x_pair(x, J0, q & 1), x1 = x_pair(x, J1, q & 1);
-                L.step((const double*)bval + 16 * t, m0, x0, q);
-                L.step((const double*)bval + 16 * (t + 1), m1, x1, q);
-            }
-            if (t < t1) L.step((const double*)bval + 16 * t, __ldg(bmap + t), x_pair(x, __ldg(bidx + t), q & 1), q);
-        } else if constexpr (!TC) {
+        if constexpr (!TC) {
             f64_tile_loop<U>(L, t0, t1, bidx, bmap, (const double*)bval, x, q);
         } else {
             // Per-tile routing: each iteration the 8 groups hold one tile each; tiles with
@@ -514,16 +506,43 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
     return AMGT_OK;
 }
 
-// SpMV kernel variant (FP64): 0 = 2 tiles/iteration, 1 = 4 tiles/iteration, 2 = 4 tiles +
-// >= 5 blocks/SM, 3 = 2 tiles + >= 6 blocks/SM.  Environment AMGT_SPMV_VARIANT overrides.
+// FP64 SpMV kernel variant (tiles per iteration U, minimum resident blocks MINB of 256
+// threads — i.e. the register budget): 0 = U4/5 (default), 1 = U8/4, 2 = U4/6, 3 = U2/6.
+// The environment variable AMGT_SPMV_VARIANT selects another for tuning.
 static int spmv_variant() {
     static int v = -1;
     if (v < 0) {
         const char* e = getenv("AMGT_SPMV_VARIANT");
         v = e ? atoi(e) : 0;
-        if (v < 0 || v > 6) v = 0;
+        if (v < 0 || v > 3) v = 0;
     }
     return v;
+}
+
+template <typename MatT, typename XT, typename YT, int MODE>
+static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
+                        int64_t long_thr, cudaStream_t s) {
+    const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE};
+    const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
+    const int tc = sizeof(MatT) == 8 ? g_tc_thr_spmv : 17;
+    auto go = [&](auto kern) {
+        kern<<<blocks, 256, 0, s>>>(I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x,
+                                    epi, long_thr, tc);
+    };
+    if constexpr (sizeof(MatT) == 8) {
+        if (tc <= 16) {  // per-tile tensor-core route (separate instantiation)
+            go(k_spmv_rows<MatT, XT, YT, MODE, 2, 1, true>);
+            return;
+        }
+        switch (spmv_variant()) {  // tuning knob AMGT_SPMV_VARIANT: tiles per iteration x min blocks/SM
+            case 1: go(k_spmv_rows<MatT, XT, YT, MODE, 8, 4>); break;
+            case 2: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 6>); break;
+            case 3: go(k_spmv_rows<MatT, XT, YT, MODE, 2, 6>); break;
+            default: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 5>);
+        }
+    } else {
+        go(k_spmv_rows<MatT, XT, YT, MODE, 2, 4>);
+    }
 }
 
 template <typename MatT, typename XT, typename YT>
@@ -533,31 +552,18 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
     if (ranged && P && P->nlong > 0) return fail(AMGT_ERR_UNSUPPORTED, "row-range SpMV on a matrix with split long rows");
     const int64_t long_thr = (P && P->nlong > 0) ? WARP_CAPACITY : INT64_MAX;
     const int64_t I0 = ranged ? ea.I0 : 0, BR = ranged ? ea.I1 : A->blc_row;
-    const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode};
     if (BR > I0) {
-        const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
-        const int tc = sizeof(MatT) == 8 ? g_tc_thr_spmv : 17;
-        auto args = [&](auto kern) {
-            kern<<<blocks, 256, 0, s>>>(I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val,
-                                        (const XT*)x, epi, long_thr, tc);
-        };
-        if (sizeof(MatT) == 8 && tc <= 16) {  // per-tile tensor-core route (separate instantiation)
-            args(k_spmv_rows<MatT, XT, YT, 2, 1, true>);
-        } else {
-            switch (sizeof(MatT) == 8 ? spmv_variant() : 0) {  // tuning knob AMGT_SPMV_VARIANT (FP64)
-                case 1: args(k_spmv_rows<MatT, XT, YT, 4, 1>); break;
-                case 2: args(k_spmv_rows<MatT, XT, YT, 4, 5>); break;
-                case 3: args(k_spmv_rows<MatT, XT, YT, 2, 6>); break;
-                case 4: args(k_spmv_rows<MatT, XT, YT, 0, 1>); break;
-                case 5: args(k_spmv_rows<MatT, XT, YT, 0, 5>); break;
-                case 6: args(k_spmv_rows<MatT, XT, YT, 8, 4>); break;
-                default: args(k_spmv_rows<MatT, XT, YT, 2, 1>);
-            }
+        switch (ea.mode) {
+            case AMGT_EPI_JACOBI: launch_rows<MatT, XT, YT, AMGT_EPI_JACOBI>(A, x, y, ea, I0, BR, long_thr, s); break;
+            case AMGT_EPI_RESIDUAL: launch_rows<MatT, XT, YT, AMGT_EPI_RESIDUAL>(A, x, y, ea, I0, BR, long_thr, s); break;
+            case AMGT_EPI_ACCUM: launch_rows<MatT, XT, YT, AMGT_EPI_ACCUM>(A, x, y, ea, I0, BR, long_thr, s); break;
+            default: launch_rows<MatT, XT, YT, AMGT_EPI_Y>(A, x, y, ea, I0, BR, long_thr, s);
         }
         AMGT_LAUNCHED();
     }
     if (!ranged && P && P->nlong > 0) {
         using Acc = typename AccOf<MatT>::type;
+        const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode};
         k_spmv_chunks<MatT, XT><<<(unsigned)ceil_div(P->nchunks * 32, 256), 256, 0, s>>>(
             P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, P->long_rows,
             P->chunk_ptr, P->chunk_lr, (Acc*)P->partial);
