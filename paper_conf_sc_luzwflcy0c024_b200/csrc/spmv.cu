@@ -6,8 +6,9 @@
 //    16-B halves {16q, 64+16q} of the 128-B tile (so every load instruction of the
 //    group covers one contiguous 64-B span) plus one 16-B x segment; FP32 lane q loads
 //    its row (16 B); FP16 lane q loads its row (8 B).  Each lane multiplies only the
-//    entries whose bitmap bit is set (Alg. 5 lines 9-11, GETBIT).  Two tiles in flight
-//    per lane per iteration.
+//    entries whose bitmap bit is set (Alg. 5 lines 9-11, GETBIT).  FP64: 8 tiles per
+//    iteration (all indices/bitmaps/values requested before the x gathers: one dependent
+//    round trip per 8 tiles) under a 64-register budget (4 blocks of 256 per SM).
 //  * Load balancing (L220, Fig. 5): with a plan (amgt_spmv_analyze), block rows longer
 //    than WARP_CAPACITY = 64 tiles are split into 64-tile warp chunks (8 groups x 8
 //    tiles, Alg. 5 lines 4-6 with reading R12); each chunk reduces its 8 groups with
@@ -507,7 +508,8 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
 }
 
 // FP64 SpMV kernel variant (tiles per iteration U, minimum resident blocks MINB of 256
-// threads — i.e. the register budget): 0 = U4/5 (default), 1 = U8/4, 2 = U4/6, 3 = U2/6.
+// threads — i.e. the register budget): 0 = U8/4 (default; measured best on B200, see
+// DESIGN.md §7), 1 = U4/5, 2 = U4/6, 3 = U2/6.
 // The environment variable AMGT_SPMV_VARIANT selects another for tuning.
 static int spmv_variant() {
     static int v = -1;
@@ -535,10 +537,10 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
             return;
         }
         switch (spmv_variant()) {  // tuning knob AMGT_SPMV_VARIANT: tiles per iteration x min blocks/SM
-            case 1: go(k_spmv_rows<MatT, XT, YT, MODE, 8, 4>); break;
+            case 1: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 5>); break;
             case 2: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 6>); break;
             case 3: go(k_spmv_rows<MatT, XT, YT, MODE, 2, 6>); break;
-            default: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 5>);
+            default: go(k_spmv_rows<MatT, XT, YT, MODE, 8, 4>);
         }
     } else {
         go(k_spmv_rows<MatT, XT, YT, MODE, 2, 4>);
