@@ -288,25 +288,39 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
         const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
         if (write) epi.finish(out_i, (q & 1) ? s1 : s0, pre);
     } else {
+        // FP32 / FP16 tiles: lane q owns tile row q; U tiles' indices, bitmaps and row values
+        // are requested before the x gathers (one dependent round trip per U tiles).
         float acc = 0.f;
-        for (int64_t t = t0; t < t1; ++t) {
-            const int32_t J = __ldg(bidx + t);
-            const uint32_t nib = (__ldg(bmap + t) >> (4 * q)) & 0xFu;
-            const float4 xv = x_quad(x, J);
-            float a0, a1, a2, a3;
-            if constexpr (sizeof(MatT) == 4) {
-                const float4 a = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * t) + q);
-                a0 = a.x; a1 = a.y; a2 = a.z; a3 = a.w;
-            } else {
-                const uint2 u = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * t) + q);
-                const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
-                const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
-                a0 = lo.x; a1 = lo.y; a2 = hi.x; a3 = hi.y;
+        for (int64_t t = t0; t < t1; t += U) {
+            int32_t J[U];
+            uint32_t nib[U];
+            float4 a[U], xv[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const bool v = t + u < t1;
+                J[u] = v ? __ldg(bidx + t + u) : 0;
+                nib[u] = v ? (__ldg(bmap + t + u) >> (4 * q)) & 0xFu : 0u;
+                a[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (v) {
+                    if constexpr (sizeof(MatT) == 4) {
+                        a[u] = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * (t + u)) + q);
+                    } else {
+                        const uint2 w = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * (t + u)) + q);
+                        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
+                        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
+                        a[u] = make_float4(lo.x, lo.y, hi.x, hi.y);
+                    }
+                }
             }
-            acc = (nib & 1u) ? fmaf(a0, xv.x, acc) : acc;
-            acc = (nib & 2u) ? fmaf(a1, xv.y, acc) : acc;
-            acc = (nib & 4u) ? fmaf(a2, xv.z, acc) : acc;
-            acc = (nib & 8u) ? fmaf(a3, xv.w, acc) : acc;
+#pragma unroll
+            for (int u = 0; u < U; ++u) xv[u] = nib[u] ? x_quad(x, J[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                acc = (nib[u] & 1u) ? fmaf(a[u].x, xv[u].x, acc) : acc;
+                acc = (nib[u] & 2u) ? fmaf(a[u].y, xv[u].y, acc) : acc;
+                acc = (nib[u] & 4u) ? fmaf(a[u].z, xv[u].z, acc) : acc;
+                acc = (nib[u] & 8u) ? fmaf(a[u].w, xv[u].w, acc) : acc;
+            }
         }
         if (write) epi.finish(out_i, acc, pre);
     }
@@ -543,7 +557,7 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
             default: go(k_spmv_rows<MatT, XT, YT, MODE, 8, 4>);
         }
     } else {
-        go(k_spmv_rows<MatT, XT, YT, MODE, 2, 4>);
+        go(k_spmv_rows<MatT, XT, YT, MODE, 8, 4>);
     }
 }
 
