@@ -153,6 +153,7 @@ amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a,
 // ------------------------------------------------------------------ instrumentation
 static std::atomic<int64_t> g_launches{0};
 void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+void count_launches(int64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
 struct TimerRec {
     int cls;
@@ -173,6 +174,8 @@ static cudaEvent_t pool_event() {
     ++g_used;
     return e;
 }
+
+unsigned timing_mask() { return g_timing; }
 
 TimerScope::TimerScope(int c, double b, cudaStream_t st) : cls(c), bytes(b), s(st), slot(-1) {
     if (!(g_timing & (1u << c))) return;

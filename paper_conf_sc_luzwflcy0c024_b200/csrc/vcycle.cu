@@ -50,6 +50,13 @@ struct amgt_hierarchy {
     double* norms = nullptr;    // per-cycle squared residual norms (device)
     int norms_cap = 0;
     int64_t spmv_calls = 0;
+    // CUDA graph of the sub-cycle below level 1 (levels 2..M down, coarse solve, up), captured
+    // once per hierarchy on an internal stream and replayed every cycle
+    cudaStream_t gs = nullptr;
+    cudaEvent_t gev[2] = {nullptr, nullptr};
+    cudaGraphExec_t gexec = nullptr;
+    bool graph_failed = false;
+    int64_t sub_calls = 0, sub_launches = 0;
     Alloc alloc() { return Alloc{has_al ? &al : nullptr, s}; }
 };
 
@@ -194,6 +201,10 @@ static void destroy(amgt_hierarchy* H) {
     a.put(H->partial, NORM_BLOCKS * sizeof(double));
     a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
     cudaStreamSynchronize(H->s);
+    if (H->gexec) cudaGraphExecDestroy(H->gexec);
+    if (H->gs) { cudaStreamSynchronize(H->gs); cudaStreamDestroy(H->gs); }
+    for (cudaEvent_t e : H->gev)
+        if (e) cudaEventDestroy(e);
     delete H;
 }
 
@@ -318,12 +329,112 @@ static amgt_status dense_solve(amgt_hierarchy* H, amgt_level& L) {
     return AMGT_OK;
 }
 
+constexpr int JAC = 1, RES = 2, ACC = 3;
+
+// Alg. 2 lines 2-4 at level k: pre-smoothing, residual, restriction into b_{k+1}.
+static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** xc, void** xa) {
+    amgt_level& L = H->L[k];
+    const void* bk = k == 0 ? b0 : L.b;
+    if (k > 0) AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, H->s));
+    for (int i = 0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
+        AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
+        std::swap(xc[k], xa[k]);
+    }
+    AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, L.r, L.vprec, k, RES, bk));  // line 3
+    amgt_level& N = H->L[k + 1];
+    return counted_spmv(H, &L.R, L.r, L.vprec, N.b, N.vprec, k);  // line 4: restriction
+}
+
+// Alg. 2 lines 8-10 at level k: interpolation + correction, post-smoothing.
+static amgt_status up_level(amgt_hierarchy* H, int k, const void* b0, void** xc, void** xa) {
+    amgt_level& L = H->L[k];
+    amgt_level& N = H->L[k + 1];
+    const void* bk = k == 0 ? b0 : L.b;
+    AMGT_TRY(counted_spmv(H, &L.P, xc[k + 1], N.vprec, xc[k], L.vprec, k, ACC));  // lines 8-9
+    for (int i = 0; i < H->o.nu2; ++i) {  // line 10: post-smoothing
+        AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
+        std::swap(xc[k], xa[k]);
+    }
+    return AMGT_OK;
+}
+
+static amgt_status coarse_solve(amgt_hierarchy* H, void** xc) {  // line 6
+    const int M = H->nlev - 1;
+    amgt_level C = H->L[M];
+    C.x = xc[M];
+    return C.vprec == AMGT_FP64 ? dense_solve<double>(H, C) : dense_solve<float>(H, C);
+}
+
+// Levels 1..M-1 down, coarsest, levels M-1..1 up (everything below level 1).
+static amgt_status subcycle_direct(amgt_hierarchy* H, void** xc, void** xa) {
+    const int M = H->nlev - 1;
+    for (int k = 1; k < M; ++k) AMGT_TRY(down_level(H, k, nullptr, xc, xa));
+    AMGT_TRY(coarse_solve(H, xc));
+    for (int k = M - 1; k >= 1; --k) AMGT_TRY(up_level(H, k, nullptr, xc, xa));
+    return AMGT_OK;
+}
+
+unsigned timing_mask();
+void count_launches(int64_t n);
+
+// The sub-cycle touches only hierarchy-owned buffers, and with nu1 + nu2 even every level's
+// ping-pong pair is back in place after a cycle, so one captured graph serves every cycle of
+// every amgt_vcycle call.  Graphs are skipped while per-class timing of the coarse classes is
+// enabled (the instrumented profile needs one event pair per launch).
+static amgt_status subcycle(amgt_hierarchy* H, void** xc, void** xa) {
+    const bool usable = !H->graph_failed && ((H->o.nu1 + H->o.nu2) % 2 == 0) && (timing_mask() & ~1u) == 0;
+    if (!usable) return subcycle_direct(H, xc, xa);
+    cudaStream_t user = H->s;
+    if (!H->gexec) {
+        if (!H->gs) AMGT_CUDA(cudaStreamCreateWithFlags(&H->gs, cudaStreamNonBlocking));
+        for (cudaEvent_t& e : H->gev)
+            if (!e) AMGT_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        void* xc0[8];
+        void* xa0[8];
+        std::copy(xc, xc + 8, xc0);
+        std::copy(xa, xa + 8, xa0);
+        const int64_t calls0 = H->spmv_calls, launches0 = amgt_launch_count();
+        AMGT_CUDA(cudaStreamSynchronize(user));
+        H->s = H->gs;
+        cudaGraph_t g = nullptr;
+        amgt_status st = AMGT_OK;
+        if (cudaStreamBeginCapture(H->gs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+            st = AMGT_ERR_CUDA;
+        } else {
+            st = subcycle_direct(H, xc, xa);
+            if (cudaStreamEndCapture(H->gs, &g) != cudaSuccess) st = AMGT_ERR_CUDA;
+        }
+        H->s = user;
+        bool same = std::equal(xc, xc + 8, xc0) && std::equal(xa, xa + 8, xa0);
+        if (st == AMGT_OK && same && g && cudaGraphInstantiate(&H->gexec, g, 0) == cudaSuccess) {
+            H->sub_calls = H->spmv_calls - calls0;
+            H->sub_launches = amgt_launch_count() - launches0;
+        } else {
+            H->gexec = nullptr;
+            H->graph_failed = true;
+        }
+        if (g) cudaGraphDestroy(g);
+        cudaGetLastError();
+        H->spmv_calls = calls0;  // the capture executed nothing
+        std::copy(xc0, xc0 + 8, xc);
+        std::copy(xa0, xa0 + 8, xa);
+        if (!H->gexec) return subcycle_direct(H, xc, xa);
+    }
+    AMGT_CUDA(cudaEventRecord(H->gev[0], user));
+    AMGT_CUDA(cudaStreamWaitEvent(H->gs, H->gev[0], 0));
+    AMGT_CUDA(cudaGraphLaunch(H->gexec, H->gs));
+    AMGT_CUDA(cudaEventRecord(H->gev[1], H->gs));
+    AMGT_CUDA(cudaStreamWaitEvent(user, H->gev[1], 0));
+    H->spmv_calls += H->sub_calls;
+    count_launches(H->sub_launches);
+    return AMGT_OK;
+}
+
 // Alg. 2 with the vector steps fused into the SpMV epilogues: each smoothing sweep is one
 // kernel (out of place, ping-pong between x and t), the residual one kernel, the
 // interpolation + correction one kernel.  SpMV calls are counted exactly as in Alg. 2.
 static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_host,
                           int64_t* calls_host) {
-    constexpr int JAC = 1, RES = 2, ACC = 3;
     cudaStream_t s = H->s;
     Alloc a = H->alloc();
     if (ncycles + 1 > H->norms_cap) {
@@ -353,33 +464,10 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
         }
     }
     for (int c = 1; c <= ncycles && M > 0; ++c) {
-        for (int k = 0; k < M; ++k) {  // Alg. 2 lines 1-5
-            amgt_level& L = H->L[k];
-            const void* bk = k == 0 ? (const void*)b : L.b;
-            if (k > 0) AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, s));
-            for (int i = 0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
-                AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
-                std::swap(xc[k], xa[k]);
-            }
-            AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, L.r, L.vprec, k, RES, bk));  // line 3
-            amgt_level& N = H->L[k + 1];
-            AMGT_TRY(counted_spmv(H, &L.R, L.r, L.vprec, N.b, N.vprec, k));  // line 4: restriction
-        }
-        {  // line 6: coarsest level
-            amgt_level C = H->L[M];
-            C.x = xc[M];
-            AMGT_TRY(C.vprec == AMGT_FP64 ? dense_solve<double>(H, C) : dense_solve<float>(H, C));
-        }
-        for (int k = M - 1; k >= 0; --k) {  // lines 7-11
-            amgt_level& L = H->L[k];
-            amgt_level& N = H->L[k + 1];
-            const void* bk = k == 0 ? (const void*)b : L.b;
-            AMGT_TRY(counted_spmv(H, &L.P, xc[k + 1], N.vprec, xc[k], L.vprec, k, ACC));  // lines 8-9
-            for (int i = 0; i < H->o.nu2; ++i) {  // line 10: post-smoothing
-                AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
-                std::swap(xc[k], xa[k]);
-            }
-        }
+        AMGT_TRY(down_level(H, 0, b, xc, xa));              // Alg. 2 lines 1-5 at level 1
+        if (M >= 2) AMGT_TRY(subcycle(H, xc, xa));          // levels 2..M (graph replay)
+        else AMGT_TRY(coarse_solve(H, xc));
+        AMGT_TRY(up_level(H, 0, b, xc, xa));                // lines 7-11 at level 1
         AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));  // residual (L308)
         AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms + c));
     }
