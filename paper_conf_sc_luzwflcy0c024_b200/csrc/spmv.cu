@@ -34,6 +34,7 @@ struct SpmvPlan {
     int32_t* chunk_lr = nullptr;   // [nchunks] -> index into long_rows
     double* partial = nullptr;     // [nchunks*4] (double or float accumulators)
     amgt_spmv_stats st{};
+    double mean_row = 0.0;  // tiles per block row
 };
 
 void spmv_plan_free(void* aux, Alloc& a) {
@@ -326,6 +327,68 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
     }
 }
 
+// ---------------------------------------------------------------- lane-per-row kernel
+// For operators with ~1 tile per block row (interpolation P, L262/Alg. 2 line 8): one lane
+// owns a whole block row (its tiles' 16 values, its x segment, its 4 outputs), 32 block rows
+// per warp, so every dependent round trip moves 32 tiles instead of 8.
+template <typename MatT, typename XT, typename YT, int MODE>
+__global__ void __launch_bounds__(256) k_spmv_lanerow(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
+                                                      const int32_t* __restrict__ bidx,
+                                                      const uint16_t* __restrict__ bmap,
+                                                      const MatT* __restrict__ bval, const XT* __restrict__ x,
+                                                      const Epi<XT, YT, MODE> epi) {
+    using Acc = typename AccOf<MatT>::type;
+    const int64_t I = I0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (I >= BR) return;
+    const int64_t t0 = __ldg(bptr + I), t1 = __ldg(bptr + I + 1);
+    typename Epi<XT, YT, MODE>::Pre pre[4];
+#pragma unroll
+    for (int r = 0; r < 4; ++r) pre[r] = epi.prefetch(4 * I + r);
+    Acc acc[4] = {Acc(0), Acc(0), Acc(0), Acc(0)};
+    for (int64_t t = t0; t < t1; ++t) {
+        const int32_t J = __ldg(bidx + t);
+        const uint32_t mp = __ldg(bmap + t);
+        Acc v[16];
+        if constexpr (sizeof(MatT) == 8) {
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const double2 d = ldg_stream(reinterpret_cast<const double2*>(bval + 16 * t) + k);
+                v[2 * k] = d.x;
+                v[2 * k + 1] = d.y;
+            }
+        } else if constexpr (sizeof(MatT) == 4) {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const float4 d = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * t) + k);
+                v[4 * k] = d.x; v[4 * k + 1] = d.y; v[4 * k + 2] = d.z; v[4 * k + 3] = d.w;
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const uint2 w = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * t) + k);
+                const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
+                const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
+                v[4 * k] = lo.x; v[4 * k + 1] = lo.y; v[4 * k + 2] = hi.x; v[4 * k + 3] = hi.y;
+            }
+        }
+        Acc xv[4];
+        if constexpr (sizeof(Acc) == 8) {
+            const double2 a = x_pair(x, J, 0), b = x_pair(x, J, 1);
+            xv[0] = a.x; xv[1] = a.y; xv[2] = b.x; xv[3] = b.y;
+        } else {
+            const float4 a = x_quad(x, J);
+            xv[0] = a.x; xv[1] = a.y; xv[2] = a.z; xv[3] = a.w;
+        }
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                acc[r] = ((mp >> (4 * r + c)) & 1u) ? fma(v[4 * r + c], xv[c], acc[r]) : acc[r];
+    }
+#pragma unroll
+    for (int r = 0; r < 4; ++r) epi.finish(4 * I + r, acc[r], pre[r]);
+}
+
 // ---------------------------------------------------------------- chunk kernel (long rows)
 template <typename MatT, typename XT>
 __global__ void __launch_bounds__(256) k_spmv_chunks(int64_t nchunks, const int64_t* __restrict__ bptr,
@@ -517,6 +580,7 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
     P->st.long_rows = nl;
     P->st.chunks = ncx;
     P->st.tc_tiles = (int64_t)ht[0];
+    P->mean_row = mean;
     A->aux = P;
     return AMGT_OK;
 }
@@ -539,6 +603,12 @@ template <typename MatT, typename XT, typename YT, int MODE>
 static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
                         int64_t long_thr, cudaStream_t s) {
     const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE};
+    const SpmvPlan* P = (const SpmvPlan*)A->aux;
+    if (P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16) {  // ~1 tile per block row
+        k_spmv_lanerow<MatT, XT, YT, MODE><<<(unsigned)ceil_div(BR - I0, 256), 256, 0, s>>>(
+            I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, epi);
+        return;
+    }
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
     const int tc = sizeof(MatT) == 8 ? g_tc_thr_spmv : 17;
     auto go = [&](auto kern) {

@@ -25,6 +25,8 @@ MATS = [
     ("irregular_small", lambda: gen.irregular_block_sparse(1 << 11)),
     ("rand_ragged", lambda: gen.random_csr(333, 271, 0.03, 9, empty_rows=20)),
     ("rand_longrows", lambda: gen.random_csr(40, 2000, 0.4, 10)),
+    ("aggregation_P", lambda: gen.aggregation_P((16, 16, 16))),            # 1 tile per block row
+    ("sparse_rows", lambda: gen.random_csr(999, 3001, 0.0004, 14, empty_rows=50)),  # <= 2 tiles per row
 ]
 
 
