@@ -414,21 +414,21 @@ def run_gpu(args):
     d2h = hx.numel() * 8 + (args.cycles + 1) * 8
     e2e_steps = args.steps
 
-    def h2d(t):
+    def to_dev(t):
         d = torch.empty(t.shape, dtype=t.dtype, device="cuda")
         d.copy_(t, non_blocking=True)
         return d
 
-    def h2d_csr(M):
-        return type(M)(M.m, M.n, h2d(M.row_ptr), h2d(M.col), h2d(M.val))
+    def to_dev_csr(M):
+        return type(M)(M.m, M.n, to_dev(M.row_ptr), to_dev(M.col), to_dev(M.val))
 
     barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     for _ in range(e2e_steps):
-        dA = h2d_csr(hA)
-        dPs = [h2d_csr(P) for P in hPs]
-        db = h2d(hb)
+        dA = to_dev_csr(hA)
+        dPs = [to_dev_csr(P) for P in hPs]
+        db = to_dev(hb)
         gpu_step(amgt, dA, dPs, db, x, args.cycles, torch)  # residual norms come back to the host here
         hx.copy_(x, non_blocking=True)
     e1.record(stream)
