@@ -47,25 +47,30 @@ struct Alloc {
     void put(void* p, size_t bytes);
 };
 
-// RAII scratch buffer from the caller's allocator (stream-ordered).
+// Library-internal temporaries: CUDA's stream-ordered pool (cudaMallocAsync on the call's
+// stream; the pool keeps freed memory cached), never the caller's allocator — outputs the
+// caller sees use the amgt_allocator, scratch does not need to cross the ABI.
+void* scratch_get(size_t bytes, cudaStream_t s);
+void scratch_put(void* p, cudaStream_t s);
+
 template <typename T>
 struct Scratch {
-    Alloc* a = nullptr;
+    cudaStream_t s = nullptr;
     T* p = nullptr;
     size_t n = 0;
     Scratch() = default;
     Scratch(const Scratch&) = delete;
     Scratch& operator=(const Scratch&) = delete;
     amgt_status init(Alloc& al, size_t count) {
-        a = &al;
+        s = al.s;
         n = count;
         if (count == 0) return AMGT_OK;
-        p = static_cast<T*>(al.get(count * sizeof(T)));
+        p = static_cast<T*>(scratch_get(count * sizeof(T), s));
         if (!p) return fail(AMGT_ERR_ALLOC, "scratch allocation of %zu bytes failed", count * sizeof(T));
         return AMGT_OK;
     }
     ~Scratch() {
-        if (a && p) a->put(p, n * sizeof(T));
+        if (p) scratch_put(p, s);
     }
 };
 

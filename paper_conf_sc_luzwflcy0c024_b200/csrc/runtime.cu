@@ -46,6 +46,30 @@ void Alloc::put(void* p, size_t bytes) {
     cudaFreeAsync(p, s);
 }
 
+void* scratch_get(size_t bytes, cudaStream_t s) {
+    static bool pool_set = false;
+    if (!pool_set) {  // keep freed pool memory cached across synchronisations
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t thr = UINT64_MAX;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        }
+        pool_set = true;
+    }
+    void* p = nullptr;
+    if (cudaMallocAsync(&p, bytes ? bytes : 16, s) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return p;
+}
+
+void scratch_put(void* p, cudaStream_t s) {
+    if (p) cudaFreeAsync(p, s);
+}
+
 size_t prec_bytes(amgt_prec p) { return p == AMGT_FP64 ? 8 : (p == AMGT_FP32 ? 4 : 2); }
 
 int num_sms() {

@@ -31,6 +31,13 @@ amgt_status mbsr_alloc(amgt_mbsr* M, int64_t m, int64_t n, int64_t T, amgt_prec 
 amgt_status mbsr_release(amgt_mbsr* M, Alloc& a);
 
 constexpr int NBINS = 8;
+// Internal row categories: the paper's 8 bins (L151) plus category 8 = the rows of bin 0
+// with Cub <= 32, which the 4-lane-group symbolic kernel takes.  stats[] layout:
+// [0..7] bins (category 8 counted separately), [8] cub_total, [9] pairs_nonzero,
+// [10] pairs_tc, [11] scalar products, [12] category-8 rows.
+constexpr int NCAT = 9;
+constexpr int SMALL_CUB = 32;
+__host__ __device__ inline int cat_stat(int c) { return c < NBINS ? c : 12; }
 constexpr int EMPTY_KEY = -1;
 
 struct SymCtx {  // device pointers shared by the symbolic kernels
@@ -47,8 +54,8 @@ template <bool STATS>
 __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, unsigned long long* __restrict__ stats,
                           int tc_thr) {
     // stats: [0..7] bin counts, [8] cub_total, [9] pairs_nonzero, [10] pairs_tc, [11] scalar products
-    __shared__ unsigned long long sh[12];
-    if (threadIdx.x < 12) sh[threadIdx.x] = 0;
+    __shared__ unsigned long long sh[13];
+    if (threadIdx.x < 13) sh[threadIdx.x] = 0;
     __syncthreads();
     unsigned long long cubs = 0, pnz = 0, ptc = 0, sp = 0;
     for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
@@ -72,8 +79,9 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
         }
         int b = 0;
         while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
+        if (b == 0 && cub <= SMALL_CUB) b = NBINS;  // category 8 (sub-bin of bin 0)
         bin_of[I] = b;
-        atomicAdd(&sh[b], 1ull);
+        atomicAdd(&sh[cat_stat(b)], 1ull);
         cubs += cub;
     }
     atomicAdd(&sh[8], cubs);
@@ -81,15 +89,15 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
     atomicAdd(&sh[10], ptc);
     atomicAdd(&sh[11], sp);
     __syncthreads();
-    if (threadIdx.x < 12 && sh[threadIdx.x]) atomicAdd(&stats[threadIdx.x], sh[threadIdx.x]);
+    if (threadIdx.x < 13 && sh[threadIdx.x]) atomicAdd(&stats[threadIdx.x], sh[threadIdx.x]);
 }
 
 __global__ void k_bin_scatter(int64_t BR, const int64_t* __restrict__ bin_of, const unsigned long long* __restrict__ stats,
                               unsigned long long* __restrict__ cursor, int32_t* __restrict__ rows) {
-    __shared__ unsigned long long off[NBINS];
+    __shared__ unsigned long long off[NCAT];
     if (threadIdx.x == 0) {
         unsigned long long s = 0;
-        for (int b = 0; b < NBINS; ++b) { off[b] = s; s += stats[b]; }
+        for (int b = 0; b < NCAT; ++b) { off[b] = s; s += stats[cat_stat(b)]; }
     }
     __syncthreads();
     const int lane = threadIdx.x & 31;
@@ -276,6 +284,94 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
         for (int j = 0; j < n; ++j) rank += keys[j] < k;
         cidx[out + rank] = k;
         cmap[out + rank] = (uint16_t)maps[i];
+    }
+}
+
+// ---------------------------------------------------------------- step kernels: tiny rows
+// Category 8 (bin-0 rows with Cub <= 32): one 4-lane group per row, 8 rows per warp.  The
+// row's distinct tile columns (<= 32) form a per-group list in shared memory (keys + OR of
+// the BITMAPMULTIPLY results); each candidate is searched by the four lanes in parallel and
+// appended when absent — the degenerate, collision-free form of the paper's hash table.
+// Deterministic, no atomics.  Step 1 writes the count, step 2 sorts (rank) and writes.
+template <int STEP>
+__global__ void __launch_bounds__(256) k_sym_group(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
+                                                   int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
+                                                   int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
+    __shared__ int keys[64][SMALL_CUB];
+    __shared__ uint32_t maps[64][SMALL_CUB];
+    const int lane = threadIdx.x & 31, r = lane & 3, gl = threadIdx.x >> 2;
+    const unsigned gm = 0xFu << (lane & ~3);
+    const int64_t rr = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2);
+    if (rr >= nrows) return;  // whole group leaves together
+    const int64_t I = rows[rr];
+    int* K = keys[gl];
+    uint32_t* Mp = maps[gl];
+    int n = 0;
+    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+    for (int64_t base = a0; base < a1; base += 4) {
+        const int64_t t = base + r;
+        const bool v = t < a1;
+        const int32_t Kc = v ? c.aidx[t] : 0;
+        const uint32_t ma = v ? c.amap[t] : 0u;
+        const int64_t b0 = v ? c.bptr[Kc] : 0;
+        const int64_t len = v ? c.bptr[Kc + 1] - b0 : 0;
+        int64_t incl = len;
+        int64_t y = __shfl_up_sync(gm, incl, 1, 4);
+        if (r >= 1) incl += y;
+        y = __shfl_up_sync(gm, incl, 2, 4);
+        if (r >= 2) incl += y;
+        const int64_t excl = incl - len;
+        const int64_t total = __shfl_sync(gm, incl, 3, 4);
+        for (int64_t p0 = 0; p0 < total; p0 += 4) {
+            const int64_t p = p0 + r;
+            int lo = 0;  // owner: largest lane with excl <= p
+            for (int step = 2; step; step >>= 1) {
+                const int cand = lo + step;
+                const int64_t e = __shfl_sync(gm, excl, cand & 3, 4);
+                if (cand < 4 && e <= p) lo = cand;
+            }
+            const int64_t ob0 = __shfl_sync(gm, b0, lo, 4), oex = __shfl_sync(gm, excl, lo, 4);
+            const uint32_t oma = __shfl_sync(gm, ma, lo, 4);
+            uint32_t mc = 0u;
+            int32_t J = -1;
+            if (p < total) {
+                const int64_t j = ob0 + (p - oex);
+                mc = bitmap_multiply(oma, c.bmap[j]);
+                if (mc) J = c.bidx[j];
+            }
+            for (int l = 0; l < 4; ++l) {  // insert the four candidates in lane order
+                const int32_t Jl = __shfl_sync(gm, J, l, 4);
+                const uint32_t ml = __shfl_sync(gm, mc, l, 4);
+                if (!ml) continue;
+                int hit = -1;
+                for (int i = r; i < n; i += 4)
+                    if (K[i] == Jl) hit = i;
+                hit = max(hit, __shfl_xor_sync(gm, hit, 1, 4));
+                hit = max(hit, __shfl_xor_sync(gm, hit, 2, 4));
+                if (r == 0) {
+                    if (hit >= 0) {
+                        Mp[hit] |= ml;
+                    } else {
+                        K[n] = Jl;
+                        Mp[n] = ml;
+                    }
+                }
+                if (hit < 0) ++n;
+                __syncwarp(gm);
+            }
+        }
+    }
+    if (STEP == 1) {
+        if (r == 0) nnz_row[I] = n;
+        return;
+    }
+    const int64_t out = cptr[I];
+    for (int i = r; i < n; i += 4) {
+        const int k = K[i];
+        int rank = 0;
+        for (int j2 = 0; j2 < n; ++j2) rank += K[j2] < k;
+        cidx[out + rank] = k;
+        cmap[out + rank] = (uint16_t)Mp[i];
     }
 }
 
@@ -1049,6 +1145,11 @@ template <int STEP>
 static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_t* rows, const SymCtx& c, int64_t BCB,
                             Alloc& a, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
                             cudaStream_t s) {
+    if (cnt[NBINS] > 0) {
+        k_sym_group<STEP><<<(unsigned)ceil_div(ceil_div(cnt[NBINS], 8) * 32, 256), 256, 0, s>>>(
+            cnt[NBINS], rows + off[NBINS], c, nnz_row, cptr, cidx, cmap);
+        AMGT_LAUNCHED();
+    }
     AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, s)));
     AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, s)));
     AMGT_TRY((launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, s)));
@@ -1073,15 +1174,15 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     const int64_t BR = A->blc_row;
     SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
     Scratch<int64_t> bin_of, nnz_row;
-    Scratch<unsigned long long> stats, cursor;
+    Scratch<unsigned long long> stats, cursor;  // stats: 16 slots (layout above)
     Scratch<int32_t> rows;
     AMGT_TRY(bin_of.init(a, BR + 1));
     AMGT_TRY(nnz_row.init(a, BR + 1));
     AMGT_TRY(stats.init(a, 16));
-    AMGT_TRY(cursor.init(a, NBINS));
+    AMGT_TRY(cursor.init(a, NCAT));
     AMGT_TRY(rows.init(a, BR + 1));
     AMGT_CUDA(cudaMemsetAsync(stats.p, 0, 16 * sizeof(unsigned long long), s));
-    AMGT_CUDA(cudaMemsetAsync(cursor.p, 0, NBINS * sizeof(unsigned long long), s));
+    AMGT_CUDA(cudaMemsetAsync(cursor.p, 0, NCAT * sizeof(unsigned long long), s));
     amgt_mbsr C{};
     C.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
     if (!C.blc_ptr) return fail(AMGT_ERR_ALLOC, "SpGEMM: blc_ptr allocation failed");
@@ -1099,8 +1200,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         }
         AMGT_CUDA(cudaMemcpyAsync(hs, stats.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
         AMGT_CUDA(cudaStreamSynchronize(s));  // sync 1: bin sizes
-        int64_t cnt[NBINS], off[NBINS], acc = 0;
-        for (int b = 0; b < NBINS; ++b) { cnt[b] = (int64_t)hs[b]; off[b] = acc; acc += cnt[b]; }
+        int64_t cnt[NCAT], off[NCAT], acc = 0;
+        for (int b = 0; b < NCAT; ++b) { cnt[b] = (int64_t)hs[cat_stat(b)]; off[b] = acc; acc += cnt[b]; }
         if (BR > 0) {
             amgt_status st = run_bins<1>(cnt, off, rows.p, c, B->blc_col, a, nnz_row.p, nullptr, nullptr, nullptr, s);
             if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
@@ -1120,6 +1221,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     }
     if (info) {
         for (int b = 0; b < NBINS; ++b) info->bin_rows[b] = (int64_t)hs[b];
+        info->bin_rows[0] += (int64_t)hs[12];  // category 8 is part of bin 0
         info->cub_total = (int64_t)hs[8];
         info->pairs_nonzero = (int64_t)hs[9];
         info->pairs_tc = (int64_t)hs[10];
