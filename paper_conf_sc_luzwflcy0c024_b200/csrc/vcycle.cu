@@ -6,9 +6,14 @@
 // applied on the device as a dense FP64 matvec (R22).
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
+#include <cstring>
 #include <vector>
 
+#include <cooperative_groups.h>
+
 #include "common.cuh"
+#include "spmv_core.cuh"
 
 namespace amgt {
 
@@ -377,13 +382,188 @@ static amgt_status subcycle_direct(amgt_hierarchy* H, void** xc, void** xa) {
 unsigned timing_mask();
 void count_launches(int64_t n);
 
+// ---------------------------------------------------------------- persistent coarse sub-cycle
+// Levels 2..M of the V-cycle (everything below level 1: a few thousand rows per level,
+// launch-latency bound) run as ONE cooperative kernel: every CTA stays resident and the
+// Alg. 2 steps are separated by grid-wide barriers instead of kernel boundaries.  Each
+// SpMV is the same 4-lane-group row code as k_spmv_rows (spmv_octet), warps striding over
+// block-row octets.  Vectors of all coarse levels share one precision VT.
+struct CoopMat {
+    const int64_t* ptr;
+    const int32_t* idx;
+    const uint16_t* map;
+    const void* val;
+    int prec;
+    int64_t BR;
+};
+struct CoopLevel {
+    CoopMat A, P, R;
+    void* b;
+    void* x[2];
+    void* r;
+    const void* dinv;
+    int64_t npad;
+};
+struct CoopArgs {
+    CoopLevel L[8];
+    int k0, M, nu1, nu2;
+    double omega;
+    int64_t nM;
+    const double* Ainv;
+};
+
+template <typename VT, int MODE>
+__device__ __forceinline__ void coop_spmv(const CoopMat& M, const VT* x, VT* y, const VT* b, const VT* dinv,
+                                          const VT* xs, double omega, int64_t gw, int64_t nw, int lane) {
+    const Epi<VT, VT, MODE> epi{y, b, dinv, xs, (VT)omega, MODE};
+    const int64_t noct = (M.BR + 7) / 8;
+    switch (M.prec) {
+        case AMGT_FP64:
+            for (int64_t o = gw; o < noct; o += nw)
+                spmv_octet<double, VT, VT, MODE, 4>(0, o, M.BR, M.ptr, M.idx, M.map, (const double*)M.val, x, epi, lane);
+            break;
+        case AMGT_FP32:
+            for (int64_t o = gw; o < noct; o += nw)
+                spmv_octet<float, VT, VT, MODE, 4>(0, o, M.BR, M.ptr, M.idx, M.map, (const float*)M.val, x, epi, lane);
+            break;
+        default:
+            for (int64_t o = gw; o < noct; o += nw)
+                spmv_octet<__half, VT, VT, MODE, 4>(0, o, M.BR, M.ptr, M.idx, M.map, (const __half*)M.val, x, epi,
+                                                    lane);
+    }
+}
+
+template <typename VT>
+__global__ void __launch_bounds__(256) k_subcycle(const CoopArgs a) {
+    namespace cg = cooperative_groups;
+    cg::grid_group grid = cg::this_grid();
+    const int lane = threadIdx.x & 31;
+    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+    const int64_t gw = gt >> 5, nw = nt >> 5;
+    int cur[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (int k = a.k0; k < a.M; ++k) {  // Alg. 2 lines 1-5
+        const CoopLevel& L = a.L[k];
+        VT* x0 = (VT*)L.x[0];
+        for (int64_t i = gt; i < L.npad; i += nt) x0[i] = VT(0);
+        cur[k] = 0;
+        grid.sync();
+        for (int s = 0; s < a.nu1; ++s) {
+            coop_spmv<VT, AMGT_EPI_JACOBI>(L.A, (const VT*)L.x[cur[k]], (VT*)L.x[1 - cur[k]], (const VT*)L.b,
+                                           (const VT*)L.dinv, (const VT*)L.x[cur[k]], a.omega, gw, nw, lane);
+            cur[k] ^= 1;
+            grid.sync();
+        }
+        coop_spmv<VT, AMGT_EPI_RESIDUAL>(L.A, (const VT*)L.x[cur[k]], (VT*)L.r, (const VT*)L.b, nullptr, nullptr,
+                                         a.omega, gw, nw, lane);
+        grid.sync();
+        coop_spmv<VT, AMGT_EPI_Y>(L.R, (const VT*)L.r, (VT*)a.L[k + 1].b, nullptr, nullptr, nullptr, a.omega, gw, nw,
+                                  lane);
+        grid.sync();
+    }
+    {  // line 6: coarsest level, x_M = A_M^{-1} b_M (dense FP64), warp per row
+        const CoopLevel& C = a.L[a.M];
+        const VT* bM = (const VT*)C.b;
+        VT* xM = (VT*)C.x[0];
+        for (int64_t row = gw; row < C.npad; row += nw) {
+            double acc = 0.0;
+            if (row < a.nM)
+                for (int64_t j = lane; j < a.nM; j += 32) acc = fma(a.Ainv[row * a.nM + j], (double)bM[j], acc);
+            for (int d = 16; d; d >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, d);
+            if (lane == 0) xM[row] = (VT)acc;
+        }
+        cur[a.M] = 0;
+        grid.sync();
+    }
+    for (int k = a.M - 1; k >= a.k0; --k) {  // lines 7-11
+        const CoopLevel& L = a.L[k];
+        coop_spmv<VT, AMGT_EPI_ACCUM>(L.P, (const VT*)a.L[k + 1].x[cur[k + 1]], (VT*)L.x[cur[k]], nullptr, nullptr,
+                                      nullptr, a.omega, gw, nw, lane);
+        grid.sync();
+        for (int s = 0; s < a.nu2; ++s) {
+            coop_spmv<VT, AMGT_EPI_JACOBI>(L.A, (const VT*)L.x[cur[k]], (VT*)L.x[1 - cur[k]], (const VT*)L.b,
+                                           (const VT*)L.dinv, (const VT*)L.x[cur[k]], a.omega, gw, nw, lane);
+            cur[k] ^= 1;
+            grid.sync();
+        }
+    }
+}
+
+static CoopMat coop_mat(const amgt_mbsr& M) {
+    return CoopMat{M.blc_ptr, M.blc_idx, M.blc_map, M.blc_val, (int)M.prec, M.blc_row};
+}
+
+// Returns AMGT_ERR_UNSUPPORTED (caller falls back) when the levels' vector precisions differ
+// or a cooperative launch is not possible.
+static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
+    const int M = H->nlev - 1, k0 = 1;
+    const amgt_prec vp = H->L[k0].vprec;
+    for (int k = k0; k <= M; ++k)
+        if (H->L[k].vprec != vp || xc[k] != H->L[k].x || xa[k] != H->L[k].t) return AMGT_ERR_UNSUPPORTED;
+    CoopArgs a{};
+    for (int k = k0; k <= M; ++k) {
+        const amgt_level& L = H->L[k];
+        CoopLevel& c = a.L[k];
+        c.A = coop_mat(L.A);
+        if (k < M) {
+            c.P = coop_mat(L.P);
+            c.R = coop_mat(L.R);
+        }
+        c.b = L.b;
+        c.x[0] = L.x;
+        c.x[1] = L.t;
+        c.r = L.r;
+        c.dinv = L.dinv;
+        c.npad = L.npad;
+    }
+    a.k0 = k0;
+    a.M = M;
+    a.nu1 = H->o.nu1;
+    a.nu2 = H->o.nu2;
+    a.omega = H->o.omega;
+    a.nM = H->nM;
+    a.Ainv = H->Ainv;
+    static int grid64 = 0, grid32 = 0;
+    int& grid = vp == AMGT_FP64 ? grid64 : grid32;
+    const void* kern = vp == AMGT_FP64 ? (const void*)k_subcycle<double> : (const void*)k_subcycle<float>;
+    if (grid == 0) {
+        int dev = 0, coop = 0, per_sm = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev);
+        if (!coop || cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, 0) != cudaSuccess || per_sm < 1) {
+            cudaGetLastError();
+            grid = -1;
+        } else {
+            grid = num_sms() * (per_sm < 2 ? per_sm : 2);
+        }
+    }
+    if (grid < 0) return AMGT_ERR_UNSUPPORTED;
+    void* args[] = {&a};
+    AMGT_CUDA(cudaLaunchCooperativeKernel(kern, dim3(grid), dim3(256), args, 0, H->s));
+    count_launch();
+    H->spmv_calls += (int64_t)(M - k0) * (H->o.nu1 + H->o.nu2 + 3);
+    return AMGT_OK;
+}
+
 // The sub-cycle touches only hierarchy-owned buffers, and with nu1 + nu2 even every level's
 // ping-pong pair is back in place after a cycle, so one captured graph serves every cycle of
 // every amgt_vcycle call.  Graphs are skipped while per-class timing of the coarse classes is
 // enabled (the instrumented profile needs one event pair per launch).
+static int coarse_mode() {  // AMGT_COARSE = coop (default) | graph | direct
+    static int m = -1;
+    if (m < 0) {
+        const char* e = getenv("AMGT_COARSE");
+        m = (e && !strcmp(e, "graph")) ? 1 : (e && !strcmp(e, "direct")) ? 2 : 0;
+    }
+    return m;
+}
+
 static amgt_status subcycle(amgt_hierarchy* H, void** xc, void** xa) {
     const bool usable = !H->graph_failed && ((H->o.nu1 + H->o.nu2) % 2 == 0) && (timing_mask() & ~1u) == 0;
-    if (!usable) return subcycle_direct(H, xc, xa);
+    if (!usable || coarse_mode() == 2) return subcycle_direct(H, xc, xa);
+    if (coarse_mode() == 0) {
+        const amgt_status st = subcycle_coop(H, xc, xa);
+        if (st != AMGT_ERR_UNSUPPORTED) return st;
+    }
     cudaStream_t user = H->s;
     if (!H->gexec) {
         if (!H->gs) AMGT_CUDA(cudaStreamCreateWithFlags(&H->gs, cudaStreamNonBlocking));
