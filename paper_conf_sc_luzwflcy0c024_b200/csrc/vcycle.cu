@@ -407,6 +407,7 @@ struct CoopLevel {
 struct CoopArgs {
     CoopLevel L[8];
     int k0, M, nu1, nu2;
+    int kb;  // levels kb..M run inside CTA 0 alone (block barriers instead of grid barriers)
     double omega;
     int64_t nM;
     const double* Ainv;
@@ -433,59 +434,82 @@ __device__ __forceinline__ void coop_spmv(const CoopMat& M, const VT* x, VT* y, 
     }
 }
 
+// One Alg. 2 step sequence on level k: grid-wide (all CTAs, grid barriers) when `grid_wide`,
+// else CTA 0 alone with block barriers (the other CTAs skip the work but keep `cur` in step).
 template <typename VT>
 __global__ void __launch_bounds__(256) k_subcycle(const CoopArgs a) {
     namespace cg = cooperative_groups;
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
-    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
-    const int64_t gw = gt >> 5, nw = nt >> 5;
     int cur[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    auto run = [&](bool grid_wide, auto&& work) {
+        if (grid_wide) {
+            const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+            work(gt, nt);
+            grid.sync();
+        } else if (blockIdx.x == 0) {
+            work((int64_t)threadIdx.x, (int64_t)blockDim.x);
+            __syncthreads();
+        }
+    };
     for (int k = a.k0; k < a.M; ++k) {  // Alg. 2 lines 1-5
         const CoopLevel& L = a.L[k];
-        VT* x0 = (VT*)L.x[0];
-        for (int64_t i = gt; i < L.npad; i += nt) x0[i] = VT(0);
+        const bool gwide = k < a.kb;
+        run(gwide, [&](int64_t gt, int64_t nt) {
+            VT* x0 = (VT*)L.x[0];
+            for (int64_t i = gt; i < L.npad; i += nt) x0[i] = VT(0);
+        });
         cur[k] = 0;
-        grid.sync();
         for (int s = 0; s < a.nu1; ++s) {
-            coop_spmv<VT, AMGT_EPI_JACOBI>(L.A, (const VT*)L.x[cur[k]], (VT*)L.x[1 - cur[k]], (const VT*)L.b,
-                                           (const VT*)L.dinv, (const VT*)L.x[cur[k]], a.omega, gw, nw, lane);
+            const int c = cur[k];
+            run(gwide, [&](int64_t gt, int64_t nt) {
+                coop_spmv<VT, AMGT_EPI_JACOBI>(L.A, (const VT*)L.x[c], (VT*)L.x[1 - c], (const VT*)L.b,
+                                               (const VT*)L.dinv, (const VT*)L.x[c], a.omega, gt >> 5, nt >> 5, lane);
+            });
             cur[k] ^= 1;
-            grid.sync();
         }
-        coop_spmv<VT, AMGT_EPI_RESIDUAL>(L.A, (const VT*)L.x[cur[k]], (VT*)L.r, (const VT*)L.b, nullptr, nullptr,
-                                         a.omega, gw, nw, lane);
-        grid.sync();
-        coop_spmv<VT, AMGT_EPI_Y>(L.R, (const VT*)L.r, (VT*)a.L[k + 1].b, nullptr, nullptr, nullptr, a.omega, gw, nw,
-                                  lane);
-        grid.sync();
+        const int c = cur[k];
+        run(gwide, [&](int64_t gt, int64_t nt) {
+            coop_spmv<VT, AMGT_EPI_RESIDUAL>(L.A, (const VT*)L.x[c], (VT*)L.r, (const VT*)L.b, nullptr, nullptr,
+                                             a.omega, gt >> 5, nt >> 5, lane);
+        });
+        run(gwide, [&](int64_t gt, int64_t nt) {
+            coop_spmv<VT, AMGT_EPI_Y>(L.R, (const VT*)L.r, (VT*)a.L[k + 1].b, nullptr, nullptr, nullptr, a.omega,
+                                      gt >> 5, nt >> 5, lane);
+        });
     }
-    {  // line 6: coarsest level, x_M = A_M^{-1} b_M (dense FP64), warp per row
+    run(a.M < a.kb, [&](int64_t gt, int64_t nt) {  // line 6: x_M = A_M^{-1} b_M (dense FP64)
         const CoopLevel& C = a.L[a.M];
         const VT* bM = (const VT*)C.b;
         VT* xM = (VT*)C.x[0];
-        for (int64_t row = gw; row < C.npad; row += nw) {
+        for (int64_t row = gt >> 5; row < C.npad; row += nt >> 5) {
             double acc = 0.0;
             if (row < a.nM)
                 for (int64_t j = lane; j < a.nM; j += 32) acc = fma(a.Ainv[row * a.nM + j], (double)bM[j], acc);
             for (int d = 16; d; d >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, d);
             if (lane == 0) xM[row] = (VT)acc;
         }
-        cur[a.M] = 0;
-        grid.sync();
-    }
+    });
+    cur[a.M] = 0;
     for (int k = a.M - 1; k >= a.k0; --k) {  // lines 7-11
         const CoopLevel& L = a.L[k];
-        coop_spmv<VT, AMGT_EPI_ACCUM>(L.P, (const VT*)a.L[k + 1].x[cur[k + 1]], (VT*)L.x[cur[k]], nullptr, nullptr,
-                                      nullptr, a.omega, gw, nw, lane);
-        grid.sync();
+        const bool gwide = k < a.kb;
+        if (k + 1 == a.kb) grid.sync();  // leaving the block-local levels: everyone sees CTA 0's result
+        const int cn = cur[k + 1], c0 = cur[k];
+        run(gwide, [&](int64_t gt, int64_t nt) {
+            coop_spmv<VT, AMGT_EPI_ACCUM>(L.P, (const VT*)a.L[k + 1].x[cn], (VT*)L.x[c0], nullptr, nullptr, nullptr,
+                                          a.omega, gt >> 5, nt >> 5, lane);
+        });
         for (int s = 0; s < a.nu2; ++s) {
-            coop_spmv<VT, AMGT_EPI_JACOBI>(L.A, (const VT*)L.x[cur[k]], (VT*)L.x[1 - cur[k]], (const VT*)L.b,
-                                           (const VT*)L.dinv, (const VT*)L.x[cur[k]], a.omega, gw, nw, lane);
+            const int c = cur[k];
+            run(gwide, [&](int64_t gt, int64_t nt) {
+                coop_spmv<VT, AMGT_EPI_JACOBI>(L.A, (const VT*)L.x[c], (VT*)L.x[1 - c], (const VT*)L.b,
+                                               (const VT*)L.dinv, (const VT*)L.x[c], a.omega, gt >> 5, nt >> 5, lane);
+            });
             cur[k] ^= 1;
-            grid.sync();
         }
     }
+    if (a.kb <= a.k0) grid.sync();  // every level was block-local
 }
 
 static CoopMat coop_mat(const amgt_mbsr& M) {
@@ -522,6 +546,15 @@ static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
     a.omega = H->o.omega;
     a.nM = H->nM;
     a.Ainv = H->Ainv;
+    // first level small enough for one CTA (AMGT_COOP_BLOCKROWS, default 128 block rows)
+    static int64_t small_br = -1;
+    if (small_br < 0) {
+        const char* e = getenv("AMGT_COOP_BLOCKROWS");
+        small_br = e ? atoll(e) : 128;
+    }
+    a.kb = M + 1;
+    for (int k = k0; k <= M; ++k)
+        if (H->L[k].A.blc_row <= small_br) { a.kb = k; break; }
     static int grid64 = 0, grid32 = 0;
     int& grid = vp == AMGT_FP64 ? grid64 : grid32;
     const void* kern = vp == AMGT_FP64 ? (const void*)k_subcycle<double> : (const void*)k_subcycle<float>;
@@ -533,7 +566,9 @@ static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
             cudaGetLastError();
             grid = -1;
         } else {
-            grid = num_sms() * (per_sm < 2 ? per_sm : 2);
+            const char* e = getenv("AMGT_COOP_PER_SM");
+            const int want = e ? atoi(e) : 1;
+            grid = num_sms() * (per_sm < want ? per_sm : want);
         }
     }
     if (grid < 0) return AMGT_ERR_UNSUPPORTED;
