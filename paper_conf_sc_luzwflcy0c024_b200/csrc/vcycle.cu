@@ -583,11 +583,13 @@ static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
 // ping-pong pair is back in place after a cycle, so one captured graph serves every cycle of
 // every amgt_vcycle call.  Graphs are skipped while per-class timing of the coarse classes is
 // enabled (the instrumented profile needs one event pair per launch).
-static int coarse_mode() {  // AMGT_COARSE = coop (default) | graph | direct
+// AMGT_COARSE = graph (default: CUDA graph replay) | coop (persistent cooperative kernel,
+// measured equal on config 2) | direct (plain launches).
+static int coarse_mode() {
     static int m = -1;
     if (m < 0) {
         const char* e = getenv("AMGT_COARSE");
-        m = (e && !strcmp(e, "graph")) ? 1 : (e && !strcmp(e, "direct")) ? 2 : 0;
+        m = (e && !strcmp(e, "coop")) ? 0 : (e && !strcmp(e, "direct")) ? 2 : 1;
     }
     return m;
 }
