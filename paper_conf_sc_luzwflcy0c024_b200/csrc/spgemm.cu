@@ -57,10 +57,14 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
     __shared__ unsigned long long sh[13];
     if (threadIdx.x < 13) sh[threadIdx.x] = 0;
     __syncthreads();
+    // one 4-lane group per block row; the lanes split the row's A tiles (independent loads)
     unsigned long long cubs = 0, pnz = 0, ptc = 0, sp = 0;
-    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+    const int r = threadIdx.x & 3;
+    const unsigned gm = 0xFu << ((threadIdx.x & 31) & ~3);
+    const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2, ng = ((int64_t)gridDim.x * blockDim.x) >> 2;
+    for (int64_t I = g0; I < BR; I += ng) {
         int64_t cub = 0;
-        for (int64_t t = c.aptr[I]; t < c.aptr[I + 1]; ++t) {
+        for (int64_t t = c.aptr[I] + r; t < c.aptr[I + 1]; t += 4) {
             const int32_t K = c.aidx[t];
             const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
             cub += b1 - b0;
@@ -77,12 +81,16 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
                 }
             }
         }
-        int b = 0;
-        while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
-        if (b == 0 && cub <= SMALL_CUB) b = NBINS;  // category 8 (sub-bin of bin 0)
-        bin_of[I] = b;
-        atomicAdd(&sh[cat_stat(b)], 1ull);
-        cubs += cub;
+        cub += __shfl_xor_sync(gm, cub, 1, 4);
+        cub += __shfl_xor_sync(gm, cub, 2, 4);
+        if (r == 0) {
+            int b = 0;
+            while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
+            if (b == 0 && cub <= SMALL_CUB) b = NBINS;  // category 8 (sub-bin of bin 0)
+            bin_of[I] = b;
+            atomicAdd(&sh[cat_stat(b)], 1ull);
+            cubs += cub;
+        }
     }
     atomicAdd(&sh[8], cubs);
     atomicAdd(&sh[9], pnz);
@@ -288,17 +296,19 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
 }
 
 // ---------------------------------------------------------------- step kernels: tiny rows
-// Category 8 (bin-0 rows with Cub <= 32): one 4-lane group per row, 8 rows per warp.  The
-// row's distinct tile columns (<= 32) form a per-group list in shared memory (keys + OR of
-// the BITMAPMULTIPLY results); each candidate is searched by the four lanes in parallel and
-// appended when absent — the degenerate, collision-free form of the paper's hash table.
-// Deterministic, no atomics.  Step 1 writes the count, step 2 sorts (rank) and writes.
+// Category 8 (bin-0 rows with Cub <= 32): one 4-lane group per row, 8 rows per warp.  All of
+// the row's candidates (tile column J of every pair with BITMAPMULTIPLY != 0) are written to
+// a per-group list in shared memory; a candidate counts when it is the first occurrence of
+// its J (the collision-free degenerate form of the paper's hash table, with the "hash" being
+// the candidate position).  Step 1 writes the distinct count; step 2 writes each distinct J
+// at its rank with the OR of the bitmaps of all its occurrences.  Deterministic, no atomics.
 template <int STEP>
 __global__ void __launch_bounds__(256) k_sym_group(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
                                                    int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
                                                    int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
     __shared__ int keys[64][SMALL_CUB];
     __shared__ uint32_t maps[64][SMALL_CUB];
+    __shared__ unsigned char first[64][SMALL_CUB];
     const int lane = threadIdx.x & 31, r = lane & 3, gl = threadIdx.x >> 2;
     const unsigned gm = 0xFu << (lane & ~3);
     const int64_t rr = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2);
@@ -306,9 +316,10 @@ __global__ void __launch_bounds__(256) k_sym_group(int64_t nrows, const int32_t*
     const int64_t I = rows[rr];
     int* K = keys[gl];
     uint32_t* Mp = maps[gl];
-    int n = 0;
+    unsigned char* F = first[gl];
+    int64_t npairs = 0;
     const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
-    for (int64_t base = a0; base < a1; base += 4) {
+    for (int64_t base = a0; base < a1; base += 4) {  // expand: every pair of the row into the list
         const int64_t t = base + r;
         const bool v = t < a1;
         const int32_t Kc = v ? c.aidx[t] : 0;
@@ -320,58 +331,46 @@ __global__ void __launch_bounds__(256) k_sym_group(int64_t nrows, const int32_t*
         if (r >= 1) incl += y;
         y = __shfl_up_sync(gm, incl, 2, 4);
         if (r >= 2) incl += y;
-        const int64_t excl = incl - len;
         const int64_t total = __shfl_sync(gm, incl, 3, 4);
-        for (int64_t p0 = 0; p0 < total; p0 += 4) {
-            const int64_t p = p0 + r;
-            int lo = 0;  // owner: largest lane with excl <= p
-            for (int step = 2; step; step >>= 1) {
-                const int cand = lo + step;
-                const int64_t e = __shfl_sync(gm, excl, cand & 3, 4);
-                if (cand < 4 && e <= p) lo = cand;
-            }
-            const int64_t ob0 = __shfl_sync(gm, b0, lo, 4), oex = __shfl_sync(gm, excl, lo, 4);
-            const uint32_t oma = __shfl_sync(gm, ma, lo, 4);
-            uint32_t mc = 0u;
-            int32_t J = -1;
-            if (p < total) {
-                const int64_t j = ob0 + (p - oex);
-                mc = bitmap_multiply(oma, c.bmap[j]);
-                if (mc) J = c.bidx[j];
-            }
-            for (int l = 0; l < 4; ++l) {  // insert the four candidates in lane order
-                const int32_t Jl = __shfl_sync(gm, J, l, 4);
-                const uint32_t ml = __shfl_sync(gm, mc, l, 4);
-                if (!ml) continue;
-                int hit = -1;
-                for (int i = r; i < n; i += 4)
-                    if (K[i] == Jl) hit = i;
-                hit = max(hit, __shfl_xor_sync(gm, hit, 1, 4));
-                hit = max(hit, __shfl_xor_sync(gm, hit, 2, 4));
-                if (r == 0) {
-                    if (hit >= 0) {
-                        Mp[hit] |= ml;
-                    } else {
-                        K[n] = Jl;
-                        Mp[n] = ml;
-                    }
-                }
-                if (hit < 0) ++n;
-                __syncwarp(gm);
-            }
+        for (int64_t jj = 0; jj < len; ++jj) {  // lane r writes its A tile's pairs
+            const int64_t j = b0 + jj;
+            const uint32_t mc = bitmap_multiply(ma, c.bmap[j]);
+            const int64_t p = npairs + incl - len + jj;
+            K[p] = mc ? c.bidx[j] : -1;
+            Mp[p] = mc;
         }
+        npairs += total;
     }
+    __syncwarp(gm);
+    const int n = (int)npairs;
+    int cnt = 0;
+    for (int i = r; i < n; i += 4) {  // first occurrences
+        const int k = K[i];
+        bool f = k >= 0;
+        for (int j = 0; j < i && f; ++j) f = K[j] != k;
+        F[i] = f;
+        cnt += f;
+    }
+    cnt += __shfl_xor_sync(gm, cnt, 1, 4);
+    cnt += __shfl_xor_sync(gm, cnt, 2, 4);
     if (STEP == 1) {
-        if (r == 0) nnz_row[I] = n;
+        if (r == 0) nnz_row[I] = cnt;
         return;
     }
+    __syncwarp(gm);
     const int64_t out = cptr[I];
     for (int i = r; i < n; i += 4) {
+        if (!F[i]) continue;
         const int k = K[i];
         int rank = 0;
-        for (int j2 = 0; j2 < n; ++j2) rank += K[j2] < k;
+        uint32_t m = 0;
+        for (int j = 0; j < n; ++j) {
+            const int kj = K[j];
+            rank += (F[j] && kj < k);
+            m |= (kj == k) ? Mp[j] : 0u;
+        }
         cidx[out + rank] = k;
-        cmap[out + rank] = (uint16_t)Mp[i];
+        cmap[out + rank] = (uint16_t)m;
     }
 }
 
@@ -908,13 +907,32 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
         t = c.aptr[I];
         a1 = c.aptr[I + 1];
     }
-    auto next_a = [&]() {  // move to the next A tile with a non-empty B row
+    // A-tile metadata cache: lane u of the group holds (bitmap, B-row range) of tile cbase + u,
+    // loaded four tiles at a time (parallel loads) instead of one dependent chain per tile.
+    const unsigned gm = 0xFu << (lane & ~3);
+    int64_t cbase = INT64_MIN, cb0 = 0, cb1 = 0;
+    uint32_t cma = 0;
+    auto load_chunk = [&](int64_t base) {
+        cbase = base;
+        const int64_t tt = base + r;
+        cb0 = cb1 = 0;
+        cma = 0;
+        if (tt < a1) {
+            const int32_t K = c.aidx[tt];
+            cma = c.amap[tt];
+            cb0 = c.bptr[K];
+            cb1 = c.bptr[K + 1];
+        }
+    };
+    auto next_a = [&]() {  // move to the next A tile with a non-empty B row (group-uniform)
         while (t < a1) {
-            const int32_t K = c.aidx[t];
-            j = c.bptr[K];
-            jend = c.bptr[K + 1];
+            if (t >= cbase + 4) load_chunk(t);
+            const int u = (int)(t - cbase);
+            j = __shfl_sync(gm, cb0, u, 4);
+            jend = __shfl_sync(gm, cb1, u, 4);
+            const uint32_t m = __shfl_sync(gm, cma, u, 4);
             if (j < jend) {
-                mA = c.amap[t];
+                mA = m;
                 RowIO<T>::load(aval + 16 * t + 4 * r, arow);
                 return;
             }
@@ -1191,9 +1209,9 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
         if (BR > 0) {
             if (info)
-                k_analyze<true><<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+                k_analyze<true><<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
             else
-                k_analyze<false><<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+                k_analyze<false><<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
             AMGT_LAUNCHED();
             k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats.p, cursor.p, rows.p);
             AMGT_LAUNCHED();
