@@ -821,6 +821,163 @@ __global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(const int32_t* __res
     }
 }
 
+// ---------------------------------------------------------------- numeric: long rows
+// C block rows with more than CAP tiles (power-law rows of config 4): one CTA per row.  The
+// row's C tile columns are copied to shared memory (when <= LONG_SMEM tiles) for the
+// position search; the row's pairs are flattened across the CTA (no serialisation over A
+// tiles).  Dense A tiles (POPCOUNT >= threshold, FP64) go to DMMA m8n8k4 exactly as Alg. 4:
+// fragA = [A;A], fragB = [B_j | B_j'], two quadrants kept; warps take the dense tiles
+// round-robin.  Accumulation: FP64/FP32 atomics into the output (FP32 workspace for FP16),
+// only at the bitmap positions a product can touch — the order of additions is not fixed,
+// so these rows are reproducible up to rounding (exact on integer/dyadic data).
+constexpr int LONG_SMEM = 16384;
+
+__device__ __forceinline__ int bsearch_any(const int32_t* idx, int n, int32_t J) {
+    int lo = 0, hi = n - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (idx[mid] < J) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict__ rows,
+                                                      const unsigned long long* __restrict__ nrows_dev, SymCtx c,
+                                                      const T* __restrict__ aval, const T* __restrict__ bval,
+                                                      const int64_t* __restrict__ cptr, const int32_t* __restrict__ cidx_g,
+                                                      const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+                                                      Acc* __restrict__ gacc, int tc_thr) {
+    extern __shared__ __align__(16) int32_t sidx[];
+    __shared__ int64_t sh_excl[256], sh_b0[256], sh_tot[9];
+    __shared__ uint32_t sh_ma[256];
+    const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    const int64_t nrows = (int64_t)*nrows_dev;
+    for (int64_t rr = blockIdx.x; rr < nrows; rr += gridDim.x) {
+        const int64_t I = rows[rr];
+        const int64_t c0 = cptr[I];
+        const int nC = (int)(cptr[I + 1] - c0);
+        const bool in_smem = nC <= LONG_SMEM;
+        const int32_t* cidx = in_smem ? sidx : cidx_g + c0;
+        if (in_smem)
+            for (int q = tid; q < nC; q += nt) sidx[q] = cidx_g[c0 + q];
+        Acc* acc = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
+        for (int64_t e = tid; e < 16 * (int64_t)nC; e += nt) acc[e] = Acc(0);
+        __syncthreads();
+        const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+        // ---- tensor-core route (FP64): warp-level DMMA per dense A tile
+        if constexpr (sizeof(T) == 8) {
+            int dense_seen = 0;
+            for (int64_t base = a0; base < a1; base += 32) {
+                const int64_t t = base + lane;
+                const uint32_t ma = t < a1 ? c.amap[t] : 0u;
+                uint32_t dense = __ballot_sync(0xffffffffu, t < a1 && __popc(ma) >= tc_thr);
+                while (dense) {
+                    const int src = __ffs(dense) - 1;
+                    dense &= dense - 1;
+                    if ((dense_seen++ % nw) != w) continue;  // round-robin over warps
+                    const int64_t ta = base + src;
+                    const uint32_t mA = __shfl_sync(0xffffffffu, ma, src);
+                    const int32_t K = c.aidx[ta];
+                    const double fa = (double)aval[16 * ta + 4 * ((lane >> 2) & 3) + (lane & 3)];
+                    const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
+                    for (int64_t jb = b0; jb < b1; jb += 32) {
+                        const int64_t j = jb + lane;
+                        const uint32_t mc = j < b1 ? bitmap_multiply(mA, c.bmap[j]) : 0u;
+                        const int q = mc ? bsearch_any(cidx, nC, c.bidx[j]) : -1;
+                        uint32_t valid = __ballot_sync(0xffffffffu, mc != 0);
+                        while (valid) {
+                            const int l1 = __ffs(valid) - 1;
+                            valid &= valid - 1;
+                            int l2 = -1;
+                            if (valid) { l2 = __ffs(valid) - 1; valid &= valid - 1; }
+                            const int q1 = __shfl_sync(0xffffffffu, q, l1);
+                            const int q2 = __shfl_sync(0xffffffffu, q, l2 < 0 ? l1 : l2);
+                            const int n8 = lane >> 2, k4 = lane & 3;
+                            double fb = 0.0;
+                            if (n8 < 4) fb = (double)bval[16 * (jb + l1) + 4 * k4 + n8];
+                            else if (l2 >= 0) fb = (double)bval[16 * (jb + l2) + 4 * k4 + (n8 - 4)];
+                            double d0 = 0.0, d1 = 0.0;
+                            dmma(d0, d1, fa, fb);
+                            if (n8 < 4 && k4 < 2) {
+                                Acc* p = acc + 16 * (int64_t)q1 + 4 * n8 + 2 * k4;
+                                atomicAdd(p, (Acc)d0);
+                                atomicAdd(p + 1, (Acc)d1);
+                            } else if (n8 >= 4 && k4 >= 2 && l2 >= 0) {
+                                Acc* p = acc + 16 * (int64_t)q2 + 4 * (n8 - 4) + 2 * (k4 - 2);
+                                atomicAdd(p, (Acc)d0);
+                                atomicAdd(p + 1, (Acc)d1);
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        // ---- CUDA-core route: every pair of the sparse A tiles, flattened across the CTA
+        const int thr = sizeof(T) == 8 ? tc_thr : 17;
+        for (int64_t base = a0; base < a1; base += nt) {
+            const int64_t t = base + tid;
+            const bool v = t < a1;
+            const uint32_t ma = v ? c.amap[t] : 0u;
+            const bool sp = v && __popc(ma) < thr;
+            const int32_t K = sp ? c.aidx[t] : 0;
+            const int64_t b0 = sp ? c.bptr[K] : 0;
+            const int64_t len = sp ? c.bptr[K + 1] - b0 : 0;
+            int64_t incl = len;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                if (lane >= d) incl += y;
+            }
+            if (lane == 31) sh_tot[w] = incl;
+            __syncthreads();
+            if (tid == 0) {
+                int64_t acc2 = 0;
+                for (int k = 0; k < nw; ++k) { const int64_t x = sh_tot[k]; sh_tot[k] = acc2; acc2 += x; }
+                sh_tot[nw] = acc2;
+            }
+            __syncthreads();
+            sh_excl[tid] = sh_tot[w] + incl - len;
+            sh_b0[tid] = b0;
+            sh_ma[tid] = ma;
+            const int64_t total = sh_tot[nw];
+            __syncthreads();
+            const int nvalid = (int)min((int64_t)nt, a1 - base);
+            for (int64_t p = tid; p < total; p += nt) {
+                int lo = 0, hi = nvalid - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (sh_excl[mid] <= p) lo = mid; else hi = mid - 1;
+                }
+                const int64_t j = sh_b0[lo] + (p - sh_excl[lo]);
+                const uint32_t mc = bitmap_multiply(sh_ma[lo], c.bmap[j]);
+                if (!mc) continue;
+                const int q = bsearch_any(cidx, nC, c.bidx[j]);
+                Acc av[16], bv[16], prod[16];
+                TileIO<T>::load(aval + 16 * (base + lo), av);
+                TileIO<T>::load(bval + 16 * j, bv);
+                tile_mma(av, bv, prod);
+                Acc* dst = acc + 16 * (int64_t)q;
+                uint32_t bits = mc;
+                while (bits) {
+                    const int b = __ffs(bits) - 1;
+                    bits &= bits - 1;
+                    atomicAdd(dst + b, prod[b]);
+                }
+            }
+            __syncthreads();
+        }
+        __syncthreads();
+        for (int64_t e = tid; e < 16 * (int64_t)nC; e += nt) {  // +0.0 where the bit is clear (R2)
+            const int q = (int)(e >> 4), b = (int)(e & 15);
+            const bool bit = (cmap_g[c0 + q] >> b) & 1u;
+            const Acc v = acc[e];
+            cval[16 * c0 + e] = bit ? from_acc<T>(v) : from_acc<T>(Acc(0));
+        }
+        __syncthreads();
+    }
+}
+
 // ---------------------------------------------------------------- numeric: group kernel
 // One 4-lane group per C block row with <= GROUP_NC tiles, 8 rows per warp.  Lane r owns
 // row r of every C tile of its row (accumulators in registers).  The group walks its
@@ -876,6 +1033,7 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
                                                        const int32_t* __restrict__ cidx_g,
                                                        const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
                                                        int32_t* __restrict__ big, unsigned long long* __restrict__ nbig,
+                                                       int32_t* __restrict__ lng, unsigned long long* __restrict__ nlng,
                                                        int tc_thr) {
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -886,8 +1044,11 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
     if (I < BR) {
         c0 = cptr[I];
         nC = (int)(cptr[I + 1] - c0);
-        if (nC > GROUP_NC) {
-            if (r == 0) big[atomicAdd(nbig, 1ull)] = (int32_t)I;
+        if (nC > GROUP_NC) {  // <= CAP: warp kernel (deterministic); longer: block kernel
+            if (r == 0) {
+                if (nC <= CAP) big[atomicAdd(nbig, 1ull)] = (int32_t)I;
+                else lng[atomicAdd(nlng, 1ull)] = (int32_t)I;
+            }
             nC = 0;
         }
     }
@@ -1266,14 +1427,15 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     const int64_t BR = A->blc_row;
     if (BR == 0 || C->blc_num == 0) return AMGT_OK;
     SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
-    Scratch<int32_t> big;
+    Scratch<int32_t> big, lng;
     Scratch<unsigned long long> nbig;
     AMGT_TRY(big.init(a, BR));
-    AMGT_TRY(nbig.init(a, 1));
-    AMGT_CUDA(cudaMemsetAsync(nbig.p, 0, sizeof(unsigned long long), s));
+    AMGT_TRY(lng.init(a, BR));
+    AMGT_TRY(nbig.init(a, 2));
+    AMGT_CUDA(cudaMemsetAsync(nbig.p, 0, 2 * sizeof(unsigned long long), s));
     k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
         BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val, big.p,
-        nbig.p, g_tc_thr_spgemm);
+        nbig.p, lng.p, nbig.p + 1, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
     Scratch<Acc> gacc;
     if (sizeof(T) < sizeof(Acc)) AMGT_TRY(gacc.init(a, 16 * (size_t)C->blc_num));
@@ -1281,6 +1443,15 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         big.p, nbig.p, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map,
         (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
+    {
+        const size_t sm = (size_t)LONG_SMEM * sizeof(int32_t);
+        auto kern = k_numeric_long<T, Acc>;
+        AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        kern<<<(unsigned)num_sms() * 2, 256, sm, s>>>(lng.p, nbig.p + 1, c, (const T*)A->blc_val, (const T*)B->blc_val,
+                                                      C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
+                                                      sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
+        AMGT_LAUNCHED();
+    }
     return AMGT_OK;
 }
 
