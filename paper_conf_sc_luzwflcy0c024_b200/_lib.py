@@ -324,7 +324,7 @@ def rap(R: Mbsr, A: Mbsr, P: Mbsr, stream=None) -> Mbsr:
     return C
 
 
-def set_tc_threshold(spgemm: int = 10, spmv: int = 17):
+def set_tc_threshold(spgemm: int = 17, spmv: int = 17):
     _check(_L.amgt_set_tc_threshold(int(spgemm), int(spmv)))
 
 

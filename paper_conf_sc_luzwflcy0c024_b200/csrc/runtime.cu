@@ -83,8 +83,14 @@ int num_sms() {
     return n;
 }
 
-int g_tc_thr_spgemm = 10;  // paper: POPCOUNT(mapA) >= 10 (L157)
-int g_tc_thr_spmv = 17;    // see DESIGN.md: TC SpMV route off by default on B200 (DMMA = DFMA rate)
+// Tensor-core routing thresholds on POPCOUNT(mapA).  The paper uses 10 (L157); north_star asks
+// for the mma route only where it beats CUDA cores.  Measured on B200 (R9/R10;
+// tools/spgemm_bench.py): DMMA m8n8k4 issues at the FP64 FMA rate and both kernels are
+// memory/latency bound, so the route is slower at every threshold (FP64 SpGEMM +6..150%,
+// FP16 HMMA +0..15%, SpMV ~same) -> default 17 (CUDA cores); amgt_set_tc_threshold(10, 10)
+// restores the paper's routing.
+int g_tc_thr_spgemm = 17;
+int g_tc_thr_spmv = 17;
 
 // ------------------------------------------------------------------ scan
 // Block-wide exclusive scan: 1024 threads x 8 items = 8192 items per block.

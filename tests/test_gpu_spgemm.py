@@ -54,7 +54,7 @@ def test_spgemm_fp64(name, mk, thr):
     try:
         C, info = amgt.spgemm(amgt.from_csr(A), amgt.from_csr(B), info=True)
     finally:
-        amgt.set_tc_threshold(10, 17)
+        amgt.set_tc_threshold(17, 17)
     integer = name.endswith("_int") or name.startswith("cfg1") or name.startswith("27pt")
     _check_product(C, Co, Cabs, exact=integer)
     deg = np.diff(Bo.row_ptr)
@@ -169,7 +169,7 @@ def test_spgemm_tc_routes_integer_exact(prec, thr):
     try:
         C, info = amgt.spgemm(amgt.from_csr(A, prec=prec), amgt.from_csr(B, prec=prec), info=True)
     finally:
-        amgt.set_tc_threshold(10, 17)
+        amgt.set_tc_threshold(17, 17)
     if thr == 0:
         assert info["pairs_tc"] == info["pairs_nonzero"]
     assert_structure_equal(C, oracle.csr_to_mbsr(Co))
@@ -188,6 +188,6 @@ def test_spgemm_fp16_tc_tolerance(thr):
         M = amgt.from_csr(A, prec="f16")
         C = amgt.spgemm(M, M)
     finally:
-        amgt.set_tc_threshold(10, 17)
+        amgt.set_tc_threshold(17, 17)
     _, _, v = tile_values_to_csr_order(C)
     assert rel_2(v, Co.val) <= 5e-3

@@ -79,7 +79,7 @@ def test_spmv_tensor_core_route(thr):
             y = amgt.spmv(M, torch.from_numpy(x).cuda()).cpu().numpy()
             check_fp64_entrywise(y[:A.m], oracle.spmv(Ao, x), oracle.spmv_abs(Ao, x))
     finally:
-        amgt.set_tc_threshold(10, 17)
+        amgt.set_tc_threshold(17, 17)
 
 
 @pytest.mark.parametrize("prec,xdt", [("f32", torch.float32), ("f32", torch.float64), ("f16", torch.float32)])
