@@ -35,6 +35,102 @@ template <> __device__ __forceinline__ bool overflows<__half>(double v) {
     return fabs(v) > 65504.0 && fabs(v) < INFINITY && __hisinf(__double2half(v));
 }
 
+// Block rows with more than LONG_CONV CSR entries (power-law rows) are handled by one CTA
+// each (k_csr2mbsr_long): the 4-lane lockstep merge would serialise them.
+constexpr int64_t LONG_CONV = 4096;
+
+// One CTA per long block row: the row's tile columns are marked in a bitmap over the tile
+// columns (shared memory when it fits, else a per-CTA global slice); popcounts give the
+// count, an exclusive scan of word popcounts gives every tile's position (ascending J by
+// construction).  Entries are placed in parallel (distinct value slots); bitmap bits are
+// ORed with 32-bit atomics on the 16-bit map array.  Validation as in the group kernel.
+template <bool FILL, typename T>
+__global__ void __launch_bounds__(512) k_csr2mbsr_long(int64_t m, int64_t n, int64_t coff, const int64_t* __restrict__ rp,
+                                                       const int32_t* __restrict__ ci, const double* __restrict__ v,
+                                                       const int32_t* __restrict__ longl,
+                                                       const unsigned long long* __restrict__ nlong, int64_t W,
+                                                       uint32_t* __restrict__ gws, int64_t* __restrict__ cnt,
+                                                       const int64_t* __restrict__ bptr, int32_t* __restrict__ bidx,
+                                                       uint16_t* __restrict__ bmap, T* __restrict__ bval,
+                                                       uint32_t* __restrict__ flag) {
+    extern __shared__ __align__(16) uint32_t smw[];
+    __shared__ long long sh_sum[17];
+    uint32_t* bm = gws ? gws + (int64_t)blockIdx.x * 2 * W : smw;
+    uint32_t* pre = bm + W;
+    const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    const int64_t nl = (int64_t)*nlong;
+    uint32_t bad = 0, range = 0;
+    for (int64_t li = blockIdx.x; li < nl; li += gridDim.x) {
+        const int64_t I = longl[li];
+        for (int64_t i = tid; i < W; i += nt) bm[i] = 0;
+        __syncthreads();
+        for (int r = 0; r < 4 && 4 * I + r < m; ++r) {
+            const int64_t a = rp[4 * I + r], b = rp[4 * I + r + 1];
+            for (int64_t p = a + tid; p < b; p += nt) {
+                const int64_t col = ci[p] - coff;
+                if (!FILL && (col < 0 || col >= n || (p > a && ci[p] <= ci[p - 1]))) bad = 1;
+                if (col >= 0 && col < n) atomicOr(bm + (col >> 7), 1u << ((col >> 2) & 31));
+            }
+        }
+        __syncthreads();
+        const int64_t per = (W + nt - 1) / nt;
+        const int64_t w0 = min(W, per * (int64_t)tid), w1 = min(W, w0 + per);
+        long long sloc = 0;
+        for (int64_t i = w0; i < w1; ++i) sloc += __popc(bm[i]);
+        long long incl = sloc;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const long long y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        if (lane == 31) sh_sum[w] = incl;
+        __syncthreads();
+        if (tid == 0) {
+            long long acc = 0;
+            for (int k = 0; k < nw; ++k) { const long long x = sh_sum[k]; sh_sum[k] = acc; acc += x; }
+            sh_sum[nw] = acc;
+        }
+        __syncthreads();
+        if (!FILL) {
+            if (tid == 0) cnt[I] = sh_sum[nw];
+            __syncthreads();
+            continue;
+        }
+        const int64_t t0 = bptr[I];
+        long long run = sh_sum[w] + incl - sloc;
+        for (int64_t i = w0; i < w1; ++i) {  // tile columns in ascending order
+            pre[i] = (uint32_t)run;
+            uint32_t bits = bm[i];
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                bits &= bits - 1;
+                bidx[t0 + run] = (int32_t)(32 * i + b);
+                ++run;
+            }
+        }
+        const int64_t ntile = sh_sum[nw];
+        for (int64_t e2 = tid; e2 < 16 * ntile; e2 += nt) bval[16 * t0 + e2] = from_f64<T>(0.0);
+        for (int64_t tt = tid; tt < ntile; tt += nt) bmap[t0 + tt] = 0;
+        __syncthreads();
+        for (int r = 0; r < 4 && 4 * I + r < m; ++r) {
+            const int64_t a = rp[4 * I + r], b = rp[4 * I + r + 1];
+            for (int64_t p = a + tid; p < b; p += nt) {
+                const int64_t col = ci[p] - coff;
+                const int64_t J = col >> 2;
+                const int64_t q = t0 + pre[J >> 5] + __popc(bm[J >> 5] & ((1u << (J & 31)) - 1u));
+                const int bit = 4 * r + (int)(col & 3);
+                const double x = v[p];
+                bval[16 * q + bit] = from_f64<T>(x);
+                if (overflows<T>(x)) range = 1;
+                atomicOr(reinterpret_cast<unsigned int*>(bmap) + (q >> 1), (1u << bit) << (16 * (q & 1)));
+            }
+        }
+        __syncthreads();
+    }
+    if (bad) atomicOr(flag, FLAG_FORMAT);
+    if (range) atomicOr(flag, FLAG_RANGE);
+}
+
 // FILL = false: count tiles per block row into cnt[I] and validate the CSR.
 // FILL = true : write blc_idx / blc_map / blc_val at offsets bptr[I].
 template <bool FILL, typename T>
@@ -43,7 +139,8 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
                                                   const double* __restrict__ v, int64_t* __restrict__ cnt,
                                                   const int64_t* __restrict__ bptr, int32_t* __restrict__ bidx,
                                                   uint16_t* __restrict__ bmap, T* __restrict__ bval,
-                                                  uint32_t* __restrict__ flag) {
+                                                  uint32_t* __restrict__ flag, int32_t* __restrict__ longl,
+                                                  unsigned long long* __restrict__ nlong) {
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
     const int64_t I = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 8 + g;
     if ((((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 8 >= BR) return;  // whole warp idle
@@ -58,6 +155,15 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
             if (p > e || p < 0 || e > nnz) { bad = 1; e = p; }
             if (row == 0 && p != 0) bad = 1;
             if (row == m - 1 && e != nnz) bad = 1;
+        }
+    }
+    {  // block rows with many entries go to the CTA-per-row kernel (k_csr2mbsr_long)
+        int64_t bn = e - p;
+        bn += __shfl_xor_sync(0xffffffffu, bn, 1);
+        bn += __shfl_xor_sync(0xffffffffu, bn, 2);
+        if (bn > LONG_CONV) {
+            if (!FILL && r == 0) longl[atomicAdd(nlong, 1ull)] = (int32_t)I;
+            e = p;
         }
     }
     int64_t t = (FILL && active) ? bptr[I] : 0;
@@ -108,7 +214,7 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
             ++t;
         }
     }
-    if (!FILL && active && r == 0) cnt[I] = c;
+    if (!FILL && active && r == 0) cnt[I] = c;  // long rows: overwritten by k_csr2mbsr_long
     if (bad) atomicOr(flag, FLAG_FORMAT);
     if (range) atomicOr(flag, FLAG_RANGE);
 }
@@ -297,9 +403,28 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     const int64_t BR = ceil_div(m, 4);
     Scratch<int64_t> cnt;
     Scratch<uint32_t> flag;
+    Scratch<int32_t> longl;
+    Scratch<unsigned long long> nlong;
     AMGT_TRY(cnt.init(a, BR + 1));
     AMGT_TRY(flag.init(a, 1));
+    AMGT_TRY(longl.init(a, BR + 1));
+    AMGT_TRY(nlong.init(a, 1));
     AMGT_CUDA(cudaMemsetAsync(flag.p, 0, sizeof(uint32_t), s));
+    AMGT_CUDA(cudaMemsetAsync(nlong.p, 0, sizeof(unsigned long long), s));
+    // long-row kernel resources: bitmap + word prefix over the tile columns
+    const int64_t W = ceil_div(ceil_div(n, 4), 32);
+    const size_t lsm = (size_t)W * 2 * sizeof(uint32_t);
+    const bool lsmem = lsm <= 160 * 1024;
+    const unsigned LG = lsmem ? (unsigned)num_sms() : 16u;
+    Scratch<uint32_t> lws;
+    if (!lsmem) AMGT_TRY(lws.init(a, (size_t)LG * 2 * W));
+    auto launch_long = [&](auto kern, int64_t* cntp, const int64_t* bp, int32_t* bi, uint16_t* bmp, auto* bv) -> amgt_status {
+        if (lsmem) AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsm));
+        kern<<<LG, 512, lsmem ? lsm : 0, s>>>(m, n, coff, rp, ci, v, longl.p, nlong.p, W, lsmem ? nullptr : lws.p, cntp,
+                                               bp, bi, bmp, bv, flag.p);
+        AMGT_LAUNCHED();
+        return AMGT_OK;
+    };
     amgt_mbsr M{};
     const double bytes_in = nnz * 12.0 + (m + 1) * 8.0;
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 256);
@@ -307,8 +432,9 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
         TimerScope ts(TC_CSR2MBSR, bytes_in, s);
         if (BR > 0) {
             k_csr2mbsr<false, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, cnt.p, nullptr, nullptr,
-                                                             nullptr, nullptr, flag.p);
+                                                             nullptr, nullptr, flag.p, longl.p, nlong.p);
             AMGT_LAUNCHED();
+            AMGT_TRY(launch_long(k_csr2mbsr_long<false, double>, cnt.p, nullptr, nullptr, nullptr, (double*)nullptr));
         }
     }
     // blc_ptr lives in the output; scan the counts into it.
@@ -334,17 +460,28 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
             switch (prec) {
                 case AMGT_FP64:
                     k_csr2mbsr<true, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
-                                                                    M.blc_idx, M.blc_map, (double*)M.blc_val, flag.p);
+                                                                    M.blc_idx, M.blc_map, (double*)M.blc_val, flag.p,
+                                                                    longl.p, nlong.p);
+                    AMGT_LAUNCHED();
+                    AMGT_TRY(launch_long(k_csr2mbsr_long<true, double>, nullptr, M.blc_ptr, M.blc_idx, M.blc_map,
+                                         (double*)M.blc_val));
                     break;
                 case AMGT_FP32:
                     k_csr2mbsr<true, float><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
-                                                                   M.blc_idx, M.blc_map, (float*)M.blc_val, flag.p);
+                                                                   M.blc_idx, M.blc_map, (float*)M.blc_val, flag.p,
+                                                                   longl.p, nlong.p);
+                    AMGT_LAUNCHED();
+                    AMGT_TRY(launch_long(k_csr2mbsr_long<true, float>, nullptr, M.blc_ptr, M.blc_idx, M.blc_map,
+                                         (float*)M.blc_val));
                     break;
                 default:
                     k_csr2mbsr<true, __half><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
-                                                                    M.blc_idx, M.blc_map, (__half*)M.blc_val, flag.p);
+                                                                    M.blc_idx, M.blc_map, (__half*)M.blc_val, flag.p,
+                                                                    longl.p, nlong.p);
+                    AMGT_LAUNCHED();
+                    AMGT_TRY(launch_long(k_csr2mbsr_long<true, __half>, nullptr, M.blc_ptr, M.blc_idx, M.blc_map,
+                                         (__half*)M.blc_val));
             }
-            AMGT_LAUNCHED();
         }
     }
     if (prec == AMGT_FP16) {

@@ -68,18 +68,6 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
             const int32_t K = c.aidx[t];
             const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
             cub += b1 - b0;
-            if (!STATS) continue;
-            const uint32_t ma = c.amap[t];
-            const bool tc = __popc(ma) >= tc_thr;
-            for (int64_t j = b0; j < b1; ++j) {  // pair statistics (info only)
-                const uint32_t mb = c.bmap[j];
-                if (bitmap_multiply(ma, mb)) {
-                    ++pnz;
-                    ptc += tc;
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) sp += __popc((ma >> k) & 0x1111u) * __popc((mb >> (4 * k)) & 0xFu);
-                }
-            }
         }
         cub += __shfl_xor_sync(gm, cub, 1, 4);
         cub += __shfl_xor_sync(gm, cub, 2, 4);
@@ -98,6 +86,35 @@ __global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, un
     atomicAdd(&sh[11], sp);
     __syncthreads();
     if (threadIdx.x < 13 && sh[threadIdx.x]) atomicAdd(&stats[threadIdx.x], sh[threadIdx.x]);
+}
+
+// Pair statistics for amgt_spgemm_info (info only): one thread per A tile over its B row.
+__global__ void k_pair_stats(int64_t TA, SymCtx c, unsigned long long* __restrict__ stats, int tc_thr) {
+    unsigned long long pnz = 0, ptc = 0, sp = 0;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < TA; t += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t K = c.aidx[t];
+        const uint32_t ma = c.amap[t];
+        const bool tc = __popc(ma) >= tc_thr;
+        for (int64_t j = c.bptr[K]; j < c.bptr[K + 1]; ++j) {
+            const uint32_t mb = c.bmap[j];
+            if (bitmap_multiply(ma, mb)) {
+                ++pnz;
+                ptc += tc;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) sp += __popc((ma >> k) & 0x1111u) * __popc((mb >> (4 * k)) & 0xFu);
+            }
+        }
+    }
+    for (int d = 16; d; d >>= 1) {
+        pnz += __shfl_xor_sync(0xffffffffu, pnz, d);
+        ptc += __shfl_xor_sync(0xffffffffu, ptc, d);
+        sp += __shfl_xor_sync(0xffffffffu, sp, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(stats + 9, pnz);
+        atomicAdd(stats + 10, ptc);
+        atomicAdd(stats + 11, sp);
+    }
 }
 
 __global__ void k_bin_scatter(int64_t BR, const int64_t* __restrict__ bin_of, const unsigned long long* __restrict__ stats,
@@ -841,20 +858,65 @@ __device__ __forceinline__ int bsearch_any(const int32_t* idx, int n, int32_t J)
     return lo;
 }
 
+constexpr int LONG_CHUNK = 256;  // A tiles per work item of a long row
+
+// chunks per long row (entries past the device-side count are 0)
+__global__ void k_long_prep(int64_t cap, const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
+                            const int64_t* __restrict__ aptr, int64_t* __restrict__ nch) {
+    const int64_t n = (int64_t)*nrows_dev;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cap; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t c = 0;
+        if (i < n) {
+            const int64_t I = rows[i];
+            c = (aptr[I + 1] - aptr[I] + LONG_CHUNK - 1) / LONG_CHUNK;
+        }
+        nch[i] = c;
+    }
+}
+
+// zero (first == true) or finalise (+0.0 where the bit is clear, FP16 from the FP32
+// workspace) the long rows' values; one CTA per row
+template <typename T, typename Acc, bool FIRST>
+__global__ void k_long_rows_pass(const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
+                                 const int64_t* __restrict__ cptr, const uint16_t* __restrict__ cmap, T* __restrict__ cval,
+                                 Acc* __restrict__ gacc) {
+    const int64_t n = (int64_t)*nrows_dev;
+    for (int64_t i = blockIdx.x; i < n; i += gridDim.x) {
+        const int64_t I = rows[i];
+        const int64_t c0 = cptr[I], len = 16 * (cptr[I + 1] - c0);
+        Acc* acc = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
+        for (int64_t e = threadIdx.x; e < len; e += blockDim.x) {
+            if (FIRST) {
+                acc[e] = Acc(0);
+            } else {
+                const bool bit = (cmap[c0 + (e >> 4)] >> (e & 15)) & 1u;
+                cval[16 * c0 + e] = bit ? from_acc<T>(acc[e]) : from_acc<T>(Acc(0));
+            }
+        }
+    }
+}
+
 template <typename T, typename Acc>
 __global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict__ rows,
-                                                      const unsigned long long* __restrict__ nrows_dev, SymCtx c,
+                                                      const unsigned long long* __restrict__ nrows_dev,
+                                                      const int64_t* __restrict__ choff, int64_t cap, SymCtx c,
                                                       const T* __restrict__ aval, const T* __restrict__ bval,
                                                       const int64_t* __restrict__ cptr, const int32_t* __restrict__ cidx_g,
-                                                      const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
-                                                      Acc* __restrict__ gacc, int tc_thr) {
+                                                      T* __restrict__ cval, Acc* __restrict__ gacc, int tc_thr) {
     extern __shared__ __align__(16) int32_t sidx[];
     __shared__ int64_t sh_excl[256], sh_b0[256], sh_tot[9];
     __shared__ uint32_t sh_ma[256];
     const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
     const int64_t nrows = (int64_t)*nrows_dev;
-    for (int64_t rr = blockIdx.x; rr < nrows; rr += gridDim.x) {
-        const int64_t I = rows[rr];
+    const int64_t nitems = choff[cap];
+    for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
+        int64_t lo = 0, hi = nrows - 1;  // long row of this item: largest li with choff[li] <= item
+        while (lo < hi) {
+            const int64_t mid = (lo + hi + 1) >> 1;
+            if (choff[mid] <= item) lo = mid; else hi = mid - 1;
+        }
+        const int64_t I = rows[lo];
+        const int64_t k = item - choff[lo];
         const int64_t c0 = cptr[I];
         const int nC = (int)(cptr[I + 1] - c0);
         const bool in_smem = nC <= LONG_SMEM;
@@ -862,9 +924,8 @@ __global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict_
         if (in_smem)
             for (int q = tid; q < nC; q += nt) sidx[q] = cidx_g[c0 + q];
         Acc* acc = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
-        for (int64_t e = tid; e < 16 * (int64_t)nC; e += nt) acc[e] = Acc(0);
         __syncthreads();
-        const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+        const int64_t a0 = c.aptr[I] + k * LONG_CHUNK, a1 = min(c.aptr[I + 1], a0 + LONG_CHUNK);
         // ---- tensor-core route (FP64): warp-level DMMA per dense A tile
         if constexpr (sizeof(T) == 8) {
             int dense_seen = 0;
@@ -966,13 +1027,6 @@ __global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict_
                 }
             }
             __syncthreads();
-        }
-        __syncthreads();
-        for (int64_t e = tid; e < 16 * (int64_t)nC; e += nt) {  // +0.0 where the bit is clear (R2)
-            const int q = (int)(e >> 4), b = (int)(e & 15);
-            const bool bit = (cmap_g[c0 + q] >> b) & 1u;
-            const Acc v = acc[e];
-            cval[16 * c0 + e] = bit ? from_acc<T>(v) : from_acc<T>(Acc(0));
         }
         __syncthreads();
     }
@@ -1369,10 +1423,11 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     {
         TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
         if (BR > 0) {
-            if (info)
-                k_analyze<true><<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
-            else
-                k_analyze<false><<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+            k_analyze<false><<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+            if (info && A->blc_num > 0) {
+                AMGT_LAUNCHED();
+                k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats.p, g_tc_thr_spgemm);
+            }
             AMGT_LAUNCHED();
             k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats.p, cursor.p, rows.p);
             AMGT_LAUNCHED();
@@ -1443,13 +1498,24 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         big.p, nbig.p, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map,
         (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
-    {
+    {  // long rows: split into (row, 256-A-tile chunk) work items over a persistent grid
+        Scratch<int64_t> nch, choff;
+        AMGT_TRY(nch.init(a, BR));
+        AMGT_TRY(choff.init(a, BR + 1));
+        Acc* ga = sizeof(T) < sizeof(Acc) ? gacc.p : nullptr;
+        const unsigned G = (unsigned)num_sms() * 2;
+        k_long_prep<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, lng.p, nbig.p + 1, A->blc_ptr, nch.p);
+        AMGT_LAUNCHED();
+        AMGT_TRY(scan_exclusive(nch.p, choff.p, BR, a, s));
+        k_long_rows_pass<T, Acc, true><<<G, 256, 0, s>>>(lng.p, nbig.p + 1, C->blc_ptr, C->blc_map, (T*)C->blc_val, ga);
+        AMGT_LAUNCHED();
         const size_t sm = (size_t)LONG_SMEM * sizeof(int32_t);
         auto kern = k_numeric_long<T, Acc>;
         AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        kern<<<(unsigned)num_sms() * 2, 256, sm, s>>>(lng.p, nbig.p + 1, c, (const T*)A->blc_val, (const T*)B->blc_val,
-                                                      C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
-                                                      sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
+        kern<<<G, 256, sm, s>>>(lng.p, nbig.p + 1, choff.p, BR, c, (const T*)A->blc_val, (const T*)B->blc_val,
+                                C->blc_ptr, C->blc_idx, (T*)C->blc_val, ga, g_tc_thr_spgemm);
+        AMGT_LAUNCHED();
+        k_long_rows_pass<T, Acc, false><<<G, 256, 0, s>>>(lng.p, nbig.p + 1, C->blc_ptr, C->blc_map, (T*)C->blc_val, ga);
         AMGT_LAUNCHED();
     }
     return AMGT_OK;
