@@ -554,9 +554,16 @@ __global__ void k_numeric_rows_stats(int64_t BR, const int64_t* __restrict__ cpt
         const int64_t n = cptr[I + 1] - cptr[I];
         if (n == 0) ++e; else if (n <= 32) ++a; else ++b;
     }
-    atomicAdd(out, a);
-    atomicAdd(out + 1, b);
-    atomicAdd(out + 2, e);
+    for (int d = 16; d; d >>= 1) {
+        a += __shfl_xor_sync(0xffffffffu, a, d);
+        b += __shfl_xor_sync(0xffffffffu, b, d);
+        e += __shfl_xor_sync(0xffffffffu, e, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(out, a);
+        atomicAdd(out + 1, b);
+        atomicAdd(out + 2, e);
+    }
 }
 
 // ---------------------------------------------------------------- numeric
@@ -593,6 +600,43 @@ template <> struct TileIO<__half> {
                 v[8 * i + 2 * k + 1] = f.y;
             }
         }
+    }
+};
+
+template <typename T> struct RowIO;
+template <> struct RowIO<double> {
+    static __device__ __forceinline__ void load(const double* p, double (&v)[4]) {
+        const double2 a = __ldg(reinterpret_cast<const double2*>(p));
+        const double2 b = __ldg(reinterpret_cast<const double2*>(p) + 1);
+        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+    }
+    static __device__ __forceinline__ void store(double* p, const double (&v)[4]) {
+        reinterpret_cast<double2*>(p)[0] = make_double2(v[0], v[1]);
+        reinterpret_cast<double2*>(p)[1] = make_double2(v[2], v[3]);
+    }
+};
+template <> struct RowIO<float> {
+    static __device__ __forceinline__ void load(const float* p, float (&v)[4]) {
+        const float4 a = __ldg(reinterpret_cast<const float4*>(p));
+        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+    }
+    static __device__ __forceinline__ void store(float* p, const float (&v)[4]) {
+        *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    }
+};
+template <> struct RowIO<__half> {
+    static __device__ __forceinline__ void load(const __half* p, float (&v)[4]) {
+        const uint2 u = __ldg(reinterpret_cast<const uint2*>(p));
+        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
+        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
+        v[0] = lo.x; v[1] = lo.y; v[2] = hi.x; v[3] = hi.y;
+    }
+    static __device__ __forceinline__ void store(__half* p, const float (&v)[4]) {
+        __half2 a = __floats2half2_rn(v[0], v[1]), b = __floats2half2_rn(v[2], v[3]);
+        uint2 u;
+        u.x = *reinterpret_cast<uint32_t*>(&a);
+        u.y = *reinterpret_cast<uint32_t*>(&b);
+        *reinterpret_cast<uint2*>(p) = u;
     }
 };
 
@@ -847,188 +891,457 @@ __global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(const int32_t* __res
 // round-robin.  Accumulation: FP64/FP32 atomics into the output (FP32 workspace for FP16),
 // only at the bitmap positions a product can touch — the order of additions is not fixed,
 // so these rows are reproducible up to rounding (exact on integer/dyadic data).
-constexpr int LONG_SMEM = 16384;
+constexpr int LONG_SMEM = 8192;
 
-__device__ __forceinline__ int bsearch_any(const int32_t* idx, int n, int32_t J) {
+// last i with idx[i] <= J (idx ascending, idx[0] <= J)
+__device__ __forceinline__ int bsearch_le(const int32_t* idx, int n, int32_t J) {
     int lo = 0, hi = n - 1;
     while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (idx[mid] < J) lo = mid + 1; else hi = mid;
+        const int mid = (lo + hi + 1) >> 1;
+        if (idx[mid] <= J) lo = mid; else hi = mid - 1;
     }
     return lo;
 }
+// warp-cooperative: largest i in [lo, hi] with key(i) <= x (key nondecreasing, key(lo) <= x);
+// each round the 32 lanes probe 32 evenly spaced candidates
+template <typename F>
+__device__ __forceinline__ int64_t warp_search_le(int64_t lo, int64_t hi, int64_t x, F key, int lane) {
+    while (hi > lo) {
+        const int64_t step = (hi - lo + 31) / 32;
+        const int64_t pos = lo + (int64_t)(lane + 1) * step;
+        const bool ok = pos <= hi && key(pos) <= x;
+        const int cnt = __popc(__ballot_sync(0xffffffffu, ok));
+        lo += cnt * step;
+        hi = min(hi, lo + step - 1);
+    }
+    return lo;
+}
+template <typename Acc, typename T> __device__ __forceinline__ Acc to_acc(T v) { return (Acc)v; }
+template <> __device__ __forceinline__ float to_acc<float, __half>(__half v) { return __half2float(v); }
+__device__ __forceinline__ double fma_acc(double a, double b, double c) { return fma(a, b, c); }
+__device__ __forceinline__ float fma_acc(float a, float b, float c) { return fmaf(a, b, c); }
 
-constexpr int LONG_CHUNK = 256;  // A tiles per work item of a long row
+constexpr int LONG_PAIRS = 2048;  // (A tile, B tile) pairs per work item of a long row
+constexpr int LONG_CTILES = 512;  // C tiles per finalising work item of a long row
 
-// chunks per long row (entries past the device-side count are 0)
+// pairs per A tile of the long rows (the other entries were zeroed)
+__global__ void k_long_plen(const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
+                            SymCtx c, int64_t* __restrict__ plen) {
+    const int64_t n = (int64_t)*nrows_dev;
+    const int lane = threadIdx.x & 31;
+    for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; wi < n;
+         wi += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t I = rows[wi];
+        for (int64_t t = c.aptr[I] + lane; t < c.aptr[I + 1]; t += 32) {
+            const int32_t K = c.aidx[t];  // an empty B row still counts one (void) pair, so a
+            plen[t] = max(c.bptr[K + 1] - c.bptr[K], (int64_t)1);  // chunk spans <= LONG_PAIRS + 1 A tiles
+        }
+    }
+}
+
+// work items per long row: ceil(pairs / LONG_PAIRS) (entries past the device-side count are 0)
 __global__ void k_long_prep(int64_t cap, const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
-                            const int64_t* __restrict__ aptr, int64_t* __restrict__ nch) {
+                            const int64_t* __restrict__ aptr, const int64_t* __restrict__ pp,
+                            int64_t* __restrict__ nch) {
     const int64_t n = (int64_t)*nrows_dev;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cap; i += (int64_t)gridDim.x * blockDim.x) {
         int64_t c = 0;
         if (i < n) {
             const int64_t I = rows[i];
-            c = (aptr[I + 1] - aptr[I] + LONG_CHUNK - 1) / LONG_CHUNK;
+            c = (pp[aptr[I + 1]] - pp[aptr[I]] + LONG_PAIRS - 1) / LONG_PAIRS;
         }
         nch[i] = c;
     }
 }
 
-// zero (first == true) or finalise (+0.0 where the bit is clear, FP16 from the FP32
-// workspace) the long rows' values; one CTA per row
-template <typename T, typename Acc, bool FIRST>
-__global__ void k_long_rows_pass(const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
-                                 const int64_t* __restrict__ cptr, const uint16_t* __restrict__ cmap, T* __restrict__ cval,
-                                 Acc* __restrict__ gacc) {
+
+__global__ void k_long_prep_c(int64_t cap, const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
+                              const int64_t* __restrict__ cptr, int64_t* __restrict__ nch) {
     const int64_t n = (int64_t)*nrows_dev;
-    for (int64_t i = blockIdx.x; i < n; i += gridDim.x) {
-        const int64_t I = rows[i];
-        const int64_t c0 = cptr[I], len = 16 * (cptr[I + 1] - c0);
-        Acc* acc = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
-        for (int64_t e = threadIdx.x; e < len; e += blockDim.x) {
-            if (FIRST) {
-                acc[e] = Acc(0);
-            } else {
-                const bool bit = (cmap[c0 + (e >> 4)] >> (e & 15)) & 1u;
-                cval[16 * c0 + e] = bit ? from_acc<T>(acc[e]) : from_acc<T>(Acc(0));
-            }
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cap; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t c = 0;
+        if (i < n) {
+            const int64_t I = rows[i];
+            c = (cptr[I + 1] - cptr[I] + LONG_CTILES - 1) / LONG_CTILES;
         }
+        nch[i] = c;
     }
 }
 
+// FP16 rows accumulated with atomics: round the FP32 workspace, +0.0 where the bit is
+// clear; work items = (row, 512-C-tile chunk) over a persistent grid
 template <typename T, typename Acc>
-__global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict__ rows,
-                                                      const unsigned long long* __restrict__ nrows_dev,
-                                                      const int64_t* __restrict__ choff, int64_t cap, SymCtx c,
-                                                      const T* __restrict__ aval, const T* __restrict__ bval,
-                                                      const int64_t* __restrict__ cptr, const int32_t* __restrict__ cidx_g,
-                                                      T* __restrict__ cval, Acc* __restrict__ gacc, int tc_thr) {
-    extern __shared__ __align__(16) int32_t sidx[];
-    __shared__ int64_t sh_excl[256], sh_b0[256], sh_tot[9];
-    __shared__ uint32_t sh_ma[256];
-    const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+__global__ void k_long_rows_finalize(const int32_t* __restrict__ rows, const unsigned long long* __restrict__ nrows_dev,
+                                     const int64_t* __restrict__ choff, int64_t cap, const int64_t* __restrict__ cptr,
+                                     const uint16_t* __restrict__ cmap, T* __restrict__ cval, const Acc* __restrict__ gacc) {
     const int64_t nrows = (int64_t)*nrows_dev;
     const int64_t nitems = choff[cap];
     for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
-        int64_t lo = 0, hi = nrows - 1;  // long row of this item: largest li with choff[li] <= item
+        int64_t lo = 0, hi = nrows - 1;
         while (lo < hi) {
             const int64_t mid = (lo + hi + 1) >> 1;
             if (choff[mid] <= item) lo = mid; else hi = mid - 1;
         }
         const int64_t I = rows[lo];
-        const int64_t k = item - choff[lo];
+        const int64_t c0 = cptr[I], q0 = c0 + (item - choff[lo]) * LONG_CTILES;
+        const int64_t q1 = min(cptr[I + 1], q0 + LONG_CTILES);
+        for (int64_t e = 16 * q0 + threadIdx.x; e < 16 * q1; e += blockDim.x) {
+            const bool bit = (cmap[e >> 4] >> (e & 15)) & 1u;
+            cval[e] = bit ? from_acc<T>(gacc[e]) : from_acc<T>(Acc(0));
+        }
+    }
+}
+
+// Pair records written by pass 0 when the long rows' pair count fits their capacity: per
+// global pair index P, the C tile (global index, -1 if the product is empty), B tile, A
+// tile and bitmap product — pass 1 then streams them (k_long_flat) with no searches.
+struct PairRec {
+    int32_t* q;
+    int32_t* j;
+    int32_t* t;
+    uint16_t* m;
+    int64_t cap;
+};
+
+template <typename T, typename Acc, int PASS>
+__global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict__ rows,
+                                                      const unsigned long long* __restrict__ nrows_dev,
+                                                      const int64_t* __restrict__ choff, int64_t cap,
+                                                      const int64_t* __restrict__ pp, const int64_t* __restrict__ pp_total,
+                                                      unsigned long long* __restrict__ next, int32_t* __restrict__ cnt,
+                                                      PairRec rec, SymCtx c, const T* __restrict__ aval,
+                                                      const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                      const int32_t* __restrict__ cidx_g, T* __restrict__ cval,
+                                                      Acc* __restrict__ gacc) {
+    extern __shared__ __align__(16) int32_t sidx[];
+    __shared__ int32_t sh_pp[LONG_PAIRS + 2];  // pair prefix of the chunk's A tiles, relative to P0
+    __shared__ int64_t sh_d[6];
+    const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5;
+    const int hl = tid & 15, hsh = tid & 16;
+    const int64_t nrows = (int64_t)*nrows_dev;
+    const int64_t nitems = choff[cap];
+    const bool records = *pp_total <= rec.cap;
+    if (PASS == 1 && records) return;  // k_long_flat streams the records instead
+    Acc* stg = reinterpret_cast<Acc*>(sidx + LONG_SMEM) + w * (32 * 16);
+    for (;;) {
+        // item descriptor (warp 0): dequeue, then 32-ary searches for the row and for the
+        // chunk's A tiles (a few dependent loads instead of ~log2 n)
+        if (w == 0) {
+            int64_t item = 0;
+            if (lane == 0) item = (int64_t)atomicAdd(next, 1ull);
+            item = __shfl_sync(0xffffffffu, item, 0);
+            if (lane == 0) sh_d[0] = item;
+            if (item < nitems) {
+                const int64_t li = warp_search_le(0, nrows - 1, item, [&](int64_t m) { return choff[m]; }, lane);
+                const int64_t I = rows[li];
+                const int64_t ta0 = c.aptr[I], ta1 = c.aptr[I + 1];
+                const int64_t P0 = pp[ta0] + (item - choff[li]) * LONG_PAIRS, P1 = min(pp[ta1], P0 + LONG_PAIRS);
+                auto key = [&](int64_t m) { return pp[m]; };
+                const int64_t a0 = warp_search_le(ta0, ta1 - 1, P0, key, lane);
+                const int64_t a1 = warp_search_le(a0, ta1 - 1, P1 - 1, key, lane) + 1;
+                if (lane == 0) { sh_d[1] = I; sh_d[2] = a0; sh_d[3] = a1; sh_d[4] = P0; sh_d[5] = P1; }
+            }
+        }
+        __syncthreads();
+        if (sh_d[0] >= nitems) break;
+        const int64_t I = sh_d[1], a0 = sh_d[2], a1 = sh_d[3], P0 = sh_d[4], P1 = sh_d[5];
         const int64_t c0 = cptr[I];
         const int nC = (int)(cptr[I + 1] - c0);
-        const bool in_smem = nC <= LONG_SMEM;
-        const int32_t* cidx = in_smem ? sidx : cidx_g + c0;
-        if (in_smem)
-            for (int q = tid; q < nC; q += nt) sidx[q] = cidx_g[c0 + q];
         Acc* acc = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
+        int32_t* rcnt = cnt + c0;
+        // position search: every S-th C tile column in shared memory (S = 1 when the row
+        // fits), then a short forward scan over the global column list
+        const int S = (nC + LONG_SMEM - 1) / LONG_SMEM, ns = (nC + S - 1) / S;
+        for (int q = tid; q < ns; q += nt) sidx[q] = cidx_g[c0 + (int64_t)q * S];
+        const int na = (int)(a1 - a0);
+        for (int i = tid; i <= na; i += nt) sh_pp[i] = (int32_t)(pp[a0 + i] - P0);
         __syncthreads();
-        const int64_t a0 = c.aptr[I] + k * LONG_CHUNK, a1 = min(c.aptr[I + 1], a0 + LONG_CHUNK);
-        // ---- tensor-core route (FP64): warp-level DMMA per dense A tile
-        if constexpr (sizeof(T) == 8) {
-            int dense_seen = 0;
-            for (int64_t base = a0; base < a1; base += 32) {
-                const int64_t t = base + lane;
-                const uint32_t ma = t < a1 ? c.amap[t] : 0u;
-                uint32_t dense = __ballot_sync(0xffffffffu, t < a1 && __popc(ma) >= tc_thr);
-                while (dense) {
-                    const int src = __ffs(dense) - 1;
-                    dense &= dense - 1;
-                    if ((dense_seen++ % nw) != w) continue;  // round-robin over warps
-                    const int64_t ta = base + src;
-                    const uint32_t mA = __shfl_sync(0xffffffffu, ma, src);
-                    const int32_t K = c.aidx[ta];
-                    const double fa = (double)aval[16 * ta + 4 * ((lane >> 2) & 3) + (lane & 3)];
-                    const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
-                    for (int64_t jb = b0; jb < b1; jb += 32) {
-                        const int64_t j = jb + lane;
-                        const uint32_t mc = j < b1 ? bitmap_multiply(mA, c.bmap[j]) : 0u;
-                        const int q = mc ? bsearch_any(cidx, nC, c.bidx[j]) : -1;
-                        uint32_t valid = __ballot_sync(0xffffffffu, mc != 0);
-                        while (valid) {
-                            const int l1 = __ffs(valid) - 1;
-                            valid &= valid - 1;
-                            int l2 = -1;
-                            if (valid) { l2 = __ffs(valid) - 1; valid &= valid - 1; }
-                            const int q1 = __shfl_sync(0xffffffffu, q, l1);
-                            const int q2 = __shfl_sync(0xffffffffu, q, l2 < 0 ? l1 : l2);
-                            const int n8 = lane >> 2, k4 = lane & 3;
-                            double fb = 0.0;
-                            if (n8 < 4) fb = (double)bval[16 * (jb + l1) + 4 * k4 + n8];
-                            else if (l2 >= 0) fb = (double)bval[16 * (jb + l2) + 4 * k4 + (n8 - 4)];
-                            double d0 = 0.0, d1 = 0.0;
-                            dmma(d0, d1, fa, fb);
-                            if (n8 < 4 && k4 < 2) {
-                                Acc* p = acc + 16 * (int64_t)q1 + 4 * n8 + 2 * k4;
-                                atomicAdd(p, (Acc)d0);
-                                atomicAdd(p + 1, (Acc)d1);
-                            } else if (n8 >= 4 && k4 >= 2 && l2 >= 0) {
-                                Acc* p = acc + 16 * (int64_t)q2 + 4 * (n8 - 4) + 2 * (k4 - 2);
-                                atomicAdd(p, (Acc)d0);
-                                atomicAdd(p + 1, (Acc)d1);
+        auto find_q = [&](int32_t J) {
+            int q = bsearch_le(sidx, ns, J) * S;
+            if (S > 1) {
+                const int e1 = min(nC, q + S);
+                while (q + 1 < e1 && cidx_g[c0 + q] != J) ++q;
+            }
+            return q;
+        };
+        auto tile_of = [&](int64_t P) {  // last chunk A tile i with pp[a0 + i] <= P
+            const int32_t x = (int32_t)(P - P0);
+            int l = 0, h = na - 1;
+            while (l < h) {
+                const int m = (l + h + 1) >> 1;
+                if (sh_pp[m] <= x) l = m; else h = m - 1;
+            }
+            return l;
+        };
+        // ---- one pair per thread per round.  Pass 0: count the products per C tile, zero
+        // the tiles that will take REDs (a second product) and write the pair records.
+        // Pass 1 (no records): the B tile and the A rows in registers, every load in flight
+        // at once; each warp stages its 32 tile products in shared memory and writes them
+        // with 16-lane coalesced accesses, two products per instruction — a plain store
+        // (+0.0 at the clear bits) into a tile with one product, REDs at the bitmap
+        // positions otherwise.
+        for (int64_t pb = P0; pb < P1; pb += nt) {
+            const int64_t p = pb + tid;
+            uint32_t mc = 0u;
+            int q = 0;
+            if (p < P1) {
+                const int i = tile_of(p);
+                const int64_t t = a0 + i;
+                const uint32_t ma = c.amap[t];
+                const int32_t K = c.aidx[t];
+                const int64_t j = c.bptr[K] + (p - P0 - sh_pp[i]);
+                if (j < c.bptr[K + 1]) {
+                    mc = bitmap_multiply(ma, c.bmap[j]);
+                    if (mc) {
+                        q = find_q(c.bidx[j]);
+                        if constexpr (PASS == 0) {
+                            const int old = atomicAdd(rcnt + q, 1);
+                            if (old == 1) {
+                                uint4* v = reinterpret_cast<uint4*>(acc + 16 * (int64_t)q);
+#pragma unroll
+                                for (int e = 0; e < (int)sizeof(Acc); ++e) v[e] = make_uint4(0u, 0u, 0u, 0u);
+                            }
+                            if (records) {
+                                rec.j[p] = (int32_t)j;
+                                rec.t[p] = (int32_t)t;
+                                rec.m[p] = (uint16_t)mc;
+                            }
+                        } else {
+                            Acc bv[16];
+                            TileIO<T>::load(bval + 16 * j, bv);
+#pragma unroll
+                            for (int r = 0; r < 4; ++r) {
+                                Acc ar[4];
+                                RowIO<T>::load(aval + 16 * t + 4 * r, ar);
+#pragma unroll
+                                for (int col = 0; col < 4; ++col) {
+                                    Acc s = ar[0] * bv[col];
+                                    s = fma_acc(ar[1], bv[4 + col], s);
+                                    s = fma_acc(ar[2], bv[8 + col], s);
+                                    s = fma_acc(ar[3], bv[12 + col], s);
+                                    stg[lane * 16 + 4 * r + col] = s;
+                                }
                             }
                         }
                     }
                 }
+                if (PASS == 0 && records) rec.q[p] = mc ? (int32_t)(c0 + q) : -1;
+            }
+            if constexpr (PASS == 1) {
+                int single = 0;
+                if (mc) single = rcnt[q] == 1;
+                __syncwarp();
+                uint32_t todo = __ballot_sync(0xffffffffu, mc != 0u);
+                while (todo) {
+                    const int s1 = __ffs(todo) - 1;
+                    todo &= todo - 1;
+                    const int s2 = todo ? __ffs(todo) - 1 : -1;
+                    if (todo) todo &= todo - 1;
+                    const int src = hsh ? s2 : s1;
+                    const int sl = src < 0 ? s1 : src;
+                    const uint32_t ms = __shfl_sync(0xffffffffu, mc, sl);
+                    const int qs = __shfl_sync(0xffffffffu, q, sl);
+                    const int one = __shfl_sync(0xffffffffu, single, sl);
+                    if (src >= 0) {
+                        const bool bit = (ms >> hl) & 1u;
+                        const Acc val = stg[src * 16 + hl];
+                        Acc* dst = acc + 16 * (int64_t)qs + hl;
+                        if (one) *dst = bit ? val : Acc(0);
+                        else if (bit) atomicAdd(dst, val);
+                    }
+                }
+                __syncwarp();
             }
         }
-        // ---- CUDA-core route: every pair of the sparse A tiles, flattened across the CTA
-        const int thr = sizeof(T) == 8 ? tc_thr : 17;
-        for (int64_t base = a0; base < a1; base += nt) {
-            const int64_t t = base + tid;
-            const bool v = t < a1;
-            const uint32_t ma = v ? c.amap[t] : 0u;
-            const bool sp = v && __popc(ma) < thr;
-            const int32_t K = sp ? c.aidx[t] : 0;
-            const int64_t b0 = sp ? c.bptr[K] : 0;
-            const int64_t len = sp ? c.bptr[K + 1] - b0 : 0;
-            int64_t incl = len;
+        __syncthreads();  // sidx / sh_pp / sh_d are rewritten by the next item
+    }
+}
+
+// Pass 1 over the pair records: a half-warp per record, lane e = 4r+c computing entry
+// (r,c) of the tile product (A row r, B column c), FLAT_U records per half-warp in flight;
+// the tile is written with one coalesced 16-lane access — a plain store (+0.0 at the clear
+// bits) into a single-product tile, REDs at the bitmap positions otherwise.
+constexpr int FLAT_U = 4;
+
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(256, 4) k_long_flat(const int64_t* __restrict__ pp_total, PairRec rec,
+                                                   const int32_t* __restrict__ cnt, const T* __restrict__ aval,
+                                                   const T* __restrict__ bval, T* __restrict__ cval,
+                                                   Acc* __restrict__ gacc) {
+    const int64_t total = *pp_total;
+    if (total > rec.cap) return;  // no records: the item kernel's pass 1 ran
+    const int hl = threadIdx.x & 15, er = hl >> 2, ec = hl & 3;
+    Acc* acc = gacc ? gacc : reinterpret_cast<Acc*>(cval);
+    const int64_t hw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4;
+    const int64_t nhw = ((int64_t)gridDim.x * blockDim.x) >> 4;
+    for (int64_t base = hw * FLAT_U; base < total; base += nhw * FLAT_U) {
+        int32_t q[FLAT_U];
+        int64_t t[FLAT_U], j[FLAT_U];
+        uint32_t m[FLAT_U];
 #pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                if (lane >= d) incl += y;
-            }
-            if (lane == 31) sh_tot[w] = incl;
-            __syncthreads();
-            if (tid == 0) {
-                int64_t acc2 = 0;
-                for (int k = 0; k < nw; ++k) { const int64_t x = sh_tot[k]; sh_tot[k] = acc2; acc2 += x; }
-                sh_tot[nw] = acc2;
-            }
-            __syncthreads();
-            sh_excl[tid] = sh_tot[w] + incl - len;
-            sh_b0[tid] = b0;
-            sh_ma[tid] = ma;
-            const int64_t total = sh_tot[nw];
-            __syncthreads();
-            const int nvalid = (int)min((int64_t)nt, a1 - base);
-            for (int64_t p = tid; p < total; p += nt) {
-                int lo = 0, hi = nvalid - 1;
-                while (lo < hi) {
-                    const int mid = (lo + hi + 1) >> 1;
-                    if (sh_excl[mid] <= p) lo = mid; else hi = mid - 1;
-                }
-                const int64_t j = sh_b0[lo] + (p - sh_excl[lo]);
-                const uint32_t mc = bitmap_multiply(sh_ma[lo], c.bmap[j]);
-                if (!mc) continue;
-                const int q = bsearch_any(cidx, nC, c.bidx[j]);
-                Acc av[16], bv[16], prod[16];
-                TileIO<T>::load(aval + 16 * (base + lo), av);
-                TileIO<T>::load(bval + 16 * j, bv);
-                tile_mma(av, bv, prod);
-                Acc* dst = acc + 16 * (int64_t)q;
-                uint32_t bits = mc;
-                while (bits) {
-                    const int b = __ffs(bits) - 1;
-                    bits &= bits - 1;
-                    atomicAdd(dst + b, prod[b]);
-                }
-            }
-            __syncthreads();
+        for (int u = 0; u < FLAT_U; ++u) {
+            const int64_t p = base + u;
+            q[u] = p < total ? __ldg(rec.q + p) : -1;
+            j[u] = q[u] >= 0 ? __ldg(rec.j + p) : 0;
+            t[u] = q[u] >= 0 ? __ldg(rec.t + p) : 0;
+            m[u] = q[u] >= 0 ? __ldg(rec.m + p) : 0u;
         }
-        __syncthreads();
+        Acc bc[FLAT_U][4];
+        int one[FLAT_U];
+#pragma unroll
+        for (int u = 0; u < FLAT_U; ++u) {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) bc[u][k] = q[u] >= 0 ? to_acc<Acc>(bval[16 * j[u] + 4 * k + ec]) : Acc(0);
+            one[u] = q[u] >= 0 ? cnt[q[u]] == 1 : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < FLAT_U; ++u) {
+            if (q[u] < 0) continue;
+            Acc ar[4];
+            RowIO<T>::load(aval + 16 * t[u] + 4 * er, ar);
+            Acc sv = ar[0] * bc[u][0];
+            sv = fma_acc(ar[1], bc[u][1], sv);
+            sv = fma_acc(ar[2], bc[u][2], sv);
+            sv = fma_acc(ar[3], bc[u][3], sv);
+            const bool bit = (m[u] >> hl) & 1u;
+            Acc* dst = acc + 16 * (int64_t)q[u] + hl;
+            if (one[u]) *dst = bit ? sv : Acc(0);
+            else if (bit) atomicAdd(dst, sv);
+        }
+    }
+}
+
+// ---------------------------------------------------------------- numeric: mid rows
+// C block rows with CAP < nC <= MIDCAP tiles (most long rows of power-law matrices): one
+// warp per row, rows dequeued dynamically, no CTA barriers.  Two passes over the row's
+// pairs (one pair per lane per round): pass 0 counts the products landing on each C tile
+// (shared-memory atomics); pass 1 computes them, stages each warp's 32 tile products in
+// shared memory and writes them with 16-lane coalesced accesses — a plain store (+0.0 at
+// the clear bits) for a tile with one product, REDs at the bitmap positions into a
+// zeroed tile otherwise.  On power-law rows almost every C tile has one product, so the
+// row is written once, without atomics.  CUDA cores only.
+constexpr int MIDCAP = 512;
+constexpr int MID_WARPS = 8;
+
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(MID_WARPS * 32) k_numeric_mid(const int32_t* __restrict__ rows,
+                                                                const unsigned long long* __restrict__ nrows_dev,
+                                                                unsigned long long* __restrict__ cursor, SymCtx c,
+                                                                const T* __restrict__ aval, const T* __restrict__ bval,
+                                                                const int64_t* __restrict__ cptr,
+                                                                const int32_t* __restrict__ cidx_g, T* __restrict__ cval,
+                                                                Acc* __restrict__ gacc) {
+    extern __shared__ __align__(16) unsigned char mid_smem[];  // per warp: staging, columns, counts
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, hl = lane & 15, hsh = lane & 16;
+    const int64_t nrows = (int64_t)*nrows_dev;
+    Acc* stg = reinterpret_cast<Acc*>(mid_smem) + w * (32 * 16);
+    int32_t* sidx = reinterpret_cast<int32_t*>(mid_smem + MID_WARPS * 32 * 16 * sizeof(Acc)) + w * (2 * MIDCAP);
+    int32_t* scnt = sidx + MIDCAP;
+    for (;;) {
+        int64_t wi = 0;
+        if (lane == 0) wi = (int64_t)atomicAdd(cursor, 1ull);
+        wi = __shfl_sync(0xffffffffu, wi, 0);
+        if (wi >= nrows) break;
+        const int64_t I = rows[wi], c0 = cptr[I];
+        const int nC = (int)(cptr[I + 1] - c0);
+        for (int q = lane; q < nC; q += 32) {
+            sidx[q] = cidx_g[c0 + q];
+            scnt[q] = 0;
+        }
+        __syncwarp();
+        Acc* acc = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
+        const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+        for (int pass = 0; pass < 2; ++pass) {
+            if (pass == 1) {  // zero the tiles that take several products
+                for (int q = lane; q < nC; q += 32)
+                    if (scnt[q] > 1) {
+                        uint4* v = reinterpret_cast<uint4*>(acc + 16 * q);
+#pragma unroll
+                        for (int e = 0; e < (int)sizeof(Acc); ++e) v[e] = make_uint4(0u, 0u, 0u, 0u);
+                    }
+                __threadfence();
+                __syncwarp();
+            }
+            for (int64_t base = a0; base < a1; base += 32) {
+                const int64_t t = base + lane;
+                const bool v = t < a1;
+                const int32_t K = v ? c.aidx[t] : 0;
+                const uint32_t ma = v ? c.amap[t] : 0u;
+                const int64_t b0 = v ? c.bptr[K] : 0;
+                const int64_t len = v ? c.bptr[K + 1] - b0 : 0;
+                int64_t incl = len;
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                    if (lane >= d) incl += y;
+                }
+                const int64_t excl = incl - len;
+                const int64_t total = __shfl_sync(0xffffffffu, incl, 31);
+                for (int64_t p0 = 0; p0 < total; p0 += 32) {
+                    const int64_t p = p0 + lane;
+                    int lo = 0;  // owner lane: last with excl <= p
+#pragma unroll
+                    for (int step = 16; step; step >>= 1) {
+                        const int cand = lo + step;
+                        const int64_t e = __shfl_sync(0xffffffffu, excl, cand & 31);
+                        if (cand < 32 && e <= p) lo = cand;
+                    }
+                    const int64_t ob0 = __shfl_sync(0xffffffffu, b0, lo);
+                    const int64_t oex = __shfl_sync(0xffffffffu, excl, lo);
+                    const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
+                    uint32_t mc = 0u;
+                    int q = 0;
+                    if (p < total) {
+                        const int64_t j = ob0 + (p - oex);
+                        mc = bitmap_multiply(oma, c.bmap[j]);
+                        if (mc) {
+                            q = bsearch_row(sidx, nC, c.bidx[j]);
+                            if (pass == 0) {
+                                atomicAdd(scnt + q, 1);
+                            } else {
+                                Acc bv[16];
+                                TileIO<T>::load(bval + 16 * j, bv);
+                                const T* ap = aval + 16 * (base + lo);
+#pragma unroll
+                                for (int r = 0; r < 4; ++r) {
+                                    Acc ar[4];
+                                    RowIO<T>::load(ap + 4 * r, ar);
+#pragma unroll
+                                    for (int col = 0; col < 4; ++col) {
+                                        Acc s = ar[0] * bv[col];
+                                        s = fma_acc(ar[1], bv[4 + col], s);
+                                        s = fma_acc(ar[2], bv[8 + col], s);
+                                        s = fma_acc(ar[3], bv[12 + col], s);
+                                        stg[lane * 16 + 4 * r + col] = s;
+                                    }
+                                }
+                            }
+                        }
+                    }
+                    if (pass == 0) continue;
+                    __syncwarp();
+                    uint32_t todo = __ballot_sync(0xffffffffu, mc != 0u);
+                    while (todo) {  // two staged products per instruction
+                        const int s1 = __ffs(todo) - 1;
+                        todo &= todo - 1;
+                        const int s2 = todo ? __ffs(todo) - 1 : -1;
+                        if (todo) todo &= todo - 1;
+                        const int src = hsh ? s2 : s1;
+                        const uint32_t ms = __shfl_sync(0xffffffffu, mc, src < 0 ? s1 : src);
+                        const int qs = __shfl_sync(0xffffffffu, q, src < 0 ? s1 : src);
+                        if (src >= 0) {
+                            const bool bit = (ms >> hl) & 1u;
+                            const Acc val = stg[src * 16 + hl];
+                            Acc* dst = acc + 16 * (int64_t)qs + hl;
+                            if (scnt[qs] == 1) *dst = bit ? val : Acc(0);
+                            else if (bit) atomicAdd(dst, val);
+                        }
+                    }
+                    __syncwarp();
+                }
+            }
+            __syncwarp();
+        }
     }
 }
 
@@ -1044,42 +1357,6 @@ __global__ void __launch_bounds__(256) k_numeric_long(const int32_t* __restrict_
 // Rows with more tiles are appended to `big` for k_numeric.
 constexpr int GROUP_NC = 8;
 
-template <typename T> struct RowIO;
-template <> struct RowIO<double> {
-    static __device__ __forceinline__ void load(const double* p, double (&v)[4]) {
-        const double2 a = __ldg(reinterpret_cast<const double2*>(p));
-        const double2 b = __ldg(reinterpret_cast<const double2*>(p) + 1);
-        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
-    }
-    static __device__ __forceinline__ void store(double* p, const double (&v)[4]) {
-        reinterpret_cast<double2*>(p)[0] = make_double2(v[0], v[1]);
-        reinterpret_cast<double2*>(p)[1] = make_double2(v[2], v[3]);
-    }
-};
-template <> struct RowIO<float> {
-    static __device__ __forceinline__ void load(const float* p, float (&v)[4]) {
-        const float4 a = __ldg(reinterpret_cast<const float4*>(p));
-        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
-    }
-    static __device__ __forceinline__ void store(float* p, const float (&v)[4]) {
-        *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
-    }
-};
-template <> struct RowIO<__half> {
-    static __device__ __forceinline__ void load(const __half* p, float (&v)[4]) {
-        const uint2 u = __ldg(reinterpret_cast<const uint2*>(p));
-        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
-        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
-        v[0] = lo.x; v[1] = lo.y; v[2] = hi.x; v[3] = hi.y;
-    }
-    static __device__ __forceinline__ void store(__half* p, const float (&v)[4]) {
-        __half2 a = __floats2half2_rn(v[0], v[1]), b = __floats2half2_rn(v[2], v[3]);
-        uint2 u;
-        u.x = *reinterpret_cast<uint32_t*>(&a);
-        u.y = *reinterpret_cast<uint32_t*>(&b);
-        *reinterpret_cast<uint2*>(p) = u;
-    }
-};
 
 template <typename T, typename Acc>
 __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, const T* __restrict__ aval,
@@ -1088,6 +1365,7 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
                                                        const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
                                                        int32_t* __restrict__ big, unsigned long long* __restrict__ nbig,
                                                        int32_t* __restrict__ lng, unsigned long long* __restrict__ nlng,
+                                                       int32_t* __restrict__ mid, unsigned long long* __restrict__ nmid,
                                                        int tc_thr) {
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -1101,6 +1379,7 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
         if (nC > GROUP_NC) {  // <= CAP: warp kernel (deterministic); longer: block kernel
             if (r == 0) {
                 if (nC <= CAP) big[atomicAdd(nbig, 1ull)] = (int32_t)I;
+                else if (nC <= MIDCAP) mid[atomicAdd(nmid, 1ull)] = (int32_t)I;
                 else lng[atomicAdd(nlng, 1ull)] = (int32_t)I;
             }
             nC = 0;
@@ -1482,15 +1761,17 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     const int64_t BR = A->blc_row;
     if (BR == 0 || C->blc_num == 0) return AMGT_OK;
     SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
-    Scratch<int32_t> big, lng;
+    Scratch<int32_t> big, lng, mid;
     Scratch<unsigned long long> nbig;
     AMGT_TRY(big.init(a, BR));
     AMGT_TRY(lng.init(a, BR));
-    AMGT_TRY(nbig.init(a, 2));
-    AMGT_CUDA(cudaMemsetAsync(nbig.p, 0, 2 * sizeof(unsigned long long), s));
+    AMGT_TRY(mid.init(a, BR));
+    // [warp rows, long rows, long-row item cursor (pass 0), mid rows, mid-row cursor, long cursor (pass 1)]
+    AMGT_TRY(nbig.init(a, 6));
+    AMGT_CUDA(cudaMemsetAsync(nbig.p, 0, 6 * sizeof(unsigned long long), s));
     k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
         BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val, big.p,
-        nbig.p, lng.p, nbig.p + 1, g_tc_thr_spgemm);
+        nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
     Scratch<Acc> gacc;
     if (sizeof(T) < sizeof(Acc)) AMGT_TRY(gacc.init(a, 16 * (size_t)C->blc_num));
@@ -1498,25 +1779,78 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         big.p, nbig.p, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map,
         (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
+    {
+        int per_sm = 0;
+        const size_t msm = MID_WARPS * (32 * 16 * sizeof(Acc) + 2 * MIDCAP * sizeof(int32_t));
+        AMGT_CUDA(cudaFuncSetAttribute(k_numeric_mid<T, Acc>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)msm));
+        AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_numeric_mid<T, Acc>, MID_WARPS * 32, msm));
+        k_numeric_mid<T, Acc><<<(unsigned)num_sms() * (unsigned)max(per_sm, 1), MID_WARPS * 32, msm, s>>>(
+            mid.p, nbig.p + 3, nbig.p + 4, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx,
+            (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr);
+        AMGT_LAUNCHED();
+    }
     {  // long rows: split into (row, 256-A-tile chunk) work items over a persistent grid
         Scratch<int64_t> nch, choff;
         AMGT_TRY(nch.init(a, BR));
         AMGT_TRY(choff.init(a, BR + 1));
         Acc* ga = sizeof(T) < sizeof(Acc) ? gacc.p : nullptr;
         const unsigned G = (unsigned)num_sms() * 2;
-        k_long_prep<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, lng.p, nbig.p + 1, A->blc_ptr, nch.p);
+        Scratch<int64_t> plen, pp;  // pairs per A tile of the long rows -> exclusive prefix
+        AMGT_TRY(plen.init(a, A->blc_num));
+        AMGT_TRY(pp.init(a, A->blc_num + 1));
+        AMGT_CUDA(cudaMemsetAsync(plen.p, 0, A->blc_num * sizeof(int64_t), s));
+        k_long_plen<<<(unsigned)num_sms() * 8, 256, 0, s>>>(lng.p, nbig.p + 1, c, plen.p);
+        AMGT_LAUNCHED();
+        AMGT_TRY(scan_exclusive(plen.p, pp.p, A->blc_num, a, s));
+        k_long_prep<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, lng.p, nbig.p + 1, A->blc_ptr, pp.p, nch.p);
         AMGT_LAUNCHED();
         AMGT_TRY(scan_exclusive(nch.p, choff.p, BR, a, s));
-        k_long_rows_pass<T, Acc, true><<<G, 256, 0, s>>>(lng.p, nbig.p + 1, C->blc_ptr, C->blc_map, (T*)C->blc_val, ga);
+        Scratch<int32_t> cnt;  // products per C tile (long rows)
+        AMGT_TRY(cnt.init(a, C->blc_num));
+        AMGT_CUDA(cudaMemsetAsync(cnt.p, 0, C->blc_num * sizeof(int32_t), s));
+        // pair records: capacity for power-law rows (about one product per C tile); past it
+        // (or past int32 indices) pass 1 re-derives the pairs instead
+        const bool fits32 = C->blc_num < INT32_MAX && B->blc_num < INT32_MAX && A->blc_num < INT32_MAX;
+        PairRec rec{nullptr, nullptr, nullptr, nullptr, fits32 ? 2 * C->blc_num + A->blc_num : -1};
+        Scratch<int32_t> rq, rj, rt;
+        Scratch<uint16_t> rm;
+        if (fits32) {
+            AMGT_TRY(rq.init(a, rec.cap));
+            AMGT_TRY(rj.init(a, rec.cap));
+            AMGT_TRY(rt.init(a, rec.cap));
+            AMGT_TRY(rm.init(a, rec.cap));
+            rec.q = rq.p; rec.j = rj.p; rec.t = rt.p; rec.m = rm.p;
+        }
+        const int64_t* pp_total = pp.p + A->blc_num;
+        for (int pass = 0; pass < 2; ++pass) {
+            // column samples (+ per-warp product staging in pass 1)
+            const size_t sm = (size_t)LONG_SMEM * sizeof(int32_t) + (pass ? 8 * 32 * 16 * sizeof(Acc) : 0);
+            auto kern = pass == 0 ? k_numeric_long<T, Acc, 0> : k_numeric_long<T, Acc, 1>;
+            AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+            int per_sm = 0;  // persistent grid: exactly the resident CTAs
+            AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, sm));
+            kern<<<(unsigned)num_sms() * (unsigned)max(per_sm, 1), 256, sm, s>>>(
+                lng.p, nbig.p + 1, choff.p, BR, pp.p, pp_total, nbig.p + 2 + 3 * pass, cnt.p, rec, c,
+                (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, (T*)C->blc_val, ga);
+            AMGT_LAUNCHED();
+        }
+        k_long_flat<T, Acc><<<(unsigned)num_sms() * 8, 256, 0, s>>>(pp_total, rec, cnt.p, (const T*)A->blc_val,
+                                                                  (const T*)B->blc_val, (T*)C->blc_val, ga);
         AMGT_LAUNCHED();
-        const size_t sm = (size_t)LONG_SMEM * sizeof(int32_t);
-        auto kern = k_numeric_long<T, Acc>;
-        AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        kern<<<G, 256, sm, s>>>(lng.p, nbig.p + 1, choff.p, BR, c, (const T*)A->blc_val, (const T*)B->blc_val,
-                                C->blc_ptr, C->blc_idx, (T*)C->blc_val, ga, g_tc_thr_spgemm);
-        AMGT_LAUNCHED();
-        k_long_rows_pass<T, Acc, false><<<G, 256, 0, s>>>(lng.p, nbig.p + 1, C->blc_ptr, C->blc_map, (T*)C->blc_val, ga);
-        AMGT_LAUNCHED();
+        if (ga) {  // FP16: round the FP32 workspace (FP64/FP32 accumulate in place: bits-only atomics)
+            Scratch<int64_t> ccoff;
+            AMGT_TRY(ccoff.init(a, BR + 1));
+            const int32_t* lists[2] = {lng.p, mid.p};
+            const unsigned long long* counts[2] = {nbig.p + 1, nbig.p + 3};
+            for (int l = 0; l < 2; ++l) {
+                k_long_prep_c<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, lists[l], counts[l], C->blc_ptr, nch.p);
+                AMGT_LAUNCHED();
+                AMGT_TRY(scan_exclusive(nch.p, ccoff.p, BR, a, s));
+                k_long_rows_finalize<T, Acc><<<G, 256, 0, s>>>(lists[l], counts[l], ccoff.p, BR, C->blc_ptr,
+                                                                C->blc_map, (T*)C->blc_val, ga);
+                AMGT_LAUNCHED();
+            }
+        }
     }
     return AMGT_OK;
 }

@@ -82,6 +82,35 @@ def test_spgemm_info_bins_and_long_rows():
     assert sum(info["bin_rows"][2:]) > 0 and info["numeric_rows"][1] > 0
 
 
+LONG = [
+    # power-law rows with > 512 C tiles, about one product per C tile: pair-record path
+    ("long_records", lambda: (gen.irregular_block_sparse(1 << 13, seed=9),) * 2),
+    # long rows with ~500 products per C tile: past the record capacity, pass 1 re-derives
+    ("long_fallback", lambda: (gen.random_csr(32, 8192, 0.3, 31), gen.random_csr(8192, 4096, 0.02, 32))),
+]
+
+
+@pytest.mark.parametrize("prec", ["f64", "f32", "f16"])
+@pytest.mark.parametrize("name,mk", LONG, ids=[p[0] for p in LONG])
+def test_spgemm_long_rows(name, mk, prec):
+    """Rows with > 512 C tiles (two-pass long-row kernels) and 32 < nC <= 512 (warp kernel)."""
+    amgt = _amgt()
+    A, B = mk()
+    Ao, Bo = oracle.as_csr(A), oracle.as_csr(B)
+    Co, Cabs = oracle.spgemm(Ao, Bo, with_abs=True)
+    C = amgt.spgemm(amgt.from_csr(A, prec=prec), amgt.from_csr(B, prec=prec))
+    assert np.diff(C.blc_ptr.cpu().numpy()).max() > 512
+    if prec == "f64":
+        _check_product(C, Co, Cabs)
+        return
+    assert_structure_equal(C, oracle.csr_to_mbsr(Co))
+    _, _, v = tile_values_to_csr_order(C)
+    if prec == "f32":
+        assert rel_inf(v, Co.val) <= 1e-5
+    else:
+        assert rel_2(v, Co.val) <= 5e-3
+
+
 @pytest.mark.parametrize("prec", ["f32", "f16"])
 def test_spgemm_low_precision(prec):
     amgt = _amgt()
