@@ -58,6 +58,11 @@ class ClockSampler:
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            # nvidia-smi's start-up (driver queries) stalls CUDA calls of this process for
+            # milliseconds: wait for its first sample so that happens before the timed region
+            t0 = time.time()
+            while not self.lines and time.time() - t0 < 5.0:
+                time.sleep(0.02)
         except Exception:
             self.proc = None
         return self
@@ -131,11 +136,14 @@ def byte_model(sz, cycles):
         num += 2 * TP * (16 * s[k] + 6)  # R = P^T (tile transpose: read + write)
     out["spgemm_symbolic"], out["spgemm_numeric"] = sym, num
     out["mbsr2csr"] = tb(lev[-1]["T"], s[-1]) + lev[-1]["m"] * 20
-    # a9/a10: per cycle 3 SpMV(A_k) + R_k + P_k per level, 1 final residual SpMV(A_1)
+    # a9/a10: per cycle 3 SpMV(A_k) + R_k + P_k per level.  The residual reported after each
+    # cycle (L308) comes out of the next cycle's first pre-smoothing pass over A_1 (same x),
+    # so A_1 is read 3 times per cycle plus once for the last residual (L > 1; a one-level
+    # hierarchy reads it once per cycle plus the initial residual)
     def spmv_b(T, BR, BC, sk, xs, ys):
         return tb(T, sk) + (BR + 1) * 8 + 4 * BC * xs + 4 * BR * ys
     sp1 = spmv_b(lev[0]["T"], lev[0]["BR"], lev[0]["BC"], s[0], vs[0], vs[0])
-    l1 = sp1 * (3 * (L > 1) + 1)
+    l1 = sp1 * (3 if L > 1 else 1)
     other, vec = 0, 0
     for k in range(L - 1):
         if k > 0:
@@ -147,7 +155,8 @@ def byte_model(sz, cycles):
         # vector operands of the Alg. 2 steps beyond the SpMV's own x/y: each Jacobi sweep
         # reads b and D^-1, the residual reads b, the correction reads x (6 vectors)
         vec += 6 * 4 * lev[k]["BR"] * vs[k]
-    vec += lev[-1]["m"] ** 2 * 8 + 2 * 4 * lev[0]["BR"] * 8  # coarse solve; final residual b + norm
+    # coarse solve; residual b + norm read; the fused pre-smoothing pass also writes r
+    vec += lev[-1]["m"] ** 2 * 8 + (3 if L > 1 else 2) * 4 * lev[0]["BR"] * 8
     out["spmv_l1"] = l1 * cycles + sp1
     out["spmv"] = other * cycles
     out["vector"] = vec * cycles

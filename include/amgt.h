@@ -65,7 +65,7 @@ typedef struct {
  *                        +0.0 where the bit is clear (R2); element type given by `prec`
  * Tiles are 4x4 because tensor-core shapes are multiples of 4 (L116).
  * blc_row = ceil(m/4), blc_col = ceil(n/4); bits outside m x n are never set (R25).
- * `own` and `aux` are library-managed (zero-initialise the struct before first use).
+ * `own`, `aux` and `row_max` are library-managed (zero-initialise the struct before first use).
  */
 typedef struct {
     int64_t m, n;
@@ -77,6 +77,9 @@ typedef struct {
     amgt_prec prec;
     uint32_t own;      /* bit0: structure arrays owned, bit1: values owned */
     void* aux;         /* library-owned analysis (SpMV plan); NULL until amgt_spmv_analyze */
+    int64_t row_max;   /* library-managed: max tiles in a block row when known (set by
+                          amgt_spgemm_symbolic, kept by cast), 0 = unknown; lets the numeric
+                          SpGEMM skip the kernels for row classes that do not occur */
 } amgt_mbsr;
 
 const char* amgt_last_error(void);
@@ -225,6 +228,16 @@ amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* 
 #define AMGT_EPI_ACCUM 3
 amgt_status amgt_spmv_fused(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec, int mode,
                             const void* b, const void* dinv, double omega, void* stream);
+
+/* Weighted Jacobi sweep that also returns the residual of its input (NEXT-1 fusion):
+ *   r = b - A x,   y = x + omega * dinv .* r        (one pass over A)
+ * After a V-cycle, r is the Alg. 2 residual reported per cycle (L308), so the first
+ * pre-smoothing sweep of the next cycle delivers it without a separate SpMV.  x, y, r, b,
+ * dinv share one precision (FP64 or FP32), length 4*blc_row; x, y, r distinct; A square.
+ * Mode value AMGT_EPI_JACOBI_RES is internal to this call (not accepted by amgt_spmv_fused). */
+#define AMGT_EPI_JACOBI_RES 4
+amgt_status amgt_spmv_fused_r(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec,
+                              const void* b, const void* dinv, double omega, void* r, void* stream);
 
 /* Row-range variant used by the distributed SpMV to overlap the halo exchange: only
  * block rows [blk_begin, blk_end) are computed; y indexed by local row; for Jacobi, x_i is

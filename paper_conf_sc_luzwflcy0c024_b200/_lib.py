@@ -38,7 +38,8 @@ class c_mbsr(ctypes.Structure):
     _fields_ = [("m", ctypes.c_int64), ("n", ctypes.c_int64), ("blc_row", ctypes.c_int64),
                 ("blc_col", ctypes.c_int64), ("blc_num", ctypes.c_int64), ("blc_ptr", ctypes.c_void_p),
                 ("blc_idx", ctypes.c_void_p), ("blc_map", ctypes.c_void_p), ("blc_val", ctypes.c_void_p),
-                ("prec", ctypes.c_int), ("own", ctypes.c_uint32), ("aux", ctypes.c_void_p)]
+                ("prec", ctypes.c_int), ("own", ctypes.c_uint32), ("aux", ctypes.c_void_p),
+                ("row_max", ctypes.c_int64)]
 
 
 _ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
@@ -104,6 +105,7 @@ _sigs = {
     "amgt_spmv_get_stats": (_int, [_P(c_mbsr), _P(c_spmv_stats)]),
     "amgt_spmv": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _vp]),
     "amgt_spmv_fused": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _int, _vp, _vp, ctypes.c_double, _vp]),
+    "amgt_spmv_fused_r": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _vp, _vp, ctypes.c_double, _vp, _vp]),
     "amgt_hierarchy_create": (_int, [_P(c_mbsr), _P(_P(c_mbsr)), _int, _P(c_vcycle_opts), _P(c_allocator), _vp,
                                      _P(_vp)]),
     "amgt_hierarchy_level": (_int, [_vp, _int, _P(_P(c_mbsr)), _P(_P(c_mbsr)), _P(_P(c_mbsr))]),
@@ -355,6 +357,15 @@ def spmv_fused(A: Mbsr, x: torch.Tensor, y: torch.Tensor, mode: str, b: torch.Te
     _check(_L.amgt_spmv_fused(ctypes.byref(A.c), x.data_ptr(), xp, y.data_ptr(), yp, EPI[mode],
                               b.data_ptr() if b is not None else None, dinv.data_ptr() if dinv is not None else None,
                               float(omega), _stream(stream)))
+    return y
+
+
+def spmv_jacobi_res(A: Mbsr, x: torch.Tensor, y: torch.Tensor, b: torch.Tensor, dinv: torch.Tensor,
+                    r: torch.Tensor, omega: float = 2.0 / 3.0, stream=None) -> torch.Tensor:
+    """amgt_spmv_fused_r: r = b - A x and y = x + omega dinv .* r in one pass over A."""
+    p = {torch.float64: FP64, torch.float32: FP32}[x.dtype]
+    _check(_L.amgt_spmv_fused_r(ctypes.byref(A.c), x.data_ptr(), p, y.data_ptr(), p, b.data_ptr(), dinv.data_ptr(),
+                                float(omega), r.data_ptr(), _stream(stream)))
     return y
 
 

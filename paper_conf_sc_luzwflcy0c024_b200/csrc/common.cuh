@@ -167,6 +167,7 @@ struct EpiArgs {
     const void* xs;
     double omega;
     int64_t I0, I1;  // block-row range [I0, I1); I1 < 0 = all rows
+    void* r = nullptr;  // AMGT_EPI_JACOBI_RES: residual output (y's precision)
 };
 
 extern int g_tc_thr_spgemm;

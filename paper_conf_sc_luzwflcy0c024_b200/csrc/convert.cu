@@ -361,6 +361,7 @@ amgt_status mbsr_alloc(amgt_mbsr* M, int64_t m, int64_t n, int64_t T, amgt_prec 
     M->prec = prec;
     M->aux = nullptr;
     M->own = 0;
+    M->row_max = 0;
     if (structure) {
         M->blc_ptr = existing_ptr ? existing_ptr : (int64_t*)a.get((M->blc_row + 1) * sizeof(int64_t));
         M->blc_idx = (int32_t*)a.get(T * sizeof(int32_t));

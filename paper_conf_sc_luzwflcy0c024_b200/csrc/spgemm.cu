@@ -548,6 +548,14 @@ __global__ void __launch_bounds__(512) k_sym_dense(int64_t nrows, const int32_t*
     }
 }
 
+__global__ void k_max_rows(int64_t BR, const int64_t* __restrict__ nrow, unsigned long long* __restrict__ out) {
+    unsigned long long m = 0;
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x)
+        m = max(m, (unsigned long long)nrow[I]);
+    for (int d = 16; d; d >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, d));
+    if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
+}
+
 __global__ void k_numeric_rows_stats(int64_t BR, const int64_t* __restrict__ cptr, unsigned long long* __restrict__ out) {
     unsigned long long a = 0, b = 0, e = 0;
     for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
@@ -1720,11 +1728,21 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
         }
         AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s));
+        Scratch<unsigned long long> rmax;  // longest C block row (numeric skips absent row classes)
+        AMGT_TRY(rmax.init(a, 1));
+        AMGT_CUDA(cudaMemsetAsync(rmax.p, 0, sizeof(unsigned long long), s));
+        if (BR > 0) {
+            k_max_rows<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, nnz_row.p, rmax.p);
+            AMGT_LAUNCHED();
+        }
         int64_t TC = 0;
+        unsigned long long hmax = 0;
         AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax.p, sizeof(hmax), cudaMemcpyDeviceToHost, s));
         AMGT_CUDA(cudaStreamSynchronize(s));  // sync 2: C tile count (L153)
         amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
         if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+        C.row_max = (int64_t)hmax;
         if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
         if (BR > 0) {
             st = run_bins<2>(cnt, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
@@ -1773,12 +1791,16 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val, big.p,
         nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, g_tc_thr_spgemm);
     AMGT_LAUNCHED();
-    Scratch<Acc> gacc;
-    if (sizeof(T) < sizeof(Acc)) AMGT_TRY(gacc.init(a, 16 * (size_t)C->blc_num));
+    // row classes present (C->row_max from symbolic; 0 = unknown: launch everything)
+    const int64_t rmax = C->row_max > 0 ? C->row_max : INT64_MAX;
+    if (rmax <= GROUP_NC) return AMGT_OK;
     k_numeric<T, Acc><<<(unsigned)num_sms() * 4, NUM_WARPS * 32, 0, s>>>(
         big.p, nbig.p, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map,
-        (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr, g_tc_thr_spgemm);
+        (T*)C->blc_val, nullptr, g_tc_thr_spgemm);  // rows <= CAP accumulate in shared memory
     AMGT_LAUNCHED();
+    if (rmax <= CAP) return AMGT_OK;
+    Scratch<Acc> gacc;  // FP16: FP32 accumulation workspace of the atomically accumulated rows
+    if (sizeof(T) < sizeof(Acc)) AMGT_TRY(gacc.init(a, 16 * (size_t)C->blc_num));
     {
         int per_sm = 0;
         const size_t msm = MID_WARPS * (32 * 16 * sizeof(Acc) + 2 * MIDCAP * sizeof(int32_t));
@@ -1789,12 +1811,12 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
             (T*)C->blc_val, sizeof(T) < sizeof(Acc) ? gacc.p : nullptr);
         AMGT_LAUNCHED();
     }
-    {  // long rows: split into (row, 256-A-tile chunk) work items over a persistent grid
+    const bool has_long = rmax > MIDCAP;
+    if (has_long) {  // long rows: (row, LONG_PAIRS-pair chunk) work items over a persistent grid
         Scratch<int64_t> nch, choff;
         AMGT_TRY(nch.init(a, BR));
         AMGT_TRY(choff.init(a, BR + 1));
         Acc* ga = sizeof(T) < sizeof(Acc) ? gacc.p : nullptr;
-        const unsigned G = (unsigned)num_sms() * 2;
         Scratch<int64_t> plen, pp;  // pairs per A tile of the long rows -> exclusive prefix
         AMGT_TRY(plen.init(a, A->blc_num));
         AMGT_TRY(pp.init(a, A->blc_num + 1));
@@ -1837,19 +1859,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         k_long_flat<T, Acc><<<(unsigned)num_sms() * 8, 256, 0, s>>>(pp_total, rec, cnt.p, (const T*)A->blc_val,
                                                                   (const T*)B->blc_val, (T*)C->blc_val, ga);
         AMGT_LAUNCHED();
-        if (ga) {  // FP16: round the FP32 workspace (FP64/FP32 accumulate in place: bits-only atomics)
-            Scratch<int64_t> ccoff;
-            AMGT_TRY(ccoff.init(a, BR + 1));
-            const int32_t* lists[2] = {lng.p, mid.p};
-            const unsigned long long* counts[2] = {nbig.p + 1, nbig.p + 3};
-            for (int l = 0; l < 2; ++l) {
-                k_long_prep_c<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, lists[l], counts[l], C->blc_ptr, nch.p);
-                AMGT_LAUNCHED();
-                AMGT_TRY(scan_exclusive(nch.p, ccoff.p, BR, a, s));
-                k_long_rows_finalize<T, Acc><<<G, 256, 0, s>>>(lists[l], counts[l], ccoff.p, BR, C->blc_ptr,
-                                                                C->blc_map, (T*)C->blc_val, ga);
-                AMGT_LAUNCHED();
-            }
+    }
+    if (sizeof(T) < sizeof(Acc)) {  // FP16: round the FP32 workspace (FP64/FP32 accumulate in place)
+        Scratch<int64_t> nch, ccoff;
+        AMGT_TRY(nch.init(a, BR));
+        AMGT_TRY(ccoff.init(a, BR + 1));
+        const int32_t* lists[2] = {mid.p, lng.p};
+        const unsigned long long* counts[2] = {nbig.p + 3, nbig.p + 1};
+        for (int l = 0; l < (has_long ? 2 : 1); ++l) {
+            k_long_prep_c<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, lists[l], counts[l], C->blc_ptr, nch.p);
+            AMGT_LAUNCHED();
+            AMGT_TRY(scan_exclusive(nch.p, ccoff.p, BR, a, s));
+            k_long_rows_finalize<T, Acc><<<(unsigned)num_sms() * 2, 256, 0, s>>>(
+                lists[l], counts[l], ccoff.p, BR, C->blc_ptr, C->blc_map, (T*)C->blc_val, gacc.p);
+            AMGT_LAUNCHED();
         }
     }
     return AMGT_OK;

@@ -189,36 +189,40 @@ __global__ void __launch_bounds__(256) k_spmv_lanerow(int64_t I0, int64_t BR, co
                                                       const int32_t* __restrict__ bidx,
                                                       const uint16_t* __restrict__ bmap,
                                                       const MatT* __restrict__ bval, const XT* __restrict__ x,
-                                                      const Epi<XT, YT, MODE> epi) {
+                                                      const Epi<XT, YT, MODE> epi, bool vec) {
     using Acc = typename AccOf<MatT>::type;
     const int64_t I = I0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (I >= BR) return;
     const int64_t t0 = __ldg(bptr + I), t1 = __ldg(bptr + I + 1);
     typename Epi<XT, YT, MODE>::Pre pre[4];
+    if (vec) {
+        epi.prefetch4(4 * I, pre);
+    } else {
 #pragma unroll
-    for (int r = 0; r < 4; ++r) pre[r] = epi.prefetch(4 * I + r);
+        for (int r = 0; r < 4; ++r) pre[r] = epi.prefetch(4 * I + r);
+    }
     Acc acc[4] = {Acc(0), Acc(0), Acc(0), Acc(0)};
     for (int64_t t = t0; t < t1; ++t) {
         const int32_t J = __ldg(bidx + t);
         const uint32_t mp = __ldg(bmap + t);
-        Acc v[16];
+        Acc v[16];  // one lane reads the whole tile: L1-allocating loads (sectors re-used)
         if constexpr (sizeof(MatT) == 8) {
 #pragma unroll
             for (int k = 0; k < 8; ++k) {
-                const double2 d = ldg_stream(reinterpret_cast<const double2*>(bval + 16 * t) + k);
+                const double2 d = __ldg(reinterpret_cast<const double2*>(bval + 16 * t) + k);
                 v[2 * k] = d.x;
                 v[2 * k + 1] = d.y;
             }
         } else if constexpr (sizeof(MatT) == 4) {
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-                const float4 d = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * t) + k);
+                const float4 d = __ldg(reinterpret_cast<const float4*>(bval + 16 * t) + k);
                 v[4 * k] = d.x; v[4 * k + 1] = d.y; v[4 * k + 2] = d.z; v[4 * k + 3] = d.w;
             }
         } else {
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-                const uint2 w = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * t) + k);
+                const uint2 w = __ldg(reinterpret_cast<const uint2*>(bval + 16 * t) + k);
                 const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
                 const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
                 v[4 * k] = lo.x; v[4 * k + 1] = lo.y; v[4 * k + 2] = hi.x; v[4 * k + 3] = hi.y;
@@ -238,8 +242,12 @@ __global__ void __launch_bounds__(256) k_spmv_lanerow(int64_t I0, int64_t BR, co
             for (int c = 0; c < 4; ++c)
                 acc[r] = ((mp >> (4 * r + c)) & 1u) ? fma(v[4 * r + c], xv[c], acc[r]) : acc[r];
     }
+    if (vec) {
+        epi.finish4(4 * I, acc, pre);
+    } else {
 #pragma unroll
-    for (int r = 0; r < 4; ++r) epi.finish(4 * I + r, acc[r], pre[r]);
+        for (int r = 0; r < 4; ++r) epi.finish(4 * I + r, acc[r], pre[r]);
+    }
 }
 
 // ---------------------------------------------------------------- chunk kernel (long rows)
@@ -455,11 +463,17 @@ static int spmv_variant() {
 template <typename MatT, typename XT, typename YT, int MODE>
 static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
                         int64_t long_thr, cudaStream_t s) {
-    const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE};
+    const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE,
+                                (YT*)ea.r};
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
     if (P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16) {  // ~1 tile per block row
+        // vector epilogue when every vector it touches is 4-element aligned
+        const uintptr_t al = 4 * sizeof(YT) - 1;
+        auto ok = [&](const void* p) { return (reinterpret_cast<uintptr_t>(p) & al) == 0; };
+        const bool vec = ok(y) && ok(ea.b) && ok(ea.dinv) && ok(ea.r) &&
+                         (reinterpret_cast<uintptr_t>(ea.xs) & (4 * sizeof(XT) - 1)) == 0;
         k_spmv_lanerow<MatT, XT, YT, MODE><<<(unsigned)ceil_div(BR - I0, 256), 256, 0, s>>>(
-            I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, epi);
+            I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, epi, vec);
         return;
     }
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
@@ -494,6 +508,9 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
     if (BR > I0) {
         switch (ea.mode) {
             case AMGT_EPI_JACOBI: launch_rows<MatT, XT, YT, AMGT_EPI_JACOBI>(A, x, y, ea, I0, BR, long_thr, s); break;
+            case AMGT_EPI_JACOBI_RES:
+                launch_rows<MatT, XT, YT, AMGT_EPI_JACOBI_RES>(A, x, y, ea, I0, BR, long_thr, s);
+                break;
             case AMGT_EPI_RESIDUAL: launch_rows<MatT, XT, YT, AMGT_EPI_RESIDUAL>(A, x, y, ea, I0, BR, long_thr, s); break;
             case AMGT_EPI_ACCUM: launch_rows<MatT, XT, YT, AMGT_EPI_ACCUM>(A, x, y, ea, I0, BR, long_thr, s); break;
             default: launch_rows<MatT, XT, YT, AMGT_EPI_Y>(A, x, y, ea, I0, BR, long_thr, s);
@@ -502,7 +519,8 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
     }
     if (!ranged && P && P->nlong > 0) {
         using Acc = typename AccOf<MatT>::type;
-        const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode};
+        const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode,
+                              (YT*)ea.r};
         k_spmv_chunks<MatT, XT><<<(unsigned)ceil_div(P->nchunks * 32, 256), 256, 0, s>>>(
             P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, P->long_rows,
             P->chunk_ptr, P->chunk_lr, (Acc*)P->partial);
@@ -532,8 +550,10 @@ double spmv_bytes(const amgt_mbsr* A, amgt_prec xp, amgt_prec yp) {
 amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, const EpiArgs& ea,
                          cudaStream_t s, int timer_class) {
     const double vec = 4.0 * A->blc_row * prec_bytes(yp);
-    // epilogue operands read once each: Jacobi b, dinv; residual b; accumulate y
-    const double extra = ea.mode == AMGT_EPI_JACOBI ? 2 * vec : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
+    // epilogue operands read once each: Jacobi b, dinv (+ r written); residual b; accumulate y
+    const double extra = ea.mode == AMGT_EPI_JACOBI ? 2 * vec
+                         : ea.mode == AMGT_EPI_JACOBI_RES ? 3 * vec
+                         : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
     TimerScope ts(timer_class, spmv_bytes(A, xp, yp) + extra, s);
     switch (A->prec) {
         case AMGT_FP64: return dispatch_xy<double>(A, x, xp, y, yp, ea, s);
@@ -572,6 +592,19 @@ amgt_status amgt_spmv(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* 
         return fail(AMGT_ERR_ARG, "amgt_spmv: x/y precision must be FP64 or FP32");
     if (!prec_valid(A->prec)) return fail(AMGT_ERR_ARG, "amgt_spmv: bad matrix precision");
     return spmv_impl(A, x, xprec, y, yprec, (cudaStream_t)stream, TC_SPMV);
+}
+
+amgt_status amgt_spmv_fused_r(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec,
+                              const void* b, const void* dinv, double omega, void* r, void* stream) {
+    if (!A || (!x && A->blc_col > 0) || (!y && A->blc_row > 0) || (!r && A->blc_row > 0))
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_r: NULL argument");
+    if ((xprec != AMGT_FP64 && xprec != AMGT_FP32) || xprec != yprec)
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_r: x/y must share one precision, FP64 or FP32");
+    if (!b || !dinv || A->m != A->n || x == y || r == x || r == y)
+        return fail(AMGT_ERR_ARG, "amgt_spmv_fused_r: needs b, dinv, a square A and distinct x, y, r");
+    EpiArgs ea{AMGT_EPI_JACOBI_RES, b, dinv, x, omega, 0, -1};
+    ea.r = r;
+    return spmv_ex_impl(A, x, xprec, y, yprec, ea, (cudaStream_t)stream, TC_SPMV);
 }
 
 amgt_status amgt_spmv_fused(const amgt_mbsr* A, const void* x, amgt_prec xprec, void* y, amgt_prec yprec, int mode,

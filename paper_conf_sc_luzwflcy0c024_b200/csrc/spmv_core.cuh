@@ -2,6 +2,8 @@
 // persistent coarse-level V-cycle kernel (vcycle.cu).  See spmv.cu for the design notes.
 #pragma once
 
+#include <type_traits>
+
 #include "common.cuh"
 
 namespace amgt {
@@ -21,6 +23,23 @@ __device__ __forceinline__ uint2 ldg_stream(const uint2* p) {
     uint2 r;
     asm volatile("ld.global.nc.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
     return r;
+}
+
+// four consecutive elements (16-byte aligned for float, 32-byte for double)
+__device__ __forceinline__ void vload4(const double* p, double (&v)[4]) {
+    const double2 a = reinterpret_cast<const double2*>(p)[0], b = reinterpret_cast<const double2*>(p)[1];
+    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+}
+__device__ __forceinline__ void vload4(const float* p, float (&v)[4]) {
+    const float4 a = *reinterpret_cast<const float4*>(p);
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+}
+__device__ __forceinline__ void vstore4(double* p, const double (&v)[4]) {
+    reinterpret_cast<double2*>(p)[0] = make_double2(v[0], v[1]);
+    reinterpret_cast<double2*>(p)[1] = make_double2(v[2], v[3]);
+}
+__device__ __forceinline__ void vstore4(float* p, const float (&v)[4]) {
+    *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
 }
 
 // x pair (elements 2h, 2h+1 of the 4-segment at 4J) as doubles.
@@ -44,6 +63,9 @@ __device__ __forceinline__ float4 x_quad(const double* x, int64_t J) {
 //   EPI_JACOBI   y_i = xs_i + w dinv_i (b_i - (A x)_i)       (out-of-place weighted Jacobi, R21)
 //   EPI_RESIDUAL y_i = b_i - (A x)_i                          (Alg. 2 line 3)
 //   EPI_ACCUM    y_i = y_i + (A x)_i                          (interpolation + correction, lines 8-9)
+//   EPI_JACOBI_RES  as EPI_JACOBI, and r_i = b_i - (A x)_i   (the residual of the sweep's input:
+//                   after a V-cycle it is the Alg. 2 / L308 residual, so the first pre-smoothing
+//                   sweep of the next cycle also delivers the previous cycle's residual)
 // Vector arithmetic is done in the y precision, as the separate vector kernels did.
 // MODE >= 0 fixes the epilogue at compile time (the row kernels); -1 reads `mode` at run time.
 template <typename XT, typename YT, int MODE = -1>
@@ -54,6 +76,7 @@ struct Epi {
     const XT* xs;
     YT omega;
     int mode;
+    YT* r = nullptr;  // EPI_JACOBI_RES only
     __device__ __forceinline__ int md() const { return MODE >= 0 ? MODE : mode; }
     // operands of row i, loaded before the tile loop so their latency overlaps it
     struct Pre {
@@ -62,7 +85,8 @@ struct Epi {
     __device__ __forceinline__ Pre prefetch(int64_t i) const {
         Pre p;
         switch (md()) {
-            case AMGT_EPI_JACOBI: p.a = b[i]; p.c = dinv[i]; p.d = (YT)xs[i]; break;
+            case AMGT_EPI_JACOBI:
+            case AMGT_EPI_JACOBI_RES: p.a = b[i]; p.c = dinv[i]; p.d = (YT)xs[i]; break;
             case AMGT_EPI_RESIDUAL: p.a = b[i]; break;
             case AMGT_EPI_ACCUM: p.a = y[i]; break;
             default: break;
@@ -74,16 +98,73 @@ struct Epi {
         const YT t = (YT)v;
         switch (md()) {
             case AMGT_EPI_JACOBI: y[i] = p.d + omega * p.c * (p.a - t); break;
+            case AMGT_EPI_JACOBI_RES: {
+                const YT res = p.a - t;
+                y[i] = p.d + omega * p.c * res;
+                r[i] = res;
+                break;
+            }
             case AMGT_EPI_RESIDUAL: y[i] = p.a - t; break;
             case AMGT_EPI_ACCUM: y[i] = p.a + t; break;
             default: y[i] = t;
         }
+    }
+    // four consecutive rows i0..i0+3 with 16/32-byte vector accesses (all vectors aligned to
+    // 4 elements: the caller checks)
+    __device__ __forceinline__ void prefetch4(int64_t i0, Pre (&p)[4]) const {
+        YT a[4], c[4], d[4];
+        switch (md()) {
+            case AMGT_EPI_JACOBI:
+            case AMGT_EPI_JACOBI_RES:
+                vload4(b + i0, a);
+                vload4(dinv + i0, c);
+                if constexpr (std::is_same<XT, YT>::value) vload4(xs + i0, d);
+                else
+                    for (int k = 0; k < 4; ++k) d[k] = (YT)xs[i0 + k];
+                for (int k = 0; k < 4; ++k) { p[k].a = a[k]; p[k].c = c[k]; p[k].d = d[k]; }
+                break;
+            case AMGT_EPI_RESIDUAL:
+                vload4(b + i0, a);
+                for (int k = 0; k < 4; ++k) p[k].a = a[k];
+                break;
+            case AMGT_EPI_ACCUM:
+                vload4(y + i0, a);
+                for (int k = 0; k < 4; ++k) p[k].a = a[k];
+                break;
+            default: break;
+        }
+    }
+    template <typename V>
+    __device__ __forceinline__ void finish4(int64_t i0, const V (&v)[4], const Pre (&p)[4]) const {
+        YT o[4], rr[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const YT t = (YT)v[k];
+            switch (md()) {
+                case AMGT_EPI_JACOBI: o[k] = p[k].d + omega * p[k].c * (p[k].a - t); break;
+                case AMGT_EPI_JACOBI_RES:
+                    rr[k] = p[k].a - t;
+                    o[k] = p[k].d + omega * p[k].c * rr[k];
+                    break;
+                case AMGT_EPI_RESIDUAL: o[k] = p[k].a - t; break;
+                case AMGT_EPI_ACCUM: o[k] = p[k].a + t; break;
+                default: o[k] = t;
+            }
+        }
+        vstore4(y + i0, o);
+        if (md() == AMGT_EPI_JACOBI_RES) vstore4(r + i0, rr);
     }
     __device__ __forceinline__ void apply(int64_t i, double v) const { put(i, (YT)v); }
     __device__ __forceinline__ void apply(int64_t i, float v) const { put(i, (YT)v); }
     __device__ __forceinline__ void put(int64_t i, YT t) const {
         switch (md()) {
             case AMGT_EPI_JACOBI: y[i] = (YT)xs[i] + omega * dinv[i] * (b[i] - t); break;
+            case AMGT_EPI_JACOBI_RES: {
+                const YT res = b[i] - t;
+                y[i] = (YT)xs[i] + omega * dinv[i] * res;
+                r[i] = res;
+                break;
+            }
             case AMGT_EPI_RESIDUAL: y[i] = b[i] - t; break;
             case AMGT_EPI_ACCUM: y[i] = y[i] + t; break;
             default: y[i] = t;

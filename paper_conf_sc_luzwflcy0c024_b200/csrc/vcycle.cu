@@ -67,7 +67,7 @@ struct amgt_hierarchy {
 
 namespace amgt {
 
-constexpr int NORM_BLOCKS = 256;
+constexpr int NORM_BLOCKS = 296;
 
 template <typename V, typename M>
 __global__ void k_dinv(int64_t BR, int64_t m, int64_t off, const int64_t* __restrict__ bptr,
@@ -83,29 +83,54 @@ __global__ void k_dinv(int64_t BR, int64_t m, int64_t off, const int64_t* __rest
     dinv[i] = (V)(d != 0.0 ? 1.0 / d : 0.0);
 }
 
-// Deterministic ||r||^2: fixed grid of NORM_BLOCKS, per-block partials, then one block.
-__global__ void k_resnorm_partial(int64_t n, const double* __restrict__ r, double* __restrict__ partial) {
-    __shared__ double sh[32];
-    double s = 0.0;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double d = r[i];
-        s = fma(d, d, s);
-    }
+// Deterministic ||r||^2 in one launch: a fixed grid of NORM_BLOCKS, per-block partial sums
+// (fixed order), and the last block to finish (ticket counter) adds the partials with a
+// fixed tree and re-arms the counter.  ws = [NORM_BLOCKS partials | counter (zeroed once)].
+__device__ __forceinline__ double block_sum(double s, double* sh) {
     for (int d = 16; d; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = s;
     __syncthreads();
-    if (threadIdx.x == 0) {
-        double a = 0.0;
+    double a = 0.0;
+    if (threadIdx.x == 0)
         for (int w = 0; w < (int)(blockDim.x >> 5); ++w) a += sh[w];
-        partial[blockIdx.x] = a;
-    }
+    return a;
 }
 
-__global__ void k_resnorm_final(const double* __restrict__ partial, double* __restrict__ out) {
-    if (threadIdx.x == 0 && blockIdx.x == 0) {
-        double a = 0.0;
-        for (int i = 0; i < NORM_BLOCKS; ++i) a += partial[i];
-        *out = a;
+__global__ void __launch_bounds__(256) k_resnorm(int64_t n, const double* __restrict__ r, double* __restrict__ ws,
+                                                 double* __restrict__ out) {
+    __shared__ double sh[32];
+    __shared__ bool last;
+    double s = 0.0;
+    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+    if ((reinterpret_cast<uintptr_t>(r) & 15) == 0) {  // 16-byte loads
+        const int64_t n2 = n >> 1;
+        const double2* r2 = reinterpret_cast<const double2*>(r);
+        for (int64_t i = gt; i < n2; i += nt) {
+            const double2 d = __ldcs(r2 + i);
+            s = fma(d.x, d.x, s);
+            s = fma(d.y, d.y, s);
+        }
+        if ((n & 1) && gt == 0) s = fma(r[n - 1], r[n - 1], s);
+    } else {
+        for (int64_t i = gt; i < n; i += nt) s = fma(r[i], r[i], s);
+    }
+    const double part = block_sum(s, sh);
+    unsigned* counter = reinterpret_cast<unsigned*>(ws + NORM_BLOCKS);
+    if (threadIdx.x == 0) {
+        ws[blockIdx.x] = part;
+        __threadfence();
+        last = atomicAdd(counter, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    double t = 0.0;
+    for (int i = threadIdx.x; i < (int)gridDim.x; i += blockDim.x) t += __ldcg(ws + i);
+    __syncthreads();
+    const double tot = block_sum(t, sh);
+    if (threadIdx.x == 0) {
+        *out = tot;
+        *counter = 0u;
     }
 }
 
@@ -203,7 +228,7 @@ static void destroy(amgt_hierarchy* H) {
         free_level_vectors(L, a);
     }
     a.put(H->Ainv, (size_t)H->nM * H->nM * sizeof(double));
-    a.put(H->partial, NORM_BLOCKS * sizeof(double));
+    a.put(H->partial, (NORM_BLOCKS + 1) * sizeof(double));
     a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
     cudaStreamSynchronize(H->s);
     if (H->gexec) cudaGraphExecDestroy(H->gexec);
@@ -300,8 +325,9 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     if (!dense_inverse(n, dense, inv)) return fail(AMGT_ERR_ARG, "coarsest operator is not SPD (Cholesky failed)");
     H->nM = n;
     H->Ainv = (double*)a.get(n * n * sizeof(double) + 8);
-    H->partial = (double*)a.get(NORM_BLOCKS * sizeof(double));
+    H->partial = (double*)a.get((NORM_BLOCKS + 1) * sizeof(double));
     if (!H->Ainv || !H->partial) return fail(AMGT_ERR_ALLOC, "coarse inverse allocation failed");
+    AMGT_CUDA(cudaMemsetAsync(H->partial, 0, (NORM_BLOCKS + 1) * sizeof(double), H->s));
     AMGT_CUDA(cudaMemcpyAsync(H->Ainv, inv.data(), n * n * sizeof(double), cudaMemcpyHostToDevice, s));
     AMGT_CUDA(cudaStreamSynchronize(s));
     return AMGT_OK;
@@ -309,18 +335,19 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
 
 static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const void* x, amgt_prec xp, void* y,
                                 amgt_prec yp, int level, int mode = 0, const void* b = nullptr,
-                                const void* dinv = nullptr) {
-    ++H->spmv_calls;
+                                const void* dinv = nullptr, void* r = nullptr) {
+    // counts Alg. 2's SpMV operations: a Jacobi sweep that also returns the residual stands
+    // for two of them (the sweep and the residual it replaces), in one pass over A
+    H->spmv_calls += mode == AMGT_EPI_JACOBI_RES ? 2 : 1;
+    EpiArgs ea{mode, b, dinv, x, H->o.omega, 0, -1};
+    ea.r = r;
     // timer class 0 = the dominant kernel: SpMV with the level-1 operator A_1 (any epilogue)
-    return spmv_ex_impl(M, x, xp, y, yp, EpiArgs{mode, b, dinv, x, H->o.omega, 0, -1}, H->s,
-                        (level == 0 && M == &H->L[0].A) ? TC_SPMV_L1 : TC_SPMV);
+    return spmv_ex_impl(M, x, xp, y, yp, ea, H->s, (level == 0 && M == &H->L[0].A) ? TC_SPMV_L1 : TC_SPMV);
 }
 
 static amgt_status norm_into(amgt_hierarchy* H, const double* r, int64_t n, double* out) {
     TimerScope ts(TC_VEC, 1.0 * n * 8, H->s);
-    k_resnorm_partial<<<NORM_BLOCKS, 256, 0, H->s>>>(n, r, H->partial);
-    AMGT_LAUNCHED();
-    k_resnorm_final<<<1, 32, 0, H->s>>>(H->partial, out);
+    k_resnorm<<<NORM_BLOCKS, 256, 0, H->s>>>(n, r, H->partial, out);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
@@ -336,13 +363,21 @@ static amgt_status dense_solve(amgt_hierarchy* H, amgt_level& L) {
 
 constexpr int JAC = 1, RES = 2, ACC = 3;
 
-// Alg. 2 lines 2-4 at level k: pre-smoothing, residual, restriction into b_{k+1}.
-static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** xc, void** xa) {
+// Alg. 2 lines 2-4 at level k: pre-smoothing, residual, restriction into b_{k+1}.  With
+// res_norm, the first sweep (level 1, nu1 >= 1) also writes r = b - A x of the incoming x
+// and its squared norm goes to *res_norm: the residual of the previous cycle (L308).
+static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** xc, void** xa,
+                              double* res_norm = nullptr) {
     amgt_level& L = H->L[k];
     const void* bk = k == 0 ? b0 : L.b;
     if (k > 0) AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, H->s));
     for (int i = 0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
-        AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
+        if (i == 0 && res_norm) {
+            AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, AMGT_EPI_JACOBI_RES, bk, L.dinv, L.r));
+            AMGT_TRY(norm_into(H, (const double*)L.r, L.npad, res_norm));
+        } else {
+            AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, JAC, bk, L.dinv));
+        }
         std::swap(xc[k], xa[k]);
     }
     AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, L.r, L.vprec, k, RES, bk));  // line 3
@@ -370,12 +405,19 @@ static amgt_status coarse_solve(amgt_hierarchy* H, void** xc) {  // line 6
     return C.vprec == AMGT_FP64 ? dense_solve<double>(H, C) : dense_solve<float>(H, C);
 }
 
-// Levels 1..M-1 down, coarsest, levels M-1..1 up (everything below level 1).
+static int tail_level(const amgt_hierarchy* H, void** xc, void** xa);
+static amgt_status subcycle_tail(amgt_hierarchy* H, int kt);
+
+// Levels 1..M-1 down, coarsest, levels M-1..1 up (everything below level 1); the small
+// tail levels kt..M go to one single-CTA kernel (block barriers instead of ~5 launches
+// per level).
 static amgt_status subcycle_direct(amgt_hierarchy* H, void** xc, void** xa) {
     const int M = H->nlev - 1;
-    for (int k = 1; k < M; ++k) AMGT_TRY(down_level(H, k, nullptr, xc, xa));
-    AMGT_TRY(coarse_solve(H, xc));
-    for (int k = M - 1; k >= 1; --k) AMGT_TRY(up_level(H, k, nullptr, xc, xa));
+    const int kt = tail_level(H, xc, xa);
+    for (int k = 1; k < std::min(kt, M); ++k) AMGT_TRY(down_level(H, k, nullptr, xc, xa));
+    if (kt <= M) AMGT_TRY(subcycle_tail(H, kt));
+    else AMGT_TRY(coarse_solve(H, xc));
+    for (int k = std::min(kt, M) - 1; k >= 1; --k) AMGT_TRY(up_level(H, k, nullptr, xc, xa));
     return AMGT_OK;
 }
 
@@ -436,17 +478,20 @@ __device__ __forceinline__ void coop_spmv(const CoopMat& M, const VT* x, VT* y, 
 
 // One Alg. 2 step sequence on level k: grid-wide (all CTAs, grid barriers) when `grid_wide`,
 // else CTA 0 alone with block barriers (the other CTAs skip the work but keep `cur` in step).
-template <typename VT>
+// COOP = false: a single-CTA launch for the tail levels (k0 == kb: every level block-local).
+template <typename VT, bool COOP = true>
 __global__ void __launch_bounds__(256) k_subcycle(const CoopArgs a) {
     namespace cg = cooperative_groups;
-    cg::grid_group grid = cg::this_grid();
+    auto gsync = [&]() {
+        if constexpr (COOP) cg::this_grid().sync();
+    };
     const int lane = threadIdx.x & 31;
     int cur[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     auto run = [&](bool grid_wide, auto&& work) {
         if (grid_wide) {
             const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
             work(gt, nt);
-            grid.sync();
+            gsync();
         } else if (blockIdx.x == 0) {
             work((int64_t)threadIdx.x, (int64_t)blockDim.x);
             __syncthreads();
@@ -494,7 +539,7 @@ __global__ void __launch_bounds__(256) k_subcycle(const CoopArgs a) {
     for (int k = a.M - 1; k >= a.k0; --k) {  // lines 7-11
         const CoopLevel& L = a.L[k];
         const bool gwide = k < a.kb;
-        if (k + 1 == a.kb) grid.sync();  // leaving the block-local levels: everyone sees CTA 0's result
+        if (k + 1 == a.kb) gsync();  // leaving the block-local levels: everyone sees CTA 0's result
         const int cn = cur[k + 1], c0 = cur[k];
         run(gwide, [&](int64_t gt, int64_t nt) {
             coop_spmv<VT, AMGT_EPI_ACCUM>(L.P, (const VT*)a.L[k + 1].x[cn], (VT*)L.x[c0], nullptr, nullptr, nullptr,
@@ -509,21 +554,15 @@ __global__ void __launch_bounds__(256) k_subcycle(const CoopArgs a) {
             cur[k] ^= 1;
         }
     }
-    if (a.kb <= a.k0) grid.sync();  // every level was block-local
+    if (a.kb <= a.k0) gsync();  // every level was block-local
 }
 
 static CoopMat coop_mat(const amgt_mbsr& M) {
     return CoopMat{M.blc_ptr, M.blc_idx, M.blc_map, M.blc_val, (int)M.prec, M.blc_row};
 }
 
-// Returns AMGT_ERR_UNSUPPORTED (caller falls back) when the levels' vector precisions differ
-// or a cooperative launch is not possible.
-static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
-    const int M = H->nlev - 1, k0 = 1;
-    const amgt_prec vp = H->L[k0].vprec;
-    for (int k = k0; k <= M; ++k)
-        if (H->L[k].vprec != vp || xc[k] != H->L[k].x || xa[k] != H->L[k].t) return AMGT_ERR_UNSUPPORTED;
-    CoopArgs a{};
+static void fill_coop_args(const amgt_hierarchy* H, int k0, CoopArgs& a) {
+    const int M = H->nlev - 1;
     for (int k = k0; k <= M; ++k) {
         const amgt_level& L = H->L[k];
         CoopLevel& c = a.L[k];
@@ -546,6 +585,48 @@ static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
     a.omega = H->o.omega;
     a.nM = H->nM;
     a.Ainv = H->Ainv;
+}
+
+// First level of the tail run by one CTA (k_subcycle<VT, false>): block rows <= TAIL_BR
+// (AMGT_TAIL_BLOCKROWS, default 128; 0 disables), every tail level with one vector
+// precision and its ping-pong buffers in place; M + 1 = no tail.
+static int tail_level(const amgt_hierarchy* H, void** xc, void** xa) {
+    static int64_t tail_br = -1;
+    if (tail_br < 0) {
+        const char* e = getenv("AMGT_TAIL_BLOCKROWS");
+        tail_br = e ? atoll(e) : 128;
+    }
+    const int M = H->nlev - 1;
+    if (tail_br == 0 || (H->o.nu1 + H->o.nu2) % 2 != 0 || (timing_mask() & ~1u) != 0) return M + 1;
+    int kt = M + 1;
+    for (int k = 1; k <= M; ++k)
+        if (H->L[k].A.blc_row <= tail_br) { kt = k; break; }
+    if (kt > M - 1) return M + 1;  // at least one level above the coarsest
+    for (int k = kt; k <= M; ++k)
+        if (H->L[k].vprec != H->L[kt].vprec || xc[k] != H->L[k].x || xa[k] != H->L[k].t) return M + 1;
+    return kt;
+}
+
+static amgt_status subcycle_tail(amgt_hierarchy* H, int kt) {
+    CoopArgs a{};
+    fill_coop_args(H, kt, a);
+    a.kb = kt;
+    if (H->L[kt].vprec == AMGT_FP64) k_subcycle<double, false><<<1, 256, 0, H->s>>>(a);
+    else k_subcycle<float, false><<<1, 256, 0, H->s>>>(a);
+    AMGT_LAUNCHED();
+    H->spmv_calls += (int64_t)(a.M - kt) * (H->o.nu1 + H->o.nu2 + 3);
+    return AMGT_OK;
+}
+
+// Returns AMGT_ERR_UNSUPPORTED (caller falls back) when the levels' vector precisions differ
+// or a cooperative launch is not possible.
+static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
+    const int M = H->nlev - 1, k0 = 1;
+    const amgt_prec vp = H->L[k0].vprec;
+    for (int k = k0; k <= M; ++k)
+        if (H->L[k].vprec != vp || xc[k] != H->L[k].x || xa[k] != H->L[k].t) return AMGT_ERR_UNSUPPORTED;
+    CoopArgs a{};
+    fill_coop_args(H, k0, a);
     // first level small enough for one CTA (AMGT_COOP_BLOCKROWS, default 128 block rows)
     static int64_t small_br = -1;
     if (small_br < 0) {
@@ -557,7 +638,7 @@ static amgt_status subcycle_coop(amgt_hierarchy* H, void** xc, void** xa) {
         if (H->L[k].A.blc_row <= small_br) { a.kb = k; break; }
     static int grid64 = 0, grid32 = 0;
     int& grid = vp == AMGT_FP64 ? grid64 : grid32;
-    const void* kern = vp == AMGT_FP64 ? (const void*)k_subcycle<double> : (const void*)k_subcycle<float>;
+    const void* kern = vp == AMGT_FP64 ? (const void*)k_subcycle<double, true> : (const void*)k_subcycle<float, true>;
     if (grid == 0) {
         int dev = 0, coop = 0, per_sm = 0;
         cudaGetDevice(&dev);
@@ -668,8 +749,13 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
     xc[0] = x;
     xa[0] = L0.t;
     for (int k = 1; k <= M; ++k) { xc[k] = H->L[k].x; xa[k] = H->L[k].t; }
-    AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));
-    AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms));
+    // residual norms: ||b - A x_c|| after cycle c is delivered by cycle c+1's first
+    // pre-smoothing sweep (same x, same arithmetic); only the last one needs its own SpMV
+    const bool fused = M > 0 && H->o.nu1 >= 1 && L0.vprec == AMGT_FP64;
+    if (!fused || ncycles == 0) {
+        AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));
+        AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms));
+    }
     if (M == 0) {
         for (int c = 1; c <= ncycles; ++c) {
             amgt_level tmp = L0;
@@ -681,12 +767,14 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
         }
     }
     for (int c = 1; c <= ncycles && M > 0; ++c) {
-        AMGT_TRY(down_level(H, 0, b, xc, xa));              // Alg. 2 lines 1-5 at level 1
+        AMGT_TRY(down_level(H, 0, b, xc, xa, fused ? H->norms + (c - 1) : nullptr));  // lines 1-5, level 1
         if (M >= 2) AMGT_TRY(subcycle(H, xc, xa));          // levels 2..M (graph replay)
         else AMGT_TRY(coarse_solve(H, xc));
         AMGT_TRY(up_level(H, 0, b, xc, xa));                // lines 7-11 at level 1
-        AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));  // residual (L308)
-        AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms + c));
+        if (!fused || c == ncycles) {                       // residual (L308)
+            AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));
+            AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms + c));
+        }
     }
     if (xc[0] != (void*)x)
         AMGT_CUDA(cudaMemcpyAsync(x, xc[0], L0.npad * sizeof(double), cudaMemcpyDeviceToDevice, s));
@@ -776,10 +864,9 @@ amgt_status amgt_norm2sq(int64_t n, const double* r, double* out_dev, void* stre
     cudaStream_t s = (cudaStream_t)stream;
     Alloc a{nullptr, s};
     Scratch<double> part;
-    AMGT_TRY(part.init(a, NORM_BLOCKS));
-    k_resnorm_partial<<<NORM_BLOCKS, 256, 0, s>>>(n, r, part.p);
-    AMGT_LAUNCHED();
-    k_resnorm_final<<<1, 32, 0, s>>>(part.p, out_dev);
+    AMGT_TRY(part.init(a, NORM_BLOCKS + 1));
+    AMGT_CUDA(cudaMemsetAsync(part.p + NORM_BLOCKS, 0, sizeof(double), s));
+    k_resnorm<<<NORM_BLOCKS, 256, 0, s>>>(n, r, part.p, out_dev);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }

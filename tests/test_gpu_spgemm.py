@@ -84,22 +84,25 @@ def test_spgemm_info_bins_and_long_rows():
 
 LONG = [
     # power-law rows with > 512 C tiles, about one product per C tile: pair-record path
-    ("long_records", lambda: (gen.irregular_block_sparse(1 << 13, seed=9),) * 2),
+    ("long_records", lambda: (gen.irregular_block_sparse(1 << 13, seed=9),) * 2, True),
     # long rows with ~500 products per C tile: past the record capacity, pass 1 re-derives
-    ("long_fallback", lambda: (gen.random_csr(32, 8192, 0.3, 31), gen.random_csr(8192, 4096, 0.02, 32))),
+    ("long_fallback", lambda: (gen.random_csr(32, 8192, 0.3, 31), gen.random_csr(8192, 4096, 0.02, 32)), True),
+    # only 32 < nC <= 512 rows (warp-per-row kernel, no long-row launches)
+    ("mid_only", lambda: (gen.random_csr(64, 3000, 0.3, 33), gen.random_csr(3000, 900, 0.01, 34)), False),
 ]
 
 
 @pytest.mark.parametrize("prec", ["f64", "f32", "f16"])
-@pytest.mark.parametrize("name,mk", LONG, ids=[p[0] for p in LONG])
-def test_spgemm_long_rows(name, mk, prec):
+@pytest.mark.parametrize("name,mk,has_long", LONG, ids=[p[0] for p in LONG])
+def test_spgemm_long_rows(name, mk, has_long, prec):
     """Rows with > 512 C tiles (two-pass long-row kernels) and 32 < nC <= 512 (warp kernel)."""
     amgt = _amgt()
     A, B = mk()
     Ao, Bo = oracle.as_csr(A), oracle.as_csr(B)
     Co, Cabs = oracle.spgemm(Ao, Bo, with_abs=True)
     C = amgt.spgemm(amgt.from_csr(A, prec=prec), amgt.from_csr(B, prec=prec))
-    assert np.diff(C.blc_ptr.cpu().numpy()).max() > 512
+    nC = np.diff(C.blc_ptr.cpu().numpy())
+    assert (nC.max() > 512) == has_long and nC.max() > 32
     if prec == "f64":
         _check_product(C, Co, Cabs)
         return

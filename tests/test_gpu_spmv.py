@@ -149,3 +149,22 @@ def test_spmv_fused_epilogues(dt):
             assert np.all(np.abs(g - expect) <= tol), mode
         else:
             assert rel_inf(g, expect) <= 1e-5, (mode, rel_inf(g, expect))
+
+
+@pytest.mark.parametrize("dt", [torch.float64, torch.float32])
+def test_spmv_jacobi_res(dt):
+    """amgt_spmv_fused_r: one pass gives the Jacobi sweep and the residual of its input,
+    bit-identical to the separate EPI_JACOBI and EPI_RESIDUAL calls."""
+    amgt = _amgt()
+    A = gen.laplacian_7pt(20, spd_seed=2)
+    Ao = oracle.as_csr(A)
+    M = amgt.from_csr(A, prec="f64" if dt == torch.float64 else "f32")
+    T = lambda v: torch.from_numpy(np.ascontiguousarray(v)).to(dt).cuda()
+    x, b = T(gen.uniform_vector(A.n, 1).numpy()), T(gen.uniform_vector(A.n, 2).numpy())
+    d = T(1.0 / Ao.dense().diagonal())
+    y, r = torch.empty_like(x), torch.empty_like(x)
+    amgt.spmv_jacobi_res(M, x, y, b, d, r)
+    y2, r2 = torch.empty_like(x), torch.empty_like(x)
+    amgt.spmv_fused(M, x, y2, "jacobi", b=b, dinv=d)
+    amgt.spmv_fused(M, x, r2, "residual", b=b)
+    assert torch.equal(y, y2) and torch.equal(r, r2)
