@@ -677,7 +677,7 @@ constexpr int CAP = 32;  // C tiles per row accumulated in shared memory
 
 template <typename Acc> struct NumSmem {
     Acc acc[CAP][16];
-    Acc stage[32][16];
+    Acc stage[32][17];  // one tile product per lane; padded rows (lane-strided writes)
     int32_t cidx[CAP];
 };
 
@@ -700,19 +700,12 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
     const int nC = (int)(cptr[I + 1] - c0);
     if (nC == 0) return;
     const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
-    const bool small = nC <= CAP;
-    // accumulator access: smem for small rows, global (C values or FP32 workspace) otherwise
-    Acc* gbase = nullptr;
-    if (small) {
-        if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
-        for (int e = lane; e < nC * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
-    } else {
-        gbase = gacc ? gacc + 16 * c0 : reinterpret_cast<Acc*>(cval + 16 * c0);
-        for (int64_t e = lane; e < 16 * (int64_t)nC; e += 32) gbase[e] = Acc(0);
-    }
+    // nC <= CAP (longer rows go to the mid/long-row kernels): shared-memory accumulators
+    if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
+    for (int e = lane; e < nC * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
     __syncwarp();
-    const int32_t* rowidx = small ? S.cidx : cidx_g + c0;
-    auto accp = [&](int q) -> Acc* { return small ? S.acc[q] : gbase + 16 * (int64_t)q; };
+    const int32_t* rowidx = S.cidx;
+    auto accp = [&](int q) -> Acc* { return S.acc[q]; };
 
     // ---- tensor-core route (FP64 only): A tiles with POPCOUNT >= tc_thr, one at a time.
     if constexpr (sizeof(T) == 8) {
@@ -768,8 +761,8 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
 
     // ---- CUDA-core route: pairs of the remaining A tiles.
     const int thr = (sizeof(T) == 8) ? tc_thr : 17;
-    if (small) {
-        // flattened pairs, conflicts resolved per round by match_any (deterministic)
+    {
+        // flattened pairs: one lane per (A tile, B tile) pair, products staged per lane
         for (int64_t base = a0; base < a1; base += 32) {
             const int64_t t = base + lane;
             const bool v = t < a1;
@@ -800,65 +793,41 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
                 const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
                 const int64_t ot = base + lo;
                 int q = -1;
-                Acc prod[16];
                 if (p < total) {
                     const int64_t j = ob0 + (p - oex);
                     const uint32_t mc = bitmap_multiply(oma, c.bmap[j]);
                     if (mc) {
                         q = bsearch_row(rowidx, nC, c.bidx[j]);
-                        Acc av[16], bv[16];
-                        TileIO<T>::load(aval + 16 * ot, av);
+                        Acc bv[16];
                         TileIO<T>::load(bval + 16 * j, bv);
-                        tile_mma(av, bv, prod);
-                    }
-                }
-                const uint32_t peers = __match_any_sync(0xffffffffu, q);
-                const bool alone = __popc(peers) == 1;
-                if (q >= 0 && alone) {
+                        const T* ap = aval + 16 * ot;
 #pragma unroll
-                    for (int e = 0; e < 16; ++e) S.acc[q][e] += prod[e];
-                }
-                const bool shared = q >= 0 && !alone;
-                if (__any_sync(0xffffffffu, shared)) {
-                    if (shared) {
+                        for (int r = 0; r < 4; ++r) {  // product rows straight to the staging row
+                            Acc ar[4];
+                            RowIO<T>::load(ap + 4 * r, ar);
 #pragma unroll
-                        for (int e = 0; e < 16; ++e) S.stage[lane][e] = prod[e];
-                    }
-                    __syncwarp();
-                    if (shared && (__ffs(peers) - 1) == lane) {  // leader: add peers in lane order
-                        uint32_t pm = peers;
-                        while (pm) {
-                            const int src = __ffs(pm) - 1;
-                            pm &= pm - 1;
-#pragma unroll
-                            for (int e = 0; e < 16; ++e) S.acc[q][e] += S.stage[src][e];
+                            for (int col = 0; col < 4; ++col) {
+                                Acc sv = ar[0] * bv[col];
+                                sv = fma(ar[1], bv[4 + col], sv);
+                                sv = fma(ar[2], bv[8 + col], sv);
+                                sv = fma(ar[3], bv[12 + col], sv);
+                                S.stage[lane][4 * r + col] = sv;
+                            }
                         }
                     }
                 }
                 __syncwarp();
+                // accumulate the staged products in lane order (deterministic): half-warp h
+                // takes the products whose C tile has (q & 1) == h, lane e of it element e
+                uint32_t todo = __ballot_sync(0xffffffffu, q >= 0);
+                while (todo) {
+                    const int sl = __ffs(todo) - 1;
+                    todo &= todo - 1;
+                    const int qs = __shfl_sync(0xffffffffu, q, sl);
+                    if ((qs & 1) == (lane >> 4)) S.acc[qs][lane & 15] += S.stage[sl][lane & 15];
+                }
+                __syncwarp();
             }
-        }
-    } else {
-        // global accumulation: one sparse A tile at a time, lanes over its B row (distinct C tiles)
-        for (int64_t t = a0; t < a1; ++t) {
-            const uint32_t ma = c.amap[t];
-            if (__popc(ma) >= thr) continue;
-            const int32_t K = c.aidx[t];
-            Acc av[16];
-            TileIO<T>::load(aval + 16 * t, av);
-            const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
-            for (int64_t j = b0 + lane; j < b1; j += 32) {
-                const uint32_t mc = bitmap_multiply(ma, c.bmap[j]);
-                if (!mc) continue;
-                const int q = bsearch_row(rowidx, nC, c.bidx[j]);
-                Acc bv[16], prod[16];
-                TileIO<T>::load(bval + 16 * j, bv);
-                tile_mma(av, bv, prod);
-                Acc* p = gbase + 16 * (int64_t)q;
-#pragma unroll
-                for (int e = 0; e < 16; ++e) p[e] += prod[e];
-            }
-            __syncwarp();
         }
     }
     __syncwarp();
@@ -866,7 +835,7 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
     for (int64_t e = lane; e < 16 * (int64_t)nC; e += 32) {
         const int q = (int)(e >> 4), b = (int)(e & 15);
         const bool bit = (cmap_g[c0 + q] >> b) & 1u;
-        const Acc v = small ? S.acc[q][b] : gbase[e];
+        const Acc v = S.acc[q][b];
         cval[16 * c0 + e] = bit ? from_acc<T>(v) : from_acc<T>(Acc(0));
     }
 }
@@ -1794,7 +1763,12 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     // row classes present (C->row_max from symbolic; 0 = unknown: launch everything)
     const int64_t rmax = C->row_max > 0 ? C->row_max : INT64_MAX;
     if (rmax <= GROUP_NC) return AMGT_OK;
-    k_numeric<T, Acc><<<(unsigned)num_sms() * 4, NUM_WARPS * 32, 0, s>>>(
+    static int warp_per_sm = 0;  // resident CTAs of the warp kernel (per instantiation)
+    if (!warp_per_sm) {
+        AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&warp_per_sm, k_numeric<T, Acc>, NUM_WARPS * 32, 0));
+        warp_per_sm = max(warp_per_sm, 1);
+    }
+    k_numeric<T, Acc><<<(unsigned)(num_sms() * warp_per_sm), NUM_WARPS * 32, 0, s>>>(
         big.p, nbig.p, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map,
         (T*)C->blc_val, nullptr, g_tc_thr_spgemm);  // rows <= CAP accumulate in shared memory
     AMGT_LAUNCHED();
