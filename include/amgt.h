@@ -329,9 +329,14 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* leve
 typedef struct {
     int max_levels;          /* <= 8 (paper: <= 7, L302) */
     int nu1, nu2;            /* pre/post smoothing sweeps (paper num_sweep = 1, L300) */
-    double omega;            /* weighted-Jacobi weight (R21; default 2/3) */
+    double omega;            /* Jacobi weight (R21; default 2/3) */
     amgt_prec level_prec[8]; /* matrix precision per level (L266: FP64, FP32, FP16...) */
+    int smoother;            /* AMGT_SMOOTH_JACOBI (default): D = diag(A_k), x += omega D^-1 (b - A x);
+                                AMGT_SMOOTH_L1_JACOBI: D_ii = sum_j |a_ij| (the l1 row norm; the
+                                paper's L1_Jacobi, L300, NEXT-3), same sweep — omega = 1 is HYPRE's */
 } amgt_vcycle_opts;
+#define AMGT_SMOOTH_JACOBI 0
+#define AMGT_SMOOTH_L1_JACOBI 1
 
 typedef struct amgt_hierarchy amgt_hierarchy;
 
@@ -360,6 +365,22 @@ int amgt_hierarchy_nlev(const amgt_hierarchy* H);
  */
 amgt_status amgt_vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_norms_host,
                         int64_t* spmv_calls_host, void* stream);
+
+/*
+ * Preconditioned conjugate gradient on A_1 x = b with one V-cycle (Alg. 2 from a zero
+ * guess, no residual norms) as the preconditioner M — the solve-phase consumer named at
+ * L92 (NEXT-1).  Textbook recurrence: r0 = b - A x0, z = M r, p = z; per iteration
+ * q = A p, alpha = (r,z)/(p,q), x += alpha p, r -= alpha q, z = M r,
+ * beta = (r,z)_new/(r,z)_old, p = z + beta p (alpha, beta = 0 when a denominator is 0).
+ * The V-cycle is symmetric when nu1 = nu2 (Jacobi before and after), so M is SPD for SPD
+ * A in exact arithmetic.  Runs maxit iterations, or stops early once ||r_k|| <= rtol ||r_0||
+ * when rtol > 0 (one host round trip per iteration for the test; rtol = 0: no sync until
+ * the end).  res_norms_host[maxit+1]: ||r_k||_2 for k = 0..*iters_host; *spmv_calls_host
+ * counts every SpMV (1 + per iteration 1 + a V-cycle's).  b, x: FP64, 4*blc_row(A_1);
+ * the level-1 vector precision must be FP64 (AMGT_ERR_UNSUPPORTED otherwise).
+ */
+amgt_status amgt_pcg(amgt_hierarchy* H, const double* b, double* x, int maxit, double rtol, double* res_norms_host,
+                     int* iters_host, int64_t* spmv_calls_host, void* stream);
 
 amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H);
 

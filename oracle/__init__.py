@@ -272,9 +272,9 @@ def build_hierarchy(A, PR_list, nthreads=None):
     return As
 
 
-def vcycle(As, PR_list, b, x0=None, ncycles=1, omega=2.0 / 3.0, nu1=1, nu2=1, nthreads=None):
-    """O6: Alg. 2 (L68-82), weighted Jacobi (R21), dense Cholesky coarsest (R22).
-    Returns (x, res_norms[ncycles+1], spmv_calls)."""
+def vcycle(As, PR_list, b, x0=None, ncycles=1, omega=2.0 / 3.0, nu1=1, nu2=1, nthreads=None, smoother="jacobi"):
+    """O6: Alg. 2 (L68-82), weighted Jacobi (R21) or L1-Jacobi (D_ii = sum_j |a_ij|, L300),
+    dense Cholesky coarsest (R22).  Returns (x, res_norms[ncycles+1], spmv_calls)."""
     nlev = len(As)
     assert len(PR_list) == nlev - 1
     Ps = [as_csr(p) for p, _ in PR_list]
@@ -301,7 +301,46 @@ def vcycle(As, PR_list, b, x0=None, ncycles=1, omega=2.0 / 3.0, nu1=1, nu2=1, nt
         arr(Rs, "row_ptr", None), arr(Rs, "col", None), arr(Rs, "val", None),
         ctypes.c_double(omega), ctypes.c_int(nu1), ctypes.c_int(nu2),
         b.ctypes.data_as(ctypes.c_void_p), x.ctypes.data_as(ctypes.c_void_p), ctypes.c_int(ncycles),
-        res.ctypes.data_as(ctypes.c_void_p), ctypes.byref(calls), ctypes.c_int(_nt(nthreads)))
+        res.ctypes.data_as(ctypes.c_void_p), ctypes.byref(calls), ctypes.c_int(_nt(nthreads)),
+        ctypes.c_int({"jacobi": 0, "l1_jacobi": 1}[smoother]))
     if st != 0:
         raise RuntimeError(f"oracle_vcycle failed ({st})")
     return x, res, int(calls.value)
+
+
+def vcycle_preconditioner(As, PR_list, omega=2.0 / 3.0, nu1=1, nu2=1, smoother="jacobi"):
+    """M r = one O6 V-cycle on A_1 z = r from z = 0 (the PCG preconditioner, NEXT-1)."""
+    def M(r):
+        z, _, _ = vcycle(As, PR_list, r, x0=None, ncycles=1, omega=omega, nu1=nu1, nu2=nu2, smoother=smoother)
+        return z
+    return M
+
+
+def pcg(A, b, M, x0=None, maxit=20):
+    """PCG (NEXT-1; PCG is the solve-phase consumer named at L92), textbook recurrence in
+    FP64, written out step by step:
+        r0 = b - A x0, z0 = M r0, p0 = z0
+        q = A p, alpha = (r,z)/(p,q), x += alpha p, r -= alpha q, z = M r,
+        beta = (r,z)_new/(r,z)_old, p = z + beta p      (alpha, beta = 0 on a zero denominator)
+    A: Csr (O3 SpMV), M: callable r -> z.  Returns (x, [||r_k||_2, k = 0..maxit])."""
+    A = as_csr(A)
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    x = np.zeros(A.m) if x0 is None else np.array(x0, dtype=np.float64)
+    r = b - spmv(A, x)
+    z = M(r)
+    p = z.copy()
+    rz = float(r @ z)
+    res = [float(np.sqrt(r @ r))]
+    for _ in range(maxit):
+        q = spmv(A, p)
+        pq = float(p @ q)
+        alpha = rz / pq if pq != 0.0 else 0.0
+        x = x + alpha * p
+        r = r - alpha * q
+        res.append(float(np.sqrt(r @ r)))
+        z = M(r)
+        rz_new = float(r @ z)
+        beta = rz_new / rz if rz != 0.0 else 0.0
+        p = z + beta * p
+        rz = rz_new
+    return x, res

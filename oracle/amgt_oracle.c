@@ -19,7 +19,8 @@
  *   O4 oracle_transpose     R = P^T by counting sort (Alg. 1 line 4, L54).
  *   O5 RAP                  A_c = O1(R, O1(A, P)) (Alg. 1 line 5, L54; reading R20).
  *   O6 oracle_vcycle        Alg. 2 (L68-82) with weighted Jacobi x += w D^-1 (b - A x)
- *                           (reading R21), dense Cholesky on the coarsest level (R22),
+ *                           (reading R21; smoother 1: L1-Jacobi, D_ii = sum_j |a_ij|,
+ *                           L300), dense Cholesky on the coarsest level (R22),
  *                           records ||r||_2 per cycle and SpMV calls (L308).
  *   O7 oracle_mbsr_to_csr_* inverse of O2 (L234, L262).
  *
@@ -311,7 +312,7 @@ int oracle_vcycle(int nlev, const int64_t* nrows,
                   const int64_t* const* Prp, const int32_t* const* Pci, const double* const* Pv,
                   const int64_t* const* Rrp, const int32_t* const* Rci, const double* const* Rv,
                   double omega, int nu1, int nu2, const double* b, double* x, int ncycles,
-                  double* res_norms, int64_t* spmv_calls, int nthreads) {
+                  double* res_norms, int64_t* spmv_calls, int nthreads, int smoother) {
     ocsr A[16], P[16], R[16];
     double *bk[16], *xk[16], *rk[16], *tk[16], *dinv[16];
     if (nlev < 1 || nlev > 16) return -2;
@@ -325,10 +326,14 @@ int oracle_vcycle(int nlev, const int64_t* nrows,
         bk[k] = (double*)calloc(1, sz); xk[k] = (double*)calloc(1, sz);
         rk[k] = (double*)calloc(1, sz); tk[k] = (double*)calloc(1, sz);
         dinv[k] = (double*)calloc(1, sz);
-        for (int64_t i = 0; i < nrows[k]; ++i) {   /* D = diag(A_k) */
+        for (int64_t i = 0; i < nrows[k]; ++i) {
             double d = 0.0;
-            for (int64_t p = Arp[k][i]; p < Arp[k][i + 1]; ++p)
-                if (Aci[k][p] == i) d = Av[k][p];
+            if (smoother == 1) {   /* L1-Jacobi (L300): D_ii = sum_j |a_ij| (l1 row norm) */
+                for (int64_t p = Arp[k][i]; p < Arp[k][i + 1]; ++p) d += fabs(Av[k][p]);
+            } else {               /* weighted Jacobi (R21): D = diag(A_k) */
+                for (int64_t p = Arp[k][i]; p < Arp[k][i + 1]; ++p)
+                    if (Aci[k][p] == i) d = Av[k][p];
+            }
             dinv[k][i] = 1.0 / d;
         }
     }

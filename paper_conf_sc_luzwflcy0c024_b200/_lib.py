@@ -68,7 +68,7 @@ class c_spmv_stats(ctypes.Structure):
 
 class c_vcycle_opts(ctypes.Structure):
     _fields_ = [("max_levels", ctypes.c_int), ("nu1", ctypes.c_int), ("nu2", ctypes.c_int), ("omega", ctypes.c_double),
-                ("level_prec", ctypes.c_int * 8)]
+                ("level_prec", ctypes.c_int * 8), ("smoother", ctypes.c_int)]
 
 
 class c_dist_level(ctypes.Structure):
@@ -105,6 +105,7 @@ _sigs = {
     "amgt_spmv_get_stats": (_int, [_P(c_mbsr), _P(c_spmv_stats)]),
     "amgt_spmv": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _vp]),
     "amgt_spmv_fused": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _int, _vp, _vp, ctypes.c_double, _vp]),
+    "amgt_pcg": (_int, [_vp, _vp, _vp, _int, ctypes.c_double, _vp, _P(ctypes.c_int), _P(ctypes.c_int64), _vp]),
     "amgt_spmv_fused_r": (_int, [_P(c_mbsr), _vp, _int, _vp, _int, _vp, _vp, ctypes.c_double, _vp, _vp]),
     "amgt_hierarchy_create": (_int, [_P(c_mbsr), _P(_P(c_mbsr)), _int, _P(c_vcycle_opts), _P(c_allocator), _vp,
                                      _P(_vp)]),
@@ -447,11 +448,12 @@ class Hierarchy:
     """amgt_hierarchy_create / amgt_vcycle / amgt_hierarchy_destroy."""
 
     def __init__(self, A: Mbsr, Ps: list, level_prec=("f64", "f32", "f16", "f16", "f16", "f16", "f16", "f16"),
-                 nu1=1, nu2=1, omega=2.0 / 3.0, stream=None):
+                 nu1=1, nu2=1, omega=2.0 / 3.0, smoother="jacobi", stream=None):
         self.nlev = len(Ps) + 1
         o = c_vcycle_opts()
         o.max_levels = self.nlev
         o.nu1, o.nu2, o.omega = int(nu1), int(nu2), float(omega)
+        o.smoother = {"jacobi": 0, "l1_jacobi": 1}[smoother]
         lp = list(level_prec) + ["f16"] * 8
         for k in range(8):
             o.level_prec[k] = PREC[lp[k]]
@@ -482,6 +484,15 @@ class Hierarchy:
         _check(_L.amgt_vcycle(self.h, b.data_ptr(), x.data_ptr(), int(ncycles), res, ctypes.byref(calls),
                               _stream(stream)))
         return list(res), int(calls.value)
+
+    def pcg(self, b: torch.Tensor, x: torch.Tensor, maxit: int, rtol: float = 0.0, stream=None):
+        """amgt_pcg: V-cycle-preconditioned CG; returns (residual norms, iterations, SpMV calls)."""
+        assert b.dtype == torch.float64 and x.dtype == torch.float64 and b.is_cuda and x.is_cuda
+        res = (ctypes.c_double * (maxit + 1))()
+        it, calls = ctypes.c_int(0), ctypes.c_int64(0)
+        _check(_L.amgt_pcg(self.h, b.data_ptr(), x.data_ptr(), int(maxit), float(rtol), res, ctypes.byref(it),
+                           ctypes.byref(calls), _stream(stream)))
+        return list(res)[:it.value + 1], int(it.value), int(calls.value)
 
     def close(self):
         if self.h:

@@ -71,15 +71,21 @@ constexpr int NORM_BLOCKS = 296;
 
 template <typename V, typename M>
 __global__ void k_dinv(int64_t BR, int64_t m, int64_t off, const int64_t* __restrict__ bptr,
-                       const int32_t* __restrict__ bidx, const M* __restrict__ bval, V* __restrict__ dinv) {
+                       const int32_t* __restrict__ bidx, const M* __restrict__ bval, V* __restrict__ dinv, bool l1) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= 4 * BR) return;
     const int64_t I = i >> 2;
     const int r = (int)(i & 3);
     double d = 0.0;
-    if (i < m)
-        for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t)
-            if (bidx[t] == (int32_t)(I + off)) { d = to_f64(bval[16 * t + 5 * r]); break; }
+    if (i < m) {
+        if (l1) {  // l1 row norm sum_j |a_ij| in column order (tiles ascending, +0.0 fill)
+            for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t)
+                for (int c = 0; c < 4; ++c) d += fabs(to_f64(bval[16 * t + 4 * r + c]));
+        } else {
+            for (int64_t t = bptr[I]; t < bptr[I + 1]; ++t)
+                if (bidx[t] == (int32_t)(I + off)) { d = to_f64(bval[16 * t + 5 * r]); break; }
+        }
+    }
     dinv[i] = (V)(d != 0.0 ? 1.0 / d : 0.0);
 }
 
@@ -96,24 +102,11 @@ __device__ __forceinline__ double block_sum(double s, double* sh) {
     return a;
 }
 
-__global__ void __launch_bounds__(256) k_resnorm(int64_t n, const double* __restrict__ r, double* __restrict__ ws,
-                                                 double* __restrict__ out) {
+// the partial of this CTA into ws[blockIdx.x]; the last CTA to arrive sums the partials
+// (fixed tree) into *out and re-arms the counter
+__device__ __forceinline__ void finish_sum(double s, double* __restrict__ ws, double* __restrict__ out) {
     __shared__ double sh[32];
     __shared__ bool last;
-    double s = 0.0;
-    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
-    if ((reinterpret_cast<uintptr_t>(r) & 15) == 0) {  // 16-byte loads
-        const int64_t n2 = n >> 1;
-        const double2* r2 = reinterpret_cast<const double2*>(r);
-        for (int64_t i = gt; i < n2; i += nt) {
-            const double2 d = __ldcs(r2 + i);
-            s = fma(d.x, d.x, s);
-            s = fma(d.y, d.y, s);
-        }
-        if ((n & 1) && gt == 0) s = fma(r[n - 1], r[n - 1], s);
-    } else {
-        for (int64_t i = gt; i < n; i += nt) s = fma(r[i], r[i], s);
-    }
     const double part = block_sum(s, sh);
     unsigned* counter = reinterpret_cast<unsigned*>(ws + NORM_BLOCKS);
     if (threadIdx.x == 0) {
@@ -132,6 +125,55 @@ __global__ void __launch_bounds__(256) k_resnorm(int64_t n, const double* __rest
         *out = tot;
         *counter = 0u;
     }
+}
+
+// *out = a . b (a == b: ||a||^2), deterministic for a fixed grid of NORM_BLOCKS
+__global__ void __launch_bounds__(256) k_dot(int64_t n, const double* __restrict__ a, const double* __restrict__ b,
+                                             double* __restrict__ ws, double* __restrict__ out) {
+    double s = 0.0;
+    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+    if (((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15) == 0) {  // 16-byte loads
+        const int64_t n2 = n >> 1;
+        const double2* a2 = reinterpret_cast<const double2*>(a);
+        const double2* b2 = reinterpret_cast<const double2*>(b);
+        for (int64_t i = gt; i < n2; i += nt) {
+            const double2 u = __ldcs(a2 + i), v = __ldcs(b2 + i);
+            s = fma(u.x, v.x, s);
+            s = fma(u.y, v.y, s);
+        }
+        if ((n & 1) && gt == 0) s = fma(a[n - 1], b[n - 1], s);
+    } else {
+        for (int64_t i = gt; i < n; i += nt) s = fma(a[i], b[i], s);
+    }
+    finish_sum(s, ws, out);
+}
+
+// PCG (NEXT-1): x += alpha p, r -= alpha q with alpha = rz / pq (0 when pq = 0), and
+// ||r||^2 of the updated r into *rr (one pass)
+__global__ void __launch_bounds__(256) k_pcg_xr(int64_t n, const double* __restrict__ rz, const double* __restrict__ pq,
+                                                double* __restrict__ x, double* __restrict__ r,
+                                                const double* __restrict__ p, const double* __restrict__ q,
+                                                double* __restrict__ ws, double* __restrict__ rr) {
+    const double den = *pq;
+    const double alpha = den != 0.0 ? *rz / den : 0.0;
+    double s = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        x[i] = fma(alpha, p[i], x[i]);
+        const double ri = fma(-alpha, q[i], r[i]);
+        r[i] = ri;
+        s = fma(ri, ri, s);
+    }
+    finish_sum(s, ws, rr);
+}
+
+// p = z + beta p, beta = rz_new / rz_old (0 when rz_old = 0)
+__global__ void __launch_bounds__(256) k_pcg_p(int64_t n, const double* __restrict__ rz_new,
+                                               const double* __restrict__ rz_old, const double* __restrict__ z,
+                                               double* __restrict__ p) {
+    const double den = *rz_old;
+    const double beta = den != 0.0 ? *rz_new / den : 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = fma(beta, p[i], z[i]);
 }
 
 // x = Ainv * b (dense FP64), one warp per row.
@@ -157,24 +199,31 @@ static unsigned vgrid(int64_t n) {
 static size_t vbytes(amgt_prec p) { return p == AMGT_FP64 ? 8 : 4; }
 
 template <typename V, typename M>
-static void launch_dinv(const amgt_mbsr& A, int64_t off, void* dinv, cudaStream_t s) {
+static void launch_dinv(const amgt_mbsr& A, int64_t off, void* dinv, bool l1, cudaStream_t s) {
     k_dinv<V, M><<<(unsigned)ceil_div(4 * A.blc_row, 256), 256, 0, s>>>(A.blc_row, A.m, off, A.blc_ptr, A.blc_idx,
-                                                                       (const M*)A.blc_val, (V*)dinv);
+                                                                       (const M*)A.blc_val, (V*)dinv, l1);
 }
 
-static amgt_status dinv_impl(const amgt_mbsr& A, int64_t off, void* dinv, amgt_prec vprec, cudaStream_t s) {
+static amgt_status dinv_impl(const amgt_mbsr& A, int64_t off, void* dinv, amgt_prec vprec, cudaStream_t s,
+                             bool l1 = false) {
     if (A.blc_row == 0) return AMGT_OK;
     const bool v64 = vprec == AMGT_FP64;
     switch (A.prec) {
-        case AMGT_FP64: v64 ? launch_dinv<double, double>(A, off, dinv, s) : launch_dinv<float, double>(A, off, dinv, s); break;
-        case AMGT_FP32: v64 ? launch_dinv<double, float>(A, off, dinv, s) : launch_dinv<float, float>(A, off, dinv, s); break;
-        default: v64 ? launch_dinv<double, __half>(A, off, dinv, s) : launch_dinv<float, __half>(A, off, dinv, s);
+        case AMGT_FP64:
+            v64 ? launch_dinv<double, double>(A, off, dinv, l1, s) : launch_dinv<float, double>(A, off, dinv, l1, s);
+            break;
+        case AMGT_FP32:
+            v64 ? launch_dinv<double, float>(A, off, dinv, l1, s) : launch_dinv<float, float>(A, off, dinv, l1, s);
+            break;
+        default: v64 ? launch_dinv<double, __half>(A, off, dinv, l1, s) : launch_dinv<float, __half>(A, off, dinv, l1, s);
     }
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
 
-static amgt_status build_dinv(amgt_level& L, cudaStream_t s) { return dinv_impl(L.A, 0, L.dinv, L.vprec, s); }
+static amgt_status build_dinv(amgt_level& L, cudaStream_t s, bool l1) {
+    return dinv_impl(L.A, 0, L.dinv, L.vprec, s, l1);
+}
 
 // Host dense Cholesky + inverse of the (SPD) coarsest operator.
 static bool dense_inverse(int64_t n, std::vector<double>& a, std::vector<double>& inv) {
@@ -266,7 +315,7 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             if (!*p) return fail(AMGT_ERR_ALLOC, "hierarchy vector allocation failed");
             AMGT_CUDA(cudaMemsetAsync(*p, 0, vb, s));
         }
-        AMGT_TRY(build_dinv(L, s));
+        AMGT_TRY(build_dinv(L, s, H->o.smoother == AMGT_SMOOTH_L1_JACOBI));
         if (k + 1 < nlev) {
             const amgt_mbsr* Pk = P[k];
             if (Pk->m != L.A.m) return fail(AMGT_ERR_ARG, "P[%d] has %lld rows, level has %lld", k, (long long)Pk->m, (long long)L.A.m);
@@ -347,7 +396,7 @@ static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const voi
 
 static amgt_status norm_into(amgt_hierarchy* H, const double* r, int64_t n, double* out) {
     TimerScope ts(TC_VEC, 1.0 * n * 8, H->s);
-    k_resnorm<<<NORM_BLOCKS, 256, 0, H->s>>>(n, r, H->partial, out);
+    k_dot<<<NORM_BLOCKS, 256, 0, H->s>>>(n, r, r, H->partial, out);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
@@ -787,6 +836,100 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
     return AMGT_OK;
 }
 
+// z = M r: one V-cycle (Alg. 2) on A_1 z = r from z = 0, no residual norms.
+static amgt_status precond(amgt_hierarchy* H, const double* r, double* z) {
+    const int M = H->nlev - 1;
+    amgt_level& L0 = H->L[0];
+    void* xc[8];
+    void* xa[8];
+    xc[0] = z;
+    xa[0] = L0.t;
+    for (int k = 1; k <= M; ++k) { xc[k] = H->L[k].x; xa[k] = H->L[k].t; }
+    AMGT_CUDA(cudaMemsetAsync(z, 0, L0.npad * sizeof(double), H->s));
+    if (M == 0) {
+        amgt_level tmp = L0;
+        tmp.b = (void*)r;
+        tmp.x = z;
+        return dense_solve<double>(H, tmp);
+    }
+    AMGT_TRY(down_level(H, 0, r, xc, xa));
+    if (M >= 2) AMGT_TRY(subcycle(H, xc, xa));
+    else AMGT_TRY(coarse_solve(H, xc));
+    AMGT_TRY(up_level(H, 0, r, xc, xa));
+    if (xc[0] != (void*)z)
+        AMGT_CUDA(cudaMemcpyAsync(z, xc[0], L0.npad * sizeof(double), cudaMemcpyDeviceToDevice, H->s));
+    return AMGT_OK;
+}
+
+// PCG on A_1 preconditioned by one V-cycle per iteration (NEXT-1; PCG is the solve-phase
+// consumer named at L92).  Textbook recurrence (r0 = b - A x0, z = M r, p = z, then
+// q = A p, alpha = (r,z)/(p,q), x += alpha p, r -= alpha q, z = M r, beta = (r,z)'/(r,z),
+// p = z + beta p); every scalar stays on the device (no host round trip per iteration
+// unless rtol > 0 asks for an early stop).  res_host[k] = ||r_k||_2, k = 0..iters.
+static amgt_status pcg(amgt_hierarchy* H, const double* b, double* x, int maxit, double rtol, double* res_host,
+                       int* iters_host, int64_t* calls_host) {
+    cudaStream_t s = H->s;
+    Alloc a = H->alloc();
+    amgt_level& L0 = H->L[0];
+    if (L0.vprec != AMGT_FP64) return fail(AMGT_ERR_UNSUPPORTED, "amgt_pcg: level-1 vectors must be FP64");
+    const int64_t n = L0.npad;
+    if (maxit + 1 > H->norms_cap) {
+        a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
+        H->norms_cap = maxit + 1;
+        H->norms = (double*)a.get((size_t)H->norms_cap * sizeof(double));
+        if (!H->norms) return fail(AMGT_ERR_ALLOC, "norm buffer allocation failed");
+    }
+    Scratch<double> r, z, p, q, sc;
+    AMGT_TRY(r.init(a, n));
+    AMGT_TRY(z.init(a, n));
+    AMGT_TRY(p.init(a, n));
+    AMGT_TRY(q.init(a, n));
+    AMGT_TRY(sc.init(a, 4));  // rz[0], rz[1] (by iteration parity), pq
+    H->spmv_calls = 0;
+    const unsigned G = (unsigned)num_sms() * 4;
+    AMGT_TRY(counted_spmv(H, &L0.A, x, AMGT_FP64, r.p, AMGT_FP64, 0, RES, b));  // r0 = b - A x0
+    AMGT_TRY(norm_into(H, r.p, n, H->norms));
+    AMGT_TRY(precond(H, r.p, z.p));
+    AMGT_CUDA(cudaMemcpyAsync(p.p, z.p, n * sizeof(double), cudaMemcpyDeviceToDevice, s));
+    k_dot<<<NORM_BLOCKS, 256, 0, s>>>(n, r.p, z.p, H->partial, sc.p);
+    AMGT_LAUNCHED();
+    double r0 = 0.0;
+    if (rtol > 0.0) {
+        AMGT_CUDA(cudaMemcpyAsync(&r0, H->norms, sizeof(double), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+    }
+    int it = 0;
+    for (int k = 0; k < maxit; ++k) {
+        if (rtol > 0.0) {
+            double rk = 0.0;
+            AMGT_CUDA(cudaMemcpyAsync(&rk, H->norms + k, sizeof(double), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaStreamSynchronize(s));
+            if (std::sqrt(rk) <= rtol * std::sqrt(r0)) break;
+        }
+        double* rz_old = sc.p + (k & 1);
+        double* rz_new = sc.p + ((k + 1) & 1);
+        AMGT_TRY(counted_spmv(H, &L0.A, p.p, AMGT_FP64, q.p, AMGT_FP64, 0));  // q = A p
+        k_dot<<<NORM_BLOCKS, 256, 0, s>>>(n, p.p, q.p, H->partial, sc.p + 2);
+        AMGT_LAUNCHED();
+        k_pcg_xr<<<NORM_BLOCKS, 256, 0, s>>>(n, rz_old, sc.p + 2, x, r.p, p.p, q.p, H->partial, H->norms + k + 1);
+        AMGT_LAUNCHED();
+        AMGT_TRY(precond(H, r.p, z.p));
+        k_dot<<<NORM_BLOCKS, 256, 0, s>>>(n, r.p, z.p, H->partial, rz_new);
+        AMGT_LAUNCHED();
+        k_pcg_p<<<G, 256, 0, s>>>(n, rz_new, rz_old, z.p, p.p);
+        AMGT_LAUNCHED();
+        it = k + 1;
+    }
+    std::vector<double> hn(it + 1);
+    AMGT_CUDA(cudaMemcpyAsync(hn.data(), H->norms, (it + 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    if (res_host)
+        for (int k = 0; k <= it; ++k) res_host[k] = std::sqrt(hn[k]);
+    if (iters_host) *iters_host = it;
+    if (calls_host) *calls_host = H->spmv_calls;
+    return AMGT_OK;
+}
+
 }  // namespace amgt
 
 extern "C" {
@@ -802,6 +945,8 @@ amgt_status amgt_hierarchy_create(const amgt_mbsr* A, const amgt_mbsr* const* P,
     for (int k = 0; k + 1 < nlev; ++k)
         if (!P[k] || P[k]->prec != AMGT_FP64) return fail(AMGT_ERR_ARG, "P[%d] missing or not FP64", k);
     if (o->nu1 < 0 || o->nu2 < 0) return fail(AMGT_ERR_ARG, "negative sweep count");
+    if (o->smoother != AMGT_SMOOTH_JACOBI && o->smoother != AMGT_SMOOTH_L1_JACOBI)
+        return fail(AMGT_ERR_ARG, "unknown smoother %d", o->smoother);
     amgt_hierarchy* H = new amgt_hierarchy();
     H->o = *o;
     H->s = (cudaStream_t)stream;
@@ -831,6 +976,13 @@ amgt_status amgt_vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycl
     if (!H || !b || !x || ncycles < 0) return fail(AMGT_ERR_ARG, "amgt_vcycle: bad argument");
     H->s = (cudaStream_t)stream;
     return vcycle(H, b, x, ncycles, res_norms_host, spmv_calls_host);
+}
+
+amgt_status amgt_pcg(amgt_hierarchy* H, const double* b, double* x, int maxit, double rtol, double* res_norms_host,
+                     int* iters_host, int64_t* spmv_calls_host, void* stream) {
+    if (!H || !b || !x || maxit < 0 || !(rtol >= 0.0)) return fail(AMGT_ERR_ARG, "amgt_pcg: bad argument");
+    H->s = (cudaStream_t)stream;
+    return pcg(H, b, x, maxit, rtol, res_norms_host, iters_host, spmv_calls_host);
 }
 
 amgt_status amgt_dinv(const amgt_mbsr* A, int64_t diag_tile_offset, void* dinv, amgt_prec vprec, void* stream) {
@@ -866,7 +1018,7 @@ amgt_status amgt_norm2sq(int64_t n, const double* r, double* out_dev, void* stre
     Scratch<double> part;
     AMGT_TRY(part.init(a, NORM_BLOCKS + 1));
     AMGT_CUDA(cudaMemsetAsync(part.p + NORM_BLOCKS, 0, sizeof(double), s));
-    k_resnorm<<<NORM_BLOCKS, 256, 0, s>>>(n, r, part.p, out_dev);
+    k_dot<<<NORM_BLOCKS, 256, 0, s>>>(n, r, r, part.p, out_dev);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }

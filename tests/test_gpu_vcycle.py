@@ -18,17 +18,19 @@ def _amgt():
     return amgt
 
 
-def _run(kind, N, nlev, prec, ncycles):
+def _run(kind, N, nlev, prec, ncycles, smoother="jacobi", omega=2.0 / 3.0, spd_seed=None):
     amgt = _amgt()
-    A = {"7pt": gen.laplacian_7pt, "27pt": gen.laplacian_27pt, "5pt": gen.laplacian_5pt}[kind](N)
+    mk = {"7pt": gen.laplacian_7pt, "27pt": gen.laplacian_27pt, "5pt": gen.laplacian_5pt}[kind]
+    A = mk(N, spd_seed=spd_seed) if spd_seed is not None else mk(N)
     dims = (N, N) if kind == "5pt" else (N, N, N)
     PR = gen.aggregation_hierarchy(dims, nlev)
     b = gen.uniform_vector(A.m, 3)
-    H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=prec)
+    H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=prec, smoother=smoother,
+                       omega=omega)
     x = torch.zeros(A.m, dtype=torch.float64, device="cuda")
     res, calls = H.vcycle(b.cuda(), x, ncycles)
     As = oracle.build_hierarchy(A, PR)
-    xo, res_o, calls_o = oracle.vcycle(As, PR, b.numpy(), ncycles=ncycles)
+    xo, res_o, calls_o = oracle.vcycle(As, PR, b.numpy(), ncycles=ncycles, smoother=smoother, omega=omega)
     return H, As, np.array(res), np.array(res_o), calls, calls_o, x.cpu().numpy(), xo
 
 
@@ -44,6 +46,22 @@ def test_vcycle_fp64_matches_oracle(kind, N, nlev):
         assert_structure_equal(Ak, oracle.csr_to_mbsr(As[k]))
         rp, ci, v = Ak.to_csr()
         assert np.array_equal(v.cpu().numpy(), As[k].val)
+    H.close()
+
+
+@pytest.mark.parametrize("prec", [("f64",) * 8, ("f64", "f32", "f16", "f16", "f16")])
+def test_vcycle_l1_jacobi(prec):
+    """L1-Jacobi smoother (D_ii = sum_j |a_ij|, L300, w = 1 as HYPRE) on the random SPD
+    7-point variant: FP64 residual history to 1e-9, mixed precision rho within 1%."""
+    H, As, res, res_o, calls, calls_o, x, xo = _run("7pt", 32, 5, prec, 8, smoother="l1_jacobi", omega=1.0,
+                                                    spd_seed=2)
+    assert calls == calls_o
+    if prec[1] == "f64":
+        np.testing.assert_allclose(res, res_o, rtol=1e-9)
+    else:
+        rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
+        live = res_o[1:] / res_o[0] > 1e-10
+        assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
     H.close()
 
 

@@ -24,13 +24,14 @@ def _dense_levels(A, PR):
     return As, Ps, Rs
 
 
-def _E(k, As, Ps, Rs, w, nu1, nu2):
+def _E(k, As, Ps, Rs, w, nu1, nu2, l1=False):
     n = As[k].shape[0]
     I = np.eye(n)
     if k == len(As) - 1:
         return np.zeros((n, n))
-    S = I - w * np.diag(1.0 / np.diag(As[k])) @ As[k]
-    Ec = _E(k + 1, As, Ps, Rs, w, nu1, nu2)
+    D = np.abs(As[k]).sum(axis=1) if l1 else np.diag(As[k])  # L1-Jacobi: l1 row norms (L300)
+    S = I - w * np.diag(1.0 / D) @ As[k]
+    Ec = _E(k + 1, As, Ps, Rs, w, nu1, nu2, l1)
     Bc = (np.eye(As[k + 1].shape[0]) - Ec) @ np.linalg.inv(As[k + 1])
     return np.linalg.matrix_power(S, nu2) @ (I - Ps[k] @ Bc @ Rs[k] @ As[k]) @ np.linalg.matrix_power(S, nu1)
 
@@ -60,6 +61,42 @@ def test_p8_error_propagation(kind, N, nlev, nu):
     assert calls == 6 * ((2 * nu + 3) * (nlev - 1) + 1) + 1
     # convergence
     assert res[-1] < 0.2 * res[0]
+
+
+@pytest.mark.parametrize("omega", [1.0, 0.8])
+def test_l1_jacobi_error_propagation(omega):
+    """L1-Jacobi smoother (NEXT-3, L300): S = I - w D_l1^-1 A with D_l1 = diag(sum_j |a_ij|),
+    on the random SPD 7-point variant (off-diagonals not all equal)."""
+    N, nlev = 8, 3
+    A = gen.laplacian_7pt(N, spd_seed=4)
+    PR = gen.aggregation_hierarchy((N, N, N), nlev)
+    b = gen.uniform_vector(A.m, 6).numpy()
+    As_o = oracle.build_hierarchy(A, PR)
+    x, res, calls = oracle.vcycle(As_o, PR, b, ncycles=5, omega=omega, smoother="l1_jacobi")
+    As, Ps, Rs = _dense_levels(A, PR)
+    E = _E(0, As, Ps, Rs, omega, 1, 1, l1=True)
+    xs = np.linalg.solve(As[0], b)
+    xc = np.zeros(A.m)
+    exp = [np.linalg.norm(b - As[0] @ xc)]
+    for _ in range(5):
+        xc = xs - E @ (xs - xc)
+        exp.append(np.linalg.norm(b - As[0] @ xc))
+    np.testing.assert_allclose(res, exp, rtol=1e-9, atol=1e-13 * exp[0])
+    # differs from weighted Jacobi with the same weight (the D really is the l1 norm)
+    _, res_j, _ = oracle.vcycle(As_o, PR, b, ncycles=5, omega=omega)
+    assert not np.allclose(res, res_j)
+
+
+def test_l1_jacobi_diagonal_exact():
+    """On a positive diagonal matrix L1-Jacobi with w = 1 is an exact solve in one sweep."""
+    n = 16
+    d = np.arange(1, n + 1, dtype=np.float64)
+    A = gen.CSR(n, n, __import__("torch").arange(n + 1, dtype=__import__("torch").int64),
+                __import__("torch").arange(n, dtype=__import__("torch").int32), __import__("torch").from_numpy(d))
+    PR = gen.aggregation_hierarchy((4, 4), 2)
+    b = gen.uniform_vector(n, 7).numpy()
+    x, res, _ = oracle.vcycle(oracle.build_hierarchy(A, PR), PR, b, ncycles=1, omega=1.0, smoother="l1_jacobi")
+    np.testing.assert_allclose(x, b / d, rtol=1e-15)
 
 
 def test_alpha_invariance_bitwise():
