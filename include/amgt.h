@@ -247,6 +247,43 @@ amgt_status amgt_spmv_fused_range(const amgt_mbsr* A, int64_t blk_begin, int64_t
                                   amgt_prec xprec, void* y, amgt_prec yprec, int mode, const void* b, const void* dinv,
                                   const void* xs, double omega, void* stream);
 
+/*
+ * Consecutive Alg. 2 steps on one square FP64 operator in one pass over HBM (§8(f) NEXT-1).
+ * Stage s computes t = A x_s and, element-wise in FP64:
+ *   AMGT_SWEEP_J   y_s = x_s + omega * dinv .* (b - t)          (Jacobi sweep, Alg. 2 lines 2/10)
+ *   AMGT_SWEEP_JR  as J; also ||b - t||^2 -> *norm_dev            (the residual of the sweep's
+ *                  input: after a V-cycle the L308 residual of that cycle)
+ *   AMGT_SWEEP_R   y_s = b - t                                   (Alg. 2 line 3)
+ *   AMGT_SWEEP_RN  as R; also ||y_s||^2 -> *norm_dev
+ * Stage s > 0 reads x_s = y_{s-1}; outputs are distinct from every vector an earlier stage
+ * reads or writes; at most one norm stage; 1..AMGT_SWEEP_MAX_STAGES stages.  Vectors: FP64,
+ * length 4*blc_row, b and dinv shared by all stages.  Each y_s is bit-identical to the
+ * amgt_spmv_fused / amgt_spmv_fused_r result of the same step (same per-row arithmetic);
+ * the norm is a deterministic sum in a different fixed order.  One kernel: stages run as a
+ * wavefront over 64-block-row chunks with acquire/release flags, lagged so the tiles a later
+ * stage re-reads are still in L2 (A read from HBM about once).  The plan (column-chunk
+ * ranges, flags, lag) belongs to one operator; calls on one plan must be stream-ordered.
+ * amgt_sweep_plan_create: no sync.  Errors: AMGT_ERR_UNSUPPORTED (not FP64), AMGT_ERR_ARG.
+ */
+#define AMGT_SWEEP_J 1
+#define AMGT_SWEEP_JR 2
+#define AMGT_SWEEP_R 3
+#define AMGT_SWEEP_RN 4
+#define AMGT_SWEEP_MAX_STAGES 4
+typedef struct {
+    int mode;
+    const void* x;
+    void* y;
+} amgt_sweep_stage;
+typedef struct amgt_sweep_plan amgt_sweep_plan;
+amgt_status amgt_sweep_plan_create(const amgt_mbsr* A, const amgt_allocator* al, void* stream, amgt_sweep_plan** out);
+amgt_status amgt_sweep_plan_destroy(amgt_sweep_plan* P, void* stream);
+/* Diagnostics (zero unless libamgt was built with -DSW_STATS=1): summed SM cycles and counts of
+ * stage-0 items, of later-stage items, cycles spent waiting, unready polls; reset on read. Syncs. */
+amgt_status amgt_sweep_plan_stats(amgt_sweep_plan* P, uint64_t* out6_host, void* stream);
+amgt_status amgt_spmv_sweeps(amgt_sweep_plan* P, const amgt_mbsr* A, int nstages, const amgt_sweep_stage* st,
+                             const void* b, const void* dinv, double omega, double* norm_dev, void* stream);
+
 /* ------------------------------------------------ distributed-path helpers (§8(e)) */
 
 /* CSR -> mBSR with column offset: column c becomes c - col_offset, which must lie in

@@ -29,12 +29,12 @@ def _deps():
     return max(os.path.getmtime(h) for h in hdrs)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, build_dir: str = BUILD, lib: str = LIB) -> str:
+    os.makedirs(build_dir, exist_ok=True)
     hdr_t = _deps()
     objs, procs = [], []
     for src in sources():
-        obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
+        obj = os.path.join(build_dir, os.path.basename(src)[:-3] + ".o")
         objs.append(obj)
         if force or not os.path.exists(obj) or os.path.getmtime(obj) < max(os.path.getmtime(src), hdr_t):
             cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
@@ -51,18 +51,24 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if failed:
         msg = "\n".join(f"--- {s}\n{o}" for s, o in failed)
         raise RuntimeError(f"nvcc failed:\n{msg}")
-    if force or procs or not os.path.exists(LIB):
-        vs = os.path.join(BUILD, "exports.map")
+    if force or procs or not os.path.exists(lib):
+        vs = os.path.join(build_dir, "exports.map")
         with open(vs, "w") as f:
             f.write("{ global: amgt_*; local: *; };\n")
-        tmp = LIB + f".tmp{os.getpid()}"
+        tmp = lib + f".tmp{os.getpid()}"
         cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs,
                "-Xlinker", f"--version-script={vs}", "-lrt", "-lpthread", "-ldl"]
         subprocess.check_call(cmd)
-        os.replace(tmp, LIB)
-    return LIB
+        os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="-v" in sys.argv)
-    print(LIB)
+    # experiments: AMGT_NVCC_EXTRA="-DX=1" python _build.py --variant NAME -> build_NAME/, libamgt_NAME.so
+    if "--variant" in sys.argv:
+        v = sys.argv[sys.argv.index("--variant") + 1]
+        print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, build_dir=BUILD + "_" + v,
+                    lib=os.path.join(PKG, f"libamgt_{v}.so")))
+    else:
+        build(force="--force" in sys.argv, verbose="-v" in sys.argv)
+        print(LIB)

@@ -13,7 +13,7 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libamgt.so")
+LIB_PATH = os.environ.get("AMGT_LIB_PATH") or os.path.join(_HERE, "libamgt.so")  # override: kernel experiments
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built — run `python __graft_entry__.py build` "
@@ -85,6 +85,10 @@ class c_dist_coarse(ctypes.Structure):
                 ("displs", ctypes.c_void_p), ("bfull", ctypes.c_void_p), ("xfull", ctypes.c_void_p)]
 
 
+class c_sweep_stage(ctypes.Structure):
+    _fields_ = [("mode", ctypes.c_int), ("x", ctypes.c_void_p), ("y", ctypes.c_void_p)]
+
+
 _vp, _i64, _i32, _int = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_int
 _P = ctypes.POINTER
 _sigs = {
@@ -127,6 +131,10 @@ _sigs = {
     "amgt_dense_spd_inverse": (_int, [_i64, _vp, _vp]),
     "amgt_dense_matvec": (_int, [_i64, _i64, _vp, _vp, _vp, _int, _vp]),
     "amgt_norm2sq": (_int, [_i64, _vp, _vp, _vp]),
+    "amgt_sweep_plan_create": (_int, [_P(c_mbsr), _P(c_allocator), _vp, _P(_vp)]),
+    "amgt_sweep_plan_destroy": (_int, [_vp, _vp]),
+    "amgt_sweep_plan_stats": (_int, [_vp, _vp, _vp]),
+    "amgt_spmv_sweeps": (_int, [_vp, _P(c_mbsr), _int, _P(c_sweep_stage), _vp, _vp, ctypes.c_double, _vp, _vp]),
     "amgt_dist_unique_id": (_int, [_vp]),
     "amgt_dist_create": (_int, [_vp, _int, _int, _P(_vp)]),
     "amgt_dist_destroy": (_int, [_vp]),
@@ -380,6 +388,45 @@ def spmv_range(A: Mbsr, blk_begin: int, blk_end: int, x: torch.Tensor, y: torch.
     _check(_L.amgt_spmv_fused_range(ctypes.byref(A.c), int(blk_begin), int(blk_end), x.data_ptr(), xp, y.data_ptr(), yp,
                                     EPI[mode], ptr(b), ptr(dinv), ptr(xs), float(omega), _stream(stream)))
     return y
+
+
+SWEEP = {"jacobi": 1, "jacobi_res": 2, "residual": 3, "residual_norm": 4}
+
+
+class SweepPlan:
+    """amgt_sweep_plan_create / amgt_spmv_sweeps / amgt_sweep_plan_destroy (FP64 square A)."""
+
+    def __init__(self, A: Mbsr, stream=None):
+        h = ctypes.c_void_p()
+        _check(_L.amgt_sweep_plan_create(ctypes.byref(A.c), _AL, _stream(stream), ctypes.byref(h)))
+        self.h, self.A = h, A
+
+    def run(self, stages, b: torch.Tensor, dinv: torch.Tensor | None = None, omega: float = 2.0 / 3.0,
+            norm: torch.Tensor | None = None, stream=None):
+        """stages: [(mode, x, y), ...] with mode in SWEEP; norm: 1-element FP64 tensor for the
+        squared residual norm of a jacobi_res / residual_norm stage."""
+        arr = (c_sweep_stage * len(stages))(*[c_sweep_stage(SWEEP[m], x.data_ptr(), y.data_ptr())
+                                              for m, x, y in stages])
+        _check(_L.amgt_spmv_sweeps(self.h, ctypes.byref(self.A.c), len(stages), arr, b.data_ptr(),
+                                   dinv.data_ptr() if dinv is not None else None, float(omega),
+                                   norm.data_ptr() if norm is not None else None, _stream(stream)))
+
+    def stats(self) -> dict:
+        """SW_STATS builds only: per-item SM-cycle accounting since the last read."""
+        o = (ctypes.c_uint64 * 6)()
+        _check(_L.amgt_sweep_plan_stats(self.h, o, _stream(None)))
+        return dict(zip(("cyc_s0", "n_s0", "cyc_later", "n_later", "cyc_wait", "polls"), list(o)))
+
+    def close(self):
+        if self.h:
+            _L.amgt_sweep_plan_destroy(self.h, _stream(None))
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def csr_to_mbsr_ex(m, n, row_ptr, col, val, col_offset: int, prec="f64", stream=None) -> Mbsr:

@@ -40,6 +40,7 @@ struct amgt_level {
     int64_t npad = 0;         // 4 * blc_row
     amgt_prec vprec = AMGT_FP64;
     void *b = nullptr, *x = nullptr, *r = nullptr, *t = nullptr, *dinv = nullptr;  // t: ping-pong partner of x
+    void* u = nullptr;        // level 1 with the fused sweeps: third iterate buffer
 };
 
 struct amgt_hierarchy {
@@ -62,6 +63,7 @@ struct amgt_hierarchy {
     cudaGraphExec_t gexec = nullptr;
     bool graph_failed = false;
     int64_t sub_calls = 0, sub_launches = 0;
+    amgt_sweep_plan* sw = nullptr;  // level-1 fused sweeps (amgt_spmv_sweeps), when usable
     Alloc alloc() { return Alloc{has_al ? &al : nullptr, s}; }
 };
 
@@ -259,7 +261,7 @@ static bool dense_inverse(int64_t n, std::vector<double>& a, std::vector<double>
 
 static void free_level_vectors(amgt_level& L, Alloc& a) {
     const size_t vb = vbytes(L.vprec) * (size_t)L.npad;
-    for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv}) {
+    for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv, &L.u}) {
         a.put(*p, vb);
         *p = nullptr;
     }
@@ -276,6 +278,7 @@ static void destroy(amgt_hierarchy* H) {
         mbsr_release(&L.R, a);
         free_level_vectors(L, a);
     }
+    if (H->sw) amgt_sweep_plan_destroy(H->sw, H->s);
     a.put(H->Ainv, (size_t)H->nM * H->nM * sizeof(double));
     a.put(H->partial, (NORM_BLOCKS + 1) * sizeof(double));
     a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
@@ -285,6 +288,13 @@ static void destroy(amgt_hierarchy* H) {
     for (cudaEvent_t e : H->gev)
         if (e) cudaEventDestroy(e);
     delete H;
+}
+
+// AMGT_SWEEP=1 runs the level-1 SpMVs of the V-cycle as fused sweeps (amgt_spmv_sweeps); off by
+// default until they beat the separate kernels on B200
+static bool sweeps_enabled() {
+    const char* e = getenv("AMGT_SWEEP");
+    return e && !strcmp(e, "1");
 }
 
 static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nlev, const amgt_vcycle_opts* o,
@@ -316,6 +326,12 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             AMGT_CUDA(cudaMemsetAsync(*p, 0, vb, s));
         }
         AMGT_TRY(build_dinv(L, s, H->o.smoother == AMGT_SMOOTH_L1_JACOBI));
+        if (k == 0 && nlev >= 2 && sweeps_enabled() && L.A.prec == AMGT_FP64 && H->o.nu1 == 1 && H->o.nu2 == 1) {
+            L.u = a.get(vb);
+            if (!L.u) return fail(AMGT_ERR_ALLOC, "hierarchy vector allocation failed");
+            AMGT_CUDA(cudaMemsetAsync(L.u, 0, vb, s));
+            AMGT_TRY(amgt_sweep_plan_create(&L.A, H->has_al ? &H->al : nullptr, s, &H->sw));
+        }
         if (k + 1 < nlev) {
             const amgt_mbsr* Pk = P[k];
             if (Pk->m != L.A.m) return fail(AMGT_ERR_ARG, "P[%d] has %lld rows, level has %lld", k, (long long)Pk->m, (long long)L.A.m);
@@ -777,6 +793,61 @@ static amgt_status subcycle(amgt_hierarchy* H, void** xc, void** xa) {
     return AMGT_OK;
 }
 
+// Level-1 steps of Alg. 2 through amgt_spmv_sweeps (one HBM pass over A_1 for consecutive
+// SpMVs): stage s reads bufs[s] and writes bufs[s+1]; SpMV operations counted as in Alg. 2.
+static amgt_status sweeps(amgt_hierarchy* H, int n, const int* modes, void* const* bufs, const double* b,
+                          double* norm) {
+    amgt_level& L0 = H->L[0];
+    amgt_sweep_stage st[AMGT_SWEEP_MAX_STAGES];
+    for (int i = 0; i < n; ++i) {
+        st[i] = amgt_sweep_stage{modes[i], bufs[i], bufs[i + 1]};
+        H->spmv_calls += modes[i] == AMGT_SWEEP_JR ? 2 : 1;
+    }
+    return amgt_spmv_sweeps(H->sw, &L0.A, n, st, b, L0.dinv, H->o.omega, norm, H->s);
+}
+
+// V-cycles with nu1 = nu2 = 1 whose level-1 SpMVs run as fused sweeps.  Per cycle c, level 1:
+// restriction of r (line 4), levels 2..M (graph replay), interpolation + correction (lines
+// 8-9), then ONE pass: post-smoothing of cycle c (line 10) -> pre-smoothing of cycle c+1
+// (line 2) with the residual norm of cycle c (L308) -> residual of cycle c+1 (line 3).  The
+// first cycle starts with {pre-smoothing + initial residual norm, residual}; the last ends
+// with {post-smoothing, residual + norm}.  Three iterate buffers rotate (x, t, u).
+static amgt_status vcycle_sweeps(amgt_hierarchy* H, const double* b, double* x, int ncycles, void** xc, void** xa) {
+    const int M = H->nlev - 1;
+    amgt_level& L0 = H->L[0];
+    amgt_level& L1 = H->L[1];
+    void* X[3] = {x, L0.t, L0.u};
+    int cur = 0;
+    auto nx = [&](int k) { return X[(cur + k) % 3]; };
+    {
+        const int modes[2] = {AMGT_SWEEP_JR, AMGT_SWEEP_R};
+        void* bufs[3] = {nx(0), nx(1), L0.r};
+        AMGT_TRY(sweeps(H, 2, modes, bufs, b, H->norms));
+        cur = (cur + 1) % 3;
+    }
+    for (int c = 1; c <= ncycles; ++c) {
+        AMGT_TRY(counted_spmv(H, &L0.R, L0.r, L0.vprec, L1.b, L1.vprec, 0));  // line 4
+        xc[0] = nx(0);
+        if (M >= 2) AMGT_TRY(subcycle(H, xc, xa));
+        else AMGT_TRY(coarse_solve(H, xc));
+        AMGT_TRY(counted_spmv(H, &L0.P, xc[1], L1.vprec, nx(0), L0.vprec, 0, ACC));  // lines 8-9
+        if (c < ncycles) {
+            const int modes[3] = {AMGT_SWEEP_J, AMGT_SWEEP_JR, AMGT_SWEEP_R};
+            void* bufs[4] = {nx(0), nx(1), nx(2), L0.r};
+            AMGT_TRY(sweeps(H, 3, modes, bufs, b, H->norms + c));
+            cur = (cur + 2) % 3;
+        } else {
+            const int modes[2] = {AMGT_SWEEP_J, AMGT_SWEEP_RN};
+            void* bufs[3] = {nx(0), nx(1), L0.r};
+            AMGT_TRY(sweeps(H, 2, modes, bufs, b, H->norms + c));
+            cur = (cur + 1) % 3;
+        }
+    }
+    xc[0] = nx(0);
+    xa[0] = nx(1);
+    return AMGT_OK;
+}
+
 // Alg. 2 with the vector steps fused into the SpMV epilogues: each smoothing sweep is one
 // kernel (out of place, ping-pong between x and t), the residual one kernel, the
 // interpolation + correction one kernel.  SpMV calls are counted exactly as in Alg. 2.
@@ -801,7 +872,8 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
     // residual norms: ||b - A x_c|| after cycle c is delivered by cycle c+1's first
     // pre-smoothing sweep (same x, same arithmetic); only the last one needs its own SpMV
     const bool fused = M > 0 && H->o.nu1 >= 1 && L0.vprec == AMGT_FP64;
-    if (!fused || ncycles == 0) {
+    int ncycles_done = 0;
+    if ((!fused || ncycles == 0) && !(H->sw && M > 0 && ncycles > 0)) {
         AMGT_TRY(counted_spmv(H, &L0.A, xc[0], AMGT_FP64, L0.r, AMGT_FP64, 0, RES, b));
         AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms));
     }
@@ -815,7 +887,11 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
             AMGT_TRY(norm_into(H, (const double*)L0.r, L0.npad, H->norms + c));
         }
     }
-    for (int c = 1; c <= ncycles && M > 0; ++c) {
+    if (H->sw && M > 0 && ncycles > 0) {
+        AMGT_TRY(vcycle_sweeps(H, b, x, ncycles, xc, xa));
+        ncycles_done = ncycles;
+    }
+    for (int c = ncycles_done + 1; c <= ncycles && M > 0; ++c) {
         AMGT_TRY(down_level(H, 0, b, xc, xa, fused ? H->norms + (c - 1) : nullptr));  // lines 1-5, level 1
         if (M >= 2) AMGT_TRY(subcycle(H, xc, xa));          // levels 2..M (graph replay)
         else AMGT_TRY(coarse_solve(H, xc));
