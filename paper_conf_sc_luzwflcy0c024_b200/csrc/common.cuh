@@ -170,6 +170,41 @@ struct EpiArgs {
     void* r = nullptr;  // AMGT_EPI_JACOBI_RES: residual output (y's precision)
 };
 
+// ------------------------------------------------------------------ programmatic dependent launch
+// Inside a PdlScope (the V-cycle and PCG solve loops, including the CUDA-graph capture of the
+// coarse sub-cycle) the solve kernels are launched with programmatic stream serialization:
+// kernel N+1's CTAs may become resident while kernel N's last wave runs, and wait in
+// pdl_wait() (griddepcontrol.wait: kernel N complete and its writes visible) before touching
+// memory.  Every kernel launched through pdl_launch must call pdl_wait() before its first
+// global memory access.  Outside a scope (or with AMGT_PDL=0) launches are ordinary.
+bool pdl_active();
+struct PdlScope {
+    PdlScope();
+    ~PdlScope();
+};
+__device__ __forceinline__ void pdl_wait() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+template <typename... KArgs, typename... Args>
+inline void pdl_launch(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+    if (pdl_active()) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = grid;
+        cfg.blockDim = block;
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+    } else {
+        kern<<<grid, block, smem, s>>>(static_cast<KArgs>(args)...);
+    }
+}
+
 extern int g_tc_thr_spgemm;
 extern int g_tc_thr_spmv;
 

@@ -1,5 +1,6 @@
 // runtime.cu — error reporting, allocator glue, device prefix sum, timing/launch counters.
 #include <atomic>
+#include <cstdlib>
 #include <cstdarg>
 #include <mutex>
 #include <vector>
@@ -182,6 +183,19 @@ amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a,
 
 // ------------------------------------------------------------------ instrumentation
 static std::atomic<int64_t> g_launches{0};
+static thread_local int g_pdl_depth = 0;
+static bool pdl_allowed() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_PDL");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+bool pdl_active() { return g_pdl_depth > 0 && pdl_allowed(); }
+PdlScope::PdlScope() { ++g_pdl_depth; }
+PdlScope::~PdlScope() { --g_pdl_depth; }
+
 void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 void count_launches(int64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 

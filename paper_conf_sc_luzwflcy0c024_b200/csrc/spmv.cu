@@ -54,6 +54,7 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
                                                    const uint16_t* __restrict__ bmap, const MatT* __restrict__ bval,
                                                    const XT* __restrict__ x, const Epi<XT, YT, MODE> epi,
                                                    int64_t long_thr, int tc_thr) {
+    pdl_wait();
     const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t I = I0 + wid * 8 + g;  // block rows [I0, BR)
@@ -190,6 +191,7 @@ __global__ void __launch_bounds__(256) k_spmv_lanerow(int64_t I0, int64_t BR, co
                                                       const uint16_t* __restrict__ bmap,
                                                       const MatT* __restrict__ bval, const XT* __restrict__ x,
                                                       const Epi<XT, YT, MODE> epi, bool vec) {
+    pdl_wait();
     using Acc = typename AccOf<MatT>::type;
     const int64_t I = I0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (I >= BR) return;
@@ -260,6 +262,7 @@ __global__ void __launch_bounds__(256) k_spmv_chunks(int64_t nchunks, const int6
                                                      const int64_t* __restrict__ chunk_ptr,
                                                      const int32_t* __restrict__ chunk_lr,
                                                      typename AccOf<MatT>::type* __restrict__ partial) {
+    pdl_wait();
     using Acc = typename AccOf<MatT>::type;
     const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -317,6 +320,7 @@ template <typename Acc, typename XT, typename YT>
 __global__ void k_spmv_combine(int64_t nlong, const int32_t* __restrict__ long_rows,
                                const int64_t* __restrict__ chunk_ptr, const Acc* __restrict__ partial,
                                const Epi<XT, YT> epi) {
+    pdl_wait();
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= 4 * nlong) return;
     const int64_t lr = i >> 2;
@@ -472,15 +476,15 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
         auto ok = [&](const void* p) { return (reinterpret_cast<uintptr_t>(p) & al) == 0; };
         const bool vec = ok(y) && ok(ea.b) && ok(ea.dinv) && ok(ea.r) &&
                          (reinterpret_cast<uintptr_t>(ea.xs) & (4 * sizeof(XT) - 1)) == 0;
-        k_spmv_lanerow<MatT, XT, YT, MODE><<<(unsigned)ceil_div(BR - I0, 256), 256, 0, s>>>(
-            I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, epi, vec);
+        pdl_launch(k_spmv_lanerow<MatT, XT, YT, MODE>, dim3((unsigned)ceil_div(BR - I0, 256)), dim3(256), 0, s, I0, BR,
+                   A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, epi, vec);
         return;
     }
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
     const int tc = sizeof(MatT) == 8 ? g_tc_thr_spmv : 17;
     auto go = [&](auto kern) {
-        kern<<<blocks, 256, 0, s>>>(I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x,
-                                    epi, long_thr, tc);
+        pdl_launch(kern, dim3(blocks), dim3(256), 0, s, I0, BR, A->blc_ptr, A->blc_idx, A->blc_map,
+                   (const MatT*)A->blc_val, (const XT*)x, epi, long_thr, tc);
     };
     if constexpr (sizeof(MatT) == 8) {
         if (tc <= 16) {  // per-tile tensor-core route (separate instantiation)
@@ -521,12 +525,12 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
         using Acc = typename AccOf<MatT>::type;
         const Epi<XT, YT> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, ea.mode,
                               (YT*)ea.r};
-        k_spmv_chunks<MatT, XT><<<(unsigned)ceil_div(P->nchunks * 32, 256), 256, 0, s>>>(
-            P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, P->long_rows,
-            P->chunk_ptr, P->chunk_lr, (Acc*)P->partial);
+        pdl_launch(k_spmv_chunks<MatT, XT>, dim3((unsigned)ceil_div(P->nchunks * 32, 256)), dim3(256), 0, s,
+                   P->nchunks, A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x,
+                   P->long_rows, P->chunk_ptr, P->chunk_lr, (Acc*)P->partial);
         AMGT_LAUNCHED();
-        k_spmv_combine<Acc, XT, YT><<<(unsigned)ceil_div(4 * P->nlong, 256), 256, 0, s>>>(
-            P->nlong, P->long_rows, P->chunk_ptr, (const Acc*)P->partial, epi);
+        pdl_launch(k_spmv_combine<Acc, XT, YT>, dim3((unsigned)ceil_div(4 * P->nlong, 256)), dim3(256), 0, s,
+                   P->nlong, P->long_rows, P->chunk_ptr, (const Acc*)P->partial, epi);
         AMGT_LAUNCHED();
     }
     return AMGT_OK;

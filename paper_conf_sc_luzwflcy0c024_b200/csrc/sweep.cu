@@ -815,7 +815,9 @@ __global__ void __launch_bounds__(TM_THREADS, 1) k_sweep_tma(SweepArgs a, TmPlan
             const int64_t mc = m.c;
             const int ms = m.s;
             bar_named(1 + g, 32 * TM_GW);  // the group's rows written, slot no longer read
-            if (wg == 0 && lane == 0) {
+            // the publishing lane rotates over the group's warps: its release fence waits for
+            // the group's stores, and rotating spreads that stall over TM_GW items
+            if (wg == (int)((i / TM_NG) % TM_GW) && lane == 0) {
                 mbar_arrive(&empty[slot]);
                 if (norm) {
                     double p = 0.0;

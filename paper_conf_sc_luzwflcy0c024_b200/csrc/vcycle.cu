@@ -132,6 +132,7 @@ __device__ __forceinline__ void finish_sum(double s, double* __restrict__ ws, do
 // *out = a . b (a == b: ||a||^2), deterministic for a fixed grid of NORM_BLOCKS
 __global__ void __launch_bounds__(256) k_dot(int64_t n, const double* __restrict__ a, const double* __restrict__ b,
                                              double* __restrict__ ws, double* __restrict__ out) {
+    pdl_wait();
     double s = 0.0;
     const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
     if (((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15) == 0) {  // 16-byte loads
@@ -179,9 +180,23 @@ __global__ void __launch_bounds__(256) k_pcg_p(int64_t n, const double* __restri
 }
 
 // x = Ainv * b (dense FP64), one warp per row.
+// First pre-smoothing sweep from the zero initial guess of a coarse level (Alg. 2 line 2 with
+// x = 0): x = 0 + w dinv .* (b - A 0) — the Epi JACOBI expression with x = 0 and A x = 0, so
+// the result is bit-identical to the SpMV kernel's, without reading A_k or zeroing x first.
+template <typename V>
+__global__ void __launch_bounds__(256) k_jacobi0(int64_t n, const V* __restrict__ b, const V* __restrict__ dinv,
+                                                 V omega, V* __restrict__ x) {
+    pdl_wait();
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const V zero = V(0), t = V(0);
+    x[i] = zero + omega * dinv[i] * (b[i] - t);
+}
+
 template <typename V>
 __global__ void k_dense_solve(int64_t n, int64_t npad, const double* __restrict__ Ainv, const V* __restrict__ b,
                               V* __restrict__ x) {
+    pdl_wait();
     const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (row >= npad) return;
@@ -412,7 +427,7 @@ static amgt_status counted_spmv(amgt_hierarchy* H, const amgt_mbsr* M, const voi
 
 static amgt_status norm_into(amgt_hierarchy* H, const double* r, int64_t n, double* out) {
     TimerScope ts(TC_VEC, 1.0 * n * 8, H->s);
-    k_dot<<<NORM_BLOCKS, 256, 0, H->s>>>(n, r, r, H->partial, out);
+    pdl_launch(k_dot, dim3(NORM_BLOCKS), dim3(256), 0, H->s, n, r, r, H->partial, out);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
@@ -420,8 +435,8 @@ static amgt_status norm_into(amgt_hierarchy* H, const double* r, int64_t n, doub
 template <typename V>
 static amgt_status dense_solve(amgt_hierarchy* H, amgt_level& L) {
     TimerScope ts(TC_VEC, (double)H->nM * H->nM * 8, H->s);
-    k_dense_solve<V><<<(unsigned)ceil_div(L.npad * 32, 256), 256, 0, H->s>>>(H->nM, L.npad, H->Ainv, (const V*)L.b,
-                                                                           (V*)L.x);
+    pdl_launch(k_dense_solve<V>, dim3((unsigned)ceil_div(L.npad * 32, 256)), dim3(256), 0, H->s, H->nM, L.npad,
+               (const double*)H->Ainv, (const V*)L.b, (V*)L.x);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
@@ -435,8 +450,24 @@ static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** x
                               double* res_norm = nullptr) {
     amgt_level& L = H->L[k];
     const void* bk = k == 0 ? b0 : L.b;
-    if (k > 0) AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, H->s));
-    for (int i = 0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
+    int i0 = 0;
+    if (k > 0 && H->o.nu1 >= 1) {  // zero initial guess: first sweep without the SpMV (k_jacobi0)
+        TimerScope ts(TC_VEC, 3.0 * vbytes(L.vprec) * L.npad, H->s);
+        const dim3 g((unsigned)ceil_div(L.npad, 256));
+        if (L.vprec == AMGT_FP64)
+            pdl_launch(k_jacobi0<double>, g, dim3(256), 0, H->s, L.npad, (const double*)bk, (const double*)L.dinv,
+                       H->o.omega, (double*)xa[k]);
+        else
+            pdl_launch(k_jacobi0<float>, g, dim3(256), 0, H->s, L.npad, (const float*)bk, (const float*)L.dinv,
+                       (float)H->o.omega, (float*)xa[k]);
+        AMGT_LAUNCHED();
+        H->spmv_calls += 1;  // Alg. 2's sweep (its SpMV is A 0 = 0)
+        std::swap(xc[k], xa[k]);
+        i0 = 1;
+    } else if (k > 0) {
+        AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, H->s));
+    }
+    for (int i = i0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
         if (i == 0 && res_norm) {
             AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, AMGT_EPI_JACOBI_RES, bk, L.dinv, L.r));
             AMGT_TRY(norm_into(H, (const double*)L.r, L.npad, res_norm));
@@ -546,6 +577,7 @@ __device__ __forceinline__ void coop_spmv(const CoopMat& M, const VT* x, VT* y, 
 // COOP = false: a single-CTA launch for the tail levels (k0 == kb: every level block-local).
 template <typename VT, bool COOP = true>
 __global__ void __launch_bounds__(256) k_subcycle(const CoopArgs a) {
+    pdl_wait();
     namespace cg = cooperative_groups;
     auto gsync = [&]() {
         if constexpr (COOP) cg::this_grid().sync();
@@ -676,8 +708,8 @@ static amgt_status subcycle_tail(amgt_hierarchy* H, int kt) {
     CoopArgs a{};
     fill_coop_args(H, kt, a);
     a.kb = kt;
-    if (H->L[kt].vprec == AMGT_FP64) k_subcycle<double, false><<<1, 256, 0, H->s>>>(a);
-    else k_subcycle<float, false><<<1, 256, 0, H->s>>>(a);
+    if (H->L[kt].vprec == AMGT_FP64) pdl_launch(k_subcycle<double, false>, dim3(1), dim3(256), 0, H->s, a);
+    else pdl_launch(k_subcycle<float, false>, dim3(1), dim3(256), 0, H->s, a);
     AMGT_LAUNCHED();
     H->spmv_calls += (int64_t)(a.M - kt) * (H->o.nu1 + H->o.nu2 + 3);
     return AMGT_OK;
@@ -853,6 +885,7 @@ static amgt_status vcycle_sweeps(amgt_hierarchy* H, const double* b, double* x, 
 // interpolation + correction one kernel.  SpMV calls are counted exactly as in Alg. 2.
 static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncycles, double* res_host,
                           int64_t* calls_host) {
+    PdlScope pdl;  // solve kernels: programmatic dependent launch
     cudaStream_t s = H->s;
     Alloc a = H->alloc();
     if (ncycles + 1 > H->norms_cap) {
@@ -944,6 +977,7 @@ static amgt_status precond(amgt_hierarchy* H, const double* r, double* z) {
 // unless rtol > 0 asks for an early stop).  res_host[k] = ||r_k||_2, k = 0..iters.
 static amgt_status pcg(amgt_hierarchy* H, const double* b, double* x, int maxit, double rtol, double* res_host,
                        int* iters_host, int64_t* calls_host) {
+    PdlScope pdl;
     cudaStream_t s = H->s;
     Alloc a = H->alloc();
     amgt_level& L0 = H->L[0];
