@@ -74,6 +74,13 @@ def lib():
         L.oracle_cholesky_solve.restype = None
         L.oracle_cholesky_solve.argtypes = [_i64, _f64p, _f64p, _f64p]
         L.oracle_vcycle.restype = ctypes.c_int
+        L.oracle_strength_count.restype = _i64
+        L.oracle_strength_count.argtypes = [_i64, _i64p, _i32p, _f64p, ctypes.c_double, _i64p]
+        L.oracle_strength_fill.restype = None
+        L.oracle_strength_fill.argtypes = [_i64, _i64p, _i32p, _f64p, ctypes.c_double, _i64p, _i32p, _f64p]
+        L.oracle_sa_combine.restype = None
+        L.oracle_sa_combine.argtypes = [_i64, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p,
+                                        ctypes.c_double]
         _lib = L
     return _lib
 
@@ -344,3 +351,44 @@ def pcg(A, b, M, x0=None, maxit=20):
         p = z + beta * p
         rz = rz_new
     return x, res
+
+
+# ---------------------------------------------------------------- NEXT-2: SA interpolation
+def strength_filter(A, theta: float = 0.25) -> Csr:
+    """O8: A_F = A without its weak off-diagonal entries, which are lumped into the diagonal
+    (classical strength -a_ij >= theta max_k(-a_ik), str_thr of L300; reading R31)."""
+    A = as_csr(A)
+    L = lib()
+    rp = np.zeros(A.m + 1, dtype=np.int64)
+    nnz = L.oracle_strength_count(A.m, A.row_ptr, A.col, A.val, float(theta), rp)
+    if nnz < 0:
+        raise ValueError("strength filter: a row with weak entries has no diagonal entry")
+    ci = np.zeros(max(nnz, 1), dtype=np.int32)
+    v = np.zeros(max(nnz, 1), dtype=np.float64)
+    L.oracle_strength_fill(A.m, A.row_ptr, A.col, A.val, float(theta), rp, ci, v)
+    return Csr(A.m, A.n, rp, ci[:nnz], v[:nnz])
+
+
+def sa_interp(A, Pt, theta: float = 0.25, omega: float = 2.0 / 3.0) -> Csr:
+    """O9: P = (I - w D_F^-1 A_F) Pt through one SpGEMM (Alg. 1 line 4, L54; [35]): T = A_F Pt
+    (O1, keeping cancelled entries), then P_ij = Pt_ij - (w / d_i) T_ij on T's structure."""
+    AF = strength_filter(A, theta)
+    Pt = as_csr(Pt)
+    T = spgemm(AF, Pt)
+    v = np.ascontiguousarray(T.val.copy())
+    lib().oracle_sa_combine(T.m, T.row_ptr, T.col, v, Pt.row_ptr, Pt.col, Pt.val, AF.row_ptr, AF.col, AF.val,
+                            float(omega))
+    return Csr(T.m, T.n, T.row_ptr, T.col, v)
+
+
+def build_hierarchy_sa(A, Pts, theta: float = 0.25, omega: float = 2.0 / 3.0, nthreads=None):
+    """Alg. 1 with SA interpolation: per level P_k = sa_interp(A_k, Pt_k), R_k = P_k^T,
+    A_{k+1} = R_k (A_k P_k) — three SpGEMM calls per level (L54, L302).  Returns (As, PR)."""
+    As = [as_csr(A)]
+    PR = []
+    for Pt in Pts:
+        P = sa_interp(As[-1], Pt, theta, omega)
+        R = transpose(P)
+        PR.append((P, R))
+        As.append(rap(R, As[-1], P, nthreads=nthreads))
+    return As, PR

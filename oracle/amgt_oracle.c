@@ -23,6 +23,13 @@
  *                           L300), dense Cholesky on the coarsest level (R22),
  *                           records ||r||_2 per cycle and SpMV calls (L308).
  *   O7 oracle_mbsr_to_csr_* inverse of O2 (L234, L262).
+ *   O8 oracle_strength_*    strength-of-connection filter (§8(f) NEXT-2; classical strength
+ *                           with str_thr = theta, L300; reading R31): off-diagonal a_ij is
+ *                           strong iff -a_ij >= theta * max_{k!=i}(-a_ik) > 0; weak entries
+ *                           are dropped and added to the diagonal in column order.
+ *   O9 oracle_sa_combine    interpolation through one SpGEMM call (Alg. 1 line 4, L54; [35]
+ *                           L385; reading R31): P = Pt - (w / d_i) * T_ij on the structure of
+ *                           T = A_F Pt (O1), Pt the tentative (aggregation) interpolation.
  *
  * No blocking, fusion or reordering beyond the definitions.  OpenMP only splits the
  * independent outer row loop; per-row arithmetic order is fixed, so results do not
@@ -386,4 +393,71 @@ int oracle_vcycle(int nlev, const int64_t* nrows,
     free(r0); free(L);
     for (int k = 0; k < nlev; ++k) { free(bk[k]); free(xk[k]); free(rk[k]); free(tk[k]); free(dinv[k]); }
     return status;
+}
+
+/* ---------------------------------------------------------------- O8 strength filter
+ * Pass 1 (count): kept entries per row -> rp_out[0..m] (exclusive prefix).  Pass 2 (fill):
+ * the kept entries in column order; the diagonal value becomes a_ii + sum of the dropped
+ * a_ij (ascending column order).  Returns -1 if a row with dropped entries has no diagonal
+ * entry (nothing to lump into), else nnz of A_F. */
+static int oracle_strong(double aij, double mi, double theta) { return mi > 0.0 && -aij >= theta * mi; }
+
+int64_t oracle_strength_count(int64_t m, const int64_t* rp, const int32_t* ci, const double* v, double theta,
+                              int64_t* rp_out) {
+    rp_out[0] = 0;
+    for (int64_t i = 0; i < m; ++i) {
+        double mi = 0.0;
+        int has_diag = 0, dropped = 0;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p)
+            if (ci[p] != i && -v[p] > mi) mi = -v[p];
+        int64_t kept = 0;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+            if (ci[p] == i) { has_diag = 1; ++kept; }
+            else if (oracle_strong(v[p], mi, theta)) ++kept;
+            else dropped = 1;
+        }
+        if (dropped && !has_diag) return -1;
+        rp_out[i + 1] = rp_out[i] + kept;
+    }
+    return rp_out[m];
+}
+
+void oracle_strength_fill(int64_t m, const int64_t* rp, const int32_t* ci, const double* v, double theta,
+                          const int64_t* rp_out, int32_t* ci_out, double* v_out) {
+    for (int64_t i = 0; i < m; ++i) {
+        double mi = 0.0;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p)
+            if (ci[p] != i && -v[p] > mi) mi = -v[p];
+        double d = 0.0;
+        int64_t dpos = -1, q = rp_out[i];
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+            if (ci[p] == i) { dpos = q; d = v[p]; ci_out[q] = ci[p]; v_out[q] = v[p]; ++q; }
+            else if (oracle_strong(v[p], mi, theta)) { ci_out[q] = ci[p]; v_out[q] = v[p]; ++q; }
+        }
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p)  /* lump the weak entries, column order */
+            if (ci[p] != i && !oracle_strong(v[p], mi, theta)) d = d + v[p];
+        if (dpos >= 0) v_out[dpos] = d;
+    }
+}
+
+/* ---------------------------------------------------------------- O9 SA combine
+ * In place on T = A_F Pt (CSR, columns sorted): T_ij <- Pt_ij - s_i * T_ij with
+ * s_i = w / (A_F)_ii (0 when the diagonal is 0 or absent); Pt_ij = 0 where Pt has no entry.
+ * Two roundings (product, difference). */
+void oracle_sa_combine(int64_t m, const int64_t* trp, const int32_t* tci, double* tv, const int64_t* prp,
+                       const int32_t* pci, const double* pv, const int64_t* arp, const int32_t* aci,
+                       const double* av, double omega) {
+    for (int64_t i = 0; i < m; ++i) {
+        double d = 0.0;
+        for (int64_t p = arp[i]; p < arp[i + 1]; ++p)
+            if (aci[p] == i) d = av[p];
+        const double si = d != 0.0 ? omega / d : 0.0;
+        for (int64_t p = trp[i]; p < trp[i + 1]; ++p) {
+            double pt = 0.0;
+            for (int64_t q = prp[i]; q < prp[i + 1]; ++q)
+                if (pci[q] == tci[p]) pt = pv[q];
+            const double prod = si * tv[p];
+            tv[p] = pt - prod;
+        }
+    }
 }
