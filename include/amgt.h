@@ -284,6 +284,27 @@ amgt_status amgt_sweep_plan_stats(amgt_sweep_plan* P, uint64_t* out6_host, void*
 amgt_status amgt_spmv_sweeps(amgt_sweep_plan* P, const amgt_mbsr* A, int nstages, const amgt_sweep_stage* st,
                              const void* b, const void* dinv, double omega, double* norm_dev, void* stream);
 
+/*
+ * Interpolation through one SpGEMM call (Alg. 1 line 4, L54; [35] L385; §8(f) NEXT-2; reading
+ * R31 in DESIGN.md: smoothed aggregation).
+ * amgt_strength_filter: A_F = A without its weak off-diagonal entries — a_ij (i != j) is strong
+ *   iff the row has a negative off-diagonal and -a_ij >= theta * max_{k != i}(-a_ik) (classical
+ *   strength, str_thr = theta, L300) — each weak entry removed from the structure (tiles left
+ *   empty disappear) and added to the diagonal in ascending column order (row sums kept).
+ *   s_out[4*blc_row] = omega / (A_F)_ii (0 where that is 0); FP64 for FP64 operators, FP32
+ *   otherwise.  A square, any precision (FP32/FP16 arithmetic in FP32).  AF allocated with al.
+ *   Errors: AMGT_ERR_ARG if a row with weak entries has no diagonal entry.  Syncs once.
+ * amgt_sa_interp: P = (I - omega D_F^-1 A_F) Pt: A_F as above, T = A_F Pt by the mBSR SpGEMM
+ *   (amgt_spgemm_symbolic/numeric), then P_ij = Pt_ij - s_i T_ij (two roundings) on T's
+ *   structure, which contains Pt's wherever A_F has its diagonal; cancelled entries stay
+ *   (R3).  Pt (the tentative interpolation, e.g. fixed aggregation, R19) has A's precision.
+ *   P allocated with al.  Syncs (filter + symbolic).
+ */
+amgt_status amgt_strength_filter(const amgt_mbsr* A, double theta, double omega, amgt_mbsr* AF, void* s_out,
+                                 const amgt_allocator* al, void* stream);
+amgt_status amgt_sa_interp(const amgt_mbsr* A, const amgt_mbsr* Pt, double theta, double omega, amgt_mbsr* P,
+                           const amgt_allocator* al, void* stream);
+
 /* ------------------------------------------------ distributed-path helpers (§8(e)) */
 
 /* CSR -> mBSR with column offset: column c becomes c - col_offset, which must lie in
@@ -371,7 +392,15 @@ typedef struct {
     int smoother;            /* AMGT_SMOOTH_JACOBI (default): D = diag(A_k), x += omega D^-1 (b - A x);
                                 AMGT_SMOOTH_L1_JACOBI: D_ii = sum_j |a_ij| (the l1 row norm; the
                                 paper's L1_Jacobi, L300, NEXT-3), same sweep — omega = 1 is HYPRE's */
+    int interp;              /* AMGT_INTERP_GIVEN (0, default): P[k] is the interpolation itself;
+                                AMGT_INTERP_SA (1): P[k] is the tentative interpolation and the level
+                                builds P_k = amgt_sa_interp(A_k, P[k], theta, omega_p) in level-k
+                                precision — three SpGEMM calls per level (L54, L302; NEXT-2) */
+    double theta;            /* strength threshold for AMGT_INTERP_SA (paper str_thr 0.25, L300) */
+    double omega_p;          /* prolongation smoothing weight for AMGT_INTERP_SA (default 2/3) */
 } amgt_vcycle_opts;
+#define AMGT_INTERP_GIVEN 0
+#define AMGT_INTERP_SA 1
 #define AMGT_SMOOTH_JACOBI 0
 #define AMGT_SMOOTH_L1_JACOBI 1
 

@@ -68,7 +68,8 @@ class c_spmv_stats(ctypes.Structure):
 
 class c_vcycle_opts(ctypes.Structure):
     _fields_ = [("max_levels", ctypes.c_int), ("nu1", ctypes.c_int), ("nu2", ctypes.c_int), ("omega", ctypes.c_double),
-                ("level_prec", ctypes.c_int * 8), ("smoother", ctypes.c_int)]
+                ("level_prec", ctypes.c_int * 8), ("smoother", ctypes.c_int), ("interp", ctypes.c_int),
+                ("theta", ctypes.c_double), ("omega_p", ctypes.c_double)]
 
 
 class c_dist_level(ctypes.Structure):
@@ -135,6 +136,10 @@ _sigs = {
     "amgt_sweep_plan_destroy": (_int, [_vp, _vp]),
     "amgt_sweep_plan_stats": (_int, [_vp, _vp, _vp]),
     "amgt_spmv_sweeps": (_int, [_vp, _P(c_mbsr), _int, _P(c_sweep_stage), _vp, _vp, ctypes.c_double, _vp, _vp]),
+    "amgt_strength_filter": (_int, [_P(c_mbsr), ctypes.c_double, ctypes.c_double, _P(c_mbsr), _vp, _P(c_allocator),
+                                     _vp]),
+    "amgt_sa_interp": (_int, [_P(c_mbsr), _P(c_mbsr), ctypes.c_double, ctypes.c_double, _P(c_mbsr), _P(c_allocator),
+                               _vp]),
     "amgt_dist_unique_id": (_int, [_vp]),
     "amgt_dist_create": (_int, [_vp, _int, _int, _P(_vp)]),
     "amgt_dist_destroy": (_int, [_vp]),
@@ -429,6 +434,24 @@ class SweepPlan:
             pass
 
 
+def strength_filter(A: Mbsr, theta: float = 0.25, omega: float = 2.0 / 3.0, stream=None):
+    """amgt_strength_filter: (A_F, s = omega / diag(A_F))."""
+    out = Mbsr()
+    sd = torch.float64 if A.prec == FP64 else torch.float32
+    sv = torch.zeros(max(4 * A.blc_row, 1), dtype=sd, device="cuda")
+    _check(_L.amgt_strength_filter(ctypes.byref(A.c), float(theta), float(omega), ctypes.byref(out.c), sv.data_ptr(),
+                                   _AL, _stream(stream)))
+    return out, sv
+
+
+def sa_interp(A: Mbsr, Pt: Mbsr, theta: float = 0.25, omega: float = 2.0 / 3.0, stream=None) -> Mbsr:
+    """amgt_sa_interp: P = (I - omega D_F^-1 A_F) Pt through one SpGEMM call."""
+    out = Mbsr()
+    _check(_L.amgt_sa_interp(ctypes.byref(A.c), ctypes.byref(Pt.c), float(theta), float(omega), ctypes.byref(out.c),
+                             _AL, _stream(stream)))
+    return out
+
+
 def csr_to_mbsr_ex(m, n, row_ptr, col, val, col_offset: int, prec="f64", stream=None) -> Mbsr:
     out = Mbsr()
     _check(_L.amgt_csr_to_mbsr_ex(int(m), int(n), int(col.numel()), row_ptr.data_ptr(), col.data_ptr(), val.data_ptr(),
@@ -495,12 +518,15 @@ class Hierarchy:
     """amgt_hierarchy_create / amgt_vcycle / amgt_hierarchy_destroy."""
 
     def __init__(self, A: Mbsr, Ps: list, level_prec=("f64", "f32", "f16", "f16", "f16", "f16", "f16", "f16"),
-                 nu1=1, nu2=1, omega=2.0 / 3.0, smoother="jacobi", stream=None):
+                 nu1=1, nu2=1, omega=2.0 / 3.0, smoother="jacobi", interp="given", theta=0.25,
+                 omega_p=2.0 / 3.0, stream=None):
         self.nlev = len(Ps) + 1
         o = c_vcycle_opts()
         o.max_levels = self.nlev
         o.nu1, o.nu2, o.omega = int(nu1), int(nu2), float(omega)
         o.smoother = {"jacobi": 0, "l1_jacobi": 1}[smoother]
+        o.interp = {"given": 0, "sa": 1}[interp]  # "sa": Ps are tentative; P_k by amgt_sa_interp
+        o.theta, o.omega_p = float(theta), float(omega_p)
         lp = list(level_prec) + ["f16"] * 8
         for k in range(8):
             o.level_prec[k] = PREC[lp[k]]

@@ -29,6 +29,8 @@ amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* 
 amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* Cout, amgt_spgemm_info* info,
                                  Alloc& a);
 amgt_status spgemm_numeric_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a);
+amgt_status sa_interp_impl(const amgt_mbsr* A, const amgt_mbsr* Pt, double theta, double omega, amgt_mbsr* P,
+                           Alloc& a);
 
 }  // namespace amgt
 
@@ -350,7 +352,18 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
         if (k + 1 < nlev) {
             const amgt_mbsr* Pk = P[k];
             if (Pk->m != L.A.m) return fail(AMGT_ERR_ARG, "P[%d] has %lld rows, level has %lld", k, (long long)Pk->m, (long long)L.A.m);
-            AMGT_TRY(cast_impl(Pk, pk, &L.P, a));  // P_k in level k precision (copy when equal)
+            if (o->interp == AMGT_INTERP_SA) {
+                // NEXT-2 / Alg. 1 line 4: P_k = (I - w D_F^-1 A_F) Pt through one SpGEMM call
+                amgt_mbsr Pt{};
+                AMGT_TRY(cast_impl(Pk, pk, &Pt, a));
+                const double th = o->theta >= 0.0 ? o->theta : 0.25;
+                const double wp = o->omega_p > 0.0 ? o->omega_p : 2.0 / 3.0;
+                const amgt_status st = sa_interp_impl(&L.A, &Pt, th, wp, &L.P, a);
+                mbsr_release(&Pt, a);
+                AMGT_TRY(st);
+            } else {
+                AMGT_TRY(cast_impl(Pk, pk, &L.P, a));  // P_k in level k precision (copy when equal)
+            }
             AMGT_TRY(transpose_impl(&L.P, &L.R, a));  // R_k = P_k^T (Alg. 1 line 4)
             // A_{k+1} = R_k (A_k P_k): two SpGEMM calls in level k precision (Alg. 1 line 5)
             amgt_mbsr AP{}, Ac{};
