@@ -464,13 +464,23 @@ static int spmv_variant() {
     return v;
 }
 
+// AMGT_LANEROW=0: ~1-tile-per-row matrices take the group kernel too (measurement knob)
+static bool lanerow_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_LANEROW");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 template <typename MatT, typename XT, typename YT, int MODE>
 static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
                         int64_t long_thr, cudaStream_t s) {
     const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE,
                                 (YT*)ea.r};
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
-    if (P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16) {  // ~1 tile per block row
+    if (P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16 && lanerow_enabled()) {  // ~1 tile per block row
         // vector epilogue when every vector it touches is 4-element aligned
         const uintptr_t al = 4 * sizeof(YT) - 1;
         auto ok = [&](const void* p) { return (reinterpret_cast<uintptr_t>(p) & al) == 0; };

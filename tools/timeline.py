@@ -162,6 +162,10 @@ def setup(args, MA, PR, prec, out, warm):
 def solve(levels, ops, prec, out):
     """Every SpMV kind of one V-cycle per level (A_k Jacobi, R_k, P_k)."""
     for k, Ak in enumerate(levels):
+        Ak.analyze()  # the SpMV plan the hierarchy builds for every A_k, P_k, R_k
+        if k < len(ops):
+            ops[k][1].analyze()
+            ops[k][2].analyze()
         vd = torch.float64 if prec[k] == "f64" else torch.float32
         n = 4 * Ak.blc_row
         x = torch.rand(4 * Ak.blc_col, dtype=vd, device="cuda")
