@@ -1576,6 +1576,240 @@ __global__ void __launch_bounds__(256) k_numeric_group(int64_t BR, SymCtx c, con
     }
 }
 
+// ---------------------------------------------------------------- staged group kernel
+// The CUDA-core route of k_numeric_group restructured for memory-level parallelism (the
+// default when the tensor-core route is off).  Same row class (<= GROUP_NC C tiles), same
+// lane roles (lane r of the group accumulates row r of every C tile in registers), same
+// pair order and arithmetic — results are bit-identical to k_numeric_group's CUDA-core
+// route.  What changes is how operands arrive: the group takes its (A tile, B tile) pairs
+// four at a time, lane u resolving pair u of the batch (owner A tile from the cached
+// metadata of four A tiles, B position, bitmap and column), and the four lanes copy the
+// batch's eight operand tiles into shared memory with cp.async (16-B pieces, independent,
+// no registers held).  Two buffers: batch k+1 is resolved and its copies issued before
+// batch k's products are formed from shared memory, and the A-tile metadata is fetched one
+// chunk ahead, so a batch costs about one exposed memory round trip instead of four
+// dependent ones per pair (ncu on k_numeric_group: 16 warps/SM, 0.27 eligible warps per
+// scheduler, DRAM 23% of peak).
+template <typename T> struct SRow;  // row / tile reads from shared memory
+template <> struct SRow<double> {
+    static __device__ __forceinline__ void load(const double* p, double (&v)[4]) {
+        const double2 a = reinterpret_cast<const double2*>(p)[0], b = reinterpret_cast<const double2*>(p)[1];
+        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+    }
+};
+template <> struct SRow<float> {
+    static __device__ __forceinline__ void load(const float* p, float (&v)[4]) {
+        const float4 a = *reinterpret_cast<const float4*>(p);
+        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+    }
+};
+template <> struct SRow<__half> {
+    static __device__ __forceinline__ void load(const __half* p, float (&v)[4]) {
+        const uint2 u = *reinterpret_cast<const uint2*>(p);
+        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
+        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
+        v[0] = lo.x; v[1] = lo.y; v[2] = hi.x; v[3] = hi.y;
+    }
+};
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+}
+
+constexpr int STAGED_WARPS = 4;  // warps per CTA of k_numeric_staged
+
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
+    int64_t BR, SymCtx c, const T* __restrict__ aval, const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+    const int32_t* __restrict__ cidx_g, const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+    int32_t* __restrict__ big, unsigned long long* __restrict__ nbig, int32_t* __restrict__ lng,
+    unsigned long long* __restrict__ nlng, int32_t* __restrict__ mid, unsigned long long* __restrict__ nmid) {
+    constexpr int TE = 16;                       // elements per tile
+    constexpr int PIECES = TE * sizeof(T) / 16;  // 16-B pieces per tile
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
+    const unsigned gm = 0xFu << (lane & ~3);
+    constexpr int GROUP_BUF = 2 * 4 * 2 * TE;   // two buffers x 4 pairs x (A tile, B tile)
+    T* buf = reinterpret_cast<T*>(smem_raw) + ((size_t)(threadIdx.x >> 5) * 8 + g) * GROUP_BUF;
+    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (wid * 8 >= BR) return;
+    const int64_t I = wid * 8 + g;
+    int64_t c0 = 0;
+    int nC = 0;
+    if (I < BR) {
+        c0 = cptr[I];
+        nC = (int)(cptr[I + 1] - c0);
+        if (nC > GROUP_NC) {
+            if (r == 0) {
+                if (nC <= CAP) big[atomicAdd(nbig, 1ull)] = (int32_t)I;
+                else if (nC <= MIDCAP) mid[atomicAdd(nmid, 1ull)] = (int32_t)I;
+                else lng[atomicAdd(nlng, 1ull)] = (int32_t)I;
+            }
+            nC = 0;
+        }
+    }
+    int32_t cid[GROUP_NC];
+#pragma unroll
+    for (int k = 0; k < GROUP_NC; ++k) cid[k] = k < nC ? cidx_g[c0 + k] : INT_MAX;
+    Acc acc[GROUP_NC][4];
+#pragma unroll
+    for (int k = 0; k < GROUP_NC; ++k)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) acc[k][e] = Acc(0);
+    // A-tile chunk cache: lane u holds tile cbase+u (bitmap, B-row start, exclusive pair
+    // offset); the next chunk's column / bitmap are prefetched one chunk ahead (pK, pma).
+    int64_t cbase = 0, a1 = 0, myb0 = 0;
+    int myE = 0, S = 0, pos = 0;
+    uint32_t mycma = 0, pma = 0;
+    int32_t pK = -1;
+    auto prefetch = [&](int64_t base) {
+        const int64_t tt = base + r;
+        pK = -1;
+        if (tt < a1) {
+            pK = c.aidx[tt];
+            pma = c.amap[tt];
+        }
+    };
+    auto load_chunk = [&](int64_t base) {  // consumes the prefetched metadata of `base`
+        cbase = base;
+        int len = 0;
+        myb0 = 0;
+        mycma = 0;
+        if (pK >= 0) {
+            mycma = pma;
+            myb0 = c.bptr[pK];
+            len = (int)(c.bptr[pK + 1] - myb0);
+        }
+        int incl = len, y = __shfl_up_sync(gm, incl, 1, 4);
+        if (r >= 1) incl += y;
+        y = __shfl_up_sync(gm, incl, 2, 4);
+        if (r >= 2) incl += y;
+        myE = incl - len;
+        S = __shfl_sync(gm, incl, 3, 4);
+        pos = 0;
+        prefetch(base + 4);
+    };
+    if (nC > 0) {
+        a1 = c.aptr[I + 1];
+        const int64_t a0 = c.aptr[I];
+        prefetch(a0);
+        load_chunk(a0);
+    }
+    // Batch = the group's next 4 pairs: lane u resolves pair u (A tile, B tile, bitmap,
+    // column; the bitmap/column loads stay in flight until the batch is computed) and the
+    // group issues the cp.async copies of the 8 operand tiles into buffer `nb`.
+    struct Batch {
+        bool valid;
+        uint32_t ma;
+        int64_t j;
+    };
+    auto issue = [&](int nb, Batch& B, uint32_t& bm, int32_t& bj) {
+        while (pos >= S && cbase + 4 < a1) load_chunk(cbase + 4);  // group-uniform
+        const bool has = pos < S;
+        const int p = pos + r;
+        B.valid = has && p < S;
+        const int E1 = __shfl_sync(gm, myE, 1, 4), E2 = __shfl_sync(gm, myE, 2, 4), E3 = __shfl_sync(gm, myE, 3, 4);
+        const int o = (p >= E1) + (p >= E2) + (p >= E3);
+        const int64_t ob0 = __shfl_sync(gm, myb0, o, 4);
+        const int oE = __shfl_sync(gm, myE, o, 4);
+        B.ma = __shfl_sync(gm, mycma, o, 4);
+        const int64_t tu = cbase + o;
+        B.j = ob0 + (p - oE);
+        bm = 0;
+        bj = 0;
+        if (B.valid) {
+            bm = c.bmap[B.j];
+            bj = c.bidx[B.j];
+        }
+        T* bb = buf + nb * (GROUP_BUF / 2);
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const int src = (lane & ~3) + v;
+            const bool vv = __shfl_sync(0xffffffffu, B.valid, src);
+            const int64_t tv = __shfl_sync(0xffffffffu, tu, src);
+            const int64_t jv = __shfl_sync(0xffffffffu, B.j, src);
+            if (vv) {
+#pragma unroll
+                for (int k = r; k < 2 * PIECES; k += 4) {
+                    const bool isB = k >= PIECES;
+                    const int pc = isB ? k - PIECES : k;
+                    const T* srcp = (isB ? bval + 16 * jv : aval + 16 * tv) + pc * (16 / sizeof(T));
+                    cp_async16(bb + (v * 2 + (isB ? 1 : 0)) * TE + pc * (16 / sizeof(T)), srcp);
+                }
+            }
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        if (has) pos += 4;
+        return has;
+    };
+    Batch cur, nxt;
+    uint32_t cbm, nbm;
+    int32_t cbj, nbj;
+    bool chas = issue(0, cur, cbm, cbj);
+    for (int k = 0;; ++k) {
+        if (!__any_sync(0xffffffffu, chas)) break;
+        const bool nhas = issue((k + 1) & 1, nxt, nbm, nbj);
+        asm volatile("cp.async.wait_group 1;" ::: "memory");  // batch k's copies have landed
+        __syncwarp();
+        uint32_t mC = 0;
+        int q = 0;
+        if (cur.valid) {
+            mC = bitmap_multiply(cur.ma, cbm);
+#pragma unroll
+            for (int kk = 0; kk < GROUP_NC; ++kk) q = (cid[kk] == cbj) ? kk : q;
+        }
+        const T* bb = buf + (k & 1) * (GROUP_BUF / 2);
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const uint32_t mv = __shfl_sync(0xffffffffu, mC, (lane & ~3) + v);
+            const int qv = __shfl_sync(0xffffffffu, q, (lane & ~3) + v);
+            if (mv) {  // lane r: row r of A_t * B_j, same FMA order as k_numeric_group
+                Acc arow[4], b0[4], b1[4], b2[4], b3[4], w[4];
+                const T* at = bb + (v * 2) * TE;
+                const T* bt = at + TE;
+                SRow<T>::load(at + 4 * r, arow);
+                SRow<T>::load(bt, b0);
+                SRow<T>::load(bt + 4, b1);
+                SRow<T>::load(bt + 8, b2);
+                SRow<T>::load(bt + 12, b3);
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    Acc s_ = arow[0] * b0[e];
+                    s_ = fma(arow[1], b1[e], s_);
+                    s_ = fma(arow[2], b2[e], s_);
+                    s_ = fma(arow[3], b3[e], s_);
+                    w[e] = s_;
+                }
+#pragma unroll
+                for (int kk = 0; kk < GROUP_NC; ++kk)
+                    if (kk == qv)
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) acc[kk][e] += w[e];
+            }
+        }
+        __syncwarp();  // buffer k&1 is refilled by the next issue
+        cur = nxt;
+        cbm = nbm;
+        cbj = nbj;
+        chas = nhas;
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+#pragma unroll
+    for (int k = 0; k < GROUP_NC; ++k) {
+        if (k < nC) {
+            const uint32_t nib = (cmap_g[c0 + k] >> (4 * r)) & 0xFu;
+            Acc o[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? acc[k][e] : Acc(0);
+            if constexpr (sizeof(T) == 8)
+                group_store_tile_f64((double*)(cval + 16 * (c0 + k)), o, r, gm, lane & ~3);
+            else
+                RowIO<T>::store(cval + 16 * (c0 + k) + 4 * r, o);
+        }
+    }
+}
+
 static unsigned capped(int64_t blocks) {
     const int64_t cap = (int64_t)num_sms() * 32;
     return (unsigned)(blocks < 1 ? 1 : (blocks > cap ? cap : blocks));
@@ -1756,9 +1990,25 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     // [warp rows, long rows, long-row item cursor (pass 0), mid rows, mid-row cursor, long cursor (pass 1)]
     AMGT_TRY(nbig.init(a, 6));
     AMGT_CUDA(cudaMemsetAsync(nbig.p, 0, 6 * sizeof(unsigned long long), s));
-    k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
-        BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val, big.p,
-        nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, g_tc_thr_spgemm);
+    // tensor-core route off (every tile on CUDA cores): the staged kernel; else the kernel
+    // with the DMMA / HMMA routes.  AMGT_NUM_STAGED=0 forces the latter (measurement).
+    static const int staged_env = [] { const char* e = getenv("AMGT_NUM_STAGED"); return e ? atoi(e) : 1; }();
+    const bool tc_route = (sizeof(T) == 8 || sizeof(T) == 2) && g_tc_thr_spgemm <= 16;
+    if (!tc_route && staged_env) {
+        constexpr size_t sm = (size_t)STAGED_WARPS * 8 * 2 * 4 * 2 * 16 * sizeof(T);
+        static bool attr = false;
+        if (!attr && sm > 48 * 1024) {
+            AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        }
+        attr = true;
+        k_numeric_staged<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8), STAGED_WARPS), STAGED_WARPS * 32, sm, s>>>(
+            BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
+            big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3);
+    } else {
+        k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
+            BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
+            big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, g_tc_thr_spgemm);
+    }
     AMGT_LAUNCHED();
     // row classes present (C->row_max from symbolic; 0 = unknown: launch everything)
     const int64_t rmax = C->row_max > 0 ? C->row_max : INT64_MAX;
