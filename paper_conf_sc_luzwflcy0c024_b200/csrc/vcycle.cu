@@ -717,7 +717,285 @@ static int tail_level(const amgt_hierarchy* H, void** xc, void** xa) {
     return kt;
 }
 
+// ---------------------------------------------------------------- shared-memory tail
+// The tail levels kt..M (a few hundred rows and below) are latency-bound: every Alg. 2 step
+// is a handful of dependent L2 round trips whatever the work.  k_tail_smem stages the tail's
+// operators (A_k, P_k, R_k in mBSR, D^-1_k, the dense coarsest inverse) and b_kt into the
+// shared memory of ONE CTA with independent 16-B loads, runs every step of levels kt..M
+// (Alg. 2 lines 1-11) from shared memory with block barriers, and writes x_kt back.  The
+// SpMV is one thread per scalar row, walking the block row's tiles in column order with
+// the bitmap predicate (Alg. 5 GETBIT) — for FP32/FP16 operators the accumulation order and
+// arithmetic of k_spmv_rows, so those levels are bit-identical to the global-memory path.
+struct SmMat {
+    int64_t ptr, idx, map, val;  // shared-memory byte offsets
+    int64_t BR;
+    int prec;
+};
+struct SmLevel {
+    SmMat A, P, R;
+    int64_t b, x, t, r, dinv;  // byte offsets of the level vectors
+    int64_t npad;
+};
+struct SmSeg {
+    const void* src;
+    int64_t off, bytes;
+};
+constexpr int SM_MAXSEG = 48;
+struct SmTailArgs {
+    SmLevel L[8];
+    SmSeg seg[SM_MAXSEG];
+    int64_t pre[SM_MAXSEG + 1];  // prefix of the 16-B chunk counts of the segments
+    int nseg, kt, M, nu1, nu2;
+    double omega;
+    int64_t nM, ainv;
+    void* xout;  // x_kt in global memory
+};
+
+// y_i = epi(i, (A x)_i) for the 4*BR rows of an mBSR operator held in shared memory
+template <typename VT, typename F>
+__device__ __forceinline__ void sm_spmv(const unsigned char* sm, const SmMat& M, const VT* x, F&& epi) {
+    const int64_t* ptr = reinterpret_cast<const int64_t*>(sm + M.ptr);
+    const int32_t* idx = reinterpret_cast<const int32_t*>(sm + M.idx);
+    const uint16_t* map = reinterpret_cast<const uint16_t*>(sm + M.map);
+    for (int64_t i = threadIdx.x; i < 4 * M.BR; i += blockDim.x) {
+        const int64_t I = i >> 2;
+        const int r = (int)(i & 3);
+        const int64_t t0 = ptr[I], t1 = ptr[I + 1];
+        if (M.prec == AMGT_FP64) {
+            const double* val = reinterpret_cast<const double*>(sm + M.val);
+            double acc = 0.0;
+            for (int64_t t = t0; t < t1; ++t) {
+                const uint32_t nib = (map[t] >> (4 * r)) & 0xFu;
+                if (!nib) continue;
+                const int64_t J = idx[t];
+#pragma unroll
+                for (int c = 0; c < 4; ++c)
+                    if ((nib >> c) & 1u) acc = fma(val[16 * t + 4 * r + c], (double)x[4 * J + c], acc);
+            }
+            epi(i, acc);
+        } else {
+            float acc = 0.f;
+            for (int64_t t = t0; t < t1; ++t) {
+                const uint32_t nib = (map[t] >> (4 * r)) & 0xFu;
+                if (!nib) continue;
+                const int64_t J = idx[t];
+                float a[4];
+                if (M.prec == AMGT_FP32) {
+                    const float4 v = *reinterpret_cast<const float4*>(sm + M.val + 4 * (16 * t + 4 * r));
+                    a[0] = v.x; a[1] = v.y; a[2] = v.z; a[3] = v.w;
+                } else {
+                    const uint2 w = *reinterpret_cast<const uint2*>(sm + M.val + 2 * (16 * t + 4 * r));
+                    const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
+                    const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
+                    a[0] = lo.x; a[1] = lo.y; a[2] = hi.x; a[3] = hi.y;
+                }
+#pragma unroll
+                for (int c = 0; c < 4; ++c)
+                    if ((nib >> c) & 1u) acc = fmaf(a[c], (float)x[4 * J + c], acc);
+            }
+            epi(i, acc);
+        }
+    }
+}
+
+template <typename VT>
+__global__ void __launch_bounds__(512) k_tail_smem(const SmTailArgs a) {
+    pdl_wait();
+    extern __shared__ __align__(16) unsigned char sm[];
+    {  // stage: all segments as one flat list of 16-B chunks, four loads in flight per thread
+        const int64_t n = a.pre[a.nseg];
+        for (int64_t c0 = threadIdx.x; c0 < n; c0 += 4 * (int64_t)blockDim.x) {
+            uint4 v[4];
+            int64_t dst[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int64_t c = c0 + (int64_t)u * blockDim.x;
+                dst[u] = -1;
+                if (c < n) {
+                    int lo = 0, hi = a.nseg - 1;  // segment: largest s with pre[s] <= c
+                    while (lo < hi) {
+                        const int mid = (lo + hi + 1) >> 1;
+                        if (a.pre[mid] <= c) lo = mid; else hi = mid - 1;
+                    }
+                    const int64_t k = c - a.pre[lo];
+                    v[u] = __ldcg(reinterpret_cast<const uint4*>(a.seg[lo].src) + k);
+                    dst[u] = a.seg[lo].off + 16 * k;
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                if (dst[u] >= 0) *reinterpret_cast<uint4*>(sm + dst[u]) = v[u];
+        }
+        // remainders (< 16 B, whole 4-B words) of the segments
+        for (int s = threadIdx.x; s < a.nseg; s += blockDim.x) {
+            const SmSeg g = a.seg[s];
+            for (int64_t w = (g.bytes >> 4) << 2; w < (g.bytes >> 2); ++w)
+                reinterpret_cast<uint32_t*>(sm + g.off)[w] = __ldcg(reinterpret_cast<const uint32_t*>(g.src) + w);
+        }
+    }
+    __syncthreads();
+    const VT om = (VT)a.omega;
+    auto V = [&](int64_t off) { return reinterpret_cast<VT*>(sm + off); };
+    int64_t xo[8], to[8];  // current / partner buffer of each level
+    for (int k = a.kt; k < a.M; ++k) {  // Alg. 2 lines 1-5
+        const SmLevel& L = a.L[k];
+        xo[k] = L.x;
+        to[k] = L.t;
+        const VT* b = V(L.b);
+        const VT* dv = V(L.dinv);
+        if (a.nu1 >= 1) {  // first sweep from x = 0 (the k_jacobi0 expression)
+            VT* x = V(xo[k]);
+            for (int64_t i = threadIdx.x; i < L.npad; i += blockDim.x) {
+                const VT zero = VT(0), t = VT(0);
+                x[i] = zero + om * dv[i] * (b[i] - t);
+            }
+        } else {
+            for (int64_t i = threadIdx.x; i < L.npad; i += blockDim.x) V(xo[k])[i] = VT(0);
+        }
+        __syncthreads();
+        for (int s = 1; s < a.nu1; ++s) {
+            const VT* x = V(xo[k]);
+            VT* y = V(to[k]);
+            sm_spmv<VT>(sm, L.A, x, [&](int64_t i, auto v) { y[i] = x[i] + om * dv[i] * (b[i] - (VT)v); });
+            __syncthreads();
+            const int64_t tmp = xo[k]; xo[k] = to[k]; to[k] = tmp;
+        }
+        {  // line 3: r = b - A x
+            VT* r = V(L.r);
+            sm_spmv<VT>(sm, L.A, V(xo[k]), [&](int64_t i, auto v) { r[i] = b[i] - (VT)v; });
+        }
+        __syncthreads();
+        {  // line 4: b_{k+1} = R r
+            VT* bn = V(a.L[k + 1].b);
+            sm_spmv<VT>(sm, L.R, V(L.r), [&](int64_t i, auto v) { bn[i] = (VT)v; });
+        }
+        __syncthreads();
+    }
+    {  // line 6: x_M = A_M^-1 b_M (dense FP64)
+        const SmLevel& C = a.L[a.M];
+        const VT* bM = V(C.b);
+        VT* xM = V(C.x);
+        const double* Ai = reinterpret_cast<const double*>(sm + a.ainv);
+        xo[a.M] = C.x;
+        for (int64_t row = threadIdx.x; row < C.npad; row += blockDim.x) {
+            double acc = 0.0;
+            if (row < a.nM)
+                for (int64_t j = 0; j < a.nM; ++j) acc = fma(Ai[row * a.nM + j], (double)bM[j], acc);
+            xM[row] = (VT)acc;
+        }
+    }
+    __syncthreads();
+    for (int k = a.M - 1; k >= a.kt; --k) {  // lines 7-11
+        const SmLevel& L = a.L[k];
+        {  // lines 8-9: x += P x_{k+1}
+            VT* x = V(xo[k]);
+            sm_spmv<VT>(sm, L.P, V(xo[k + 1]), [&](int64_t i, auto v) { x[i] = x[i] + (VT)v; });
+        }
+        __syncthreads();
+        const VT* b = V(L.b);
+        const VT* dv = V(L.dinv);
+        for (int s = 0; s < a.nu2; ++s) {  // line 10
+            const VT* x = V(xo[k]);
+            VT* y = V(to[k]);
+            sm_spmv<VT>(sm, L.A, x, [&](int64_t i, auto v) { y[i] = x[i] + om * dv[i] * (b[i] - (VT)v); });
+            __syncthreads();
+            const int64_t tmp = xo[k]; xo[k] = to[k]; to[k] = tmp;
+        }
+    }
+    VT* out = reinterpret_cast<VT*>(a.xout);
+    const VT* xk = V(xo[a.kt]);
+    for (int64_t i = threadIdx.x; i < a.L[a.kt].npad; i += blockDim.x) out[i] = xk[i];
+}
+
+// Plans the shared-memory tail of levels kt..M; false when it does not fit (or too many
+// segments): the caller then uses the global-memory tail kernel.
+static bool plan_tail_smem(const amgt_hierarchy* H, int kt, void* xout, SmTailArgs& a, size_t& bytes) {
+    static int budget = -1;
+    if (budget < 0) {
+        int dev = 0, optin = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        const char* e = getenv("AMGT_TAIL_SMEM");
+        budget = e ? atoi(e) : std::min(optin, 200 * 1024);
+    }
+    if (budget <= 0) return false;
+    const int M = H->nlev - 1;
+    a = SmTailArgs{};
+    int64_t cur = 0;
+    auto place = [&](int64_t nb) {
+        const int64_t off = (cur + 15) & ~int64_t(15);
+        cur = off + nb;
+        return off;
+    };
+    auto stage = [&](const void* src, int64_t nb) -> int64_t {
+        const int64_t off = place(nb);
+        if (a.nseg < SM_MAXSEG && nb > 0) {
+            a.seg[a.nseg] = SmSeg{src, off, nb};
+            a.pre[a.nseg + 1] = a.pre[a.nseg] + (nb >> 4);
+            ++a.nseg;
+        } else if (nb > 0) {
+            a.nseg = SM_MAXSEG + 1;  // overflow marker
+        }
+        return off;
+    };
+    auto mat = [&](const amgt_mbsr& X) {
+        SmMat m{};
+        m.BR = X.blc_row;
+        m.prec = (int)X.prec;
+        m.ptr = stage(X.blc_ptr, (X.blc_row + 1) * 8);
+        m.idx = stage(X.blc_idx, X.blc_num * 4);
+        m.map = stage(X.blc_map, ((X.blc_num + 1) & ~int64_t(1)) * 2);
+        m.val = stage(X.blc_val, 16 * X.blc_num * (int64_t)prec_bytes(X.prec));
+        return m;
+    };
+    const size_t vs = vbytes(H->L[kt].vprec);
+    for (int k = kt; k <= M; ++k) {
+        const amgt_level& L = H->L[k];
+        if (L.vprec != H->L[kt].vprec) return false;
+        SmLevel& s = a.L[k];
+        s.npad = L.npad;
+        const int64_t vb = (int64_t)vs * L.npad;
+        s.b = k == kt ? stage(L.b, vb) : place(vb);
+        s.x = place(vb);
+        s.t = place(vb);
+        if (k < M) {
+            s.r = place(vb);
+            s.dinv = stage(L.dinv, vb);
+            s.A = mat(L.A);
+            s.P = mat(L.P);
+            s.R = mat(L.R);
+        }
+    }
+    a.ainv = stage(H->Ainv, H->nM * H->nM * 8);
+    if (a.nseg > SM_MAXSEG || cur > budget) return false;
+    a.kt = kt;
+    a.M = M;
+    a.nu1 = H->o.nu1;
+    a.nu2 = H->o.nu2;
+    a.omega = H->o.omega;
+    a.nM = H->nM;
+    a.xout = xout;
+    bytes = (size_t)cur;
+    return true;
+}
+
 static amgt_status subcycle_tail(amgt_hierarchy* H, int kt) {
+    {
+        SmTailArgs* sa = new SmTailArgs();
+        size_t bytes = 0;
+        const bool ok = plan_tail_smem(H, kt, H->L[kt].x, *sa, bytes);
+        if (ok) {
+            const bool f64 = H->L[kt].vprec == AMGT_FP64;
+            auto kern = f64 ? k_tail_smem<double> : k_tail_smem<float>;
+            AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+            pdl_launch(kern, dim3(1), dim3(512), bytes, H->s, *sa);
+            delete sa;
+            AMGT_LAUNCHED();
+            H->spmv_calls += (int64_t)(H->nlev - 1 - kt) * (H->o.nu1 + H->o.nu2 + 3);
+            return AMGT_OK;
+        }
+        delete sa;
+    }
     CoopArgs a{};
     fill_coop_args(H, kt, a);
     a.kb = kt;
