@@ -187,7 +187,11 @@ amgt_status amgt_rap(const amgt_mbsr* R, const amgt_mbsr* A, const amgt_mbsr* P,
  * variation (coefficient of variation of tiles per block row, R11) and the
  * load-balancing work list (block rows longer than 64 tiles are split into chunks of
  * WARP_CAPACITY = 64 tiles, Alg. 5, R12).  Stored in A->aux (freed by amgt_mbsr_free).
- * Without it amgt_spmv still works (no row splitting).  Syncs once.
+ * Without it amgt_spmv still works (no row splitting).  Syncs once — except when A->row_max
+ * is known (set by conversion, SpGEMM symbolic, transpose inside amgt_hierarchy_create;
+ * kept by cast) and <= 64: then nothing needs splitting, the call launches nothing and
+ * returns at once, and the statistics below are computed (one sync on the legacy default
+ * stream) by the first amgt_spmv_get_stats.
  */
 amgt_status amgt_spmv_analyze(amgt_mbsr* A, const amgt_allocator* al, void* stream);
 

@@ -150,6 +150,10 @@ enum TimerClass : int {
     TC_VEC = 7
 };
 void count_launch();
+void trace_point(const char* name, cudaStream_t s);  // AMGT_TRACE=1 only (measurement)
+constexpr int PINNED_SLOTS = 64;
+int64_t* pinned_slots();  // per-thread pinned host int64[PINNED_SLOTS], NULL if unavailable
+void trace_dump();
 struct TimerScope {  // records start/end events on `s` when timing is enabled
     int cls;
     double bytes;

@@ -343,6 +343,8 @@ __global__ void k_tr_gather(int64_t T_, const int64_t* __restrict__ perm, const 
     }
 }
 
+__global__ void k_max_rows(int64_t BR, const int64_t* __restrict__ nrow, unsigned long long* __restrict__ out);  // spgemm.cu
+
 static unsigned grid_for(int64_t work, int threads) {
     int64_t b = ceil_div(work, threads);
     int64_t cap = (int64_t)num_sms() * 16;
@@ -442,10 +444,19 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     M.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
     if (!M.blc_ptr) return fail(AMGT_ERR_ALLOC, "blc_ptr allocation failed");
     AMGT_TRY(scan_exclusive(cnt.p, M.blc_ptr, BR, a, s));
+    Scratch<unsigned long long> rmax;  // longest block row (lets the SpMV analysis skip its sync)
+    AMGT_TRY(rmax.init(a, 1));
+    AMGT_CUDA(cudaMemsetAsync(rmax.p, 0, sizeof(unsigned long long), s));
+    if (BR > 0) {
+        k_max_rows<<<grid_for(BR, 256), 256, 0, s>>>(BR, cnt.p, rmax.p);
+        AMGT_LAUNCHED();
+    }
     int64_t hT[1] = {0};
     uint32_t hflag = 0;
+    unsigned long long hmax = 0;
     AMGT_CUDA(cudaMemcpyAsync(hT, M.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     AMGT_CUDA(cudaMemcpyAsync(&hflag, flag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax.p, sizeof(hmax), cudaMemcpyDeviceToHost, s));
     AMGT_CUDA(cudaStreamSynchronize(s));
     if (hflag & FLAG_FORMAT) {
         a.put(M.blc_ptr, (BR + 1) * sizeof(int64_t));
@@ -454,6 +465,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     const int64_t T = hT[0];
     amgt_status st = mbsr_alloc(&M, m, n, T, prec, a, true, true, M.blc_ptr);
     if (st != AMGT_OK) { mbsr_release(&M, a); return st; }
+    M.row_max = (int64_t)hmax;
     {
         const double bytes = bytes_in + T * (16.0 * prec_bytes(prec) + 6.0) + (BR + 1) * 8.0;
         TimerScope ts(TC_CSR2MBSR, bytes, s);
@@ -527,7 +539,9 @@ amgt_status mbsr_to_csr_impl(const amgt_mbsr* A, int64_t* rp, int32_t* ci, doubl
     return AMGT_OK;
 }
 
-amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& a) {
+// dflag (optional, device): the FP16 range flag is OR-ed there and NOT read back (no sync);
+// the caller checks it after a later synchronisation (amgt_hierarchy_create)
+amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& a, uint32_t* dflag) {
     cudaStream_t s = a.s;
     if (prec_bytes(to) > prec_bytes(in->prec)) return fail(AMGT_ERR_ARG, "cast must not widen (from %d to %d)", in->prec, to);
     amgt_mbsr M = *in;
@@ -538,9 +552,13 @@ amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& 
     M.blc_val = a.get(n * prec_bytes(to));
     if (!M.blc_val) return fail(AMGT_ERR_ALLOC, "cast value allocation failed");
     M.own = 2u;
-    Scratch<uint32_t> flag;
-    AMGT_TRY(flag.init(a, 1));
-    AMGT_CUDA(cudaMemsetAsync(flag.p, 0, sizeof(uint32_t), s));
+    Scratch<uint32_t> own_flag;
+    uint32_t* fl = dflag;
+    if (!fl) {
+        AMGT_TRY(own_flag.init(a, 1));
+        AMGT_CUDA(cudaMemsetAsync(own_flag.p, 0, sizeof(uint32_t), s));
+        fl = own_flag.p;
+    }
     {
         TimerScope ts(TC_CAST, (double)n * (prec_bytes(in->prec) + prec_bytes(to)), s);
         if (n > 0) {
@@ -548,20 +566,20 @@ amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& 
             if (in->prec == to) {
                 AMGT_CUDA(cudaMemcpyAsync(M.blc_val, in->blc_val, n * prec_bytes(to), cudaMemcpyDeviceToDevice, s));
             } else if (in->prec == AMGT_FP64 && to == AMGT_FP32) {
-                k_cast<double, float><<<g, 256, 0, s>>>(n, (const double*)in->blc_val, (float*)M.blc_val, flag.p);
+                k_cast<double, float><<<g, 256, 0, s>>>(n, (const double*)in->blc_val, (float*)M.blc_val, fl);
                 AMGT_LAUNCHED();
             } else if (in->prec == AMGT_FP64 && to == AMGT_FP16) {
-                k_cast<double, __half><<<g, 256, 0, s>>>(n, (const double*)in->blc_val, (__half*)M.blc_val, flag.p);
+                k_cast<double, __half><<<g, 256, 0, s>>>(n, (const double*)in->blc_val, (__half*)M.blc_val, fl);
                 AMGT_LAUNCHED();
             } else {
-                k_cast<float, __half><<<g, 256, 0, s>>>(n, (const float*)in->blc_val, (__half*)M.blc_val, flag.p);
+                k_cast<float, __half><<<g, 256, 0, s>>>(n, (const float*)in->blc_val, (__half*)M.blc_val, fl);
                 AMGT_LAUNCHED();
             }
         }
     }
-    if (to == AMGT_FP16 && in->prec != AMGT_FP16) {
+    if (to == AMGT_FP16 && in->prec != AMGT_FP16 && !dflag) {
         uint32_t hflag = 0;
-        AMGT_TRY(read_flag(flag.p, s, &hflag));
+        AMGT_TRY(read_flag(fl, s, &hflag));
         if (hflag & FLAG_RANGE) {
             a.put(M.blc_val, n * prec_bytes(to));
             return fail(AMGT_ERR_RANGE, "value exceeds the FP16 range (65504)");
@@ -577,7 +595,9 @@ static void launch_tr_gather(const amgt_mbsr* in, const int64_t* perm, amgt_mbsr
                                                              o->blc_map, (T*)o->blc_val);
 }
 
-amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a) {
+// dmax (optional, device): atomicMax of the longest block row of the transpose, for callers
+// that read it after a later synchronisation (amgt_hierarchy_create)
+amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a, unsigned long long* dmax) {
     cudaStream_t s = a.s;
     amgt_mbsr M{};
     AMGT_TRY(mbsr_alloc(&M, in->n, in->m, in->blc_num, in->prec, a, true, true, nullptr));
@@ -593,6 +613,10 @@ amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a) {
         AMGT_LAUNCHED();
     }
     AMGT_TRY(scan_exclusive((const int64_t*)cnt.p, M.blc_ptr, BRo, a, s));
+    if (dmax && BRo > 0) {
+        k_max_rows<<<grid_for(BRo, 256), 256, 0, s>>>(BRo, (const int64_t*)cnt.p, dmax);
+        AMGT_LAUNCHED();
+    }
     AMGT_CUDA(cudaMemsetAsync(cnt.p, 0, (BRo + 1) * sizeof(unsigned long long), s));
     if (T > 0) {
         k_tr_scatter<<<grid_for(in->blc_row, 128), 128, 0, s>>>(in->blc_row, in->blc_ptr, in->blc_idx, M.blc_ptr, cnt.p,
@@ -717,7 +741,7 @@ amgt_status amgt_mbsr_to_csr(const amgt_mbsr* A, int64_t* row_ptr, int32_t* col_
 amgt_status amgt_mbsr_cast(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, const amgt_allocator* al, void* stream) {
     if (!in || !out || !prec_valid(to)) return fail(AMGT_ERR_ARG, "amgt_mbsr_cast: bad argument");
     Alloc a{al, (cudaStream_t)stream};
-    return cast_impl(in, to, out, a);
+    return cast_impl(in, to, out, a, nullptr);
 }
 
 amgt_status amgt_mbsr_free(amgt_mbsr* A, const amgt_allocator* al, void* stream) {
@@ -728,7 +752,7 @@ amgt_status amgt_mbsr_free(amgt_mbsr* A, const amgt_allocator* al, void* stream)
 amgt_status amgt_mbsr_transpose(const amgt_mbsr* in, amgt_mbsr* out, const amgt_allocator* al, void* stream) {
     if (!in || !out) return fail(AMGT_ERR_ARG, "amgt_mbsr_transpose: NULL argument");
     Alloc a{al, (cudaStream_t)stream};
-    return transpose_impl(in, out, a);
+    return transpose_impl(in, out, a, nullptr);
 }
 
 amgt_status amgt_mbsr_shift_cols(amgt_mbsr* A, int64_t delta_tiles, int64_t new_n, void* stream) {

@@ -1,5 +1,6 @@
 // runtime.cu — error reporting, allocator glue, device prefix sum, timing/launch counters.
 #include <atomic>
+#include <ctime>
 #include <cstdlib>
 #include <cstdarg>
 #include <mutex>
@@ -195,6 +196,52 @@ static bool pdl_allowed() {
 bool pdl_active() { return g_pdl_depth > 0 && pdl_allowed(); }
 PdlScope::PdlScope() { ++g_pdl_depth; }
 PdlScope::~PdlScope() { --g_pdl_depth; }
+
+// AMGT_TRACE=1 (measurement only): named points; at each point the host time when the
+// step's work was enqueued and, after a stream synchronisation, when the device finished it.
+// (The synchronisations change the overlap; per-step device and host costs still separate.)
+struct TracePt {
+    const char* name;
+    double enq_ms, done_ms;
+};
+static std::vector<TracePt> g_trace;
+static bool trace_on() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_TRACE");
+        v = (e && e[0] == '1') ? 1 : 0;
+    }
+    return v == 1;
+}
+static double host_ms() {
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return ts.tv_sec * 1e3 + ts.tv_nsec * 1e-6;
+}
+void trace_point(const char* name, cudaStream_t s) {
+    if (!trace_on()) return;
+    const double e = host_ms();
+    cudaStreamSynchronize(s);
+    g_trace.push_back(TracePt{name, e, host_ms()});
+}
+void trace_dump() {
+    if (!trace_on() || g_trace.empty()) return;
+    double prev = g_trace.front().done_ms;
+    for (const TracePt& t : g_trace) {
+        fprintf(stderr, "trace %-20s enqueue %8.3f ms  device-done %8.3f ms\n", t.name, t.enq_ms - prev,
+                t.done_ms - t.enq_ms);
+        prev = t.done_ms;
+    }
+    g_trace.clear();
+}
+
+// Small pinned host buffer (per thread, allocated once) for device values read back after a
+// later synchronisation point instead of with a synchronisation of their own.
+int64_t* pinned_slots() {
+    static thread_local int64_t* p = nullptr;
+    if (!p && cudaMallocHost(&p, PINNED_SLOTS * sizeof(int64_t)) != cudaSuccess) p = nullptr;
+    return p;
+}
 
 void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 void count_launches(int64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }

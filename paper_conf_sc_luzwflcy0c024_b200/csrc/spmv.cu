@@ -35,7 +35,8 @@ struct SpmvPlan {
     int32_t* chunk_lr = nullptr;   // [nchunks] -> index into long_rows
     double* partial = nullptr;     // [nchunks*4] (double or float accumulators)
     amgt_spmv_stats st{};
-    double mean_row = 0.0;  // tiles per block row
+    bool stats_ready = false;  // st computed (the fast path defers it to amgt_spmv_get_stats)
+    double mean_row = 0.0;     // tiles per block row
 };
 
 void spmv_plan_free(void* aux, Alloc& a) {
@@ -387,10 +388,57 @@ static unsigned grid_cap(int64_t work, int threads) {
     return (unsigned)(b < 1 ? 1 : (b > cap ? cap : b));
 }
 
+// The reported statistics of a plan (amgt_spmv_get_stats; no effect on the SpMV): mean and
+// coefficient of variation of tiles per block row (R11), popcount sum, tensor-core tiles.
+static amgt_status plan_stats(const amgt_mbsr* A, SpmvPlan* P, cudaStream_t s) {
+    Alloc a{nullptr, s};
+    const int64_t BR = A->blc_row;
+    Scratch<int64_t> islong, nch;
+    Scratch<double> sums;
+    Scratch<unsigned long long> tcc;
+    AMGT_TRY(islong.init(a, BR + 1));
+    AMGT_TRY(nch.init(a, BR + 1));
+    AMGT_TRY(sums.init(a, 2));
+    AMGT_TRY(tcc.init(a, 2));
+    AMGT_CUDA(cudaMemsetAsync(sums.p, 0, 2 * sizeof(double), s));
+    AMGT_CUDA(cudaMemsetAsync(tcc.p, 0, 2 * sizeof(unsigned long long), s));
+    if (BR > 0) {
+        k_plan_rows<<<grid_cap(BR, 256), 256, 0, s>>>(BR, A->blc_ptr, islong.p, nch.p, sums.p);
+        AMGT_LAUNCHED();
+    }
+    if (A->blc_num > 0) {
+        k_count_tc<<<grid_cap(A->blc_num, 256), 256, 0, s>>>(A->blc_num, A->blc_map, g_tc_thr_spmv, tcc.p);
+        AMGT_LAUNCHED();
+    }
+    double hs[2];
+    unsigned long long ht[2];
+    AMGT_CUDA(cudaMemcpyAsync(hs, sums.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaMemcpyAsync(ht, tcc.p, sizeof(ht), cudaMemcpyDeviceToHost, s));
+    AMGT_CUDA(cudaStreamSynchronize(s));
+    const double mean = BR ? hs[0] / BR : 0.0;
+    const double var = BR ? hs[1] / BR - mean * mean : 0.0;
+    P->st.avg_nnz_blc = A->blc_num ? (double)ht[1] / (double)A->blc_num : 0.0;
+    P->st.variation = mean > 0 ? sqrt(var > 0 ? var : 0) / mean : 0.0;
+    P->st.long_rows = P->nlong;
+    P->st.chunks = P->nchunks;
+    P->st.tc_tiles = (int64_t)ht[0];
+    P->stats_ready = true;
+    return AMGT_OK;
+}
+
 amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
     cudaStream_t s = a.s;
     if (A->aux) { spmv_plan_free(A->aux, a); A->aux = nullptr; }
     const int64_t BR = A->blc_row;
+    if (A->row_max > 0 && A->row_max <= WARP_CAPACITY) {
+        // longest block row known (conversion / SpGEMM / transpose) and within one warp chunk:
+        // no long rows, nothing to split, no device work and no synchronisation; the reported
+        // statistics are computed on first request
+        SpmvPlan* P = new SpmvPlan();
+        P->mean_row = BR ? (double)A->blc_num / (double)BR : 0.0;
+        A->aux = P;
+        return AMGT_OK;
+    }
     Scratch<int64_t> islong, nch, lpos, cpos;
     Scratch<double> sums;
     Scratch<unsigned long long> tcc;
@@ -445,6 +493,7 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
     P->st.long_rows = nl;
     P->st.chunks = ncx;
     P->st.tc_tiles = (int64_t)ht[0];
+    P->stats_ready = true;
     P->mean_row = mean;
     A->aux = P;
     return AMGT_OK;
@@ -596,7 +645,9 @@ amgt_status amgt_spmv_analyze(amgt_mbsr* A, const amgt_allocator* al, void* stre
 amgt_status amgt_spmv_get_stats(const amgt_mbsr* A, amgt_spmv_stats* st) {
     if (!A || !st) return fail(AMGT_ERR_ARG, "amgt_spmv_get_stats: NULL argument");
     if (!A->aux) return fail(AMGT_ERR_ARG, "amgt_spmv_get_stats: matrix not analysed");
-    *st = ((const SpmvPlan*)A->aux)->st;
+    SpmvPlan* P = (SpmvPlan*)A->aux;
+    if (!P->stats_ready) AMGT_TRY(plan_stats(A, P, (cudaStream_t)0));  // legacy stream: ordered after prior work
+    *st = P->st;
     return AMGT_OK;
 }
 

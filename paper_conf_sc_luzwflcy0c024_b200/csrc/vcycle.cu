@@ -18,8 +18,8 @@
 namespace amgt {
 
 amgt_status mbsr_release(amgt_mbsr* M, Alloc& a);
-amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& a);
-amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a);
+amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& a, uint32_t* dflag = nullptr);
+amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a, unsigned long long* dmax = nullptr);
 amgt_status mbsr_to_csr_impl(const amgt_mbsr* A, int64_t* rp, int32_t* ci, double* v, Alloc& a);
 amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a);
 amgt_status spmv_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* y, amgt_prec yp, cudaStream_t s,
@@ -71,7 +71,7 @@ struct amgt_hierarchy {
 
 namespace amgt {
 
-constexpr int NORM_BLOCKS = 296;
+constexpr int NORM_BLOCKS = 592;  // one wave: 4 CTAs of 256 per SM (k_dot, k_pcg_xr: <= 64 registers)
 
 template <typename V, typename M>
 __global__ void k_dinv(int64_t BR, int64_t m, int64_t off, const int64_t* __restrict__ bptr,
@@ -131,8 +131,9 @@ __device__ __forceinline__ void finish_sum(double s, double* __restrict__ ws, do
     }
 }
 
-// *out = a . b (a == b: ||a||^2), deterministic for a fixed grid of NORM_BLOCKS
-__global__ void __launch_bounds__(256) k_dot(int64_t n, const double* __restrict__ a, const double* __restrict__ b,
+// *out = a . b (a == b: ||a||^2), deterministic for a fixed grid of NORM_BLOCKS.  16-B loads,
+// four per thread in flight (a == b: one stream), summed in a fixed order.
+__global__ void __launch_bounds__(256, 4) k_dot(int64_t n, const double* __restrict__ a, const double* __restrict__ b,
                                              double* __restrict__ ws, double* __restrict__ out) {
     pdl_wait();
     double s = 0.0;
@@ -141,7 +142,26 @@ __global__ void __launch_bounds__(256) k_dot(int64_t n, const double* __restrict
         const int64_t n2 = n >> 1;
         const double2* a2 = reinterpret_cast<const double2*>(a);
         const double2* b2 = reinterpret_cast<const double2*>(b);
-        for (int64_t i = gt; i < n2; i += nt) {
+        const bool same = a == b;
+        int64_t i = gt;
+        for (; i + 3 * nt < n2; i += 4 * nt) {
+            double2 u[4], v[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) u[k] = __ldcs(a2 + i + k * nt);
+            if (same) {
+#pragma unroll
+                for (int k = 0; k < 4; ++k) v[k] = u[k];
+            } else {
+#pragma unroll
+                for (int k = 0; k < 4; ++k) v[k] = __ldcs(b2 + i + k * nt);
+            }
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                s = fma(u[k].x, v[k].x, s);
+                s = fma(u[k].y, v[k].y, s);
+            }
+        }
+        for (; i < n2; i += nt) {
             const double2 u = __ldcs(a2 + i), v = __ldcs(b2 + i);
             s = fma(u.x, v.x, s);
             s = fma(u.y, v.y, s);
@@ -155,7 +175,7 @@ __global__ void __launch_bounds__(256) k_dot(int64_t n, const double* __restrict
 
 // PCG (NEXT-1): x += alpha p, r -= alpha q with alpha = rz / pq (0 when pq = 0), and
 // ||r||^2 of the updated r into *rr (one pass)
-__global__ void __launch_bounds__(256) k_pcg_xr(int64_t n, const double* __restrict__ rz, const double* __restrict__ pq,
+__global__ void __launch_bounds__(256, 4) k_pcg_xr(int64_t n, const double* __restrict__ rz, const double* __restrict__ pq,
                                                 double* __restrict__ x, double* __restrict__ r,
                                                 const double* __restrict__ p, const double* __restrict__ q,
                                                 double* __restrict__ ws, double* __restrict__ rr) {
@@ -319,6 +339,16 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     cudaStream_t s = H->s;
     Alloc a = H->alloc();
     H->nlev = nlev;
+    trace_point("create", s);
+    // Values read back at later synchronisation points instead of with their own: the FP16
+    // range flag of every cast (checked at the end) and the longest block row of each R_k
+    // (it arrives with the SpGEMM syncs that follow the transpose; lets the SpMV analysis of
+    // R_k skip its sync).  dev = [flag | row max of R_0..R_6].
+    Scratch<unsigned long long> dev;
+    AMGT_TRY(dev.init(a, 8));
+    AMGT_CUDA(cudaMemsetAsync(dev.p, 0, 8 * sizeof(unsigned long long), s));
+    uint32_t* dflag = reinterpret_cast<uint32_t*>(dev.p);
+    int64_t* pin = pinned_slots();
     for (int k = 0; k < nlev; ++k) {
         amgt_level& L = H->L[k];
         const amgt_prec pk = o->level_prec[k];
@@ -330,12 +360,13 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
                 L.A.aux = nullptr;
                 L.ownA = false;
             } else {
-                AMGT_TRY(cast_impl(A, pk, &L.A, a));
+                AMGT_TRY(cast_impl(A, pk, &L.A, a, dflag));
                 L.ownA = true;
             }
         }
         L.npad = 4 * L.A.blc_row;
         AMGT_TRY(spmv_analyze_impl(&L.A, a));
+        trace_point("analyze A", s);
         const size_t vb = vbytes(L.vprec) * (size_t)L.npad;
         for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv}) {
             *p = a.get(vb);
@@ -343,6 +374,7 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             AMGT_CUDA(cudaMemsetAsync(*p, 0, vb, s));
         }
         AMGT_TRY(build_dinv(L, s, H->o.smoother == AMGT_SMOOTH_L1_JACOBI));
+        trace_point("vectors+dinv", s);
         if (k == 0 && nlev >= 2 && sweeps_enabled() && L.A.prec == AMGT_FP64 && H->o.nu1 == 1 && H->o.nu2 == 1) {
             L.u = a.get(vb);
             if (!L.u) return fail(AMGT_ERR_ALLOC, "hierarchy vector allocation failed");
@@ -355,28 +387,35 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             if (o->interp == AMGT_INTERP_SA) {
                 // NEXT-2 / Alg. 1 line 4: P_k = (I - w D_F^-1 A_F) Pt through one SpGEMM call
                 amgt_mbsr Pt{};
-                AMGT_TRY(cast_impl(Pk, pk, &Pt, a));
+                AMGT_TRY(cast_impl(Pk, pk, &Pt, a, dflag));
                 const double th = o->theta >= 0.0 ? o->theta : 0.25;
                 const double wp = o->omega_p > 0.0 ? o->omega_p : 2.0 / 3.0;
                 const amgt_status st = sa_interp_impl(&L.A, &Pt, th, wp, &L.P, a);
                 mbsr_release(&Pt, a);
                 AMGT_TRY(st);
             } else {
-                AMGT_TRY(cast_impl(Pk, pk, &L.P, a));  // P_k in level k precision (copy when equal)
+                AMGT_TRY(cast_impl(Pk, pk, &L.P, a, dflag));  // P_k in level k precision (copy when equal)
             }
-            AMGT_TRY(transpose_impl(&L.P, &L.R, a));  // R_k = P_k^T (Alg. 1 line 4)
+            trace_point("P cast", s);
+            AMGT_TRY(transpose_impl(&L.P, &L.R, a, pin ? dev.p + 1 + k : nullptr));  // R_k = P_k^T (Alg. 1 line 4)
+            if (pin) AMGT_CUDA(cudaMemcpyAsync(pin + k, dev.p + 1 + k, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            trace_point("transpose", s);
             // A_{k+1} = R_k (A_k P_k): two SpGEMM calls in level k precision (Alg. 1 line 5)
             amgt_mbsr AP{}, Ac{};
             AMGT_TRY(spgemm_symbolic_impl(&L.A, &L.P, &AP, nullptr, a));
+            trace_point("sym AP", s);
             amgt_status st = spgemm_numeric_impl(&L.A, &L.P, &AP, a);
+            trace_point("num AP", s);
             if (st == AMGT_OK) st = spgemm_symbolic_impl(&L.R, &AP, &Ac, nullptr, a);
+            trace_point("sym RAP", s);
             if (st == AMGT_OK) st = spgemm_numeric_impl(&L.R, &AP, &Ac, a);
+            trace_point("num RAP", s);
             mbsr_release(&AP, a);
             if (st != AMGT_OK) { mbsr_release(&Ac, a); return st; }
             amgt_level& N = H->L[k + 1];
             const amgt_prec pn = o->level_prec[k + 1];
             if (pn != Ac.prec) {
-                st = cast_impl(&Ac, pn, &N.A, a);
+                st = cast_impl(&Ac, pn, &N.A, a, dflag);
                 if (st != AMGT_OK) { mbsr_release(&Ac, a); return st; }
                 Ac.own &= ~1u;  // the cast shares Ac's structure: move its ownership to N.A
                 mbsr_release(&Ac, a);  // frees Ac's values only
@@ -385,8 +424,11 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
                 N.A = Ac;
             }
             N.ownA = true;
+            trace_point("cast Ac", s);
             AMGT_TRY(spmv_analyze_impl(&L.P, a));
+            if (pin) L.R.row_max = pin[k];  // arrived: the SpGEMM symbolic phases synchronised since
             AMGT_TRY(spmv_analyze_impl(&L.R, a));
+            trace_point("analyze P R", s);
         }
     }
     // coarsest level: MBSR2CSR, dense inverse on the host (FP64)
@@ -400,7 +442,10 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     AMGT_TRY(mbsr_to_csr_impl(&C.A, rp, ci, v, a));
     std::vector<int64_t> hrp(n + 1);
     AMGT_CUDA(cudaMemcpyAsync(hrp.data(), rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    uint32_t hflag = 0;  // FP16 range flag of every cast above
+    AMGT_CUDA(cudaMemcpyAsync(&hflag, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     AMGT_CUDA(cudaStreamSynchronize(s));
+    if (hflag & FLAG_RANGE) return fail(AMGT_ERR_RANGE, "hierarchy: a level value exceeds the FP16 range (65504)");
     const int64_t nnz = hrp[n];
     std::vector<int32_t> hci(nnz);
     std::vector<double> hv(nnz);
@@ -423,6 +468,8 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     AMGT_CUDA(cudaMemsetAsync(H->partial, 0, (NORM_BLOCKS + 1) * sizeof(double), H->s));
     AMGT_CUDA(cudaMemcpyAsync(H->Ainv, inv.data(), n * n * sizeof(double), cudaMemcpyHostToDevice, s));
     AMGT_CUDA(cudaStreamSynchronize(s));
+    trace_point("coarse inverse", s);
+    trace_dump();
     return AMGT_OK;
 }
 
@@ -751,47 +798,72 @@ struct SmTailArgs {
     void* xout;  // x_kt in global memory
 };
 
-// y_i = epi(i, (A x)_i) for the 4*BR rows of an mBSR operator held in shared memory
+// y_i = epi(i, (A x)_i) for the 4*BR rows of an mBSR operator held in shared memory.  Tiles
+// in groups of four: the group's bitmaps, columns and row values are read before its x
+// entries (independent shared-memory loads), then accumulated in tile / column order.
 template <typename VT, typename F>
 __device__ __forceinline__ void sm_spmv(const unsigned char* sm, const SmMat& M, const VT* x, F&& epi) {
     const int64_t* ptr = reinterpret_cast<const int64_t*>(sm + M.ptr);
     const int32_t* idx = reinterpret_cast<const int32_t*>(sm + M.idx);
     const uint16_t* map = reinterpret_cast<const uint16_t*>(sm + M.map);
+    constexpr int U = 4, U2 = 2;  // tiles per group (FP32/FP16, FP64)
     for (int64_t i = threadIdx.x; i < 4 * M.BR; i += blockDim.x) {
         const int64_t I = i >> 2;
         const int r = (int)(i & 3);
-        const int64_t t0 = ptr[I], t1 = ptr[I + 1];
+        const int t0 = (int)ptr[I], t1 = (int)ptr[I + 1];
         if (M.prec == AMGT_FP64) {
             const double* val = reinterpret_cast<const double*>(sm + M.val);
             double acc = 0.0;
-            for (int64_t t = t0; t < t1; ++t) {
-                const uint32_t nib = (map[t] >> (4 * r)) & 0xFu;
-                if (!nib) continue;
-                const int64_t J = idx[t];
+            for (int t = t0; t < t1; t += U2) {
+                uint32_t nib[U2];
+                int J[U2];
+                double a[U2][4];
 #pragma unroll
-                for (int c = 0; c < 4; ++c)
-                    if ((nib >> c) & 1u) acc = fma(val[16 * t + 4 * r + c], (double)x[4 * J + c], acc);
+                for (int u = 0; u < U2; ++u) {
+                    const bool v = t + u < t1;
+                    nib[u] = v ? (map[t + u] >> (4 * r)) & 0xFu : 0u;
+                    J[u] = v ? idx[t + u] : 0;
+                    if (v) {
+                        const double2 p0 = reinterpret_cast<const double2*>(val + 16 * (t + u) + 4 * r)[0];
+                        const double2 p1 = reinterpret_cast<const double2*>(val + 16 * (t + u) + 4 * r)[1];
+                        a[u][0] = p0.x; a[u][1] = p0.y; a[u][2] = p1.x; a[u][3] = p1.y;
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < U2; ++u)
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if ((nib[u] >> c) & 1u) acc = fma(a[u][c], (double)x[4 * J[u] + c], acc);
             }
             epi(i, acc);
         } else {
             float acc = 0.f;
-            for (int64_t t = t0; t < t1; ++t) {
-                const uint32_t nib = (map[t] >> (4 * r)) & 0xFu;
-                if (!nib) continue;
-                const int64_t J = idx[t];
-                float a[4];
-                if (M.prec == AMGT_FP32) {
-                    const float4 v = *reinterpret_cast<const float4*>(sm + M.val + 4 * (16 * t + 4 * r));
-                    a[0] = v.x; a[1] = v.y; a[2] = v.z; a[3] = v.w;
-                } else {
-                    const uint2 w = *reinterpret_cast<const uint2*>(sm + M.val + 2 * (16 * t + 4 * r));
-                    const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
-                    const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
-                    a[0] = lo.x; a[1] = lo.y; a[2] = hi.x; a[3] = hi.y;
+            for (int t = t0; t < t1; t += U) {
+                uint32_t nib[U];
+                int J[U];
+                float a[U][4];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const bool v = t + u < t1;
+                    nib[u] = v ? (map[t + u] >> (4 * r)) & 0xFu : 0u;
+                    J[u] = v ? idx[t + u] : 0;
+                    if (v) {
+                        if (M.prec == AMGT_FP32) {
+                            const float4 w = *reinterpret_cast<const float4*>(sm + M.val + 4 * (16 * (int64_t)(t + u) + 4 * r));
+                            a[u][0] = w.x; a[u][1] = w.y; a[u][2] = w.z; a[u][3] = w.w;
+                        } else {
+                            const uint2 w = *reinterpret_cast<const uint2*>(sm + M.val + 2 * (16 * (int64_t)(t + u) + 4 * r));
+                            const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
+                            const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
+                            a[u][0] = lo.x; a[u][1] = lo.y; a[u][2] = hi.x; a[u][3] = hi.y;
+                        }
+                    }
                 }
 #pragma unroll
-                for (int c = 0; c < 4; ++c)
-                    if ((nib >> c) & 1u) acc = fmaf(a[c], (float)x[4 * J + c], acc);
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if ((nib[u] >> c) & 1u) acc = fmaf(a[u][c], (float)x[4 * J[u] + c], acc);
             }
             epi(i, acc);
         }
@@ -803,7 +875,14 @@ __global__ void __launch_bounds__(512) k_tail_smem(const SmTailArgs a) {
     pdl_wait();
     extern __shared__ __align__(16) unsigned char sm[];
     {  // stage: all segments as one flat list of 16-B chunks, four loads in flight per thread
-        const int64_t n = a.pre[a.nseg];
+        __shared__ int64_t s_pre[SM_MAXSEG + 1], s_off[SM_MAXSEG];
+        __shared__ const void* s_src[SM_MAXSEG];
+        for (int k = threadIdx.x; k <= a.nseg; k += blockDim.x) {
+            s_pre[k] = a.pre[k];
+            if (k < a.nseg) { s_off[k] = a.seg[k].off; s_src[k] = a.seg[k].src; }
+        }
+        __syncthreads();
+        const int64_t n = s_pre[a.nseg];
         for (int64_t c0 = threadIdx.x; c0 < n; c0 += 4 * (int64_t)blockDim.x) {
             uint4 v[4];
             int64_t dst[4];
@@ -815,11 +894,11 @@ __global__ void __launch_bounds__(512) k_tail_smem(const SmTailArgs a) {
                     int lo = 0, hi = a.nseg - 1;  // segment: largest s with pre[s] <= c
                     while (lo < hi) {
                         const int mid = (lo + hi + 1) >> 1;
-                        if (a.pre[mid] <= c) lo = mid; else hi = mid - 1;
+                        if (s_pre[mid] <= c) lo = mid; else hi = mid - 1;
                     }
-                    const int64_t k = c - a.pre[lo];
-                    v[u] = __ldcg(reinterpret_cast<const uint4*>(a.seg[lo].src) + k);
-                    dst[u] = a.seg[lo].off + 16 * k;
+                    const int64_t k = c - s_pre[lo];
+                    v[u] = __ldcg(reinterpret_cast<const uint4*>(s_src[lo]) + k);
+                    dst[u] = s_off[lo] + 16 * k;
                 }
             }
 #pragma unroll

@@ -84,3 +84,21 @@ def test_vcycle_cfg3_shape_mixed():
     live = res_o[1:] / res_o[0] > 1e-10
     assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
     H.close()
+
+
+def test_hierarchy_fp16_overflow_reported():
+    """R18: a coarse FP16 level whose values exceed 65504 makes amgt_hierarchy_create return
+    AMGT_ERR_RANGE (the FP16 range flags of the casts are read back at the hierarchy's
+    coarse-level synchronisation): the 27-point operator scaled by 1e4 (diagonal 2.6e5,
+    in range for the FP64 / FP32 levels, not for the FP16 ones) fails, the unscaled one
+    builds."""
+    amgt = _amgt()
+    A = gen.laplacian_27pt(16)
+    PR = gen.aggregation_hierarchy((16, 16, 16), 4)
+    prec = ("f64", "f32", "f16", "f16")
+    As = type(A)(A.m, A.n, A.row_ptr, A.col, A.val * 1e4)
+    with pytest.raises(amgt.AmgtError) as ei:
+        amgt.Hierarchy(amgt.from_csr(As), [amgt.from_csr(P) for P, _ in PR], level_prec=prec)
+    assert "RANGE" in str(ei.value)
+    H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=prec)
+    H.close()
