@@ -135,8 +135,10 @@ __device__ __forceinline__ void group_store_tile_f64(double* tile, const double 
 enum : uint32_t { FLAG_FORMAT = 1u, FLAG_RANGE = 2u };
 
 // ------------------------------------------------------------------ scan
-// out[0] = 0, out[i+1] = in[0] + ... + in[i]  (int64, n >= 0).  `in` may alias `out+1`? no.
-amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a, cudaStream_t s);
+// out[0] = 0, out[i+1] = in[0] + ... + in[i]  (int64, n >= 0, inputs >= 0); one launch
+// (decoupled look-back).  dmax (optional, device, pre-set by the caller): atomicMax of the inputs.
+amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a, cudaStream_t s,
+                           unsigned long long* dmax = nullptr);
 
 // ------------------------------------------------------------------ instrumentation
 enum TimerClass : int {

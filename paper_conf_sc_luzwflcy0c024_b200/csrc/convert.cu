@@ -343,8 +343,6 @@ __global__ void k_tr_gather(int64_t T_, const int64_t* __restrict__ perm, const 
     }
 }
 
-__global__ void k_max_rows(int64_t BR, const int64_t* __restrict__ nrow, unsigned long long* __restrict__ out);  // spgemm.cu
-
 static unsigned grid_for(int64_t work, int threads) {
     int64_t b = ceil_div(work, threads);
     int64_t cap = (int64_t)num_sms() * 16;
@@ -443,14 +441,10 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     // blc_ptr lives in the output; scan the counts into it.
     M.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
     if (!M.blc_ptr) return fail(AMGT_ERR_ALLOC, "blc_ptr allocation failed");
-    AMGT_TRY(scan_exclusive(cnt.p, M.blc_ptr, BR, a, s));
     Scratch<unsigned long long> rmax;  // longest block row (lets the SpMV analysis skip its sync)
     AMGT_TRY(rmax.init(a, 1));
     AMGT_CUDA(cudaMemsetAsync(rmax.p, 0, sizeof(unsigned long long), s));
-    if (BR > 0) {
-        k_max_rows<<<grid_for(BR, 256), 256, 0, s>>>(BR, cnt.p, rmax.p);
-        AMGT_LAUNCHED();
-    }
+    AMGT_TRY(scan_exclusive(cnt.p, M.blc_ptr, BR, a, s, rmax.p));
     int64_t hT[1] = {0};
     uint32_t hflag = 0;
     unsigned long long hmax = 0;
@@ -612,11 +606,7 @@ amgt_status transpose_impl(const amgt_mbsr* in, amgt_mbsr* out, Alloc& a, unsign
         k_tr_count<<<grid_for(T, 256), 256, 0, s>>>(T, in->blc_idx, cnt.p);
         AMGT_LAUNCHED();
     }
-    AMGT_TRY(scan_exclusive((const int64_t*)cnt.p, M.blc_ptr, BRo, a, s));
-    if (dmax && BRo > 0) {
-        k_max_rows<<<grid_for(BRo, 256), 256, 0, s>>>(BRo, (const int64_t*)cnt.p, dmax);
-        AMGT_LAUNCHED();
-    }
+    AMGT_TRY(scan_exclusive((const int64_t*)cnt.p, M.blc_ptr, BRo, a, s, dmax));
     AMGT_CUDA(cudaMemsetAsync(cnt.p, 0, (BRo + 1) * sizeof(unsigned long long), s));
     if (T > 0) {
         k_tr_scatter<<<grid_for(in->blc_row, 128), 128, 0, s>>>(in->blc_row, in->blc_ptr, in->blc_idx, M.blc_ptr, cnt.p,

@@ -125,59 +125,93 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t* sh_warp, 
     return r;
 }
 
-__global__ void k_scan_reduce(const int64_t* __restrict__ in, int64_t n, int64_t* __restrict__ bsum) {
-    __shared__ int64_t sh[32];
-    int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_I;
-    int64_t s = 0;
-#pragma unroll
-    for (int i = 0; i < SCAN_I; ++i)
-        if (base + i < n) s += in[base + i];
-    int64_t tot;
-    block_excl_scan(s, sh, &tot);
-    if (threadIdx.x == 0) bsum[blockIdx.x] = tot;
+// Single-pass exclusive scan (decoupled look-back): one launch.  Each CTA takes a ticket
+// (logical tile order = scheduling order, so every predecessor is resident or done), publishes
+// its tile aggregate, then warp 0 looks back over 32 predecessors at a time, summing
+// aggregates until it meets a published inclusive prefix; the CTA publishes its own inclusive
+// prefix and scans its tile.  st = [ticket | one status word per tile], zeroed by the host;
+// status word = flag << 62 | value (flag 1 aggregate, 2 inclusive prefix; value < 2^62).
+// Optionally also the maximum input (dmax, atomicMax).
+constexpr unsigned long long ST_AGG = 1ull << 62, ST_INC = 2ull << 62, ST_VAL = (1ull << 62) - 1;
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
 }
 
-// Scan of `in` (n items) into out (out[0]=0 ... out[n]) adding boff[blockIdx] (exclusive
-// block offsets, or nullptr).
-__global__ void k_scan_tile(const int64_t* __restrict__ in, int64_t n, const int64_t* __restrict__ boff,
-                            int64_t* __restrict__ out) {
+__global__ void __launch_bounds__(SCAN_T) k_scan(const int64_t* __restrict__ in, int64_t n,
+                                                 unsigned long long* __restrict__ st, int64_t* __restrict__ out,
+                                                 unsigned long long* __restrict__ dmax) {
     __shared__ int64_t sh[32];
-    int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_I;
+    __shared__ int64_t s_tile, s_excl;
+    if (threadIdx.x == 0) s_tile = (int64_t)atomicAdd(st, 1ull);
+    __syncthreads();
+    const int64_t tile = s_tile;
+    const int64_t base = tile * SCAN_TILE + (int64_t)threadIdx.x * SCAN_I;
     int64_t v[SCAN_I];
-    int64_t s = 0;
+    int64_t s = 0, mx = 0;
 #pragma unroll
     for (int i = 0; i < SCAN_I; ++i) {
         v[i] = (base + i < n) ? in[base + i] : 0;
         s += v[i];
+        mx = max(mx, v[i]);
     }
     int64_t tot;
-    int64_t off = block_excl_scan(s, sh, &tot) + (boff ? boff[blockIdx.x] : 0);
-    if (blockIdx.x == 0 && threadIdx.x == 0) out[0] = 0;
+    const int64_t off = block_excl_scan(s, sh, &tot);
+    unsigned long long* status = st + 1;
+    if (threadIdx.x == 0) st_release(status + tile, (tile == 0 ? ST_INC : ST_AGG) | (unsigned long long)tot);
+    if (threadIdx.x < 32) {
+        const int lane = threadIdx.x;
+        int64_t excl = 0;
+        int64_t j = tile - 1;  // look back over status[j - lane], j decreasing by 32
+        while (j >= 0) {
+            const int64_t k = j - lane;
+            unsigned long long w = k >= 0 ? ld_acquire(status + k) : ST_INC;  // before tile 0: prefix 0
+            while (__any_sync(0xffffffffu, (w >> 62) == 0)) {
+                if ((w >> 62) == 0) w = ld_acquire(status + k);
+            }
+            const unsigned inc = __ballot_sync(0xffffffffu, (w >> 62) == 2);
+            const int stop = inc ? __ffs(inc) - 1 : 32;  // first lane (nearest tile) with a prefix
+            int64_t val = (lane <= stop && k >= 0) ? (int64_t)(w & ST_VAL) : 0;
+#pragma unroll
+            for (int d = 16; d; d >>= 1) val += __shfl_xor_sync(0xffffffffu, val, d);
+            excl += val;
+            if (inc) break;
+            j -= 32;
+        }
+        if (lane == 0) {
+            s_excl = excl;
+            if (tile > 0) st_release(status + tile, ST_INC | (unsigned long long)(excl + tot));
+        }
+    }
+    __syncthreads();
+    int64_t o = s_excl + off;
+    if (tile == 0 && threadIdx.x == 0) out[0] = 0;
 #pragma unroll
     for (int i = 0; i < SCAN_I; ++i) {
-        off += v[i];
-        if (base + i < n) out[base + i + 1] = off;
+        o += v[i];
+        if (base + i < n) out[base + i + 1] = o;
+    }
+    if (dmax) {
+        for (int d = 16; d; d >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, d));
+        if ((threadIdx.x & 31) == 0 && mx > 0) atomicMax(dmax, (unsigned long long)mx);
     }
 }
 
-amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a, cudaStream_t s) {
+amgt_status scan_exclusive(const int64_t* in, int64_t* out, int64_t n, Alloc& a, cudaStream_t s,
+                           unsigned long long* dmax) {
     if (n <= 0) {
         AMGT_CUDA(cudaMemsetAsync(out, 0, sizeof(int64_t), s));
         return AMGT_OK;
     }
-    int64_t nb = ceil_div(n, SCAN_TILE);
-    if (nb == 1) {
-        k_scan_tile<<<1, SCAN_T, 0, s>>>(in, n, nullptr, out);
-        AMGT_LAUNCHED();
-        return AMGT_OK;
-    }
-    Scratch<int64_t> bsum, boff;
-    AMGT_TRY(bsum.init(a, nb));
-    AMGT_TRY(boff.init(a, nb + 1));
-    k_scan_reduce<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, bsum.p);
-    AMGT_LAUNCHED();
-    AMGT_TRY(scan_exclusive(bsum.p, boff.p, nb, a, s));
-    k_scan_tile<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, boff.p, out);
+    const int64_t nb = ceil_div(n, SCAN_TILE);
+    Scratch<unsigned long long> st;
+    AMGT_TRY(st.init(a, nb + 1));
+    AMGT_CUDA(cudaMemsetAsync(st.p, 0, (nb + 1) * sizeof(unsigned long long), s));
+    k_scan<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, st.p, out, dmax);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }

@@ -1,19 +1,20 @@
 // spgemm.cu — C = A*B over mBSR (§IV.C; Alg. 3; Alg. 4).
 //
-// Pipeline (all on the device; host syncs: bin sizes, then the C tile count, L153):
-//   k_analyze     Cub_per_row(I) = sum_{K in A(I,:)} #tiles(B(K,:)) and bin(I) (L149-151;
-//                 8 bins, edges 128*2^b, reading R7); also the pair statistics.
-//   k_bin_*       row lists per bin (stable order irrelevant: rows are independent).
-//   step 1        per bin: distinct tile columns J with BITMAPMULTIPLY(mapA, mapB) != 0
-//                 (Alg. 3 lines 1-13) -> nnzC_row; prefix sum -> blc_ptrC; allocation.
-//   step 2        per bin: insert again, OR the bitmaps (R15), compress, sort ascending
-//                 (Alg. 3 lines 13-14) -> blc_idxC, blc_mapC.
-//   numeric       one warp per C block row (L155).  A tiles with POPCOUNT >= threshold go
+// Pipeline (all on the device; one host sync when every row has <= 32 candidates, else two):
+//   step 1        k_sym_group<1, true> over every block row: Cub(I) = sum_{K in A(I,:)}
+//                 #tiles(B(K,:)) and bin(I) (L149-151; 8 bins, edges 128*2^b, reading R7)
+//                 and, for the rows with Cub <= 32 (category 8), the distinct tile columns J
+//                 with BITMAPMULTIPLY(mapA, mapB) != 0 (Alg. 3 lines 1-13) -> nnzC_row;
+//                 prefix sum -> blc_ptrC; host reads the bins and the C tile count (L153).
+//   long rows     (only when some row has Cub > 32) row lists per bin (k_bin_scatter), the
+//                 per-bin hash kernels of step 1, prefix sum again, second host sync.
+//   step 2        insert again, OR the bitmaps (R15), compress, sort ascending (Alg. 3 lines
+//                 13-14) -> blc_idxC, blc_mapC: k_sym_group<2, true> + the per-bin kernels.
+//   numeric       rows by C-row length (<= 8 C tiles: staged 4-lane-group kernel; 9-32: warp
+//                 per row; 33-512; > 512: two passes).  A tiles with POPCOUNT >= threshold go
 //                 to the tensor-core route (DMMA m8n8k4: fragA = [A;A], fragB = [Bj|Bj'],
-//                 keep the two diagonal quadrants, L157-171); the others to CUDA cores,
-//                 one lane per (A tile, B tile) pair (L173).  Accumulation in shared
-//                 memory for rows with <= 32 C tiles, in global memory (conflict-free, one
-//                 A tile at a time) for longer rows.  Deterministic.
+//                 keep the two diagonal quadrants, L157-171); the others to CUDA cores
+//                 (L173).  Deterministic for rows with <= 32 C tiles.
 //
 // Hash tables (R8): power-of-two, >= 2x the bin's Cub upper bound, multiplicative hash,
 // linear probing.  Bins 0-1: one warp per row, table per warp; bins 2-6: one block per
@@ -50,43 +51,7 @@ struct SymCtx {  // device pointers shared by the symbolic kernels
 };
 
 // ---------------------------------------------------------------- analysis + binning
-template <bool STATS>
-__global__ void k_analyze(int64_t BR, SymCtx c, int64_t* __restrict__ bin_of, unsigned long long* __restrict__ stats,
-                          int tc_thr) {
-    // stats: [0..7] bin counts, [8] cub_total, [9] pairs_nonzero, [10] pairs_tc, [11] scalar products
-    __shared__ unsigned long long sh[13];
-    if (threadIdx.x < 13) sh[threadIdx.x] = 0;
-    __syncthreads();
-    // one 4-lane group per block row; the lanes split the row's A tiles (independent loads)
-    unsigned long long cubs = 0, pnz = 0, ptc = 0, sp = 0;
-    const int r = threadIdx.x & 3;
-    const unsigned gm = 0xFu << ((threadIdx.x & 31) & ~3);
-    const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2, ng = ((int64_t)gridDim.x * blockDim.x) >> 2;
-    for (int64_t I = g0; I < BR; I += ng) {
-        int64_t cub = 0;
-        for (int64_t t = c.aptr[I] + r; t < c.aptr[I + 1]; t += 4) {
-            const int32_t K = c.aidx[t];
-            const int64_t b0 = c.bptr[K], b1 = c.bptr[K + 1];
-            cub += b1 - b0;
-        }
-        cub += __shfl_xor_sync(gm, cub, 1, 4);
-        cub += __shfl_xor_sync(gm, cub, 2, 4);
-        if (r == 0) {
-            int b = 0;
-            while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
-            if (b == 0 && cub <= SMALL_CUB) b = NBINS;  // category 8 (sub-bin of bin 0)
-            bin_of[I] = b;
-            atomicAdd(&sh[cat_stat(b)], 1ull);
-            cubs += cub;
-        }
-    }
-    atomicAdd(&sh[8], cubs);
-    atomicAdd(&sh[9], pnz);
-    atomicAdd(&sh[10], ptc);
-    atomicAdd(&sh[11], sp);
-    __syncthreads();
-    if (threadIdx.x < 13 && sh[threadIdx.x]) atomicAdd(&stats[threadIdx.x], sh[threadIdx.x]);
-}
+// (Cub and the bins are computed by k_sym_group<1, true> below, L149-151.)
 
 // Pair statistics for amgt_spgemm_info (info only): one thread per A tile over its B row.
 __global__ void k_pair_stats(int64_t TA, SymCtx c, unsigned long long* __restrict__ stats, int tc_thr) {
@@ -319,18 +284,63 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
 // its J (the collision-free degenerate form of the paper's hash table, with the "hash" being
 // the candidate position).  Step 1 writes the distinct count; step 2 writes each distinct J
 // at its rank with the OR of the bitmaps of all its occurrences.  Deterministic, no atomics.
-template <int STEP>
+//
+// ALL = true: the kernel runs over every block row (rows == nullptr) and does the analysis
+// and binning itself (k_analyze's Cub and bin, L149-151): step 1 computes Cub, writes
+// bin_of[I] and the category counts / Cub total into stats (warp-aggregated atomics), and
+// continues only for category-8 rows (others: nnz_row = 0 here, counted later by their bin's
+// kernel); step 2 processes the rows whose bin_of is 8.  For operators whose rows are all
+// category 8 (every Laplacian RAP) the symbolic phase is then two kernels, one scan and one
+// host synchronisation.
+template <int STEP, bool ALL = false>
 __global__ void __launch_bounds__(256) k_sym_group(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
                                                    int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
-                                                   int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
+                                                   int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap,
+                                                   int64_t* __restrict__ bin_of = nullptr,
+                                                   unsigned long long* __restrict__ stats = nullptr) {
     __shared__ int keys[64][SMALL_CUB];
     __shared__ uint32_t maps[64][SMALL_CUB];
     __shared__ unsigned char first[64][SMALL_CUB];
     const int lane = threadIdx.x & 31, r = lane & 3, gl = threadIdx.x >> 2;
     const unsigned gm = 0xFu << (lane & ~3);
     const int64_t rr = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2);
-    if (rr >= nrows) return;  // whole group leaves together
-    const int64_t I = rows[rr];
+    if constexpr (ALL) {
+        const bool valid = rr < nrows;
+        if (STEP == 1) {
+            int64_t cub = 0;
+            if (valid)
+                for (int64_t t = c.aptr[rr] + r; t < c.aptr[rr + 1]; t += 4) {
+                    const int32_t Kc = c.aidx[t];
+                    cub += c.bptr[Kc + 1] - c.bptr[Kc];
+                }
+            cub += __shfl_xor_sync(0xffffffffu, cub, 1);
+            cub += __shfl_xor_sync(0xffffffffu, cub, 2);
+            int b = 0;
+            while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
+            if (b == 0 && cub <= SMALL_CUB) b = NBINS;  // category 8
+            const bool lead = valid && r == 0;
+            if (lead) {
+                bin_of[rr] = b;
+                if (b != NBINS) {
+                    nnz_row[rr] = 0;
+                    atomicAdd(&stats[cat_stat(b)], 1ull);  // rare: rows longer than 32 candidates
+                }
+            }
+            const unsigned n8 = __ballot_sync(0xffffffffu, lead && b == NBINS);
+            unsigned long long ct = lead ? (unsigned long long)cub : 0ull;
+            for (int d = 16; d; d >>= 1) ct += __shfl_xor_sync(0xffffffffu, ct, d);
+            if (lane == 0) {
+                if (n8) atomicAdd(&stats[cat_stat(NBINS)], (unsigned long long)__popc(n8));
+                if (ct) atomicAdd(&stats[8], ct);
+            }
+            if (!valid || b != NBINS) return;  // whole group leaves together
+        } else {
+            if (!valid || bin_of[rr] != NBINS) return;
+        }
+    } else {
+        if (rr >= nrows) return;  // whole group leaves together
+    }
+    const int64_t I = ALL ? rr : rows[rr];
     int* K = keys[gl];
     uint32_t* Mp = maps[gl];
     unsigned char* F = first[gl];
@@ -546,14 +556,6 @@ __global__ void __launch_bounds__(512) k_sym_dense(int64_t nrows, const int32_t*
         });
         __syncthreads();
     }
-}
-
-__global__ void k_max_rows(int64_t BR, const int64_t* __restrict__ nrow, unsigned long long* __restrict__ out) {
-    unsigned long long m = 0;
-    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x)
-        m = max(m, (unsigned long long)nrow[I]);
-    for (int d = 16; d; d >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, d));
-    if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
 }
 
 __global__ void k_numeric_rows_stats(int64_t BR, const int64_t* __restrict__ cptr, unsigned long long* __restrict__ out) {
@@ -1869,7 +1871,7 @@ static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_
                             Alloc& a, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
                             cudaStream_t s) {
     if (cnt[NBINS] > 0) {
-        k_sym_group<STEP><<<(unsigned)ceil_div(ceil_div(cnt[NBINS], 8) * 32, 256), 256, 0, s>>>(
+        k_sym_group<STEP, false><<<(unsigned)ceil_div(ceil_div(cnt[NBINS], 8) * 32, 256), 256, 0, s>>>(
             cnt[NBINS], rows + off[NBINS], c, nnz_row, cptr, cidx, cmap);
         AMGT_LAUNCHED();
     }
@@ -1897,59 +1899,69 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     const int64_t BR = A->blc_row;
     SymCtx c{A->blc_ptr, A->blc_idx, A->blc_map, B->blc_ptr, B->blc_idx, B->blc_map};
     Scratch<int64_t> bin_of, nnz_row;
-    Scratch<unsigned long long> stats, cursor;  // stats: 16 slots (layout above)
+    Scratch<unsigned long long> ctr;  // [0..15] stats (layout above) | [16..24] bin cursors | [25] longest C row
     Scratch<int32_t> rows;
     AMGT_TRY(bin_of.init(a, BR + 1));
     AMGT_TRY(nnz_row.init(a, BR + 1));
-    AMGT_TRY(stats.init(a, 16));
-    AMGT_TRY(cursor.init(a, NCAT));
-    AMGT_TRY(rows.init(a, BR + 1));
-    AMGT_CUDA(cudaMemsetAsync(stats.p, 0, 16 * sizeof(unsigned long long), s));
-    AMGT_CUDA(cudaMemsetAsync(cursor.p, 0, NCAT * sizeof(unsigned long long), s));
+    AMGT_TRY(ctr.init(a, 32));
+    AMGT_CUDA(cudaMemsetAsync(ctr.p, 0, 32 * sizeof(unsigned long long), s));
+    unsigned long long* stats = ctr.p;
+    unsigned long long* cursor = ctr.p + 16;
+    unsigned long long* rmax = ctr.p + 25;
     amgt_mbsr C{};
     C.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
     if (!C.blc_ptr) return fail(AMGT_ERR_ALLOC, "SpGEMM: blc_ptr allocation failed");
     unsigned long long hs[16];
     {
         TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
+        // step 1 over every block row: Cub + bins (L149-151) and, for the category-8 rows
+        // (Cub <= 32), the distinct tile columns (Alg. 3 lines 1-13)
         if (BR > 0) {
-            k_analyze<false><<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, c, bin_of.p, stats.p, g_tc_thr_spgemm);
+            k_sym_group<1, true><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
+                BR, nullptr, c, nnz_row.p, nullptr, nullptr, nullptr, bin_of.p, stats);
+            AMGT_LAUNCHED();
             if (info && A->blc_num > 0) {
+                k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats, g_tc_thr_spgemm);
                 AMGT_LAUNCHED();
-                k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats.p, g_tc_thr_spgemm);
             }
-            AMGT_LAUNCHED();
-            k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats.p, cursor.p, rows.p);
-            AMGT_LAUNCHED();
         }
-        AMGT_CUDA(cudaMemcpyAsync(hs, stats.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaStreamSynchronize(s));  // sync 1: bin sizes
-        int64_t cnt[NCAT], off[NCAT], acc = 0;
-        for (int b = 0; b < NCAT; ++b) { cnt[b] = (int64_t)hs[cat_stat(b)]; off[b] = acc; acc += cnt[b]; }
-        if (BR > 0) {
-            amgt_status st = run_bins<1>(cnt, off, rows.p, c, B->blc_col, a, nnz_row.p, nullptr, nullptr, nullptr, s);
-            if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
-        }
-        AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s));
-        Scratch<unsigned long long> rmax;  // longest C block row (numeric skips absent row classes)
-        AMGT_TRY(rmax.init(a, 1));
-        AMGT_CUDA(cudaMemsetAsync(rmax.p, 0, sizeof(unsigned long long), s));
-        if (BR > 0) {
-            k_max_rows<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, nnz_row.p, rmax.p);
-            AMGT_LAUNCHED();
-        }
+        AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
         int64_t TC = 0;
         unsigned long long hmax = 0;
+        AMGT_CUDA(cudaMemcpyAsync(hs, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
         AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax.p, sizeof(hmax), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaStreamSynchronize(s));  // sync 2: C tile count (L153)
+        AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));  // sync 1: bins, C tile count (L153)
+        int64_t cnt[NCAT], off[NCAT], acc = 0;
+        for (int b = 0; b < NCAT; ++b) { cnt[b] = (int64_t)hs[cat_stat(b)]; off[b] = acc; acc += cnt[b]; }
+        int64_t big = 0;
+        for (int b = 0; b < NBINS; ++b) big += cnt[b];
+        int64_t cnt_big[NCAT];  // the rows the per-bin kernels take (category 8 is done)
+        for (int b = 0; b < NCAT; ++b) cnt_big[b] = b < NBINS ? cnt[b] : 0;
+        if (big > 0) {  // rows with more than 32 candidates: per-bin hash kernels, then rescan
+            AMGT_TRY(rows.init(a, BR + 1));
+            k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats, cursor, rows.p);
+            AMGT_LAUNCHED();
+            amgt_status st = run_bins<1>(cnt_big, off, rows.p, c, B->blc_col, a, nnz_row.p, nullptr, nullptr, nullptr, s);
+            if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
+            AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
+            AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
+            AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaStreamSynchronize(s));  // sync 2: C tile count with the long rows
+        }
         amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
         if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
         C.row_max = (int64_t)hmax;
         if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
-        if (BR > 0) {
-            st = run_bins<2>(cnt, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
-            if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+        if (BR > 0) {  // step 2 (Alg. 3 lines 13-14 + bitmap OR, R15)
+            k_sym_group<2, true><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
+                BR, nullptr, c, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, bin_of.p, nullptr);
+            AMGT_LAUNCHED();
+            if (big > 0) {
+                st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
+                if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+            }
         }
         ts.bytes = (A->blc_num + B->blc_num) * 6.0 * 2 + (A->blc_row + B->blc_row) * 8.0 + TC * 6.0 + (BR + 1) * 8.0;
     }
