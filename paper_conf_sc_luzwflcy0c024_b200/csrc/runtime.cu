@@ -96,7 +96,7 @@ int g_tc_thr_spmv = 17;
 
 // ------------------------------------------------------------------ scan
 // Block-wide exclusive scan: 1024 threads x 8 items = 8192 items per block.
-constexpr int SCAN_T = 1024, SCAN_I = 8, SCAN_TILE = SCAN_T * SCAN_I;
+constexpr int SCAN_T = 256, SCAN_I = 8, SCAN_TILE = SCAN_T * SCAN_I;  // 2048 items per CTA
 
 __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t* sh_warp, int64_t* total) {
     int lane = threadIdx.x & 31, w = threadIdx.x >> 5;

@@ -1,7 +1,7 @@
 // spgemm.cu — C = A*B over mBSR (§IV.C; Alg. 3; Alg. 4).
 //
 // Pipeline (all on the device; one host sync when every row has <= 32 candidates, else two):
-//   step 1        k_sym_group<1, true> over every block row: Cub(I) = sum_{K in A(I,:)}
+//   step 1        k_sym_flat<1> over every block row: Cub(I) = sum_{K in A(I,:)}
 //                 #tiles(B(K,:)) and bin(I) (L149-151; 8 bins, edges 128*2^b, reading R7)
 //                 and, for the rows with Cub <= 32 (category 8), the distinct tile columns J
 //                 with BITMAPMULTIPLY(mapA, mapB) != 0 (Alg. 3 lines 1-13) -> nnzC_row;
@@ -9,7 +9,7 @@
 //   long rows     (only when some row has Cub > 32) row lists per bin (k_bin_scatter), the
 //                 per-bin hash kernels of step 1, prefix sum again, second host sync.
 //   step 2        insert again, OR the bitmaps (R15), compress, sort ascending (Alg. 3 lines
-//                 13-14) -> blc_idxC, blc_mapC: k_sym_group<2, true> + the per-bin kernels.
+//                 13-14) -> blc_idxC, blc_mapC: k_sym_flat<2> + the per-bin kernels.
 //   numeric       rows by C-row length (<= 8 C tiles: staged 4-lane-group kernel; 9-32: warp
 //                 per row; 33-512; > 512: two passes).  A tiles with POPCOUNT >= threshold go
 //                 to the tensor-core route (DMMA m8n8k4: fragA = [A;A], fragB = [Bj|Bj'],
@@ -51,7 +51,7 @@ struct SymCtx {  // device pointers shared by the symbolic kernels
 };
 
 // ---------------------------------------------------------------- analysis + binning
-// (Cub and the bins are computed by k_sym_group<1, true> below, L149-151.)
+// (Cub and the bins are computed by k_sym_flat<1> below, L149-151.)
 
 // Pair statistics for amgt_spgemm_info (info only): one thread per A tile over its B row.
 __global__ void k_pair_stats(int64_t TA, SymCtx c, unsigned long long* __restrict__ stats, int tc_thr) {
@@ -278,126 +278,159 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
 }
 
 // ---------------------------------------------------------------- step kernels: tiny rows
-// Category 8 (bin-0 rows with Cub <= 32): one 4-lane group per row, 8 rows per warp.  All of
-// the row's candidates (tile column J of every pair with BITMAPMULTIPLY != 0) are written to
-// a per-group list in shared memory; a candidate counts when it is the first occurrence of
-// its J (the collision-free degenerate form of the paper's hash table, with the "hash" being
-// the candidate position).  Step 1 writes the distinct count; step 2 writes each distinct J
-// at its rank with the OR of the bitmaps of all its occurrences.  Deterministic, no atomics.
-//
-// ALL = true: the kernel runs over every block row (rows == nullptr) and does the analysis
-// and binning itself (k_analyze's Cub and bin, L149-151): step 1 computes Cub, writes
-// bin_of[I] and the category counts / Cub total into stats (warp-aggregated atomics), and
-// continues only for category-8 rows (others: nnz_row = 0 here, counted later by their bin's
-// kernel); step 2 processes the rows whose bin_of is 8.  For operators whose rows are all
-// category 8 (every Laplacian RAP) the symbolic phase is then two kernels, one scan and one
-// host synchronisation.
-template <int STEP, bool ALL = false>
-__global__ void __launch_bounds__(256) k_sym_group(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
-                                                   int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
-                                                   int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap,
-                                                   int64_t* __restrict__ bin_of = nullptr,
-                                                   unsigned long long* __restrict__ stats = nullptr) {
-    __shared__ int keys[64][SMALL_CUB];
-    __shared__ uint32_t maps[64][SMALL_CUB];
-    __shared__ unsigned char first[64][SMALL_CUB];
-    const int lane = threadIdx.x & 31, r = lane & 3, gl = threadIdx.x >> 2;
+// Every block row goes through k_sym_flat, which also does the analysis and binning (L149-151:
+// Cub(I) = sum_{K in A(I,:)} #tiles(B(K,:)), bin edges 128*2^b, reading R7).  One warp takes
+// SF_ROWS = 16 consecutive block rows; their A tiles are one contiguous range, which the 32
+// lanes walk 128 tiles at a time (4 per lane: columns, bitmaps, B-row ranges all requested
+// together, so a few dependent round trips per warp instead of per tile).  Each lane appends its tile's (A tile, B tile) pairs to
+// its row's candidate list in shared memory at the row-local pair position (A-tile order, then
+// B order): the candidate is the tile column J when BITMAPMULTIPLY(mapA, mapB) != 0 (Alg. 3
+// lines 7-8).  The list length is Cub.  Rows with Cub <= 32 (category 8) are finished here by
+// one 4-lane group: a candidate counts when it is the first occurrence of its J (the
+// collision-free degenerate form of the paper's hash table, Alg. 3 lines 9-11); step 1 writes
+// the distinct count, step 2 writes each distinct J at its rank with the OR of the bitmaps of
+// all its occurrences (lines 13-14, R15).  Deterministic, no atomics on the data.  Rows with
+// Cub > 32 are only binned here (bin_of, stats) and left to the per-bin hash kernels.
+// (A 4-lane group per row walking its own tiles measured 92 + 104 us for the config-2 A*P
+// steps: latency-bound dependent chains.)
+constexpr int SF_ROWS = 16;  // block rows per warp in k_sym_flat
+constexpr int SF_U = 4;      // A tiles per lane per round (all their loads in flight together)
+template <int STEP>
+__global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t* __restrict__ nnz_row,
+                                                  const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx,
+                                                  uint16_t* __restrict__ cmap, int64_t* __restrict__ bin_of,
+                                                  unsigned long long* __restrict__ stats) {
+    // row stride padded by one word: the 8 groups of a warp read the same position of 8
+    // different rows at once (an unpadded 128-B stride puts them all in one bank)
+    __shared__ int keys[8][SF_ROWS][SMALL_CUB + 1];
+    __shared__ uint32_t maps[8][SF_ROWS][SMALL_CUB + 1];
+    __shared__ unsigned char first[8][SF_ROWS][SMALL_CUB + 4];
+    __shared__ int npair[8][SF_ROWS];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, g = lane >> 2, r = lane & 3;
     const unsigned gm = 0xFu << (lane & ~3);
-    const int64_t rr = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2);
-    if constexpr (ALL) {
-        const bool valid = rr < nrows;
+    const int64_t I0 = ((int64_t)blockIdx.x * 8 + w) * SF_ROWS;
+    if (I0 >= BR) return;  // whole warp
+    const int nr = (int)min((int64_t)SF_ROWS, BR - I0);
+    const int64_t ap = lane <= nr ? c.aptr[I0 + lane] : 0;  // lane k: start of row I0 + k
+    const int64_t T0 = __shfl_sync(0xffffffffu, ap, 0), T1 = __shfl_sync(0xffffffffu, ap, nr);
+    if (lane < SF_ROWS) npair[w][lane] = 0;
+    __syncwarp();
+    for (int64_t base = T0; base < T1; base += 32 * SF_U) {
+        int32_t K[SF_U];
+        uint32_t ma[SF_U];
+        int64_t b0[SF_U];
+        int len[SF_U];
+#pragma unroll
+        for (int u = 0; u < SF_U; ++u) {  // tile base + 32u + lane
+            const int64_t t = base + 32 * u + lane;
+            K[u] = t < T1 ? c.aidx[t] : -1;
+            ma[u] = t < T1 ? c.amap[t] : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < SF_U; ++u) {
+            b0[u] = K[u] >= 0 ? c.bptr[K[u]] : 0;
+            len[u] = K[u] >= 0 ? (int)(c.bptr[K[u] + 1] - b0[u]) : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < SF_U; ++u) {
+            const int64_t t = base + 32 * u + lane;
+            if (__all_sync(0xffffffffu, t >= T1)) break;
+            int row = 0;  // the tile's row within the warp: #{k in 1..nr-1 : start(k) <= t}
+#pragma unroll
+            for (int k = 1; k < SF_ROWS; ++k) {
+                const int64_t sk = __shfl_sync(0xffffffffu, ap, k);
+                row += (k < nr && sk <= t);
+            }
+            int incl = len[u];
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const int y = __shfl_up_sync(0xffffffffu, incl, d);
+                if (lane >= d) incl += y;
+            }
+            const int excl = incl - len[u];
+            const int prow = __shfl_up_sync(0xffffffffu, row, 1);
+            const unsigned seg = __ballot_sync(0xffffffffu, lane == 0 || row != prow);  // segment starts
+            const int start = 31 - __clz(seg & (0xffffffffu >> (31 - lane)));
+            const int excl0 = __shfl_sync(0xffffffffu, excl, start);
+            const int off = npair[w][row] + excl - excl0;
+            int* Kl = keys[w][row];
+            uint32_t* Ml = maps[w][row];
+            for (int jj = 0; jj < len[u] && off + jj < SMALL_CUB; ++jj) {
+                const int64_t j = b0[u] + jj;
+                const uint32_t mc = bitmap_multiply(ma[u], c.bmap[j]);
+                Kl[off + jj] = mc ? c.bidx[j] : -1;
+                Ml[off + jj] = mc;
+            }
+            const bool last = lane == 31 || ((seg >> (lane + 1)) & 1u);
+            __syncwarp();
+            if (last) npair[w][row] += incl - excl0;
+            __syncwarp();
+        }
+    }
+    // rows g and g + 8 of the warp: one 4-lane group each, in turn
+    for (int h = 0; h < SF_ROWS / 8; ++h) {
+        const int gr = g + 8 * h;
+        const bool own = gr < nr;
+        const int64_t I = I0 + gr;
+        const int64_t cub = own ? npair[w][gr] : 0;
+        bool small = false;
         if (STEP == 1) {
-            int64_t cub = 0;
-            if (valid)
-                for (int64_t t = c.aptr[rr] + r; t < c.aptr[rr + 1]; t += 4) {
-                    const int32_t Kc = c.aidx[t];
-                    cub += c.bptr[Kc + 1] - c.bptr[Kc];
-                }
-            cub += __shfl_xor_sync(0xffffffffu, cub, 1);
-            cub += __shfl_xor_sync(0xffffffffu, cub, 2);
             int b = 0;
             while (b < NBINS - 1 && cub >= (128ll << b)) ++b;
             if (b == 0 && cub <= SMALL_CUB) b = NBINS;  // category 8
-            const bool lead = valid && r == 0;
+            small = b == NBINS;
+            const bool lead = own && r == 0;
             if (lead) {
-                bin_of[rr] = b;
-                if (b != NBINS) {
-                    nnz_row[rr] = 0;
-                    atomicAdd(&stats[cat_stat(b)], 1ull);  // rare: rows longer than 32 candidates
+                bin_of[I] = b;
+                if (!small) {
+                    nnz_row[I] = 0;  // counted by its bin's kernel
+                    atomicAdd(&stats[cat_stat(b)], 1ull);
                 }
             }
-            const unsigned n8 = __ballot_sync(0xffffffffu, lead && b == NBINS);
+            const unsigned n8 = __ballot_sync(0xffffffffu, lead && small);
             unsigned long long ct = lead ? (unsigned long long)cub : 0ull;
             for (int d = 16; d; d >>= 1) ct += __shfl_xor_sync(0xffffffffu, ct, d);
             if (lane == 0) {
                 if (n8) atomicAdd(&stats[cat_stat(NBINS)], (unsigned long long)__popc(n8));
                 if (ct) atomicAdd(&stats[8], ct);
             }
-            if (!valid || b != NBINS) return;  // whole group leaves together
         } else {
-            if (!valid || bin_of[rr] != NBINS) return;
+            small = own && cub <= SMALL_CUB;  // same classification as step 1
         }
-    } else {
-        if (rr >= nrows) return;  // whole group leaves together
-    }
-    const int64_t I = ALL ? rr : rows[rr];
-    int* K = keys[gl];
-    uint32_t* Mp = maps[gl];
-    unsigned char* F = first[gl];
-    int64_t npairs = 0;
-    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
-    for (int64_t base = a0; base < a1; base += 4) {  // expand: every pair of the row into the list
-        const int64_t t = base + r;
-        const bool v = t < a1;
-        const int32_t Kc = v ? c.aidx[t] : 0;
-        const uint32_t ma = v ? c.amap[t] : 0u;
-        const int64_t b0 = v ? c.bptr[Kc] : 0;
-        const int64_t len = v ? c.bptr[Kc + 1] - b0 : 0;
-        int64_t incl = len;
-        int64_t y = __shfl_up_sync(gm, incl, 1, 4);
-        if (r >= 1) incl += y;
-        y = __shfl_up_sync(gm, incl, 2, 4);
-        if (r >= 2) incl += y;
-        const int64_t total = __shfl_sync(gm, incl, 3, 4);
-        for (int64_t jj = 0; jj < len; ++jj) {  // lane r writes its A tile's pairs
-            const int64_t j = b0 + jj;
-            const uint32_t mc = bitmap_multiply(ma, c.bmap[j]);
-            const int64_t p = npairs + incl - len + jj;
-            K[p] = mc ? c.bidx[j] : -1;
-            Mp[p] = mc;
+        if (!own || !small) continue;  // group-uniform
+        const int* Kr = keys[w][gr];
+        const uint32_t* Mr = maps[w][gr];
+        unsigned char* F = first[w][gr];
+        const int n = (int)cub;
+        int cnt = 0;
+        for (int i = r; i < n; i += 4) {  // first occurrences
+            const int k = Kr[i];
+            bool f = k >= 0;
+            for (int j = 0; j < i && f; ++j) f = Kr[j] != k;
+            F[i] = f;
+            cnt += f;
         }
-        npairs += total;
-    }
-    __syncwarp(gm);
-    const int n = (int)npairs;
-    int cnt = 0;
-    for (int i = r; i < n; i += 4) {  // first occurrences
-        const int k = K[i];
-        bool f = k >= 0;
-        for (int j = 0; j < i && f; ++j) f = K[j] != k;
-        F[i] = f;
-        cnt += f;
-    }
-    cnt += __shfl_xor_sync(gm, cnt, 1, 4);
-    cnt += __shfl_xor_sync(gm, cnt, 2, 4);
-    if (STEP == 1) {
-        if (r == 0) nnz_row[I] = cnt;
-        return;
-    }
-    __syncwarp(gm);
-    const int64_t out = cptr[I];
-    for (int i = r; i < n; i += 4) {
-        if (!F[i]) continue;
-        const int k = K[i];
-        int rank = 0;
-        uint32_t m = 0;
-        for (int j = 0; j < n; ++j) {
-            const int kj = K[j];
-            rank += (F[j] && kj < k);
-            m |= (kj == k) ? Mp[j] : 0u;
+        cnt += __shfl_xor_sync(gm, cnt, 1, 4);
+        cnt += __shfl_xor_sync(gm, cnt, 2, 4);
+        if (STEP == 1) {
+            if (r == 0) nnz_row[I] = cnt;
+            continue;
         }
-        cidx[out + rank] = k;
-        cmap[out + rank] = (uint16_t)m;
+        __syncwarp(gm);
+        const int64_t out = cptr[I];
+        for (int i = r; i < n; i += 4) {
+            if (!F[i]) continue;
+            const int k = Kr[i];
+            int rank = 0;
+            uint32_t m = 0;
+            for (int j = 0; j < n; ++j) {
+                const int kj = Kr[j];
+                rank += (F[j] && kj < k);
+                m |= (kj == k) ? Mr[j] : 0u;
+            }
+            cidx[out + rank] = k;
+            cmap[out + rank] = (uint16_t)m;
+        }
     }
 }
 
@@ -1870,11 +1903,6 @@ template <int STEP>
 static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_t* rows, const SymCtx& c, int64_t BCB,
                             Alloc& a, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
                             cudaStream_t s) {
-    if (cnt[NBINS] > 0) {
-        k_sym_group<STEP, false><<<(unsigned)ceil_div(ceil_div(cnt[NBINS], 8) * 32, 256), 256, 0, s>>>(
-            cnt[NBINS], rows + off[NBINS], c, nnz_row, cptr, cidx, cmap);
-        AMGT_LAUNCHED();
-    }
     AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, s)));
     AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, s)));
     AMGT_TRY((launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, s)));
@@ -1917,8 +1945,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         // step 1 over every block row: Cub + bins (L149-151) and, for the category-8 rows
         // (Cub <= 32), the distinct tile columns (Alg. 3 lines 1-13)
         if (BR > 0) {
-            k_sym_group<1, true><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
-                BR, nullptr, c, nnz_row.p, nullptr, nullptr, nullptr, bin_of.p, stats);
+            k_sym_flat<1><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nnz_row.p, nullptr, nullptr, nullptr,
+                                                                     bin_of.p, stats);
             AMGT_LAUNCHED();
             if (info && A->blc_num > 0) {
                 k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats, g_tc_thr_spgemm);
@@ -1955,8 +1983,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         C.row_max = (int64_t)hmax;
         if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
         if (BR > 0) {  // step 2 (Alg. 3 lines 13-14 + bitmap OR, R15)
-            k_sym_group<2, true><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
-                BR, nullptr, c, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, bin_of.p, nullptr);
+            k_sym_flat<2><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nullptr, C.blc_ptr, C.blc_idx, C.blc_map,
+                                                                     bin_of.p, nullptr);
             AMGT_LAUNCHED();
             if (big > 0) {
                 st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
