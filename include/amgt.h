@@ -462,6 +462,10 @@ amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H);
 #define AMGT_TIMER_CLASSES 8
 /* on: 0 = off, -1 = all classes, otherwise a bitmask (bit c enables class c). */
 amgt_status amgt_timing_enable(int on);
+/* Record events for one call in `every` (>= 1, default 1) of each enabled class: an event
+ * pair between two programmatically dependent launches breaks their overlap, so sampling
+ * keeps a live measurement from slowing the run it measures.  Reset by nothing. */
+amgt_status amgt_timing_sample(int every);
 amgt_status amgt_timing_reset(void);
 /* Syncs the recorded events; fills ms_total[8], launches[8] and bytes[8] (algorithmic
  * bytes of SURVEY §8(d) per class) on the host. */

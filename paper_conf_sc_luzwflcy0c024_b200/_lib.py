@@ -120,6 +120,7 @@ _sigs = {
     "amgt_hierarchy_destroy": (_int, [_vp]),
     "amgt_timing_enable": (_int, [_int]),
     "amgt_timing_reset": (_int, []),
+    "amgt_timing_sample": (_int, [_int]),
     "amgt_timing_read": (_int, [_P(ctypes.c_double), _P(_i64), _P(ctypes.c_double)]),
     "amgt_launch_count": (_i64, []),
     "amgt_spmv_fused_range": (_int, [_P(c_mbsr), _i64, _i64, _vp, _int, _vp, _int, _int, _vp, _vp, _vp, ctypes.c_double,
@@ -590,6 +591,11 @@ def timing_enable(on=True):
 
 def timing_reset():
     _check(_L.amgt_timing_reset())
+
+
+def timing_sample(every: int = 1):
+    """Time one call in `every` of each enabled class (amgt_timing_sample)."""
+    _check(_L.amgt_timing_sample(int(every)))
 
 
 def timing_read() -> dict:

@@ -302,9 +302,13 @@ static cudaEvent_t pool_event() {
 
 unsigned timing_mask() { return g_timing; }
 
+static int g_sample_every = 1;  // time one scope in N of each class
+static int64_t g_scope_count[AMGT_TIMER_CLASSES] = {};
+
 TimerScope::TimerScope(int c, double b, cudaStream_t st) : cls(c), bytes(b), s(st), slot(-1) {
     if (!(g_timing & (1u << c))) return;
     std::lock_guard<std::mutex> lk(g_tmu);
+    if (g_scope_count[c]++ % g_sample_every != 0) return;
     TimerRec r{c, b, pool_event(), pool_event()};
     cudaEventRecord(r.e0, s);
     g_recs.push_back(r);
@@ -342,8 +346,16 @@ amgt_status amgt_timing_enable(int on) {
     return AMGT_OK;
 }
 
+amgt_status amgt_timing_sample(int every) {
+    if (every < 1) return fail(AMGT_ERR_ARG, "amgt_timing_sample: every must be >= 1");
+    std::lock_guard<std::mutex> lk(g_tmu);
+    g_sample_every = every;
+    return AMGT_OK;
+}
+
 amgt_status amgt_timing_reset(void) {
     std::lock_guard<std::mutex> lk(g_tmu);
+    for (int64_t& n : g_scope_count) n = 0;
     g_recs.clear();
     g_used = 0;
     g_launches.store(0);
