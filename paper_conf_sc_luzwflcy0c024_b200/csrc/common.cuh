@@ -174,7 +174,13 @@ struct EpiArgs {
     double omega;
     int64_t I0, I1;  // block-row range [I0, I1); I1 < 0 = all rows
     void* r = nullptr;  // AMGT_EPI_JACOBI_RES: residual output (y's precision)
+    void* x1 = nullptr;  // EPI_RES_X0: the zero-guess sweep's iterate (y's precision)
 };
+// Internal epilogue (not in the ABI): the residual of the first pre-smoothing sweep from a
+// zero guess, r = b - A x1 with x1 = 0 + w dinv .* (b - 0) formed on the fly at every
+// gathered column (the k_jacobi0 expression, bit-identical), and x1 of the row written too:
+// Alg. 2 lines 2-3 on a coarse level in one pass.  FP32 vectors, FP32/FP16 operators.
+constexpr int EPI_RES_X0 = 5;
 
 // ------------------------------------------------------------------ programmatic dependent launch
 // Inside a PdlScope (the V-cycle and PCG solve loops, including the CUDA-graph capture of the

@@ -19,6 +19,7 @@
 //    default on B200 (DMMA rate == DFMA rate), enabled by
 //    amgt_set_tc_threshold.
 #include <climits>
+#include <type_traits>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -168,8 +169,22 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
                     }
                 }
             }
+            if constexpr (MODE == EPI_RES_X0) {  // x1_J = 0 + w dinv_J (b_J - 0), the k_jacobi0 expression
+                const float om = (float)epi.omega;
 #pragma unroll
-            for (int u = 0; u < U; ++u) xv[u] = nib[u] ? x_quad(x, J[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int u = 0; u < U; ++u) {
+                    xv[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (nib[u]) {
+                        const float4 bq = x_quad((const float*)epi.b, J[u]), dq = x_quad((const float*)epi.dinv, J[u]);
+                        const float zero = 0.f, t0 = 0.f;
+                        xv[u] = make_float4(zero + om * dq.x * (bq.x - t0), zero + om * dq.y * (bq.y - t0),
+                                            zero + om * dq.z * (bq.z - t0), zero + om * dq.w * (bq.w - t0));
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; ++u) xv[u] = nib[u] ? x_quad(x, J[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 acc = (nib[u] & 1u) ? fmaf(a[u].x, xv[u].x, acc) : acc;
@@ -527,9 +542,10 @@ template <typename MatT, typename XT, typename YT, int MODE>
 static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
                         int64_t long_thr, cudaStream_t s) {
     const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE,
-                                (YT*)ea.r};
+                                (YT*)ea.r, (YT*)ea.x1};
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
-    if (P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16 && lanerow_enabled()) {  // ~1 tile per block row
+    if (MODE != EPI_RES_X0 && P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16 &&
+        lanerow_enabled()) {  // ~1 tile per block row
         // vector epilogue when every vector it touches is 4-element aligned
         const uintptr_t al = 4 * sizeof(YT) - 1;
         auto ok = [&](const void* p) { return (reinterpret_cast<uintptr_t>(p) & al) == 0; };
@@ -576,6 +592,14 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
                 break;
             case AMGT_EPI_RESIDUAL: launch_rows<MatT, XT, YT, AMGT_EPI_RESIDUAL>(A, x, y, ea, I0, BR, long_thr, s); break;
             case AMGT_EPI_ACCUM: launch_rows<MatT, XT, YT, AMGT_EPI_ACCUM>(A, x, y, ea, I0, BR, long_thr, s); break;
+            case EPI_RES_X0:
+                if constexpr (sizeof(MatT) < 8 && std::is_same<XT, float>::value && std::is_same<YT, float>::value) {
+                    if (P && P->nlong > 0) return fail(AMGT_ERR_UNSUPPORTED, "zero-guess residual with split long rows");
+                    launch_rows<MatT, XT, YT, EPI_RES_X0>(A, x, y, ea, I0, BR, long_thr, s);
+                } else {
+                    return fail(AMGT_ERR_UNSUPPORTED, "zero-guess residual: FP32 vectors, FP32/FP16 operator only");
+                }
+                break;
             default: launch_rows<MatT, XT, YT, AMGT_EPI_Y>(A, x, y, ea, I0, BR, long_thr, s);
         }
         AMGT_LAUNCHED();
@@ -615,7 +639,7 @@ amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* 
     const double vec = 4.0 * A->blc_row * prec_bytes(yp);
     // epilogue operands read once each: Jacobi b, dinv (+ r written); residual b; accumulate y
     const double extra = ea.mode == AMGT_EPI_JACOBI ? 2 * vec
-                         : ea.mode == AMGT_EPI_JACOBI_RES ? 3 * vec
+                         : (ea.mode == AMGT_EPI_JACOBI_RES || ea.mode == EPI_RES_X0) ? 3 * vec
                          : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
     TimerScope ts(timer_class, spmv_bytes(A, xp, yp) + extra, s);
     switch (A->prec) {

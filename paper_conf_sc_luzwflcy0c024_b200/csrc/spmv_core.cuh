@@ -76,7 +76,8 @@ struct Epi {
     const XT* xs;
     YT omega;
     int mode;
-    YT* r = nullptr;  // EPI_JACOBI_RES only
+    YT* r = nullptr;   // EPI_JACOBI_RES only
+    YT* x1 = nullptr;  // EPI_RES_X0 only
     __device__ __forceinline__ int md() const { return MODE >= 0 ? MODE : mode; }
     // operands of row i, loaded before the tile loop so their latency overlaps it
     struct Pre {
@@ -89,6 +90,7 @@ struct Epi {
             case AMGT_EPI_JACOBI_RES: p.a = b[i]; p.c = dinv[i]; p.d = (YT)xs[i]; break;
             case AMGT_EPI_RESIDUAL: p.a = b[i]; break;
             case AMGT_EPI_ACCUM: p.a = y[i]; break;
+            case EPI_RES_X0: p.a = b[i]; p.c = dinv[i]; break;
             default: break;
         }
         return p;
@@ -106,6 +108,12 @@ struct Epi {
             }
             case AMGT_EPI_RESIDUAL: y[i] = p.a - t; break;
             case AMGT_EPI_ACCUM: y[i] = p.a + t; break;
+            case EPI_RES_X0: {
+                y[i] = p.a - t;
+                const YT zero = YT(0), t0 = YT(0);
+                x1[i] = zero + omega * p.c * (p.a - t0);
+                break;
+            }
             default: y[i] = t;
         }
     }

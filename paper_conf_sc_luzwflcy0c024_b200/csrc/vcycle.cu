@@ -61,7 +61,6 @@ struct amgt_hierarchy {
     // CUDA graph of the sub-cycle below level 1 (levels 2..M down, coarse solve, up), captured
     // once per hierarchy on an internal stream and replayed every cycle
     cudaStream_t gs = nullptr;
-    cudaEvent_t gev[2] = {nullptr, nullptr};
     cudaGraphExec_t gexec = nullptr;
     bool graph_failed = false;
     int64_t sub_calls = 0, sub_launches = 0;
@@ -322,8 +321,6 @@ static void destroy(amgt_hierarchy* H) {
     cudaStreamSynchronize(H->s);
     if (H->gexec) cudaGraphExecDestroy(H->gexec);
     if (H->gs) { cudaStreamSynchronize(H->gs); cudaStreamDestroy(H->gs); }
-    for (cudaEvent_t e : H->gev)
-        if (e) cudaEventDestroy(e);
     delete H;
 }
 
@@ -503,6 +500,17 @@ static amgt_status dense_solve(amgt_hierarchy* H, amgt_level& L) {
 
 constexpr int JAC = 1, RES = 2, ACC = 3;
 
+// AMGT_ZERO_GUESS_FUSED=0: coarse levels run the zero-guess sweep (k_jacobi0) and the residual
+// as two kernels (measurement knob; the results are bit-identical either way)
+static bool zero_guess_fused() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_ZERO_GUESS_FUSED");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 // Alg. 2 lines 2-4 at level k: pre-smoothing, residual, restriction into b_{k+1}.  With
 // res_norm, the first sweep (level 1, nu1 >= 1) also writes r = b - A x of the incoming x
 // and its squared norm goes to *res_norm: the residual of the previous cycle (L308).
@@ -511,6 +519,20 @@ static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** x
     amgt_level& L = H->L[k];
     const void* bk = k == 0 ? b0 : L.b;
     int i0 = 0;
+    if (k > 0 && H->o.nu1 == 1 && L.vprec == AMGT_FP32 && L.A.prec != AMGT_FP64 && zero_guess_fused()) {
+        // lines 2-3 from the zero guess in one pass: r = b - A x1, x1 = w D^-1 b formed on the
+        // fly (EPI_RES_X0); two of Alg. 2's SpMV operations (the sweep's is A 0 = 0)
+        EpiArgs ea{EPI_RES_X0, bk, L.dinv, nullptr, H->o.omega, 0, -1};
+        ea.x1 = xa[k];
+        const amgt_status st = spmv_ex_impl(&L.A, bk, L.vprec, L.r, L.vprec, ea, H->s, TC_SPMV);
+        if (st == AMGT_OK) {
+            H->spmv_calls += 2;
+            std::swap(xc[k], xa[k]);
+            amgt_level& N = H->L[k + 1];
+            return counted_spmv(H, &L.R, L.r, L.vprec, N.b, N.vprec, k);  // line 4: restriction
+        }
+        if (st != AMGT_ERR_UNSUPPORTED) return st;
+    }
     if (k > 0 && H->o.nu1 >= 1) {  // zero initial guess: first sweep without the SpMV (k_jacobi0)
         TimerScope ts(TC_VEC, 3.0 * vbytes(L.vprec) * L.npad, H->s);
         const dim3 g((unsigned)ceil_div(L.npad, 256));
@@ -1152,8 +1174,6 @@ static amgt_status subcycle(amgt_hierarchy* H, void** xc, void** xa) {
     cudaStream_t user = H->s;
     if (!H->gexec) {
         if (!H->gs) AMGT_CUDA(cudaStreamCreateWithFlags(&H->gs, cudaStreamNonBlocking));
-        for (cudaEvent_t& e : H->gev)
-            if (!e) AMGT_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         void* xc0[8];
         void* xa0[8];
         std::copy(xc, xc + 8, xc0);
@@ -1185,11 +1205,7 @@ static amgt_status subcycle(amgt_hierarchy* H, void** xc, void** xa) {
         std::copy(xa0, xa0 + 8, xa);
         if (!H->gexec) return subcycle_direct(H, xc, xa);
     }
-    AMGT_CUDA(cudaEventRecord(H->gev[0], user));
-    AMGT_CUDA(cudaStreamWaitEvent(H->gs, H->gev[0], 0));
-    AMGT_CUDA(cudaGraphLaunch(H->gexec, H->gs));
-    AMGT_CUDA(cudaEventRecord(H->gev[1], H->gs));
-    AMGT_CUDA(cudaStreamWaitEvent(user, H->gev[1], 0));
+    AMGT_CUDA(cudaGraphLaunch(H->gexec, user));  // replayed on the caller's stream (captured on gs)
     H->spmv_calls += H->sub_calls;
     count_launches(H->sub_launches);
     return AMGT_OK;

@@ -102,3 +102,41 @@ def test_hierarchy_fp16_overflow_reported():
     assert "RANGE" in str(ei.value)
     H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=prec)
     H.close()
+
+
+_ZG_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import gen, paper_conf_sc_luzwflcy0c024_b200 as amgt
+A = gen.laplacian_27pt(32)
+PR = gen.aggregation_hierarchy((32, 32, 32), 5)
+H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=("f64", "f32", "f16", "f16", "f16"))
+b = gen.uniform_vector(A.m, 3).cuda()
+x = torch.zeros(A.m, dtype=torch.float64, device="cuda")
+res, calls = H.vcycle(b, x, 6)
+np.save(sys.argv[2], x.cpu().numpy())
+print(calls)
+"""
+
+
+def test_zero_guess_fused_bit_identical(tmp_path):
+    """The coarse-level zero-guess sweep + residual in one pass (EPI_RES_X0) gives the same
+    iterates, bit for bit, as k_jacobi0 followed by the residual SpMV (separate processes:
+    AMGT_ZERO_GUESS_FUSED is read once per process), and the same SpMV call count."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "zg.py"
+    script.write_text(_ZG_SCRIPT)
+    outs, calls = [], []
+    for flag in ("1", "0"):
+        out = tmp_path / f"x{flag}.npy"
+        env = dict(os.environ, AMGT_ZERO_GUESS_FUSED=flag)
+        p = subprocess.run([sys.executable, str(script), root, str(out)], env=env, capture_output=True, text=True,
+                           timeout=300)
+        assert p.returncode == 0, p.stderr[-2000:]
+        calls.append(int(p.stdout.strip().splitlines()[-1]))
+        outs.append(np.load(out))
+    assert calls[0] == calls[1] == 1 + 6 * (5 * 4 + 1)
+    assert np.array_equal(outs[0].view(np.uint64), outs[1].view(np.uint64))
