@@ -21,6 +21,7 @@
 // row, table per block; bin 7 (Cub >= 8192): dense bitmap over B's tile columns
 // (shared memory when it fits, else a per-block global slice) — sorted by construction.
 #include <algorithm>
+#include <cmath>
 #include <climits>
 
 #include "common.cuh"
@@ -1653,65 +1654,101 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
 }
 
 constexpr int STAGED_WARPS = 4;  // warps per CTA of k_numeric_staged
+constexpr int STAGED_RPG = 4;    // consecutive block rows streamed by one 4-lane group
 
+// The group streams STAGED_RPG consecutive block rows: their A tiles are one contiguous range,
+// walked four tiles per chunk, so the batch pipeline runs across row boundaries and the
+// per-row chain (C row pointers and columns, A row pointers) is loaded once for the four rows
+// up front (lane u: row R0 + u).  A pair carries its row; when the pair being multiplied
+// belongs to a new row, the group writes out the finished row's tiles and switches its
+// column list (kept in shared memory).  Rows with more than GROUP_NC C tiles are listed for
+// the warp / mid / long-row kernels and their A tiles contribute no pairs here.
 template <typename T, typename Acc>
 __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
     int64_t BR, SymCtx c, const T* __restrict__ aval, const T* __restrict__ bval, const int64_t* __restrict__ cptr,
     const int32_t* __restrict__ cidx_g, const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
     int32_t* __restrict__ big, unsigned long long* __restrict__ nbig, int32_t* __restrict__ lng,
-    unsigned long long* __restrict__ nlng, int32_t* __restrict__ mid, unsigned long long* __restrict__ nmid) {
+    unsigned long long* __restrict__ nlng, int32_t* __restrict__ mid, unsigned long long* __restrict__ nmid,
+    int rpg) {
     constexpr int TE = 16;                       // elements per tile
     constexpr int PIECES = TE * sizeof(T) / 16;  // 16-B pieces per tile
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ int32_t s_cid[STAGED_WARPS * 8][STAGED_RPG][GROUP_NC];
+    __shared__ uint16_t s_cmap[STAGED_WARPS * 8][STAGED_RPG][GROUP_NC];
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
+    const int gi = (threadIdx.x >> 5) * 8 + g;  // group index in the CTA
     const unsigned gm = 0xFu << (lane & ~3);
     constexpr int GROUP_BUF = 2 * 4 * 2 * TE;   // two buffers x 4 pairs x (A tile, B tile)
-    T* buf = reinterpret_cast<T*>(smem_raw) + ((size_t)(threadIdx.x >> 5) * 8 + g) * GROUP_BUF;
+    T* buf = reinterpret_cast<T*>(smem_raw) + (size_t)gi * GROUP_BUF;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (wid * 8 >= BR) return;
-    const int64_t I = wid * 8 + g;
-    int64_t c0 = 0;
-    int nC = 0;
-    if (I < BR) {
-        c0 = cptr[I];
-        nC = (int)(cptr[I + 1] - c0);
-        if (nC > GROUP_NC) {
-            if (r == 0) {
-                if (nC <= CAP) big[atomicAdd(nbig, 1ull)] = (int32_t)I;
-                else if (nC <= MIDCAP) mid[atomicAdd(nmid, 1ull)] = (int32_t)I;
-                else lng[atomicAdd(nlng, 1ull)] = (int32_t)I;
-            }
-            nC = 0;
+    if (wid * 8 * rpg >= BR) return;
+    const int64_t R0 = (wid * 8 + g) * rpg;
+    // lane u < rpg: row R0 + u (C range, class; A range start)
+    const int64_t Ir = R0 + r;
+    int64_t rc0 = 0, ra0 = 0;
+    int rnC = 0;
+    if (r < rpg && Ir < BR) {
+        rc0 = cptr[Ir];
+        rnC = (int)(cptr[Ir + 1] - rc0);
+        ra0 = c.aptr[Ir];
+        if (rnC > GROUP_NC) {
+            if (rnC <= CAP) big[atomicAdd(nbig, 1ull)] = (int32_t)Ir;
+            else if (rnC <= MIDCAP) mid[atomicAdd(nmid, 1ull)] = (int32_t)Ir;
+            else lng[atomicAdd(nlng, 1ull)] = (int32_t)Ir;
+            rnC = 0;  // not this kernel's row: its A tiles give no pairs here
         }
     }
-    int32_t cid[GROUP_NC];
+    const int64_t last = min(R0 + rpg, BR);  // one past the group's last row
+    const int64_t A1 = R0 < BR ? c.aptr[last] : 0;
 #pragma unroll
-    for (int k = 0; k < GROUP_NC; ++k) cid[k] = k < nC ? cidx_g[c0 + k] : INT_MAX;
+    for (int k = 0; k < GROUP_NC; ++k) {
+        s_cid[gi][r][k] = k < rnC ? cidx_g[rc0 + k] : INT_MAX;
+        s_cmap[gi][r][k] = k < rnC ? cmap_g[rc0 + k] : (uint16_t)0;
+    }
+    // row starts / sizes of the four rows, in every lane of the group
+    int64_t rs[STAGED_RPG];
+    int rn[STAGED_RPG];
+#pragma unroll
+    for (int u = 0; u < STAGED_RPG; ++u) {
+        rs[u] = __shfl_sync(gm, ra0, u, 4);
+        rn[u] = __shfl_sync(gm, rnC, u, 4);
+    }
+    const int nrows = (int)max(last - R0, (int64_t)0);
     Acc acc[GROUP_NC][4];
 #pragma unroll
     for (int k = 0; k < GROUP_NC; ++k)
 #pragma unroll
         for (int e = 0; e < 4; ++e) acc[k][e] = Acc(0);
+    int32_t cid[GROUP_NC];
+    int cur = -1;  // row (0..3) whose C tiles acc holds
     // A-tile chunk cache: lane u holds tile cbase+u (bitmap, B-row start, exclusive pair
-    // offset); the next chunk's column / bitmap are prefetched one chunk ahead (pK, pma).
-    int64_t cbase = 0, a1 = 0, myb0 = 0;
-    int myE = 0, S = 0, pos = 0;
+    // offset, row); the next chunk's column / bitmap are prefetched one chunk ahead (pK, pma).
+    int64_t cbase = 0, myb0 = 0;
+    int myE = 0, S = 0, pos = 0, myrow = 0;
     uint32_t mycma = 0, pma = 0;
     int32_t pK = -1;
     auto prefetch = [&](int64_t base) {
         const int64_t tt = base + r;
         pK = -1;
-        if (tt < a1) {
+        if (tt < A1) {
             pK = c.aidx[tt];
             pma = c.amap[tt];
         }
     };
     auto load_chunk = [&](int64_t base) {  // consumes the prefetched metadata of `base`
         cbase = base;
+        const int64_t tt = base + r;
+        int ri = 0;
+#pragma unroll
+        for (int u = 1; u < STAGED_RPG; ++u) ri += (u < nrows && rs[u] <= tt);
+        int rnc = 0;
+#pragma unroll
+        for (int u = 0; u < STAGED_RPG; ++u) rnc = (u == ri) ? rn[u] : rnc;
+        myrow = ri;
         int len = 0;
         myb0 = 0;
         mycma = 0;
-        if (pK >= 0) {
+        if (pK >= 0 && rnc > 0) {
             mycma = pma;
             myb0 = c.bptr[pK];
             len = (int)(c.bptr[pK + 1] - myb0);
@@ -1725,22 +1762,19 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         pos = 0;
         prefetch(base + 4);
     };
-    if (nC > 0) {
-        a1 = c.aptr[I + 1];
-        const int64_t a0 = c.aptr[I];
-        prefetch(a0);
-        load_chunk(a0);
-    }
+    const int64_t A0 = nrows > 0 ? rs[0] : 0;
+    prefetch(A0);
+    load_chunk(A0);
     // Batch = the group's next 4 pairs: lane u resolves pair u (A tile, B tile, bitmap,
-    // column; the bitmap/column loads stay in flight until the batch is computed) and the
-    // group issues the cp.async copies of the 8 operand tiles into buffer `nb`.
+    // column, row; the bitmap/column loads stay in flight until the batch is computed) and
+    // the group issues the cp.async copies of the 8 operand tiles into buffer `nb`.
     struct Batch {
         bool valid;
         uint32_t ma;
-        int64_t j;
+        int row;
     };
     auto issue = [&](int nb, Batch& B, uint32_t& bm, int32_t& bj) {
-        while (pos >= S && cbase + 4 < a1) load_chunk(cbase + 4);  // group-uniform
+        while (pos >= S && cbase + 4 < A1) load_chunk(cbase + 4);  // group-uniform
         const bool has = pos < S;
         const int p = pos + r;
         B.valid = has && p < S;
@@ -1749,13 +1783,14 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         const int64_t ob0 = __shfl_sync(gm, myb0, o, 4);
         const int oE = __shfl_sync(gm, myE, o, 4);
         B.ma = __shfl_sync(gm, mycma, o, 4);
+        B.row = __shfl_sync(gm, myrow, o, 4);
         const int64_t tu = cbase + o;
-        B.j = ob0 + (p - oE);
+        const int64_t ju = ob0 + (p - oE);
         bm = 0;
         bj = 0;
         if (B.valid) {
-            bm = c.bmap[B.j];
-            bj = c.bidx[B.j];
+            bm = c.bmap[ju];
+            bj = c.bidx[ju];
         }
         T* bb = buf + nb * (GROUP_BUF / 2);
 #pragma unroll
@@ -1763,7 +1798,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
             const int src = (lane & ~3) + v;
             const bool vv = __shfl_sync(0xffffffffu, B.valid, src);
             const int64_t tv = __shfl_sync(0xffffffffu, tu, src);
-            const int64_t jv = __shfl_sync(0xffffffffu, B.j, src);
+            const int64_t jv = __shfl_sync(0xffffffffu, ju, src);
             if (vv) {
 #pragma unroll
                 for (int k = r; k < 2 * PIECES; k += 4) {
@@ -1778,28 +1813,57 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         if (has) pos += 4;
         return has;
     };
-    Batch cur, nxt;
+    // write row `row`'s tiles: lane r writes row r of each tile, +0.0 where the bit is clear (R2)
+    auto flush = [&](int row) {
+        int64_t c0 = 0;
+        int nC = 0;
+#pragma unroll
+        for (int u = 0; u < STAGED_RPG; ++u) nC = (u == row) ? rn[u] : nC;
+        c0 = __shfl_sync(gm, rc0, row, 4);
+#pragma unroll
+        for (int k = 0; k < GROUP_NC; ++k) {
+            if (k < nC) {
+                const uint32_t nib = (s_cmap[gi][row][k] >> (4 * r)) & 0xFu;
+                Acc o[4];
+#pragma unroll
+                for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? acc[k][e] : Acc(0);
+                if constexpr (sizeof(T) == 8)
+                    group_store_tile_f64((double*)(cval + 16 * (c0 + k)), o, r, gm, lane & ~3);
+                else
+                    RowIO<T>::store(cval + 16 * (c0 + k) + 4 * r, o);
+            }
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[k][e] = Acc(0);
+        }
+    };
+    __syncwarp();  // s_cid / s_cmap written by the group's lanes
+    Batch curb, nxtb;
     uint32_t cbm, nbm;
     int32_t cbj, nbj;
-    bool chas = issue(0, cur, cbm, cbj);
+    bool chas = issue(0, curb, cbm, cbj);
     for (int k = 0;; ++k) {
         if (!__any_sync(0xffffffffu, chas)) break;
-        const bool nhas = issue((k + 1) & 1, nxt, nbm, nbj);
+        const bool nhas = issue((k + 1) & 1, nxtb, nbm, nbj);
         asm volatile("cp.async.wait_group 1;" ::: "memory");  // batch k's copies have landed
         __syncwarp();
-        uint32_t mC = 0;
-        int q = 0;
-        if (cur.valid) {
-            mC = bitmap_multiply(cur.ma, cbm);
-#pragma unroll
-            for (int kk = 0; kk < GROUP_NC; ++kk) q = (cid[kk] == cbj) ? kk : q;
-        }
+        const uint32_t mC = curb.valid ? bitmap_multiply(curb.ma, cbm) : 0u;
         const T* bb = buf + (k & 1) * (GROUP_BUF / 2);
 #pragma unroll
         for (int v = 0; v < 4; ++v) {
-            const uint32_t mv = __shfl_sync(0xffffffffu, mC, (lane & ~3) + v);
-            const int qv = __shfl_sync(0xffffffffu, q, (lane & ~3) + v);
+            const int src = (lane & ~3) + v;
+            const uint32_t mv = __shfl_sync(0xffffffffu, mC, src);
+            const int rv = __shfl_sync(0xffffffffu, curb.row, src);
+            const int32_t Jv = __shfl_sync(0xffffffffu, cbj, src);
             if (mv) {  // lane r: row r of A_t * B_j, same FMA order as k_numeric_group
+                if (rv != cur) {  // group-uniform: a new C block row starts
+                    if (cur >= 0) flush(cur);
+                    cur = rv;
+#pragma unroll
+                    for (int kk = 0; kk < GROUP_NC; ++kk) cid[kk] = s_cid[gi][cur][kk];
+                }
+                int q = 0;
+#pragma unroll
+                for (int kk = 0; kk < GROUP_NC; ++kk) q = (cid[kk] == Jv) ? kk : q;
                 Acc arow[4], b0[4], b1[4], b2[4], b3[4], w[4];
                 const T* at = bb + (v * 2) * TE;
                 const T* bt = at + TE;
@@ -1818,31 +1882,19 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
                 }
 #pragma unroll
                 for (int kk = 0; kk < GROUP_NC; ++kk)
-                    if (kk == qv)
+                    if (kk == q)
 #pragma unroll
                         for (int e = 0; e < 4; ++e) acc[kk][e] += w[e];
             }
         }
         __syncwarp();  // buffer k&1 is refilled by the next issue
-        cur = nxt;
+        curb = nxtb;
         cbm = nbm;
         cbj = nbj;
         chas = nhas;
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
-#pragma unroll
-    for (int k = 0; k < GROUP_NC; ++k) {
-        if (k < nC) {
-            const uint32_t nib = (cmap_g[c0 + k] >> (4 * r)) & 0xFu;
-            Acc o[4];
-#pragma unroll
-            for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? acc[k][e] : Acc(0);
-            if constexpr (sizeof(T) == 8)
-                group_store_tile_f64((double*)(cval + 16 * (c0 + k)), o, r, gm, lane & ~3);
-            else
-                RowIO<T>::store(cval + 16 * (c0 + k) + 4 * r, o);
-        }
-    }
+    if (cur >= 0) flush(cur);
 }
 
 static unsigned capped(int64_t blocks) {
@@ -2041,9 +2093,13 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
             AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
         }
         attr = true;
-        k_numeric_staged<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8), STAGED_WARPS), STAGED_WARPS * 32, sm, s>>>(
+        // rows per group: several when rows are short (mean pairs per row ~ (T_A/BR_A)(T_B/BR_B)),
+        // one when a row alone keeps the batch pipeline busy (and the grid large)
+        const double mp = (BR ? (double)A->blc_num / BR : 0.0) * (B->blc_row ? (double)B->blc_num / B->blc_row : 0.0);
+        const int rpg = (int)std::max(1.0, std::min((double)STAGED_RPG, std::floor(32.0 / std::max(mp, 1.0))));
+        k_numeric_staged<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8 * rpg), STAGED_WARPS), STAGED_WARPS * 32, sm, s>>>(
             BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
-            big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3);
+            big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, rpg);
     } else {
         k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
             BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
