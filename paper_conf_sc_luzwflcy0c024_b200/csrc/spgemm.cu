@@ -1955,14 +1955,29 @@ template <int STEP>
 static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_t* rows, const SymCtx& c, int64_t BCB,
                             Alloc& a, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
                             cudaStream_t s) {
+    // Bins >= dense_from take the dense-bitmap kernel (a bitmap over B's W = BC/32 column
+    // words: sorted by construction, cost ~ W + Cub per row) instead of a hash table + bitonic
+    // sort (~ Cub log^2 Cub): from the first bin whose lower edge 128*2^(b-1) reaches W/16,
+    // while the bitmap fits in shared memory (measured on config 4, W = 8192: bins >= 3
+    // 2.2 ms symbolic vs 3.6 ms with bin 7 alone dense).  AMGT_DENSE_FROM_BIN overrides.
+    static const int dense_env = [] { const char* e = getenv("AMGT_DENSE_FROM_BIN"); return e ? atoi(e) : -1; }();
+    const int64_t W = ceil_div(BCB, 32);
+    int dense_from = 7;
+    if (W * 2 * (int64_t)sizeof(uint32_t) <= 160 * 1024)
+        for (int b = 2; b < 7; ++b)
+            if ((128ll << (b - 1)) * 16 >= W) { dense_from = b; break; }
+    if (dense_env >= 2 && dense_env <= 7) dense_from = dense_env;
+    auto block_bin = [&](int b, auto launch) -> amgt_status { return b < dense_from ? launch() : AMGT_OK; };
     AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, s)));
     AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_dense_bin<STEP>(cnt[7], rows + off[7], c, BCB, a, nnz_row, cptr, cidx, cmap, s)));
+    AMGT_TRY(block_bin(2, [&] { return launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, s); }));
+    AMGT_TRY(block_bin(3, [&] { return launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, s); }));
+    AMGT_TRY(block_bin(4, [&] { return launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, s); }));
+    AMGT_TRY(block_bin(5, [&] { return launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, s); }));
+    AMGT_TRY(block_bin(6, [&] { return launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, s); }));
+    int64_t nd = 0;  // bins dense_from..7 are contiguous in the row lists
+    for (int b = dense_from; b < NBINS; ++b) nd += cnt[b];
+    AMGT_TRY((launch_dense_bin<STEP>(nd, rows + off[dense_from], c, BCB, a, nnz_row, cptr, cidx, cmap, s)));
     return AMGT_OK;
 }
 

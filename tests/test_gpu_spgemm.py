@@ -223,3 +223,40 @@ def test_spgemm_fp16_tc_tolerance(thr):
         amgt.set_tc_threshold(17, 17)
     _, _, v = tile_values_to_csr_order(C)
     assert rel_2(v, Co.val) <= 5e-3
+
+
+_BINS_SCRIPT = r"""
+import sys, numpy as np
+sys.path.insert(0, sys.argv[1])
+import gen, paper_conf_sc_luzwflcy0c024_b200 as amgt
+A = gen.irregular_block_sparse(1 << 11, seed=5)
+M = amgt.from_csr(A)
+C = amgt.spgemm(M, M)
+np.savez(sys.argv[2], ptr=C.blc_ptr.cpu().numpy(), idx=C.blc_idx.cpu().numpy(), map=C.map_u16().cpu().numpy(),
+         val=C.blc_val.cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("dense_from", ["2", "7"])
+def test_spgemm_hash_and_dense_bins_agree(tmp_path, dense_from):
+    """The per-bin hash kernels (bins 2-6) and the dense-bitmap kernel give the same C:
+    AMGT_DENSE_FROM_BIN = 7 (hash for bins 2-6) and 2 (dense for all of them) in separate
+    processes (the knob is read once), each bit-exact in structure against the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "bins.py"
+    script.write_text(_BINS_SCRIPT)
+    out = tmp_path / "c.npz"
+    env = dict(os.environ, AMGT_DENSE_FROM_BIN=dense_from)
+    p = subprocess.run([sys.executable, str(script), root, str(out)], env=env, capture_output=True, text=True,
+                       timeout=300)
+    assert p.returncode == 0, p.stderr[-2000:]
+    got = np.load(out)
+    A = gen.irregular_block_sparse(1 << 11, seed=5)
+    Ao = oracle.as_csr(A)
+    Co = oracle.csr_to_mbsr(oracle.spgemm(Ao, Ao))
+    assert np.array_equal(got["ptr"], Co.blc_ptr)
+    assert np.array_equal(got["idx"], Co.blc_idx)
+    assert np.array_equal(got["map"], Co.blc_map.astype(np.int32))
