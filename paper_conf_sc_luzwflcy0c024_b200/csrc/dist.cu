@@ -152,14 +152,18 @@ amgt_status halo_begin(Ctx& c, const amgt_dist_level& L, void* xe) {
 }
 
 // distributed A_k SpMV with epilogue: y = epi(A xe)
-amgt_status dspmv(Ctx& c, const amgt_dist_level& L, int k, void* xe, void* y, int mode, const void* b, const void* xs) {
-    ++c.calls;
+// r (AMGT_EPI_JACOBI_RES only): the residual of the sweep's input, written in the same pass
+amgt_status dspmv(Ctx& c, const amgt_dist_level& L, int k, void* xe, void* y, int mode, const void* b, const void* xs,
+                  void* r = nullptr) {
+    c.calls += mode == AMGT_EPI_JACOBI_RES ? 2 : 1;  // the fused sweep stands for two of Alg. 2's SpMVs
     AMGT_TRY(halo_begin(c, L, xe));
     const int tcls = k == 0 ? TC_SPMV_L1 : TC_SPMV;
     const int64_t BR = L.A->blc_row;
     auto run = [&](int64_t i0, int64_t i1) -> amgt_status {
         if (i1 <= i0) return AMGT_OK;
-        return spmv_ex_impl(L.A, xe, L.vprec, y, L.vprec, EpiArgs{mode, b, L.dinv, xs, c.omega, i0, i1}, c.s, tcls);
+        EpiArgs ea{mode, b, L.dinv, xs, c.omega, i0, i1};
+        ea.r = r;
+        return spmv_ex_impl(L.A, xe, L.vprec, y, L.vprec, ea, c.s, tcls);
     };
     const bool has_int = L.int1 > L.int0 && (L.nsend + L.nrecv) > 0;  // no halo: one launch
     if (has_int) AMGT_TRY(run(L.int0, L.int1));
@@ -248,8 +252,7 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* Ls, 
     std::vector<int> cur(nlev, 0);
     const amgt_dist_level& L0 = Ls[0];
     AMGT_CUDA(cudaMemcpyAsync(own(L0, 0), x, L0.m * sizeof(double), cudaMemcpyDeviceToDevice, s));
-    auto resnorm = [&](int slot) -> amgt_status {
-        AMGT_TRY(dspmv(c, L0, 0, L0.xe[cur[0]], L0.r, RES, b, nullptr));
+    auto norm_of_r = [&](int slot) -> amgt_status {  // ||r_1||^2 into norms[slot] (all ranks)
         k_sq_partial<<<NB, 256, 0, s>>>(4 * L0.A->blc_row, (const double*)L0.r, part.p);
         AMGT_LAUNCHED();
         k_sq_final<<<1, 32, 0, s>>>(part.p, norms.p + slot);
@@ -258,16 +261,30 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* Ls, 
             AMGT_NCCL(g_nccl.AllReduce(norms.p + slot, norms.p + slot, 1, NCCL_FLOAT64, NCCL_SUM, D->comm, s));
         return AMGT_OK;
     };
-    auto smooth = [&](int k, const void* bk, int sweeps) -> amgt_status {
+    auto resnorm = [&](int slot) -> amgt_status {
+        AMGT_TRY(dspmv(c, L0, 0, L0.xe[cur[0]], L0.r, RES, b, nullptr));
+        return norm_of_r(slot);
+    };
+    // The residual after cycle c (L308) is what cycle c+1's first level-1 pre-smoothing sweep
+    // computes anyway (same x, same arithmetic): that sweep also writes r (AMGT_EPI_JACOBI_RES)
+    // and the norm is taken from it, as in the single-GPU amgt_vcycle; only the last cycle's
+    // residual needs its own pass over A_1.
+    const bool fused = nu1 >= 1 && M > 0;
+    auto smooth = [&](int k, const void* bk, int sweeps, int norm_slot = -1) -> amgt_status {
         const amgt_dist_level& L = Ls[k];
         for (int i = 0; i < sweeps; ++i) {
             const int src = cur[k], dst = 1 - src;
-            AMGT_TRY(dspmv(c, L, k, L.xe[src], own(L, dst), JAC, bk, own(L, src)));
+            if (i == 0 && norm_slot >= 0) {
+                AMGT_TRY(dspmv(c, L, k, L.xe[src], own(L, dst), AMGT_EPI_JACOBI_RES, bk, own(L, src), L.r));
+                AMGT_TRY(norm_of_r(norm_slot));
+            } else {
+                AMGT_TRY(dspmv(c, L, k, L.xe[src], own(L, dst), JAC, bk, own(L, src)));
+            }
             cur[k] = dst;
         }
         return AMGT_OK;
     };
-    AMGT_TRY(resnorm(0));
+    if (!fused || ncycles == 0) AMGT_TRY(resnorm(0));
     for (int cyc = 1; cyc <= ncycles; ++cyc) {
         for (int k = 0; k < M; ++k) {  // Alg. 2 lines 1-5
             const amgt_dist_level& L = Ls[k];
@@ -276,7 +293,7 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* Ls, 
                 cur[k] = 0;
                 AMGT_CUDA(cudaMemsetAsync(own(L, 0), 0, 4 * L.A->blc_row * vb(L.vprec), s));
             }
-            AMGT_TRY(smooth(k, bk, nu1));
+            AMGT_TRY(smooth(k, bk, nu1, (k == 0 && fused) ? cyc - 1 : -1));
             AMGT_TRY(dspmv(c, L, k, L.xe[cur[k]], L.r, RES, bk, nullptr));
             AMGT_TRY(local_spmv(c, L.R, L.r, L.vprec, Ls[k + 1].b, Ls[k + 1].vprec, 0));
         }
@@ -312,7 +329,7 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* Ls, 
             AMGT_TRY(local_spmv(c, L.P, own(N, cur[k + 1]), N.vprec, own(L, cur[k]), L.vprec, ACC));
             AMGT_TRY(smooth(k, bk, nu2));
         }
-        AMGT_TRY(resnorm(cyc));
+        if (!fused || cyc == ncycles) AMGT_TRY(resnorm(cyc));
     }
     AMGT_CUDA(cudaMemcpyAsync(x, own(L0, cur[0]), L0.m * sizeof(double), cudaMemcpyDeviceToDevice, s));
     std::vector<double> hn(ncycles + 1);
