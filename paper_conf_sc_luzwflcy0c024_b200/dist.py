@@ -68,6 +68,20 @@ class Comm:
         return t
 
     def allgather_obj(self, obj):
+        """All-gather a small Python value.  Integers and tuples of integers (every use in the
+        setup: row ranges, extended ranges, counts) go through one int64 tensor all-gather;
+        anything else through all_gather_object (pickled)."""
+        if self.size == 1:
+            return [obj]
+        ints = isinstance(obj, int) or (isinstance(obj, tuple) and all(isinstance(v, int) for v in obj))
+        if ints:
+            vals = [obj] if isinstance(obj, int) else list(obj)
+            dev = torch.device("cuda", torch.cuda.current_device()) if self.nccl else torch.device("cpu")
+            t = torch.tensor(vals, dtype=torch.int64, device=dev)
+            outs = [torch.empty_like(t) for _ in range(self.size)]
+            dist.all_gather(outs, t, group=self.group)
+            host = torch.stack(outs).cpu().tolist()
+            return [h[0] if isinstance(obj, int) else tuple(h) for h in host]
         out = [None] * self.size
         dist.all_gather_object(out, obj, group=self.group)
         return out
