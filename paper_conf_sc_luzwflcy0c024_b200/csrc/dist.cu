@@ -115,6 +115,18 @@ __global__ void k_sq_final(const double* __restrict__ part, double* __restrict__
         *out = a;
     }
 }
+// first pre-smoothing sweep of a coarse level from x = 0: x = 0 + w dinv .* (b - 0) on the own
+// rows (the SpMV of the zero vector and its halo exchange are skipped; same expression as the
+// single-GPU k_jacobi0)
+template <typename V>
+__global__ void k_zero_sweep(int64_t n, const V* __restrict__ b, const V* __restrict__ dinv, V omega,
+                             V* __restrict__ x) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const V zero = V(0), t = V(0);
+    x[i] = zero + omega * dinv[i] * (b[i] - t);
+}
+
 template <typename V>
 __global__ void k_dense_apply(int64_t n, const double* __restrict__ Ainv, const V* __restrict__ b, V* __restrict__ x) {
     const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -289,11 +301,27 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* Ls, 
         for (int k = 0; k < M; ++k) {  // Alg. 2 lines 1-5
             const amgt_dist_level& L = Ls[k];
             const void* bk = k == 0 ? (const void*)b : L.b;
+            int sweeps = nu1;
             if (k > 0) {
-                cur[k] = 0;
-                AMGT_CUDA(cudaMemsetAsync(own(L, 0), 0, 4 * L.A->blc_row * vb(L.vprec), s));
+                const int64_t nk = 4 * L.A->blc_row;
+                if (nu1 >= 1) {  // zero initial guess: the first sweep is w D^-1 b (no SpMV, no halo)
+                    const unsigned g = (unsigned)ceil_div(nk, 256);
+                    if (L.vprec == AMGT_FP64)
+                        k_zero_sweep<double><<<g, 256, 0, s>>>(nk, (const double*)bk, (const double*)L.dinv, omega,
+                                                                (double*)own(L, 1));
+                    else
+                        k_zero_sweep<float><<<g, 256, 0, s>>>(nk, (const float*)bk, (const float*)L.dinv, (float)omega,
+                                                               (float*)own(L, 1));
+                    AMGT_LAUNCHED();
+                    ++c.calls;  // Alg. 2's sweep (its SpMV is A 0 = 0)
+                    cur[k] = 1;
+                    sweeps = nu1 - 1;
+                } else {
+                    cur[k] = 0;
+                    AMGT_CUDA(cudaMemsetAsync(own(L, 0), 0, nk * vb(L.vprec), s));
+                }
             }
-            AMGT_TRY(smooth(k, bk, nu1, (k == 0 && fused) ? cyc - 1 : -1));
+            AMGT_TRY(smooth(k, bk, sweeps, (k == 0 && fused) ? cyc - 1 : -1));
             AMGT_TRY(dspmv(c, L, k, L.xe[cur[k]], L.r, RES, bk, nullptr));
             AMGT_TRY(local_spmv(c, L.R, L.r, L.vprec, Ls[k + 1].b, Ls[k + 1].vprec, 0));
         }
