@@ -175,12 +175,20 @@ struct EpiArgs {
     int64_t I0, I1;  // block-row range [I0, I1); I1 < 0 = all rows
     void* r = nullptr;  // AMGT_EPI_JACOBI_RES: residual output (y's precision)
     void* x1 = nullptr;  // EPI_RES_X0: the zero-guess sweep's iterate (y's precision)
+    double* nws = nullptr;  // EPI_JACOBI_NORM: one partial per warp
 };
 // Internal epilogue (not in the ABI): the residual of the first pre-smoothing sweep from a
 // zero guess, r = b - A x1 with x1 = 0 + w dinv .* (b - 0) formed on the fly at every
 // gathered column (the k_jacobi0 expression, bit-identical), and x1 of the row written too:
 // Alg. 2 lines 2-3 on a coarse level in one pass.  FP32 vectors, FP32/FP16 operators.
 constexpr int EPI_RES_X0 = 5;
+// Internal epilogue: the Jacobi sweep (as AMGT_EPI_JACOBI) plus, per warp of the row kernel,
+// the sum of (b_i - (A x)_i)^2 over its rows (xor-tree) into nws[warp] — the residual norm of
+// the sweep's input without writing r (a deterministic fixed-order sum of the partials
+// follows).  FP64 operator and vectors, no long rows (spmv_warp_norm_ok).
+constexpr int EPI_JACOBI_NORM = 6;
+bool spmv_warp_norm_ok(const amgt_mbsr* A);
+int64_t spmv_warp_norm_count(const amgt_mbsr* A);  // partials written (warps of the row kernel)
 
 // ------------------------------------------------------------------ programmatic dependent launch
 // Inside a PdlScope (the V-cycle and PCG solve loops, including the CUDA-graph capture of the

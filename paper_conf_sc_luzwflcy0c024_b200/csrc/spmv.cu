@@ -142,8 +142,17 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
         }
         const double s0 = L.acc0 + __shfl_xor_sync(0xffffffffu, L.acc0, 1);
         const double s1 = L.acc1 + __shfl_xor_sync(0xffffffffu, L.acc1, 1);
-        const int myrow = (q == 0) ? 0 : (q == 1) ? 2 : (q == 2) ? 1 : 3;
-        if (write) epi.finish(out_i, (q & 1) ? s1 : s0, pre);
+        if constexpr (MODE == EPI_JACOBI_NORM) {  // per-warp partial of the residual norm
+            double sq = 0.0;
+            if (write) {
+                const double res = (double)epi.finish(out_i, (q & 1) ? s1 : s0, pre);
+                sq = res * res;
+            }
+            for (int d = 16; d; d >>= 1) sq += __shfl_xor_sync(0xffffffffu, sq, d);
+            if (lane == 0) epi.nws[wid] = sq;
+        } else {
+            if (write) epi.finish(out_i, (q & 1) ? s1 : s0, pre);
+        }
     } else {
         // FP32 / FP16 tiles: lane q owns tile row q; U tiles' indices, bitmaps and row values
         // are requested before the x gathers (one dependent round trip per U tiles).
@@ -538,11 +547,18 @@ static bool lanerow_enabled() {
     return v == 1;
 }
 
+bool spmv_warp_norm_ok(const amgt_mbsr* A) {
+    const SpmvPlan* P = (const SpmvPlan*)A->aux;
+    return A->prec == AMGT_FP64 && g_tc_thr_spmv > 16 && P && P->nlong == 0 &&
+           !(P->mean_row <= 2.0 && lanerow_enabled());
+}
+int64_t spmv_warp_norm_count(const amgt_mbsr* A) { return ceil_div(A->blc_row, 8); }
+
 template <typename MatT, typename XT, typename YT, int MODE>
 static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
                         int64_t long_thr, cudaStream_t s) {
     const Epi<XT, YT, MODE> epi{(YT*)y, (const YT*)ea.b, (const YT*)ea.dinv, (const XT*)ea.xs, (YT)ea.omega, MODE,
-                                (YT*)ea.r, (YT*)ea.x1};
+                                (YT*)ea.r, (YT*)ea.x1, ea.nws};
     const SpmvPlan* P = (const SpmvPlan*)A->aux;
     if (MODE != EPI_RES_X0 && P && P->nlong == 0 && P->mean_row <= 2.0 && g_tc_thr_spmv > 16 &&
         lanerow_enabled()) {  // ~1 tile per block row
@@ -592,6 +608,14 @@ static amgt_status launch_spmv(const amgt_mbsr* A, const void* x, void* y, const
                 break;
             case AMGT_EPI_RESIDUAL: launch_rows<MatT, XT, YT, AMGT_EPI_RESIDUAL>(A, x, y, ea, I0, BR, long_thr, s); break;
             case AMGT_EPI_ACCUM: launch_rows<MatT, XT, YT, AMGT_EPI_ACCUM>(A, x, y, ea, I0, BR, long_thr, s); break;
+            case EPI_JACOBI_NORM:
+                if constexpr (sizeof(MatT) == 8 && std::is_same<XT, double>::value && std::is_same<YT, double>::value) {
+                    if (!spmv_warp_norm_ok(A) || ranged) return fail(AMGT_ERR_UNSUPPORTED, "warp-partial norm");
+                    launch_rows<MatT, XT, YT, EPI_JACOBI_NORM>(A, x, y, ea, I0, BR, long_thr, s);
+                } else {
+                    return fail(AMGT_ERR_UNSUPPORTED, "warp-partial norm: FP64 only");
+                }
+                break;
             case EPI_RES_X0:
                 if constexpr (sizeof(MatT) < 8 && std::is_same<XT, float>::value && std::is_same<YT, float>::value) {
                     if (P && P->nlong > 0) return fail(AMGT_ERR_UNSUPPORTED, "zero-guess residual with split long rows");
@@ -638,7 +662,7 @@ amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* 
                          cudaStream_t s, int timer_class) {
     const double vec = 4.0 * A->blc_row * prec_bytes(yp);
     // epilogue operands read once each: Jacobi b, dinv (+ r written); residual b; accumulate y
-    const double extra = ea.mode == AMGT_EPI_JACOBI ? 2 * vec
+    const double extra = (ea.mode == AMGT_EPI_JACOBI || ea.mode == EPI_JACOBI_NORM) ? 2 * vec
                          : (ea.mode == AMGT_EPI_JACOBI_RES || ea.mode == EPI_RES_X0) ? 3 * vec
                          : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
     TimerScope ts(timer_class, spmv_bytes(A, xp, yp) + extra, s);

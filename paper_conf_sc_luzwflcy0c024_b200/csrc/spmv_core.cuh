@@ -78,6 +78,7 @@ struct Epi {
     int mode;
     YT* r = nullptr;   // EPI_JACOBI_RES only
     YT* x1 = nullptr;  // EPI_RES_X0 only
+    double* nws = nullptr;  // EPI_JACOBI_NORM only
     __device__ __forceinline__ int md() const { return MODE >= 0 ? MODE : mode; }
     // operands of row i, loaded before the tile loop so their latency overlaps it
     struct Pre {
@@ -87,6 +88,7 @@ struct Epi {
         Pre p;
         switch (md()) {
             case AMGT_EPI_JACOBI:
+            case EPI_JACOBI_NORM:
             case AMGT_EPI_JACOBI_RES: p.a = b[i]; p.c = dinv[i]; p.d = (YT)xs[i]; break;
             case AMGT_EPI_RESIDUAL: p.a = b[i]; break;
             case AMGT_EPI_ACCUM: p.a = y[i]; break;
@@ -95,11 +97,17 @@ struct Epi {
         }
         return p;
     }
+    // returns b_i - (A x)_i for EPI_JACOBI_NORM (0 otherwise)
     template <typename V>
-    __device__ __forceinline__ void finish(int64_t i, V v, const Pre& p) const {
+    __device__ __forceinline__ YT finish(int64_t i, V v, const Pre& p) const {
         const YT t = (YT)v;
         switch (md()) {
             case AMGT_EPI_JACOBI: y[i] = p.d + omega * p.c * (p.a - t); break;
+            case EPI_JACOBI_NORM: {
+                const YT res = p.a - t;
+                y[i] = p.d + omega * p.c * res;
+                return res;
+            }
             case AMGT_EPI_JACOBI_RES: {
                 const YT res = p.a - t;
                 y[i] = p.d + omega * p.c * res;
@@ -116,6 +124,7 @@ struct Epi {
             }
             default: y[i] = t;
         }
+        return YT(0);
     }
     // four consecutive rows i0..i0+3 with 16/32-byte vector accesses (all vectors aligned to
     // 4 elements: the caller checks)

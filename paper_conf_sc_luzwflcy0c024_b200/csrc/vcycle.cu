@@ -55,6 +55,8 @@ struct amgt_hierarchy {
     int64_t nM = 0;
     double* Ainv = nullptr;     // dense inverse of the coarsest operator (FP64, nM x nM)
     double* partial = nullptr;  // norm partial sums
+    double* nws = nullptr;      // per-warp residual partials of the level-1 sweep (EPI_JACOBI_NORM)
+    int64_t nws_n = 0;
     double* norms = nullptr;    // per-cycle squared residual norms (device)
     int norms_cap = 0;
     int64_t spmv_calls = 0;
@@ -169,6 +171,17 @@ __global__ void __launch_bounds__(256, 4) k_dot(int64_t n, const double* __restr
     } else {
         for (int64_t i = gt; i < n; i += nt) s = fma(a[i], b[i], s);
     }
+    finish_sum(s, ws, out);
+}
+
+// *out = sum of a[0..n) (the per-warp residual partials of EPI_JACOBI_NORM), deterministic for
+// the fixed grid of NORM_BLOCKS
+__global__ void __launch_bounds__(256, 4) k_sum(int64_t n, const double* __restrict__ a, double* __restrict__ ws,
+                                                double* __restrict__ out) {
+    pdl_wait();
+    double s = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        s += a[i];
     finish_sum(s, ws, out);
 }
 
@@ -317,6 +330,7 @@ static void destroy(amgt_hierarchy* H) {
     if (H->sw) amgt_sweep_plan_destroy(H->sw, H->s);
     a.put(H->Ainv, (size_t)H->nM * H->nM * sizeof(double));
     a.put(H->partial, (NORM_BLOCKS + 1) * sizeof(double));
+    a.put(H->nws, (size_t)H->nws_n * sizeof(double));
     a.put(H->norms, (size_t)H->norms_cap * sizeof(double));
     cudaStreamSynchronize(H->s);
     if (H->gexec) cudaGraphExecDestroy(H->gexec);
@@ -463,6 +477,9 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     H->partial = (double*)a.get((NORM_BLOCKS + 1) * sizeof(double));
     if (!H->Ainv || !H->partial) return fail(AMGT_ERR_ALLOC, "coarse inverse allocation failed");
     AMGT_CUDA(cudaMemsetAsync(H->partial, 0, (NORM_BLOCKS + 1) * sizeof(double), H->s));
+    H->nws_n = std::max<int64_t>(spmv_warp_norm_count(&H->L[0].A), 1);
+    H->nws = (double*)a.get((size_t)H->nws_n * sizeof(double));
+    if (!H->nws) return fail(AMGT_ERR_ALLOC, "norm partial allocation failed");
     AMGT_CUDA(cudaMemcpyAsync(H->Ainv, inv.data(), n * n * sizeof(double), cudaMemcpyHostToDevice, s));
     AMGT_CUDA(cudaStreamSynchronize(s));
     trace_point("coarse inverse", s);
@@ -550,7 +567,17 @@ static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** x
         AMGT_CUDA(cudaMemsetAsync(xc[k], 0, vbytes(L.vprec) * L.npad, H->s));
     }
     for (int i = i0; i < H->o.nu1; ++i) {  // line 2: pre-smoothing
-        if (i == 0 && res_norm) {
+        if (i == 0 && res_norm && H->nws && L.vprec == AMGT_FP64 && spmv_warp_norm_ok(&L.A)) {
+            // the sweep also sums (b - A x)^2 per warp (r is not written); partials summed in order
+            EpiArgs ea{EPI_JACOBI_NORM, bk, L.dinv, xc[k], H->o.omega, 0, -1};
+            ea.nws = H->nws;
+            AMGT_TRY(spmv_ex_impl(&L.A, xc[k], L.vprec, xa[k], L.vprec, ea, H->s, TC_SPMV_L1));
+            H->spmv_calls += 2;  // Alg. 2's sweep and the residual it delivers (L308)
+            TimerScope ts(TC_VEC, 8.0 * spmv_warp_norm_count(&L.A), H->s);
+            pdl_launch(k_sum, dim3(NORM_BLOCKS), dim3(256), 0, H->s, spmv_warp_norm_count(&L.A), (const double*)H->nws,
+                       H->partial, res_norm);
+            AMGT_LAUNCHED();
+        } else if (i == 0 && res_norm) {
             AMGT_TRY(counted_spmv(H, &L.A, xc[k], L.vprec, xa[k], L.vprec, k, AMGT_EPI_JACOBI_RES, bk, L.dinv, L.r));
             AMGT_TRY(norm_into(H, (const double*)L.r, L.npad, res_norm));
         } else {
