@@ -155,6 +155,11 @@ void count_launch();
 void trace_point(const char* name, cudaStream_t s);  // AMGT_TRACE=1 only (measurement)
 constexpr int PINNED_SLOTS = 64;
 int64_t* pinned_slots();  // per-thread pinned host int64[PINNED_SLOTS], NULL if unavailable
+// slot ranges (a pageable-memory cudaMemcpyAsync D2H stages through the driver and costs
+// tens of microseconds; these small read-backs go to pinned memory instead)
+constexpr int PIN_CREATE = 0;  // [0, 16): hierarchy creation, R_k row maxima (read at later syncs)
+constexpr int PIN_SYM = 16;    // [16, 36): SpGEMM symbolic (16 stats, C tile count, longest row)
+constexpr int PIN_CONV = 40;   // [40, 44): CSR -> mBSR (tile count, flags, longest row)
 void trace_dump();
 struct TimerScope {  // records start/end events on `s` when timing is enabled
     int cls;

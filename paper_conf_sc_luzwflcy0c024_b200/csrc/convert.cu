@@ -448,10 +448,22 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     int64_t hT[1] = {0};
     uint32_t hflag = 0;
     unsigned long long hmax = 0;
-    AMGT_CUDA(cudaMemcpyAsync(hT, M.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    AMGT_CUDA(cudaMemcpyAsync(&hflag, flag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax.p, sizeof(hmax), cudaMemcpyDeviceToHost, s));
-    AMGT_CUDA(cudaStreamSynchronize(s));
+    if (int64_t* pin = pinned_slots()) {  // pinned read-back (pageable D2H copies stage through the driver)
+        int64_t* pc = pin + PIN_CONV;
+        pc[1] = 0;
+        AMGT_CUDA(cudaMemcpyAsync(pc, M.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(pc + 1, flag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(pc + 2, rmax.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+        hT[0] = pc[0];
+        hflag = (uint32_t)pc[1];
+        hmax = (unsigned long long)pc[2];
+    } else {
+        AMGT_CUDA(cudaMemcpyAsync(hT, M.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(&hflag, flag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax.p, sizeof(hmax), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+    }
     if (hflag & FLAG_FORMAT) {
         a.put(M.blc_ptr, (BR + 1) * sizeof(int64_t));
         return fail(AMGT_ERR_FORMAT, "CSR input: row_ptr not monotone from 0 to nnz, or columns unsorted/duplicate/out of range");

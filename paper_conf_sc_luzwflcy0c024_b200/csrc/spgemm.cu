@@ -23,6 +23,7 @@
 #include <algorithm>
 #include <cmath>
 #include <climits>
+#include <cstring>
 
 #include "common.cuh"
 
@@ -2023,10 +2024,26 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
         int64_t TC = 0;
         unsigned long long hmax = 0;
-        AMGT_CUDA(cudaMemcpyAsync(hs, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaStreamSynchronize(s));  // sync 1: bins, C tile count (L153)
+        int64_t* pin = pinned_slots();
+        auto read_back = [&](bool with_stats) -> amgt_status {  // pinned when available
+            if (pin) {
+                int64_t* ps = pin + PIN_SYM;
+                if (with_stats) AMGT_CUDA(cudaMemcpyAsync(ps, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaMemcpyAsync(ps + 16, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaMemcpyAsync(ps + 17, rmax, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaStreamSynchronize(s));
+                if (with_stats) memcpy(hs, ps, sizeof(hs));
+                TC = ps[16];
+                hmax = (unsigned long long)ps[17];
+            } else {
+                if (with_stats) AMGT_CUDA(cudaMemcpyAsync(hs, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaStreamSynchronize(s));
+            }
+            return AMGT_OK;
+        };
+        AMGT_TRY(read_back(true));  // sync 1: bins, C tile count (L153)
         int64_t cnt[NCAT], off[NCAT], acc = 0;
         for (int b = 0; b < NCAT; ++b) { cnt[b] = (int64_t)hs[cat_stat(b)]; off[b] = acc; acc += cnt[b]; }
         int64_t big = 0;
@@ -2041,9 +2058,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
             AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
             AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
-            AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-            AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
-            AMGT_CUDA(cudaStreamSynchronize(s));  // sync 2: C tile count with the long rows
+            AMGT_TRY(read_back(false));  // sync 2: C tile count with the long rows
         }
         amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
         if (st != AMGT_OK) { mbsr_release(&C, a); return st; }

@@ -409,7 +409,7 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             }
             trace_point("P cast", s);
             AMGT_TRY(transpose_impl(&L.P, &L.R, a, pin ? dev.p + 1 + k : nullptr));  // R_k = P_k^T (Alg. 1 line 4)
-            if (pin) AMGT_CUDA(cudaMemcpyAsync(pin + k, dev.p + 1 + k, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            if (pin) AMGT_CUDA(cudaMemcpyAsync(pin + PIN_CREATE + k, dev.p + 1 + k, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
             trace_point("transpose", s);
             // A_{k+1} = R_k (A_k P_k): two SpGEMM calls in level k precision (Alg. 1 line 5)
             amgt_mbsr AP{}, Ac{};
@@ -437,7 +437,7 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             N.ownA = true;
             trace_point("cast Ac", s);
             AMGT_TRY(spmv_analyze_impl(&L.P, a));
-            if (pin) L.R.row_max = pin[k];  // arrived: the SpGEMM symbolic phases synchronised since
+            if (pin) L.R.row_max = pin[PIN_CREATE + k];  // arrived: the SpGEMM symbolic phases synchronised since
             AMGT_TRY(spmv_analyze_impl(&L.R, a));
             trace_point("analyze P R", s);
         }
