@@ -153,13 +153,15 @@ enum TimerClass : int {
 };
 void count_launch();
 void trace_point(const char* name, cudaStream_t s);  // AMGT_TRACE=1 only (measurement)
-constexpr int PINNED_SLOTS = 64;
+constexpr int PINNED_SLOTS = 16384;  // 128 KB
 int64_t* pinned_slots();  // per-thread pinned host int64[PINNED_SLOTS], NULL if unavailable
 // slot ranges (a pageable-memory cudaMemcpyAsync D2H stages through the driver and costs
 // tens of microseconds; these small read-backs go to pinned memory instead)
 constexpr int PIN_CREATE = 0;  // [0, 16): hierarchy creation, R_k row maxima (read at later syncs)
 constexpr int PIN_SYM = 16;    // [16, 36): SpGEMM symbolic (16 stats, C tile count, longest row)
 constexpr int PIN_CONV = 40;   // [40, 44): CSR -> mBSR (tile count, flags, longest row)
+constexpr int PIN_NORMS = 64;  // [64, 1088): V-cycle / PCG residual norms
+constexpr int PIN_COARSE = 2048;  // [2048, 16384): coarsest-level CSR on its way to the host factorisation
 void trace_dump();
 struct TimerScope {  // records start/end events on `s` when timing is enabled
     int cls;

@@ -451,20 +451,43 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     double* v = (double*)a.get(16 * C.A.blc_num * sizeof(double) + 8);
     if (!rp || !ci || !v) return fail(AMGT_ERR_ALLOC, "coarse CSR allocation failed");
     AMGT_TRY(mbsr_to_csr_impl(&C.A, rp, ci, v, a));
+    // read back through the pinned buffer when the coarse CSR fits (pageable D2H copies stage
+    // through the driver); the row pointers and the range flag first, then columns and values
+    int64_t* pc = pin ? pin + PIN_COARSE : nullptr;
+    const int64_t pcap = PINNED_SLOTS - PIN_COARSE;
+    const bool pin_rp = pc && n + 2 <= pcap;
     std::vector<int64_t> hrp(n + 1);
-    AMGT_CUDA(cudaMemcpyAsync(hrp.data(), rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     uint32_t hflag = 0;  // FP16 range flag of every cast above
-    AMGT_CUDA(cudaMemcpyAsync(&hflag, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    AMGT_CUDA(cudaStreamSynchronize(s));
+    if (pin_rp) {
+        pc[n + 1] = 0;
+        AMGT_CUDA(cudaMemcpyAsync(pc, rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(pc + n + 1, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+        std::copy(pc, pc + n + 1, hrp.begin());
+        hflag = (uint32_t)pc[n + 1];
+    } else {
+        AMGT_CUDA(cudaMemcpyAsync(hrp.data(), rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaMemcpyAsync(&hflag, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+    }
     if (hflag & FLAG_RANGE) return fail(AMGT_ERR_RANGE, "hierarchy: a level value exceeds the FP16 range (65504)");
     const int64_t nnz = hrp[n];
     std::vector<int32_t> hci(nnz);
     std::vector<double> hv(nnz);
     if (nnz) {
-        AMGT_CUDA(cudaMemcpyAsync(hci.data(), ci, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaMemcpyAsync(hv.data(), v, nnz * sizeof(double), cudaMemcpyDeviceToHost, s));
+        const int64_t need = nnz + (nnz + 1) / 2;  // values (8 B) then columns (4 B) in int64 slots
+        if (pc && need <= pcap) {
+            AMGT_CUDA(cudaMemcpyAsync(pc, v, nnz * sizeof(double), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaMemcpyAsync(pc + nnz, ci, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaStreamSynchronize(s));
+            memcpy(hv.data(), pc, nnz * sizeof(double));
+            memcpy(hci.data(), pc + nnz, nnz * sizeof(int32_t));
+        } else {
+            AMGT_CUDA(cudaMemcpyAsync(hci.data(), ci, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaMemcpyAsync(hv.data(), v, nnz * sizeof(double), cudaMemcpyDeviceToHost, s));
+            AMGT_CUDA(cudaStreamSynchronize(s));
+        }
     }
-    AMGT_CUDA(cudaStreamSynchronize(s));
     a.put(rp, (n + 1) * sizeof(int64_t));
     a.put(ci, 16 * C.A.blc_num * sizeof(int32_t) + 4);
     a.put(v, 16 * C.A.blc_num * sizeof(double) + 8);
@@ -1350,8 +1373,15 @@ static amgt_status vcycle(amgt_hierarchy* H, const double* b, double* x, int ncy
     if (xc[0] != (void*)x)
         AMGT_CUDA(cudaMemcpyAsync(x, xc[0], L0.npad * sizeof(double), cudaMemcpyDeviceToDevice, s));
     std::vector<double> hn(ncycles + 1);
-    AMGT_CUDA(cudaMemcpyAsync(hn.data(), H->norms, (ncycles + 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
-    AMGT_CUDA(cudaStreamSynchronize(s));
+    int64_t* pin = pinned_slots();
+    if (pin && ncycles + 1 <= PIN_COARSE - PIN_NORMS) {  // pinned read-back
+        AMGT_CUDA(cudaMemcpyAsync(pin + PIN_NORMS, H->norms, (ncycles + 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+        memcpy(hn.data(), pin + PIN_NORMS, (ncycles + 1) * sizeof(double));
+    } else {
+        AMGT_CUDA(cudaMemcpyAsync(hn.data(), H->norms, (ncycles + 1) * sizeof(double), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+    }
     if (res_host)
         for (int c = 0; c <= ncycles; ++c) res_host[c] = std::sqrt(hn[c]);
     if (calls_host) *calls_host = H->spmv_calls;
