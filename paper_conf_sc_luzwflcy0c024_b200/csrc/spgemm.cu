@@ -1664,7 +1664,9 @@ constexpr int STAGED_RPG = 4;    // consecutive block rows streamed by one 4-lan
 // belongs to a new row, the group writes out the finished row's tiles and switches its
 // column list (kept in shared memory).  Rows with more than GROUP_NC C tiles are listed for
 // the warp / mid / long-row kernels and their A tiles contribute no pairs here.
-template <typename T, typename Acc>
+// NC: C tiles per row held in registers (4 when the longest C row has <= 4 tiles: fewer
+// registers, more resident warps), rows with more than GROUP_NC tiles go to the other kernels.
+template <typename T, typename Acc, int NC>
 __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
     int64_t BR, SymCtx c, const T* __restrict__ aval, const T* __restrict__ bval, const int64_t* __restrict__ cptr,
     const int32_t* __restrict__ cidx_g, const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
@@ -1715,12 +1717,12 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         rn[u] = __shfl_sync(gm, rnC, u, 4);
     }
     const int nrows = (int)max(last - R0, (int64_t)0);
-    Acc acc[GROUP_NC][4];
+    Acc acc[NC][4];
 #pragma unroll
-    for (int k = 0; k < GROUP_NC; ++k)
+    for (int k = 0; k < NC; ++k)
 #pragma unroll
         for (int e = 0; e < 4; ++e) acc[k][e] = Acc(0);
-    int32_t cid[GROUP_NC];
+    int32_t cid[NC];
     int cur = -1;  // row (0..3) whose C tiles acc holds
     // A-tile chunk cache: lane u holds tile cbase+u (bitmap, B-row start, exclusive pair
     // offset, row); the next chunk's column / bitmap are prefetched one chunk ahead (pK, pma).
@@ -1822,7 +1824,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         for (int u = 0; u < STAGED_RPG; ++u) nC = (u == row) ? rn[u] : nC;
         c0 = __shfl_sync(gm, rc0, row, 4);
 #pragma unroll
-        for (int k = 0; k < GROUP_NC; ++k) {
+        for (int k = 0; k < NC; ++k) {
             if (k < nC) {
                 const uint32_t nib = (s_cmap[gi][row][k] >> (4 * r)) & 0xFu;
                 Acc o[4];
@@ -1860,11 +1862,11 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
                     if (cur >= 0) flush(cur);
                     cur = rv;
 #pragma unroll
-                    for (int kk = 0; kk < GROUP_NC; ++kk) cid[kk] = s_cid[gi][cur][kk];
+                    for (int kk = 0; kk < NC; ++kk) cid[kk] = s_cid[gi][cur][kk];
                 }
                 int q = 0;
 #pragma unroll
-                for (int kk = 0; kk < GROUP_NC; ++kk) q = (cid[kk] == Jv) ? kk : q;
+                for (int kk = 0; kk < NC; ++kk) q = (cid[kk] == Jv) ? kk : q;
                 Acc arow[4], b0[4], b1[4], b2[4], b3[4], w[4];
                 const T* at = bb + (v * 2) * TE;
                 const T* bt = at + TE;
@@ -1882,7 +1884,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
                     w[e] = s_;
                 }
 #pragma unroll
-                for (int kk = 0; kk < GROUP_NC; ++kk)
+                for (int kk = 0; kk < NC; ++kk)
                     if (kk == q)
 #pragma unroll
                         for (int e = 0; e < 4; ++e) acc[kk][e] += w[e];
@@ -2118,16 +2120,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     const bool tc_route = (sizeof(T) == 8 || sizeof(T) == 2) && g_tc_thr_spgemm <= 16;
     if (!tc_route && staged_env) {
         constexpr size_t sm = (size_t)STAGED_WARPS * 8 * 2 * 4 * 2 * 16 * sizeof(T);
+        const bool nc4 = C->row_max > 0 && C->row_max <= 4;
+        auto kern = nc4 ? k_numeric_staged<T, Acc, 4> : k_numeric_staged<T, Acc, GROUP_NC>;
         static bool attr = false;
         if (!attr && sm > 48 * 1024) {
-            AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+            AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+            AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc, GROUP_NC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           (int)sm));
         }
         attr = true;
         // rows per group: several when rows are short (mean pairs per row ~ (T_A/BR_A)(T_B/BR_B)),
         // one when a row alone keeps the batch pipeline busy (and the grid large)
         const double mp = (BR ? (double)A->blc_num / BR : 0.0) * (B->blc_row ? (double)B->blc_num / B->blc_row : 0.0);
         const int rpg = (int)std::max(1.0, std::min((double)STAGED_RPG, std::floor(32.0 / std::max(mp, 1.0))));
-        k_numeric_staged<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8 * rpg), STAGED_WARPS), STAGED_WARPS * 32, sm, s>>>(
+        kern<<<(unsigned)ceil_div(ceil_div(BR, 8 * rpg), STAGED_WARPS), STAGED_WARPS * 32, sm, s>>>(
             BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
             big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, rpg);
     } else {
