@@ -1666,7 +1666,7 @@ constexpr int STAGED_RPG = 4;    // consecutive block rows streamed by one 4-lan
 // the warp / mid / long-row kernels and their A tiles contribute no pairs here.
 // NC: C tiles per row held in registers (4 when the longest C row has <= 4 tiles: fewer
 // registers, more resident warps), rows with more than GROUP_NC tiles go to the other kernels.
-template <typename T, typename Acc, int NC>
+template <typename T, typename Acc, int NC, int NBUF>
 __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
     int64_t BR, SymCtx c, const T* __restrict__ aval, const T* __restrict__ bval, const int64_t* __restrict__ cptr,
     const int32_t* __restrict__ cidx_g, const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
@@ -1681,7 +1681,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
     const int gi = (threadIdx.x >> 5) * 8 + g;  // group index in the CTA
     const unsigned gm = 0xFu << (lane & ~3);
-    constexpr int GROUP_BUF = 2 * 4 * 2 * TE;   // two buffers x 4 pairs x (A tile, B tile)
+    constexpr int GROUP_BUF = NBUF * 4 * 2 * TE;  // NBUF buffers x 4 pairs x (A tile, B tile)
     T* buf = reinterpret_cast<T*>(smem_raw) + (size_t)gi * GROUP_BUF;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (wid * 8 * rpg >= BR) return;
@@ -1795,7 +1795,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
             bm = c.bmap[ju];
             bj = c.bidx[ju];
         }
-        T* bb = buf + nb * (GROUP_BUF / 2);
+        T* bb = buf + nb * (GROUP_BUF / NBUF);
 #pragma unroll
         for (int v = 0; v < 4; ++v) {
             const int src = (lane & ~3) + v;
@@ -1846,11 +1846,16 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
     bool chas = issue(0, curb, cbm, cbj);
     for (int k = 0;; ++k) {
         if (!__any_sync(0xffffffffu, chas)) break;
-        const bool nhas = issue((k + 1) & 1, nxtb, nbm, nbj);
-        asm volatile("cp.async.wait_group 1;" ::: "memory");  // batch k's copies have landed
+        bool nhas = false;
+        if constexpr (NBUF == 2) {  // batch k+1's copies fly while batch k is multiplied
+            nhas = issue((k + 1) & 1, nxtb, nbm, nbj);
+            asm volatile("cp.async.wait_group 1;" ::: "memory");  // batch k's copies have landed
+        } else {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
         __syncwarp();
         const uint32_t mC = curb.valid ? bitmap_multiply(curb.ma, cbm) : 0u;
-        const T* bb = buf + (k & 1) * (GROUP_BUF / 2);
+        const T* bb = buf + (NBUF == 2 ? (k & 1) : 0) * (GROUP_BUF / NBUF);
 #pragma unroll
         for (int v = 0; v < 4; ++v) {
             const int src = (lane & ~3) + v;
@@ -1891,6 +1896,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
             }
         }
         __syncwarp();  // buffer k&1 is refilled by the next issue
+        if constexpr (NBUF == 1) nhas = issue(0, nxtb, nbm, nbj);
         curb = nxtb;
         cbm = nbm;
         cbj = nbj;
@@ -2119,16 +2125,13 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     static const int staged_env = [] { const char* e = getenv("AMGT_NUM_STAGED"); return e ? atoi(e) : 1; }();
     const bool tc_route = (sizeof(T) == 8 || sizeof(T) == 2) && g_tc_thr_spgemm <= 16;
     if (!tc_route && staged_env) {
-        constexpr size_t sm = (size_t)STAGED_WARPS * 8 * 2 * 4 * 2 * 16 * sizeof(T);
+        static const int nbuf_env = [] { const char* e = getenv("AMGT_STAGED_NBUF"); return e ? atoi(e) : 2; }();
+        const int nbuf = nbuf_env == 1 ? 1 : 2;
+        const size_t sm = (size_t)STAGED_WARPS * 8 * nbuf * 4 * 2 * 16 * sizeof(T);
         const bool nc4 = C->row_max > 0 && C->row_max <= 4;
-        auto kern = nc4 ? k_numeric_staged<T, Acc, 4> : k_numeric_staged<T, Acc, GROUP_NC>;
-        static bool attr = false;
-        if (!attr && sm > 48 * 1024) {
-            AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-            AMGT_CUDA(cudaFuncSetAttribute(k_numeric_staged<T, Acc, GROUP_NC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                           (int)sm));
-        }
-        attr = true;
+        auto kern = nc4 ? (nbuf == 2 ? k_numeric_staged<T, Acc, 4, 2> : k_numeric_staged<T, Acc, 4, 1>)
+                        : (nbuf == 2 ? k_numeric_staged<T, Acc, GROUP_NC, 2> : k_numeric_staged<T, Acc, GROUP_NC, 1>);
+        if (sm > 48 * 1024) AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
         // rows per group: several when rows are short (mean pairs per row ~ (T_A/BR_A)(T_B/BR_B)),
         // one when a row alone keeps the batch pipeline busy (and the grid large)
         const double mp = (BR ? (double)A->blc_num / BR : 0.0) * (B->blc_row ? (double)B->blc_num / B->blc_row : 0.0);
