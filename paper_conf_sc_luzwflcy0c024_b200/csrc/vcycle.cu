@@ -43,6 +43,8 @@ struct amgt_level {
     amgt_prec vprec = AMGT_FP64;
     void *b = nullptr, *x = nullptr, *r = nullptr, *t = nullptr, *dinv = nullptr;  // t: ping-pong partner of x
     void* u = nullptr;        // level 1 with the fused sweeps: third iterate buffer
+    void* vblock = nullptr;   // the allocation holding b, x, r, t, dinv
+    size_t vblock_bytes = 0;
 };
 
 struct amgt_hierarchy {
@@ -310,10 +312,11 @@ static bool dense_inverse(int64_t n, std::vector<double>& a, std::vector<double>
 
 static void free_level_vectors(amgt_level& L, Alloc& a) {
     const size_t vb = vbytes(L.vprec) * (size_t)L.npad;
-    for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv, &L.u}) {
-        a.put(*p, vb);
-        *p = nullptr;
-    }
+    a.put(L.vblock, L.vblock_bytes);  // b, x, r, t, dinv
+    L.vblock = nullptr;
+    L.b = L.x = L.r = L.t = L.dinv = nullptr;
+    a.put(L.u, vb);
+    L.u = nullptr;
 }
 
 static void destroy(amgt_hierarchy* H) {
@@ -379,10 +382,18 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
         AMGT_TRY(spmv_analyze_impl(&L.A, a));
         trace_point("analyze A", s);
         const size_t vb = vbytes(L.vprec) * (size_t)L.npad;
-        for (void** p : {&L.b, &L.x, &L.r, &L.t, &L.dinv}) {
-            *p = a.get(vb);
-            if (!*p) return fail(AMGT_ERR_ALLOC, "hierarchy vector allocation failed");
-            AMGT_CUDA(cudaMemsetAsync(*p, 0, vb, s));
+        {  // the five level vectors in one allocation (one allocator call, one memset)
+            const size_t va = (vb + 255) & ~size_t(255);
+            L.vblock = a.get(5 * va);
+            if (!L.vblock) return fail(AMGT_ERR_ALLOC, "hierarchy vector allocation failed");
+            L.vblock_bytes = 5 * va;
+            AMGT_CUDA(cudaMemsetAsync(L.vblock, 0, 5 * va, s));
+            char* base = (char*)L.vblock;
+            L.b = base;
+            L.x = base + va;
+            L.r = base + 2 * va;
+            L.t = base + 3 * va;
+            L.dinv = base + 4 * va;
         }
         AMGT_TRY(build_dinv(L, s, H->o.smoother == AMGT_SMOOTH_L1_JACOBI));
         trace_point("vectors+dinv", s);
