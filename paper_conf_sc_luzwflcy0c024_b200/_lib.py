@@ -175,11 +175,19 @@ def _stream(stream=None) -> int:
 _live: dict[int, int] = {}
 
 
+_ext_streams: dict[int, "torch.cuda.ExternalStream"] = {}  # stream handle -> wrapper (built once)
+
+
 @_ALLOC_FN
 def _torch_alloc(nbytes, stream, ctx):
     try:
-        p = torch.cuda.caching_allocator_alloc(int(nbytes), torch.cuda.current_device(),
-                                               torch.cuda.ExternalStream(stream) if stream else None)
+        st = None
+        if stream:
+            st = _ext_streams.get(stream)
+            if st is None:
+                st = _ext_streams[stream] = torch.cuda.ExternalStream(stream)
+        p = torch.cuda.caching_allocator_alloc(int(nbytes), st.device_index if st is not None else
+                                               torch.cuda.current_device(), st)
         _live[p] = int(nbytes)
         return p
     except Exception:  # allocation failure is reported by the library as AMGT_ERR_ALLOC
