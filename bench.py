@@ -253,8 +253,11 @@ def run_dist(args, rank, world, local):
     import paper_conf_sc_luzwflcy0c024_b200 as amgt
     from paper_conf_sc_luzwflcy0c024_b200.dist import Comm, DistHierarchy
 
-    if os.environ.get("NCCL_DEBUG", "VERSION").upper() == "VERSION":  # keep stdout to the one JSON line
-        os.environ["NCCL_DEBUG"] = "WARN"
+    # stdout carries the one JSON line: library banners printed from C (the NCCL version line)
+    # go to stderr while the run is set up and measured
+    sys.stdout.flush()
+    json_fd = os.dup(1)
+    os.dup2(2, 1)
     dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     comm = Comm()
     cfg = gen.configs.CONFIGS["cfg2"]
@@ -318,27 +321,41 @@ def run_dist(args, rank, world, local):
     h2d = sum(t.numel() * t.element_size() for M in [hA, *hPs] for t in (M.row_ptr, M.col, M.val)) + hb.numel() * 8
     d2h = hx.numel() * 8 + (args.cycles + 1) * 8
 
-    def dev(t):
-        d = torch.empty(t.shape, dtype=t.dtype, device="cuda")
-        d.copy_(t, non_blocking=True)
-        return d
+    # as the single-GPU leg: uploads on a copy stream into two buffer sets, step i+1's upload
+    # enqueued once step i's hierarchy exists (it overlaps step i's V-cycles)
+    host_in = [hA.row_ptr, hA.col, hA.val] + [t for P in hPs for t in (P.row_ptr, P.col, P.val)] + [hb]
+    dev_in = [[torch.empty(t.shape, dtype=t.dtype, device="cuda") for t in host_in] for _ in range(2)]
+    cs = torch.cuda.Stream()
+    ev_in = [torch.cuda.Event(), torch.cuda.Event()]
 
-    def e2e_step():
-        dA = CSR(hA.m, hA.n, dev(hA.row_ptr), dev(hA.col), dev(hA.val))
-        dPs = [CSR(P.m, P.n, dev(P.row_ptr), dev(P.col), dev(P.val)) for P in hPs]
-        db = dev(hb)
+    def upload(k):
+        with torch.cuda.stream(cs):
+            for d, h in zip(dev_in[k], host_in):
+                d.copy_(h, non_blocking=True)
+            ev_in[k].record(cs)
+
+    def e2e_step(k, nxt):
+        stream.wait_event(ev_in[k])
+        d = dev_in[k]
+        dA = CSR(hA.m, hA.n, d[0], d[1], d[2])
+        dPs = [CSR(P.m, P.n, d[3 + 3 * i], d[4 + 3 * i], d[5 + 3 * i]) for i, P in enumerate(hPs)]
         H_ = DistHierarchy(comm, dA, rows, n, dPs, level_prec=LEVEL_PREC[:nlev])
+        if nxt is not None:
+            upload(nxt)
         x.zero_()
-        H_.native_vcycle(native, db, x, args.cycles)
+        H_.native_vcycle(native, d[-1], x, args.cycles)
         hx.copy_(x, non_blocking=True)
 
-    e2e_step()
+    upload(0)
+    e2e_step(0, None)
     dist.barrier()
     torch.cuda.synchronize()
     f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     f0.record(stream)
-    for _ in range(args.steps):
-        e2e_step()
+    cs.wait_event(f0)
+    upload(0)
+    for i in range(args.steps):
+        e2e_step(i % 2, (i + 1) % 2 if i + 1 < args.steps else None)
     f1.record(stream)
     dist.barrier()
     torch.cuda.synchronize()
@@ -349,6 +366,9 @@ def run_dist(args, rank, world, local):
     sp_bytes = l0["T"] * (16 * 8 + 6) + (l0["BR"] + 1) * 8 + 8 * 4 * l0["BC"] + 8 * 4 * l0["BR"]
     peak, peak_kind = _peaks()
     achieved = sp_bytes / (spmv_ms * 1e-3) / 1e9
+    sys.stdout.flush()
+    os.dup2(json_fd, 1)
+    os.close(json_fd)
     if rank == 0:
         print(json.dumps({
             "metric": METRIC, "value": round(bytes_rank * world / (ms_step * 1e-3) / 1e9, 2), "unit": "GB/s",
@@ -366,7 +386,8 @@ def run_dist(args, rank, world, local):
             "components": {"final_rel_residual": res[-1] / res[0], "bytes_per_rank_step": bytes_rank},
             "e2e": {"value": round(bytes_rank * world / (e2e_ms * 1e-3) / 1e9, 2), "unit": "GB/s",
                     "ms_per_step": round(e2e_ms, 3), "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
-                    "copies": "each rank uploads its slab inputs from pinned host memory every step and reads x back"},
+                    "copies": "each rank uploads its slab inputs from pinned host memory every step (copy stream, "
+                              "double-buffered, overlapping the previous step's V-cycles) and reads x back"},
             "gpu_launches": launches, "clocks": clk.summary(),
         }), flush=True)
     dist.destroy_process_group()
