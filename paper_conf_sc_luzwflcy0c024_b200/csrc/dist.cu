@@ -254,6 +254,9 @@ amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* Ls, 
         if (!Ls[k].A || !Ls[k].xe[0] || !Ls[k].xe[1] || !Ls[k].r || (k + 1 < nlev && (!Ls[k].P || !Ls[k].R)))
             return fail(AMGT_ERR_ARG, "amgt_dist_vcycle: incomplete level %d", k);
     cudaStream_t s = (cudaStream_t)stream;
+    // SpMV kernels with programmatic dependent launch, as in amgt_vcycle: a launch that follows
+    // an event wait (the halo) or a non-PDL kernel gets an ordinary full dependency
+    PdlScope pdl;
     Ctx c{D, s, omega};
     const int M = nlev - 1;
     constexpr int JAC = 1, RES = 2, ACC = 3;
