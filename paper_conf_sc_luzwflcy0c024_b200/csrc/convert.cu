@@ -323,23 +323,32 @@ __global__ void k_tr_sort(int64_t BRo, const int64_t* __restrict__ optr, int32_t
     }
 }
 
+// Output tile d = (input tile perm[d])^T.  One 4-lane group per tile: lane q gathers column q
+// of the input tile (its four rows' q-th entries: each load instruction of the group reads
+// the 32-B row r) and writes it as row q of the output tile (the group's stores cover the
+// output tile contiguously); the bitmap is transposed by lane 0.
 template <typename T>
 __global__ void k_tr_gather(int64_t T_, const int64_t* __restrict__ perm, const uint16_t* __restrict__ bmap,
                             const T* __restrict__ bval, uint16_t* __restrict__ omap, T* __restrict__ oval) {
-    for (int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; d < T_; d += (int64_t)gridDim.x * blockDim.x) {
+    const int q = threadIdx.x & 3;
+    for (int64_t d = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2; d < T_;
+         d += ((int64_t)gridDim.x * blockDim.x) >> 2) {
         const int64_t s = perm[d];
-        const uint32_t mp = bmap[s];
-        uint32_t tm = 0;
+        T v[4];
 #pragma unroll
-        for (int r = 0; r < 4; ++r)
+        for (int r = 0; r < 4; ++r) v[r] = bval[16 * s + 4 * r + q];
 #pragma unroll
-            for (int c = 0; c < 4; ++c)
-                if (mp & (1u << (4 * r + c))) tm |= 1u << (4 * c + r);
-        omap[d] = (uint16_t)tm;
+        for (int r = 0; r < 4; ++r) oval[16 * d + 4 * q + r] = v[r];
+        if (q == 0) {
+            const uint32_t mp = bmap[s];
+            uint32_t tm = 0;
 #pragma unroll
-        for (int r = 0; r < 4; ++r)
+            for (int r = 0; r < 4; ++r)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) oval[16 * d + 4 * c + r] = bval[16 * s + 4 * r + c];
+                for (int c = 0; c < 4; ++c)
+                    if (mp & (1u << (4 * r + c))) tm |= 1u << (4 * c + r);
+            omap[d] = (uint16_t)tm;
+        }
     }
 }
 
@@ -597,7 +606,7 @@ amgt_status cast_impl(const amgt_mbsr* in, amgt_prec to, amgt_mbsr* out, Alloc& 
 
 template <typename T>
 static void launch_tr_gather(const amgt_mbsr* in, const int64_t* perm, amgt_mbsr* o, cudaStream_t s) {
-    k_tr_gather<T><<<grid_for(in->blc_num, 256), 256, 0, s>>>(in->blc_num, perm, in->blc_map, (const T*)in->blc_val,
+    k_tr_gather<T><<<grid_for(4 * in->blc_num, 256), 256, 0, s>>>(in->blc_num, perm, in->blc_map, (const T*)in->blc_val,
                                                              o->blc_map, (T*)o->blc_val);
 }
 
