@@ -297,11 +297,16 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
 // steps: latency-bound dependent chains.)
 constexpr int SF_ROWS = 16;  // block rows per warp in k_sym_flat
 constexpr int SF_U = 4;      // A tiles per lane per round (all their loads in flight together)
+// sidx/smap (step 1, optional): the finished sorted list of every category-8 row is also
+// written to its slot [32 I, 32 I + n) of these scratch arrays, and k_sym_copy moves it into C
+// once the row offsets exist — step 2's re-expansion of the pairs is then skipped.
 template <int STEP>
 __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t* __restrict__ nnz_row,
                                                   const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx,
                                                   uint16_t* __restrict__ cmap, int64_t* __restrict__ bin_of,
-                                                  unsigned long long* __restrict__ stats) {
+                                                  unsigned long long* __restrict__ stats,
+                                                  int32_t* __restrict__ sidx = nullptr,
+                                                  uint16_t* __restrict__ smap = nullptr) {
     // row stride padded by one word: the 8 groups of a warp read the same position of 8
     // different rows at once (an unpadded 128-B stride puts them all in one bank)
     __shared__ int keys[8][SF_ROWS][SMALL_CUB + 1];
@@ -416,10 +421,11 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
         cnt += __shfl_xor_sync(gm, cnt, 2, 4);
         if (STEP == 1) {
             if (r == 0) nnz_row[I] = cnt;
-            continue;
+            if (!sidx) continue;
         }
         __syncwarp(gm);
-        const int64_t out = cptr[I];
+        int32_t* oi = STEP == 1 ? sidx + SMALL_CUB * I : cidx + cptr[I];
+        uint16_t* om = STEP == 1 ? smap + SMALL_CUB * I : cmap + cptr[I];
         for (int i = r; i < n; i += 4) {
             if (!F[i]) continue;
             const int k = Kr[i];
@@ -430,8 +436,27 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
                 rank += (F[j] && kj < k);
                 m |= (kj == k) ? Mr[j] : 0u;
             }
-            cidx[out + rank] = k;
-            cmap[out + rank] = (uint16_t)m;
+            oi[rank] = k;
+            om[rank] = (uint16_t)m;
+        }
+    }
+}
+
+// Step 2 of the category-8 rows when step 1 kept their sorted lists: copy slot [32 I, +n) to
+// C at cptr[I] (4-lane group per row).
+__global__ void __launch_bounds__(256) k_sym_copy(int64_t BR, const int64_t* __restrict__ bin_of,
+                                                  const int64_t* __restrict__ cptr, const int32_t* __restrict__ sidx,
+                                                  const uint16_t* __restrict__ smap, int32_t* __restrict__ cidx,
+                                                  uint16_t* __restrict__ cmap) {
+    const int r = threadIdx.x & 3;
+    for (int64_t I = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2; I < BR;
+         I += ((int64_t)gridDim.x * blockDim.x) >> 2) {
+        if (bin_of[I] != NBINS) continue;  // group-uniform
+        const int64_t c0 = cptr[I];
+        const int n = (int)(cptr[I + 1] - c0);
+        for (int i = r; i < n; i += 4) {
+            cidx[c0 + i] = sidx[SMALL_CUB * I + i];
+            cmap[c0 + i] = smap[SMALL_CUB * I + i];
         }
     }
 }
@@ -2020,9 +2045,18 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
         // step 1 over every block row: Cub + bins (L149-151) and, for the category-8 rows
         // (Cub <= 32), the distinct tile columns (Alg. 3 lines 1-13)
+        // keep the category-8 rows' sorted lists from step 1 (32 slots per row) when the scratch
+        // stays moderate; step 2 is then a copy
+        Scratch<int32_t> sidx;
+        Scratch<uint16_t> smap;
+        const bool keep = BR > 0 && (double)BR * SMALL_CUB * 6.0 <= 2e9;
+        if (keep) {
+            AMGT_TRY(sidx.init(a, (size_t)BR * SMALL_CUB));
+            AMGT_TRY(smap.init(a, (size_t)BR * SMALL_CUB));
+        }
         if (BR > 0) {
             k_sym_flat<1><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nnz_row.p, nullptr, nullptr, nullptr,
-                                                                     bin_of.p, stats);
+                                                                     bin_of.p, stats, sidx.p, smap.p);
             AMGT_LAUNCHED();
             if (info && A->blc_num > 0) {
                 k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats, g_tc_thr_spgemm);
@@ -2073,8 +2107,12 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         C.row_max = (int64_t)hmax;
         if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
         if (BR > 0) {  // step 2 (Alg. 3 lines 13-14 + bitmap OR, R15)
-            k_sym_flat<2><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nullptr, C.blc_ptr, C.blc_idx, C.blc_map,
-                                                                     bin_of.p, nullptr);
+            if (keep)
+                k_sym_copy<<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, bin_of.p, C.blc_ptr, sidx.p, smap.p,
+                                                                       C.blc_idx, C.blc_map);
+            else
+                k_sym_flat<2><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nullptr, C.blc_ptr, C.blc_idx,
+                                                                         C.blc_map, bin_of.p, nullptr);
             AMGT_LAUNCHED();
             if (big > 0) {
                 st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
