@@ -277,6 +277,52 @@ __global__ void __launch_bounds__(256) k_spmv_lanerow(int64_t I0, int64_t BR, co
     }
 }
 
+// FP64 operators with ~1 tile per block row (the level-1 interpolation P): two lanes per block
+// row, lane h owning tile rows 2h and 2h+1 (64 contiguous bytes: four 16-B loads).  The
+// lane-per-row kernel's loads touch 32 lines per warp instruction (8 instructions per tile:
+// L1-wavefront bound, ncu 82% L1/TEX); here each tile line is touched by 4 instructions.  Same
+// per-row accumulation order as k_spmv_lanerow (tiles in order, columns in order).
+template <typename XT, typename YT, int MODE>
+__global__ void __launch_bounds__(256) k_spmv_lanepair(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
+                                                       const int32_t* __restrict__ bidx,
+                                                       const uint16_t* __restrict__ bmap,
+                                                       const double* __restrict__ bval, const XT* __restrict__ x,
+                                                       const Epi<XT, YT, MODE> epi) {
+    pdl_wait();
+    const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t I = I0 + (gt >> 1);
+    const int h = (int)(gt & 1);
+    if (I >= BR) return;  // both lanes of the pair
+    const int64_t t0 = __ldg(bptr + I), t1 = __ldg(bptr + I + 1);
+    typename Epi<XT, YT, MODE>::Pre pre[2];
+#pragma unroll
+    for (int rr = 0; rr < 2; ++rr) pre[rr] = epi.prefetch(4 * I + 2 * h + rr);
+    double acc[2] = {0.0, 0.0};
+    for (int64_t t = t0; t < t1; ++t) {
+        const int32_t J = __ldg(bidx + t);
+        const uint32_t mp = __ldg(bmap + t);
+        double v[8];
+        const double2* tp = reinterpret_cast<const double2*>(bval + 16 * t + 8 * h);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const double2 d = __ldg(tp + k);
+            v[2 * k] = d.x;
+            v[2 * k + 1] = d.y;
+        }
+        const double2 xa = x_pair(x, J, 0), xb = x_pair(x, J, 1);
+        const double xv[4] = {xa.x, xa.y, xb.x, xb.y};
+#pragma unroll
+        for (int rr = 0; rr < 2; ++rr) {
+            const int r = 2 * h + rr;
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                acc[rr] = ((mp >> (4 * r + c)) & 1u) ? fma(v[4 * rr + c], xv[c], acc[rr]) : acc[rr];
+        }
+    }
+#pragma unroll
+    for (int rr = 0; rr < 2; ++rr) epi.finish(4 * I + 2 * h + rr, acc[rr], pre[rr]);
+}
+
 // ---------------------------------------------------------------- chunk kernel (long rows)
 template <typename MatT, typename XT>
 __global__ void __launch_bounds__(256) k_spmv_chunks(int64_t nchunks, const int64_t* __restrict__ bptr,
@@ -537,6 +583,16 @@ static int spmv_variant() {
     return v;
 }
 
+// AMGT_LANEPAIR=0: FP64 ~1-tile-per-row matrices take the lane-per-row kernel (measurement knob)
+static bool lanepair_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_LANEPAIR");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 // AMGT_LANEROW=0: ~1-tile-per-row matrices take the group kernel too (measurement knob)
 static bool lanerow_enabled() {
     static int v = -1;
@@ -567,6 +623,13 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
         auto ok = [&](const void* p) { return (reinterpret_cast<uintptr_t>(p) & al) == 0; };
         const bool vec = ok(y) && ok(ea.b) && ok(ea.dinv) && ok(ea.r) &&
                          (reinterpret_cast<uintptr_t>(ea.xs) & (4 * sizeof(XT) - 1)) == 0;
+        if constexpr (sizeof(MatT) == 8) {
+            if (lanepair_enabled()) {
+                pdl_launch(k_spmv_lanepair<XT, YT, MODE>, dim3((unsigned)ceil_div(2 * (BR - I0), 256)), dim3(256), 0, s,
+                           I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const double*)A->blc_val, (const XT*)x, epi);
+                return;
+            }
+        }
         pdl_launch(k_spmv_lanerow<MatT, XT, YT, MODE>, dim3((unsigned)ceil_div(BR - I0, 256)), dim3(256), 0, s, I0, BR,
                    A->blc_ptr, A->blc_idx, A->blc_map, (const MatT*)A->blc_val, (const XT*)x, epi, vec);
         return;
