@@ -277,34 +277,37 @@ __global__ void __launch_bounds__(256) k_spmv_lanerow(int64_t I0, int64_t BR, co
     }
 }
 
-// FP64 operators with ~1 tile per block row (the level-1 interpolation P): two lanes per block
-// row, lane h owning tile rows 2h and 2h+1 (64 contiguous bytes: four 16-B loads).  The
-// lane-per-row kernel's loads touch 32 lines per warp instruction (8 instructions per tile:
-// L1-wavefront bound, ncu 82% L1/TEX); here each tile line is touched by 4 instructions.  Same
+// FP64 operators with ~1 tile per block row (the level-1 interpolation P): LPR lanes per block
+// row (2 by default), lane h owning tile rows [h 4/LPR, (h+1) 4/LPR) (contiguous 16-B loads).
+// The lane-per-row kernel's loads touch 32 lines per warp instruction (8 instructions per
+// tile: L1-wavefront bound, ncu 82% L1/TEX); with 2 lanes each tile line is touched by 4.  Same
 // per-row accumulation order as k_spmv_lanerow (tiles in order, columns in order).
-template <typename XT, typename YT, int MODE>
+template <typename XT, typename YT, int MODE, int LPR>
 __global__ void __launch_bounds__(256) k_spmv_lanepair(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
                                                        const int32_t* __restrict__ bidx,
                                                        const uint16_t* __restrict__ bmap,
                                                        const double* __restrict__ bval, const XT* __restrict__ x,
                                                        const Epi<XT, YT, MODE> epi) {
+    constexpr int RPL = 4 / LPR;  // tile rows per lane
     pdl_wait();
     const int64_t gt = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t I = I0 + (gt >> 1);
-    const int h = (int)(gt & 1);
-    if (I >= BR) return;  // both lanes of the pair
+    const int64_t I = I0 + gt / LPR;
+    const int h = (int)(gt % LPR);
+    if (I >= BR) return;  // all lanes of the row
     const int64_t t0 = __ldg(bptr + I), t1 = __ldg(bptr + I + 1);
-    typename Epi<XT, YT, MODE>::Pre pre[2];
+    typename Epi<XT, YT, MODE>::Pre pre[RPL];
 #pragma unroll
-    for (int rr = 0; rr < 2; ++rr) pre[rr] = epi.prefetch(4 * I + 2 * h + rr);
-    double acc[2] = {0.0, 0.0};
+    for (int rr = 0; rr < RPL; ++rr) pre[rr] = epi.prefetch(4 * I + RPL * h + rr);
+    double acc[RPL];
+#pragma unroll
+    for (int rr = 0; rr < RPL; ++rr) acc[rr] = 0.0;
     for (int64_t t = t0; t < t1; ++t) {
         const int32_t J = __ldg(bidx + t);
         const uint32_t mp = __ldg(bmap + t);
-        double v[8];
-        const double2* tp = reinterpret_cast<const double2*>(bval + 16 * t + 8 * h);
+        double v[4 * RPL];
+        const double2* tp = reinterpret_cast<const double2*>(bval + 16 * t + 4 * RPL * h);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
+        for (int k = 0; k < 2 * RPL; ++k) {
             const double2 d = __ldg(tp + k);
             v[2 * k] = d.x;
             v[2 * k + 1] = d.y;
@@ -312,15 +315,15 @@ __global__ void __launch_bounds__(256) k_spmv_lanepair(int64_t I0, int64_t BR, c
         const double2 xa = x_pair(x, J, 0), xb = x_pair(x, J, 1);
         const double xv[4] = {xa.x, xa.y, xb.x, xb.y};
 #pragma unroll
-        for (int rr = 0; rr < 2; ++rr) {
-            const int r = 2 * h + rr;
+        for (int rr = 0; rr < RPL; ++rr) {
+            const int r = RPL * h + rr;
 #pragma unroll
             for (int c = 0; c < 4; ++c)
                 acc[rr] = ((mp >> (4 * r + c)) & 1u) ? fma(v[4 * rr + c], xv[c], acc[rr]) : acc[rr];
         }
     }
 #pragma unroll
-    for (int rr = 0; rr < 2; ++rr) epi.finish(4 * I + 2 * h + rr, acc[rr], pre[rr]);
+    for (int rr = 0; rr < RPL; ++rr) epi.finish(4 * I + RPL * h + rr, acc[rr], pre[rr]);
 }
 
 // ---------------------------------------------------------------- chunk kernel (long rows)
@@ -583,14 +586,15 @@ static int spmv_variant() {
     return v;
 }
 
-// AMGT_LANEPAIR=0: FP64 ~1-tile-per-row matrices take the lane-per-row kernel (measurement knob)
-static bool lanepair_enabled() {
+// lanes per block row of k_spmv_lanepair for FP64 ~1-tile-per-row operators (AMGT_LANEPAIR:
+// 2 default, 4, or 0 = the lane-per-row kernel; measurement knob)
+static int lanepair_lanes() {
     static int v = -1;
     if (v < 0) {
         const char* e = getenv("AMGT_LANEPAIR");
-        v = (e && e[0] == '0') ? 0 : 1;
+        v = e ? atoi(e) : 2;
     }
-    return v == 1;
+    return v;
 }
 
 // AMGT_LANEROW=0: ~1-tile-per-row matrices take the group kernel too (measurement knob)
@@ -624,9 +628,11 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
         const bool vec = ok(y) && ok(ea.b) && ok(ea.dinv) && ok(ea.r) &&
                          (reinterpret_cast<uintptr_t>(ea.xs) & (4 * sizeof(XT) - 1)) == 0;
         if constexpr (sizeof(MatT) == 8) {
-            if (lanepair_enabled()) {
-                pdl_launch(k_spmv_lanepair<XT, YT, MODE>, dim3((unsigned)ceil_div(2 * (BR - I0), 256)), dim3(256), 0, s,
-                           I0, BR, A->blc_ptr, A->blc_idx, A->blc_map, (const double*)A->blc_val, (const XT*)x, epi);
+            const int lpr = lanepair_lanes();
+            if (lpr == 2 || lpr == 4) {
+                auto kern = lpr == 2 ? k_spmv_lanepair<XT, YT, MODE, 2> : k_spmv_lanepair<XT, YT, MODE, 4>;
+                pdl_launch(kern, dim3((unsigned)ceil_div(lpr * (BR - I0), 256)), dim3(256), 0, s, I0, BR, A->blc_ptr,
+                           A->blc_idx, A->blc_map, (const double*)A->blc_val, (const XT*)x, epi);
                 return;
             }
         }
