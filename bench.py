@@ -17,6 +17,7 @@ the same workload (setup + a few cycles) in the same unit.
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import os
 import statistics
@@ -290,6 +291,8 @@ def run_dist(args, rank, world, local):
     torch.cuda.synchronize()
     launches0 = amgt.launch_count()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gc.collect()
+    gc.disable()  # no collector pause inside the timed region (host stalls starve the GPU queue)
     with ClockSampler(local) as clk:
         e0.record(stream)
         for _ in range(args.steps):
@@ -297,6 +300,7 @@ def run_dist(args, rank, world, local):
         e1.record(stream)
         dist.barrier()
         torch.cuda.synchronize()
+    gc.enable()
     ms = torch.tensor([e0.elapsed_time(e1) / args.steps], dtype=torch.float64, device="cuda")
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms_step = float(ms.item())
@@ -449,6 +453,8 @@ def run_gpu(args):
     amgt.timing_sample(L1_SAMPLE)  # on one launch in L1_SAMPLE (an event pair breaks the PDL overlap)
     launches0 = amgt.launch_count()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gc.collect()
+    gc.disable()  # no collector pause inside the timed region (host stalls starve the GPU queue)
     with ClockSampler(local) as clk:
         barrier()
         ev0.record(stream)
@@ -456,6 +462,7 @@ def run_gpu(args):
             gpu_step(amgt, A, Ps, b, x, args.cycles, torch)
         ev1.record(stream)
         barrier()
+    gc.enable()
     launches = amgt.launch_count() - launches0
     live = amgt.timing_read()
     amgt.timing_enable(False)

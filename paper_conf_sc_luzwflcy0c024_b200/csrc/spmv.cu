@@ -205,8 +205,9 @@ __device__ __forceinline__ void spmv_rows_octet(int64_t wid, int64_t I0, int64_t
 }
 
 // Row kernel: warps take row octets in a grid-stride loop (one octet per warp when the grid
-// covers the rows, AMGT_SPMV_PERSIST=0; by default a grid of exactly the resident CTAs, so
-// no partial last wave: 386.8 vs 399.8 us per config-2 V-cycle).
+// covers the rows, AMGT_SPMV_PERSIST=0; by default a grid of exactly the resident CTAs while
+// the launch is <= kPersistMaxWaves waves, so no partial last wave: 386.8 vs 399.8 us per
+// config-2 V-cycle; longer launches keep the full grid: config-3 A_1 2.42 vs 2.53 ms).
 template <typename MatT, typename XT, typename YT, int MODE, int U = 2, int MINB = 1, bool TC = false>
 __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
                                                    const int32_t* __restrict__ bidx,
@@ -589,6 +590,10 @@ amgt_status spmv_analyze_impl(amgt_mbsr* A, Alloc& a) {
 // threads — i.e. the register budget): 0 = U8/4 (default; measured best on B200, see
 // DESIGN.md §7), 1 = U4/5, 2 = U4/6, 3 = U2/6.
 // The environment variable AMGT_SPMV_VARIANT selects another for tuning.
+// AMGT_SPMV_PERSIST: 0 = one warp per row octet over a full grid, 1 = grid of exactly the
+// resident CTAs while the launch is at most kPersistMaxWaves waves (default), 2 = always.
+static constexpr unsigned kPersistMaxWaves = 32;
+
 static int spmv_variant() {
     static int v = -1;
     if (v < 0) {
@@ -662,7 +667,10 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
             int per_sm = 0;
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, 0);
             const unsigned cap = (unsigned)num_sms() * (unsigned)std::max(per_sm, 1);
-            g = std::min(g, cap);
+            // auto (1): only while the partial last wave is a visible share of the launch; over
+            // many waves a grid-stride loop lets the warps drift apart in the address space
+            // (config-3 A_1, ~110 octets per warp: 2.53 ms vs 2.37 ms for the full grid)
+            if (persist > 1 || g <= kPersistMaxWaves * cap) g = std::min(g, cap);
         }
         pdl_launch(kern, dim3(g), dim3(256), 0, s, I0, BR, A->blc_ptr, A->blc_idx, A->blc_map,
                    (const MatT*)A->blc_val, (const XT*)x, epi, long_thr, tc);
