@@ -53,6 +53,32 @@ class ClockSampler:
         self.lines = []
 
     def __enter__(self):
+        mode = os.environ.get("AMGT_BENCH_CLOCKS", "smi")  # smi | nvml (in-process) | off (testing only)
+        if mode == "off":
+            return self
+        if mode == "nvml":
+            try:
+                import pynvml
+                pynvml.nvmlInit()
+                h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+                mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+                bits = (pynvml.nvmlClocksEventReasonHwSlowdown, pynvml.nvmlClocksEventReasonHwThermalSlowdown,
+                        pynvml.nvmlClocksEventReasonSwThermalSlowdown, pynvml.nvmlClocksEventReasonSwPowerCap)
+                self.stop = threading.Event()
+
+                def poll():
+                    while not self.stop.is_set():
+                        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                        r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                        self.lines.append(", ".join([str(sm), str(mx)] +
+                                                    ["Active" if r & b else "Not Active" for b in bits]))
+                        self.stop.wait(0.1)
+
+                self.t = threading.Thread(target=poll, daemon=True)
+                self.t.start()
+            except Exception:
+                self.stop = None
+            return self
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
                                           "--format=csv,noheader,nounits", "-lms", "100"],
@@ -73,6 +99,9 @@ class ClockSampler:
             self.lines.append(line.strip())
 
     def __exit__(self, *a):
+        if getattr(self, "stop", None) is not None:
+            self.stop.set()
+            self.t.join(timeout=5)
         if self.proc:
             self.proc.terminate()
             try:
