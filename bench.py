@@ -324,12 +324,16 @@ def run_dist(args, rank, world, local):
     gc.disable()  # no collector pause inside the timed region (host stalls starve the GPU queue)
     with ClockSampler(local) as clk:
         e0.record(stream)
+        host_ms = []
         for _ in range(args.steps):
+            t_h = time.perf_counter()
             H, res, calls = step()
+            host_ms.append(round((time.perf_counter() - t_h) * 1e3, 2))
         e1.record(stream)
         dist.barrier()
         torch.cuda.synchronize()
     gc.enable()
+    print(f"[bench] host ms per timed step (enqueue + host syncs): {host_ms}", file=sys.stderr)
     ms = torch.tensor([e0.elapsed_time(e1) / args.steps], dtype=torch.float64, device="cuda")
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms_step = float(ms.item())
@@ -487,11 +491,15 @@ def run_gpu(args):
     with ClockSampler(local) as clk:
         barrier()
         ev0.record(stream)
+        host_ms = []
         for _ in range(args.steps):
+            t_h = time.perf_counter()
             gpu_step(amgt, A, Ps, b, x, args.cycles, torch)
+            host_ms.append(round((time.perf_counter() - t_h) * 1e3, 2))
         ev1.record(stream)
         barrier()
     gc.enable()
+    print(f"[bench] host ms per timed step (enqueue + host syncs): {host_ms}", file=sys.stderr)
     launches = amgt.launch_count() - launches0
     live = amgt.timing_read()
     amgt.timing_enable(False)
