@@ -333,59 +333,6 @@ amgt_status amgt_dense_matvec(int64_t n, int64_t npad, const double* Ainv, const
 /* *out_dev = sum r_i^2 (deterministic two-pass reduction, FP64). */
 amgt_status amgt_norm2sq(int64_t n, const double* r, double* out_dev, void* stream);
 
-/* ------------------------------------------- native distributed V-cycle (§8(e)) */
-
-/* Communicator for the row-slab path: NCCL, loaded at run time (libnccl.so.2). */
-typedef struct amgt_dist amgt_dist;
-amgt_status amgt_dist_unique_id(void* id128_host);               /* on one rank; broadcast the 128 bytes */
-amgt_status amgt_dist_create(const void* id128_host, int rank, int size, amgt_dist** D);
-amgt_status amgt_dist_destroy(amgt_dist* D);
-amgt_status amgt_dist_allreduce_sum(amgt_dist* D, double* buf, int64_t count, void* stream);
-
-/* One level of a rank's distributed hierarchy (built by the host-side setup).
- *   A: own rows, columns in the extended range [eb, ee) (eb 4-aligned) ; P, R: rank-local.
- *   xe[2]: extended vectors (ping-pong), own rows at element offset `off`; b, r, dinv: own.
- *   Halo plan: send own elements [send_off, +send_cnt) of xe to send_peer; receive halo
- *   elements into [recv_off, +recv_cnt) from recv_peer (offsets in elements of xe; host
- *   arrays).  Block rows [int0, int1) touch no halo (computed while the halo is in flight). */
-typedef struct {
-    const amgt_mbsr* A;
-    const amgt_mbsr* P;
-    const amgt_mbsr* R;
-    int64_t m, off, int0, int1;
-    void* xe[2];
-    void* b;
-    void* r;
-    void* dinv;
-    amgt_prec vprec;
-    int nsend, nrecv;
-    const int32_t* send_peer;
-    const int64_t* send_off;
-    const int64_t* send_cnt;
-    const int32_t* recv_peer;
-    const int64_t* recv_off;
-    const int64_t* recv_cnt;
-} amgt_dist_level;
-
-/* Coarsest level: n global rows, dense FP64 inverse (device), per-rank counts/displacements of
- * its rows (host arrays of `size` entries), device buffers bfull/xfull of n elements. */
-typedef struct {
-    int64_t n;
-    const double* Ainv;
-    const int64_t* counts;
-    const int64_t* displs;
-    void* bfull;
-    void* xfull;
-} amgt_dist_coarse;
-
-/* Alg. 2 (L68-82) on a row-slab hierarchy: every A_k SpMV exchanges its halo (ncclSend/Recv on
- * a side stream, overlapped with the interior block rows); residual norms are all-reduced; the
- * coarsest right-hand side is all-gathered and solved redundantly.  b, x: own rows of level 1
- * (FP64).  res_norms_host[ncycles+1] (global), spmv_calls_host (this rank).  Syncs at the end. */
-amgt_status amgt_dist_vcycle(amgt_dist* D, int nlev, const amgt_dist_level* levels, const amgt_dist_coarse* coarse,
-                             double omega, int nu1, int nu2, const double* b, double* x, int ncycles,
-                             double* res_norms_host, int64_t* spmv_calls_host, void* stream);
-
 /* ------------------------------------------------------ hierarchy + V-cycle (§II) */
 
 typedef struct {
@@ -453,6 +400,119 @@ amgt_status amgt_pcg(amgt_hierarchy* H, const double* b, double* x, int maxit, d
                      int* iters_host, int64_t* spmv_calls_host, void* stream);
 
 amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H);
+
+/* ------------------------------------------------------ distributed path (§8(e)) */
+/*
+ * Row partition (the paper's 8-GPU runs, L363-365): rank r owns a contiguous range
+ * of rows of every distributed matrix, ranks in ascending order; every range except the last
+ * covers whole 4-row block rows (rows % 4 == 0).  A rank's matrices hold ITS rows with GLOBAL
+ * column indices (m = own rows, n = global columns); its vectors hold its own rows, padded to
+ * 4*ceil(m/4) elements.  The library derives the rest: the contiguous block-row range a rank's
+ * columns touch (its halo), which pieces other ranks own, which of its own rows they need — from
+ * one host all-gather of (rows, min tile column, max tile column) per rank.
+ * All calls below except amgt_dist_plan_host are COLLECTIVE: every rank calls them in the same
+ * order.  Transfers are stream-ordered on the call's stream (halo exchanges on an internal
+ * communication stream, joined with events).
+ */
+typedef struct amgt_dist amgt_dist;
+
+/* NCCL transport (one process per GPU).  amgt_nccl_unique_id on one rank, broadcast the 128
+ * bytes, then amgt_dist_create on every rank with its level-1 row range [row_begin, row_end).
+ * libnccl.so.2 is loaded at run time (AMGT_ERR_NCCL if absent). */
+amgt_status amgt_nccl_unique_id(void* id128_host);
+amgt_status amgt_dist_create(const void* id128_host, int rank, int size, int64_t row_begin, int64_t row_end,
+                             amgt_dist** D);
+
+/* Loopback transport: `size` (<= 16) virtual ranks in ONE process on ONE GPU, each driven by its
+ * own host thread with its own stream.  Point-to-point messages are device-to-device copies
+ * ordered by CUDA events; all-reduce sums the ranks' buffers in rank order (deterministic, the
+ * same bits on every rank).  Same semantics as the NCCL transport — it runs the multi-rank code
+ * paths on a single GPU.  A mismatched call sequence fails with AMGT_ERR_NCCL after 300 s. */
+typedef struct amgt_dist_group amgt_dist_group;
+amgt_status amgt_dist_group_create(int size, amgt_dist_group** G);
+amgt_status amgt_dist_group_destroy(amgt_dist_group* G);  /* after every member's amgt_dist_destroy */
+/* A member failed outside the library: every call waiting on the group returns AMGT_ERR_NCCL. */
+amgt_status amgt_dist_group_abort(amgt_dist_group* G);
+amgt_status amgt_dist_create_loopback(amgt_dist_group* G, int rank, int64_t row_begin, int64_t row_end,
+                                      amgt_dist** D);
+amgt_status amgt_dist_destroy(amgt_dist* D);
+
+/* In-place sum over ranks of count doubles (device buffer). */
+amgt_status amgt_dist_allreduce_sum(amgt_dist* D, double* buf, int64_t count, void* stream);
+
+/*
+ * y_local = (A x)_own rows (§IV.D SpMV, L218-230, over a row partition).  A_local: own rows, global
+ * columns (square A; any precision).  x_local/y_local: own rows, FP64 for an FP64 matrix, else
+ * FP32 (R16).  The halo of x is exchanged (one point-to-point group on the communication stream)
+ * while the interior block rows (rows whose columns are all owned) run; the boundary rows follow.
+ * The first call for a matrix builds its plan (syncs; a shifted column array + an extended x
+ * buffer, cached in D and keyed by A's arrays — A must stay alive and unchanged while D uses it;
+ * freed by amgt_dist_destroy).  Values equal amgt_spmv's on the assembled matrix bit for bit.
+ */
+amgt_status amgt_dist_spmv(amgt_dist* D, const amgt_mbsr* A_local, const void* x_local, void* y_local, void* stream);
+
+/*
+ * Ac_l = own rows of R (A P) (Alg. 1 line 5, L54; R20) over a row partition: R_l = own COARSE
+ * rows of R (global fine columns), A_l = own fine rows of A (global columns), P_l = own fine rows
+ * of P (global coarse columns); one precision.  The rows of P that A_l's columns reach are
+ * gathered from their owners (row lengths, then tiles: one host sync), AP_l = A_l P_ext locally;
+ * the rows of AP that R_l's columns reach likewise (none when aggregates are rank-local); then
+ * Ac_l = R_l AP_ext.  Ac_l: own coarse rows, global coarse columns, allocated with al.  The
+ * structure equals the corresponding rows of the single-GPU R (A P) bit for bit.
+ */
+amgt_status amgt_dist_rap(amgt_dist* D, const amgt_mbsr* R_l, const amgt_mbsr* A_l, const amgt_mbsr* P_l,
+                          amgt_mbsr* Ac_l, const amgt_allocator* al, void* stream);
+
+/* M_full = every rank's rows of a row-partitioned matrix, in rank order (agglomeration). */
+amgt_status amgt_dist_allgather_mbsr(amgt_dist* D, const amgt_mbsr* M_local, amgt_mbsr* M_full,
+                                     const amgt_allocator* al, void* stream);
+
+/*
+ * Distributed hierarchy (Alg. 1 with fixed interpolation, L52-58) and V-cycle (Alg. 2, L68-82).
+ *   A_l: own rows of A_1 (FP64, global columns, rows [row_begin, row_end) of amgt_dist_create).
+ *   P_l[k]: own fine rows of P_k (FP64, global coarse columns); a rank's coarse rows are the
+ *   columns its P rows reach, which must form contiguous ranges in rank order (aggregates never
+ *   straddle ranks — true for the z-slab partition; else AMGT_ERR_UNSUPPORTED).
+ * Levels whose global row count is at most agg_rows (from level 2 on; the coarsest always) are
+ * AGGLOMERATED: their operators are all-gathered at setup and the single-GPU V-cycle machinery
+ * runs on them redundantly on every rank (one all-gather of the right-hand side per cycle instead
+ * of a halo exchange per coarse-level SpMV).  With one rank the whole hierarchy is the
+ * single-GPU one.  o: as amgt_hierarchy_create (level 1 FP64, interp = AMGT_INTERP_GIVEN).
+ * A_l and P_l are borrowed (keep them alive until amgt_dist_hierarchy_destroy).  Syncs.
+ */
+typedef struct amgt_dist_hierarchy amgt_dist_hierarchy;
+amgt_status amgt_dist_hierarchy_create(amgt_dist* D, const amgt_mbsr* A_l, const amgt_mbsr* const* P_l, int nlev,
+                                       const amgt_vcycle_opts* o, int64_t agg_rows, const amgt_allocator* al,
+                                       void* stream, amgt_dist_hierarchy** H);
+/* ncycles V-cycles; b_local, x_local: own rows of level 1 (FP64, 4*ceil(m/4) elements).
+ * res_norms_host[ncycles+1]: global ||b - A x|| (all-reduced); *spmv_calls_host: this rank's
+ * SpMV operations of Alg. 2 (the same count on every rank and as amgt_vcycle).  Syncs at the end. */
+amgt_status amgt_dist_vcycle(amgt_dist_hierarchy* H, const double* b_local, double* x_local, int ncycles,
+                             double* res_norms_host, int64_t* spmv_calls_host, void* stream);
+typedef struct {
+    int nlev, agg_level;         /* levels [0, agg_level) distributed, the rest agglomerated */
+    int64_t rows[8];             /* own rows (distributed levels) / global rows (agglomerated) */
+    int64_t tiles[8];            /* own tiles / global tiles */
+    int64_t row_begin[8];        /* first own row (distributed levels) */
+    int64_t ext_begin[8], ext_end[8];  /* the row range the own rows' columns touch */
+    int halo_recv[8], halo_send[8];    /* halo pieces received / sent per SpMV */
+    int64_t interior[8][2];      /* interior block rows [begin, end) (computed while the halo flies) */
+} amgt_dist_hier_info;
+amgt_status amgt_dist_hierarchy_info(const amgt_dist_hierarchy* H, amgt_dist_hier_info* out);
+amgt_status amgt_dist_hierarchy_destroy(amgt_dist_hierarchy* H);
+
+/* Host only (no GPU, not collective): the halo plan of rank `rank` from the all-gathered metadata
+ * — rows[q] own rows of the gathered operand per rank, colmin[q] / colmax[q] the min / max tile
+ * column of rank q's matrix (colmin > colmax: no tiles).  ext_host = {eb, ee} (block rows);
+ * recv: pieces [begin, end) of [eb, ee) owned by other ranks; send: pieces of the own block rows
+ * in other ranks' ranges; at most cap each. */
+typedef struct {
+    int32_t peer;
+    int64_t begin, end; /* global block rows */
+} amgt_dist_piece;
+amgt_status amgt_dist_plan_host(int rank, int size, const int64_t* rows, const int64_t* colmin, const int64_t* colmax,
+                                int64_t* ext_host, amgt_dist_piece* recv, int* nrecv, amgt_dist_piece* send, int* nsend,
+                                int cap);
 
 /* ------------------------------------------------------------- instrumentation */
 

@@ -72,18 +72,15 @@ class c_vcycle_opts(ctypes.Structure):
                 ("theta", ctypes.c_double), ("omega_p", ctypes.c_double)]
 
 
-class c_dist_level(ctypes.Structure):
-    _fields_ = [("A", ctypes.c_void_p), ("P", ctypes.c_void_p), ("R", ctypes.c_void_p), ("m", ctypes.c_int64),
-                ("off", ctypes.c_int64), ("int0", ctypes.c_int64), ("int1", ctypes.c_int64), ("xe", ctypes.c_void_p * 2),
-                ("b", ctypes.c_void_p), ("r", ctypes.c_void_p), ("dinv", ctypes.c_void_p), ("vprec", ctypes.c_int),
-                ("nsend", ctypes.c_int), ("nrecv", ctypes.c_int), ("send_peer", ctypes.c_void_p),
-                ("send_off", ctypes.c_void_p), ("send_cnt", ctypes.c_void_p), ("recv_peer", ctypes.c_void_p),
-                ("recv_off", ctypes.c_void_p), ("recv_cnt", ctypes.c_void_p)]
+class c_dist_piece(ctypes.Structure):
+    _fields_ = [("peer", ctypes.c_int32), ("begin", ctypes.c_int64), ("end", ctypes.c_int64)]
 
 
-class c_dist_coarse(ctypes.Structure):
-    _fields_ = [("n", ctypes.c_int64), ("Ainv", ctypes.c_void_p), ("counts", ctypes.c_void_p),
-                ("displs", ctypes.c_void_p), ("bfull", ctypes.c_void_p), ("xfull", ctypes.c_void_p)]
+class c_dist_hier_info(ctypes.Structure):
+    _fields_ = [("nlev", ctypes.c_int), ("agg_level", ctypes.c_int), ("rows", ctypes.c_int64 * 8),
+                ("tiles", ctypes.c_int64 * 8), ("row_begin", ctypes.c_int64 * 8), ("ext_begin", ctypes.c_int64 * 8),
+                ("ext_end", ctypes.c_int64 * 8), ("halo_recv", ctypes.c_int * 8), ("halo_send", ctypes.c_int * 8),
+                ("interior", (ctypes.c_int64 * 2) * 8)]
 
 
 class c_sweep_stage(ctypes.Structure):
@@ -141,12 +138,24 @@ _sigs = {
                                      _vp]),
     "amgt_sa_interp": (_int, [_P(c_mbsr), _P(c_mbsr), ctypes.c_double, ctypes.c_double, _P(c_mbsr), _P(c_allocator),
                                _vp]),
-    "amgt_dist_unique_id": (_int, [_vp]),
-    "amgt_dist_create": (_int, [_vp, _int, _int, _P(_vp)]),
+    "amgt_nccl_unique_id": (_int, [_vp]),
+    "amgt_dist_create": (_int, [_vp, _int, _int, _i64, _i64, _P(_vp)]),
+    "amgt_dist_group_create": (_int, [_int, _P(_vp)]),
+    "amgt_dist_group_destroy": (_int, [_vp]),
+    "amgt_dist_group_abort": (_int, [_vp]),
+    "amgt_dist_create_loopback": (_int, [_vp, _int, _i64, _i64, _P(_vp)]),
     "amgt_dist_destroy": (_int, [_vp]),
     "amgt_dist_allreduce_sum": (_int, [_vp, _vp, _i64, _vp]),
-    "amgt_dist_vcycle": (_int, [_vp, _int, _P(c_dist_level), _P(c_dist_coarse), ctypes.c_double, _int, _int, _vp, _vp,
-                                _int, _P(ctypes.c_double), _P(_i64), _vp]),
+    "amgt_dist_spmv": (_int, [_vp, _P(c_mbsr), _vp, _vp, _vp]),
+    "amgt_dist_rap": (_int, [_vp, _P(c_mbsr), _P(c_mbsr), _P(c_mbsr), _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_dist_allgather_mbsr": (_int, [_vp, _P(c_mbsr), _P(c_mbsr), _P(c_allocator), _vp]),
+    "amgt_dist_hierarchy_create": (_int, [_vp, _P(c_mbsr), _P(_P(c_mbsr)), _int, _P(c_vcycle_opts), _i64,
+                                          _P(c_allocator), _vp, _P(_vp)]),
+    "amgt_dist_vcycle": (_int, [_vp, _vp, _vp, _int, _P(ctypes.c_double), _P(_i64), _vp]),
+    "amgt_dist_hierarchy_info": (_int, [_vp, _P(c_dist_hier_info)]),
+    "amgt_dist_hierarchy_destroy": (_int, [_vp]),
+    "amgt_dist_plan_host": (_int, [_int, _int, _vp, _vp, _vp, _vp, _P(c_dist_piece), _P(_int), _P(c_dist_piece),
+                                   _P(_int), _int]),
 }
 for _name, (_res, _args) in _sigs.items():
     _f = getattr(_L, _name)
@@ -540,6 +549,7 @@ class Hierarchy:
         for k in range(8):
             o.level_prec[k] = PREC[lp[k]]
         self._keep = [A, *Ps]
+        self.npad = 4 * A.blc_row  # length of the level-1 vectors the library reads and writes
         arr = (_P(c_mbsr) * max(len(Ps), 1))(*[ctypes.pointer(p.c) for p in Ps])
         h = ctypes.c_void_p()
         _check(_L.amgt_hierarchy_create(ctypes.byref(A.c), arr, self.nlev, ctypes.byref(o), _AL, _stream(stream),
@@ -559,8 +569,17 @@ class Hierarchy:
             return M
         return mk(a), mk(p), mk(r)
 
+    def _check_vectors(self, b: torch.Tensor, x: torch.Tensor):
+        """The ABI reads b and writes x over 4*blc_row(A_1) elements (include/amgt.h)."""
+        for name, t in (("b", b), ("x", x)):
+            if t.dtype != torch.float64 or not t.is_cuda or not t.is_contiguous():
+                raise TypeError(f"{name}: expected a contiguous CUDA float64 tensor")
+            if t.numel() < self.npad:
+                raise ValueError(f"{name} has {t.numel()} elements; the level-1 vectors need 4*blc_row = {self.npad} "
+                                 "(zero-pad to a multiple of 4)")
+
     def vcycle(self, b: torch.Tensor, x: torch.Tensor, ncycles: int, stream=None):
-        assert b.dtype == torch.float64 and x.dtype == torch.float64 and b.is_cuda and x.is_cuda
+        self._check_vectors(b, x)
         res = (ctypes.c_double * (ncycles + 1))()
         calls = ctypes.c_int64(0)
         _check(_L.amgt_vcycle(self.h, b.data_ptr(), x.data_ptr(), int(ncycles), res, ctypes.byref(calls),
@@ -569,7 +588,7 @@ class Hierarchy:
 
     def pcg(self, b: torch.Tensor, x: torch.Tensor, maxit: int, rtol: float = 0.0, stream=None):
         """amgt_pcg: V-cycle-preconditioned CG; returns (residual norms, iterations, SpMV calls)."""
-        assert b.dtype == torch.float64 and x.dtype == torch.float64 and b.is_cuda and x.is_cuda
+        self._check_vectors(b, x)
         res = (ctypes.c_double * (maxit + 1))()
         it, calls = ctypes.c_int(0), ctypes.c_int64(0)
         _check(_L.amgt_pcg(self.h, b.data_ptr(), x.data_ptr(), int(maxit), float(rtol), res, ctypes.byref(it),

@@ -33,6 +33,16 @@ amgt_status fail(amgt_status st, const char* fmt, ...);
                                 cudaGetErrorString(e_));                                         \
     } while (0)
 
+// An error a previous CUDA call left pending in this host thread would be reported by the next
+// launch check of a library call that did nothing wrong: name it at the entry point instead.
+#define AMGT_NO_PENDING(fn)                                                                      \
+    do {                                                                                         \
+        cudaError_t e_ = cudaGetLastError();                                                     \
+        if (e_ != cudaSuccess)                                                                   \
+            return ::amgt::fail(AMGT_ERR_CUDA, "%s: CUDA error pending from an earlier call: %s", fn, \
+                                cudaGetErrorString(e_));                                         \
+    } while (0)
+
 #define AMGT_TRY(expr)                       \
     do {                                     \
         amgt_status s_ = (expr);             \
@@ -68,6 +78,13 @@ struct Scratch {
         p = static_cast<T*>(scratch_get(count * sizeof(T), s));
         if (!p) return fail(AMGT_ERR_ALLOC, "scratch allocation of %zu bytes failed", count * sizeof(T));
         return AMGT_OK;
+    }
+    bool try_init(Alloc& al, size_t count) {  // optional scratch: false (no error set) on failure
+        s = al.s;
+        n = count;
+        if (count == 0) return true;
+        p = static_cast<T*>(scratch_get(count * sizeof(T), s));
+        return p != nullptr;
     }
     ~Scratch() {
         if (p) scratch_put(p, s);

@@ -710,6 +710,7 @@ amgt_status amgt_csr_to_mbsr(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     if (m > 0 && !row_ptr) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: row_ptr is NULL");
     if (nnz > 0 && (!col_idx || !val)) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: col/val NULL");
     if (ceil_div(n, 4) > INT32_MAX) return fail(AMGT_ERR_ARG, "amgt_csr_to_mbsr: too many columns for int32 tile indices");
+    AMGT_NO_PENDING("amgt_csr_to_mbsr");
     Alloc a{al, (cudaStream_t)stream};
     return csr_to_mbsr_impl(m, n, nnz, row_ptr, col_idx, val, prec, out, a, 0);
 }

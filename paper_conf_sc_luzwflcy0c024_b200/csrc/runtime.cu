@@ -48,20 +48,42 @@ void Alloc::put(void* p, size_t bytes) {
     cudaFreeAsync(p, s);
 }
 
-void* scratch_get(size_t bytes, cudaStream_t s) {
-    static bool pool_set = false;
-    if (!pool_set) {  // keep freed pool memory cached across synchronisations
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaMemPool_t pool;
-        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-            uint64_t thr = UINT64_MAX;
-            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+// Scratch comes from a library-owned stream-ordered pool (not the device default pool, which
+// torch or the caller may configure).  Freed scratch stays cached up to a release threshold
+// (AMGT_SCRATCH_CACHE_MB, default 1024 MB); beyond it the pool returns memory to the device at
+// the next synchronisation, so large transient buffers (SpGEMM candidate lists, hash tables)
+// do not stay reserved for the life of the process.
+static cudaMemPool_t scratch_pool() {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!pools[dev]) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
         }
-        pool_set = true;
+        const char* e = getenv("AMGT_SCRATCH_CACHE_MB");
+        uint64_t thr = (uint64_t)(e ? atoll(e) : 1024) << 20;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[dev] = p;
     }
+    return pools[dev];
+}
+
+void* scratch_get(size_t bytes, cudaStream_t s) {
     void* p = nullptr;
-    if (cudaMallocAsync(&p, bytes ? bytes : 16, s) != cudaSuccess) {
+    cudaMemPool_t pool = scratch_pool();
+    const cudaError_t e = pool ? cudaMallocFromPoolAsync(&p, bytes ? bytes : 16, pool, s)
+                               : cudaMallocAsync(&p, bytes ? bytes : 16, s);
+    if (e != cudaSuccess) {
         cudaGetLastError();
         return nullptr;
     }
@@ -252,14 +274,18 @@ static double host_ms() {
     clock_gettime(CLOCK_MONOTONIC, &ts);
     return ts.tv_sec * 1e3 + ts.tv_nsec * 1e-6;
 }
+static std::mutex g_trace_mu;  // loopback ranks trace from several threads
 void trace_point(const char* name, cudaStream_t s) {
     if (!trace_on()) return;
     const double e = host_ms();
     cudaStreamSynchronize(s);
+    std::lock_guard<std::mutex> lk(g_trace_mu);
     g_trace.push_back(TracePt{name, e, host_ms()});
 }
 void trace_dump() {
-    if (!trace_on() || g_trace.empty()) return;
+    if (!trace_on()) return;
+    std::lock_guard<std::mutex> lk(g_trace_mu);
+    if (g_trace.empty()) return;
     double prev = g_trace.front().done_ms;
     for (const TracePt& t : g_trace) {
         fprintf(stderr, "trace %-20s enqueue %8.3f ms  device-done %8.3f ms\n", t.name, t.enq_ms - prev,

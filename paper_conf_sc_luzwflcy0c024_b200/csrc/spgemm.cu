@@ -2040,6 +2040,19 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     amgt_mbsr C{};
     C.blc_ptr = (int64_t*)a.get((BR + 1) * sizeof(int64_t));
     if (!C.blc_ptr) return fail(AMGT_ERR_ALLOC, "SpGEMM: blc_ptr allocation failed");
+    // every error return below releases what C holds (blc_ptr alone before mbsr_alloc)
+    bool done = false;
+    struct CGuard {
+        amgt_mbsr& C;
+        Alloc& a;
+        bool& done;
+        int64_t BR;
+        ~CGuard() {
+            if (done) return;
+            if (C.own) mbsr_release(&C, a);
+            else a.put(C.blc_ptr, (BR + 1) * sizeof(int64_t));
+        }
+    } cguard{C, a, done, BR};
     unsigned long long hs[16];
     {
         TimerScope ts(TC_SPGEMM_SYM, (A->blc_num + B->blc_num) * 6.0 + (A->blc_row + B->blc_row) * 8.0, s);
@@ -2049,11 +2062,9 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         // stays moderate; step 2 is then a copy
         Scratch<int32_t> sidx;
         Scratch<uint16_t> smap;
-        const bool keep = BR > 0 && (double)BR * SMALL_CUB * 6.0 <= 2e9;
-        if (keep) {
-            AMGT_TRY(sidx.init(a, (size_t)BR * SMALL_CUB));
-            AMGT_TRY(smap.init(a, (size_t)BR * SMALL_CUB));
-        }
+        bool keep = BR > 0 && (double)BR * SMALL_CUB * 6.0 <= 2e9;
+        if (keep)  // optional: without it step 2 re-expands the rows (k_sym_flat<2>)
+            keep = sidx.try_init(a, (size_t)BR * SMALL_CUB) && smap.try_init(a, (size_t)BR * SMALL_CUB);
         if (BR > 0) {
             k_sym_flat<1><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nnz_row.p, nullptr, nullptr, nullptr,
                                                                      bin_of.p, stats, sidx.p, smap.p);
@@ -2097,13 +2108,13 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats, cursor, rows.p);
             AMGT_LAUNCHED();
             amgt_status st = run_bins<1>(cnt_big, off, rows.p, c, B->blc_col, a, nnz_row.p, nullptr, nullptr, nullptr, s);
-            if (st != AMGT_OK) { a.put(C.blc_ptr, (BR + 1) * 8); return st; }
+            if (st != AMGT_OK) return st;
             AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
             AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
             AMGT_TRY(read_back(false));  // sync 2: C tile count with the long rows
         }
         amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
-        if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+        if (st != AMGT_OK) return st;
         C.row_max = (int64_t)hmax;
         if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
         if (BR > 0) {  // step 2 (Alg. 3 lines 13-14 + bitmap OR, R15)
@@ -2116,7 +2127,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             AMGT_LAUNCHED();
             if (big > 0) {
                 st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
-                if (st != AMGT_OK) { mbsr_release(&C, a); return st; }
+                if (st != AMGT_OK) return st;
             }
         }
         ts.bytes = (A->blc_num + B->blc_num) * 6.0 * 2 + (A->blc_row + B->blc_row) * 8.0 + TC * 6.0 + (BR + 1) * 8.0;
@@ -2140,6 +2151,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         AMGT_CUDA(cudaStreamSynchronize(s));
         for (int k = 0; k < 3; ++k) info->numeric_rows[k] = (int64_t)h3[k];
     }
+    done = true;
     *Cout = C;
     return AMGT_OK;
 }

@@ -23,10 +23,31 @@
 #include <type_traits>
 #include <cstdlib>
 
+#include <mutex>
+#include <unordered_map>
+
 #include "common.cuh"
 #include "spmv_core.cuh"
 
 namespace amgt {
+
+// resident 256-thread CTAs per SM of a kernel, queried once per kernel (the level-1 SpMVs of the
+// V-cycle loop are launched directly: no host-side occupancy query per launch)
+static int occupancy_256(const void* kern) {
+    static std::mutex mu;
+    static std::unordered_map<const void*, int> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(kern);
+    if (it != cache.end()) return it->second;
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, 0) != cudaSuccess) {
+        cudaGetLastError();
+        per_sm = 0;
+    }
+    cache[kern] = per_sm;
+    return per_sm;
+}
+
 
 constexpr int WARP_CAPACITY = 64;  // tiles per warp chunk (L220)
 
@@ -664,8 +685,7 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
     auto go = [&](auto kern) {
         unsigned g = blocks;
         if (persist > 0) {  // exactly the resident CTAs (no partial last wave)
-            int per_sm = 0;
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, 0);
+            const int per_sm = occupancy_256(reinterpret_cast<const void*>(kern));
             const unsigned cap = (unsigned)num_sms() * (unsigned)std::max(per_sm, 1);
             // auto (1): only while the partial last wave is a visible share of the launch; over
             // many waves a grid-stride loop lets the warps drift apart in the address space
@@ -763,7 +783,11 @@ amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* 
     const double extra = (ea.mode == AMGT_EPI_JACOBI || ea.mode == EPI_JACOBI_NORM) ? 2 * vec
                          : (ea.mode == AMGT_EPI_JACOBI_RES || ea.mode == EPI_RES_X0) ? 3 * vec
                          : (ea.mode == AMGT_EPI_Y ? 0.0 : vec);
-    TimerScope ts(timer_class, spmv_bytes(A, xp, yp) + extra, s);
+    // a block-row range (the distributed path's interior / boundary launches) counts its share
+    const double frac = (ea.I1 >= 0 && A->blc_row > 0)
+                            ? (double)(std::min<int64_t>(ea.I1, A->blc_row) - ea.I0) / (double)A->blc_row
+                            : 1.0;
+    TimerScope ts(timer_class, (spmv_bytes(A, xp, yp) + extra) * frac, s);
     switch (A->prec) {
         case AMGT_FP64: return dispatch_xy<double>(A, x, xp, y, yp, ea, s);
         case AMGT_FP32: return dispatch_xy<float>(A, x, xp, y, yp, ea, s);

@@ -69,6 +69,9 @@ struct amgt_hierarchy {
     bool graph_failed = false;
     int64_t sub_calls = 0, sub_launches = 0;
     amgt_sweep_plan* sw = nullptr;  // level-1 fused sweeps (amgt_spmv_sweeps), when usable
+    // replicated tail of a distributed hierarchy (dist.cu): level 0 is a coarse level, so its
+    // vectors follow its precision (FP32 below FP64, R16) instead of the level-1 FP64 rule
+    bool vec_from_prec = false;
     Alloc alloc() { return Alloc{has_al ? &al : nullptr, s}; }
 };
 
@@ -257,8 +260,8 @@ static void launch_dinv(const amgt_mbsr& A, int64_t off, void* dinv, bool l1, cu
                                                                        (const M*)A.blc_val, (V*)dinv, l1);
 }
 
-static amgt_status dinv_impl(const amgt_mbsr& A, int64_t off, void* dinv, amgt_prec vprec, cudaStream_t s,
-                             bool l1 = false) {
+amgt_status dinv_impl(const amgt_mbsr& A, int64_t off, void* dinv, amgt_prec vprec, cudaStream_t s,
+                      bool l1 = false) {
     if (A.blc_row == 0) return AMGT_OK;
     const bool v64 = vprec == AMGT_FP64;
     switch (A.prec) {
@@ -308,6 +311,88 @@ static bool dense_inverse(int64_t n, std::vector<double>& a, std::vector<double>
         }
     }
     return true;
+}
+
+// ---------------------------------------------------------------- coarsest level (R22)
+// The coarsest operator A_M (n <= 4096 rows) as a dense FP64 matrix on the device: one thread
+// per tile scatters its bitmap-marked entries (values widened exactly).
+template <typename T>
+__global__ void k_dense_scatter(int64_t BR, int64_t n, const int64_t* __restrict__ ptr,
+                                const int32_t* __restrict__ idx, const uint16_t* __restrict__ map,
+                                const T* __restrict__ val, double* __restrict__ D) {
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t t = ptr[I]; t < ptr[I + 1]; ++t) {
+            const uint32_t mp = map[t];
+            const int64_t J = idx[t];
+            for (int e = 0; e < 16; ++e)
+                if ((mp >> e) & 1u) D[(4 * I + (e >> 2)) * n + 4 * J + (e & 3)] = to_f64(val[16 * t + e]);
+        }
+}
+
+// In-place Gauss-Jordan inversion of an SPD matrix without pivoting (every pivot of an SPD
+// matrix is positive), one cooperative grid: step k scales the pivot row (r_j = a_kj / a_kk,
+// r_k = 1 / a_kk) and keeps the pivot column c_i = a_ik, then a_ij -= c_i r_j for i != k (with
+// a_ik taken as 0) and row k = r.  A non-positive pivot sets FLAG_SPD (not SPD).  n^3 FMAs over
+// every SM, two grid barriers per step.
+constexpr uint32_t FLAG_SPD = 4u;
+__global__ void __launch_bounds__(256) k_gauss_jordan(int64_t n, double* __restrict__ a, double* __restrict__ rbuf,
+                                                      double* __restrict__ cbuf, uint32_t* __restrict__ flag) {
+    namespace cg = cooperative_groups;
+    cg::grid_group g = cg::this_grid();
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t k = 0; k < n; ++k) {
+        const double piv = a[k * n + k];
+        if (tid == 0 && !(piv > 0.0)) atomicOr(flag, FLAG_SPD);
+        for (int64_t j = tid; j < n; j += nt) {
+            rbuf[j] = (j == k ? 1.0 : a[k * n + j]) / piv;
+            cbuf[j] = a[j * n + k];
+        }
+        g.sync();
+        for (int64_t e = tid; e < n * n; e += nt) {
+            const int64_t i = e / n, j = e - i * n;
+            a[e] = i == k ? rbuf[j] : (j == k ? 0.0 : a[e]) - cbuf[i] * rbuf[j];
+        }
+        g.sync();
+    }
+}
+
+// Ainv = A_M^-1 on the device (dense scatter + Gauss-Jordan); FLAG_SPD into dflag.
+static amgt_status device_coarse_inverse(const amgt_mbsr& C, double* Ainv, uint32_t* dflag, Alloc& a) {
+    cudaStream_t s = a.s;
+    const int64_t n = C.m;
+    AMGT_CUDA(cudaMemsetAsync(Ainv, 0, n * n * sizeof(double), s));
+    const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(C.blc_row, 128), 1024));
+    switch (C.prec) {
+        case AMGT_FP64:
+            k_dense_scatter<double><<<g, 128, 0, s>>>(C.blc_row, n, C.blc_ptr, C.blc_idx, C.blc_map,
+                                                      (const double*)C.blc_val, Ainv);
+            break;
+        case AMGT_FP32:
+            k_dense_scatter<float><<<g, 128, 0, s>>>(C.blc_row, n, C.blc_ptr, C.blc_idx, C.blc_map,
+                                                     (const float*)C.blc_val, Ainv);
+            break;
+        default:
+            k_dense_scatter<__half><<<g, 128, 0, s>>>(C.blc_row, n, C.blc_ptr, C.blc_idx, C.blc_map,
+                                                      (const __half*)C.blc_val, Ainv);
+    }
+    AMGT_LAUNCHED();
+    if (n == 0) return AMGT_OK;
+    Scratch<double> buf;
+    AMGT_TRY(buf.init(a, 2 * n));
+    static int per_sm = -1;
+    if (per_sm < 0) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_gauss_jordan, 256, 0) != cudaSuccess) per_sm = 1;
+        per_sm = std::max(per_sm, 1);
+    }
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * per_sm,
+                                                                           ceil_div(n * n, 256)));
+    int64_t nn = n;
+    double* rb = buf.p;
+    double* cb = buf.p + n;
+    void* args[] = {&nn, &Ainv, &rb, &cb, &dflag};
+    AMGT_CUDA(cudaLaunchCooperativeKernel((const void*)k_gauss_jordan, dim3(grid), dim3(256), args, 0, s));
+    count_launch();
+    return AMGT_OK;
 }
 
 static void free_level_vectors(amgt_level& L, Alloc& a) {
@@ -366,7 +451,7 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
     for (int k = 0; k < nlev; ++k) {
         amgt_level& L = H->L[k];
         const amgt_prec pk = o->level_prec[k];
-        L.vprec = (k == 0 || pk == AMGT_FP64) ? AMGT_FP64 : AMGT_FP32;  // R16
+        L.vprec = ((k == 0 && !H->vec_from_prec) || pk == AMGT_FP64) ? AMGT_FP64 : AMGT_FP32;  // R16
         if (k == 0) {
             if (pk == A->prec) {
                 L.A = *A;  // borrowed
@@ -453,69 +538,30 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             trace_point("analyze P R", s);
         }
     }
-    // coarsest level: MBSR2CSR, dense inverse on the host (FP64)
+    // coarsest level (R22): dense inverse in FP64 on the device (Gauss-Jordan on the SPD A_M)
     amgt_level& C = H->L[nlev - 1];
     const int64_t n = C.A.m;
     if (n > 4096) return fail(AMGT_ERR_UNSUPPORTED, "coarsest level has %lld rows (dense solve limit 4096)", (long long)n);
-    int64_t* rp = (int64_t*)a.get((n + 1) * sizeof(int64_t));
-    int32_t* ci = (int32_t*)a.get(16 * C.A.blc_num * sizeof(int32_t) + 4);
-    double* v = (double*)a.get(16 * C.A.blc_num * sizeof(double) + 8);
-    if (!rp || !ci || !v) return fail(AMGT_ERR_ALLOC, "coarse CSR allocation failed");
-    AMGT_TRY(mbsr_to_csr_impl(&C.A, rp, ci, v, a));
-    // read back through the pinned buffer when the coarse CSR fits (pageable D2H copies stage
-    // through the driver); the row pointers and the range flag first, then columns and values
-    int64_t* pc = pin ? pin + PIN_COARSE : nullptr;
-    const int64_t pcap = PINNED_SLOTS - PIN_COARSE;
-    const bool pin_rp = pc && n + 2 <= pcap;
-    std::vector<int64_t> hrp(n + 1);
-    uint32_t hflag = 0;  // FP16 range flag of every cast above
-    if (pin_rp) {
-        pc[n + 1] = 0;
-        AMGT_CUDA(cudaMemcpyAsync(pc, rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaMemcpyAsync(pc + n + 1, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaStreamSynchronize(s));
-        std::copy(pc, pc + n + 1, hrp.begin());
-        hflag = (uint32_t)pc[n + 1];
-    } else {
-        AMGT_CUDA(cudaMemcpyAsync(hrp.data(), rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaMemcpyAsync(&hflag, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-        AMGT_CUDA(cudaStreamSynchronize(s));
-    }
-    if (hflag & FLAG_RANGE) return fail(AMGT_ERR_RANGE, "hierarchy: a level value exceeds the FP16 range (65504)");
-    const int64_t nnz = hrp[n];
-    std::vector<int32_t> hci(nnz);
-    std::vector<double> hv(nnz);
-    if (nnz) {
-        const int64_t need = nnz + (nnz + 1) / 2;  // values (8 B) then columns (4 B) in int64 slots
-        if (pc && need <= pcap) {
-            AMGT_CUDA(cudaMemcpyAsync(pc, v, nnz * sizeof(double), cudaMemcpyDeviceToHost, s));
-            AMGT_CUDA(cudaMemcpyAsync(pc + nnz, ci, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-            AMGT_CUDA(cudaStreamSynchronize(s));
-            memcpy(hv.data(), pc, nnz * sizeof(double));
-            memcpy(hci.data(), pc + nnz, nnz * sizeof(int32_t));
-        } else {
-            AMGT_CUDA(cudaMemcpyAsync(hci.data(), ci, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-            AMGT_CUDA(cudaMemcpyAsync(hv.data(), v, nnz * sizeof(double), cudaMemcpyDeviceToHost, s));
-            AMGT_CUDA(cudaStreamSynchronize(s));
-        }
-    }
-    a.put(rp, (n + 1) * sizeof(int64_t));
-    a.put(ci, 16 * C.A.blc_num * sizeof(int32_t) + 4);
-    a.put(v, 16 * C.A.blc_num * sizeof(double) + 8);
-    std::vector<double> dense(n * n, 0.0), inv;
-    for (int64_t i = 0; i < n; ++i)
-        for (int64_t p = hrp[i]; p < hrp[i + 1]; ++p) dense[i * n + hci[p]] = hv[p];
-    if (!dense_inverse(n, dense, inv)) return fail(AMGT_ERR_ARG, "coarsest operator is not SPD (Cholesky failed)");
     H->nM = n;
     H->Ainv = (double*)a.get(n * n * sizeof(double) + 8);
     H->partial = (double*)a.get((NORM_BLOCKS + 1) * sizeof(double));
     if (!H->Ainv || !H->partial) return fail(AMGT_ERR_ALLOC, "coarse inverse allocation failed");
+    AMGT_TRY(device_coarse_inverse(C.A, H->Ainv, dflag, a));
     AMGT_CUDA(cudaMemsetAsync(H->partial, 0, (NORM_BLOCKS + 1) * sizeof(double), H->s));
     H->nws_n = std::max<int64_t>(spmv_warp_norm_count(&H->L[0].A), 1);
     H->nws = (double*)a.get((size_t)H->nws_n * sizeof(double));
     if (!H->nws) return fail(AMGT_ERR_ALLOC, "norm partial allocation failed");
-    AMGT_CUDA(cudaMemcpyAsync(H->Ainv, inv.data(), n * n * sizeof(double), cudaMemcpyHostToDevice, s));
-    AMGT_CUDA(cudaStreamSynchronize(s));
+    uint32_t hflag = 0;  // FP16 range flag of every cast above + the SPD flag of the inverse
+    if (pin) {
+        AMGT_CUDA(cudaMemcpyAsync(pin + PIN_CREATE + 8, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+        hflag = (uint32_t)pin[PIN_CREATE + 8];
+    } else {
+        AMGT_CUDA(cudaMemcpyAsync(&hflag, dflag, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        AMGT_CUDA(cudaStreamSynchronize(s));
+    }
+    if (hflag & FLAG_RANGE) return fail(AMGT_ERR_RANGE, "hierarchy: a level value exceeds the FP16 range (65504)");
+    if (hflag & FLAG_SPD) return fail(AMGT_ERR_ARG, "coarsest operator is not SPD (non-positive pivot)");
     trace_point("coarse inverse", s);
     trace_dump();
     return AMGT_OK;
@@ -1491,6 +1537,61 @@ static amgt_status pcg(amgt_hierarchy* H, const double* b, double* x, int maxit,
         for (int k = 0; k <= it; ++k) res_host[k] = std::sqrt(hn[k]);
     if (iters_host) *iters_host = it;
     if (calls_host) *calls_host = H->spmv_calls;
+    return AMGT_OK;
+}
+
+// ---------------------------------------------------------------- internal: distributed tail
+// (dist.cu) The levels a distributed hierarchy agglomerates onto every rank form an ordinary
+// hierarchy whose level 0 is a coarse level: created from an operator in its level precision,
+// applied as one V-cycle from a zero guess per distributed cycle (Alg. 2 lines 2-10 below the
+// agglomeration level).
+amgt_status hierarchy_create_tail(const amgt_mbsr* A, const amgt_mbsr* const* P, int nlev, const amgt_vcycle_opts* o,
+                                  const amgt_allocator* al, cudaStream_t s, amgt_hierarchy** Hout) {
+    amgt_hierarchy* H = new amgt_hierarchy();
+    H->o = *o;
+    H->s = s;
+    H->vec_from_prec = true;
+    if (al) { H->al = *al; H->has_al = true; }
+    amgt_status st = create(A, P, nlev, o, H);
+    if (st != AMGT_OK) {
+        destroy(H);
+        return st;
+    }
+    *Hout = H;
+    return AMGT_OK;
+}
+
+void hierarchy_free(amgt_hierarchy* H) { destroy(H); }
+
+amgt_prec hierarchy_vprec0(const amgt_hierarchy* H) { return H->L[0].vprec; }
+int64_t hierarchy_npad0(const amgt_hierarchy* H) { return H->L[0].npad; }
+
+// x = one V-cycle on A_0 x = b from x = 0 (level-0 vector precision); adds its SpMV count.
+amgt_status hierarchy_apply(amgt_hierarchy* H, const void* b, void* x, cudaStream_t s, int64_t* calls) {
+    H->s = s;
+    H->spmv_calls = 0;
+    const int M = H->nlev - 1;
+    amgt_level& L0 = H->L[0];
+    void* xc[8];
+    void* xa[8];
+    xc[0] = x;
+    xa[0] = L0.t;
+    for (int k = 1; k <= M; ++k) { xc[k] = H->L[k].x; xa[k] = H->L[k].t; }
+    if (M == 0) {
+        amgt_level tmp = L0;
+        tmp.b = (void*)b;
+        tmp.x = x;
+        AMGT_TRY(L0.vprec == AMGT_FP64 ? dense_solve<double>(H, tmp) : dense_solve<float>(H, tmp));
+        H->spmv_calls = 0;
+    } else {
+        AMGT_CUDA(cudaMemsetAsync(x, 0, vbytes(L0.vprec) * L0.npad, s));
+        AMGT_TRY(down_level(H, 0, b, xc, xa));
+        if (M >= 2) AMGT_TRY(subcycle(H, xc, xa));
+        else AMGT_TRY(coarse_solve(H, xc));
+        AMGT_TRY(up_level(H, 0, b, xc, xa));
+        if (xc[0] != x) AMGT_CUDA(cudaMemcpyAsync(x, xc[0], vbytes(L0.vprec) * L0.npad, cudaMemcpyDeviceToDevice, s));
+    }
+    if (calls) *calls += H->spmv_calls;
     return AMGT_OK;
 }
 
