@@ -348,10 +348,21 @@ typedef struct {
                                 builds P_k = amgt_sa_interp(A_k, P[k], theta, omega_p) in level-k
                                 precision — three SpGEMM calls per level (L54, L302; NEXT-2) */
     double theta;            /* strength threshold for AMGT_INTERP_SA (paper str_thr 0.25, L300) */
-    double omega_p;          /* prolongation smoothing weight for AMGT_INTERP_SA (default 2/3) */
+    double omega_p;          /* prolongation smoothing weight for AMGT_INTERP_SA / _PMIS (default 2/3) */
+    /* AMGT_INTERP_PMIS (2): no P is given; every level is coarsened on the device — PMIS C/F
+       splitting of the strength graph (str_thr = theta, max_row_sum; L300) with aggregates
+       around the C points (amgt_pmis_aggregate, reading R32) — and P_k is the smoothed
+       aggregation amgt_sa_interp(A_k, Pt_k) (one SpGEMM, L54).  The hierarchy stops at
+       nlev levels, at the first level with at most max_coarse_size rows (L300: 3), or when
+       the coarsening stalls; amgt_hierarchy_nlev gives the number built. */
+    int max_coarse_size;     /* 0: no size criterion */
+    double max_row_sum;      /* PMIS strength: rows with |sum_j a_ij| > max_row_sum |a_ii| have no strong
+                                dependencies (L300: 0.8); >= 1 or <= 0 disables */
+    uint64_t seed;           /* PMIS random weights: the counter-based generator of R32 (seed, level) */
 } amgt_vcycle_opts;
 #define AMGT_INTERP_GIVEN 0
 #define AMGT_INTERP_SA 1
+#define AMGT_INTERP_PMIS 2
 #define AMGT_SMOOTH_JACOBI 0
 #define AMGT_SMOOTH_L1_JACOBI 1
 
@@ -400,6 +411,29 @@ amgt_status amgt_pcg(amgt_hierarchy* H, const double* b, double* x, int maxit, d
                      int* iters_host, int64_t* spmv_calls_host, void* stream);
 
 amgt_status amgt_hierarchy_destroy(amgt_hierarchy* H);
+
+/* ------------------------------------------------------- coarsening (§8(f) NEXT-2) */
+/*
+ * PMIS coarsening with aggregation (Alg. 1 line 3, L54; the paper's PMIS, str_thr, max_row_sum,
+ * L300; [71] L385; reading R32 in DESIGN.md).  A square, any precision (strength decisions in FP64
+ * of the stored values):
+ *   S_i = {j != i : -a_ij >= theta max_{k!=i}(-a_ik)}, empty when that max <= 0 or when
+ *         |sum_j a_ij| > max_row_sum |a_ii| (max_row_sum < 1);
+ *   lambda_i = |{j : i in S_j}| + w_i, w_i = weights[i] (device, m) or, when weights is NULL, the
+ *         counter-based generator u(seed, level, i) of R32;
+ *   PMIS rounds: points influencing nobody are F; every undecided point beating every undecided
+ *         neighbour in S u S^T becomes C, then undecided points with a new C point in S_i become F;
+ *   aggregates: C points in row order; F points join their strongest (largest lambda) C point in
+ *         S_i, then the points of S_i assigned that way; the rest are singletons.
+ * agg[m] (device): aggregate of each row; is_c[m] (device, nullable): 1 for C points;
+ * *n_agg_host; *rounds_host (nullable): PMIS rounds.  Deterministic.  Syncs once per round.
+ */
+amgt_status amgt_pmis_aggregate(const amgt_mbsr* A, double theta, double max_row_sum, const double* weights,
+                                uint64_t seed, int level, int32_t* agg, int8_t* is_c, int64_t* n_agg_host,
+                                int* rounds_host, void* stream);
+/* The tentative interpolation of an aggregation: Pt (m x n_agg, precision prec) with Pt(i, agg_i) = 1. */
+amgt_status amgt_aggregation_p(int64_t m, int64_t n_agg, const int32_t* agg, amgt_prec prec, amgt_mbsr* Pt,
+                               const amgt_allocator* al, void* stream);
 
 /* ------------------------------------------------------ distributed path (§8(e)) */
 /*

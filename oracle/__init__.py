@@ -31,6 +31,7 @@ _i64p = np.ctypeslib.ndpointer(dtype=np.int64, flags="C_CONTIGUOUS")
 _i32p = np.ctypeslib.ndpointer(dtype=np.int32, flags="C_CONTIGUOUS")
 _f64p = np.ctypeslib.ndpointer(dtype=np.float64, flags="C_CONTIGUOUS")
 _u16p = np.ctypeslib.ndpointer(dtype=np.uint16, flags="C_CONTIGUOUS")
+_i8p = np.ctypeslib.ndpointer(dtype=np.int8, flags="C_CONTIGUOUS")
 _i64 = ctypes.c_int64
 
 
@@ -78,6 +79,11 @@ def lib():
         L.oracle_strength_count.argtypes = [_i64, _i64p, _i32p, _f64p, ctypes.c_double, _i64p]
         L.oracle_strength_fill.restype = None
         L.oracle_strength_fill.argtypes = [_i64, _i64p, _i32p, _f64p, ctypes.c_double, _i64p, _i32p, _f64p]
+        L.oracle_pmis_aggregate.restype = _i64
+        L.oracle_pmis_aggregate.argtypes = [_i64, _i64p, _i32p, _f64p, ctypes.c_double, ctypes.c_double, _f64p,
+                                            _i8p, _i32p, ctypes.POINTER(ctypes.c_int)]
+        L.oracle_pmis_weights.restype = None
+        L.oracle_pmis_weights.argtypes = [_i64, ctypes.c_uint64, ctypes.c_int, _f64p]
         L.oracle_sa_combine.restype = None
         L.oracle_sa_combine.argtypes = [_i64, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p, _i64p, _i32p, _f64p,
                                         ctypes.c_double]
@@ -391,4 +397,57 @@ def build_hierarchy_sa(A, Pts, theta: float = 0.25, omega: float = 2.0 / 3.0, nt
         R = transpose(P)
         PR.append((P, R))
         As.append(rap(R, As[-1], P, nthreads=nthreads))
+    return As, PR
+
+
+# ---------------------------------------------------------------- O10 PMIS aggregation
+def pmis_weights(n: int, seed: int, level: int = 0) -> np.ndarray:
+    """PMIS's random weights w_i in [0, 1): the counter-based generator both sides implement
+    (splitmix64 of seed + golden * (1 + i + 2^40 level); R32)."""
+    w = np.zeros(max(n, 1), dtype=np.float64)
+    lib().oracle_pmis_weights(int(n), int(seed) & 0xFFFFFFFFFFFFFFFF, int(level), w)
+    return w[:n]
+
+
+def pmis_aggregate(A, weights, theta: float = 0.25, max_row_sum: float = 0.8):
+    """O10: PMIS C/F splitting on the strength graph (str_thr, max_row_sum, L300; [71] L385) and
+    aggregates around the C points (reading R32).  Returns (agg int32[n], is_c int8[n],
+    n_agg, rounds)."""
+    A = as_csr(A)
+    w = np.ascontiguousarray(weights, dtype=np.float64)
+    assert w.size >= A.m
+    st = np.zeros(max(A.m, 1), dtype=np.int8)
+    agg = np.zeros(max(A.m, 1), dtype=np.int32)
+    rounds = ctypes.c_int(0)
+    nagg = lib().oracle_pmis_aggregate(A.m, A.row_ptr, A.col, A.val, float(theta), float(max_row_sum), w, st, agg,
+                                       ctypes.byref(rounds))
+    return agg[:A.m], st[:A.m], int(nagg), int(rounds.value)
+
+
+def aggregation_from_labels(agg, nagg: int) -> Csr:
+    """The tentative interpolation of an aggregation: Pt(i, agg_i) = 1."""
+    agg = np.asarray(agg, dtype=np.int32)
+    m = agg.size
+    return Csr(m, int(nagg), np.arange(m + 1, dtype=np.int64), agg.copy(), np.ones(m, dtype=np.float64))
+
+
+def build_hierarchy_pmis(A, max_levels: int, theta: float = 0.25, max_row_sum: float = 0.8, seed: int = 0,
+                         max_coarse_size: int = 0, omega: float = 2.0 / 3.0, nthreads=None):
+    """Alg. 1 with PMIS coarsening (O10, lines 2-3) and SA interpolation through one SpGEMM (O9,
+    line 4), A_{k+1} = R_k (A_k P_k) (O5, line 5); stops at max_levels, at the first level with at
+    most max_coarse_size rows (L300), or when the coarsening stalls.  Level k's PMIS weights are
+    pmis_weights(n_k, seed, k).  Returns (As, PR)."""
+    As = [as_csr(A)]
+    PR = []
+    while len(As) < max_levels:
+        Ak = As[-1]
+        if max_coarse_size > 0 and Ak.m <= max_coarse_size:
+            break
+        agg, _, nagg, _ = pmis_aggregate(Ak, pmis_weights(Ak.m, seed, len(As) - 1), theta, max_row_sum)
+        if nagg == 0 or nagg >= Ak.m:
+            break
+        P = sa_interp(Ak, aggregation_from_labels(agg, nagg), theta, omega)
+        R = transpose(P)
+        PR.append((P, R))
+        As.append(rap(R, Ak, P, nthreads=nthreads))
     return As, PR

@@ -461,3 +461,136 @@ void oracle_sa_combine(int64_t m, const int64_t* trp, const int32_t* tci, double
         }
     }
 }
+
+/* ---------------------------------------------------------------- O10 PMIS aggregation
+ * Coarsening (Alg. 1 line 3, L54; PMIS with str_thr and max_row_sum, L300, [71] L385; reading
+ * R32 in DESIGN.md), written out step by step:
+ *   1. strength: S_i = {j != i : -a_ij >= theta * max_{k!=i}(-a_ik)}, empty when that max is
+ *      <= 0 or when |sum_j a_ij| > max_row_sum * |a_ii| (max_row_sum < 1);
+ *   2. measure: lambda_i = |{j : i in S_j}| + w_i (w_i in [0, 1): the random numbers PMIS draws,
+ *      an input);
+ *   3. points that influence nobody (|{j : i in S_j}| = 0) are F; the rest undecided (U);
+ *   4. rounds until no U: every U point whose lambda exceeds the lambda of every U point in
+ *      S_i u S_i^T becomes C; then every U point with a new C point in S_i becomes F;
+ *   5. aggregates: the C points in row order are aggregates 0..nC-1; (a) an F point with a C
+ *      point in S_i joins the aggregate of the one with the largest lambda (ties: smaller
+ *      index); (b) an F point still without one joins, among the points of S_i assigned in
+ *      (a), the one with the largest lambda; (c) every point still unassigned is a new
+ *      aggregate (row order).
+ * state_out[i]: 1 = C, 0 = F; agg_out[i]; *rounds_out = PMIS rounds.  Returns the number of
+ * aggregates.  Parity unpinned parts: none (hand-worked example + invariants, tests). */
+enum { O_F = 0, O_C = 1, O_U = 2 };
+
+static int oracle_row_strength_ok(int64_t i, const int64_t* rp, const int32_t* ci, const double* v,
+                                  double max_row_sum, double* mi_out) {
+    double mi = 0.0, rs = 0.0, d = 0.0;
+    for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+        rs = rs + v[p];
+        if (ci[p] == i) d = v[p];
+        else if (-v[p] > mi) mi = -v[p];
+    }
+    *mi_out = mi;
+    if (max_row_sum < 1.0 && fabs(rs) > max_row_sum * fabs(d)) return 0;
+    return mi > 0.0;
+}
+
+/* 1 if j (!= i) is in S_i (row i's strong dependencies) */
+static int oracle_in_S(int64_t i, int64_t p, const int32_t* ci, const double* v, double theta, double mi, int ok) {
+    return ok && ci[p] != i && oracle_strong(v[p], mi, theta);
+}
+
+int64_t oracle_pmis_aggregate(int64_t n, const int64_t* rp, const int32_t* ci, const double* v, double theta,
+                              double max_row_sum, const double* w, int8_t* state_out, int32_t* agg_out,
+                              int* rounds_out) {
+    double* mi = (double*)malloc((size_t)(n + 1) * sizeof(double));
+    int* ok = (int*)malloc((size_t)(n + 1) * sizeof(int));
+    int64_t* infl = (int64_t*)calloc((size_t)(n + 1), sizeof(int64_t));
+    double* lam = (double*)malloc((size_t)(n + 1) * sizeof(double));
+    int8_t* st = state_out;
+    int8_t* newc = (int8_t*)calloc((size_t)(n + 1), 1);
+    int8_t* cand = (int8_t*)calloc((size_t)(n + 1), 1);
+    int32_t* aggA = (int32_t*)malloc((size_t)(n + 1) * sizeof(int32_t));
+    /* 1-2: strength and measure */
+    for (int64_t i = 0; i < n; ++i) ok[i] = oracle_row_strength_ok(i, rp, ci, v, max_row_sum, &mi[i]);
+    for (int64_t i = 0; i < n; ++i)
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p)
+            if (oracle_in_S(i, p, ci, v, theta, mi[i], ok[i])) infl[ci[p]] += 1;
+    for (int64_t i = 0; i < n; ++i) {
+        lam[i] = (double)infl[i] + w[i];
+        st[i] = infl[i] == 0 ? O_F : O_U;  /* 3 */
+    }
+    /* 4: PMIS rounds */
+    int rounds = 0;
+    for (;;) {
+        int64_t undecided = 0;
+        for (int64_t i = 0; i < n; ++i) undecided += st[i] == O_U;
+        if (!undecided) break;
+        ++rounds;
+        for (int64_t i = 0; i < n; ++i) cand[i] = st[i] == O_U;
+        for (int64_t i = 0; i < n; ++i)  /* compare across every strong edge i -> j (S_i u S_i^T) */
+            for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+                if (!oracle_in_S(i, p, ci, v, theta, mi[i], ok[i])) continue;
+                const int64_t j = ci[p];
+                if (st[i] != O_U || st[j] != O_U) continue;
+                if (!(lam[i] > lam[j])) cand[i] = 0;
+                if (!(lam[j] > lam[i])) cand[j] = 0;
+            }
+        for (int64_t i = 0; i < n; ++i) {
+            newc[i] = cand[i];
+            if (cand[i]) st[i] = O_C;
+        }
+        for (int64_t i = 0; i < n; ++i) {
+            if (st[i] != O_U) continue;
+            for (int64_t p = rp[i]; p < rp[i + 1]; ++p)
+                if (oracle_in_S(i, p, ci, v, theta, mi[i], ok[i]) && newc[ci[p]]) {
+                    st[i] = O_F;
+                    break;
+                }
+        }
+    }
+    /* 5: aggregates */
+    int32_t nagg = 0;
+    for (int64_t i = 0; i < n; ++i) agg_out[i] = st[i] == O_C ? nagg++ : -1;
+    for (int64_t i = 0; i < n; ++i) {  /* (a) */
+        if (st[i] == O_C) continue;
+        int64_t best = -1;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+            if (!oracle_in_S(i, p, ci, v, theta, mi[i], ok[i])) continue;
+            const int64_t j = ci[p];
+            if (st[j] != O_C) continue;
+            if (best < 0 || lam[j] > lam[best] || (lam[j] == lam[best] && j < best)) best = j;
+        }
+        if (best >= 0) agg_out[i] = agg_out[best];
+    }
+    for (int64_t i = 0; i < n; ++i) aggA[i] = agg_out[i];
+    for (int64_t i = 0; i < n; ++i) {  /* (b): neighbours assigned in (a) */
+        if (aggA[i] >= 0) continue;
+        int64_t best = -1;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+            if (!oracle_in_S(i, p, ci, v, theta, mi[i], ok[i])) continue;
+            const int64_t j = ci[p];
+            if (aggA[j] < 0 || st[j] == O_C) continue;
+            if (best < 0 || lam[j] > lam[best] || (lam[j] == lam[best] && j < best)) best = j;
+        }
+        if (best >= 0) agg_out[i] = aggA[best];
+    }
+    for (int64_t i = 0; i < n; ++i)  /* (c) */
+        if (agg_out[i] < 0) agg_out[i] = nagg++;
+    for (int64_t i = 0; i < n; ++i) st[i] = st[i] == O_C ? 1 : 0;
+    *rounds_out = rounds;
+    free(mi); free(ok); free(infl); free(lam); free(newc); free(cand); free(aggA);
+    return nagg;
+}
+
+/* The counter-based uniform generator of PMIS's random weights (both sides implement it):
+ * z = seed + 0x9E3779B97F4A7C15 * (1 + i + 2^40 * level) (mod 2^64), splitmix64 finaliser,
+ * u = (z >> 11) * 2^-53 in [0, 1). */
+void oracle_pmis_weights(int64_t n, uint64_t seed, int level, double* w) {
+    for (int64_t i = 0; i < n; ++i) {
+        uint64_t z = seed + 0x9E3779B97F4A7C15ull * (1ull + (uint64_t)i + ((uint64_t)level << 40));
+        z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+        z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+        z = z ^ (z >> 31);
+        w[i] = (double)(z >> 11) * (1.0 / 9007199254740992.0);
+    }
+}

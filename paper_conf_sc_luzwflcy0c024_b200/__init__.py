@@ -5,6 +5,6 @@ include/amgt.h (libamgt.so).  This package is the thin Python binding (ctypes).
 """
 from ._lib import (  # noqa: F401
     FP16, FP32, FP64, EXPORTED, LIB_PATH, AmgtError, Hierarchy, Mbsr, csr_to_mbsr, from_csr, launch_count, rap,
-    set_tc_threshold, SweepPlan, sa_interp, spgemm, strength_filter, spgemm_numeric, spgemm_symbolic, spmv, spmv_fused, spmv_jacobi_res, timing_enable, timing_read, timing_reset, timing_sample,
+    set_tc_threshold, SweepPlan, pmis_aggregate, aggregation_p, sa_interp, spgemm, strength_filter, spgemm_numeric, spgemm_symbolic, spmv, spmv_fused, spmv_jacobi_res, timing_enable, timing_read, timing_reset, timing_sample,
     version, wrap,
 )

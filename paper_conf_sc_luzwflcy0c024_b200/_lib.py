@@ -69,7 +69,8 @@ class c_spmv_stats(ctypes.Structure):
 class c_vcycle_opts(ctypes.Structure):
     _fields_ = [("max_levels", ctypes.c_int), ("nu1", ctypes.c_int), ("nu2", ctypes.c_int), ("omega", ctypes.c_double),
                 ("level_prec", ctypes.c_int * 8), ("smoother", ctypes.c_int), ("interp", ctypes.c_int),
-                ("theta", ctypes.c_double), ("omega_p", ctypes.c_double)]
+                ("theta", ctypes.c_double), ("omega_p", ctypes.c_double), ("max_coarse_size", ctypes.c_int),
+                ("max_row_sum", ctypes.c_double), ("seed", ctypes.c_uint64)]
 
 
 class c_dist_piece(ctypes.Structure):
@@ -138,6 +139,9 @@ _sigs = {
                                      _vp]),
     "amgt_sa_interp": (_int, [_P(c_mbsr), _P(c_mbsr), ctypes.c_double, ctypes.c_double, _P(c_mbsr), _P(c_allocator),
                                _vp]),
+    "amgt_pmis_aggregate": (_int, [_P(c_mbsr), ctypes.c_double, ctypes.c_double, _vp, ctypes.c_uint64, _int, _vp, _vp,
+                                   _P(_i64), _P(_int), _vp]),
+    "amgt_aggregation_p": (_int, [_i64, _i64, _vp, _int, _P(c_mbsr), _P(c_allocator), _vp]),
     "amgt_nccl_unique_id": (_int, [_vp]),
     "amgt_dist_create": (_int, [_vp, _int, _int, _i64, _i64, _P(_vp)]),
     "amgt_dist_group_create": (_int, [_int, _P(_vp)]),
@@ -470,6 +474,29 @@ def sa_interp(A: Mbsr, Pt: Mbsr, theta: float = 0.25, omega: float = 2.0 / 3.0, 
     return out
 
 
+def pmis_aggregate(A: Mbsr, theta: float = 0.25, max_row_sum: float = 0.8, weights: torch.Tensor | None = None,
+                   seed: int = 0, level: int = 0, stream=None):
+    """amgt_pmis_aggregate: (agg int32[m], is_c int8[m], n_agg, rounds) on the device."""
+    agg = torch.empty(max(A.m, 1), dtype=torch.int32, device="cuda")
+    isc = torch.empty(max(A.m, 1), dtype=torch.int8, device="cuda")
+    if weights is not None:
+        assert weights.dtype == torch.float64 and weights.is_cuda and weights.numel() >= A.m
+    n, r = ctypes.c_int64(0), ctypes.c_int(0)
+    _check(_L.amgt_pmis_aggregate(ctypes.byref(A.c), float(theta), float(max_row_sum),
+                                  weights.data_ptr() if weights is not None else None, int(seed) & 0xFFFFFFFFFFFFFFFF,
+                                  int(level), agg.data_ptr(), isc.data_ptr(), ctypes.byref(n), ctypes.byref(r),
+                                  _stream(stream)))
+    return agg[:A.m], isc[:A.m], int(n.value), int(r.value)
+
+
+def aggregation_p(agg: torch.Tensor, n_agg: int, prec="f64", stream=None) -> Mbsr:
+    """amgt_aggregation_p: Pt(i, agg_i) = 1."""
+    out = Mbsr()
+    _check(_L.amgt_aggregation_p(int(agg.numel()), int(n_agg), agg.data_ptr(), PREC[prec], ctypes.byref(out.c), _AL,
+                                 _stream(stream)))
+    return out
+
+
 def csr_to_mbsr_ex(m, n, row_ptr, col, val, col_offset: int, prec="f64", stream=None) -> Mbsr:
     out = Mbsr()
     _check(_L.amgt_csr_to_mbsr_ex(int(m), int(n), int(col.numel()), row_ptr.data_ptr(), col.data_ptr(), val.data_ptr(),
@@ -537,14 +564,17 @@ class Hierarchy:
 
     def __init__(self, A: Mbsr, Ps: list, level_prec=("f64", "f32", "f16", "f16", "f16", "f16", "f16", "f16"),
                  nu1=1, nu2=1, omega=2.0 / 3.0, smoother="jacobi", interp="given", theta=0.25,
-                 omega_p=2.0 / 3.0, stream=None):
-        self.nlev = len(Ps) + 1
+                 omega_p=2.0 / 3.0, max_levels=None, max_coarse_size=0, max_row_sum=0.8, seed=0, stream=None):
+        # interp "pmis": no Ps; every level coarsened on the device (amgt_pmis_aggregate + SA),
+        # up to max_levels levels (L300: PMIS, str_thr, max_row_sum, max_coarse_size)
+        self.nlev = int(max_levels) if interp == "pmis" else len(Ps) + 1
         o = c_vcycle_opts()
         o.max_levels = self.nlev
         o.nu1, o.nu2, o.omega = int(nu1), int(nu2), float(omega)
         o.smoother = {"jacobi": 0, "l1_jacobi": 1}[smoother]
-        o.interp = {"given": 0, "sa": 1}[interp]  # "sa": Ps are tentative; P_k by amgt_sa_interp
+        o.interp = {"given": 0, "sa": 1, "pmis": 2}[interp]  # "sa": Ps are tentative; P_k by amgt_sa_interp
         o.theta, o.omega_p = float(theta), float(omega_p)
+        o.max_coarse_size, o.max_row_sum, o.seed = int(max_coarse_size), float(max_row_sum), int(seed)
         lp = list(level_prec) + ["f16"] * 8
         for k in range(8):
             o.level_prec[k] = PREC[lp[k]]
@@ -555,6 +585,7 @@ class Hierarchy:
         _check(_L.amgt_hierarchy_create(ctypes.byref(A.c), arr, self.nlev, ctypes.byref(o), _AL, _stream(stream),
                                         ctypes.byref(h)))
         self.h = h
+        self.nlev = int(_L.amgt_hierarchy_nlev(h))
 
     def level(self, k: int):
         a, p, r = _P(c_mbsr)(), _P(c_mbsr)(), _P(c_mbsr)()

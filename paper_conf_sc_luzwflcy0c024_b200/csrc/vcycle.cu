@@ -29,6 +29,9 @@ amgt_status spmv_ex_impl(const amgt_mbsr* A, const void* x, amgt_prec xp, void* 
 amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* Cout, amgt_spgemm_info* info,
                                  Alloc& a);
 amgt_status spgemm_numeric_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a);
+amgt_status pmis_aggregate_impl(const amgt_mbsr* A, double theta, double mrs, const double* weights, uint64_t seed,
+                                int level, int32_t* agg, int8_t* is_c, int64_t* nagg_host, int* rounds_host, Alloc& a);
+amgt_status aggregation_p_impl(int64_t m, int64_t nagg, const int32_t* agg, amgt_prec prec, amgt_mbsr* Pt, Alloc& a);
 amgt_status sa_interp_impl(const amgt_mbsr* A, const amgt_mbsr* Pt, double theta, double omega, amgt_mbsr* P,
                            Alloc& a);
 
@@ -488,15 +491,41 @@ static amgt_status create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nle
             AMGT_CUDA(cudaMemsetAsync(L.u, 0, vb, s));
             AMGT_TRY(amgt_sweep_plan_create(&L.A, H->has_al ? &H->al : nullptr, s, &H->sw));
         }
+        const double th = o->theta >= 0.0 ? o->theta : 0.25;
+        const double wp = o->omega_p > 0.0 ? o->omega_p : 2.0 / 3.0;
+        if (k + 1 < nlev && o->interp == AMGT_INTERP_PMIS) {
+            // NEXT-2 / Alg. 1 lines 2-4: stop at max_coarse_size; else PMIS aggregation of A_k (R32)
+            // and P_k = (I - w D_F^-1 A_F) Pt through one SpGEMM call
+            bool stop = o->max_coarse_size > 0 && L.A.m <= o->max_coarse_size;
+            amgt_mbsr Pt{};
+            if (!stop) {
+                Scratch<int32_t> agg;
+                AMGT_TRY(agg.init(a, L.A.m + 1));
+                int64_t nagg = 0;
+                const double mrs = o->max_row_sum > 0.0 ? o->max_row_sum : 1.0;
+                AMGT_TRY(pmis_aggregate_impl(&L.A, th, mrs, nullptr, o->seed, k, agg.p, nullptr, &nagg, nullptr, a));
+                stop = nagg == 0 || nagg >= L.A.m;
+                if (!stop) AMGT_TRY(aggregation_p_impl(L.A.m, nagg, agg.p, pk, &Pt, a));
+            }
+            if (stop) {
+                nlev = k + 1;
+                H->nlev = nlev;
+            } else {
+                const amgt_status st = sa_interp_impl(&L.A, &Pt, th, wp, &L.P, a);
+                mbsr_release(&Pt, a);
+                AMGT_TRY(st);
+            }
+            trace_point("PMIS + SA", s);
+        }
         if (k + 1 < nlev) {
-            const amgt_mbsr* Pk = P[k];
-            if (Pk->m != L.A.m) return fail(AMGT_ERR_ARG, "P[%d] has %lld rows, level has %lld", k, (long long)Pk->m, (long long)L.A.m);
-            if (o->interp == AMGT_INTERP_SA) {
+            const amgt_mbsr* Pk = o->interp == AMGT_INTERP_PMIS ? nullptr : P[k];
+            if (Pk && Pk->m != L.A.m) return fail(AMGT_ERR_ARG, "P[%d] has %lld rows, level has %lld", k, (long long)Pk->m, (long long)L.A.m);
+            if (!Pk) {
+                // built above
+            } else if (o->interp == AMGT_INTERP_SA) {
                 // NEXT-2 / Alg. 1 line 4: P_k = (I - w D_F^-1 A_F) Pt through one SpGEMM call
                 amgt_mbsr Pt{};
                 AMGT_TRY(cast_impl(Pk, pk, &Pt, a, dflag));
-                const double th = o->theta >= 0.0 ? o->theta : 0.25;
-                const double wp = o->omega_p > 0.0 ? o->omega_p : 2.0 / 3.0;
                 const amgt_status st = sa_interp_impl(&L.A, &Pt, th, wp, &L.P, a);
                 mbsr_release(&Pt, a);
                 AMGT_TRY(st);
@@ -1601,13 +1630,14 @@ extern "C" {
 
 amgt_status amgt_hierarchy_create(const amgt_mbsr* A, const amgt_mbsr* const* P, int nlev, const amgt_vcycle_opts* o,
                                   const amgt_allocator* al, void* stream, amgt_hierarchy** Hout) {
-    if (!A || !o || !Hout || nlev < 1 || nlev > 8 || (nlev > 1 && !P))
+    const bool pmis = o && o->interp == AMGT_INTERP_PMIS;
+    if (!A || !o || !Hout || nlev < 1 || nlev > 8 || (nlev > 1 && !P && !pmis))
         return fail(AMGT_ERR_ARG, "amgt_hierarchy_create: bad argument");
     if (A->prec != AMGT_FP64) return fail(AMGT_ERR_ARG, "amgt_hierarchy_create: A must be FP64");
     if (A->m != A->n) return fail(AMGT_ERR_ARG, "amgt_hierarchy_create: A must be square");
     for (int k = 0; k < nlev; ++k)
         if (!prec_valid(o->level_prec[k])) return fail(AMGT_ERR_ARG, "bad level precision %d", k);
-    for (int k = 0; k + 1 < nlev; ++k)
+    for (int k = 0; k + 1 < nlev && !pmis; ++k)
         if (!P[k] || P[k]->prec != AMGT_FP64) return fail(AMGT_ERR_ARG, "P[%d] missing or not FP64", k);
     if (o->nu1 < 0 || o->nu2 < 0) return fail(AMGT_ERR_ARG, "negative sweep count");
     if (o->smoother != AMGT_SMOOTH_JACOBI && o->smoother != AMGT_SMOOTH_L1_JACOBI)

@@ -69,7 +69,7 @@ def _raw(rep, metrics):
 def _num(v, unit):
     v = float(str(v).replace(",", ""))
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-9, "usecond": 1e-6,
-             "msecond": 1e-3, "second": 1}.get(unit, 1)
+             "msecond": 1e-3, "second": 1, "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "s": 1}[unit]
     return v * scale
 
 
