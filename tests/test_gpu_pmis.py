@@ -128,3 +128,42 @@ def test_pmis_hierarchy_mixed_precision_rho():
     rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
     live = res_o[1:] / res_o[0] > 1e-10
     assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
+
+
+def test_table2_shape_pres_poisson():
+    """NEXT-3 (L300-331): the Pres_Poisson-shaped synthetic matrix (14,822 rows, 715,804 nonzeros,
+    gen/table2.py) with the paper's settings — PMIS (str_thr 0.25, max_row_sum 0.8), SA
+    interpolation, max_coarse_size 3, at most 7 levels, L1-Jacobi — parity level by level and
+    convergence against the oracle; plus A*A through the SpGEMM against O1."""
+    amgt = _amgt()
+    import gen.table2 as t2
+    from gpu_helpers import check_fp64_entrywise, tile_values_to_csr_order
+    A = t2.table2_matrix("Pres_Poisson")
+    Ao = oracle.as_csr(A)
+    M = amgt.from_csr(A)
+    C = amgt.spgemm(M, M)
+    Co, Cabs = oracle.spgemm(Ao, Ao, with_abs=True)
+    assert_structure_equal(C, oracle.csr_to_mbsr(Co))
+    _, _, cv = tile_values_to_csr_order(C)
+    check_fp64_entrywise(cv, Co.val, Cabs)
+    H = amgt.Hierarchy(M, [], level_prec=("f64",) * 8, interp="pmis", max_levels=7, max_coarse_size=3, seed=1,
+                       smoother="l1_jacobi", omega=1.0)
+    for k in range(H.nlev - 1):
+        Ak, Pk, _ = H.level(k)
+        Ah = _host_csr(Ak)
+        agg, _, n, _ = amgt.pmis_aggregate(Ak, seed=1, level=k)
+        ao, _, no, _ = oracle.pmis_aggregate(Ah, oracle.pmis_weights(Ah.m, 1, k))
+        assert n == no and np.array_equal(agg.cpu().numpy(), ao)
+        assert_structure_equal(Pk, oracle.csr_to_mbsr(oracle.sa_interp(Ah, oracle.aggregation_from_labels(ao, no))))
+    As, PR = oracle.build_hierarchy_pmis(A, 7, seed=1, max_coarse_size=3)
+    assert H.nlev == len(As)
+    b = gen.uniform_vector(A.m, 3)
+    x = torch.zeros(4 * M.blc_row, dtype=torch.float64, device="cuda")
+    bb = torch.zeros_like(x)
+    bb[:A.m] = b.cuda()
+    res, calls = H.vcycle(bb, x, 6)
+    _, res_o, calls_o = oracle.vcycle(As, PR, b.numpy(), ncycles=6, omega=1.0, smoother="l1_jacobi")
+    assert calls == calls_o
+    res, res_o = np.array(res), np.array(res_o)
+    rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
+    assert np.all(np.abs(rho - rho_o) <= 0.01 * rho_o), (rho, rho_o)
