@@ -653,6 +653,199 @@ bool spmv_warp_norm_ok(const amgt_mbsr* A) {
 }
 int64_t spmv_warp_norm_count(const amgt_mbsr* A) { return ceil_div(A->blc_row, 8); }
 
+// ---------------------------------------------------------------- tensor-core routes (L222-228)
+// FP64 (DMMA m8n8k4): one warp per block row walks its tiles in consecutive pairs (t, t+1).  The
+// A fragment [A_t; A_t+1] is ONE coalesced 256-byte load: lane l holds element l % 16 of tile
+// t + l / 16, i.e. row l / 4, column l % 4 of the 8x4 fragment (a[row8][k4], lane = 4 row8 + k4).
+// The B fragment is [x_J | x_J' | 0 ...] (lane 4n + k holds B[k][n]).  C accumulates over the whole
+// row; y_r = C[r][0] + C[4 + r][1] ("diagonal of fragY", L228).  Per-tile routing (R10): a tile
+// with POPCOUNT(map) < tc_thr is multiplied by the CUDA cores of the 16 lanes that loaded it
+// (bitmap-predicated FMAs) and enters the mma with a zero B column; a pair without a dense tile
+// skips the mma.  Values: route-independent up to rounding.  Rows longer than long_thr are the
+// chunk kernel's.
+__device__ __forceinline__ double ldg_f64(const double* p) {
+    double r;
+    asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(r) : "l"(p));
+    return r;
+}
+
+template <typename XT, typename YT, int MODE, int UP>
+__global__ void __launch_bounds__(256) k_spmv_tc64(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
+                                                   const int32_t* __restrict__ bidx, const uint16_t* __restrict__ bmap,
+                                                   const double* __restrict__ bval, const XT* __restrict__ x,
+                                                   Epi<XT, YT, MODE> epi, int64_t long_thr, int tc_thr) {
+    pdl_wait();
+    constexpr unsigned FULL = 0xffffffffu;
+    const int lane = threadIdx.x & 31, h = lane >> 4, e = lane & 15, n = lane >> 2, k = lane & 3;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t I = I0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); I < BR; I += nw) {
+        const int64_t t0 = __ldg(bptr + I), t1 = __ldg(bptr + I + 1);
+        if (t1 - t0 > long_thr) continue;  // warp-uniform
+        typename Epi<XT, YT, MODE>::Pre pre;
+        if (lane < 4) pre = epi.prefetch(4 * I + lane);
+        double c0 = 0.0, c1 = 0.0, cc = 0.0;
+        for (int64_t p = t0; p < t1; p += 2 * UP) {
+            double a[UP];
+            uint32_t mp[UP];
+            int32_t J[UP];
+            bool v[UP];
+#pragma unroll
+            for (int u = 0; u < UP; ++u) {  // every load of the UP pairs in flight together
+                const int64_t t = p + 2 * u + h;
+                v[u] = t < t1;
+                a[u] = v[u] ? ldg_f64(bval + 16 * t + e) : 0.0;
+                mp[u] = v[u] ? __ldg(bmap + t) : 0u;
+                J[u] = v[u] ? __ldg(bidx + t) : 0;
+            }
+            // x operands of all UP pairs requested before any mma (one dependent round trip)
+            double xb[UP], xc[UP];
+            bool dn[UP], any[UP];
+#pragma unroll
+            for (int u = 0; u < UP; ++u) {
+                dn[u] = v[u] && __popc(mp[u]) >= tc_thr;
+                const int32_t Jb = __shfl_sync(FULL, J[u], n == 1 ? 16 : 0);
+                const bool db = __shfl_sync(FULL, dn[u] ? 1 : 0, n == 1 ? 16 : 0) != 0;
+                any[u] = __any_sync(FULL, dn[u]);
+                xb[u] = (n < 2 && db) ? (double)__ldg(x + 4 * (int64_t)Jb + k) : 0.0;
+                xc[u] = (v[u] && !dn[u] && ((mp[u] >> e) & 1u)) ? (double)__ldg(x + 4 * (int64_t)J[u] + (e & 3)) : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < UP; ++u) {
+                if (v[u] && !dn[u]) cc = fma(a[u], xc[u], cc);  // xc = 0 at the clear bits
+                if (any[u]) dmma_884(c0, c1, dn[u] ? a[u] : 0.0, xb[u]);
+            }
+        }
+        double cs = cc + __shfl_xor_sync(FULL, cc, 1);
+        cs += __shfl_xor_sync(FULL, cs, 2);
+        cs += __shfl_xor_sync(FULL, cs, 16);  // lanes 4r.. and 16+4r..: the CUDA-core sum of row r
+        const int r = lane & 3;
+        const double ya = __shfl_sync(FULL, c0, 4 * r), yb = __shfl_sync(FULL, c1, 16 + 4 * r);
+        const double yc = __shfl_sync(FULL, cs, 4 * r);
+        if (lane < 4) epi.finish(4 * I + lane, ya + yb + yc, pre);
+    }
+}
+
+// FP16 (HMMA m16n8k16, FP16 operands, FP32 accumulation, R18): a warp takes FOUR block rows g =
+// 0..3 and their tiles four at a time: A[4g + r][4i + c] = tile i of row g (row r, column c),
+// B[4i + c][g] = x_J(g,i)[c] (x rounded to FP16 for the mma), so C[4g + r][g] = the four tiles'
+// contribution to row r of block row g — 16 tile products per instruction, the diagonal column
+// blocks of C kept.  Tiles with POPCOUNT < tc_thr go through CUDA-core FMAs (FP32, x in FP32) of
+// the lanes that hold them and enter the mma as zeros.
+__device__ __forceinline__ void hmma_16816(float (&c)[4], const uint32_t (&a)[4], const uint32_t (&b)[2]) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+        "{%0, %1, %2, %3};"
+        : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b[0]), "r"(b[1]));
+}
+
+template <typename XT, typename YT, int MODE>
+__global__ void __launch_bounds__(256) k_spmv_tc16(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
+                                                   const int32_t* __restrict__ bidx, const uint16_t* __restrict__ bmap,
+                                                   const __half* __restrict__ bval, const XT* __restrict__ x,
+                                                   Epi<XT, YT, MODE> epi, int64_t long_thr, int tc_thr) {
+    pdl_wait();
+    constexpr unsigned FULL = 0xffffffffu;
+    const int lane = threadIdx.x & 31, gid = lane >> 2, tig = lane & 3;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t Q = I0 + 4 * (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); Q < BR; Q += 4 * nw) {
+        // this lane's two A rows: (g0 = gid / 4, r = gid % 4) and (g0 + 2, r); its B column gid (< 4)
+        const int r = gid & 3, gA = gid >> 2, gB = gA + 2;
+        int64_t ta0 = 0, ta1 = 0, tb0 = 0, tb1 = 0, tn0 = 0, tn1 = 0;
+        auto range = [&](int g, int64_t& lo, int64_t& hi) {
+            const int64_t I = Q + g;
+            lo = hi = 0;
+            if (I < BR) {
+                lo = __ldg(bptr + I);
+                hi = __ldg(bptr + I + 1);
+                if (hi - lo > long_thr) hi = lo;  // chunk kernel's row
+            }
+        };
+        range(gA, ta0, ta1);
+        range(gB, tb0, tb1);
+        if (gid < 4) range(gid, tn0, tn1);
+        int64_t len = max(ta1 - ta0, tb1 - tb0);
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) len = max(len, __shfl_xor_sync(FULL, len, d));
+        typename Epi<XT, YT, MODE>::Pre pre;
+        const int64_t out_i = 4 * (Q + (lane >> 2 & 3)) + (lane & 3);  // lanes 0-15: rows of the quad
+        const bool writer = lane < 16 && Q + (lane >> 2) < BR;
+        if (writer) pre = epi.prefetch(out_i);
+        float c[4] = {0.f, 0.f, 0.f, 0.f};
+        float ccA = 0.f, ccB = 0.f;  // CUDA-core sums of rows (gA, r) and (gB, r)
+        for (int64_t w = 0; w < len; w += 4) {
+            // phase 1: the A side (tile values of this lane's two rows, 4 tile slots) and the B
+            // side (bitmaps and columns of block row gid's tiles), all requested together
+            uint32_t raw[4], mpA[4], mpB[2];
+            int64_t tA[4], JA[4], JB[2];
+            bool vA[4], vB[2];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const bool rowB = q & 1;
+                const int i = (tig >> 1) + ((q >> 1) << 1);
+                const int64_t lo = rowB ? tb0 : ta0, hi = rowB ? tb1 : ta1;
+                tA[q] = lo + w + i;
+                vA[q] = tA[q] < hi;
+                raw[q] = vA[q] ? __ldg(reinterpret_cast<const uint32_t*>(bval + 16 * tA[q] + 4 * r) + (tig & 1)) : 0u;
+                mpA[q] = vA[q] ? (uint32_t)__ldg(bmap + tA[q]) : 0u;
+                JA[q] = vA[q] ? (int64_t)__ldg(bidx + tA[q]) : 0;
+            }
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                const int64_t t = tn0 + w + (tig >> 1) + 2 * q;
+                vB[q] = gid < 4 && t < tn1;
+                mpB[q] = vB[q] ? (uint32_t)__ldg(bmap + t) : 0u;
+                JB[q] = vB[q] ? (int64_t)__ldg(bidx + t) : 0;
+            }
+            // phase 2: x operands (B fragment in FP16; the sparse tiles' entries in FP32)
+            const int cb = 2 * (tig & 1);
+            uint32_t a[4], b[2];
+            float2 xs[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const bool dense = vA[q] && __popc(mpA[q]) >= tc_thr;
+                a[q] = dense ? raw[q] : 0u;
+                const uint32_t bits = (vA[q] && !dense) ? (mpA[q] >> (4 * r + cb)) & 3u : 0u;
+                xs[q] = make_float2(bits & 1u ? (float)__ldg(x + 4 * JA[q] + cb) : 0.f,
+                                    bits & 2u ? (float)__ldg(x + 4 * JA[q] + cb + 1) : 0.f);
+            }
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                b[q] = 0u;
+                if (vB[q] && __popc(mpB[q]) >= tc_thr) {
+                    const __half2 xv = __floats2half2_rn((float)__ldg(x + 4 * JB[q] + cb), (float)__ldg(x + 4 * JB[q] + cb + 1));
+                    b[q] = *reinterpret_cast<const uint32_t*>(&xv);
+                }
+            }
+            // phase 3: the sparse tiles on CUDA cores, the dense ones through the mma
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                if (a[q] == 0u && vA[q]) {
+                    const float2 av = __half22float2(*reinterpret_cast<const __half2*>(&raw[q]));
+                    const float sv = fmaf(av.y, xs[q].y, av.x * xs[q].x);
+                    if (q & 1) ccB += sv; else ccA += sv;
+                }
+            }
+            hmma_16816(c, a, b);
+        }
+        // C[4g + r][g]: g = 0 -> c[0] of lanes 4r (tig 0), g = 1 -> c[1] of lanes 16 + 4r, g = 2 ->
+        // c[2] of lanes 4r + 1, g = 3 -> c[3] of lanes 16 + 4r + 1
+        float sA = ccA + __shfl_xor_sync(FULL, ccA, 1);
+        sA += __shfl_xor_sync(FULL, sA, 2);
+        float sB = ccB + __shfl_xor_sync(FULL, ccB, 1);
+        sB += __shfl_xor_sync(FULL, sB, 2);  // group gid: rows (gA, r) and (gB, r) summed over tig
+        const int g = lane >> 2 & 3, rr = lane & 3;  // this writer lane's block row g and row rr
+        const int srcC = (g & 1 ? 16 : 0) + 4 * rr + (g >> 1);
+        const float v0 = __shfl_sync(FULL, c[0], srcC), v1 = __shfl_sync(FULL, c[1], srcC);
+        const float v2 = __shfl_sync(FULL, c[2], srcC), v3 = __shfl_sync(FULL, c[3], srcC);
+        const float cv = g == 0 ? v0 : g == 1 ? v1 : g == 2 ? v2 : v3;
+        // CUDA-core part of (g, rr): group gid' = 4 (g & 1) + rr holds it in sA (g < 2) or sB (g >= 2)
+        const int srcS = 4 * (4 * (g & 1) + rr);
+        const float vA = __shfl_sync(FULL, sA, srcS), vB = __shfl_sync(FULL, sB, srcS);
+        if (writer) epi.finish(out_i, cv + (g < 2 ? vA : vB), pre);
+    }
+}
+
 template <typename MatT, typename XT, typename YT, int MODE>
 static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArgs& ea, int64_t I0, int64_t BR,
                         int64_t long_thr, cudaStream_t s) {
@@ -680,7 +873,22 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
         return;
     }
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
-    const int tc = sizeof(MatT) == 8 ? g_tc_thr_spmv : 17;
+    const int tc = sizeof(MatT) != 4 ? g_tc_thr_spmv : 17;  // FP32: CUDA cores (no TF32, R17)
+    if (tc <= 16 && MODE != EPI_JACOBI_NORM && MODE != EPI_RES_X0) {  // tensor-core routes (L222-228)
+        const int per_sm_cap = 8;  // 256-thread CTAs: persistent grid over the rows
+        if constexpr (sizeof(MatT) == 8) {
+            const unsigned g = (unsigned)std::min<int64_t>(ceil_div((BR - I0) * 32, 256), (int64_t)num_sms() * per_sm_cap);
+            pdl_launch(k_spmv_tc64<XT, YT, MODE, 4>, dim3(std::max(g, 1u)), dim3(256), 0, s, I0, BR, A->blc_ptr,
+                       A->blc_idx, A->blc_map, (const double*)A->blc_val, (const XT*)x, epi, long_thr, tc);
+            return;
+        } else if constexpr (sizeof(MatT) == 2) {
+            const unsigned g =
+                (unsigned)std::min<int64_t>(ceil_div(ceil_div(BR - I0, 4) * 32, 256), (int64_t)num_sms() * per_sm_cap);
+            pdl_launch(k_spmv_tc16<XT, YT, MODE>, dim3(std::max(g, 1u)), dim3(256), 0, s, I0, BR, A->blc_ptr,
+                       A->blc_idx, A->blc_map, (const __half*)A->blc_val, (const XT*)x, epi, long_thr, tc);
+            return;
+        }
+    }
     static const int persist = [] { const char* e = getenv("AMGT_SPMV_PERSIST"); return e ? atoi(e) : 1; }();
     auto go = [&](auto kern) {
         unsigned g = blocks;
@@ -696,10 +904,6 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
                    (const MatT*)A->blc_val, (const XT*)x, epi, long_thr, tc);
     };
     if constexpr (sizeof(MatT) == 8) {
-        if (tc <= 16) {  // per-tile tensor-core route (separate instantiation)
-            go(k_spmv_rows<MatT, XT, YT, MODE, 2, 1, true>);
-            return;
-        }
         switch (spmv_variant()) {  // tuning knob AMGT_SPMV_VARIANT: tiles per iteration x min blocks/SM
             case 1: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 5>); break;
             case 2: go(k_spmv_rows<MatT, XT, YT, MODE, 4, 6>); break;

@@ -628,6 +628,7 @@ constexpr int JAC = 1, RES = 2, ACC = 3;
 
 // AMGT_ZERO_GUESS_FUSED=0: coarse levels run the zero-guess sweep (k_jacobi0) and the residual
 // as two kernels (measurement knob; the results are bit-identical either way)
+constexpr int64_t kZeroGuessFusedMaxBR = 131072;
 static bool zero_guess_fused() {
     static int v = -1;
     if (v < 0) {
@@ -645,7 +646,10 @@ static amgt_status down_level(amgt_hierarchy* H, int k, const void* b0, void** x
     amgt_level& L = H->L[k];
     const void* bk = k == 0 ? b0 : L.b;
     int i0 = 0;
-    if (k > 0 && H->o.nu1 == 1 && L.vprec == AMGT_FP32 && L.A.prec != AMGT_FP64 && zero_guess_fused()) {
+    // (large levels excluded: forming x1 at every gathered column doubles the gathered vector loads;
+    // config-3 level 2, 524,288 block rows: 274 us fused vs ~175 us for k_jacobi0 + the residual)
+    if (k > 0 && H->o.nu1 == 1 && L.vprec == AMGT_FP32 && L.A.prec != AMGT_FP64 && zero_guess_fused() &&
+        L.A.blc_row <= kZeroGuessFusedMaxBR && !(L.A.prec == AMGT_FP16 && g_tc_thr_spmv <= 16)) {
         // lines 2-3 from the zero guess in one pass: r = b - A x1, x1 = w D^-1 b formed on the
         // fly (EPI_RES_X0); two of Alg. 2's SpMV operations (the sweep's is A 0 = 0)
         EpiArgs ea{EPI_RES_X0, bk, L.dinv, nullptr, H->o.omega, 0, -1};

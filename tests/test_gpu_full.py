@@ -52,3 +52,47 @@ def test_cfg3_full():
     live = res_o[1:] / res_o[0] > 1e-10
     assert np.all(np.abs(rho[live] - rho_o[live]) <= 0.01 * rho_o[live]), (rho, rho_o)
     H.close()
+
+
+def _block_rows(M, I0, I1):
+    """Block rows [I0, I1) of a device mBSR as host arrays (pointers rebased to 0)."""
+    ptr = M.blc_ptr[I0:I1 + 1].cpu().numpy()
+    t0, t1 = int(ptr[0]), int(ptr[-1])
+    return (ptr - t0, M.blc_idx[t0:t1].cpu().numpy(), (M.blc_map[t0:t1].to(torch.int32) & 0xFFFF).cpu().numpy()
+            .astype(np.uint16))
+
+
+def test_cfg5_full_g1_shardwise():
+    """Config 5 at full size on one GPU (7-point 512^3: 134,217,728 rows, 937,951,232 nonzeros;
+    the G = 1 point of the strong-scaling runs): the CSR->mBSR conversion of A_1 and the A_1 P_1
+    SpGEMM of the setup, structure bit-exact against the oracle run shard-wise (the
+    full 512^3 oracle would need ~22 GB of host CSR) on the first, a middle and the last 8-plane
+    z-slab, plus the exact total tile counts of SURVEY 8(a) (closed forms P3)."""
+    import paper_conf_sc_luzwflcy0c024_b200 as amgt
+    N, planes = 512, 8
+    plane = N * N
+    A = gen.laplacian_7pt(N, device="cuda")
+    assert A.nnz == 937_951_232
+    M = amgt.from_csr(A)
+    del A
+    torch.cuda.empty_cache()
+    assert M.blc_num == 234_094_592 == N * N * (7 * N // 4 - 3)
+    P = amgt.from_csr(gen.aggregation_P((N, N, N), 0.5, device="cuda"))
+    AP = amgt.spgemm_symbolic(M, P)
+    assert AP.blc_num == 133_431_296 == N * N * (N - 3)  # AP tiles = N^2 (N - 3)
+    for z0 in (0, N // 2 - planes // 2, N - planes):
+        r0, r1 = z0 * plane, (z0 + planes) * plane
+        As = oracle.as_csr(gen.laplacian_7pt(N, rows=(r0, r1)))  # global columns
+        Ms = oracle.csr_to_mbsr(As)
+        bp, bi, bm = _block_rows(M, r0 // 4, r1 // 4)
+        assert np.array_equal(bp, Ms.blc_ptr) and np.array_equal(bi, Ms.blc_idx) and np.array_equal(bm, Ms.blc_map)
+        # A P of the slab: the P rows its columns reach (one plane either side), global coarse columns
+        e0, e1 = max(0, r0 - plane), min(N ** 3, r1 + plane)
+        Pe = oracle.as_csr(gen.aggregation_P((N, N, N), 0.5, rows=(e0, e1)))
+        Ash = oracle.Csr(As.m, e1 - e0, As.row_ptr, (As.col.astype(np.int64) - e0).astype(np.int32), As.val)
+        APs = oracle.csr_to_mbsr(oracle.spgemm(Ash, Pe))
+        bp, bi, bm = _block_rows(AP, r0 // 4, r1 // 4)
+        assert np.array_equal(bp, APs.blc_ptr) and np.array_equal(bi, APs.blc_idx) and np.array_equal(bm, APs.blc_map)
+    AP.free()
+    P.free()
+    M.free()

@@ -65,19 +65,68 @@ def test_spmv_long_rows_plan():
     check_fp64_entrywise(y[:A.m], oracle.spmv(Ao, x), oracle.spmv_abs(Ao, x))
 
 
-@pytest.mark.parametrize("thr", [0, 4, 10])
-def test_spmv_tensor_core_route(thr):
-    """Per-tile DMMA route (popcount >= thr) gives the same result within FP64 tolerance."""
+@pytest.mark.parametrize("thr", [0, 4, 10, 16])
+@pytest.mark.parametrize("name,mk", MATS, ids=[m[0] for m in MATS])
+def test_spmv_tensor_core_route(name, mk, thr):
+    """Per-tile tensor-core route (R10; DMMA m8n8k4 with [A_t; A_t+1] fragments, L222-228): tiles
+    with popcount >= thr through the mma, the rest on CUDA cores, long rows through the chunk
+    kernel.  FP64 within 1e-12 scaled; integer data exact; every fused epilogue equals the
+    CUDA-core route's within FP64 rounding."""
+    amgt = _amgt()
+    A = mk()
+    Ao = oracle.as_csr(A)
+    try:
+        amgt.set_tc_threshold(17, thr)
+        M = amgt.from_csr(A).analyze()
+        x = gen.uniform_vector(A.n, 3).numpy()
+        y = amgt.spmv(M, torch.from_numpy(x).cuda()).cpu().numpy()
+        assert np.all(y[A.m:] == 0)
+        check_fp64_entrywise(y[:A.m], oracle.spmv(Ao, x), oracle.spmv_abs(Ao, x))
+        xi = gen.integer_vector(A.n, 12).numpy()
+        Ai = oracle.Csr(Ao.m, Ao.n, Ao.row_ptr, Ao.col, np.round(Ao.val * 8))
+        Mi = amgt.from_csr(gen.CSR(A.m, A.n, A.row_ptr, A.col, torch.from_numpy(Ai.val))).analyze()
+        yi = amgt.spmv(Mi, torch.from_numpy(xi).cuda()).cpu().numpy()
+        assert np.array_equal(yi[:A.m], oracle.spmv(Ai, xi))
+        if A.m == A.n:  # fused epilogues against the plain result
+            n4 = 4 * M.blc_row
+            xv = torch.zeros(n4, dtype=torch.float64, device="cuda")
+            xv[:A.m] = torch.from_numpy(x[:A.m])
+            b = torch.from_numpy(gen.uniform_vector(n4, 5).numpy()).cuda()
+            d = torch.from_numpy(gen.uniform_vector(n4, 6, 0.5, 1.0).numpy()).cuda()
+            t = torch.from_numpy(y).cuda()
+            for mode in ("jacobi", "residual", "accum"):
+                out = torch.from_numpy(gen.uniform_vector(n4, 7).numpy()).cuda()
+                ref = {"jacobi": xv + (2.0 / 3.0) * d * (b - t), "residual": b - t, "accum": out + t}[mode]
+                amgt.spmv_fused(M, xv, out, mode, b=b, dinv=d)
+                scale = torch.from_numpy(oracle.spmv_abs(Ao, np.abs(x)))
+                err = (out - ref).abs().cpu()[:A.m]
+                assert torch.all(err <= 1e-12 * (scale + ref.abs().cpu()[:A.m] + 1)), (mode, float(err.max()))
+    finally:
+        amgt.set_tc_threshold(17, 17)
+
+
+@pytest.mark.parametrize("thr", [0, 10])
+def test_spmv_fp16_tensor_core_route(thr):
+    """FP16 levels on HMMA m16n8k16 (FP16 operands, x rounded to FP16, FP32 accumulation, R18): 16
+    tile products per instruction from four block rows; exact on small-integer data, within the
+    FP16-level tolerance (5e-3 in the 2-norm) on random data."""
     amgt = _amgt()
     try:
-        amgt.set_tc_threshold(10, thr)
-        for mk in (lambda: gen.laplacian_27pt(12), lambda: gen.irregular_block_sparse(1 << 10)):
+        amgt.set_tc_threshold(17, thr)
+        for mk in (lambda: gen.laplacian_27pt(12), lambda: gen.irregular_block_sparse(1 << 11),
+                   lambda: gen.random_csr(333, 333, 0.03, 9, empty_rows=20)):
             A = mk()
             Ao = oracle.as_csr(A)
-            M = amgt.from_csr(A)
-            x = gen.uniform_vector(A.n, 3).numpy()
-            y = amgt.spmv(M, torch.from_numpy(x).cuda()).cpu().numpy()
-            check_fp64_entrywise(y[:A.m], oracle.spmv(Ao, x), oracle.spmv_abs(Ao, x))
+            M = amgt.from_csr(A, prec="f16").analyze()
+            x = gen.uniform_vector(A.n, 4).numpy()
+            y = torch.empty(4 * M.blc_row, dtype=torch.float32, device="cuda")
+            amgt.spmv(M, torch.from_numpy(x).float().cuda(), y)
+            assert rel_2(y.double().cpu().numpy()[:A.m], oracle.spmv(Ao, x)) <= 5e-3
+            Ai = oracle.Csr(Ao.m, Ao.n, Ao.row_ptr, Ao.col, np.round(Ao.val * 8))
+            Mi = amgt.from_csr(gen.CSR(A.m, A.n, A.row_ptr, A.col, torch.from_numpy(Ai.val)), prec="f16").analyze()
+            xi = gen.integer_vector(A.n, 12).numpy()
+            amgt.spmv(Mi, torch.from_numpy(xi).float().cuda(), y)
+            assert np.array_equal(y.double().cpu().numpy()[:A.m], oracle.spmv(Ai, xi))
     finally:
         amgt.set_tc_threshold(17, 17)
 
@@ -168,3 +217,30 @@ def test_spmv_jacobi_res(dt):
     amgt.spmv_fused(M, x, y2, "jacobi", b=b, dinv=d)
     amgt.spmv_fused(M, x, r2, "residual", b=b)
     assert torch.equal(y, y2) and torch.equal(r, r2)
+
+
+@pytest.mark.parametrize("prec", [("f64",) * 4, ("f64", "f32", "f16", "f16")])
+def test_vcycle_with_tensor_core_spmv(prec):
+    """The V-cycle with every SpMV tile on the tensor-core routes (threshold 0): FP64 residual
+    history within 1e-9 of the oracle, mixed precision within 1% per cycle, same call count."""
+    amgt = _amgt()
+    N, nlev = 24, 4
+    A = gen.laplacian_27pt(N)
+    PR = gen.aggregation_hierarchy((N, N, N), nlev)
+    b = gen.uniform_vector(A.m, 3)
+    try:
+        amgt.set_tc_threshold(17, 0)
+        H = amgt.Hierarchy(amgt.from_csr(A), [amgt.from_csr(P) for P, _ in PR], level_prec=prec)
+        x = torch.zeros(A.m, dtype=torch.float64, device="cuda")
+        res, calls = H.vcycle(b.cuda(), x, 6)
+        H.close()
+    finally:
+        amgt.set_tc_threshold(17, 17)
+    _, res_o, calls_o = oracle.vcycle(oracle.build_hierarchy(A, PR), PR, b.numpy(), ncycles=6)
+    assert calls == calls_o
+    if prec[1] == "f64":
+        np.testing.assert_allclose(res, res_o, rtol=1e-9)
+    else:
+        res, res_o = np.array(res), np.array(res_o)
+        rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
+        assert np.all(np.abs(rho - rho_o) <= 0.01 * rho_o), (rho, rho_o)
