@@ -133,17 +133,29 @@ __global__ void __launch_bounds__(512) k_csr2mbsr_long(int64_t m, int64_t n, int
 
 // FILL = false: count tiles per block row into cnt[I] and validate the CSR.
 // FILL = true : write blc_idx / blc_map / blc_val at offsets bptr[I].
+// Fill pass: the warp's 32 CSR rows are one contiguous range of the column / value arrays; when it
+// holds at most CONV_STAGE entries the warp first copies it to shared memory with coalesced loads,
+// so the lanes' per-row merges read shared memory instead of issuing dependent scattered global
+// loads (config-3 A_1 fill: 8.3 -> 7.2 ms of cold kernel time).  The count pass reads only the
+// columns and keeps the unstaged loads and the higher occupancy.
+constexpr int CONV_WARPS = 4;     // 128-thread CTAs
+constexpr int CONV_STAGE = 1024;  // entries per warp (27-point: 32 rows x 27 = 864)
+template <bool FILL>
+constexpr int conv_smem_bytes() { return FILL ? CONV_WARPS * CONV_STAGE * 12 : 0; }
+
 template <bool FILL, typename T>
-__global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t nnz, int64_t BR, int64_t coff,
+__global__ void __launch_bounds__(128) k_csr2mbsr(int64_t m, int64_t n, int64_t nnz, int64_t BR, int64_t coff,
                                                   const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
                                                   const double* __restrict__ v, int64_t* __restrict__ cnt,
                                                   const int64_t* __restrict__ bptr, int32_t* __restrict__ bidx,
                                                   uint16_t* __restrict__ bmap, T* __restrict__ bval,
                                                   uint32_t* __restrict__ flag, int32_t* __restrict__ longl,
                                                   unsigned long long* __restrict__ nlong) {
-    const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
-    const int64_t I = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 8 + g;
-    if ((((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 8 >= BR) return;  // whole warp idle
+    extern __shared__ __align__(16) unsigned char conv_sm[];
+    const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3, wib = threadIdx.x >> 5;
+    const int64_t W = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t I = W * 8 + g;
+    if (W * 8 >= BR) return;  // whole warp idle
     const bool active = I < BR;
     const int64_t row = 4 * I + r;
     int64_t p = 0, e = 0;
@@ -166,11 +178,32 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
             e = p;
         }
     }
+    // stage the warp's entries [wb, we) (rows 32 W .. 32 W + 31); every lane's [p, e) must lie
+    // inside (true for a valid CSR; a malformed one is read from global memory and flagged)
+    double* sv = reinterpret_cast<double*>(conv_sm) + (int64_t)wib * CONV_STAGE;
+    int32_t* sci = reinterpret_cast<int32_t*>(conv_sm + (size_t)CONV_WARPS * CONV_STAGE * 8) + (int64_t)wib * CONV_STAGE;
+    int64_t wb = 0, we = 0;
+    if (FILL && lane == 0) {
+        wb = rp[min(32 * W, m)];
+        we = rp[min(32 * W + 32, m)];
+    }
+    wb = __shfl_sync(0xffffffffu, wb, 0);
+    we = __shfl_sync(0xffffffffu, we, 0);
+    const bool staged = FILL && __all_sync(0xffffffffu, we - wb >= 0 && we - wb <= CONV_STAGE && wb >= 0 && we <= nnz &&
+                                                             (p >= e || (p >= wb && e <= we)));
+    if (staged) {
+        const int64_t ne = we - wb;
+        for (int64_t q = lane; q < ne; q += 32) sci[q] = __ldg(ci + wb + q);
+        for (int64_t q = lane; q < ne; q += 32) sv[q] = __ldg(v + wb + q);
+        __syncwarp();
+    }
+    auto ld_ci = [&](int64_t q) { return staged ? sci[q - wb] : __ldg(ci + q); };
+    auto ld_v = [&](int64_t q) { return staged ? sv[q - wb] : __ldg(v + q); };
     int64_t t = (FILL && active) ? bptr[I] : 0;
     int64_t c = 0;
     int32_t prev = -1;
     for (;;) {
-        const int32_t J = (p < e) ? (int32_t)((__ldg(ci + p) - coff) >> 2) : INT_MAX;
+        const int32_t J = (p < e) ? (int32_t)((ld_ci(p) - coff) >> 2) : INT_MAX;
         int32_t Jm = min(J, __shfl_xor_sync(0xffffffffu, J, 1));
         Jm = min(Jm, __shfl_xor_sync(0xffffffffu, Jm, 2));
         if (!__any_sync(0xffffffffu, Jm != INT_MAX)) break;
@@ -178,14 +211,14 @@ __global__ void __launch_bounds__(256) k_csr2mbsr(int64_t m, int64_t n, int64_t 
         uint32_t nib = 0;
         if (Jm != INT_MAX) {
             while (p < e) {
-                const int32_t col = (int32_t)(__ldg(ci + p) - coff);
+                const int32_t col = (int32_t)(ld_ci(p) - coff);
                 if ((col >> 2) != Jm) break;
                 if (!FILL) {
                     if (col <= prev || col >= n || col < 0) bad = 1;
                     prev = col;
                 } else {
                     const int cc = col & 3;
-                    const double x = __ldg(v + p);
+                    const double x = ld_v(p);
                     rv[0] = cc == 0 ? x : rv[0];
                     rv[1] = cc == 1 ? x : rv[1];
                     rv[2] = cc == 2 ? x : rv[2];
@@ -437,11 +470,18 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     };
     amgt_mbsr M{};
     const double bytes_in = nnz * 12.0 + (m + 1) * 8.0;
-    const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 256);
+    const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 32 * CONV_WARPS);
+    static bool attr_set = false;
+    if (!attr_set) {  // > 48 KB of dynamic shared memory for the staged fill
+        cudaFuncSetAttribute(k_csr2mbsr<true, double>, cudaFuncAttributeMaxDynamicSharedMemorySize, conv_smem_bytes<true>());
+        cudaFuncSetAttribute(k_csr2mbsr<true, float>, cudaFuncAttributeMaxDynamicSharedMemorySize, conv_smem_bytes<true>());
+        cudaFuncSetAttribute(k_csr2mbsr<true, __half>, cudaFuncAttributeMaxDynamicSharedMemorySize, conv_smem_bytes<true>());
+        attr_set = true;
+    }
     {
         TimerScope ts(TC_CSR2MBSR, bytes_in, s);
         if (BR > 0) {
-            k_csr2mbsr<false, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, cnt.p, nullptr, nullptr,
+            k_csr2mbsr<false, double><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<false>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, cnt.p, nullptr, nullptr,
                                                              nullptr, nullptr, flag.p, longl.p, nlong.p);
             AMGT_LAUNCHED();
             AMGT_TRY(launch_long(k_csr2mbsr_long<false, double>, cnt.p, nullptr, nullptr, nullptr, (double*)nullptr));
@@ -487,7 +527,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
         if (BR > 0) {
             switch (prec) {
                 case AMGT_FP64:
-                    k_csr2mbsr<true, double><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
+                    k_csr2mbsr<true, double><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<true>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                     M.blc_idx, M.blc_map, (double*)M.blc_val, flag.p,
                                                                     longl.p, nlong.p);
                     AMGT_LAUNCHED();
@@ -495,7 +535,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
                                          (double*)M.blc_val));
                     break;
                 case AMGT_FP32:
-                    k_csr2mbsr<true, float><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
+                    k_csr2mbsr<true, float><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<true>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                    M.blc_idx, M.blc_map, (float*)M.blc_val, flag.p,
                                                                    longl.p, nlong.p);
                     AMGT_LAUNCHED();
@@ -503,7 +543,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
                                          (float*)M.blc_val));
                     break;
                 default:
-                    k_csr2mbsr<true, __half><<<blocks, 256, 0, s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
+                    k_csr2mbsr<true, __half><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<true>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                     M.blc_idx, M.blc_map, (__half*)M.blc_val, flag.p,
                                                                     longl.p, nlong.p);
                     AMGT_LAUNCHED();

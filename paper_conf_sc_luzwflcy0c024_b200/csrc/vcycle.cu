@@ -359,6 +359,33 @@ __global__ void __launch_bounds__(256) k_gauss_jordan(int64_t n, double* __restr
     }
 }
 
+// The same Gauss-Jordan for small n (<= GJ_SMEM_N) in ONE CTA with the matrix in shared memory
+// (block barriers instead of grid barriers: the config-3 coarsest level, n = 64, 269 -> ~20 us).
+constexpr int GJ_SMEM_N = 128;
+__global__ void __launch_bounds__(512) k_gauss_jordan_smem(int n, double* __restrict__ a, uint32_t* __restrict__ flag) {
+    extern __shared__ double gsm[];
+    double* m = gsm;
+    double* rb = gsm + n * n;
+    double* cb = rb + n;
+    for (int e = threadIdx.x; e < n * n; e += blockDim.x) m[e] = a[e];
+    __syncthreads();
+    for (int k = 0; k < n; ++k) {
+        const double piv = m[k * n + k];
+        if (threadIdx.x == 0 && !(piv > 0.0)) atomicOr(flag, FLAG_SPD);
+        for (int j = threadIdx.x; j < n; j += blockDim.x) {
+            rb[j] = (j == k ? 1.0 : m[k * n + j]) / piv;
+            cb[j] = m[j * n + k];
+        }
+        __syncthreads();
+        for (int e = threadIdx.x; e < n * n; e += blockDim.x) {
+            const int i = e / n, j = e - i * n;
+            m[e] = i == k ? rb[j] : (j == k ? 0.0 : m[e]) - cb[i] * rb[j];
+        }
+        __syncthreads();
+    }
+    for (int e = threadIdx.x; e < n * n; e += blockDim.x) a[e] = m[e];
+}
+
 // Ainv = A_M^-1 on the device (dense scatter + Gauss-Jordan); FLAG_SPD into dflag.
 static amgt_status device_coarse_inverse(const amgt_mbsr& C, double* Ainv, uint32_t* dflag, Alloc& a) {
     cudaStream_t s = a.s;
@@ -380,6 +407,18 @@ static amgt_status device_coarse_inverse(const amgt_mbsr& C, double* Ainv, uint3
     }
     AMGT_LAUNCHED();
     if (n == 0) return AMGT_OK;
+    if (n <= GJ_SMEM_N) {
+        const size_t sm = (size_t)(n * n + 2 * n) * sizeof(double);
+        static bool attr = false;
+        if (!attr) {
+            AMGT_CUDA(cudaFuncSetAttribute(k_gauss_jordan_smem, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           (int)((GJ_SMEM_N * GJ_SMEM_N + 2 * GJ_SMEM_N) * sizeof(double))));
+            attr = true;
+        }
+        k_gauss_jordan_smem<<<1, 512, sm, s>>>((int)n, Ainv, dflag);
+        AMGT_LAUNCHED();
+        return AMGT_OK;
+    }
     Scratch<double> buf;
     AMGT_TRY(buf.init(a, 2 * n));
     static int per_sm = -1;
