@@ -38,7 +38,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "SpMV GB/s, SpGEMM GFLOP/s (mBSR, 1–8 B200); AMG setup+solve s"
 LEVEL_PREC = ("f64", "f32", "f16", "f16", "f16", "f16", "f16")
-AGG_ROWS = 32768  # distributed path: levels with <= 32^3 global rows agglomerated on every rank
+AGG_ROWS = 262144  # distributed path: levels with <= 64^3 global rows agglomerated on every rank (DESIGN 9)
 FLUSH_BYTES = 512 << 20  # > 2x the 126 MB L2
 
 
@@ -591,14 +591,18 @@ def run_dist(args, rank, world, local):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     gc.collect()
     gc.disable()
+    host_ms = []
     with ClockSampler(local) as clk:
         e0.record(stream)
         for _ in range(args.steps):
+            t_h = time.perf_counter()
             step()
+            host_ms.append(round((time.perf_counter() - t_h) * 1e3, 2))
         e1.record(stream)
         dist.barrier()
         torch.cuda.synchronize()
     gc.enable()
+    print(f"[bench] rank {rank} host ms per timed step (enqueue + host syncs): {host_ms}", file=sys.stderr)
     t = torch.tensor([e0.elapsed_time(e1) / args.steps], dtype=torch.float64, device="cuda")
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_step = float(t.item())
@@ -685,7 +689,7 @@ def run_dist(args, rank, world, local):
                          "peak_source": peak_kind, "bytes_per_launch": sp_bytes,
                          "avg_launch_us": round(spmv_ms * 1e3, 2), "traffic": None},
             "components": {"setup_ms_rank0": round(setup_ms, 3), "bytes_per_step": bytes_job,
-                           "final_rel_residual": res[-1] / res[0]},
+                           "final_rel_residual": res[-1] / res[0], "host_ms_per_step_rank0": host_ms},
             "e2e": {"value": round(bytes_job / (e2e_ms * 1e-3) / 1e9, 2), "unit": "GB/s", "ms_per_step": round(e2e_ms, 3),
                     "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
                     "copies": "each rank uploads its slab inputs from pinned host memory every step (copy stream, "

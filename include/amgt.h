@@ -166,7 +166,9 @@ amgt_status amgt_spgemm_symbolic(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
  * quadrants, L157-171; FP16: HMMA m16n8k16 with FP32 accumulation, 8 tile products per
  * instruction); otherwise the thread-level CUDA-core route.  FP32 always takes the
  * CUDA-core route (no TF32, R17).  C must come from amgt_spgemm_symbolic(A, B).
- * Values: deterministic.
+ * Values: deterministic for C block rows with at most 32 tiles (fixed lane order); longer rows
+ * accumulate tiles that receive three or more products with FP atomics and are reproducible up
+ * to rounding only (exact on integer / dyadic data).
  */
 amgt_status amgt_spgemm_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, void* stream);
 
