@@ -8,6 +8,7 @@
 // sequential in its row.  Two passes (count, fill) around a device prefix sum; one
 // host sync to size the tile arrays.
 #include <climits>
+#include <cstdlib>
 
 #include "common.cuh"
 
@@ -138,6 +139,15 @@ __global__ void __launch_bounds__(512) k_csr2mbsr_long(int64_t m, int64_t n, int
 // so the lanes' per-row merges read shared memory instead of issuing dependent scattered global
 // loads (config-3 A_1 fill: 8.3 -> 7.2 ms of cold kernel time).  The count pass reads only the
 // columns and keeps the unstaged loads and the higher occupancy.
+// AMGT_CONV_STAGE=0: the fill pass without the shared-memory staging (measurement knob)
+static bool conv_stage() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_CONV_STAGE");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
 constexpr int CONV_WARPS = 4;     // 128-thread CTAs
 constexpr int CONV_STAGE = 1024;  // entries per warp (27-point: 32 rows x 27 = 864)
 template <bool FILL>
@@ -150,7 +160,7 @@ __global__ void __launch_bounds__(128) k_csr2mbsr(int64_t m, int64_t n, int64_t 
                                                   const int64_t* __restrict__ bptr, int32_t* __restrict__ bidx,
                                                   uint16_t* __restrict__ bmap, T* __restrict__ bval,
                                                   uint32_t* __restrict__ flag, int32_t* __restrict__ longl,
-                                                  unsigned long long* __restrict__ nlong) {
+                                                  unsigned long long* __restrict__ nlong, bool stage_ok) {
     extern __shared__ __align__(16) unsigned char conv_sm[];
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3, wib = threadIdx.x >> 5;
     const int64_t W = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -189,7 +199,7 @@ __global__ void __launch_bounds__(128) k_csr2mbsr(int64_t m, int64_t n, int64_t 
     }
     wb = __shfl_sync(0xffffffffu, wb, 0);
     we = __shfl_sync(0xffffffffu, we, 0);
-    const bool staged = FILL && __all_sync(0xffffffffu, we - wb >= 0 && we - wb <= CONV_STAGE && wb >= 0 && we <= nnz &&
+    const bool staged = FILL && stage_ok && __all_sync(0xffffffffu, we - wb >= 0 && we - wb <= CONV_STAGE && wb >= 0 && we <= nnz &&
                                                              (p >= e || (p >= wb && e <= we)));
     if (staged) {
         const int64_t ne = we - wb;
@@ -482,7 +492,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
         TimerScope ts(TC_CSR2MBSR, bytes_in, s);
         if (BR > 0) {
             k_csr2mbsr<false, double><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<false>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, cnt.p, nullptr, nullptr,
-                                                             nullptr, nullptr, flag.p, longl.p, nlong.p);
+                                                             nullptr, nullptr, flag.p, longl.p, nlong.p, false);
             AMGT_LAUNCHED();
             AMGT_TRY(launch_long(k_csr2mbsr_long<false, double>, cnt.p, nullptr, nullptr, nullptr, (double*)nullptr));
         }
@@ -529,7 +539,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
                 case AMGT_FP64:
                     k_csr2mbsr<true, double><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<true>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                     M.blc_idx, M.blc_map, (double*)M.blc_val, flag.p,
-                                                                    longl.p, nlong.p);
+                                                                    longl.p, nlong.p, conv_stage());
                     AMGT_LAUNCHED();
                     AMGT_TRY(launch_long(k_csr2mbsr_long<true, double>, nullptr, M.blc_ptr, M.blc_idx, M.blc_map,
                                          (double*)M.blc_val));
@@ -537,7 +547,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
                 case AMGT_FP32:
                     k_csr2mbsr<true, float><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<true>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                    M.blc_idx, M.blc_map, (float*)M.blc_val, flag.p,
-                                                                   longl.p, nlong.p);
+                                                                   longl.p, nlong.p, conv_stage());
                     AMGT_LAUNCHED();
                     AMGT_TRY(launch_long(k_csr2mbsr_long<true, float>, nullptr, M.blc_ptr, M.blc_idx, M.blc_map,
                                          (float*)M.blc_val));
@@ -545,7 +555,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
                 default:
                     k_csr2mbsr<true, __half><<<blocks, 32 * CONV_WARPS, conv_smem_bytes<true>(), s>>>(m, n, nnz, BR, coff, rp, ci, v, nullptr, M.blc_ptr,
                                                                     M.blc_idx, M.blc_map, (__half*)M.blc_val, flag.p,
-                                                                    longl.p, nlong.p);
+                                                                    longl.p, nlong.p, conv_stage());
                     AMGT_LAUNCHED();
                     AMGT_TRY(launch_long(k_csr2mbsr_long<true, __half>, nullptr, M.blc_ptr, M.blc_idx, M.blc_map,
                                          (__half*)M.blc_val));

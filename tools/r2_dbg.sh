@@ -1,3 +1,4 @@
-cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/r2
-timeout 900 python -m pytest tests/test_gpu_convert.py tests/test_gpu_spgemm.py tests/test_gpu_pmis.py -q -m gpu -x > gpurun_out/r2/conv_tests.log 2>&1; echo "rc=$?" >> gpurun_out/r2/conv_tests.log
-timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --nvtx --nvtx-include 'setup/' --csv --log-file gpurun_out/r2/setup_cfg3_launches_c.csv python tools/setup_kernels.py cfg3 > gpurun_out/r2/setup_cfg3.log 2>&1
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/r2d
+timeout 900 python tools/dist_overhead.py --n 512 --cycles 2 --agg-rows 262144 --G 8 > gpurun_out/r2d/g8_a.jsonl 2> gpurun_out/r2d/g8_a.err
+AMGT_CONV_STAGE=0 timeout 900 python tools/dist_overhead.py --n 512 --cycles 2 --agg-rows 262144 --G 8 > gpurun_out/r2d/g8_nostage.jsonl 2> gpurun_out/r2d/g8_nostage.err
+CUDA_LAUNCH_BLOCKING=1 timeout 900 python tools/dist_overhead.py --n 512 --cycles 2 --agg-rows 262144 --G 8 > gpurun_out/r2d/g8_block.jsonl 2> gpurun_out/r2d/g8_block.err

@@ -11,3 +11,5 @@ run var3 AMGT_SPMV_VARIANT=3
 run nopdl AMGT_PDL=0
 run persist0 AMGT_SPMV_PERSIST=0
 run persist2 AMGT_SPMV_PERSIST=2
+timeout 1500 python tools/dist_overhead.py --n 512 --cycles 10 --agg-rows 262144 > gpurun_out/r2k/dist_overhead_512.jsonl 2> gpurun_out/r2k/dist_overhead_512.err
+for i in $(seq 1 12); do timeout 300 python bench.py --force-dist --config cfg2 --steps 10 --warmup 3 --no-cfg4 > gpurun_out/r2k/forced_cfg2_$i.json 2> gpurun_out/r2k/forced_cfg2_$i.err; done
