@@ -255,4 +255,11 @@ extern int g_tc_thr_spmv;
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 int num_sms();
 
+// Opt a kernel into `bytes` of dynamic shared memory.  The attribute is process-wide while the
+// loopback ranks launch from several host threads with different sizes, so it only ever rises
+// (under a lock): a launch never finds it lowered below what its own call raised it to.
+cudaError_t dyn_smem_optin(const void* kern, size_t bytes);
+template <typename K>
+inline cudaError_t dyn_smem(K* kern, size_t bytes) { return dyn_smem_optin((const void*)kern, bytes); }
+
 }  // namespace amgt

@@ -472,7 +472,7 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     Scratch<uint32_t> lws;
     if (!lsmem) AMGT_TRY(lws.init(a, (size_t)LG * 2 * W));
     auto launch_long = [&](auto kern, int64_t* cntp, const int64_t* bp, int32_t* bi, uint16_t* bmp, auto* bv) -> amgt_status {
-        if (lsmem) AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsm));
+        if (lsmem) AMGT_CUDA(dyn_smem(kern, lsm));
         kern<<<LG, 512, lsmem ? lsm : 0, s>>>(m, n, coff, rp, ci, v, longl.p, nlong.p, W, lsmem ? nullptr : lws.p, cntp,
                                                bp, bi, bmp, bv, flag.p);
         AMGT_LAUNCHED();
@@ -481,13 +481,10 @@ amgt_status csr_to_mbsr_impl(int64_t m, int64_t n, int64_t nnz, const int64_t* r
     amgt_mbsr M{};
     const double bytes_in = nnz * 12.0 + (m + 1) * 8.0;
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR, 8) * 32, 32 * CONV_WARPS);
-    static bool attr_set = false;
-    if (!attr_set) {  // > 48 KB of dynamic shared memory for the staged fill
-        cudaFuncSetAttribute(k_csr2mbsr<true, double>, cudaFuncAttributeMaxDynamicSharedMemorySize, conv_smem_bytes<true>());
-        cudaFuncSetAttribute(k_csr2mbsr<true, float>, cudaFuncAttributeMaxDynamicSharedMemorySize, conv_smem_bytes<true>());
-        cudaFuncSetAttribute(k_csr2mbsr<true, __half>, cudaFuncAttributeMaxDynamicSharedMemorySize, conv_smem_bytes<true>());
-        attr_set = true;
-    }
+    // > 48 KB of dynamic shared memory for the staged fill
+    AMGT_CUDA(dyn_smem(k_csr2mbsr<true, double>, conv_smem_bytes<true>()));
+    AMGT_CUDA(dyn_smem(k_csr2mbsr<true, float>, conv_smem_bytes<true>()));
+    AMGT_CUDA(dyn_smem(k_csr2mbsr<true, __half>, conv_smem_bytes<true>()));
     {
         TimerScope ts(TC_CSR2MBSR, bytes_in, s);
         if (BR > 0) {

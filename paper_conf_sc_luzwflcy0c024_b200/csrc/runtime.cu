@@ -4,6 +4,7 @@
 #include <cstdlib>
 #include <cstdarg>
 #include <mutex>
+#include <unordered_map>
 #include <vector>
 
 #include "common.cuh"
@@ -105,6 +106,19 @@ int num_sms() {
         if (n <= 0) n = 148;
     }
     return n;
+}
+
+cudaError_t dyn_smem_optin(const void* kern, size_t bytes) {
+    // (no shortcut at <= 48 KB: the default limit counts the kernel's static shared memory too)
+    if (bytes == 0) return cudaSuccess;
+    static std::mutex mu;
+    static std::unordered_map<const void*, size_t> cur;
+    std::lock_guard<std::mutex> g(mu);
+    size_t& c = cur[kern];
+    if (c >= bytes) return cudaSuccess;
+    const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    if (e == cudaSuccess) c = bytes;
+    return e;
 }
 
 // Tensor-core routing thresholds on POPCOUNT(mapA).  The paper uses 10 (L157); north_star asks

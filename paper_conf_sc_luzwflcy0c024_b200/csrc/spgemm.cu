@@ -1942,7 +1942,7 @@ static amgt_status launch_warp_bin(int64_t n, const int32_t* rows, const SymCtx&
     if (n == 0) return AMGT_OK;
     const size_t sm = (size_t)8 * 2 * (1 << LOGS) * sizeof(int);
     auto kern = k_sym_warp<LOGS, STEP>;
-    if (sm > 48 * 1024) AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    AMGT_CUDA(dyn_smem(kern, sm));
     kern<<<(unsigned)ceil_div(n * 32, 256), 256, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap);
     AMGT_LAUNCHED();
     return AMGT_OK;
@@ -1956,7 +1956,7 @@ static amgt_status launch_block_bin(int64_t n, const int32_t* rows, const SymCtx
     const size_t sm = (size_t)S * 4 * 2 + (STEP == 2 ? (size_t)S / 2 * 8 : 0);
     const int threads = LOGS >= 12 ? 512 : 256;
     auto kern = k_sym_block<LOGS, STEP>;
-    AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    AMGT_CUDA(dyn_smem(kern, sm));
     kern<<<capped(n), threads, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap);
     AMGT_LAUNCHED();
     return AMGT_OK;
@@ -1972,7 +1972,7 @@ static amgt_status launch_dense_bin(int64_t n, const int32_t* rows, const SymCtx
     auto kern = k_sym_dense<STEP>;
     const size_t max_dyn = 160 * 1024;
     if (need <= max_dyn) {
-        AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)need));
+        AMGT_CUDA(dyn_smem(kern, need));
         kern<<<capped(n), 512, need, s>>>(n, rows, c, W, nullptr, nnz_row, cptr, cidx, cmap);
         AMGT_LAUNCHED();
     } else {
@@ -2156,6 +2156,92 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     return AMGT_OK;
 }
 
+// ---------------------------------------------------------------- numeric: B with one tile per row
+// C = A B when every block row of B holds at most one tile (the aggregation P of the RAP's A P,
+// R19): each A tile (I, K) meets at most one B tile (K, J_K), so C row I (<= NC tiles, positions
+// from the symbolic phase) is a sum of A tile x single B tile products.  A 4-lane group per C
+// block row, lane r owning row r of every C tile in registers; the A tiles of the row are walked
+// U at a time with all their loads in flight (column, B row pointer, B column, A row, B row — the
+// B tile arrives as four rows, one per lane, and is broadcast by shuffles); the product is formed
+// as in tile_mma and added in A-tile order (deterministic, the staged kernel's arithmetic); C
+// rows written once with full-line stores (+0.0 at the clear bits, R2).  No shared-memory
+// staging buffers, so the kernel runs at full occupancy: it is the A stream that bounds it.
+template <typename T, typename Acc, int NC, int U>
+__global__ void __launch_bounds__(256, 2) k_numeric_b1(int64_t BR, SymCtx c, const T* __restrict__ aval,
+                                                   const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                   const int32_t* __restrict__ cidx, const uint16_t* __restrict__ cmap,
+                                                   T* __restrict__ cval) {
+    const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
+    const unsigned gm = 0xFu << (lane & ~3);
+    const int gb = lane & ~3;
+    const int64_t ng = ((int64_t)gridDim.x * blockDim.x) >> 2;
+    for (int64_t I = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2; I < BR; I += ng) {
+        const int64_t c0 = cptr[I];
+        const int nC = (int)(cptr[I + 1] - c0);
+        int32_t cj[NC];
+#pragma unroll
+        for (int q = 0; q < NC; ++q) cj[q] = q < nC ? __ldg(cidx + c0 + q) : -1;
+        Acc acc[NC][4];
+#pragma unroll
+        for (int q = 0; q < NC; ++q)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[q][e] = Acc(0);
+        const int64_t t0 = c.aptr[I], t1 = c.aptr[I + 1];
+        for (int64_t t = t0; t < t1; t += U) {
+            int32_t K[U];
+            int64_t b[U];
+            bool hb[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) K[u] = t + u < t1 ? __ldg(c.aidx + t + u) : -1;
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                b[u] = K[u] >= 0 ? __ldg(c.bptr + K[u]) : 0;
+                hb[u] = K[u] >= 0 && __ldg(c.bptr + K[u] + 1) > b[u];
+            }
+            int32_t J[U];
+            Acc ar[U][4], br[U][4];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                J[u] = hb[u] ? __ldg(c.bidx + b[u]) : -1;
+                if (hb[u]) {
+                    RowIO<T>::load(aval + 16 * (t + u) + 4 * r, ar[u]);
+                    RowIO<T>::load(bval + 16 * b[u] + 4 * r, br[u]);  // B row r: this lane's share
+                } else {
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) ar[u][e] = br[u][e] = Acc(0);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                if (!hb[u]) continue;  // uniform across the group (same tile)
+                Acc pr[4];  // row r of A_t B: B element (k, col) from lane k of the group
+#pragma unroll
+                for (int col = 0; col < 4; ++col) {
+                    Acc s2 = ar[u][0] * __shfl_sync(gm, br[u][col], gb);
+                    s2 = fma_acc(ar[u][1], __shfl_sync(gm, br[u][col], gb + 1), s2);
+                    s2 = fma_acc(ar[u][2], __shfl_sync(gm, br[u][col], gb + 2), s2);
+                    s2 = fma_acc(ar[u][3], __shfl_sync(gm, br[u][col], gb + 3), s2);
+                    pr[col] = s2;
+                }
+#pragma unroll
+                for (int q = 0; q < NC; ++q)
+                    if (cj[q] == J[u])
+#pragma unroll
+                        for (int col = 0; col < 4; ++col) acc[q][col] = acc[q][col] + pr[col];
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < NC; ++q) {
+            if (q >= nC) break;
+            const uint32_t mp = (__ldg(cmap + c0 + q) >> (4 * r)) & 0xFu;
+            Acc o[4];
+#pragma unroll
+            for (int col = 0; col < 4; ++col) o[col] = ((mp >> col) & 1u) ? acc[q][col] : Acc(0);
+            RowIO<T>::store(cval + 16 * (c0 + q) + 4 * r, o);
+        }
+    }
+}
+
 template <typename T, typename Acc>
 static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a) {
     cudaStream_t s = a.s;
@@ -2174,6 +2260,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     // with the DMMA / HMMA routes.  AMGT_NUM_STAGED=0 forces the latter (measurement).
     static const int staged_env = [] { const char* e = getenv("AMGT_NUM_STAGED"); return e ? atoi(e) : 1; }();
     const bool tc_route = (sizeof(T) == 8 || sizeof(T) == 2) && g_tc_thr_spgemm <= 16;
+    static const int b1_env = [] { const char* e = getenv("AMGT_NUM_B1"); return e ? atoi(e) : 1; }();
+    if (!tc_route && b1_env && B->row_max == 1 && C->row_max > 0 && C->row_max <= GROUP_NC) {
+        // every B block row holds at most one tile (aggregation P): k_numeric_b1 over all rows
+        const unsigned grid = (unsigned)std::min<int64_t>(ceil_div(4 * BR, 256), (int64_t)num_sms() * 8);
+        if (C->row_max <= 4)
+            k_numeric_b1<T, Acc, 4, 4><<<grid, 256, 0, s>>>(BR, c, (const T*)A->blc_val, (const T*)B->blc_val,
+                                                            C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val);
+        else
+            k_numeric_b1<T, Acc, GROUP_NC, 2><<<grid, 256, 0, s>>>(BR, c, (const T*)A->blc_val, (const T*)B->blc_val,
+                                                                   C->blc_ptr, C->blc_idx, C->blc_map,
+                                                                   (T*)C->blc_val);
+        AMGT_LAUNCHED();
+        return AMGT_OK;
+    }
     if (!tc_route && staged_env) {
         static const int nbuf_env = [] { const char* e = getenv("AMGT_STAGED_NBUF"); return e ? atoi(e) : 2; }();
         const int nbuf = nbuf_env == 1 ? 1 : 2;
@@ -2181,7 +2281,7 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         const bool nc4 = C->row_max > 0 && C->row_max <= 4;
         auto kern = nc4 ? (nbuf == 2 ? k_numeric_staged<T, Acc, 4, 2> : k_numeric_staged<T, Acc, 4, 1>)
                         : (nbuf == 2 ? k_numeric_staged<T, Acc, GROUP_NC, 2> : k_numeric_staged<T, Acc, GROUP_NC, 1>);
-        if (sm > 48 * 1024) AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        AMGT_CUDA(dyn_smem(kern, sm));
         // rows per group: several when rows are short (mean pairs per row ~ (T_A/BR_A)(T_B/BR_B)),
         // one when a row alone keeps the batch pipeline busy (and the grid large)
         const double mp = (BR ? (double)A->blc_num / BR : 0.0) * (B->blc_row ? (double)B->blc_num / B->blc_row : 0.0);
@@ -2213,7 +2313,7 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     {
         int per_sm = 0;
         const size_t msm = MID_WARPS * (32 * 16 * sizeof(Acc) + 2 * MIDCAP * sizeof(int32_t));
-        AMGT_CUDA(cudaFuncSetAttribute(k_numeric_mid<T, Acc>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)msm));
+        AMGT_CUDA(dyn_smem(k_numeric_mid<T, Acc>, msm));
         AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_numeric_mid<T, Acc>, MID_WARPS * 32, msm));
         k_numeric_mid<T, Acc><<<(unsigned)num_sms() * (unsigned)max(per_sm, 1), MID_WARPS * 32, msm, s>>>(
             mid.p, nbig.p + 3, nbig.p + 4, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx,
@@ -2257,7 +2357,7 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
             // column samples (+ per-warp product staging in pass 1)
             const size_t sm = (size_t)LONG_SMEM * sizeof(int32_t) + (pass ? 8 * 32 * 16 * sizeof(Acc) : 0);
             auto kern = pass == 0 ? k_numeric_long<T, Acc, 0> : k_numeric_long<T, Acc, 1>;
-            AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+            AMGT_CUDA(dyn_smem(kern, sm));
             int per_sm = 0;  // persistent grid: exactly the resident CTAs
             AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, sm));
             kern<<<(unsigned)num_sms() * (unsigned)max(per_sm, 1), 256, sm, s>>>(

@@ -1039,11 +1039,7 @@ amgt_status amgt_sweep_plan_create(const amgt_mbsr* A, const amgt_allocator* al,
     p.nchunks = ceil_div(A->blc_row, SW_CHUNK);
     p.tma = sweep_use_tma() && A->blc_num < ((int64_t)1 << 31);  // 32-bit tile offsets in the TMA descriptors
     if (p.tma) {
-        static bool attr = false;
-        if (!attr) {
-            cudaFuncSetAttribute(k_sweep_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, TM_SMEM);
-            attr = true;
-        }
+        AMGT_CUDA(dyn_smem(k_sweep_tma, TM_SMEM));
         p.grid = num_sms();
     } else {
         p.grid = num_sms() * sweep_ctas_per_sm();

@@ -409,12 +409,7 @@ static amgt_status device_coarse_inverse(const amgt_mbsr& C, double* Ainv, uint3
     if (n == 0) return AMGT_OK;
     if (n <= GJ_SMEM_N) {
         const size_t sm = (size_t)(n * n + 2 * n) * sizeof(double);
-        static bool attr = false;
-        if (!attr) {
-            AMGT_CUDA(cudaFuncSetAttribute(k_gauss_jordan_smem, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                           (int)((GJ_SMEM_N * GJ_SMEM_N + 2 * GJ_SMEM_N) * sizeof(double))));
-            attr = true;
-        }
+        AMGT_CUDA(dyn_smem(k_gauss_jordan_smem, (GJ_SMEM_N * GJ_SMEM_N + 2 * GJ_SMEM_N) * sizeof(double)));
         k_gauss_jordan_smem<<<1, 512, sm, s>>>((int)n, Ainv, dflag);
         AMGT_LAUNCHED();
         return AMGT_OK;
@@ -1267,7 +1262,7 @@ static amgt_status subcycle_tail(amgt_hierarchy* H, int kt) {
         if (ok) {
             const bool f64 = H->L[kt].vprec == AMGT_FP64;
             auto kern = f64 ? k_tail_smem<double> : k_tail_smem<float>;
-            AMGT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+            AMGT_CUDA(dyn_smem(kern, bytes));
             pdl_launch(kern, dim3(1), dim3(512), bytes, H->s, *sa);
             delete sa;
             AMGT_LAUNCHED();
