@@ -2160,20 +2160,67 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
 // C = A B when every block row of B holds at most one tile (the aggregation P of the RAP's A P,
 // R19): each A tile (I, K) meets at most one B tile (K, J_K), so C row I (<= NC tiles, positions
 // from the symbolic phase) is a sum of A tile x single B tile products.  A 4-lane group per C
-// block row, lane r owning row r of every C tile in registers; the A tiles of the row are walked
-// U at a time with all their loads in flight (column, B row pointer, B column, A row, B row — the
-// B tile arrives as four rows, one per lane, and is broadcast by shuffles); the product is formed
-// as in tile_mma and added in A-tile order (deterministic, the staged kernel's arithmetic); C
-// rows written once with full-line stores (+0.0 at the clear bits, R2).  No shared-memory
-// staging buffers, so the kernel runs at full occupancy: it is the A stream that bounds it.
-template <typename T, typename Acc, int NC, int U>
-__global__ void __launch_bounds__(256, 2) k_numeric_b1(int64_t BR, SymCtx c, const T* __restrict__ aval,
-                                                   const T* __restrict__ bval, const int64_t* __restrict__ cptr,
-                                                   const int32_t* __restrict__ cidx, const uint16_t* __restrict__ cmap,
-                                                   T* __restrict__ cval) {
+// block row, lane r owning row r of every C tile.  The row's A tiles are taken 32 at a time: the
+// group first resolves each tile's B position and C slot (lane r, slot s <- tile 4s + r: column,
+// B row pointers, B column — three rounds of independent loads for the whole chunk), then streams
+// the chunk four tiles per step with no dependent load left (A row r and B row r of four tiles in
+// flight per lane; the B tile is broadcast in the group by shuffles).  The products are formed as
+// in tile_mma and added in A-tile order into the lane's rows of the C tiles in shared memory
+// (lane-private, deterministic: the staged kernel's arithmetic); C rows written once with
+// full-line stores (+0.0 at the clear bits, R2).  Group buffers are padded by 16 B so the eight
+// groups of a warp spread over the banks.
+constexpr int B1_WARPS = 8;
+template <typename Acc, int NC>
+constexpr int b1_gstride() { return NC * 16 + 16 / (int)sizeof(Acc); }
+template <typename Acc, int NC>
+constexpr size_t b1_smem_bytes() { return (size_t)B1_WARPS * 8 * b1_gstride<Acc, NC>() * sizeof(Acc); }
+
+template <typename Acc> struct SmemRow;
+template <> struct SmemRow<double> {
+    static __device__ __forceinline__ void add(double* p, const double (&v)[4]) {
+        double2* q = reinterpret_cast<double2*>(p);
+        double2 a = q[0], b = q[1];
+        a.x += v[0]; a.y += v[1]; b.x += v[2]; b.y += v[3];
+        q[0] = a; q[1] = b;
+    }
+    static __device__ __forceinline__ void take(double* p, double (&v)[4]) {
+        double2* q = reinterpret_cast<double2*>(p);
+        const double2 a = q[0], b = q[1];
+        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+        q[0] = q[1] = make_double2(0.0, 0.0);
+    }
+    static __device__ __forceinline__ void zero(double* p) {
+        reinterpret_cast<double2*>(p)[0] = reinterpret_cast<double2*>(p)[1] = make_double2(0.0, 0.0);
+    }
+};
+template <> struct SmemRow<float> {
+    static __device__ __forceinline__ void add(float* p, const float (&v)[4]) {
+        float4* q = reinterpret_cast<float4*>(p);
+        float4 a = *q;
+        a.x += v[0]; a.y += v[1]; a.z += v[2]; a.w += v[3];
+        *q = a;
+    }
+    static __device__ __forceinline__ void take(float* p, float (&v)[4]) {
+        float4* q = reinterpret_cast<float4*>(p);
+        const float4 a = *q;
+        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+        *q = make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    static __device__ __forceinline__ void zero(float* p) { *reinterpret_cast<float4*>(p) = make_float4(0.f, 0.f, 0.f, 0.f); }
+};
+
+template <typename T, typename Acc, int NC>
+__global__ void __launch_bounds__(B1_WARPS * 32, 2) k_numeric_b1(int64_t BR, SymCtx c, const T* __restrict__ aval,
+                                                             const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                             const int32_t* __restrict__ cidx,
+                                                             const uint16_t* __restrict__ cmap, T* __restrict__ cval) {
+    extern __shared__ __align__(16) unsigned char b1_smem[];
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
     const unsigned gm = 0xFu << (lane & ~3);
     const int gb = lane & ~3;
+    Acc* acc = reinterpret_cast<Acc*>(b1_smem) + ((threadIdx.x >> 5) * 8 + g) * b1_gstride<Acc, NC>() + 4 * r;
+#pragma unroll
+    for (int q = 0; q < NC; ++q) SmemRow<Acc>::zero(acc + 16 * q);
     const int64_t ng = ((int64_t)gridDim.x * blockDim.x) >> 2;
     for (int64_t I = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2; I < BR; I += ng) {
         const int64_t c0 = cptr[I];
@@ -2181,65 +2228,94 @@ __global__ void __launch_bounds__(256, 2) k_numeric_b1(int64_t BR, SymCtx c, con
         int32_t cj[NC];
 #pragma unroll
         for (int q = 0; q < NC; ++q) cj[q] = q < nC ? __ldg(cidx + c0 + q) : -1;
-        Acc acc[NC][4];
-#pragma unroll
-        for (int q = 0; q < NC; ++q)
-#pragma unroll
-            for (int e = 0; e < 4; ++e) acc[q][e] = Acc(0);
         const int64_t t0 = c.aptr[I], t1 = c.aptr[I + 1];
-        for (int64_t t = t0; t < t1; t += U) {
-            int32_t K[U];
-            int64_t b[U];
-            bool hb[U];
+        for (int64_t tc = t0; tc < t1; tc += 32) {
+            // chunk metadata: lane r resolves tiles tc + 4s + r
+            int32_t K[8], bp[8];
 #pragma unroll
-            for (int u = 0; u < U; ++u) K[u] = t + u < t1 ? __ldg(c.aidx + t + u) : -1;
+            for (int s = 0; s < 8; ++s) K[s] = tc + 4 * s + r < t1 ? __ldg(c.aidx + tc + 4 * s + r) : -1;
+            int64_t b0[8];
+            bool has[8];
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                b[u] = K[u] >= 0 ? __ldg(c.bptr + K[u]) : 0;
-                hb[u] = K[u] >= 0 && __ldg(c.bptr + K[u] + 1) > b[u];
+            for (int s = 0; s < 8; ++s) {
+                b0[s] = K[s] >= 0 ? __ldg(c.bptr + K[s]) : 0;
+                has[s] = K[s] >= 0 && __ldg(c.bptr + K[s] + 1) > b0[s];
             }
-            int32_t J[U];
-            Acc ar[U][4], br[U][4];
+            uint32_t qq = 0;
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                J[u] = hb[u] ? __ldg(c.bidx + b[u]) : -1;
-                if (hb[u]) {
-                    RowIO<T>::load(aval + 16 * (t + u) + 4 * r, ar[u]);
-                    RowIO<T>::load(bval + 16 * b[u] + 4 * r, br[u]);  // B row r: this lane's share
-                } else {
+            for (int s = 0; s < 8; ++s) {
+                const int32_t J = has[s] ? __ldg(c.bidx + b0[s]) : -1;
+                int q = 15;
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) ar[u][e] = br[u][e] = Acc(0);
-                }
+                for (int k = 0; k < NC; ++k)
+                    if (cj[k] == J && J >= 0) q = k;
+                bp[s] = q < NC ? (int32_t)b0[s] : -1;
+                qq |= (uint32_t)q << (4 * s);
             }
+            const int ns = (int)(t1 - tc < 32 ? t1 - tc : 32);
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                if (!hb[u]) continue;  // uniform across the group (same tile)
-                Acc pr[4];  // row r of A_t B: B element (k, col) from lane k of the group
+            for (int s = 0; s < 8; ++s) {
+                if (4 * s >= ns) break;  // uniform across the group
+                int qv[4];
+                Acc ar[4][4], br[4][4];
 #pragma unroll
-                for (int col = 0; col < 4; ++col) {
-                    Acc s2 = ar[u][0] * __shfl_sync(gm, br[u][col], gb);
-                    s2 = fma_acc(ar[u][1], __shfl_sync(gm, br[u][col], gb + 1), s2);
-                    s2 = fma_acc(ar[u][2], __shfl_sync(gm, br[u][col], gb + 2), s2);
-                    s2 = fma_acc(ar[u][3], __shfl_sync(gm, br[u][col], gb + 3), s2);
-                    pr[col] = s2;
+                for (int u = 0; u < 4; ++u) {
+                    const int32_t bpu = __shfl_sync(gm, bp[s], gb + u);
+                    qv[u] = (int)((__shfl_sync(gm, qq, gb + u) >> (4 * s)) & 15u);
+                    if (bpu >= 0) {
+                        RowIO<T>::load(aval + 16 * (tc + 4 * s + u) + 4 * r, ar[u]);
+                        RowIO<T>::load(bval + 16 * (int64_t)bpu + 4 * r, br[u]);  // B row r: this lane's share
+                    } else {
+                        qv[u] = 15;
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) ar[u][e] = br[u][e] = Acc(0);
+                    }
                 }
 #pragma unroll
-                for (int q = 0; q < NC; ++q)
-                    if (cj[q] == J[u])
+                for (int u = 0; u < 4; ++u) {
+                    if (qv[u] >= NC) continue;  // uniform across the group (same tile)
+                    Acc pr[4];  // row r of A_t B: B element (k, col) from lane k of the group
 #pragma unroll
-                        for (int col = 0; col < 4; ++col) acc[q][col] = acc[q][col] + pr[col];
+                    for (int col = 0; col < 4; ++col) {
+                        Acc s2 = ar[u][0] * __shfl_sync(gm, br[u][col], gb);
+                        s2 = fma_acc(ar[u][1], __shfl_sync(gm, br[u][col], gb + 1), s2);
+                        s2 = fma_acc(ar[u][2], __shfl_sync(gm, br[u][col], gb + 2), s2);
+                        s2 = fma_acc(ar[u][3], __shfl_sync(gm, br[u][col], gb + 3), s2);
+                        pr[col] = s2;
+                    }
+                    SmemRow<Acc>::add(acc + 16 * qv[u], pr);
+                }
             }
         }
 #pragma unroll
         for (int q = 0; q < NC; ++q) {
             if (q >= nC) break;
             const uint32_t mp = (__ldg(cmap + c0 + q) >> (4 * r)) & 0xFu;
-            Acc o[4];
+            Acc v[4], o[4];
+            SmemRow<Acc>::take(acc + 16 * q, v);
 #pragma unroll
-            for (int col = 0; col < 4; ++col) o[col] = ((mp >> col) & 1u) ? acc[q][col] : Acc(0);
+            for (int col = 0; col < 4; ++col) o[col] = ((mp >> col) & 1u) ? v[col] : Acc(0);
             RowIO<T>::store(cval + 16 * (c0 + q) + 4 * r, o);
         }
     }
+}
+
+template <typename T, typename Acc, int NC>
+static amgt_status launch_b1(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, const SymCtx& c, cudaStream_t s) {
+    auto kern = k_numeric_b1<T, Acc, NC>;
+    const size_t sm = b1_smem_bytes<Acc, NC>();
+    AMGT_CUDA(dyn_smem(kern, sm));
+    static const int per_sm = [&] {
+        int n = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, B1_WARPS * 32, sm);
+        return n > 0 ? n : 1;
+    }();
+    const int64_t BR = A->blc_row;
+    const unsigned grid = (unsigned)std::min<int64_t>(ceil_div(4 * BR, B1_WARPS * 32), (int64_t)num_sms() * per_sm);
+    kern<<<grid, B1_WARPS * 32, sm, s>>>(BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx,
+                                         C->blc_map, (T*)C->blc_val);
+    AMGT_LAUNCHED();
+    return AMGT_OK;
 }
 
 template <typename T, typename Acc>
@@ -2261,18 +2337,10 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     static const int staged_env = [] { const char* e = getenv("AMGT_NUM_STAGED"); return e ? atoi(e) : 1; }();
     const bool tc_route = (sizeof(T) == 8 || sizeof(T) == 2) && g_tc_thr_spgemm <= 16;
     static const int b1_env = [] { const char* e = getenv("AMGT_NUM_B1"); return e ? atoi(e) : 1; }();
-    if (!tc_route && b1_env && B->row_max == 1 && C->row_max > 0 && C->row_max <= GROUP_NC) {
+    if (!tc_route && b1_env && B->row_max == 1 && C->row_max > 0 && C->row_max <= GROUP_NC &&
+        B->blc_num < ((int64_t)1 << 31)) {
         // every B block row holds at most one tile (aggregation P): k_numeric_b1 over all rows
-        const unsigned grid = (unsigned)std::min<int64_t>(ceil_div(4 * BR, 256), (int64_t)num_sms() * 8);
-        if (C->row_max <= 4)
-            k_numeric_b1<T, Acc, 4, 4><<<grid, 256, 0, s>>>(BR, c, (const T*)A->blc_val, (const T*)B->blc_val,
-                                                            C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val);
-        else
-            k_numeric_b1<T, Acc, GROUP_NC, 2><<<grid, 256, 0, s>>>(BR, c, (const T*)A->blc_val, (const T*)B->blc_val,
-                                                                   C->blc_ptr, C->blc_idx, C->blc_map,
-                                                                   (T*)C->blc_val);
-        AMGT_LAUNCHED();
-        return AMGT_OK;
+        return C->row_max <= 4 ? launch_b1<T, Acc, 4>(A, B, C, c, s) : launch_b1<T, Acc, GROUP_NC>(A, B, C, c, s);
     }
     if (!tc_route && staged_env) {
         static const int nbuf_env = [] { const char* e = getenv("AMGT_STAGED_NBUF"); return e ? atoi(e) : 2; }();
