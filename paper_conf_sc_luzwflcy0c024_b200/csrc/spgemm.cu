@@ -2172,8 +2172,42 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
 constexpr int B1_WARPS = 8;
 template <typename Acc, int NC>
 constexpr int b1_gstride() { return NC * 16 + 16 / (int)sizeof(Acc); }
-template <typename Acc, int NC>
-constexpr size_t b1_smem_bytes() { return (size_t)B1_WARPS * 8 * b1_gstride<Acc, NC>() * sizeof(Acc); }
+// per group: the C-row accumulators (b1_gstride Acc) + the step's four B tiles (64 T, 16-B padded)
+template <typename T>
+constexpr int b1_bstride() { return 64 + 16 / (int)sizeof(T); }
+template <typename T, typename Acc, int NC>
+constexpr size_t b1_smem_bytes() {
+    return (size_t)B1_WARPS * 8 * (b1_gstride<Acc, NC>() * sizeof(Acc) + b1_bstride<T>() * sizeof(T));
+}
+
+// Row r of a B tile: global -> shared memory without registers (cp.async), and shared -> Acc.
+template <typename T> struct B1Row;
+template <> struct B1Row<double> {
+    static __device__ __forceinline__ void copy(double* d, const double* g) { cp_async16(d, g); cp_async16(d + 2, g + 2); }
+    static __device__ __forceinline__ void read(const double* p, double (&v)[4]) {
+        const double2 a = reinterpret_cast<const double2*>(p)[0], b = reinterpret_cast<const double2*>(p)[1];
+        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+    }
+};
+template <> struct B1Row<float> {
+    static __device__ __forceinline__ void copy(float* d, const float* g) { cp_async16(d, g); }
+    static __device__ __forceinline__ void read(const float* p, float (&v)[4]) {
+        const float4 a = *reinterpret_cast<const float4*>(p);
+        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+    }
+};
+template <> struct B1Row<__half> {
+    static __device__ __forceinline__ void copy(__half* d, const __half* g) {
+        const uint32_t sa = (uint32_t)__cvta_generic_to_shared(d);
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(sa), "l"(g) : "memory");
+    }
+    static __device__ __forceinline__ void read(const __half* p, float (&v)[4]) {
+        const uint2 u = *reinterpret_cast<const uint2*>(p);
+        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&u.x));
+        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&u.y));
+        v[0] = lo.x; v[1] = lo.y; v[2] = hi.x; v[3] = hi.y;
+    }
+};
 
 template <typename Acc> struct SmemRow;
 template <> struct SmemRow<double> {
@@ -2218,7 +2252,10 @@ __global__ void __launch_bounds__(B1_WARPS * 32, 2) k_numeric_b1(int64_t BR, Sym
     const int lane = threadIdx.x & 31, g = lane >> 2, r = lane & 3;
     const unsigned gm = 0xFu << (lane & ~3);
     const int gb = lane & ~3;
-    Acc* acc = reinterpret_cast<Acc*>(b1_smem) + ((threadIdx.x >> 5) * 8 + g) * b1_gstride<Acc, NC>() + 4 * r;
+    const int gid = (threadIdx.x >> 5) * 8 + g;
+    Acc* acc = reinterpret_cast<Acc*>(b1_smem) + gid * b1_gstride<Acc, NC>() + 4 * r;
+    T* sB = reinterpret_cast<T*>(b1_smem + (size_t)B1_WARPS * 8 * b1_gstride<Acc, NC>() * sizeof(Acc)) +
+            gid * b1_bstride<T>();  // tile u at sB + 16 u (row-major)
 #pragma unroll
     for (int q = 0; q < NC; ++q) SmemRow<Acc>::zero(acc + 16 * q);
     const int64_t ng = ((int64_t)gridDim.x * blockDim.x) >> 2;
@@ -2257,34 +2294,41 @@ __global__ void __launch_bounds__(B1_WARPS * 32, 2) k_numeric_b1(int64_t BR, Sym
             for (int s = 0; s < 8; ++s) {
                 if (4 * s >= ns) break;  // uniform across the group
                 int qv[4];
-                Acc ar[4][4], br[4][4];
+                Acc ar[4][4];
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
+                for (int u = 0; u < 4; ++u) {  // B row r of the four tiles -> shared memory, A row r -> registers
                     const int32_t bpu = __shfl_sync(gm, bp[s], gb + u);
                     qv[u] = (int)((__shfl_sync(gm, qq, gb + u) >> (4 * s)) & 15u);
                     if (bpu >= 0) {
+                        B1Row<T>::copy(sB + 16 * u + 4 * r, bval + 16 * (int64_t)bpu + 4 * r);
                         RowIO<T>::load(aval + 16 * (tc + 4 * s + u) + 4 * r, ar[u]);
-                        RowIO<T>::load(bval + 16 * (int64_t)bpu + 4 * r, br[u]);  // B row r: this lane's share
                     } else {
                         qv[u] = 15;
-#pragma unroll
-                        for (int e = 0; e < 4; ++e) ar[u][e] = br[u][e] = Acc(0);
                     }
                 }
+                asm volatile("cp.async.commit_group;" ::: "memory");
+                asm volatile("cp.async.wait_group 0;" ::: "memory");
+                __syncwarp(gm);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) {
                     if (qv[u] >= NC) continue;  // uniform across the group (same tile)
-                    Acc pr[4];  // row r of A_t B: B element (k, col) from lane k of the group
+                    Acc pr[4];  // row r of A_t B, in tile_mma's order (k = 0..3)
+                    {
+                        Acc b0[4];
+                        B1Row<T>::read(sB + 16 * u, b0);
 #pragma unroll
-                    for (int col = 0; col < 4; ++col) {
-                        Acc s2 = ar[u][0] * __shfl_sync(gm, br[u][col], gb);
-                        s2 = fma_acc(ar[u][1], __shfl_sync(gm, br[u][col], gb + 1), s2);
-                        s2 = fma_acc(ar[u][2], __shfl_sync(gm, br[u][col], gb + 2), s2);
-                        s2 = fma_acc(ar[u][3], __shfl_sync(gm, br[u][col], gb + 3), s2);
-                        pr[col] = s2;
+                        for (int col = 0; col < 4; ++col) pr[col] = ar[u][0] * b0[col];
+                    }
+#pragma unroll
+                    for (int k = 1; k < 4; ++k) {
+                        Acc bk[4];
+                        B1Row<T>::read(sB + 16 * u + 4 * k, bk);
+#pragma unroll
+                        for (int col = 0; col < 4; ++col) pr[col] = fma_acc(ar[u][k], bk[col], pr[col]);
                     }
                     SmemRow<Acc>::add(acc + 16 * qv[u], pr);
                 }
+                __syncwarp(gm);  // the step's B tiles are consumed before the next step's copies
             }
         }
 #pragma unroll
@@ -2303,7 +2347,7 @@ __global__ void __launch_bounds__(B1_WARPS * 32, 2) k_numeric_b1(int64_t BR, Sym
 template <typename T, typename Acc, int NC>
 static amgt_status launch_b1(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, const SymCtx& c, cudaStream_t s) {
     auto kern = k_numeric_b1<T, Acc, NC>;
-    const size_t sm = b1_smem_bytes<Acc, NC>();
+    const size_t sm = b1_smem_bytes<T, Acc, NC>();
     AMGT_CUDA(dyn_smem(kern, sm));
     static const int per_sm = [&] {
         int n = 0;
