@@ -442,6 +442,84 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
     }
 }
 
+// Symbolic step 1 when every block row of B holds at most one tile (A P with an aggregation P,
+// R19) and every row of A at most 32 tiles: Cub(I) = the A tiles of row I whose B row is not
+// empty (all category 8).  A 4-lane group per row resolves them (lane r: tiles 4s + r, s < 8 —
+// column and bitmap, B row pointers, B column and bitmap: three rounds of independent loads) and
+// extracts the distinct columns J with BITMAPMULTIPLY != 0 in ascending order, each with the OR
+// of its bitmap products (group min / OR by shuffles; no shared memory, no pair lists).  The
+// sorted list goes to the row's 32-slot scratch row for k_sym_copy, the count to nnz_row: the
+// same outputs as k_sym_flat<1> for these rows.
+__global__ void __launch_bounds__(256) k_sym_b1(int64_t BR, SymCtx c, int64_t* __restrict__ nnz_row,
+                                                int64_t* __restrict__ bin_of, unsigned long long* __restrict__ stats,
+                                                int32_t* __restrict__ sidx, uint16_t* __restrict__ smap) {
+    const int lane = threadIdx.x & 31, r = lane & 3;
+    const unsigned gm = 0xFu << (lane & ~3);
+    unsigned long long rows8 = 0, cubs = 0;
+    for (int64_t I = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2; I < BR;
+         I += ((int64_t)gridDim.x * blockDim.x) >> 2) {
+        const int64_t t0 = c.aptr[I], t1 = c.aptr[I + 1];
+        int32_t K[8], J[8];
+        uint32_t ma[8], mc[8];
+        int64_t b0[8];
+        bool has[8];
+#pragma unroll
+        for (int s = 0; s < 8; ++s) {
+            const int64_t t = t0 + 4 * s + r;
+            K[s] = t < t1 ? __ldg(c.aidx + t) : -1;
+            ma[s] = t < t1 ? __ldg(c.amap + t) : 0u;
+        }
+#pragma unroll
+        for (int s = 0; s < 8; ++s) {
+            b0[s] = K[s] >= 0 ? __ldg(c.bptr + K[s]) : 0;
+            has[s] = K[s] >= 0 && __ldg(c.bptr + K[s] + 1) > b0[s];
+        }
+        int cub = 0;
+#pragma unroll
+        for (int s = 0; s < 8; ++s) {
+            mc[s] = has[s] ? bitmap_multiply(ma[s], __ldg(c.bmap + b0[s])) : 0u;
+            J[s] = mc[s] ? __ldg(c.bidx + b0[s]) : INT_MAX;
+            cub += has[s];
+        }
+        cub += __shfl_xor_sync(gm, cub, 1, 4);
+        cub += __shfl_xor_sync(gm, cub, 2, 4);
+        int n = 0, prev = -1;
+        for (;;) {  // group-uniform: ascending distinct columns
+            int m = INT_MAX;
+#pragma unroll
+            for (int s = 0; s < 8; ++s) m = (J[s] > prev && J[s] < m) ? J[s] : m;
+            m = min(m, __shfl_xor_sync(gm, m, 1, 4));
+            m = min(m, __shfl_xor_sync(gm, m, 2, 4));
+            if (m == INT_MAX) break;
+            uint32_t o = 0;
+#pragma unroll
+            for (int s = 0; s < 8; ++s) o |= (J[s] == m) ? mc[s] : 0u;
+            o |= __shfl_xor_sync(gm, o, 1, 4);
+            o |= __shfl_xor_sync(gm, o, 2, 4);
+            if (r == 0) {
+                sidx[SMALL_CUB * I + n] = m;
+                smap[SMALL_CUB * I + n] = (uint16_t)o;
+            }
+            ++n;
+            prev = m;
+        }
+        if (r == 0) {
+            nnz_row[I] = n;
+            bin_of[I] = NBINS;
+            rows8 += 1;
+            cubs += (unsigned long long)cub;
+        }
+    }
+    for (int d = 16; d; d >>= 1) {
+        rows8 += __shfl_xor_sync(0xffffffffu, rows8, d);
+        cubs += __shfl_xor_sync(0xffffffffu, cubs, d);
+    }
+    if (lane == 0) {
+        if (rows8) atomicAdd(&stats[cat_stat(NBINS)], rows8);
+        if (cubs) atomicAdd(&stats[8], cubs);
+    }
+}
+
 // Step 2 of the category-8 rows when step 1 kept their sorted lists: copy slot [32 I, +n) to
 // C at cptr[I] (4-lane group per row).
 __global__ void __launch_bounds__(256) k_sym_copy(int64_t BR, const int64_t* __restrict__ bin_of,
@@ -2065,7 +2143,19 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         bool keep = BR > 0 && (double)BR * SMALL_CUB * 6.0 <= 2e9;
         if (keep)  // optional: without it step 2 re-expands the rows (k_sym_flat<2>)
             keep = sidx.try_init(a, (size_t)BR * SMALL_CUB) && smap.try_init(a, (size_t)BR * SMALL_CUB);
-        if (BR > 0) {
+        // B rows of at most one tile and A rows of at most 32 (A P with an aggregation P):
+        // k_sym_b1 (needs the kept scratch rows; AMGT_SYM_B1=0 forces the general kernel)
+        static const int symb1_env = [] { const char* e = getenv("AMGT_SYM_B1"); return e ? atoi(e) : 1; }();
+        const bool b1 = symb1_env && keep && B->row_max == 1 && A->row_max > 0 && A->row_max <= SMALL_CUB;
+        if (BR > 0 && b1) {
+            k_sym_b1<<<(unsigned)std::min<int64_t>(ceil_div(4 * BR, 256), (int64_t)num_sms() * 8), 256, 0, s>>>(
+                BR, c, nnz_row.p, bin_of.p, stats, sidx.p, smap.p);
+            AMGT_LAUNCHED();
+            if (info && A->blc_num > 0) {
+                k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats, g_tc_thr_spgemm);
+                AMGT_LAUNCHED();
+            }
+        } else if (BR > 0) {
             k_sym_flat<1><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nnz_row.p, nullptr, nullptr, nullptr,
                                                                      bin_of.p, stats, sidx.p, smap.p);
             AMGT_LAUNCHED();
@@ -2163,8 +2253,9 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
 // block row, lane r owning row r of every C tile.  The row's A tiles are taken 32 at a time: the
 // group first resolves each tile's B position and C slot (lane r, slot s <- tile 4s + r: column,
 // B row pointers, B column — three rounds of independent loads for the whole chunk), then streams
-// the chunk four tiles per step with no dependent load left (A row r and B row r of four tiles in
-// flight per lane; the B tile is broadcast in the group by shuffles).  The products are formed as
+// the chunk four tiles per step with no dependent load left (A row r of four tiles in flight per
+// lane in registers, their B tiles copied row by row into a per-group shared-memory buffer with
+// cp.async and read back as broadcasts).  The products are formed as
 // in tile_mma and added in A-tile order into the lane's rows of the C tiles in shared memory
 // (lane-private, deterministic: the staged kernel's arithmetic); C rows written once with
 // full-line stores (+0.0 at the clear bits, R2).  Group buffers are padded by 16 B so the eight
