@@ -149,7 +149,7 @@ static bool conv_stage() {
     return v == 1;
 }
 constexpr int CONV_WARPS = 4;     // 128-thread CTAs
-constexpr int CONV_STAGE = 1024;  // entries per warp (27-point: 32 rows x 27 = 864)
+constexpr int CONV_STAGE = 896;  // entries per warp (27-point: 32 rows x 27 = 864; 5 CTAs per SM)
 template <bool FILL>
 constexpr int conv_smem_bytes() { return FILL ? CONV_WARPS * CONV_STAGE * 12 : 0; }
 
@@ -212,23 +212,26 @@ __global__ void __launch_bounds__(128) k_csr2mbsr(int64_t m, int64_t n, int64_t 
     int64_t t = (FILL && active) ? bptr[I] : 0;
     int64_t c = 0;
     int32_t prev = -1;
+    // the lane's next entry's column, loaded one entry ahead (the merge chain then waits for
+    // one shared-memory / global load per entry, not two)
+    int32_t col = (p < e) ? (int32_t)(ld_ci(p) - coff) : 0;
     for (;;) {
-        const int32_t J = (p < e) ? (int32_t)((ld_ci(p) - coff) >> 2) : INT_MAX;
+        const int32_t J = (p < e) ? (col >> 2) : INT_MAX;
         int32_t Jm = min(J, __shfl_xor_sync(0xffffffffu, J, 1));
         Jm = min(Jm, __shfl_xor_sync(0xffffffffu, Jm, 2));
         if (!__any_sync(0xffffffffu, Jm != INT_MAX)) break;
         double rv[4] = {0.0, 0.0, 0.0, 0.0};
         uint32_t nib = 0;
         if (Jm != INT_MAX) {
-            while (p < e) {
-                const int32_t col = (int32_t)(ld_ci(p) - coff);
-                if ((col >> 2) != Jm) break;
+            while (p < e && (col >> 2) == Jm) {
+                const int64_t pc = p++;
+                const int32_t ncol = (p < e) ? (int32_t)(ld_ci(p) - coff) : 0;
                 if (!FILL) {
                     if (col <= prev || col >= n || col < 0) bad = 1;
                     prev = col;
                 } else {
                     const int cc = col & 3;
-                    const double x = ld_v(p);
+                    const double x = ld_v(pc);
                     rv[0] = cc == 0 ? x : rv[0];
                     rv[1] = cc == 1 ? x : rv[1];
                     rv[2] = cc == 2 ? x : rv[2];
@@ -236,7 +239,7 @@ __global__ void __launch_bounds__(128) k_csr2mbsr(int64_t m, int64_t n, int64_t 
                     if (overflows<T>(x)) range = 1;
                 }
                 nib |= 1u << (col & 3);
-                ++p;
+                col = ncol;
             }
         }
         uint32_t mp = nib << (4 * r);
