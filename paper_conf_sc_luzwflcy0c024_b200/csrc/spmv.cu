@@ -241,6 +241,92 @@ __global__ void __launch_bounds__(256, MINB) k_spmv_rows(int64_t I0, int64_t BR,
         spmv_rows_octet<MatT, XT, YT, MODE, U, TC>(wid, I0, BR, bptr, bidx, bmap, bval, x, epi, long_thr, tc_thr);
 }
 
+// ---------------------------------------------------------------- warp-per-row kernel
+// FP32 / FP16 coarse operators of up to AMGT_SPMV_WROW block columns (default 65,536: config 3's
+// levels 3-5) with >= 16 tiles per block row on average (~27 there): a warp per block row, the 8 four-lane groups take tiles
+// g, g + 8, g + 16, g + 24 of the row (32 per iteration: one dependent round trip for the tiles
+// and one for x, where the octet kernel needs four pairs for a 27-tile row), lane q of a group
+// accumulates tile row q; the 8 group partials are added by a fixed 3-step xor tree
+// (deterministic).  The small levels are latency-bound, so fewer round trips per row is the gain.
+template <typename MatT, typename XT, typename YT, int MODE>
+__global__ void __launch_bounds__(256) k_spmv_wrow(int64_t I0, int64_t BR, const int64_t* __restrict__ bptr,
+                                                   const int32_t* __restrict__ bidx, const uint16_t* __restrict__ bmap,
+                                                   const MatT* __restrict__ bval, const XT* __restrict__ x,
+                                                   const Epi<XT, YT, MODE> epi, int64_t long_thr) {
+    pdl_wait();
+    const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t I = I0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); I < BR; I += nw) {
+        const int64_t t0 = __ldg(bptr + I);
+        int64_t t1 = __ldg(bptr + I + 1);
+        if (t1 - t0 > long_thr) continue;  // warp-uniform: the chunk kernel takes long rows
+        const int64_t out_i = 4 * I + q;
+        typename Epi<XT, YT, MODE>::Pre pre;
+        if (g == 0) pre = epi.prefetch(out_i);
+        constexpr int U = 4;
+        float acc = 0.f;
+        for (int64_t t = t0 + g; t < t1; t += 8 * U) {
+            int32_t J[U];
+            uint32_t nib[U];
+            float4 a[U], xv[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int64_t tt = t + 8 * u;
+                const bool v = tt < t1;
+                J[u] = v ? __ldg(bidx + tt) : 0;
+                nib[u] = v ? (__ldg(bmap + tt) >> (4 * q)) & 0xFu : 0u;
+                a[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (v) {
+                    if constexpr (sizeof(MatT) == 4) {
+                        a[u] = ldg_stream(reinterpret_cast<const float4*>(bval + 16 * tt) + q);
+                    } else {
+                        const uint2 w = ldg_stream(reinterpret_cast<const uint2*>(bval + 16 * tt) + q);
+                        const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&w.x));
+                        const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&w.y));
+                        a[u] = make_float4(lo.x, lo.y, hi.x, hi.y);
+                    }
+                }
+            }
+            if constexpr (MODE == EPI_RES_X0) {  // x1_J = 0 + w dinv_J (b_J - 0), the k_jacobi0 expression
+                const float om = (float)epi.omega;
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    xv[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (nib[u]) {
+                        const float4 bq = x_quad((const float*)epi.b, J[u]), dq = x_quad((const float*)epi.dinv, J[u]);
+                        const float zero = 0.f, z0 = 0.f;
+                        xv[u] = make_float4(zero + om * dq.x * (bq.x - z0), zero + om * dq.y * (bq.y - z0),
+                                            zero + om * dq.z * (bq.z - z0), zero + om * dq.w * (bq.w - z0));
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; ++u) xv[u] = nib[u] ? x_quad(x, J[u]) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                acc = (nib[u] & 1u) ? fmaf(a[u].x, xv[u].x, acc) : acc;
+                acc = (nib[u] & 2u) ? fmaf(a[u].y, xv[u].y, acc) : acc;
+                acc = (nib[u] & 4u) ? fmaf(a[u].z, xv[u].z, acc) : acc;
+                acc = (nib[u] & 8u) ? fmaf(a[u].w, xv[u].w, acc) : acc;
+            }
+        }
+        acc += __shfl_xor_sync(0xffffffffu, acc, 4);
+        acc += __shfl_xor_sync(0xffffffffu, acc, 8);
+        acc += __shfl_xor_sync(0xffffffffu, acc, 16);
+        if (g == 0) epi.finish(out_i, acc, pre);
+    }
+}
+
+static int64_t wrow_max_br() {
+    static int64_t v = -1;
+    if (v < 0) {
+        const char* e = getenv("AMGT_SPMV_WROW");
+        v = e ? atoll(e) : 65536;
+    }
+    return v;
+}
+
 // ---------------------------------------------------------------- lane-per-row kernel
 // For operators with ~1 tile per block row (interpolation P, L262/Alg. 2 line 8): one lane
 // owns a whole block row (its tiles' 16 values, its x segment, its 4 outputs), 32 block rows
@@ -874,6 +960,20 @@ static void launch_rows(const amgt_mbsr* A, const void* x, void* y, const EpiArg
     }
     const unsigned blocks = (unsigned)ceil_div(ceil_div(BR - I0, 8) * 32, 256);
     const int tc = sizeof(MatT) != 4 ? g_tc_thr_spmv : 17;  // FP32: CUDA cores (no TF32, R17)
+    if constexpr (sizeof(MatT) <= 4 && MODE != EPI_JACOBI_NORM) {
+        // small coarse levels with long rows (decided per operator — block columns, mean row
+        // length — so a row range of a distributed operator takes the same arithmetic)
+        const double mean = A->blc_row > 0 ? (double)A->blc_num / (double)A->blc_row : 0.0;
+        if (tc > 16 && A->blc_col <= wrow_max_br() && mean >= 16.0) {
+            auto kern = k_spmv_wrow<MatT, XT, YT, MODE>;
+            const int per_sm = occupancy_256(reinterpret_cast<const void*>(kern));
+            const int64_t cap = (int64_t)num_sms() * std::max(per_sm, 1);
+            const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(BR - I0, 8), cap));
+            pdl_launch(kern, dim3(g), dim3(256), 0, s, I0, BR, A->blc_ptr, A->blc_idx, A->blc_map,
+                       (const MatT*)A->blc_val, (const XT*)x, epi, long_thr);
+            return;
+        }
+    }
     if (tc <= 16 && MODE != EPI_JACOBI_NORM && MODE != EPI_RES_X0) {  // tensor-core routes (L222-228)
         const int per_sm_cap = 8;  // 256-thread CTAs: persistent grid over the rows
         if constexpr (sizeof(MatT) == 8) {

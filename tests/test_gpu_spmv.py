@@ -244,3 +244,47 @@ def test_vcycle_with_tensor_core_spmv(prec):
         res, res_o = np.array(res), np.array(res_o)
         rho, rho_o = res[1:] / res[:-1], res_o[1:] / res_o[:-1]
         assert np.all(np.abs(rho - rho_o) <= 0.01 * rho_o), (rho, rho_o)
+
+
+def _long_row_ragged(n=1536, seed=11):
+    """Rows of 1..17 entries spread over the whole column range (block rows of ~4-60 tiles, mean
+    >= 16): the warp-per-row kernel's loop over several 32-tile batches and its near-empty rows."""
+    rng = np.random.default_rng(seed)
+    rp, cols = [0], []
+    for i in range(n):
+        k = 0 if i % 97 == 5 else int(rng.integers(4, 17))
+        c = np.unique(np.concatenate([[i], rng.integers(0, n, size=k)]))
+        cols.append(c)
+        rp.append(rp[-1] + len(c))
+    col = np.concatenate(cols).astype(np.int32)
+    val = np.round(rng.uniform(-4, 4, size=len(col))) / 4
+    return gen.CSR(n, n, torch.tensor(rp, dtype=torch.int64), torch.from_numpy(col), torch.from_numpy(val))
+
+
+@pytest.mark.parametrize("prec", ["f32", "f16"])
+@pytest.mark.parametrize("name,mk", [("27pt_16", lambda: gen.laplacian_27pt(16)), ("long_ragged", _long_row_ragged)])
+def test_spmv_warp_per_row(prec, name, mk):
+    """FP32 / FP16 operators with >= 16 tiles per block row and <= 65,536 block columns take the
+    warp-per-row kernel (k_spmv_wrow): dyadic data with few significant bits is exact in FP16 and
+    FP32 with FP32 accumulation; every fused epilogue equals its definition on the plain product."""
+    amgt = _amgt()
+    A = mk()
+    Ao = oracle.as_csr(A)
+    M = amgt.from_csr(A, prec=prec).analyze()
+    assert M.blc_num / M.blc_row >= 16
+    x = (gen.integer_vector(A.n, 13).numpy() / 4).astype(np.float32)
+    y = amgt.spmv(M, torch.from_numpy(x).cuda(), torch.zeros(4 * M.blc_row, dtype=torch.float32,
+                                                                device="cuda")).cpu().numpy()
+    assert np.array_equal(y[:A.m].astype(np.float64), oracle.spmv(Ao, x.astype(np.float64)))
+    n4 = 4 * M.blc_row
+    xv = torch.zeros(n4, dtype=torch.float32, device="cuda")
+    xv[:A.m] = torch.from_numpy(x[:A.m])
+    t = torch.from_numpy(y).cuda()
+    b = torch.from_numpy((gen.integer_vector(n4, 5).numpy() / 8).astype(np.float32)).cuda()
+    d = torch.full((n4,), 0.25, dtype=torch.float32, device="cuda")
+    w = torch.tensor(2.0 / 3.0, dtype=torch.float32)
+    for mode in ("jacobi", "residual", "accum"):
+        out = torch.from_numpy((gen.integer_vector(n4, 7).numpy() / 2).astype(np.float32)).cuda()
+        ref = {"jacobi": xv + w.item() * d * (b - t), "residual": b - t, "accum": out + t}[mode]
+        amgt.spmv_fused(M, xv, out, mode, b=b, dinv=d)
+        assert torch.allclose(out[:A.m], ref[:A.m], rtol=1e-6, atol=1e-6), mode
