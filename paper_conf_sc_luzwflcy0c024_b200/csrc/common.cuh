@@ -62,6 +62,8 @@ struct Alloc {
 // caller sees use the amgt_allocator, scratch does not need to cross the ABI.
 void* scratch_get(size_t bytes, cudaStream_t s);
 void scratch_put(void* p, cudaStream_t s);
+// drops the SpGEMM numeric plan keyed by a C structure array being released (spgemm.cu)
+void spgemm_plan_drop(const void* key, cudaStream_t s);
 
 template <typename T>
 struct Scratch {

@@ -438,6 +438,7 @@ amgt_status mbsr_release(amgt_mbsr* M, Alloc& a) {
     if (!M) return AMGT_OK;
     if (M->aux) spmv_plan_free(M->aux, a);
     if (M->own & 1u) {
+        spgemm_plan_drop(M->blc_idx, a.s);
         a.put(M->blc_ptr, (M->blc_row + 1) * sizeof(int64_t));
         a.put(M->blc_idx, M->blc_num * sizeof(int32_t));
         a.put(M->blc_map, ((M->blc_num + 1) & ~int64_t(1)) * sizeof(uint16_t));

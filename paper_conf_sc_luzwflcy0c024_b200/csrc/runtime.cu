@@ -51,7 +51,7 @@ void Alloc::put(void* p, size_t bytes) {
 
 // Scratch comes from a library-owned stream-ordered pool (not the device default pool, which
 // torch or the caller may configure).  Freed scratch stays cached up to a release threshold
-// (AMGT_SCRATCH_CACHE_MB, default 1024 MB); beyond it the pool returns memory to the device at
+// (AMGT_SCRATCH_CACHE_MB, default 4096 MB); beyond it the pool returns memory to the device at
 // the next synchronisation, so large transient buffers (SpGEMM candidate lists, hash tables)
 // do not stay reserved for the life of the process.
 static cudaMemPool_t scratch_pool() {
@@ -72,7 +72,7 @@ static cudaMemPool_t scratch_pool() {
             return nullptr;
         }
         const char* e = getenv("AMGT_SCRATCH_CACHE_MB");
-        uint64_t thr = (uint64_t)(e ? atoll(e) : 1024) << 20;
+        uint64_t thr = (uint64_t)(e ? atoll(e) : 4096) << 20;
         cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
         pools[dev] = p;
     }

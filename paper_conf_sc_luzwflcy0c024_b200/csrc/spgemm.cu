@@ -24,8 +24,12 @@
 #include <cmath>
 #include <climits>
 #include <cstring>
+#include <mutex>
+#include <vector>
 
 #include "common.cuh"
+
+#include <cub/block/block_radix_sort.cuh>
 
 namespace amgt {
 
@@ -174,10 +178,10 @@ __device__ __forceinline__ void warp_pairs(const SymCtx& c, int64_t I, int lane,
 }
 
 // Block-cooperative version: chunks of blockDim A tiles, owner search in shared memory.
+constexpr int PAIR_U = 4;
 template <typename F>
-__device__ __forceinline__ void block_pairs(const SymCtx& c, int64_t I, int64_t* sh_excl, int64_t* sh_b0,
-                                            uint32_t* sh_ma, int64_t* sh_tot, F&& fn) {
-    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+__device__ __forceinline__ void block_pairs_range(const SymCtx& c, int64_t a0, int64_t a1, int64_t* sh_excl,
+                                                  int64_t* sh_b0, uint32_t* sh_ma, int64_t* sh_tot, F&& fn) {
     const int nt = blockDim.x, tid = threadIdx.x;
     const int lane = tid & 31, w = tid >> 5, nw = nt >> 5;
     for (int64_t base = a0; base < a1; base += nt) {
@@ -209,18 +213,109 @@ __device__ __forceinline__ void block_pairs(const SymCtx& c, int64_t I, int64_t*
         const int64_t total = sh_tot[nw];
         __syncthreads();
         const int nvalid = (int)min((int64_t)nt, a1 - base);
-        for (int64_t p = tid; p < total; p += nt) {
-            int lo = 0, hi = nvalid - 1;  // largest o with excl[o] <= p
-            while (lo < hi) {
-                const int mid = (lo + hi + 1) >> 1;
-                if (sh_excl[mid] <= p) lo = mid; else hi = mid - 1;
+        // PAIR_U pairs per thread per round: their B-tile loads are all in flight together
+        for (int64_t p0 = tid; p0 < total; p0 += (int64_t)nt * PAIR_U) {
+            int lo_[PAIR_U];
+            int64_t j_[PAIR_U];
+            uint32_t mb_[PAIR_U];
+            int32_t J_[PAIR_U];
+#pragma unroll
+            for (int u = 0; u < PAIR_U; ++u) {
+                const int64_t p = p0 + (int64_t)u * nt;
+                int lo = 0, hi = nvalid - 1;  // largest o with excl[o] <= p
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (sh_excl[mid] <= p) lo = mid; else hi = mid - 1;
+                }
+                lo_[u] = lo;
+                j_[u] = p < total ? sh_b0[lo] + (p - sh_excl[lo]) : -1;
             }
-            const int64_t j = sh_b0[lo] + (p - sh_excl[lo]);
-            const uint32_t mc = bitmap_multiply(sh_ma[lo], c.bmap[j]);
-            if (mc) fn(c.bidx[j], mc);
+#pragma unroll
+            for (int u = 0; u < PAIR_U; ++u) {
+                mb_[u] = j_[u] >= 0 ? c.bmap[j_[u]] : 0u;
+                J_[u] = j_[u] >= 0 ? c.bidx[j_[u]] : 0;
+            }
+#pragma unroll
+            for (int u = 0; u < PAIR_U; ++u) {
+                const uint32_t mc = j_[u] >= 0 ? bitmap_multiply(sh_ma[lo_[u]], mb_[u]) : 0u;
+                if (mc) fn(J_[u], mc);
+            }
         }
         __syncthreads();
     }
+}
+// block_pairs_range that also hands fn the pair's A tile t, B tile j and aux(t) + (j - first
+// tile of B row K): aux(t, K) is evaluated once per A tile (the plan's record position base).
+template <typename G, typename F>
+__device__ __forceinline__ void block_pairs_aux(const SymCtx& c, int64_t a0, int64_t a1, int64_t* sh_excl,
+                                                int64_t* sh_b0, uint32_t* sh_ma, int64_t* sh_tot, int64_t* sh_aux,
+                                                G&& aux, F&& fn) {
+    const int nt = blockDim.x, tid = threadIdx.x;
+    const int lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    for (int64_t base = a0; base < a1; base += nt) {
+        const int64_t t = base + tid;
+        const bool v = t < a1;
+        const int32_t K = v ? c.aidx[t] : 0;
+        const uint32_t ma = v ? c.amap[t] : 0u;
+        const int64_t b0 = v ? c.bptr[K] : 0;
+        const int64_t len = v ? c.bptr[K + 1] - b0 : 0;
+        int64_t incl = len;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        if (lane == 31) sh_tot[w] = incl;
+        __syncthreads();
+        if (tid == 0) {
+            int64_t s = 0;
+            for (int k = 0; k < nw; ++k) { const int64_t x = sh_tot[k]; sh_tot[k] = s; s += x; }
+            sh_tot[nw] = s;
+        }
+        __syncthreads();
+        const int64_t excl = sh_tot[w] + incl - len;
+        sh_excl[tid] = excl;
+        sh_b0[tid] = b0;
+        sh_ma[tid] = ma;
+        sh_aux[tid] = v ? aux(t, K) : 0;
+        const int64_t total = sh_tot[nw];
+        __syncthreads();
+        const int nvalid = (int)min((int64_t)nt, a1 - base);
+        for (int64_t p0 = tid; p0 < total; p0 += (int64_t)nt * PAIR_U) {
+            int lo_[PAIR_U];
+            int64_t j_[PAIR_U], off_[PAIR_U];
+            uint32_t mb_[PAIR_U];
+            int32_t J_[PAIR_U];
+#pragma unroll
+            for (int u = 0; u < PAIR_U; ++u) {
+                const int64_t p = p0 + (int64_t)u * nt;
+                int lo = 0, hi = nvalid - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (sh_excl[mid] <= p) lo = mid; else hi = mid - 1;
+                }
+                lo_[u] = lo;
+                off_[u] = p - sh_excl[lo];
+                j_[u] = p < total ? sh_b0[lo] + off_[u] : -1;
+            }
+#pragma unroll
+            for (int u = 0; u < PAIR_U; ++u) {
+                mb_[u] = j_[u] >= 0 ? c.bmap[j_[u]] : 0u;
+                J_[u] = j_[u] >= 0 ? c.bidx[j_[u]] : 0;
+            }
+#pragma unroll
+            for (int u = 0; u < PAIR_U; ++u) {
+                const uint32_t mc = j_[u] >= 0 ? bitmap_multiply(sh_ma[lo_[u]], mb_[u]) : 0u;
+                if (mc) fn(J_[u], mc, base + lo_[u], j_[u], sh_aux[lo_[u]] + off_[u]);
+            }
+        }
+        __syncthreads();
+    }
+}
+template <typename F>
+__device__ __forceinline__ void block_pairs(const SymCtx& c, int64_t I, int64_t* sh_excl, int64_t* sh_b0,
+                                            uint32_t* sh_ma, int64_t* sh_tot, F&& fn) {
+    block_pairs_range(c, c.aptr[I], c.aptr[I + 1], sh_excl, sh_b0, sh_ma, sh_tot, fn);
 }
 
 // ---------------------------------------------------------------- step kernels: warp bins
@@ -306,7 +401,11 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
                                                   uint16_t* __restrict__ cmap, int64_t* __restrict__ bin_of,
                                                   unsigned long long* __restrict__ stats,
                                                   int32_t* __restrict__ sidx = nullptr,
-                                                  uint16_t* __restrict__ smap = nullptr) {
+                                                  uint16_t* __restrict__ smap = nullptr,
+                                                  const int64_t* __restrict__ pp = nullptr) {
+    // pp (optional): pair prefix over A tiles -> Cub(I) = pp[aptr[I+1]] - pp[aptr[I]] directly;
+    // the tiles of rows with Cub > SMALL_CUB (power-law rows of thousands of tiles) are then
+    // jumped over instead of walked.
     // row stride padded by one word: the 8 groups of a warp read the same position of 8
     // different rows at once (an unpadded 128-B stride puts them all in one bank)
     __shared__ int keys[8][SF_ROWS][SMALL_CUB + 1];
@@ -320,9 +419,33 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
     const int nr = (int)min((int64_t)SF_ROWS, BR - I0);
     const int64_t ap = lane <= nr ? c.aptr[I0 + lane] : 0;  // lane k: start of row I0 + k
     const int64_t T0 = __shfl_sync(0xffffffffu, ap, 0), T1 = __shfl_sync(0xffffffffu, ap, nr);
+    // lane k < nr: Cub of row I0 + k from pp (pp[ap] at lane k, pp[ap of k+1] from lane k+1)
+    int64_t pcub = 0;
+    if (pp) {
+        const int64_t pk = lane <= nr ? pp[ap] : 0;
+        const int64_t pk1 = __shfl_down_sync(0xffffffffu, pk, 1);
+        pcub = lane < nr ? pk1 - pk : 0;
+    }
+    const unsigned bigrows = __ballot_sync(0xffffffffu, pp != nullptr && lane < nr && pcub > SMALL_CUB);
     if (lane < SF_ROWS) npair[w][lane] = 0;
     __syncwarp();
     for (int64_t base = T0; base < T1; base += 32 * SF_U) {
+        if (bigrows) {  // warp-uniform: skip whole chunks that start inside a big row
+            int rb = 0;
+#pragma unroll
+            for (int k = 1; k < SF_ROWS; ++k) {
+                const int64_t sk = __shfl_sync(0xffffffffu, ap, k);
+                rb += (k < nr && sk <= base);
+            }
+            bool jumped = false;
+            while (rb < nr && ((bigrows >> rb) & 1u)) {
+                base = __shfl_sync(0xffffffffu, ap, rb + 1);  // start of the next row
+                ++rb;
+                jumped = true;
+            }
+            if (base >= T1) break;
+            (void)jumped;
+        }
         int32_t K[SF_U];
         uint32_t ma[SF_U];
         int64_t b0[SF_U];
@@ -379,7 +502,8 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
         const int gr = g + 8 * h;
         const bool own = gr < nr;
         const int64_t I = I0 + gr;
-        const int64_t cub = own ? npair[w][gr] : 0;
+        const int64_t pc = __shfl_sync(0xffffffffu, pcub, gr);
+        const int64_t cub = own ? (pp ? pc : (int64_t)npair[w][gr]) : 0;
         bool small = false;
         if (STEP == 1) {
             int b = 0;
@@ -542,7 +666,8 @@ __global__ void __launch_bounds__(256) k_sym_copy(int64_t BR, const int64_t* __r
 // ---------------------------------------------------------------- step kernels: block bins
 template <int LOGS, int STEP>
 __global__ void k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c, int64_t* __restrict__ nnz_row,
-                            const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
+                            const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap,
+                            int jbits) {
     constexpr int S = 1 << LOGS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     // layout: keys[S] | maps[S] | list u64[S/2] (step 2) ; pair-search scratch in static smem
@@ -573,6 +698,42 @@ __global__ void k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, Sym
                 int s = 0;
                 for (int k = 0; k < nw; ++k) s += sh_cnt[k];
                 nnz_row[I] = s;
+            }
+            __syncthreads();
+            continue;
+        }
+        if constexpr (LOGS <= 12) {
+            // sort the whole table as packed keys (J << 16 | map; empty slots = ~0 sort last)
+            // with a block radix sort over J's bits: no compress pass, ~nbits/4 passes instead
+            // of the log^2 N stages of a bitonic network (Alg. 3 line 14)
+            constexpr int THREADS = LOGS >= 12 ? 512 : 256;
+            constexpr int IPT = S / THREADS;
+            using Sorter = cub::BlockRadixSort<unsigned long long, THREADS, IPT>;
+            __shared__ typename Sorter::TempStorage rs_tmp;
+            unsigned long long kv[IPT];
+            int nv = 0;
+#pragma unroll
+            for (int u = 0; u < IPT; ++u) {
+                const int slot = tid * IPT + u;
+                const int k = keys[slot];
+                nv += k != EMPTY_KEY;
+                kv[u] = k != EMPTY_KEY ? (((unsigned long long)(uint32_t)k << 16) | (maps[slot] & 0xFFFFu)) : ~0ull;
+            }
+#pragma unroll
+            for (int d = 16; d; d >>= 1) nv += __shfl_xor_sync(0xffffffffu, nv, d);
+            if (lane == 0) sh_cnt[w] = nv;
+            __syncthreads();  // keys/maps read into registers; sh_cnt complete
+            int n = 0;
+            for (int q = 0; q < nw; ++q) n += sh_cnt[q];
+            Sorter(rs_tmp).Sort(kv, 16, 17 + jbits);  // one bit above J: empty slots (~0) last
+            const int64_t out = cptr[I];
+#pragma unroll
+            for (int u = 0; u < IPT; ++u) {
+                const int pos = tid * IPT + u;
+                if (pos < n) {
+                    cidx[out + pos] = (int32_t)(kv[u] >> 16);
+                    cmap[out + pos] = (uint16_t)(kv[u] & 0xFFFFu);
+                }
             }
             __syncthreads();
             continue;
@@ -693,6 +854,176 @@ __global__ void __launch_bounds__(512) k_sym_dense(int64_t nrows, const int32_t*
             atomicOr(reinterpret_cast<unsigned int*>(cmap) + (q >> 1), mc << (16 * (q & 1)));
         });
         __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------- dense rows, whole-GPU form
+// Same bitmap idea as k_sym_dense, with the row bitmaps in global memory (W words per dense
+// row) so that one row is spread over many CTAs: work items are (row, GD_CH consecutive A
+// tiles), each expanded by block_pairs_range.  Step 1 ORs the bit of every candidate column
+// J into its row's bitmap; k_gdense_count turns each bitmap into per-word exclusive prefix
+// counts and the row's distinct count (Alg. 3 lines 9-12); step 2 writes the columns in word
+// order (sorted by construction, line 14) and ORs each pair's bitmap product into its C tile
+// at rank(J) = prefix(word) + popcount of the lower bits (R15).  No per-row serial walk: the
+// 107K-pair rows of config 4 take ~400 items instead of one CTA.
+constexpr int GD_CH = 256;  // A tiles per work item (= the block size: one block_pairs round)
+
+__global__ void k_gdense_items(int64_t nd, const int32_t* __restrict__ rows, const int64_t* __restrict__ aptr,
+                               int64_t* __restrict__ nitem) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nd; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t I = rows[i];
+        nitem[i] = (aptr[I + 1] - aptr[I] + GD_CH - 1) / GD_CH;
+    }
+}
+
+__global__ void k_gdense_item_rows(int64_t nd, const int64_t* __restrict__ ioff, int32_t* __restrict__ item_row) {
+    for (int64_t i = blockIdx.x; i < nd; i += gridDim.x)
+        for (int64_t k = ioff[i] + threadIdx.x; k < ioff[i + 1]; k += blockDim.x) item_row[k] = (int32_t)i;
+}
+
+// Numeric plan records written by step 2 (band-major positions, see SpgemmPlan below).
+struct PlanRec {
+    const int64_t* pp;    // [TA+1] global pair prefix over A tiles
+    const int64_t* tl;    // [nd][nb+1] pair index of the row's first tile in band b
+    const int64_t* ioffB; // [nb*nd+1] band-major offsets of the (band, row) items
+    int64_t nd, BW;
+    int nb;
+    int4* rec;      // {C tile q, B tile j, A tile t, bitmap product}; q = -1: empty product
+    uint32_t* cnt;  // [TC] products per C tile
+};
+
+// mflag bit q <- C tile q takes more than one product
+__global__ void k_plan_mark(int64_t TC, const uint32_t* __restrict__ cnt, uint32_t* __restrict__ mflag) {
+    const int64_t nw = (TC + 31) / 32;
+    const int lane = threadIdx.x & 31;
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 32 * nw; q += (int64_t)gridDim.x * blockDim.x) {
+        const bool m = q < TC && cnt[q] > 1u;
+        const unsigned b = __ballot_sync(0xffffffffu, m);
+        if (lane == 0) mflag[q >> 5] = b;
+    }
+}
+
+template <int STEP>
+__global__ void __launch_bounds__(GD_CH) k_gdense_pairs(const int64_t* __restrict__ nitems_dev,
+                                                      const int32_t* __restrict__ item_row,
+                                                      const int64_t* __restrict__ ioff, const int32_t* __restrict__ rows,
+                                                      SymCtx c, int64_t W, uint32_t* __restrict__ gbm,
+                                                      uint32_t* __restrict__ gbm2,
+                                                      const uint32_t* __restrict__ gpre, const int64_t* __restrict__ cptr,
+                                                      uint32_t* __restrict__ cmap32, PlanRec pr,
+                                                      unsigned long long* __restrict__ npairs) {
+    __shared__ int64_t sh_excl[GD_CH], sh_b0[GD_CH], sh_tot[GD_CH / 32 + 1], sh_aux[GD_CH];
+    __shared__ uint32_t sh_ma[GD_CH];
+    const int64_t nitems = *nitems_dev;
+    for (int64_t item = blockIdx.x; item < nitems; item += gridDim.x) {
+        const int64_t li = item_row[item];
+        const int64_t I = rows[li];
+        const int64_t a0 = c.aptr[I] + (item - ioff[li]) * GD_CH;
+        const int64_t a1 = min(c.aptr[I + 1], a0 + GD_CH);
+        uint32_t* bm = gbm + li * W;
+        if (STEP == 1) {
+            if (npairs) {  // the item's (A tile, B tile) pairs: the plan's record count
+                const int64_t t = a0 + threadIdx.x;
+                unsigned long long len = 0;
+                if (t < a1) {
+                    const int32_t K = c.aidx[t];
+                    len = (unsigned long long)(c.bptr[K + 1] - c.bptr[K]);
+                }
+#pragma unroll
+                for (int d = 16; d; d >>= 1) len += __shfl_xor_sync(0xffffffffu, len, d);
+                if ((threadIdx.x & 31) == 0 && len) atomicAdd(npairs, len);
+            }
+            block_pairs_range(c, a0, a1, sh_excl, sh_b0, sh_ma, sh_tot,
+                              [&](int32_t J, uint32_t) { atomicOr(bm + (J >> 5), 1u << (J & 31)); });
+        } else {
+            const uint32_t* pre = gpre + li * W;
+            const int64_t c0 = cptr[I];
+            auto rank = [&](int32_t J) {
+                const int wd = J >> 5;
+                return c0 + pre[wd] + __popc(bm[wd] & ((1u << (J & 31)) - 1u));
+            };
+            if (pr.rec) {
+                const int64_t* tlr = pr.tl + li * (pr.nb + 1);
+                block_pairs_aux(
+                    c, a0, a1, sh_excl, sh_b0, sh_ma, sh_tot, sh_aux,
+                    [&](int64_t t, int32_t K) {
+                        const int b = (int)(K / pr.BW);
+                        return pr.ioffB[(int64_t)b * pr.nd + li] + (pr.pp[t] - tlr[b]);
+                    },
+                    [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
+                        const int64_t q = rank(J);
+                        atomicOr(cmap32 + (q >> 1), mc << (16 * (q & 1)));
+                        atomicAdd(pr.cnt + q, 1u);  // products per C tile (k_plan_mark)
+                        pr.rec[pos] = make_int4((int)q, (int)j, (int)t, (int)mc);
+                    });
+            } else {
+                block_pairs_range(c, a0, a1, sh_excl, sh_b0, sh_ma, sh_tot, [&](int32_t J, uint32_t mc) {
+                    const int64_t q = rank(J);
+                    atomicOr(cmap32 + (q >> 1), mc << (16 * (q & 1)));
+                });
+            }
+        }
+    }
+}
+
+// per dense row: exclusive prefix popcount per bitmap word (gpre) and the distinct count
+constexpr int GD_CNT_THREADS = 512;
+__global__ void __launch_bounds__(GD_CNT_THREADS) k_gdense_count(int64_t nd, const int32_t* __restrict__ rows, int64_t W,
+                                                                 const uint32_t* __restrict__ gbm,
+                                                                 uint32_t* __restrict__ gpre, int64_t* __restrict__ nnz_row) {
+    __shared__ uint32_t sh[GD_CNT_THREADS / 32 + 1];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    constexpr int NW = GD_CNT_THREADS / 32;
+    for (int64_t li = blockIdx.x; li < nd; li += gridDim.x) {
+        const uint32_t* bm = gbm + li * W;
+        uint32_t* pre = gpre + li * W;
+        uint32_t run = 0;
+        for (int64_t base = 0; base < W; base += GD_CNT_THREADS) {
+            const int64_t i = base + tid;
+            const uint32_t v = i < W ? (uint32_t)__popc(bm[i]) : 0u;
+            uint32_t incl = v;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                if (lane >= d) incl += y;
+            }
+            if (lane == 31) sh[w] = incl;
+            __syncthreads();
+            if (w == 0) {
+                const uint32_t x = lane < NW ? sh[lane] : 0u;
+                uint32_t xi = x;
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, xi, d);
+                    if (lane >= d) xi += y;
+                }
+                if (lane < NW) sh[lane] = xi - x;
+                if (lane == NW - 1) sh[NW] = xi;
+            }
+            __syncthreads();
+            if (i < W) pre[i] = run + sh[w] + incl - v;
+            run += sh[NW];
+            __syncthreads();
+        }
+        if (tid == 0) nnz_row[rows[li]] = run;
+    }
+}
+
+// step 2 columns: every set bit of word i of dense row li goes to cptr + gpre + its rank
+__global__ void k_gdense_out(int64_t nd, const int32_t* __restrict__ rows, int64_t W, const uint32_t* __restrict__ gbm,
+                             const uint32_t* __restrict__ gpre, const int64_t* __restrict__ cptr,
+                             int32_t* __restrict__ cidx) {
+    const int64_t n = nd * W;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t bits = gbm[i];
+        if (!bits) continue;
+        const int64_t li = i / W, wd = i - li * W;
+        int64_t q = cptr[rows[li]] + gpre[i];
+        while (bits) {
+            const int b = __ffs(bits) - 1;
+            bits &= bits - 1;
+            cidx[q++] = (int32_t)(32 * wd + b);
+        }
     }
 }
 
@@ -1775,7 +2106,7 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
     const int32_t* __restrict__ cidx_g, const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
     int32_t* __restrict__ big, unsigned long long* __restrict__ nbig, int32_t* __restrict__ lng,
     unsigned long long* __restrict__ nlng, int32_t* __restrict__ mid, unsigned long long* __restrict__ nmid,
-    int rpg) {
+    int rpg, const uint8_t* __restrict__ skip) {
     constexpr int TE = 16;                       // elements per tile
     constexpr int PIECES = TE * sizeof(T) / 16;  // 16-B pieces per tile
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -1797,7 +2128,9 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         rc0 = cptr[Ir];
         rnC = (int)(cptr[Ir + 1] - rc0);
         ra0 = c.aptr[Ir];
-        if (rnC > GROUP_NC) {
+        if (skip && skip[Ir]) {
+            rnC = 0;  // computed from the symbolic phase's records (SpgemmPlan)
+        } else if (rnC > GROUP_NC) {
             if (rnC <= CAP) big[atomicAdd(nbig, 1ull)] = (int32_t)Ir;
             else if (rnC <= MIDCAP) mid[atomicAdd(nmid, 1ull)] = (int32_t)Ir;
             else lng[atomicAdd(nlng, 1ull)] = (int32_t)Ir;
@@ -1879,8 +2212,32 @@ __global__ void __launch_bounds__(STAGED_WARPS * 32) k_numeric_staged(
         uint32_t ma;
         int row;
     };
+    // first chunk base >= b that lies in a row of this kernel: the A tiles of rows handed to the
+    // other kernels (rn = 0; power-law rows of thousands of tiles) are jumped over, not walked
+    auto skip_rows = [&](int64_t b) {
+        for (;;) {
+            if (b >= A1) return b;
+            int ri = 0;
+#pragma unroll
+            for (int u = 1; u < STAGED_RPG; ++u) ri += (u < nrows && rs[u] <= b);
+            int rnc = 0;
+            int64_t nxt = A1;
+#pragma unroll
+            for (int u = 0; u < STAGED_RPG; ++u) {
+                rnc = (u == ri) ? rn[u] : rnc;
+                nxt = (u == ri + 1 && u < nrows) ? rs[u] : nxt;
+            }
+            if (rnc > 0) return b;
+            b = nxt;
+        }
+    };
     auto issue = [&](int nb, Batch& B, uint32_t& bm, int32_t& bj) {
-        while (pos >= S && cbase + 4 < A1) load_chunk(cbase + 4);  // group-uniform
+        while (pos >= S) {  // group-uniform
+            const int64_t nbse = skip_rows(cbase + 4);
+            if (nbse >= A1) break;
+            if (nbse != cbase + 4) prefetch(nbse);
+            load_chunk(nbse);
+        }
         const bool has = pos < S;
         const int p = pos + r;
         B.valid = has && p < S;
@@ -2028,14 +2385,16 @@ static amgt_status launch_warp_bin(int64_t n, const int32_t* rows, const SymCtx&
 
 template <int LOGS, int STEP>
 static amgt_status launch_block_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t* nnz_row,
-                                    const int64_t* cptr, int32_t* cidx, uint16_t* cmap, cudaStream_t s) {
+                                    const int64_t* cptr, int32_t* cidx, uint16_t* cmap, int64_t BCB, cudaStream_t s) {
+    int jbits = 1;  // bits of a tile column (the radix sort's key width)
+    while (jbits < 31 && ((int64_t)1 << jbits) < BCB) ++jbits;
     if (n == 0) return AMGT_OK;
     constexpr int S = 1 << LOGS;
     const size_t sm = (size_t)S * 4 * 2 + (STEP == 2 ? (size_t)S / 2 * 8 : 0);
     const int threads = LOGS >= 12 ? 512 : 256;
     auto kern = k_sym_block<LOGS, STEP>;
     AMGT_CUDA(dyn_smem(kern, sm));
-    kern<<<capped(n), threads, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap);
+    kern<<<capped(n), threads, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap, jbits);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
@@ -2063,33 +2422,298 @@ static amgt_status launch_dense_bin(int64_t n, const int32_t* rows, const SymCtx
     return AMGT_OK;
 }
 
+// State of the whole-GPU dense rows between symbolic steps 1 and 2 (row bitmaps, prefixes, items).
+struct GDense {
+    bool on = false;
+    bool plan = false;      // leave numeric records for the dense rows (SpgemmPlan)
+    int dense_from = 7;
+    int64_t nd = 0, W = 0;
+    int64_t cub_total = 0;  // all (A tile, B tile) pairs
+    unsigned long long* npairs_dev = nullptr;  // pairs of the dense rows (counted in step 1)
+    int64_t npairs = -1;                       // ... read back with the C tile count
+    int64_t TB = 0, BRB = 0, vbytes = 8;
+    const int64_t* pp = nullptr;  // pair prefix over A tiles, when computed before step 1
+    Scratch<uint32_t> bm, pre;
+    Scratch<int64_t> nitem, ioff;
+    Scratch<int32_t> item_row;
+};
+
+// ---------------------------------------------------------------- numeric plan of the dense rows
+// The whole-GPU symbolic step 2 already resolves, for every (A tile, B tile) pair of the dense
+// rows, the rank of its C tile (the bitmap prefix of R15).  It records (C tile q, B tile j, A
+// tile t) per pair and flags the C tiles that take more than one product, the way a two-phase
+// SpGEMM keeps its work buffers between the phases (cuSPARSE's SpGEMM keeps a user buffer):
+// the numeric phase of these rows is then one streaming pass with no searches.  Records are
+// stored band-major: the pairs of all dense rows whose A column K (= B row) lies in band b
+// precede those of band b + 1, so the B rows the concurrently running CTAs read are one band
+// (~24 MB, L2-resident) instead of all of B.  A plan is keyed by C's blc_idx pointer, consumed
+// by the first amgt_spgemm_numeric on that C (a second call recomputes) and dropped when C's
+// structure is released.
+struct SpgemmPlan {
+    const void* key = nullptr;
+    const int64_t* aptr = nullptr;
+    const int32_t* aidx = nullptr;
+    const int64_t* bptr = nullptr;
+    int64_t BR = 0, TC = 0;
+    int64_t* np = nullptr;  // device: number of records
+    int4* rec = nullptr;    // records (PlanRec)
+    size_t bytes = 0;       // device bytes held
+    uint32_t* mflag = nullptr;  // bit q: C tile q takes several products
+    uint8_t* rowf = nullptr;    // per C block row: 1 = computed from the records
+};
+
+static std::mutex g_plan_mu;
+static std::vector<SpgemmPlan*> g_plans;
+constexpr size_t MAX_PLANS = 4;
+constexpr size_t MAX_PLAN_BYTES = (size_t)2 << 30;  // least recently built plans dropped beyond
+
+static void plan_free(SpgemmPlan* P, cudaStream_t s) {
+    if (!P) return;
+    scratch_put(P->np, s);
+    scratch_put(P->rec, s);
+    scratch_put(P->mflag, s);
+    scratch_put(P->rowf, s);
+    delete P;
+}
+
+static void plan_put(SpgemmPlan* P, cudaStream_t s) {
+    std::vector<SpgemmPlan*> old;
+    {
+        std::lock_guard<std::mutex> lk(g_plan_mu);
+        for (size_t i = 0; i < g_plans.size();)
+            if (g_plans[i]->key == P->key) { old.push_back(g_plans[i]); g_plans.erase(g_plans.begin() + i); }
+            else ++i;
+        g_plans.push_back(P);
+        size_t held = 0;
+        for (SpgemmPlan* q : g_plans) held += q->bytes;
+        while (g_plans.size() > 1 && (g_plans.size() > MAX_PLANS || held > MAX_PLAN_BYTES)) {
+            held -= g_plans.front()->bytes;
+            old.push_back(g_plans.front());
+            g_plans.erase(g_plans.begin());
+        }
+    }
+    for (SpgemmPlan* q : old) plan_free(q, s);
+}
+
+static SpgemmPlan* plan_take(const void* key) {
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    for (size_t i = 0; i < g_plans.size(); ++i)
+        if (g_plans[i]->key == key) {
+            SpgemmPlan* P = g_plans[i];
+            g_plans.erase(g_plans.begin() + i);
+            return P;
+        }
+    return nullptr;
+}
+
+void spgemm_plan_drop(const void* key, cudaStream_t s) {
+    if (!key) return;
+    SpgemmPlan* P = plan_take(key);
+    if (P) plan_free(P, s);
+}
+
+// pairs per A tile (all tiles): the global pair index space of the records
+__global__ void k_plan_plen(int64_t TA, SymCtx c, int64_t* __restrict__ plen) {
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < TA; t += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t K = c.aidx[t];
+        plen[t] = c.bptr[K + 1] - c.bptr[K];
+    }
+}
+
+// tl[li][b] = pp of the first A tile of dense row li with column >= b * BW (b = 0..nb)
+__global__ void k_plan_bands(int64_t nd, int nb, int64_t BW, const int32_t* __restrict__ rows, SymCtx c,
+                             const int64_t* __restrict__ pp, int64_t* __restrict__ tl) {
+    const int64_t n = nd * (nb + 1);
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t li = i / (nb + 1);
+        const int b = (int)(i - li * (nb + 1));
+        const int64_t I = rows[li];
+        int64_t lo = c.aptr[I], hi = c.aptr[I + 1];
+        if (b < nb) {
+            const int64_t x = (int64_t)b * BW;
+            while (lo < hi) {
+                const int64_t mid = (lo + hi) >> 1;
+                if ((int64_t)c.aidx[mid] < x) lo = mid + 1; else hi = mid;
+            }
+        } else {
+            lo = hi;
+        }
+        tl[i] = pp[lo];
+    }
+}
+
+// band-major item sizes sz[b * nd + li] = pairs of row li in band b
+__global__ void k_plan_sizes(int64_t nd, int nb, const int64_t* __restrict__ tl, int64_t* __restrict__ sz) {
+    const int64_t n = nd * nb;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t b = i / nd, li = i - b * nd;
+        sz[i] = tl[li * (nb + 1) + b + 1] - tl[li * (nb + 1) + b];
+    }
+}
+
+__global__ void k_plan_rowf(int64_t nd, const int32_t* __restrict__ rows, uint8_t* __restrict__ rowf) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nd; i += (int64_t)gridDim.x * blockDim.x)
+        rowf[rows[i]] = 1;
+}
+
+template <int STEP>
+static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& c, int64_t BCB, int64_t TA, Alloc& a,
+                                 GDense& g, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
+                                 int64_t BR, int64_t TC, const void* key, cudaStream_t s) {
+    if (nd == 0) return AMGT_OK;
+    static int per_sm = 0;
+    if (!per_sm) {
+        AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_gdense_pairs<1>, GD_CH, 0));
+        per_sm = max(per_sm, 1);
+    }
+    const unsigned pgrid = (unsigned)(num_sms() * per_sm);
+    const int64_t W = g.W;
+    PlanRec pr{};
+    if (STEP == 1) {
+        g.nd = nd;
+        const int64_t cap_items = TA / GD_CH + nd + 1;  // >= sum over the rows of ceil(tiles / GD_CH)
+        AMGT_TRY(g.bm.init(a, (size_t)nd * W));
+        AMGT_TRY(g.pre.init(a, (size_t)nd * W));
+        AMGT_TRY(g.nitem.init(a, nd));
+        AMGT_TRY(g.ioff.init(a, nd + 1));
+        AMGT_TRY(g.item_row.init(a, (size_t)cap_items));
+        AMGT_CUDA(cudaMemsetAsync(g.bm.p, 0, (size_t)nd * W * sizeof(uint32_t), s));
+        k_gdense_items<<<capped(ceil_div(nd, 256)), 256, 0, s>>>(nd, rows, c.aptr, g.nitem.p);
+        AMGT_LAUNCHED();
+        AMGT_TRY(scan_exclusive(g.nitem.p, g.ioff.p, nd, a, s));
+        k_gdense_item_rows<<<capped(nd), 256, 0, s>>>(nd, g.ioff.p, g.item_row.p);
+        AMGT_LAUNCHED();
+        k_gdense_pairs<1><<<pgrid, GD_CH, 0, s>>>(g.ioff.p + nd, g.item_row.p, g.ioff.p, rows, c, W, g.bm.p,
+                                                nullptr, nullptr, nullptr, nullptr, pr,
+                                                g.plan ? g.npairs_dev : nullptr);
+        AMGT_LAUNCHED();
+        k_gdense_count<<<capped(nd), GD_CNT_THREADS, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, nnz_row);
+        AMGT_LAUNCHED();
+        return AMGT_OK;
+    }
+    // step 2 (+ the numeric plan when every index fits int32)
+    SpgemmPlan* P = nullptr;
+    Scratch<int64_t> plen, pp, tl, sz, ioffB;
+    Scratch<uint32_t> pcnt;
+    if (g.plan && TC < INT32_MAX && g.npairs > 0) {
+        static const double band_bytes = [] {
+            const char* e = getenv("AMGT_PLAN_BAND_MB");
+            return (e ? atof(e) : 24.0) * 1e6;
+        }();
+        const double row_bytes = g.BRB ? (double)g.TB / g.BRB * (16.0 * g.vbytes + 6.0) : 1.0;
+        int64_t BW = std::max<int64_t>(1, (int64_t)(band_bytes / std::max(row_bytes, 1.0)));
+        BW = std::max<int64_t>(BW, ceil_div(std::max<int64_t>(g.BRB, 1), 64));  // at most 64 bands
+        const int nb = (int)ceil_div(std::max<int64_t>(g.BRB, 1), BW);
+        P = new SpgemmPlan();
+        P->key = key;
+        P->aptr = c.aptr;
+        P->aidx = c.aidx;
+        P->bptr = c.bptr;
+        P->BR = BR;
+        P->TC = TC;
+        const size_t cap = (size_t)g.npairs;
+        const size_t nf = (size_t)ceil_div(TC, 32);
+        P->np = (int64_t*)scratch_get(sizeof(int64_t), s);
+        P->rec = (int4*)scratch_get(cap * sizeof(int4), s);
+        P->mflag = (uint32_t*)scratch_get(nf * sizeof(uint32_t), s);
+        P->rowf = (uint8_t*)scratch_get((size_t)BR, s);
+        P->bytes = cap * sizeof(int4) + nf * sizeof(uint32_t) + (size_t)BR;
+        const bool have_pp = g.pp != nullptr;
+        const bool ok = P->np && P->rec && P->mflag && P->rowf && (have_pp || (plen.try_init(a, TA) &&
+                        pp.try_init(a, TA + 1))) && tl.try_init(a, (size_t)nd * (nb + 1)) &&
+                        sz.try_init(a, (size_t)nd * nb) && ioffB.try_init(a, (size_t)nd * nb + 1) &&
+                        pcnt.try_init(a, (size_t)TC);
+        if (!ok) {
+            plan_free(P, s);
+            P = nullptr;
+        } else {
+            const int64_t* ppp = g.pp;
+            if (!have_pp) {
+                k_plan_plen<<<capped(ceil_div(TA, 256)), 256, 0, s>>>(TA, c, plen.p);
+                AMGT_LAUNCHED();
+                AMGT_TRY(scan_exclusive(plen.p, pp.p, TA, a, s));
+                ppp = pp.p;
+            }
+            k_plan_bands<<<capped(ceil_div(nd * (nb + 1), 256)), 256, 0, s>>>(nd, nb, BW, rows, c, ppp, tl.p);
+            AMGT_LAUNCHED();
+            k_plan_sizes<<<capped(ceil_div(nd * nb, 256)), 256, 0, s>>>(nd, nb, tl.p, sz.p);
+            AMGT_LAUNCHED();
+            AMGT_TRY(scan_exclusive(sz.p, ioffB.p, nd * nb, a, s));
+            AMGT_CUDA(cudaMemcpyAsync(P->np, ioffB.p + nd * nb, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+            AMGT_CUDA(cudaMemsetAsync(P->rec, 0xFF, cap * sizeof(int4), s));
+            AMGT_CUDA(cudaMemsetAsync(pcnt.p, 0, (size_t)TC * sizeof(uint32_t), s));
+            AMGT_CUDA(cudaMemsetAsync(P->rowf, 0, (size_t)BR, s));
+            k_plan_rowf<<<capped(ceil_div(nd, 256)), 256, 0, s>>>(nd, rows, P->rowf);
+            AMGT_LAUNCHED();
+            pr = PlanRec{ppp, tl.p, ioffB.p, nd, BW, nb, P->rec, pcnt.p};
+        }
+    }
+    k_gdense_out<<<capped(ceil_div(nd * W, 256)), 256, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, cptr, cidx);
+    AMGT_LAUNCHED();
+    k_gdense_pairs<2><<<pgrid, GD_CH, 0, s>>>(g.ioff.p + nd, g.item_row.p, g.ioff.p, rows, c, W, g.bm.p,
+                                            nullptr, g.pre.p, cptr, reinterpret_cast<uint32_t*>(cmap), pr, nullptr);
+    AMGT_LAUNCHED();
+    if (P) {
+        k_plan_mark<<<capped(ceil_div(TC, 256)), 256, 0, s>>>(TC, pcnt.p, P->mflag);
+        AMGT_LAUNCHED();
+    }
+    if (P) plan_put(P, s);
+    return AMGT_OK;
+}
+
 template <int STEP>
 static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_t* rows, const SymCtx& c, int64_t BCB,
-                            Alloc& a, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx, uint16_t* cmap,
-                            cudaStream_t s) {
+                            int64_t TA, Alloc& a, GDense& g, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx,
+                            uint16_t* cmap, int64_t BR, int64_t TC, const void* key, cudaStream_t s) {
     // Bins >= dense_from take the dense-bitmap kernel (a bitmap over B's W = BC/32 column
     // words: sorted by construction, cost ~ W + Cub per row) instead of a hash table + bitonic
     // sort (~ Cub log^2 Cub): from the first bin whose lower edge 128*2^(b-1) reaches W/16,
     // while the bitmap fits in shared memory (measured on config 4, W = 8192: bins >= 3
     // 2.2 ms symbolic vs 3.6 ms with bin 7 alone dense).  AMGT_DENSE_FROM_BIN overrides.
     static const int dense_env = [] { const char* e = getenv("AMGT_DENSE_FROM_BIN"); return e ? atoi(e) : -1; }();
+    // Whole-GPU form (global row bitmaps, k_gdense_*; AMGT_GDENSE=0 keeps k_sym_dense): from the
+    // first bin whose lower edge reaches W / 8 words (cost ~ W words per row of memset + scan +
+    // expansion against ~Cub pairs), while the bitmaps and prefixes stay under 4 GB.
+    static const int gd_env = [] { const char* e = getenv("AMGT_GDENSE"); return e ? atoi(e) : 1; }();
     const int64_t W = ceil_div(BCB, 32);
     int dense_from = 7;
-    if (W * 2 * (int64_t)sizeof(uint32_t) <= 160 * 1024)
-        for (int b = 2; b < 7; ++b)
-            if ((128ll << (b - 1)) * 16 >= W) { dense_from = b; break; }
-    if (dense_env >= 2 && dense_env <= 7) dense_from = dense_env;
+    if (STEP == 1) {
+        g.on = false;
+        g.W = W;
+        if (gd_env) {
+            for (int b = 2; b < 7; ++b)
+                if ((128ll << (b - 1)) * 8 >= W) { dense_from = b; break; }
+            if (dense_env >= 2 && dense_env <= 7) dense_from = dense_env;
+            int64_t nd = 0;
+            for (int b = dense_from; b < NBINS; ++b) nd += cnt[b];
+            g.on = (double)nd * W * 8.0 <= 4e9;
+            g.dense_from = dense_from;
+        }
+    }
+    if (g.on) {
+        dense_from = g.dense_from;
+    } else {
+        dense_from = 7;
+        if (W * 2 * (int64_t)sizeof(uint32_t) <= 160 * 1024)
+            for (int b = 2; b < 7; ++b)
+                if ((128ll << (b - 1)) * 16 >= W) { dense_from = b; break; }
+        if (dense_env >= 2 && dense_env <= 7) dense_from = dense_env;
+    }
     auto block_bin = [&](int b, auto launch) -> amgt_status { return b < dense_from ? launch() : AMGT_OK; };
     AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, s)));
     AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY(block_bin(2, [&] { return launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, s); }));
-    AMGT_TRY(block_bin(3, [&] { return launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, s); }));
-    AMGT_TRY(block_bin(4, [&] { return launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, s); }));
-    AMGT_TRY(block_bin(5, [&] { return launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, s); }));
-    AMGT_TRY(block_bin(6, [&] { return launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, s); }));
+    AMGT_TRY(block_bin(2, [&] { return launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
+    AMGT_TRY(block_bin(3, [&] { return launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
+    AMGT_TRY(block_bin(4, [&] { return launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
+    AMGT_TRY(block_bin(5, [&] { return launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
+    AMGT_TRY(block_bin(6, [&] { return launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
     int64_t nd = 0;  // bins dense_from..7 are contiguous in the row lists
     for (int b = dense_from; b < NBINS; ++b) nd += cnt[b];
-    AMGT_TRY((launch_dense_bin<STEP>(nd, rows + off[dense_from], c, BCB, a, nnz_row, cptr, cidx, cmap, s)));
+    if (g.on)
+        AMGT_TRY((launch_gdense<STEP>(nd, rows + off[dense_from], c, BCB, TA, a, g, nnz_row, cptr, cidx, cmap, BR, TC,
+                                      key, s)));
+    else
+        AMGT_TRY((launch_dense_bin<STEP>(nd, rows + off[dense_from], c, BCB, a, nnz_row, cptr, cidx, cmap, s)));
     return AMGT_OK;
 }
 
@@ -2108,6 +2732,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     Scratch<int64_t> bin_of, nnz_row;
     Scratch<unsigned long long> ctr;  // [0..15] stats (layout above) | [16..24] bin cursors | [25] longest C row
     Scratch<int32_t> rows;
+    GDense gd;  // whole-GPU dense rows (steps 1 and 2)
+    Scratch<int64_t> plen_s, pp_s;  // pair prefix over A tiles (rows longer than SMALL_CUB tiles)
     AMGT_TRY(bin_of.init(a, BR + 1));
     AMGT_TRY(nnz_row.init(a, BR + 1));
     AMGT_TRY(ctr.init(a, 32));
@@ -2156,8 +2782,17 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_LAUNCHED();
             }
         } else if (BR > 0) {
+            // rows of A longer than SMALL_CUB tiles: the pair prefix over A tiles first (Cub per row
+            // without a walk; reused by the whole-GPU dense rows' records)
+            if ((A->row_max == 0 || A->row_max > SMALL_CUB) && A->blc_num > 0 && plen_s.try_init(a, A->blc_num) &&
+                pp_s.try_init(a, A->blc_num + 1)) {
+                k_plan_plen<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, plen_s.p);
+                AMGT_LAUNCHED();
+                AMGT_TRY(scan_exclusive(plen_s.p, pp_s.p, A->blc_num, a, s));
+                gd.pp = pp_s.p;
+            }
             k_sym_flat<1><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nnz_row.p, nullptr, nullptr, nullptr,
-                                                                     bin_of.p, stats, sidx.p, smap.p);
+                                                                     bin_of.p, stats, sidx.p, smap.p, gd.pp);
             AMGT_LAUNCHED();
             if (info && A->blc_num > 0) {
                 k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats, g_tc_thr_spgemm);
@@ -2174,14 +2809,17 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 if (with_stats) AMGT_CUDA(cudaMemcpyAsync(ps, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(ps + 16, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(ps + 17, rmax, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaMemcpyAsync(ps + 18, ctr.p + 26, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaStreamSynchronize(s));
                 if (with_stats) memcpy(hs, ps, sizeof(hs));
                 TC = ps[16];
                 hmax = (unsigned long long)ps[17];
+                gd.npairs = ps[18];
             } else {
                 if (with_stats) AMGT_CUDA(cudaMemcpyAsync(hs, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
+                AMGT_CUDA(cudaMemcpyAsync(&gd.npairs, ctr.p + 26, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaStreamSynchronize(s));
             }
             return AMGT_OK;
@@ -2197,7 +2835,16 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             AMGT_TRY(rows.init(a, BR + 1));
             k_bin_scatter<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, stats, cursor, rows.p);
             AMGT_LAUNCHED();
-            amgt_status st = run_bins<1>(cnt_big, off, rows.p, c, B->blc_col, a, nnz_row.p, nullptr, nullptr, nullptr, s);
+            static const int plan_env = [] { const char* e = getenv("AMGT_SPGEMM_PLAN"); return e ? atoi(e) : 1; }();
+            gd.plan = plan_env && A->blc_num < INT32_MAX && B->blc_num < INT32_MAX &&
+                      (double)hs[8] * 12.0 <= 6e9;  // records: 12 B per pair
+            gd.cub_total = (int64_t)hs[8];
+            gd.npairs_dev = ctr.p + 26;
+            gd.TB = B->blc_num;
+            gd.BRB = B->blc_row;
+            gd.vbytes = (int64_t)prec_bytes(B->prec);
+            amgt_status st = run_bins<1>(cnt_big, off, rows.p, c, B->blc_col, A->blc_num, a, gd, nnz_row.p, nullptr,
+                                         nullptr, nullptr, BR, 0, nullptr, s);
             if (st != AMGT_OK) return st;
             AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
             AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
@@ -2216,7 +2863,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                                                                          C.blc_map, bin_of.p, nullptr);
             AMGT_LAUNCHED();
             if (big > 0) {
-                st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, a, nullptr, C.blc_ptr, C.blc_idx, C.blc_map, s);
+                st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, A->blc_num, a, gd, nullptr, C.blc_ptr, C.blc_idx,
+                                 C.blc_map, BR, TC, C.blc_idx, s);
                 if (st != AMGT_OK) return st;
             }
         }
@@ -2453,6 +3101,188 @@ static amgt_status launch_b1(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* 
     return AMGT_OK;
 }
 
+// ---------------------------------------------------------------- numeric: plan rows
+// Multi-product C tiles of the plan rows start at zero (the accumulation target: C values, or
+// the FP32 workspace for FP16).
+template <typename Acc>
+__global__ void k_plan_zero(int64_t TC, const uint32_t* __restrict__ mflag, Acc* __restrict__ acc) {
+    const int64_t nw = (TC + 31) / 32;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t f = mflag[i];
+        while (f) {
+            const int b = __ffs(f) - 1;
+            f &= f - 1;
+            uint4* v = reinterpret_cast<uint4*>(acc + 16 * (32 * i + b));
+#pragma unroll
+            for (int e = 0; e < (int)sizeof(Acc); ++e) v[e] = make_uint4(0u, 0u, 0u, 0u);
+        }
+    }
+}
+
+// One pass over the records, PLAN_R records per block of work: the records arrive in registers
+// one block ahead, the A and B tiles of a block are copied to shared memory with cp.async one
+// block ahead (double-buffered), and four threads per record each form one row of A_t * B_j
+// (the tile_mma arithmetic, k = 0..3).  A single-product tile is written with full-line
+// stores (the four threads' rows are one 128-B line for FP64; +0.0 at the clear bits, R2); a
+// multi-product tile takes REDs at its bitmap positions (zeroed by k_plan_zero).
+constexpr int PLAN_R = 64;  // records per block of work (4 threads each)
+template <typename T>
+__device__ __forceinline__ void cp_async16_g(void* smem, const void* gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+}
+// the same with an L2 eviction-priority policy (createpolicy)
+__device__ __forceinline__ void cp_async16_hint(void* smem, const void* gmem, uint64_t pol) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(sa), "l"(gmem), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// streaming (evict-first) row stores of the C tiles: the product is not read again here
+template <typename T> struct RowCS;
+template <> struct RowCS<double> {
+    static __device__ __forceinline__ void store(double* p, const double (&v)[4]) {
+        __stcs(reinterpret_cast<double2*>(p), make_double2(v[0], v[1]));
+        __stcs(reinterpret_cast<double2*>(p) + 1, make_double2(v[2], v[3]));
+    }
+};
+template <> struct RowCS<float> {
+    static __device__ __forceinline__ void store(float* p, const float (&v)[4]) {
+        __stcs(reinterpret_cast<float4*>(p), make_float4(v[0], v[1], v[2], v[3]));
+    }
+};
+template <> struct RowCS<__half> {
+    static __device__ __forceinline__ void store(__half* p, const float (&v)[4]) { RowIO<__half>::store(p, v); }
+};
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(const int64_t* __restrict__ np_dev, const int4* __restrict__ rec,
+                                                         const uint32_t* __restrict__ mflag,
+                                                         const T* __restrict__ aval, const T* __restrict__ bval,
+                                                         T* __restrict__ cval, Acc* __restrict__ gacc,
+                                                         int hints) {
+    constexpr int TE = 16;
+    constexpr int CH = 16 / (int)sizeof(T);       // elements per 16-B piece
+    constexpr int PC = TE / CH;                   // 16-B pieces per tile
+    constexpr int TS = TE + CH;                   // padded tile stride: the 8 records a warp reads
+                                                  // at once fall on different banks
+    __shared__ __align__(16) T sA[2][PLAN_R][TS];
+    __shared__ __align__(16) T sB[2][PLAN_R][TS];
+    __shared__ int4 sr[2][PLAN_R];
+    __shared__ int sa[2][PLAN_R];  // record whose A copy this record uses (runs of one A tile)
+    const int tid = threadIdx.x;
+    const int64_t total = *np_dev;
+    const int64_t nblk = (total + PLAN_R - 1) / PLAN_R;
+    Acc* acc = gacc ? gacc : reinterpret_cast<Acc*>(cval);
+    const uint64_t pol = policy_evict_last();
+    auto load_rec = [&](int64_t blk) {
+        int4 r = make_int4(-1, 0, 0, 0);
+        if (tid < PLAN_R && blk < nblk) {
+            const int64_t p = blk * PLAN_R + tid;
+            if (p < total) r = __ldg(rec + p);
+        }
+        return r;
+    };
+    auto stage = [&](int buf, const int4& r) {  // warps 0-1: record + A-run slot
+        if (tid < PLAN_R) {
+            const int lane = tid & 31;
+            const int zp = __shfl_up_sync(0xffffffffu, r.z, 1);
+            const unsigned bal = __ballot_sync(0xffffffffu, lane == 0 || r.x < 0 || r.z != zp);
+            sr[buf][tid] = r;
+            sa[buf][tid] = (tid & ~31) + 31 - __clz(bal & (0xffffffffu >> (31 - lane)));
+        }
+    };
+    auto issue = [&](int buf) {  // tiles of the records in sr[buf]
+        for (int k = tid; k < PLAN_R * 2 * PC; k += PLAN_R * 4) {
+            const int ri = k / (2 * PC), part = k - ri * 2 * PC;
+            const int4 r = sr[buf][ri];
+            if (r.x < 0) continue;
+            if (part < PC) {
+                if (sa[buf][ri] == ri) cp_async16_g<T>(&sA[buf][ri][part * CH], aval + 16 * (int64_t)r.z + part * CH);
+            } else if (hints & 1) {
+                cp_async16_hint(&sB[buf][ri][(part - PC) * CH], bval + 16 * (int64_t)r.y + (part - PC) * CH, pol);
+            } else {
+                cp_async16_g<T>(&sB[buf][ri][(part - PC) * CH], bval + 16 * (int64_t)r.y + (part - PC) * CH);
+            }
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    int64_t blk = blockIdx.x;
+    if (blk >= nblk) return;
+    stage(0, load_rec(blk));
+    __syncthreads();
+    issue(0);
+    int4 rnext = load_rec(blk + gridDim.x);
+    const int ri = tid >> 2, row = tid & 3;
+    for (int it = 0; blk < nblk; ++it, blk += gridDim.x) {
+        const int buf = it & 1;
+        const bool more = blk + gridDim.x < nblk;
+        if (more) {
+            stage(buf ^ 1, rnext);
+            __syncthreads();
+            issue(buf ^ 1);
+            rnext = load_rec(blk + 2 * (int64_t)gridDim.x);
+            asm volatile("cp.async.wait_group 1;" ::: "memory");
+        } else {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
+        __syncthreads();
+        const int4 r = sr[buf][ri];
+        if (r.x >= 0) {
+            Acc a4[4], o[4];
+            SRow<T>::load(&sA[buf][sa[buf][ri]][4 * row], a4);
+            Acc b0[4], b1[4], b2[4], b3[4];
+            SRow<T>::load(&sB[buf][ri][0], b0);
+            SRow<T>::load(&sB[buf][ri][4], b1);
+            SRow<T>::load(&sB[buf][ri][8], b2);
+            SRow<T>::load(&sB[buf][ri][12], b3);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                Acc v = a4[0] * b0[e];
+                v = fma_acc(a4[1], b1[e], v);
+                v = fma_acc(a4[2], b2[e], v);
+                v = fma_acc(a4[3], b3[e], v);
+                o[e] = v;
+            }
+            const uint32_t nib = ((uint32_t)r.w >> (4 * row)) & 0xFu;
+            const bool multi = (__ldg(mflag + (r.x >> 5)) >> (r.x & 31)) & 1u;
+            const int64_t q = r.x;
+            if (!multi) {
+#pragma unroll
+                for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? o[e] : Acc(0);
+                if (hints & 2) RowCS<T>::store(cval + 16 * q + 4 * row, o);
+                else RowIO<T>::store(cval + 16 * q + 4 * row, o);
+            } else {
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                    if ((nib >> e) & 1u) atomicAdd(acc + 16 * q + 4 * row + e, o[e]);
+            }
+        }
+        __syncthreads();  // buffer `buf` is refilled two iterations on
+    }
+}
+
+// FP16: round the multi-product tiles from the FP32 workspace (+0.0 where the bit is clear)
+template <typename T, typename Acc>
+__global__ void k_plan_finalize(int64_t TC, const uint32_t* __restrict__ mflag, const uint16_t* __restrict__ cmap,
+                                const Acc* __restrict__ gacc, T* __restrict__ cval) {
+    const int64_t nw = (TC + 31) / 32;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t f = mflag[i];
+        while (f) {
+            const int b = __ffs(f) - 1;
+            f &= f - 1;
+            const int64_t q = 32 * i + b;
+            const uint32_t mp = cmap[q];
+#pragma unroll
+            for (int e = 0; e < 16; ++e) cval[16 * q + e] = ((mp >> e) & 1u) ? from_acc<T>(gacc[16 * q + e]) : from_acc<T>(Acc(0));
+        }
+    }
+}
+
 template <typename T, typename Acc>
 static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, Alloc& a) {
     cudaStream_t s = a.s;
@@ -2471,6 +3301,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     // with the DMMA / HMMA routes.  AMGT_NUM_STAGED=0 forces the latter (measurement).
     static const int staged_env = [] { const char* e = getenv("AMGT_NUM_STAGED"); return e ? atoi(e) : 1; }();
     const bool tc_route = (sizeof(T) == 8 || sizeof(T) == 2) && g_tc_thr_spgemm <= 16;
+    // the symbolic phase's records for its dense rows (consumed here; used on the staged path)
+    SpgemmPlan* plan = plan_take(C->blc_idx);
+    struct PlanGuard {  // the plan stays with C (structure-only records) for later numeric calls
+        SpgemmPlan*& p;
+        cudaStream_t s;
+        ~PlanGuard() {
+            if (p) plan_put(p, s);
+        }
+    } plan_guard{plan, s};
+    if (plan && (tc_route || !staged_env || plan->aptr != A->blc_ptr || plan->aidx != A->blc_idx ||
+                 plan->bptr != B->blc_ptr || plan->TC != C->blc_num || plan->BR != BR)) {
+        plan_free(plan, s);
+        plan = nullptr;
+    }
     static const int b1_env = [] { const char* e = getenv("AMGT_NUM_B1"); return e ? atoi(e) : 1; }();
     if (!tc_route && b1_env && B->row_max == 1 && C->row_max > 0 && C->row_max <= GROUP_NC &&
         B->blc_num < ((int64_t)1 << 31)) {
@@ -2491,13 +3335,37 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         const int rpg = (int)std::max(1.0, std::min((double)STAGED_RPG, std::floor(32.0 / std::max(mp, 1.0))));
         kern<<<(unsigned)ceil_div(ceil_div(BR, 8 * rpg), STAGED_WARPS), STAGED_WARPS * 32, sm, s>>>(
             BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
-            big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, rpg);
+            big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, rpg, plan ? plan->rowf : nullptr);
     } else {
         k_numeric_group<T, Acc><<<(unsigned)ceil_div(ceil_div(BR, 8) * 32, 256), 256, 0, s>>>(
             BR, c, (const T*)A->blc_val, (const T*)B->blc_val, C->blc_ptr, C->blc_idx, C->blc_map, (T*)C->blc_val,
             big.p, nbig.p, lng.p, nbig.p + 1, mid.p, nbig.p + 3, g_tc_thr_spgemm);
     }
     AMGT_LAUNCHED();
+    if (plan) {  // the dense rows: one pass over the symbolic phase's records
+        Scratch<Acc> pacc;  // FP16: FP32 workspace of the multi-product tiles
+        if (sizeof(T) < sizeof(Acc)) AMGT_TRY(pacc.init(a, 16 * (size_t)C->blc_num));
+        Acc* acc = sizeof(T) < sizeof(Acc) ? pacc.p : reinterpret_cast<Acc*>(C->blc_val);
+        const int64_t nw = ceil_div(C->blc_num, 32);
+        k_plan_zero<Acc><<<capped(ceil_div(nw, 256)), 256, 0, s>>>(C->blc_num, plan->mflag, acc);
+        AMGT_LAUNCHED();
+        // L2 policies: bit 0 B tiles evict-last, bit 1 C stores evict-first (AMGT_PLAN_HINTS)
+        static const int plan_hints = [] { const char* e = getenv("AMGT_PLAN_HINTS"); return e ? atoi(e) : 3; }();
+        static int flat_per_sm = 0;
+        if (!flat_per_sm) {
+            AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&flat_per_sm, k_plan_flat<T, Acc>, PLAN_R * 4, 0));
+            flat_per_sm = max(flat_per_sm, 1);
+        }
+        k_plan_flat<T, Acc><<<(unsigned)(num_sms() * flat_per_sm), PLAN_R * 4, 0, s>>>(
+            plan->np, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
+            sizeof(T) < sizeof(Acc) ? pacc.p : nullptr, plan_hints);
+        AMGT_LAUNCHED();
+        if (sizeof(T) < sizeof(Acc)) {
+            k_plan_finalize<T, Acc><<<capped(ceil_div(nw, 256)), 256, 0, s>>>(C->blc_num, plan->mflag, C->blc_map,
+                                                                            pacc.p, (T*)C->blc_val);
+            AMGT_LAUNCHED();
+        }
+    }
     // row classes present (C->row_max from symbolic; 0 = unknown: launch everything)
     const int64_t rmax = C->row_max > 0 ? C->row_max : INT64_MAX;
     if (rmax <= GROUP_NC) return AMGT_OK;

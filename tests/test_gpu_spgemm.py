@@ -260,3 +260,24 @@ def test_spgemm_hash_and_dense_bins_agree(tmp_path, dense_from):
     assert np.array_equal(got["ptr"], Co.blc_ptr)
     assert np.array_equal(got["idx"], Co.blc_idx)
     assert np.array_equal(got["map"], Co.blc_map.astype(np.int32))
+
+
+def test_spgemm_plan_reused_after_value_change():
+    """The symbolic phase's numeric plan (records of the whole-GPU dense rows) depends on the
+    structure only: a second numeric call on the same C, and one after A's values are scaled in
+    place by 2, both match the oracle (the latter against 4x the product; power-of-two scaling is
+    exact) within the FP64 bound."""
+    amgt = _amgt()
+    A = gen.irregular_block_sparse(1 << 12, seed=11)
+    Ao = oracle.as_csr(A)
+    Co, Cabs = oracle.spgemm(Ao, Ao, with_abs=True)
+    M = amgt.from_csr(A)
+    C, info = amgt.spgemm(M, M, info=True)
+    assert sum(info["bin_rows"][2:]) > 0
+    _check_product(C, Co, Cabs)
+    amgt.spgemm_numeric(M, M, C)  # same inputs again
+    _check_product(C, Co, Cabs)
+    M.blc_val.mul_(2.0)
+    amgt.spgemm_numeric(M, M, C)
+    Co4 = oracle.Csr(Co.m, Co.n, Co.row_ptr, Co.col, 4.0 * Co.val)
+    _check_product(C, Co4, 4.0 * Cabs)

@@ -1,0 +1,9 @@
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r3; mkdir -p $O
+timeout 900 python -m pytest tests/test_gpu_spgemm.py -x -q -m gpu > $O/t_spgemm3.log 2>&1; tail -15 $O/t_spgemm3.log
+rm -f $O/cfg4_knobs3.txt
+for v in "AMGT_SPGEMM_PLAN=0" "AMGT_SPGEMM_PLAN=1" "AMGT_PLAN_BAND_MB=8" "AMGT_PLAN_BAND_MB=1000" "AMGT_DENSE_FROM_BIN=4" "AMGT_DENSE_FROM_BIN=3"; do
+  echo "$v $(env $v python tools/spgemm_time.py cfg4 5 2>&1 | tail -1)" >> $O/cfg4_knobs3.txt
+done
+cat $O/cfg4_knobs3.txt
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:'^k_' --csv --log-file $O/cfg4_launches4.csv python tools/profile_cfg4.py 2 > $O/cfg4_ncu4.log 2>&1
+python tools/ncu_sum_launches.py $O/cfg4_launches4.csv --per-launch > $O/cfg4_launches4.txt 2>&1

@@ -1,0 +1,9 @@
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r3; mkdir -p $O
+timeout 900 python -m pytest tests/test_gpu_spgemm.py -x -q -m gpu > $O/t_spgemm5.log 2>&1; tail -3 $O/t_spgemm5.log
+rm -f $O/cfg4_knobs5.txt
+for v in "AMGT_PLAN_HINTS=0" "AMGT_PLAN_HINTS=3" "AMGT_PLAN_HINTS=3 AMGT_PLAN_BAND_MB=1000"; do
+  echo "$v $(env $v python tools/spgemm_time.py cfg4 5 2>&1 | tail -1 | cut -c1-300)" >> $O/cfg4_knobs5.txt
+done
+cat $O/cfg4_knobs5.txt
+timeout 900 ncu --set full --clock-control none -k regex:'k_plan_flat' -c 1 -o $O/plan_flat_full2 python tools/profile_cfg4.py 1 > $O/ncu_pf2.log 2>&1
+ncu -i $O/plan_flat_full2.ncu-rep --page details --csv > $O/plan_flat_full2.csv 2>&1
