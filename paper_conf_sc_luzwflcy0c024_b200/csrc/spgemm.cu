@@ -25,6 +25,7 @@
 #include <climits>
 #include <cstring>
 #include <mutex>
+#include <type_traits>
 #include <vector>
 
 #include "common.cuh"
@@ -137,10 +138,12 @@ __device__ __forceinline__ bool hash_insert(int* keys, uint32_t* maps, int logS,
 
 // Warp-cooperative enumeration of the (A tile, B tile) pairs of block row I: lanes take
 // up to 32 A tiles, warp-scan their B-row lengths, then spread the pairs over lanes.
-// fn(J, mapC) is called for every pair with mapC != 0.
+// fn(J, mapC) is called for every pair with mapC != 0 — or fn(J, mapC, t, j, pos) with the
+// pair's A tile t, B tile j and its ordinal among the row's pairs (A-tile order, then B order).
 template <typename F>
 __device__ __forceinline__ void warp_pairs(const SymCtx& c, int64_t I, int lane, F&& fn) {
     const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+    int64_t rbase = 0;  // pairs of the previous 32-tile chunks
     for (int64_t base = a0; base < a1; base += 32) {
         const int64_t t = base + lane;
         const bool v = t < a1;
@@ -171,9 +174,14 @@ __device__ __forceinline__ void warp_pairs(const SymCtx& c, int64_t I, int lane,
             if (p < total) {
                 const int64_t j = ob0 + (p - oex);
                 const uint32_t mc = bitmap_multiply(oma, c.bmap[j]);
-                if (mc) fn(c.bidx[j], mc);
+                if constexpr (std::is_invocable_v<F, int32_t, uint32_t, int64_t, int64_t, int64_t>) {
+                    if (mc) fn(c.bidx[j], mc, base + lo, j, rbase + p);
+                } else {
+                    if (mc) fn(c.bidx[j], mc);
+                }
             }
         }
+        rbase += total;
     }
 }
 
@@ -245,13 +253,15 @@ __device__ __forceinline__ void block_pairs_range(const SymCtx& c, int64_t a0, i
     }
 }
 // block_pairs_range that also hands fn the pair's A tile t, B tile j and aux(t) + (j - first
-// tile of B row K): aux(t, K) is evaluated once per A tile (the plan's record position base).
+// tile of B row K): aux(t, K, pos0) is evaluated once per A tile (pos0: the ordinal of the
+// tile's first pair in the range; the plan's record position base).
 template <typename G, typename F>
 __device__ __forceinline__ void block_pairs_aux(const SymCtx& c, int64_t a0, int64_t a1, int64_t* sh_excl,
                                                 int64_t* sh_b0, uint32_t* sh_ma, int64_t* sh_tot, int64_t* sh_aux,
                                                 G&& aux, F&& fn) {
     const int nt = blockDim.x, tid = threadIdx.x;
     const int lane = tid & 31, w = tid >> 5, nw = nt >> 5;
+    int64_t rbase = 0;  // pairs of the previous chunks of the range
     for (int64_t base = a0; base < a1; base += nt) {
         const int64_t t = base + tid;
         const bool v = t < a1;
@@ -277,7 +287,7 @@ __device__ __forceinline__ void block_pairs_aux(const SymCtx& c, int64_t a0, int
         sh_excl[tid] = excl;
         sh_b0[tid] = b0;
         sh_ma[tid] = ma;
-        sh_aux[tid] = v ? aux(t, K) : 0;
+        sh_aux[tid] = v ? aux(t, K, rbase + excl) : 0;
         const int64_t total = sh_tot[nw];
         __syncthreads();
         const int nvalid = (int)min((int64_t)nt, a1 - base);
@@ -309,6 +319,7 @@ __device__ __forceinline__ void block_pairs_aux(const SymCtx& c, int64_t a0, int
                 if (mc) fn(J_[u], mc, base + lo_[u], j_[u], sh_aux[lo_[u]] + off_[u]);
             }
         }
+        rbase += total;
         __syncthreads();
     }
 }
@@ -318,13 +329,31 @@ __device__ __forceinline__ void block_pairs(const SymCtx& c, int64_t I, int64_t*
     block_pairs_range(c, c.aptr[I], c.aptr[I + 1], sh_excl, sh_b0, sh_ma, sh_tot, fn);
 }
 
+// Numeric plan records of the hash-bin rows with more than CAP C tiles (written by symbolic
+// step 2 after the sort): rec[hoff[I] + pos] for the row's pos-th pair (A-tile order, then B
+// order), products per C tile counted in cnt, rowf[I] = 1.
+struct HRec {
+    const int64_t* hoff;  // [BR+1] record offsets per row (0-length: no records)
+    int4* rec;
+    uint32_t* cnt;
+    uint8_t* rowf;
+};
+__device__ __forceinline__ int lower_pos(const int* keys, int n, int J) {  // keys ascending, J present
+    int lo = 0, hi = n - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (keys[mid] < J) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
 // ---------------------------------------------------------------- step kernels: warp bins
 // LOGS = log2(table slots per warp).  STEP 1: count -> nnz_row[I].  STEP 2: write sorted
 // idx/map at ptrC[I].
 template <int LOGS, int STEP>
 __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
                                                   int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
-                                                  int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap) {
+                                                  int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap, HRec hr) {
     constexpr int S = 1 << LOGS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -363,14 +392,28 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
         n += __popc(bal);
         __syncwarp();
     }
-    // rank sort (n <= S/2 distinct keys)
+    // rank sort (n <= S/2 distinct keys); the sorted keys also go to keys[S/2 ..)
     const int64_t out = cptr[I];
+    int* sorted = keys + S / 2;
     for (int i = lane; i < n; i += 32) {
         const int k = keys[i];
         int rank = 0;
         for (int j = 0; j < n; ++j) rank += keys[j] < k;
         cidx[out + rank] = k;
         cmap[out + rank] = (uint16_t)maps[i];
+        sorted[rank] = k;
+    }
+    if (hr.rec) {
+        const int64_t r0 = hr.hoff[I];
+        if (hr.hoff[I + 1] > r0) {  // records: C tile of every pair (third walk)
+            __syncwarp();
+            if (lane == 0) hr.rowf[I] = 1;
+            warp_pairs(c, I, lane, [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
+                const int64_t q = out + lower_pos(sorted, n, J);
+                atomicAdd(hr.cnt + q, 1u);
+                hr.rec[r0 + pos] = make_int4((int)q, (int)j, (int)t, (int)mc);
+            });
+        }
     }
 }
 
@@ -402,7 +445,8 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
                                                   unsigned long long* __restrict__ stats,
                                                   int32_t* __restrict__ sidx = nullptr,
                                                   uint16_t* __restrict__ smap = nullptr,
-                                                  const int64_t* __restrict__ pp = nullptr) {
+                                                  const int64_t* __restrict__ pp = nullptr,
+                                                  int64_t* __restrict__ cub_row = nullptr) {
     // pp (optional): pair prefix over A tiles -> Cub(I) = pp[aptr[I+1]] - pp[aptr[I]] directly;
     // the tiles of rows with Cub > SMALL_CUB (power-law rows of thousands of tiles) are then
     // jumped over instead of walked.
@@ -516,6 +560,7 @@ __global__ void __launch_bounds__(256) k_sym_flat(int64_t BR, SymCtx c, int64_t*
                 if (!small) {
                     nnz_row[I] = 0;  // counted by its bin's kernel
                     atomicAdd(&stats[cat_stat(b)], 1ull);
+                    if (cub_row) cub_row[I] = cub;
                 }
             }
             const unsigned n8 = __ballot_sync(0xffffffffu, lead && small);
@@ -667,14 +712,14 @@ __global__ void __launch_bounds__(256) k_sym_copy(int64_t BR, const int64_t* __r
 template <int LOGS, int STEP>
 __global__ void k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c, int64_t* __restrict__ nnz_row,
                             const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap,
-                            int jbits) {
+                            int jbits, HRec hr) {
     constexpr int S = 1 << LOGS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     // layout: keys[S] | maps[S] | list u64[S/2] (step 2) ; pair-search scratch in static smem
     int* keys = reinterpret_cast<int*>(smem_raw);
     uint32_t* maps = reinterpret_cast<uint32_t*>(keys + S);
     unsigned long long* list = reinterpret_cast<unsigned long long*>(maps + S);
-    __shared__ int64_t sh_excl[512], sh_b0[512], sh_tot[17];
+    __shared__ int64_t sh_excl[512], sh_b0[512], sh_tot[17], sh_aux[512];
     __shared__ uint32_t sh_ma[512];
     __shared__ int sh_cnt[17];
     const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, w = tid >> 5, nw = nt >> 5;
@@ -733,9 +778,24 @@ __global__ void k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, Sym
                 if (pos < n) {
                     cidx[out + pos] = (int32_t)(kv[u] >> 16);
                     cmap[out + pos] = (uint16_t)(kv[u] & 0xFFFFu);
+                    keys[pos] = (int)(kv[u] >> 16);  // sorted columns for the record walk
                 }
             }
             __syncthreads();
+            if (hr.rec) {
+                const int64_t r0 = hr.hoff[I];
+                if (hr.hoff[I + 1] > r0) {  // block-uniform: records (third walk)
+                    if (tid == 0) hr.rowf[I] = 1;
+                    block_pairs_aux(
+                        c, c.aptr[I], c.aptr[I + 1], sh_excl, sh_b0, sh_ma, sh_tot, sh_aux,
+                        [&](int64_t, int32_t, int64_t pos0) { return r0 + pos0; },
+                        [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
+                            const int64_t q = out + lower_pos(keys, n, J);
+                            atomicAdd(hr.cnt + q, 1u);
+                            hr.rec[pos] = make_int4((int)q, (int)j, (int)t, (int)mc);
+                        });
+                }
+            }
             continue;
         }
         // compress into list (packed key<<16 | map), block-wide ballot prefix per round
@@ -946,7 +1006,7 @@ __global__ void __launch_bounds__(GD_CH) k_gdense_pairs(const int64_t* __restric
                 const int64_t* tlr = pr.tl + li * (pr.nb + 1);
                 block_pairs_aux(
                     c, a0, a1, sh_excl, sh_b0, sh_ma, sh_tot, sh_aux,
-                    [&](int64_t t, int32_t K) {
+                    [&](int64_t t, int32_t K, int64_t) {
                         const int b = (int)(K / pr.BW);
                         return pr.ioffB[(int64_t)b * pr.nd + li] + (pr.pp[t] - tlr[b]);
                     },
@@ -1118,6 +1178,11 @@ template <> struct RowIO<__half> {
         *reinterpret_cast<uint2*>(p) = u;
     }
 };
+
+template <typename Acc, typename T> __device__ __forceinline__ Acc to_acc(T v) { return (Acc)v; }
+template <> __device__ __forceinline__ float to_acc<float, __half>(__half v) { return __half2float(v); }
+__device__ __forceinline__ double fma_acc(double a, double b, double c) { return fma(a, b, c); }
+__device__ __forceinline__ float fma_acc(float a, float b, float c) { return fmaf(a, b, c); }
 
 // C tile += A tile * B tile on CUDA cores (64 FMAs, fixed order k = 0..3).
 template <typename Acc>
@@ -1311,6 +1376,101 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
     }
 }
 
+// CUDA-core form of numeric_warp_row without per-lane tile products: the lanes resolve 32 pairs
+// of the row (A-tile order, then B order), then the two half-warps form them four at a time,
+// lane e = 4r+c computing entry (r,c) of A_t * B_j (A row r, B column c: the tile_mma order) —
+// the 16 lanes of a product read one A tile and one B tile with coalesced accesses, and the
+// loads of four products are in flight together.  The products are added into the row's
+// shared-memory accumulators in pair order (one half-warp at a time), so the sums are
+// bit-identical to numeric_warp_row's.
+template <typename T, typename Acc>
+__device__ __forceinline__ void numeric_warp_row_hw(int64_t I, const SymCtx& c, const T* __restrict__ aval,
+                                                    const T* __restrict__ bval, const int64_t* __restrict__ cptr,
+                                                    const int32_t* __restrict__ cidx_g,
+                                                    const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
+                                                    NumSmem<Acc>& S, int lane) {
+    const int64_t c0 = cptr[I];
+    const int nC = (int)(cptr[I + 1] - c0);
+    if (nC == 0) return;
+    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
+    if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
+    for (int e = lane; e < nC * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
+    __syncwarp();
+    const int h = lane >> 4, e = lane & 15, er = e >> 2, ec = e & 3;
+    for (int64_t base = a0; base < a1; base += 32) {
+        const int64_t t = base + lane;
+        const bool v = t < a1;
+        const uint32_t ma = v ? c.amap[t] : 0u;
+        const int32_t K = v ? c.aidx[t] : 0;
+        const int64_t b0 = v ? c.bptr[K] : 0;
+        const int64_t len = v ? c.bptr[K + 1] - b0 : 0;
+        int64_t incl = len;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        const int64_t excl = incl - len;
+        const int64_t total = __shfl_sync(0xffffffffu, incl, 31);
+        for (int64_t p0 = 0; p0 < total; p0 += 32) {
+            const int64_t p = p0 + lane;
+            int lo = 0;
+#pragma unroll
+            for (int step = 16; step; step >>= 1) {
+                const int cand = lo + step;
+                const int64_t ex = __shfl_sync(0xffffffffu, excl, cand & 31);
+                if (cand < 32 && ex <= p) lo = cand;
+            }
+            const int64_t ob0 = __shfl_sync(0xffffffffu, b0, lo);
+            const int64_t oex = __shfl_sync(0xffffffffu, excl, lo);
+            const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
+            int q = -1;
+            int64_t j = 0;
+            if (p < total) {
+                j = ob0 + (p - oex);
+                if (bitmap_multiply(oma, c.bmap[j])) q = bsearch_row(S.cidx, nC, c.bidx[j]);
+            }
+            const int64_t ta = base + lo;
+            const unsigned any = __ballot_sync(0xffffffffu, q >= 0);
+            for (int sr = 0; sr < 32; sr += 8) {
+                if (!((any >> sr) & 0xFFu)) continue;  // warp-uniform
+                int qq[4];
+                Acc prod[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int src = sr + 2 * u + h;
+                    qq[u] = __shfl_sync(0xffffffffu, q, src);
+                    const int64_t tu = __shfl_sync(0xffffffffu, ta, src);
+                    const int64_t ju = __shfl_sync(0xffffffffu, j, src);
+                    Acc ar[4], bc[4];
+                    if (qq[u] >= 0) {
+                        RowIO<T>::load(aval + 16 * tu + 4 * er, ar);
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) bc[k] = to_acc<Acc>(bval[16 * ju + 4 * k + ec]);
+                        Acc sv = ar[0] * bc[0];
+                        sv = fma_acc(ar[1], bc[1], sv);
+                        sv = fma_acc(ar[2], bc[2], sv);
+                        sv = fma_acc(ar[3], bc[3], sv);
+                        prod[u] = sv;
+                    }
+                }
+                // pair order: sr+0 (half 0), sr+1 (half 1), sr+2 (half 0), ...
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    if (h == (k & 1) && qq[k >> 1] >= 0) S.acc[qq[k >> 1]][e] += prod[k >> 1];
+                    __syncwarp();
+                }
+            }
+        }
+    }
+    __syncwarp();
+    for (int64_t x = lane; x < 16 * (int64_t)nC; x += 32) {  // +0.0 where the bitmap bit is clear (R2)
+        const int qx = (int)(x >> 4), b = (int)(x & 15);
+        const bool bit = (cmap_g[c0 + qx] >> b) & 1u;
+        cval[16 * c0 + x] = bit ? from_acc<T>(S.acc[qx][b]) : from_acc<T>(Acc(0));
+    }
+}
+
 // Warp per C block row for the rows in `rows` (count read from the device: the rows the
 // group kernel could not take, nC > GROUP_NC).  Persistent grid-stride over the list.
 template <typename T, typename Acc>
@@ -1324,8 +1484,10 @@ __global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(const int32_t* __res
     __shared__ NumSmem<Acc> sm[NUM_WARPS];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t nrows = (int64_t)*nrows_dev;
+    const bool hw = tc_thr > 16 || sizeof(T) == 4;  // every tile on CUDA cores: the half-warp form
     for (int64_t wi = (int64_t)blockIdx.x * NUM_WARPS + w; wi < nrows; wi += (int64_t)gridDim.x * NUM_WARPS) {
-        numeric_warp_row<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, gacc, tc_thr, sm[w], lane);
+        if (hw) numeric_warp_row_hw<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, sm[w], lane);
+        else numeric_warp_row<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, gacc, tc_thr, sm[w], lane);
         __syncwarp();
     }
 }
@@ -1364,10 +1526,6 @@ __device__ __forceinline__ int64_t warp_search_le(int64_t lo, int64_t hi, int64_
     }
     return lo;
 }
-template <typename Acc, typename T> __device__ __forceinline__ Acc to_acc(T v) { return (Acc)v; }
-template <> __device__ __forceinline__ float to_acc<float, __half>(__half v) { return __half2float(v); }
-__device__ __forceinline__ double fma_acc(double a, double b, double c) { return fma(a, b, c); }
-__device__ __forceinline__ float fma_acc(float a, float b, float c) { return fmaf(a, b, c); }
 
 constexpr int LONG_PAIRS = 2048;  // (A tile, B tile) pairs per work item of a long row
 constexpr int LONG_CTILES = 512;  // C tiles per finalising work item of a long row
@@ -2373,19 +2531,20 @@ static unsigned capped(int64_t blocks) {
 
 template <int LOGS, int STEP>
 static amgt_status launch_warp_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t* nnz_row, const int64_t* cptr,
-                                   int32_t* cidx, uint16_t* cmap, cudaStream_t s) {
+                                   int32_t* cidx, uint16_t* cmap, HRec hr, cudaStream_t s) {
     if (n == 0) return AMGT_OK;
     const size_t sm = (size_t)8 * 2 * (1 << LOGS) * sizeof(int);
     auto kern = k_sym_warp<LOGS, STEP>;
     AMGT_CUDA(dyn_smem(kern, sm));
-    kern<<<(unsigned)ceil_div(n * 32, 256), 256, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap);
+    kern<<<(unsigned)ceil_div(n * 32, 256), 256, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap, hr);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
 
 template <int LOGS, int STEP>
 static amgt_status launch_block_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t* nnz_row,
-                                    const int64_t* cptr, int32_t* cidx, uint16_t* cmap, int64_t BCB, cudaStream_t s) {
+                                    const int64_t* cptr, int32_t* cidx, uint16_t* cmap, int64_t BCB, HRec hr,
+                                    cudaStream_t s) {
     int jbits = 1;  // bits of a tile column (the radix sort's key width)
     while (jbits < 31 && ((int64_t)1 << jbits) < BCB) ++jbits;
     if (n == 0) return AMGT_OK;
@@ -2394,7 +2553,7 @@ static amgt_status launch_block_bin(int64_t n, const int32_t* rows, const SymCtx
     const int threads = LOGS >= 12 ? 512 : 256;
     auto kern = k_sym_block<LOGS, STEP>;
     AMGT_CUDA(dyn_smem(kern, sm));
-    kern<<<capped(n), threads, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap, jbits);
+    kern<<<capped(n), threads, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap, jbits, hr);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }
@@ -2422,17 +2581,21 @@ static amgt_status launch_dense_bin(int64_t n, const int32_t* rows, const SymCtx
     return AMGT_OK;
 }
 
+struct SpgemmPlan;
 // State of the whole-GPU dense rows between symbolic steps 1 and 2 (row bitmaps, prefixes, items).
 struct GDense {
     bool on = false;
     bool plan = false;      // leave numeric records for the dense rows (SpgemmPlan)
     int dense_from = 7;
+    int dense_from_eff = 7;  // the bins >= this took the dense kernels (either form)
     int64_t nd = 0, W = 0;
     int64_t cub_total = 0;  // all (A tile, B tile) pairs
     unsigned long long* npairs_dev = nullptr;  // pairs of the dense rows (counted in step 1)
     int64_t npairs = -1;                       // ... read back with the C tile count
     int64_t TB = 0, BRB = 0, vbytes = 8;
     const int64_t* pp = nullptr;  // pair prefix over A tiles, when computed before step 1
+    SpgemmPlan* P = nullptr;      // step 2: the plan receiving the dense rows' records
+    uint32_t* pcnt = nullptr;     // step 2: products per C tile
     Scratch<uint32_t> bm, pre;
     Scratch<int64_t> nitem, ioff;
     Scratch<int32_t> item_row;
@@ -2455,8 +2618,8 @@ struct SpgemmPlan {
     const int32_t* aidx = nullptr;
     const int64_t* bptr = nullptr;
     int64_t BR = 0, TC = 0;
-    int64_t* np = nullptr;  // device: number of records
-    int4* rec = nullptr;    // records (PlanRec)
+    int64_t nrec = 0;       // records: [0, dense pairs) band-major, then the hash-bin rows'
+    int4* rec = nullptr;    // records (PlanRec / HRec)
     size_t bytes = 0;       // device bytes held
     uint32_t* mflag = nullptr;  // bit q: C tile q takes several products
     uint8_t* rowf = nullptr;    // per C block row: 1 = computed from the records
@@ -2469,7 +2632,6 @@ constexpr size_t MAX_PLAN_BYTES = (size_t)2 << 30;  // least recently built plan
 
 static void plan_free(SpgemmPlan* P, cudaStream_t s) {
     if (!P) return;
-    scratch_put(P->np, s);
     scratch_put(P->rec, s);
     scratch_put(P->mflag, s);
     scratch_put(P->rowf, s);
@@ -2551,6 +2713,15 @@ __global__ void k_plan_sizes(int64_t nd, int nb, const int64_t* __restrict__ tl,
     }
 }
 
+// records of a hash-bin row (bin < hb_hi) with more than CAP C tiles: its Cub pairs
+__global__ void k_plan_hcount(int64_t BR, const int64_t* __restrict__ bin_of, const int64_t* __restrict__ nnz_row,
+                              const int64_t* __restrict__ cub_row, int hb_hi, int64_t* __restrict__ hcnt) {
+    for (int64_t I = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; I < BR; I += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t b = bin_of[I];
+        hcnt[I] = (b < hb_hi && nnz_row[I] > CAP) ? cub_row[I] : 0;
+    }
+}
+
 __global__ void k_plan_rowf(int64_t nd, const int32_t* __restrict__ rows, uint8_t* __restrict__ rowf) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nd; i += (int64_t)gridDim.x * blockDim.x)
         rowf[rows[i]] = 1;
@@ -2591,11 +2762,9 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
         AMGT_LAUNCHED();
         return AMGT_OK;
     }
-    // step 2 (+ the numeric plan when every index fits int32)
-    SpgemmPlan* P = nullptr;
+    // step 2 (+ the dense rows' records of the numeric plan, positions [0, npairs) band-major)
     Scratch<int64_t> plen, pp, tl, sz, ioffB;
-    Scratch<uint32_t> pcnt;
-    if (g.plan && TC < INT32_MAX && g.npairs > 0) {
+    if (g.P && g.plan && g.npairs > 0) {
         static const double band_bytes = [] {
             const char* e = getenv("AMGT_PLAN_BAND_MB");
             return (e ? atof(e) : 24.0) * 1e6;
@@ -2604,29 +2773,11 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
         int64_t BW = std::max<int64_t>(1, (int64_t)(band_bytes / std::max(row_bytes, 1.0)));
         BW = std::max<int64_t>(BW, ceil_div(std::max<int64_t>(g.BRB, 1), 64));  // at most 64 bands
         const int nb = (int)ceil_div(std::max<int64_t>(g.BRB, 1), BW);
-        P = new SpgemmPlan();
-        P->key = key;
-        P->aptr = c.aptr;
-        P->aidx = c.aidx;
-        P->bptr = c.bptr;
-        P->BR = BR;
-        P->TC = TC;
-        const size_t cap = (size_t)g.npairs;
-        const size_t nf = (size_t)ceil_div(TC, 32);
-        P->np = (int64_t*)scratch_get(sizeof(int64_t), s);
-        P->rec = (int4*)scratch_get(cap * sizeof(int4), s);
-        P->mflag = (uint32_t*)scratch_get(nf * sizeof(uint32_t), s);
-        P->rowf = (uint8_t*)scratch_get((size_t)BR, s);
-        P->bytes = cap * sizeof(int4) + nf * sizeof(uint32_t) + (size_t)BR;
         const bool have_pp = g.pp != nullptr;
-        const bool ok = P->np && P->rec && P->mflag && P->rowf && (have_pp || (plen.try_init(a, TA) &&
-                        pp.try_init(a, TA + 1))) && tl.try_init(a, (size_t)nd * (nb + 1)) &&
-                        sz.try_init(a, (size_t)nd * nb) && ioffB.try_init(a, (size_t)nd * nb + 1) &&
-                        pcnt.try_init(a, (size_t)TC);
-        if (!ok) {
-            plan_free(P, s);
-            P = nullptr;
-        } else {
+        const bool ok = (have_pp || (plen.try_init(a, TA) && pp.try_init(a, TA + 1))) &&
+                        tl.try_init(a, (size_t)nd * (nb + 1)) && sz.try_init(a, (size_t)nd * nb) &&
+                        ioffB.try_init(a, (size_t)nd * nb + 1);
+        if (ok) {
             const int64_t* ppp = g.pp;
             if (!have_pp) {
                 k_plan_plen<<<capped(ceil_div(TA, 256)), 256, 0, s>>>(TA, c, plen.p);
@@ -2639,13 +2790,12 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
             k_plan_sizes<<<capped(ceil_div(nd * nb, 256)), 256, 0, s>>>(nd, nb, tl.p, sz.p);
             AMGT_LAUNCHED();
             AMGT_TRY(scan_exclusive(sz.p, ioffB.p, nd * nb, a, s));
-            AMGT_CUDA(cudaMemcpyAsync(P->np, ioffB.p + nd * nb, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
-            AMGT_CUDA(cudaMemsetAsync(P->rec, 0xFF, cap * sizeof(int4), s));
-            AMGT_CUDA(cudaMemsetAsync(pcnt.p, 0, (size_t)TC * sizeof(uint32_t), s));
-            AMGT_CUDA(cudaMemsetAsync(P->rowf, 0, (size_t)BR, s));
-            k_plan_rowf<<<capped(ceil_div(nd, 256)), 256, 0, s>>>(nd, rows, P->rowf);
+            k_plan_rowf<<<capped(ceil_div(nd, 256)), 256, 0, s>>>(nd, rows, g.P->rowf);
             AMGT_LAUNCHED();
-            pr = PlanRec{ppp, tl.p, ioffB.p, nd, BW, nb, P->rec, pcnt.p};
+            pr = PlanRec{ppp, tl.p, ioffB.p, nd, BW, nb, g.P->rec, g.pcnt};
+        } else {
+            // no dense records: these rows' slots stay empty (q = -1) and they take the other kernels
+            g.plan = false;
         }
     }
     k_gdense_out<<<capped(ceil_div(nd * W, 256)), 256, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, cptr, cidx);
@@ -2653,18 +2803,13 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
     k_gdense_pairs<2><<<pgrid, GD_CH, 0, s>>>(g.ioff.p + nd, g.item_row.p, g.ioff.p, rows, c, W, g.bm.p,
                                             nullptr, g.pre.p, cptr, reinterpret_cast<uint32_t*>(cmap), pr, nullptr);
     AMGT_LAUNCHED();
-    if (P) {
-        k_plan_mark<<<capped(ceil_div(TC, 256)), 256, 0, s>>>(TC, pcnt.p, P->mflag);
-        AMGT_LAUNCHED();
-    }
-    if (P) plan_put(P, s);
     return AMGT_OK;
 }
 
 template <int STEP>
 static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_t* rows, const SymCtx& c, int64_t BCB,
                             int64_t TA, Alloc& a, GDense& g, int64_t* nnz_row, const int64_t* cptr, int32_t* cidx,
-                            uint16_t* cmap, int64_t BR, int64_t TC, const void* key, cudaStream_t s) {
+                            uint16_t* cmap, int64_t BR, int64_t TC, const void* key, HRec hr, cudaStream_t s) {
     // Bins >= dense_from take the dense-bitmap kernel (a bitmap over B's W = BC/32 column
     // words: sorted by construction, cost ~ W + Cub per row) instead of a hash table + bitonic
     // sort (~ Cub log^2 Cub): from the first bin whose lower edge 128*2^(b-1) reaches W/16,
@@ -2699,14 +2844,15 @@ static amgt_status run_bins(const int64_t* cnt, const int64_t* off, const int32_
                 if ((128ll << (b - 1)) * 16 >= W) { dense_from = b; break; }
         if (dense_env >= 2 && dense_env <= 7) dense_from = dense_env;
     }
+    g.dense_from_eff = dense_from;
     auto block_bin = [&](int b, auto launch) -> amgt_status { return b < dense_from ? launch() : AMGT_OK; };
-    AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, s)));
-    AMGT_TRY(block_bin(2, [&] { return launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
-    AMGT_TRY(block_bin(3, [&] { return launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
-    AMGT_TRY(block_bin(4, [&] { return launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
-    AMGT_TRY(block_bin(5, [&] { return launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
-    AMGT_TRY(block_bin(6, [&] { return launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, BCB, s); }));
+    AMGT_TRY((launch_warp_bin<8, STEP>(cnt[0], rows + off[0], c, nnz_row, cptr, cidx, cmap, hr, s)));
+    AMGT_TRY((launch_warp_bin<9, STEP>(cnt[1], rows + off[1], c, nnz_row, cptr, cidx, cmap, hr, s)));
+    AMGT_TRY(block_bin(2, [&] { return launch_block_bin<10, STEP>(cnt[2], rows + off[2], c, nnz_row, cptr, cidx, cmap, BCB, hr, s); }));
+    AMGT_TRY(block_bin(3, [&] { return launch_block_bin<11, STEP>(cnt[3], rows + off[3], c, nnz_row, cptr, cidx, cmap, BCB, hr, s); }));
+    AMGT_TRY(block_bin(4, [&] { return launch_block_bin<12, STEP>(cnt[4], rows + off[4], c, nnz_row, cptr, cidx, cmap, BCB, hr, s); }));
+    AMGT_TRY(block_bin(5, [&] { return launch_block_bin<13, STEP>(cnt[5], rows + off[5], c, nnz_row, cptr, cidx, cmap, BCB, HRec{}, s); }));
+    AMGT_TRY(block_bin(6, [&] { return launch_block_bin<14, STEP>(cnt[6], rows + off[6], c, nnz_row, cptr, cidx, cmap, BCB, HRec{}, s); }));
     int64_t nd = 0;  // bins dense_from..7 are contiguous in the row lists
     for (int b = dense_from; b < NBINS; ++b) nd += cnt[b];
     if (g.on)
@@ -2734,6 +2880,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     Scratch<int32_t> rows;
     GDense gd;  // whole-GPU dense rows (steps 1 and 2)
     Scratch<int64_t> plen_s, pp_s;  // pair prefix over A tiles (rows longer than SMALL_CUB tiles)
+    Scratch<int64_t> cub_row, hcnt, hoff;  // hash-bin rows: Cub, record counts and offsets
+    int64_t nH = 0;                        // records of the hash-bin rows (numeric plan)
     AMGT_TRY(bin_of.init(a, BR + 1));
     AMGT_TRY(nnz_row.init(a, BR + 1));
     AMGT_TRY(ctr.init(a, 32));
@@ -2791,8 +2939,10 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_TRY(scan_exclusive(plen_s.p, pp_s.p, A->blc_num, a, s));
                 gd.pp = pp_s.p;
             }
+            AMGT_TRY(cub_row.init(a, BR));
             k_sym_flat<1><<<(unsigned)ceil_div(BR, 8 * SF_ROWS), 256, 0, s>>>(BR, c, nnz_row.p, nullptr, nullptr, nullptr,
-                                                                     bin_of.p, stats, sidx.p, smap.p, gd.pp);
+                                                                     bin_of.p, stats, sidx.p, smap.p, gd.pp,
+                                                                     cub_row.p);
             AMGT_LAUNCHED();
             if (info && A->blc_num > 0) {
                 k_pair_stats<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, stats, g_tc_thr_spgemm);
@@ -2810,16 +2960,19 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_CUDA(cudaMemcpyAsync(ps + 16, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(ps + 17, rmax, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(ps + 18, ctr.p + 26, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                if (hoff.p) AMGT_CUDA(cudaMemcpyAsync(ps + 19, hoff.p + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaStreamSynchronize(s));
                 if (with_stats) memcpy(hs, ps, sizeof(hs));
                 TC = ps[16];
                 hmax = (unsigned long long)ps[17];
                 gd.npairs = ps[18];
+                if (hoff.p) nH = ps[19];
             } else {
                 if (with_stats) AMGT_CUDA(cudaMemcpyAsync(hs, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&gd.npairs, ctr.p + 26, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                if (hoff.p) AMGT_CUDA(cudaMemcpyAsync(&nH, hoff.p + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaStreamSynchronize(s));
             }
             return AMGT_OK;
@@ -2844,16 +2997,65 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             gd.BRB = B->blc_row;
             gd.vbytes = (int64_t)prec_bytes(B->prec);
             amgt_status st = run_bins<1>(cnt_big, off, rows.p, c, B->blc_col, A->blc_num, a, gd, nnz_row.p, nullptr,
-                                         nullptr, nullptr, BR, 0, nullptr, s);
+                                         nullptr, nullptr, BR, 0, nullptr, HRec{}, s);
             if (st != AMGT_OK) return st;
             AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
             AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
+            // hash-bin rows (bins < min(dense, 5): the kernels that sort in shared memory) with more
+            // than CAP C tiles: their pair counts -> record offsets
+            if (plan_env && cub_row.p && hcnt.try_init(a, BR) && hoff.try_init(a, BR + 1)) {
+                const int hb_hi = std::min(gd.dense_from_eff, 5);
+                k_plan_hcount<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, nnz_row.p, cub_row.p, hb_hi,
+                                                                      hcnt.p);
+                AMGT_LAUNCHED();
+                AMGT_TRY(scan_exclusive(hcnt.p, hoff.p, BR, a, s));
+            }
             AMGT_TRY(read_back(false));  // sync 2: C tile count with the long rows
         }
         amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
         if (st != AMGT_OK) return st;
         C.row_max = (int64_t)hmax;
         if (TC > 0) AMGT_CUDA(cudaMemsetAsync(C.blc_map, 0, ((TC + 1) & ~int64_t(1)) * sizeof(uint16_t), s));
+        // numeric plan: records of the whole-GPU dense rows ([0, npD), band-major) and of the
+        // hash-bin rows with more than CAP C tiles ([npD, npD + nH), row-major)
+        SpgemmPlan* P = nullptr;
+        Scratch<uint32_t> pcnt;
+        const int64_t npD = gd.on && gd.plan ? std::max<int64_t>(gd.npairs, 0) : 0;
+        if (big > 0 && TC > 0 && TC < INT32_MAX && npD + nH > 0 && A->blc_num < INT32_MAX && B->blc_num < INT32_MAX) {
+            P = new SpgemmPlan();
+            P->key = C.blc_idx;
+            P->aptr = A->blc_ptr;
+            P->aidx = A->blc_idx;
+            P->bptr = B->blc_ptr;
+            P->BR = BR;
+            P->TC = TC;
+            P->nrec = npD + nH;
+            const size_t nf = (size_t)ceil_div(TC, 32);
+            P->rec = (int4*)scratch_get((size_t)P->nrec * sizeof(int4), s);
+            P->mflag = (uint32_t*)scratch_get(nf * sizeof(uint32_t), s);
+            P->rowf = (uint8_t*)scratch_get((size_t)BR, s);
+            P->bytes = (size_t)P->nrec * sizeof(int4) + nf * sizeof(uint32_t) + (size_t)BR;
+            if (!P->rec || !P->mflag || !P->rowf || !pcnt.try_init(a, (size_t)TC)) {
+                plan_free(P, s);
+                P = nullptr;
+            } else {
+                AMGT_CUDA(cudaMemsetAsync(P->rec, 0xFF, (size_t)P->nrec * sizeof(int4), s));
+                AMGT_CUDA(cudaMemsetAsync(pcnt.p, 0, (size_t)TC * sizeof(uint32_t), s));
+                AMGT_CUDA(cudaMemsetAsync(P->rowf, 0, (size_t)BR, s));
+            }
+        }
+        gd.P = npD > 0 ? P : nullptr;
+        gd.pcnt = pcnt.p;
+        HRec hr{};
+        if (P && nH > 0) hr = HRec{hoff.p, P->rec + npD, pcnt.p, P->rowf};
+        struct PlanScope {  // the plan goes to the cache once step 2 has filled it (freed on errors)
+            SpgemmPlan*& P;
+            cudaStream_t s;
+            bool ok = false;
+            ~PlanScope() {
+                if (P && !ok) plan_free(P, s);
+            }
+        } pscope{P, s};
         if (BR > 0) {  // step 2 (Alg. 3 lines 13-14 + bitmap OR, R15)
             if (keep)
                 k_sym_copy<<<capped(ceil_div(4 * BR, 256)), 256, 0, s>>>(BR, bin_of.p, C.blc_ptr, sidx.p, smap.p,
@@ -2864,9 +3066,15 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             AMGT_LAUNCHED();
             if (big > 0) {
                 st = run_bins<2>(cnt_big, off, rows.p, c, B->blc_col, A->blc_num, a, gd, nullptr, C.blc_ptr, C.blc_idx,
-                                 C.blc_map, BR, TC, C.blc_idx, s);
+                                 C.blc_map, BR, TC, C.blc_idx, hr, s);
                 if (st != AMGT_OK) return st;
             }
+        }
+        if (P) {
+            k_plan_mark<<<capped(ceil_div(TC, 256)), 256, 0, s>>>(TC, pcnt.p, P->mflag);
+            AMGT_LAUNCHED();
+            pscope.ok = true;
+            plan_put(P, s);
         }
         ts.bytes = (A->blc_num + B->blc_num) * 6.0 * 2 + (A->blc_row + B->blc_row) * 8.0 + TC * 6.0 + (BR + 1) * 8.0;
     }
@@ -3159,7 +3367,7 @@ template <> struct RowCS<__half> {
     static __device__ __forceinline__ void store(__half* p, const float (&v)[4]) { RowIO<__half>::store(p, v); }
 };
 template <typename T, typename Acc>
-__global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(const int64_t* __restrict__ np_dev, const int4* __restrict__ rec,
+__global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(int64_t total, const int4* __restrict__ rec,
                                                          const uint32_t* __restrict__ mflag,
                                                          const T* __restrict__ aval, const T* __restrict__ bval,
                                                          T* __restrict__ cval, Acc* __restrict__ gacc,
@@ -3174,7 +3382,6 @@ __global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(const int64_t* __restr
     __shared__ int4 sr[2][PLAN_R];
     __shared__ int sa[2][PLAN_R];  // record whose A copy this record uses (runs of one A tile)
     const int tid = threadIdx.x;
-    const int64_t total = *np_dev;
     const int64_t nblk = (total + PLAN_R - 1) / PLAN_R;
     Acc* acc = gacc ? gacc : reinterpret_cast<Acc*>(cval);
     const uint64_t pol = policy_evict_last();
@@ -3262,6 +3469,133 @@ __global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(const int64_t* __restr
             }
         }
         __syncthreads();  // buffer `buf` is refilled two iterations on
+    }
+}
+
+// Bulk-copy (TMA 1-D, cp.async.bulk) form of k_plan_flat: per record, the thread owning it in
+// warps 0-1 arms the stage's mbarrier with its byte count and issues one bulk copy per tile (B,
+// and A at the start of a run of one A tile) — 1-2 instructions per record instead of sixteen
+// 16-B cp.async spread over the block, and the copies bypass the LSU/L1 request path.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(smem_u32(b)), "r"(parity)
+            : "memory");
+    }
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(b))
+                 : "memory");
+}
+
+template <typename T, typename Acc>
+__global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat_bulk(int64_t total, const int4* __restrict__ rec,
+                                                              const uint32_t* __restrict__ mflag,
+                                                              const T* __restrict__ aval, const T* __restrict__ bval,
+                                                              T* __restrict__ cval, Acc* __restrict__ gacc, int hints) {
+    constexpr int TE = 16;
+    constexpr int CH = 16 / (int)sizeof(T);
+    constexpr int TS = TE + CH;  // padded tile stride (bank spread), 16-B multiple
+    constexpr uint32_t TB = TE * sizeof(T);
+    __shared__ __align__(16) T sA[2][PLAN_R][TS];
+    __shared__ __align__(16) T sB[2][PLAN_R][TS];
+    __shared__ int4 sr[2][PLAN_R];
+    __shared__ int sa[2][PLAN_R];
+    __shared__ __align__(8) uint64_t mbar[2];
+    const int tid = threadIdx.x;
+    const int64_t nblk = (total + PLAN_R - 1) / PLAN_R;
+    Acc* acc = gacc ? gacc : reinterpret_cast<Acc*>(cval);
+    int64_t blk = blockIdx.x;
+    if (blk >= nblk) return;
+    if (tid == 0) {
+        mbar_init(&mbar[0], PLAN_R);
+        mbar_init(&mbar[1], PLAN_R);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    auto load_rec = [&](int64_t b) {
+        int4 r = make_int4(-1, 0, 0, 0);
+        if (tid < PLAN_R && b < nblk) {
+            const int64_t p = b * PLAN_R + tid;
+            if (p < total) r = __ldg(rec + p);
+        }
+        return r;
+    };
+    // warps 0-1: stage the record, its A-run slot, arm the barrier and issue its copies
+    auto produce = [&](int buf, const int4& r) {
+        if (tid < PLAN_R) {
+            const int lane = tid & 31;
+            const int zp = __shfl_up_sync(0xffffffffu, r.z, 1);
+            const unsigned bal = __ballot_sync(0xffffffffu, lane == 0 || r.x < 0 || r.z != zp);
+            const int slot = (tid & ~31) + 31 - __clz(bal & (0xffffffffu >> (31 - lane)));
+            sr[buf][tid] = r;
+            sa[buf][tid] = slot;
+            const bool own_a = r.x >= 0 && slot == tid;
+            const uint32_t bytes = r.x >= 0 ? TB * (own_a ? 2u : 1u) : 0u;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of the buffer
+            mbar_arrive_tx(&mbar[buf], bytes);
+            if (r.x >= 0) {
+                bulk_g2s(&sB[buf][tid][0], bval + 16 * (int64_t)r.y, TB, &mbar[buf]);
+                if (own_a) bulk_g2s(&sA[buf][tid][0], aval + 16 * (int64_t)r.z, TB, &mbar[buf]);
+            }
+        }
+    };
+    uint32_t par[2] = {0u, 0u};
+    produce(0, load_rec(blk));
+    int4 rnext = load_rec(blk + gridDim.x);
+    const int ri = tid >> 2, row = tid & 3;
+    for (int it = 0; blk < nblk; ++it, blk += gridDim.x) {
+        const int buf = it & 1;
+        if (blk + gridDim.x < nblk) {
+            produce(buf ^ 1, rnext);
+            rnext = load_rec(blk + 2 * (int64_t)gridDim.x);
+        }
+        mbar_wait(&mbar[buf], par[buf]);
+        par[buf] ^= 1u;
+        const int4 r = sr[buf][ri];
+        if (r.x >= 0) {
+            Acc a4[4], o[4];
+            SRow<T>::load(&sA[buf][sa[buf][ri]][4 * row], a4);
+            Acc b0[4], b1[4], b2[4], b3[4];
+            SRow<T>::load(&sB[buf][ri][0], b0);
+            SRow<T>::load(&sB[buf][ri][4], b1);
+            SRow<T>::load(&sB[buf][ri][8], b2);
+            SRow<T>::load(&sB[buf][ri][12], b3);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                Acc v = a4[0] * b0[e];
+                v = fma_acc(a4[1], b1[e], v);
+                v = fma_acc(a4[2], b2[e], v);
+                v = fma_acc(a4[3], b3[e], v);
+                o[e] = v;
+            }
+            const uint32_t nib = ((uint32_t)r.w >> (4 * row)) & 0xFu;
+            const bool multi = (__ldg(mflag + (r.x >> 5)) >> (r.x & 31)) & 1u;
+            const int64_t q = r.x;
+            if (!multi) {
+#pragma unroll
+                for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? o[e] : Acc(0);
+                if (hints & 2) RowCS<T>::store(cval + 16 * q + 4 * row, o);
+                else RowIO<T>::store(cval + 16 * q + 4 * row, o);
+            } else {
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                    if ((nib >> e) & 1u) atomicAdd(acc + 16 * q + 4 * row + e, o[e]);
+            }
+        }
+        __syncthreads();  // buffer `buf` is refilled by the next iteration's producers
     }
 }
 
@@ -3356,8 +3690,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
             AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&flat_per_sm, k_plan_flat<T, Acc>, PLAN_R * 4, 0));
             flat_per_sm = max(flat_per_sm, 1);
         }
+        static const int bulk_env = [] { const char* e = getenv("AMGT_PLAN_BULK"); return e ? atoi(e) : 0; }();  // measured slower (cfg4 1.80 vs 1.67 ms)
+        if (bulk_env) {
+            static int bulk_per_sm = 0;
+            if (!bulk_per_sm) {
+                AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bulk_per_sm, k_plan_flat_bulk<T, Acc>,
+                                                                        PLAN_R * 4, 0));
+                bulk_per_sm = max(bulk_per_sm, 1);
+            }
+            k_plan_flat_bulk<T, Acc><<<(unsigned)(num_sms() * bulk_per_sm), PLAN_R * 4, 0, s>>>(
+                plan->nrec, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
+                sizeof(T) < sizeof(Acc) ? pacc.p : nullptr, plan_hints);
+        } else
         k_plan_flat<T, Acc><<<(unsigned)(num_sms() * flat_per_sm), PLAN_R * 4, 0, s>>>(
-            plan->np, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
+            plan->nrec, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
             sizeof(T) < sizeof(Acc) ? pacc.p : nullptr, plan_hints);
         AMGT_LAUNCHED();
         if (sizeof(T) < sizeof(Acc)) {
