@@ -401,7 +401,7 @@ __global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* 
         for (int j = 0; j < n; ++j) rank += keys[j] < k;
         cidx[out + rank] = k;
         cmap[out + rank] = (uint16_t)maps[i];
-        sorted[rank] = k;
+        if (hr.rec) sorted[rank] = k;
     }
     if (hr.rec) {
         const int64_t r0 = hr.hoff[I];
@@ -1376,101 +1376,6 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
     }
 }
 
-// CUDA-core form of numeric_warp_row without per-lane tile products: the lanes resolve 32 pairs
-// of the row (A-tile order, then B order), then the two half-warps form them four at a time,
-// lane e = 4r+c computing entry (r,c) of A_t * B_j (A row r, B column c: the tile_mma order) —
-// the 16 lanes of a product read one A tile and one B tile with coalesced accesses, and the
-// loads of four products are in flight together.  The products are added into the row's
-// shared-memory accumulators in pair order (one half-warp at a time), so the sums are
-// bit-identical to numeric_warp_row's.
-template <typename T, typename Acc>
-__device__ __forceinline__ void numeric_warp_row_hw(int64_t I, const SymCtx& c, const T* __restrict__ aval,
-                                                    const T* __restrict__ bval, const int64_t* __restrict__ cptr,
-                                                    const int32_t* __restrict__ cidx_g,
-                                                    const uint16_t* __restrict__ cmap_g, T* __restrict__ cval,
-                                                    NumSmem<Acc>& S, int lane) {
-    const int64_t c0 = cptr[I];
-    const int nC = (int)(cptr[I + 1] - c0);
-    if (nC == 0) return;
-    const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
-    if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
-    for (int e = lane; e < nC * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
-    __syncwarp();
-    const int h = lane >> 4, e = lane & 15, er = e >> 2, ec = e & 3;
-    for (int64_t base = a0; base < a1; base += 32) {
-        const int64_t t = base + lane;
-        const bool v = t < a1;
-        const uint32_t ma = v ? c.amap[t] : 0u;
-        const int32_t K = v ? c.aidx[t] : 0;
-        const int64_t b0 = v ? c.bptr[K] : 0;
-        const int64_t len = v ? c.bptr[K + 1] - b0 : 0;
-        int64_t incl = len;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
-            if (lane >= d) incl += y;
-        }
-        const int64_t excl = incl - len;
-        const int64_t total = __shfl_sync(0xffffffffu, incl, 31);
-        for (int64_t p0 = 0; p0 < total; p0 += 32) {
-            const int64_t p = p0 + lane;
-            int lo = 0;
-#pragma unroll
-            for (int step = 16; step; step >>= 1) {
-                const int cand = lo + step;
-                const int64_t ex = __shfl_sync(0xffffffffu, excl, cand & 31);
-                if (cand < 32 && ex <= p) lo = cand;
-            }
-            const int64_t ob0 = __shfl_sync(0xffffffffu, b0, lo);
-            const int64_t oex = __shfl_sync(0xffffffffu, excl, lo);
-            const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
-            int q = -1;
-            int64_t j = 0;
-            if (p < total) {
-                j = ob0 + (p - oex);
-                if (bitmap_multiply(oma, c.bmap[j])) q = bsearch_row(S.cidx, nC, c.bidx[j]);
-            }
-            const int64_t ta = base + lo;
-            const unsigned any = __ballot_sync(0xffffffffu, q >= 0);
-            for (int sr = 0; sr < 32; sr += 8) {
-                if (!((any >> sr) & 0xFFu)) continue;  // warp-uniform
-                int qq[4];
-                Acc prod[4];
-#pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const int src = sr + 2 * u + h;
-                    qq[u] = __shfl_sync(0xffffffffu, q, src);
-                    const int64_t tu = __shfl_sync(0xffffffffu, ta, src);
-                    const int64_t ju = __shfl_sync(0xffffffffu, j, src);
-                    Acc ar[4], bc[4];
-                    if (qq[u] >= 0) {
-                        RowIO<T>::load(aval + 16 * tu + 4 * er, ar);
-#pragma unroll
-                        for (int k = 0; k < 4; ++k) bc[k] = to_acc<Acc>(bval[16 * ju + 4 * k + ec]);
-                        Acc sv = ar[0] * bc[0];
-                        sv = fma_acc(ar[1], bc[1], sv);
-                        sv = fma_acc(ar[2], bc[2], sv);
-                        sv = fma_acc(ar[3], bc[3], sv);
-                        prod[u] = sv;
-                    }
-                }
-                // pair order: sr+0 (half 0), sr+1 (half 1), sr+2 (half 0), ...
-#pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    if (h == (k & 1) && qq[k >> 1] >= 0) S.acc[qq[k >> 1]][e] += prod[k >> 1];
-                    __syncwarp();
-                }
-            }
-        }
-    }
-    __syncwarp();
-    for (int64_t x = lane; x < 16 * (int64_t)nC; x += 32) {  // +0.0 where the bitmap bit is clear (R2)
-        const int qx = (int)(x >> 4), b = (int)(x & 15);
-        const bool bit = (cmap_g[c0 + qx] >> b) & 1u;
-        cval[16 * c0 + x] = bit ? from_acc<T>(S.acc[qx][b]) : from_acc<T>(Acc(0));
-    }
-}
-
 // Warp per C block row for the rows in `rows` (count read from the device: the rows the
 // group kernel could not take, nC > GROUP_NC).  Persistent grid-stride over the list.
 template <typename T, typename Acc>
@@ -1484,10 +1389,8 @@ __global__ void __launch_bounds__(NUM_WARPS * 32) k_numeric(const int32_t* __res
     __shared__ NumSmem<Acc> sm[NUM_WARPS];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t nrows = (int64_t)*nrows_dev;
-    const bool hw = tc_thr > 16 || sizeof(T) == 4;  // every tile on CUDA cores: the half-warp form
     for (int64_t wi = (int64_t)blockIdx.x * NUM_WARPS + w; wi < nrows; wi += (int64_t)gridDim.x * NUM_WARPS) {
-        if (hw) numeric_warp_row_hw<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, sm[w], lane);
-        else numeric_warp_row<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, gacc, tc_thr, sm[w], lane);
+        numeric_warp_row<T, Acc>(rows[wi], c, aval, bval, cptr, cidx_g, cmap_g, cval, gacc, tc_thr, sm[w], lane);
         __syncwarp();
     }
 }
@@ -2930,9 +2833,9 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_LAUNCHED();
             }
         } else if (BR > 0) {
-            // rows of A longer than SMALL_CUB tiles: the pair prefix over A tiles first (Cub per row
+            // rows of A longer than 4 SMALL_CUB tiles: the pair prefix over A tiles first (Cub per row
             // without a walk; reused by the whole-GPU dense rows' records)
-            if ((A->row_max == 0 || A->row_max > SMALL_CUB) && A->blc_num > 0 && plen_s.try_init(a, A->blc_num) &&
+            if (A->row_max > 4 * SMALL_CUB && A->blc_num > 0 && plen_s.try_init(a, A->blc_num) &&
                 pp_s.try_init(a, A->blc_num + 1)) {
                 k_plan_plen<<<capped(ceil_div(A->blc_num, 256)), 256, 0, s>>>(A->blc_num, c, plen_s.p);
                 AMGT_LAUNCHED();
