@@ -351,7 +351,7 @@ __device__ __forceinline__ int lower_pos(const int* keys, int n, int J) {  // ke
 // LOGS = log2(table slots per warp).  STEP 1: count -> nnz_row[I].  STEP 2: write sorted
 // idx/map at ptrC[I].
 template <int LOGS, int STEP>
-__global__ void __launch_bounds__(256) k_sym_warp(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
+__global__ void __launch_bounds__(256, 8) k_sym_warp(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c,
                                                   int64_t* __restrict__ nnz_row, const int64_t* __restrict__ cptr,
                                                   int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap, HRec hr) {
     constexpr int S = 1 << LOGS;
@@ -710,7 +710,7 @@ __global__ void __launch_bounds__(256) k_sym_copy(int64_t BR, const int64_t* __r
 
 // ---------------------------------------------------------------- step kernels: block bins
 template <int LOGS, int STEP>
-__global__ void k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c, int64_t* __restrict__ nnz_row,
+__global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_sym_block(int64_t nrows, const int32_t* __restrict__ rows, SymCtx c, int64_t* __restrict__ nnz_row,
                             const int64_t* __restrict__ cptr, int32_t* __restrict__ cidx, uint16_t* __restrict__ cmap,
                             int jbits, HRec hr) {
     constexpr int S = 1 << LOGS;
@@ -2452,7 +2452,7 @@ static amgt_status launch_block_bin(int64_t n, const int32_t* rows, const SymCtx
     while (jbits < 31 && ((int64_t)1 << jbits) < BCB) ++jbits;
     if (n == 0) return AMGT_OK;
     constexpr int S = 1 << LOGS;
-    const size_t sm = (size_t)S * 4 * 2 + (STEP == 2 ? (size_t)S / 2 * 8 : 0);
+    const size_t sm = (size_t)S * 4 * 2 + (STEP == 2 && LOGS > 12 ? (size_t)S / 2 * 8 : 0);  // list: bitonic path
     const int threads = LOGS >= 12 ? 512 : 256;
     auto kern = k_sym_block<LOGS, STEP>;
     AMGT_CUDA(dyn_smem(kern, sm));
@@ -2784,7 +2784,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     GDense gd;  // whole-GPU dense rows (steps 1 and 2)
     Scratch<int64_t> plen_s, pp_s;  // pair prefix over A tiles (rows longer than SMALL_CUB tiles)
     Scratch<int64_t> cub_row, hcnt, hoff;  // hash-bin rows: Cub, record counts and offsets
-    int64_t nH = 0;                        // records of the hash-bin rows (numeric plan)
+    int64_t nH = 0;                        // record slots of the hash-bin rows (an upper bound)
     AMGT_TRY(bin_of.init(a, BR + 1));
     AMGT_TRY(nnz_row.init(a, BR + 1));
     AMGT_TRY(ctr.init(a, 32));
@@ -2863,19 +2863,16 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_CUDA(cudaMemcpyAsync(ps + 16, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(ps + 17, rmax, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(ps + 18, ctr.p + 26, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-                if (hoff.p) AMGT_CUDA(cudaMemcpyAsync(ps + 19, hoff.p + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaStreamSynchronize(s));
                 if (with_stats) memcpy(hs, ps, sizeof(hs));
                 TC = ps[16];
                 hmax = (unsigned long long)ps[17];
                 gd.npairs = ps[18];
-                if (hoff.p) nH = ps[19];
             } else {
                 if (with_stats) AMGT_CUDA(cudaMemcpyAsync(hs, stats, sizeof(hs), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&TC, C.blc_ptr + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&hmax, rmax, sizeof(hmax), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaMemcpyAsync(&gd.npairs, ctr.p + 26, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-                if (hoff.p) AMGT_CUDA(cudaMemcpyAsync(&nH, hoff.p + BR, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
                 AMGT_CUDA(cudaStreamSynchronize(s));
             }
             return AMGT_OK;
@@ -2904,16 +2901,19 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             if (st != AMGT_OK) return st;
             AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
             AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
+            AMGT_TRY(read_back(false));  // sync 2: C tile count with the long rows
             // hash-bin rows (bins < min(dense, 5): the kernels that sort in shared memory) with more
-            // than CAP C tiles: their pair counts -> record offsets
-            if (plan_env && cub_row.p && hcnt.try_init(a, BR) && hoff.try_init(a, BR + 1)) {
+            // than CAP C tiles (some exist only if the longest C row has more): their pair counts ->
+            // record offsets; the records are allocated for an upper bound (all pairs outside the
+            // dense rows), so no further synchronisation
+            if (plan_env && cub_row.p && (int64_t)hmax > CAP && hcnt.try_init(a, BR) && hoff.try_init(a, BR + 1)) {
                 const int hb_hi = std::min(gd.dense_from_eff, 5);
                 k_plan_hcount<<<capped(ceil_div(BR, 256)), 256, 0, s>>>(BR, bin_of.p, nnz_row.p, cub_row.p, hb_hi,
                                                                       hcnt.p);
                 AMGT_LAUNCHED();
                 AMGT_TRY(scan_exclusive(hcnt.p, hoff.p, BR, a, s));
+                nH = std::max<int64_t>((int64_t)hs[8] - (gd.on && gd.plan ? std::max<int64_t>(gd.npairs, 0) : 0), 0);
             }
-            AMGT_TRY(read_back(false));  // sync 2: C tile count with the long rows
         }
         amgt_status st = mbsr_alloc(&C, A->m, B->n, TC, A->prec, a, true, true, C.blc_ptr);
         if (st != AMGT_OK) return st;
