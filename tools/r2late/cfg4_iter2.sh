@@ -1,4 +1,4 @@
-cd $GRAFT_REPO_ROOT; O=gpurun_out/r3; mkdir -p $O
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late; mkdir -p $O
 timeout 900 python -m pytest tests/test_gpu_spgemm.py -x -q -m gpu > $O/t_spgemm2.log 2>&1; tail -15 $O/t_spgemm2.log
 rm -f $O/cfg4_knobs2.txt
 for v in "AMGT_SPGEMM_PLAN=0" "AMGT_SPGEMM_PLAN=1" "AMGT_DENSE_FROM_BIN=3" "AMGT_DENSE_FROM_BIN=4"; do

@@ -1,4 +1,4 @@
-cd $GRAFT_REPO_ROOT; O=gpurun_out/r3; mkdir -p $O
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late; mkdir -p $O
 timeout 900 python -m pytest tests/test_gpu_spgemm.py -x -q -m gpu > $O/t_spgemm5.log 2>&1; tail -3 $O/t_spgemm5.log
 rm -f $O/cfg4_knobs5.txt
 for v in "AMGT_PLAN_HINTS=0" "AMGT_PLAN_HINTS=3" "AMGT_PLAN_HINTS=3 AMGT_PLAN_BAND_MB=1000"; do

@@ -1,7 +1,7 @@
-cd $GRAFT_REPO_ROOT; O=gpurun_out/r3; mkdir -p $O
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late; mkdir -p $O
 timeout 900 python -m pytest tests/test_gpu_spgemm.py -x -q -m gpu > $O/t_spgemm7.log 2>&1; tail -3 $O/t_spgemm7.log
-python tools/r3/sym_var.py 2>&1 | tail -3
-AMGT_PLAN_BAND_MB=1000 python tools/r3/sym_var.py 2>&1 | tail -2
-AMGT_PLAN_BAND_MB=6 python tools/r3/sym_var.py 2>&1 | tail -2
+python tools/r2late/sym_var.py 2>&1 | tail -3
+AMGT_PLAN_BAND_MB=1000 python tools/r2late/sym_var.py 2>&1 | tail -2
+AMGT_PLAN_BAND_MB=6 python tools/r2late/sym_var.py 2>&1 | tail -2
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:'^k_' --csv --log-file $O/cfg4_launches7.csv python tools/profile_cfg4.py 2 > $O/cfg4_ncu7.log 2>&1
 python tools/ncu_sum_launches.py $O/cfg4_launches7.csv --per-launch > $O/cfg4_launches7.txt 2>&1

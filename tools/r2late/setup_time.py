@@ -1,5 +1,5 @@
 """Config-3 (or other) hierarchy setup: wall time (CUDA events) of several setups after a warm-up,
-and the per-class device timers of the last one.  usage: python tools/r3/setup_time.py [cfg3] [reps]"""
+and the per-class device timers of the last one.  usage: python tools/r2late/setup_time.py [cfg3] [reps]"""
 import json, os, sys, statistics
 sys.path.insert(0, os.getcwd())
 import torch
