@@ -1212,8 +1212,7 @@ constexpr int NUM_WARPS = 4;
 constexpr int CAP = 32;  // C tiles per row accumulated in shared memory
 
 template <typename Acc> struct NumSmem {
-    Acc acc[CAP][16];
-    Acc stage[32][17];  // one tile product per lane; padded rows (lane-strided writes)
+    Acc acc[CAP][17];  // C tiles of the row; padded: lanes adding different tiles spread over banks
     int32_t cidx[CAP];
 };
 
@@ -1238,7 +1237,7 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
     const int64_t a0 = c.aptr[I], a1 = c.aptr[I + 1];
     // nC <= CAP (longer rows go to the mid/long-row kernels): shared-memory accumulators
     if (lane < nC) S.cidx[lane] = cidx_g[c0 + lane];
-    for (int e = lane; e < nC * 16; e += 32) (&S.acc[0][0])[e] = Acc(0);
+    for (int e = lane; e < nC * 16; e += 32) S.acc[e >> 4][e & 15] = Acc(0);
     __syncwarp();
     const int32_t* rowidx = S.cidx;
     auto accp = [&](int q) -> Acc* { return S.acc[q]; };
@@ -1329,6 +1328,7 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
                 const uint32_t oma = __shfl_sync(0xffffffffu, ma, lo);
                 const int64_t ot = base + lo;
                 int q = -1;
+                Acc pr[16];
                 if (p < total) {
                     const int64_t j = ob0 + (p - oex);
                     const uint32_t mc = bitmap_multiply(oma, c.bmap[j]);
@@ -1338,7 +1338,7 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
                         TileIO<T>::load(bval + 16 * j, bv);
                         const T* ap = aval + 16 * ot;
 #pragma unroll
-                        for (int r = 0; r < 4; ++r) {  // product rows straight to the staging row
+                        for (int r = 0; r < 4; ++r) {  // the product in registers (tile_mma order)
                             Acc ar[4];
                             RowIO<T>::load(ap + 4 * r, ar);
 #pragma unroll
@@ -1347,22 +1347,24 @@ __device__ __forceinline__ void numeric_warp_row(int64_t I, const SymCtx& c, con
                                 sv = fma(ar[1], bv[4 + col], sv);
                                 sv = fma(ar[2], bv[8 + col], sv);
                                 sv = fma(ar[3], bv[12 + col], sv);
-                                S.stage[lane][4 * r + col] = sv;
+                                pr[4 * r + col] = sv;
                             }
                         }
                     }
                 }
-                __syncwarp();
-                // accumulate the staged products in lane order (deterministic): half-warp h
-                // takes the products whose C tile has (q & 1) == h, lane e of it element e
-                uint32_t todo = __ballot_sync(0xffffffffu, q >= 0);
-                while (todo) {
-                    const int sl = __ffs(todo) - 1;
-                    todo &= todo - 1;
-                    const int qs = __shfl_sync(0xffffffffu, q, sl);
-                    if ((qs & 1) == (lane >> 4)) S.acc[qs][lane & 15] += S.stage[sl][lane & 15];
+                // accumulate in lane order per C tile (deterministic): the k-th lane of a group
+                // of lanes with the same tile adds in round k, so lanes of different tiles add
+                // concurrently (usually one to three rounds instead of 32 serial steps)
+                const unsigned peers = __match_any_sync(0xffffffffu, q);
+                const int rank = __popc(peers & ((1u << lane) - 1u));
+                const int rmax = (int)__reduce_max_sync(0xffffffffu, q >= 0 ? (unsigned)rank : 0u);
+                for (int k = 0; k <= rmax; ++k) {
+                    if (q >= 0 && rank == k) {
+#pragma unroll
+                        for (int x = 0; x < 16; ++x) S.acc[q][x] += pr[x];
+                    }
+                    __syncwarp();
                 }
-                __syncwarp();
             }
         }
     }
