@@ -1,0 +1,17 @@
+# late-round measurement batch: GPU suite, smoke, bench x2 (the driver's command), reference arm,
+# bench launch list (ncu), config-4 SpGEMM traffic capture (ncu --set full), sanitizer on SpGEMM
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late/final; mkdir -p $O
+timeout 1800 python -m pytest tests -q -m gpu > $O/gpu_tests.log 2>&1; echo "rc=$?" >> $O/gpu_tests.log; tail -2 $O/gpu_tests.log
+python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log; tail -2 $O/smoke.log
+timeout 900 python bench.py > $O/bench_1.json 2> $O/bench_1.err
+timeout 900 python bench.py > $O/bench_2.json 2> $O/bench_2.err
+timeout 900 python bench.py --impl reference > $O/bench_ref.json 2> $O/bench_ref.err
+timeout 1500 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"^k_" -c 20000 --csv --log-file $O/bench_launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-cfg4 > $O/bench_ncu.log 2>&1
+timeout 1500 ncu --set full --clock-control none --nvtx --nvtx-include 'amgt_spgemm/' -o $O/ncu_spgemm_cfg4 python tools/ncu_traffic.py run cfg4 > $O/ncu_cfg4.log 2>&1
+python tools/ncu_traffic.py summarize cfg4 $O/ncu_spgemm_cfg4.ncu-rep > $O/ncu_cfg4_sum.log 2>&1
+export PYTORCH_NO_CUDA_MEMORY_CACHING=1
+CS="compute-sanitizer --print-limit 20 --error-exitcode 99"
+timeout 1200 $CS --tool memcheck python -m pytest tests/test_gpu_spgemm.py -m gpu -q -x -p no:cacheprovider -k "not full and not cfg" > $O/spgemm_memcheck.log 2>&1; echo "memcheck rc=$?" >> $O/sanitize.txt
+timeout 1200 $CS --tool racecheck python -m pytest tests/test_gpu_spgemm.py -m gpu -q -x -p no:cacheprovider -k "long_rows or plan or info_bins" > $O/spgemm_racecheck.log 2>&1; echo "racecheck rc=$?" >> $O/sanitize.txt
+grep -h "ERROR SUMMARY" $O/*check.log >> $O/sanitize.txt
+echo done > $O/done
