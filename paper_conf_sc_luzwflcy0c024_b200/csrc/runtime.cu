@@ -132,7 +132,13 @@ int g_tc_thr_spmv = 17;
 
 // ------------------------------------------------------------------ scan
 // Block-wide exclusive scan: 1024 threads x 8 items = 8192 items per block.
-constexpr int SCAN_T = 256, SCAN_I = 8, SCAN_TILE = SCAN_T * SCAN_I;  // 2048 items per CTA
+#ifndef AMGT_SCAN_T  // experiments: -DAMGT_SCAN_T=.. -DAMGT_SCAN_I=.. (AMGT_NVCC_EXTRA)
+#define AMGT_SCAN_T 256
+#endif
+#ifndef AMGT_SCAN_I
+#define AMGT_SCAN_I 8
+#endif
+constexpr int SCAN_T = AMGT_SCAN_T, SCAN_I = AMGT_SCAN_I, SCAN_TILE = SCAN_T * SCAN_I;  // 2048 items per CTA (4096 / 8192 measured equal)
 
 __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t* sh_warp, int64_t* total) {
     int lane = threadIdx.x & 31, w = threadIdx.x >> 5;

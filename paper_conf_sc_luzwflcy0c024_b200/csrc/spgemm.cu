@@ -2879,6 +2879,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             }
             return AMGT_OK;
         };
+        trace_point("sym step1", s);
         AMGT_TRY(read_back(true));  // sync 1: bins, C tile count (L153)
         int64_t cnt[NCAT], off[NCAT], acc = 0;
         for (int b = 0; b < NCAT; ++b) { cnt[b] = (int64_t)hs[cat_stat(b)]; off[b] = acc; acc += cnt[b]; }
@@ -2903,6 +2904,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             if (st != AMGT_OK) return st;
             AMGT_CUDA(cudaMemsetAsync(rmax, 0, sizeof(unsigned long long), s));
             AMGT_TRY(scan_exclusive(nnz_row.p, C.blc_ptr, BR, a, s, rmax));
+            trace_point("sym bins step1", s);
             AMGT_TRY(read_back(false));  // sync 2: C tile count with the long rows
             // hash-bin rows (bins < min(dense, 5): the kernels that sort in shared memory) with more
             // than CAP C tiles (some exist only if the longest C row has more): their pair counts ->
@@ -2949,6 +2951,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_CUDA(cudaMemsetAsync(P->rowf, 0, (size_t)BR, s));
             }
         }
+        trace_point("sym alloc", s);
         gd.P = npD > 0 ? P : nullptr;
         gd.pcnt = pcnt.p;
         HRec hr{};
@@ -2975,6 +2978,7 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 if (st != AMGT_OK) return st;
             }
         }
+        trace_point("sym step2", s);
         if (P) {
             k_plan_mark<<<capped(ceil_div(TC, 256)), 256, 0, s>>>(TC, pcnt.p, P->mflag);
             AMGT_LAUNCHED();
@@ -3004,6 +3008,8 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
     }
     done = true;
     *Cout = C;
+    trace_point("sym end", s);
+    trace_dump();
     return AMGT_OK;
 }
 

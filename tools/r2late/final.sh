@@ -7,8 +7,10 @@ timeout 900 python bench.py > $O/bench_1.json 2> $O/bench_1.err
 timeout 900 python bench.py > $O/bench_2.json 2> $O/bench_2.err
 timeout 900 python bench.py --impl reference > $O/bench_ref.json 2> $O/bench_ref.err
 timeout 1500 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"^k_" -c 20000 --csv --log-file $O/bench_launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-cfg4 > $O/bench_ncu.log 2>&1
-timeout 1500 ncu --set full --clock-control none --nvtx --nvtx-include 'amgt_spgemm/' -o $O/ncu_spgemm_cfg4 python tools/ncu_traffic.py run cfg4 > $O/ncu_cfg4.log 2>&1
-python tools/ncu_traffic.py summarize cfg4 $O/ncu_spgemm_cfg4.ncu-rep > $O/ncu_cfg4_sum.log 2>&1
+timeout 1500 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none --nvtx --nvtx-include 'amgt_spgemm/' -o /tmp/ncu_spgemm_cfg4 python tools/ncu_traffic.py run cfg4 > $O/ncu_cfg4.log 2>&1
+python tools/ncu_traffic.py summarize cfg4 /tmp/ncu_spgemm_cfg4.ncu-rep > $O/ncu_cfg4_sum.log 2>&1
+cp profiles/ncu_traffic_cfg4.json $O/ncu_traffic_cfg4.json
+gzip -f $O/bench_launches.csv
 export PYTORCH_NO_CUDA_MEMORY_CACHING=1
 CS="compute-sanitizer --print-limit 20 --error-exitcode 99"
 timeout 1200 $CS --tool memcheck python -m pytest tests/test_gpu_spgemm.py -m gpu -q -x -p no:cacheprovider -k "not full and not cfg" > $O/spgemm_memcheck.log 2>&1; echo "memcheck rc=$?" >> $O/sanitize.txt
