@@ -2528,6 +2528,8 @@ struct SpgemmPlan {
     size_t bytes = 0;       // device bytes held
     uint32_t* mflag = nullptr;  // bit q: C tile q takes several products
     uint8_t* rowf = nullptr;    // per C block row: 1 = computed from the records
+    cudaEvent_t used = nullptr;  // recorded after the last work that reads the plan (any stream)
+    bool covers_all = false;     // every row with more than CAP C tiles has records
 };
 
 static std::mutex g_plan_mu;
@@ -2535,8 +2537,15 @@ static std::vector<SpgemmPlan*> g_plans;
 constexpr size_t MAX_PLANS = 4;
 constexpr size_t MAX_PLAN_BYTES = (size_t)2 << 30;  // least recently built plans dropped beyond
 
+// Frees on stream s after the plan's last use, wherever that ran (virtual ranks share the cache
+// from several threads and streams: an eviction on one stream must not free records another
+// stream's kernels still read).
 static void plan_free(SpgemmPlan* P, cudaStream_t s) {
     if (!P) return;
+    if (P->used) {
+        cudaStreamWaitEvent(s, P->used, 0);
+        cudaEventDestroy(P->used);
+    }
     scratch_put(P->rec, s);
     scratch_put(P->mflag, s);
     scratch_put(P->rowf, s);
@@ -2544,6 +2553,11 @@ static void plan_free(SpgemmPlan* P, cudaStream_t s) {
 }
 
 static void plan_put(SpgemmPlan* P, cudaStream_t s) {
+    if (!P->used && cudaEventCreateWithFlags(&P->used, cudaEventDisableTiming) != cudaSuccess) {
+        cudaGetLastError();
+        P->used = nullptr;
+    }
+    if (P->used) cudaEventRecord(P->used, s);  // the work just enqueued on s is the latest use
     std::vector<SpgemmPlan*> old;
     {
         std::lock_guard<std::mutex> lk(g_plan_mu);
@@ -2980,6 +2994,14 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
         }
         trace_point("sym step2", s);
         if (P) {
+            // rows past CAP C tiles without records: dense rows whose records failed, hash rows when
+            // the longest C row exceeds CAP and no offsets were computed, bins 5-6 (bitonic kernels)
+            int64_t dense_rows = 0, bitonic_rows = 0;
+            for (int b = gd.dense_from_eff; b < NBINS; ++b) dense_rows += cnt_big[b];
+            for (int b = 5; b < std::min(gd.dense_from_eff, NBINS); ++b) bitonic_rows += cnt_big[b];
+            const bool dense_ok = dense_rows == 0 || (gd.on && gd.plan && npD > 0);
+            const bool hash_ok = (int64_t)hmax <= CAP || (hoff.p != nullptr && nH > 0);
+            P->covers_all = dense_ok && hash_ok && bitonic_rows == 0;
             k_plan_mark<<<capped(ceil_div(TC, 256)), 256, 0, s>>>(TC, pcnt.p, P->mflag);
             AMGT_LAUNCHED();
             pscope.ok = true;
@@ -3624,7 +3646,8 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
         }
     }
     // row classes present (C->row_max from symbolic; 0 = unknown: launch everything)
-    const int64_t rmax = C->row_max > 0 ? C->row_max : INT64_MAX;
+    int64_t rmax = C->row_max > 0 ? C->row_max : INT64_MAX;
+    if (plan && plan->covers_all) rmax = std::min<int64_t>(rmax, CAP);  // longer rows: records only
     if (rmax <= GROUP_NC) return AMGT_OK;
     static int warp_per_sm = 0;  // resident CTAs of the warp kernel (per instantiation)
     if (!warp_per_sm) {

@@ -281,3 +281,64 @@ def test_spgemm_plan_reused_after_value_change():
     amgt.spgemm_numeric(M, M, C)
     Co4 = oracle.Csr(Co.m, Co.n, Co.row_ptr, Co.col, 4.0 * Co.val)
     _check_product(C, Co4, 4.0 * Cabs)
+
+
+_NOPLAN_SCRIPT = r"""
+import sys, numpy as np
+sys.path.insert(0, sys.argv[1])
+import gen, paper_conf_sc_luzwflcy0c024_b200 as amgt
+cases = {
+    "power_law": lambda: (gen.irregular_block_sparse(1 << 13, seed=9),) * 2,
+    "long_dense": lambda: (gen.random_csr(32, 8192, 0.3, 31), gen.random_csr(8192, 4096, 0.02, 32)),
+    "mid_only": lambda: (gen.random_csr(64, 3000, 0.3, 33), gen.random_csr(3000, 900, 0.01, 34)),
+}
+A, B = cases[sys.argv[3]]()
+C = amgt.spgemm(amgt.from_csr(A, prec=sys.argv[4]), amgt.from_csr(B, prec=sys.argv[4]))
+np.savez(sys.argv[2], ptr=C.blc_ptr.cpu().numpy(), idx=C.blc_idx.cpu().numpy(), map=C.map_u16().cpu().numpy(),
+         val=C.blc_val.float().double().cpu().numpy() if sys.argv[4] == "f16" else C.blc_val.double().cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("prec", ["f64", "f16"])
+@pytest.mark.parametrize("case", ["power_law", "long_dense", "mid_only"])
+def test_spgemm_searching_kernels_without_plan(tmp_path, case, prec):
+    """AMGT_SPGEMM_PLAN=0 (separate process; the knob is read once): the rows past 32 C tiles take
+    the searching kernels (warp rows 33-512, two-pass long rows with pair records) instead of the
+    symbolic phase's records (R34) — structure bit-exact, FP64 values within 1e-12 (|A||B|),
+    FP16 within 5e-3 (2-norm)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "noplan.py"
+    script.write_text(_NOPLAN_SCRIPT)
+    out = tmp_path / "c.npz"
+    env = dict(os.environ, AMGT_SPGEMM_PLAN="0")
+    p = subprocess.run([sys.executable, str(script), root, str(out), case, prec], env=env, capture_output=True,
+                       text=True, timeout=300)
+    assert p.returncode == 0, p.stderr[-2000:]
+    got = np.load(out)
+    A, B = {
+        "power_law": lambda: (gen.irregular_block_sparse(1 << 13, seed=9),) * 2,
+        "long_dense": lambda: (gen.random_csr(32, 8192, 0.3, 31), gen.random_csr(8192, 4096, 0.02, 32)),
+        "mid_only": lambda: (gen.random_csr(64, 3000, 0.3, 33), gen.random_csr(3000, 900, 0.01, 34)),
+    }[case]()
+    Ao, Bo = oracle.as_csr(A), oracle.as_csr(B)
+    Co, Cabs = oracle.spgemm(Ao, Bo, with_abs=True)
+    Cm = oracle.csr_to_mbsr(Co)
+    assert np.array_equal(got["ptr"], Cm.blc_ptr)
+    assert np.array_equal(got["idx"], Cm.blc_idx)
+    assert np.array_equal(got["map"], Cm.blc_map.astype(np.int32))
+    assert np.diff(got["ptr"]).max() > 32
+    # values in CSR order from the dense tiles (bits set in the bitmap, row-major within a tile row)
+    om = oracle.csr_to_mbsr(Co)
+    vals = got["val"].reshape(-1, 16)
+    ref = np.asarray(om.blc_val).reshape(-1, 16)
+    bits = ((got["map"][:, None] >> np.arange(16)) & 1).astype(bool)
+    g, r = vals[bits], ref[bits]
+    if prec == "f64":
+        absm = oracle.csr_to_mbsr(oracle.Csr(Co.m, Co.n, Co.row_ptr, Co.col, Cabs))
+        bound = 1e-12 * np.asarray(absm.blc_val).reshape(-1, 16)[bits]
+        assert np.all(np.abs(g - r) <= bound + 1e-300)
+    else:
+        assert np.linalg.norm(g - r) <= 5e-3 * np.linalg.norm(r)
