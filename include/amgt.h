@@ -153,8 +153,16 @@ typedef struct {
  * blc_ptrC, allocation, step 2 re-inserts, compresses and sorts -> blc_idxC) and, in
  * this build, the OR of BITMAPMULTIPLY results into blc_mapC (R15).
  * A, B: same precision, A.n == B.m.  C: output; structure allocated and filled, values
- * allocated (not computed).  info may be NULL.  Syncs once (the C tile count, L153)
- * plus once more if info != NULL.
+ * allocated (not computed).  info may be NULL.  Syncs once (the C tile count, L153) — twice when
+ * some block row has more than 32 candidate tiles (its bin kernels count before the allocation)
+ * — plus once more if info != NULL.
+ * Numeric plan (R34): for the block rows of C with more than 32 tiles, step 2 also keeps
+ * one 16-B record per (A tile, B tile) pair (C tile, B tile, A tile, bitmap product) and a
+ * "several products" bit per C tile in library-owned device memory keyed by C's blc_idx; the
+ * numeric call then streams them instead of searching C's rows.  The plan depends on the
+ * structure only (values of A, B may change between numeric calls), is freed with C's structure
+ * (amgt_mbsr_free) and at most 4 plans / 2 GB are cached (least recently built dropped).
+ * AMGT_SPGEMM_PLAN=0 disables it.
  */
 amgt_status amgt_spgemm_symbolic(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, amgt_spgemm_info* info,
                                  const amgt_allocator* al, void* stream);
@@ -165,7 +173,8 @@ amgt_status amgt_spgemm_symbolic(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
  * DMMA m8n8k4 with fragA = [A;A], fragB = [B_j | B_j'], keeping the two diagonal 4x4
  * quadrants, L157-171; FP16: HMMA m16n8k16 with FP32 accumulation, 8 tile products per
  * instruction); otherwise the thread-level CUDA-core route.  FP32 always takes the
- * CUDA-core route (no TF32, R17).  C must come from amgt_spgemm_symbolic(A, B).
+ * CUDA-core route (no TF32, R17).  C must come from amgt_spgemm_symbolic(A, B) (same A and B
+ * structure arrays; the symbolic phase's numeric plan is used when present, see above).
  * Values: deterministic for C block rows with at most 32 tiles (fixed lane order); longer rows
  * accumulate tiles that receive three or more products with FP atomics and are reproducible up
  * to rounding only (exact on integer / dyadic data).
