@@ -136,6 +136,28 @@ __device__ __forceinline__ bool hash_insert(int* keys, uint32_t* maps, int logS,
     }
 }
 
+// hash_insert that also returns the slot holding J (the plan's records refer to it until the
+// sort has fixed the columns' ranks)
+__device__ __forceinline__ int hash_insert_at(int* keys, uint32_t* maps, int logS, int32_t J, uint32_t mapC) {
+    const uint32_t mask = (1u << logS) - 1u;
+    uint32_t h = hash_slot(J, logS);
+    for (;;) {
+        const int k = ((volatile int*)keys)[h];
+        if (k == J) {
+            atomicOr(maps + h, mapC);
+            return (int)h;
+        }
+        if (k == EMPTY_KEY) {
+            const int old = atomicCAS(keys + h, EMPTY_KEY, J);
+            if (old == EMPTY_KEY || old == J) {
+                atomicOr(maps + h, mapC);
+                return (int)h;
+            }
+        }
+        h = (h + 1) & mask;
+    }
+}
+
 // Warp-cooperative enumeration of the (A tile, B tile) pairs of block row I: lanes take
 // up to 32 A tiles, warp-scan their B-row lengths, then spread the pairs over lanes.
 // fn(J, mapC) is called for every pair with mapC != 0 — or fn(J, mapC, t, j, pos) with the
@@ -357,8 +379,9 @@ __global__ void __launch_bounds__(256, 8) k_sym_warp(int64_t nrows, const int32_
     constexpr int S = 1 << LOGS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    int* keys = reinterpret_cast<int*>(smem_raw) + w * 2 * S;
+    int* keys = reinterpret_cast<int*>(smem_raw) + w * (2 * S + S / 2);
     uint32_t* maps = reinterpret_cast<uint32_t*>(keys + S);
+    int* oslot = keys + 2 * S;  // step 2, rows with records: hash slot of each compressed entry
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (wg >= nrows) return;
     const int64_t I = rows[wg];
@@ -367,8 +390,20 @@ __global__ void __launch_bounds__(256, 8) k_sym_warp(int64_t nrows, const int32_
         maps[i] = 0;
     }
     __syncwarp();
+    int64_t r0 = 0, r1 = 0;
+    if (STEP == 2 && hr.rec) {
+        r0 = hr.hoff[I];
+        r1 = hr.hoff[I + 1];
+    }
     int cnt = 0;
-    warp_pairs(c, I, lane, [&](int32_t J, uint32_t mc) { cnt += hash_insert(keys, maps, LOGS, J, mc, STEP == 2); });
+    if (STEP == 2 && r1 > r0) {  // records {hash slot, B tile, A tile, bitmap product} (R34)
+        warp_pairs(c, I, lane, [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
+            const int h = hash_insert_at(keys, maps, LOGS, J, mc);
+            hr.rec[r0 + pos] = make_int4(h, (int)j, (int)t, (int)mc);
+        });
+    } else {
+        warp_pairs(c, I, lane, [&](int32_t J, uint32_t mc) { cnt += hash_insert(keys, maps, LOGS, J, mc, STEP == 2); });
+    }
     __syncwarp();
     if (STEP == 1) {
 #pragma unroll
@@ -388,31 +423,42 @@ __global__ void __launch_bounds__(256, 8) k_sym_warp(int64_t nrows, const int32_
             const int pos = n + __popc(bal & ((1u << lane) - 1u));
             keys[pos] = k;
             maps[pos] = mp;
+            oslot[pos] = base + lane;
         }
         n += __popc(bal);
         __syncwarp();
     }
-    // rank sort (n <= S/2 distinct keys); the sorted keys also go to keys[S/2 ..)
+    // rank sort (n <= S/2 distinct keys); with records, maps[i] <- rank of entry i
     const int64_t out = cptr[I];
-    int* sorted = keys + S / 2;
     for (int i = lane; i < n; i += 32) {
         const int k = keys[i];
         int rank = 0;
         for (int j = 0; j < n; ++j) rank += keys[j] < k;
         cidx[out + rank] = k;
         cmap[out + rank] = (uint16_t)maps[i];
-        if (hr.rec) sorted[rank] = k;
+        maps[i] = (uint32_t)rank;
     }
-    if (hr.rec) {
-        const int64_t r0 = hr.hoff[I];
-        if (hr.hoff[I + 1] > r0) {  // records: C tile of every pair (third walk)
-            __syncwarp();
-            if (lane == 0) hr.rowf[I] = 1;
-            warp_pairs(c, I, lane, [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
-                const int64_t q = out + lower_pos(sorted, n, J);
-                atomicAdd(hr.cnt + q, 1u);
-                hr.rec[r0 + pos] = make_int4((int)q, (int)j, (int)t, (int)mc);
-            });
+    if (r1 > r0) {  // slot -> rank table in keys[], then the row's records get their C tiles
+        __syncwarp();
+        if (lane == 0) hr.rowf[I] = 1;
+        int sl[S / 64 > 0 ? S / 64 : 1], rk[S / 64 > 0 ? S / 64 : 1];
+#pragma unroll
+        for (int u = 0; u < (S / 64 > 0 ? S / 64 : 1); ++u) {
+            const int i = lane + 32 * u;
+            sl[u] = i < n ? oslot[i] : -1;
+            rk[u] = i < n ? (int)maps[i] : 0;
+        }
+        __syncwarp();
+#pragma unroll
+        for (int u = 0; u < (S / 64 > 0 ? S / 64 : 1); ++u)
+            if (sl[u] >= 0) keys[sl[u]] = rk[u];
+        __syncwarp();
+        for (int64_t p = r0 + lane; p < r1; p += 32) {
+            const int h = hr.rec[p].x;
+            if (h < 0) continue;
+            const int64_t q = out + keys[h];
+            hr.rec[p].x = (int)q;
+            atomicAdd(hr.cnt + q, 1u);
         }
     }
 }
@@ -730,9 +776,24 @@ __global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_
             maps[i] = 0;
         }
         __syncthreads();
+        int64_t r0 = 0, r1 = 0;
+        if (STEP == 2 && LOGS <= 12 && hr.rec) {
+            r0 = hr.hoff[I];
+            r1 = hr.hoff[I + 1];
+        }
         int cnt = 0;
-        block_pairs(c, I, sh_excl, sh_b0, sh_ma, sh_tot,
-                    [&](int32_t J, uint32_t mc) { cnt += hash_insert(keys, maps, LOGS, J, mc, STEP == 2); });
+        if (STEP == 2 && r1 > r0) {  // block-uniform: records {hash slot, B tile, A tile, product} (R34)
+            block_pairs_aux(
+                c, c.aptr[I], c.aptr[I + 1], sh_excl, sh_b0, sh_ma, sh_tot, sh_aux,
+                [&](int64_t, int32_t, int64_t pos0) { return r0 + pos0; },
+                [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
+                    const int h = hash_insert_at(keys, maps, LOGS, J, mc);
+                    hr.rec[pos] = make_int4(h, (int)j, (int)t, (int)mc);
+                });
+        } else {
+            block_pairs(c, I, sh_excl, sh_b0, sh_ma, sh_tot,
+                        [&](int32_t J, uint32_t mc) { cnt += hash_insert(keys, maps, LOGS, J, mc, STEP == 2); });
+        }
         __syncthreads();
         if (STEP == 1) {
 #pragma unroll
@@ -753,9 +814,10 @@ __global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_
             // of the log^2 N stages of a bitonic network (Alg. 3 line 14)
             constexpr int THREADS = LOGS >= 12 ? 512 : 256;
             constexpr int IPT = S / THREADS;
-            using Sorter = cub::BlockRadixSort<unsigned long long, THREADS, IPT>;
+            using Sorter = cub::BlockRadixSort<unsigned long long, THREADS, IPT, int>;  // value: hash slot
             __shared__ typename Sorter::TempStorage rs_tmp;
             unsigned long long kv[IPT];
+            int sv[IPT];
             int nv = 0;
 #pragma unroll
             for (int u = 0; u < IPT; ++u) {
@@ -763,6 +825,7 @@ __global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_
                 const int k = keys[slot];
                 nv += k != EMPTY_KEY;
                 kv[u] = k != EMPTY_KEY ? (((unsigned long long)(uint32_t)k << 16) | (maps[slot] & 0xFFFFu)) : ~0ull;
+                sv[u] = slot;
             }
 #pragma unroll
             for (int d = 16; d; d >>= 1) nv += __shfl_xor_sync(0xffffffffu, nv, d);
@@ -770,7 +833,7 @@ __global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_
             __syncthreads();  // keys/maps read into registers; sh_cnt complete
             int n = 0;
             for (int q = 0; q < nw; ++q) n += sh_cnt[q];
-            Sorter(rs_tmp).Sort(kv, 16, 17 + jbits);  // one bit above J: empty slots (~0) last
+            Sorter(rs_tmp).Sort(kv, sv, 16, 17 + jbits);  // one bit above J: empty slots (~0) last
             const int64_t out = cptr[I];
 #pragma unroll
             for (int u = 0; u < IPT; ++u) {
@@ -778,23 +841,20 @@ __global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_
                 if (pos < n) {
                     cidx[out + pos] = (int32_t)(kv[u] >> 16);
                     cmap[out + pos] = (uint16_t)(kv[u] & 0xFFFFu);
-                    keys[pos] = (int)(kv[u] >> 16);  // sorted columns for the record walk
+                    if (r1 > r0) keys[sv[u]] = pos;  // slot -> rank (keys were read before the sort)
                 }
             }
             __syncthreads();
-            if (hr.rec) {
-                const int64_t r0 = hr.hoff[I];
-                if (hr.hoff[I + 1] > r0) {  // block-uniform: records (third walk)
-                    if (tid == 0) hr.rowf[I] = 1;
-                    block_pairs_aux(
-                        c, c.aptr[I], c.aptr[I + 1], sh_excl, sh_b0, sh_ma, sh_tot, sh_aux,
-                        [&](int64_t, int32_t, int64_t pos0) { return r0 + pos0; },
-                        [&](int32_t J, uint32_t mc, int64_t t, int64_t j, int64_t pos) {
-                            const int64_t q = out + lower_pos(keys, n, J);
-                            atomicAdd(hr.cnt + q, 1u);
-                            hr.rec[pos] = make_int4((int)q, (int)j, (int)t, (int)mc);
-                        });
+            if (r1 > r0) {  // the row's records get their C tiles
+                if (tid == 0) hr.rowf[I] = 1;
+                for (int64_t p = r0 + tid; p < r1; p += nt) {
+                    const int h = hr.rec[p].x;
+                    if (h < 0) continue;
+                    const int64_t q = out + keys[h];
+                    hr.rec[p].x = (int)q;
+                    atomicAdd(hr.cnt + q, 1u);
                 }
+                __syncthreads();
             }
             continue;
         }
@@ -2438,7 +2498,7 @@ template <int LOGS, int STEP>
 static amgt_status launch_warp_bin(int64_t n, const int32_t* rows, const SymCtx& c, int64_t* nnz_row, const int64_t* cptr,
                                    int32_t* cidx, uint16_t* cmap, HRec hr, cudaStream_t s) {
     if (n == 0) return AMGT_OK;
-    const size_t sm = (size_t)8 * 2 * (1 << LOGS) * sizeof(int);
+    const size_t sm = (size_t)8 * (2 * (1 << LOGS) + (1 << LOGS) / 2) * sizeof(int);
     auto kern = k_sym_warp<LOGS, STEP>;
     AMGT_CUDA(dyn_smem(kern, sm));
     kern<<<(unsigned)ceil_div(n * 32, 256), 256, sm, s>>>(n, rows, c, nnz_row, cptr, cidx, cmap, hr);
