@@ -1098,9 +1098,20 @@ __global__ void __launch_bounds__(GD_CNT_THREADS) k_gdense_count(int64_t nd, con
         const uint32_t* bm = gbm + li * W;
         uint32_t* pre = gpre + li * W;
         uint32_t run = 0;
-        for (int64_t base = 0; base < W; base += GD_CNT_THREADS) {
-            const int64_t i = base + tid;
-            const uint32_t v = i < W ? (uint32_t)__popc(bm[i]) : 0u;
+        // four consecutive words per thread per round (one 16-B load when W is a multiple of 4)
+        for (int64_t base = 0; base < W; base += 4 * GD_CNT_THREADS) {
+            const int64_t i = base + 4 * tid;
+            uint32_t wv[4];
+            if ((W & 3) == 0 && i + 3 < W) {
+                const uint4 q4 = *reinterpret_cast<const uint4*>(bm + i);
+                wv[0] = q4.x; wv[1] = q4.y; wv[2] = q4.z; wv[3] = q4.w;
+            } else {
+#pragma unroll
+                for (int u = 0; u < 4; ++u) wv[u] = i + u < W ? bm[i + u] : 0u;
+            }
+            uint32_t pc[4], v = 0;
+#pragma unroll
+            for (int u = 0; u < 4; ++u) { pc[u] = (uint32_t)__popc(wv[u]); v += pc[u]; }
             uint32_t incl = v;
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
@@ -1121,7 +1132,21 @@ __global__ void __launch_bounds__(GD_CNT_THREADS) k_gdense_count(int64_t nd, con
                 if (lane == NW - 1) sh[NW] = xi;
             }
             __syncthreads();
-            if (i < W) pre[i] = run + sh[w] + incl - v;
+            uint32_t ex = run + sh[w] + incl - v;
+            if ((W & 3) == 0 && i + 3 < W) {
+                uint4 o;
+                o.x = ex; ex += pc[0];
+                o.y = ex; ex += pc[1];
+                o.z = ex; ex += pc[2];
+                o.w = ex;
+                *reinterpret_cast<uint4*>(pre + i) = o;
+            } else {
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    if (i + u < W) pre[i + u] = ex;
+                    ex += pc[u];
+                }
+            }
             run += sh[NW];
             __syncthreads();
         }
@@ -1133,16 +1158,34 @@ __global__ void __launch_bounds__(GD_CNT_THREADS) k_gdense_count(int64_t nd, con
 __global__ void k_gdense_out(int64_t nd, const int32_t* __restrict__ rows, int64_t W, const uint32_t* __restrict__ gbm,
                              const uint32_t* __restrict__ gpre, const int64_t* __restrict__ cptr,
                              int32_t* __restrict__ cidx) {
+    // four consecutive words of one row per thread (W a multiple of 4), else one
     const int64_t n = nd * W;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        uint32_t bits = gbm[i];
-        if (!bits) continue;
-        const int64_t li = i / W, wd = i - li * W;
-        int64_t q = cptr[rows[li]] + gpre[i];
-        while (bits) {
-            const int b = __ffs(bits) - 1;
-            bits &= bits - 1;
-            cidx[q++] = (int32_t)(32 * wd + b);
+    const int V = (W & 3) == 0 ? 4 : 1;
+    for (int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * V; g < n;
+         g += (int64_t)gridDim.x * blockDim.x * V) {
+        uint32_t wv[4] = {0u, 0u, 0u, 0u}, pv[4] = {0u, 0u, 0u, 0u};
+        if (V == 4) {
+            const uint4 b4 = *reinterpret_cast<const uint4*>(gbm + g);
+            if ((b4.x | b4.y | b4.z | b4.w) == 0u) continue;
+            const uint4 p4 = *reinterpret_cast<const uint4*>(gpre + g);
+            wv[0] = b4.x; wv[1] = b4.y; wv[2] = b4.z; wv[3] = b4.w;
+            pv[0] = p4.x; pv[1] = p4.y; pv[2] = p4.z; pv[3] = p4.w;
+        } else {
+            wv[0] = gbm[g];
+            if (!wv[0]) continue;
+            pv[0] = gpre[g];
+        }
+        const int64_t li = g / W, wd0 = g - li * W;
+        const int64_t c0 = cptr[rows[li]];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            uint32_t bits = wv[u];
+            int64_t q = c0 + pv[u];
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                bits &= bits - 1;
+                cidx[q++] = (int32_t)(32 * (wd0 + u) + b);
+            }
         }
     }
 }
@@ -2777,7 +2820,7 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
             g.plan = false;
         }
     }
-    k_gdense_out<<<capped(ceil_div(nd * W, 256)), 256, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, cptr, cidx);
+    k_gdense_out<<<capped(ceil_div(nd * W, 1024)), 256, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, cptr, cidx);
     AMGT_LAUNCHED();
     k_gdense_pairs<2><<<pgrid, GD_CH, 0, s>>>(g.ioff.p + nd, g.item_row.p, g.ioff.p, rows, c, W, g.bm.p,
                                             nullptr, g.pre.p, cptr, reinterpret_cast<uint32_t*>(cmap), pr, nullptr);
