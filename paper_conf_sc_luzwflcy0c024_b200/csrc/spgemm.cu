@@ -453,12 +453,17 @@ __global__ void __launch_bounds__(256, 8) k_sym_warp(int64_t nrows, const int32_
         for (int u = 0; u < (S / 64 > 0 ? S / 64 : 1); ++u)
             if (sl[u] >= 0) keys[sl[u]] = rk[u];
         __syncwarp();
-        for (int64_t p = r0 + lane; p < r1; p += 32) {
-            const int h = hr.rec[p].x;
-            if (h < 0) continue;
-            const int64_t q = out + keys[h];
-            hr.rec[p].x = (int)q;
-            atomicAdd(hr.cnt + q, 1u);
+        for (int64_t pb = r0 + lane; pb < r1; pb += 4 * 32) {  // four records per lane in flight
+            int hv[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) hv[u] = pb + 32 * u < r1 ? reinterpret_cast<const int*>(hr.rec + pb + 32 * u)[0] : -1;
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                if (hv[u] < 0) continue;
+                const int64_t q = out + keys[hv[u]];
+                reinterpret_cast<int*>(hr.rec + pb + 32 * u)[0] = (int)q;
+                atomicAdd(hr.cnt + q, 1u);
+            }
         }
     }
 }
@@ -847,12 +852,18 @@ __global__ void __launch_bounds__(LOGS >= 12 ? 512 : 256, LOGS >= 12 ? 2 : 5) k_
             __syncthreads();
             if (r1 > r0) {  // the row's records get their C tiles
                 if (tid == 0) hr.rowf[I] = 1;
-                for (int64_t p = r0 + tid; p < r1; p += nt) {
-                    const int h = hr.rec[p].x;
-                    if (h < 0) continue;
-                    const int64_t q = out + keys[h];
-                    hr.rec[p].x = (int)q;
-                    atomicAdd(hr.cnt + q, 1u);
+                for (int64_t pb = r0 + tid; pb < r1; pb += 4 * (int64_t)nt) {  // four records per thread in flight
+                    int hv[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        hv[u] = pb + (int64_t)nt * u < r1 ? reinterpret_cast<const int*>(hr.rec + pb + (int64_t)nt * u)[0] : -1;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        if (hv[u] < 0) continue;
+                        const int64_t q = out + keys[hv[u]];
+                        reinterpret_cast<int*>(hr.rec + pb + (int64_t)nt * u)[0] = (int)q;
+                        atomicAdd(hr.cnt + q, 1u);
+                    }
                 }
                 __syncthreads();
             }
