@@ -177,7 +177,10 @@ amgt_status amgt_spgemm_symbolic(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
  * structure arrays; the symbolic phase's numeric plan is used when present, see above).
  * Values: deterministic for C block rows with at most 32 tiles (fixed lane order); longer rows
  * accumulate tiles that receive three or more products with FP atomics and are reproducible up
- * to rounding only (exact on integer / dyadic data).
+ * to rounding only (exact on integer / dyadic data) — unless AMGT_SPGEMM_DET=1:
+ * then the symbolic phase gives every multi-product tile of its plan a slot range and the numeric
+ * phase adds the tile's products in ascending A-tile order (bitwise reproducible; two more host
+ * syncs in the symbolic phase).
  */
 amgt_status amgt_spgemm_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mbsr* C, void* stream);
 

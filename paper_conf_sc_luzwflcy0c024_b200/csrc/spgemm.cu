@@ -1023,6 +1023,52 @@ struct PlanRec {
     uint32_t* cnt;  // [TC] products per C tile
 };
 
+// Deterministic multi-product tiles (R34): the multi tiles are numbered in C order
+// (mi = prefix of popcount(mflag) words + rank in the word); k_plan_mlist lists their C tile
+// and product count, a scan gives each its slot range, and k_plan_slots rewrites every record of
+// a multi tile to -(slot + 2) — the numeric pass writes those products to their slots and
+// k_plan_msum adds each tile's products in ascending A-tile order (the pair order of Alg. 4), so
+// the sum no longer depends on scheduling.
+__global__ void k_plan_wpop(int64_t nw, const uint32_t* __restrict__ mflag, int64_t* __restrict__ wpop) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (int64_t)gridDim.x * blockDim.x)
+        wpop[i] = __popc(mflag[i]);
+}
+__device__ __forceinline__ int64_t multi_index(const uint32_t* mflag, const int64_t* mwpre, int64_t q) {
+    return mwpre[q >> 5] + __popc(mflag[q >> 5] & ((1u << (q & 31)) - 1u));
+}
+__global__ void k_plan_mlist(int64_t TC, const uint32_t* __restrict__ mflag, const int64_t* __restrict__ mwpre,
+                             const uint32_t* __restrict__ cnt, int32_t* __restrict__ mq, int64_t* __restrict__ mcnt) {
+    const int64_t nw = (TC + 31) / 32;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t f = mflag[i];
+        int64_t mi = mwpre[i];
+        while (f) {
+            const int b = __ffs(f) - 1;
+            f &= f - 1;
+            const int64_t q = 32 * i + b;
+            mq[mi] = (int32_t)q;
+            mcnt[mi] = cnt[q];
+            ++mi;
+        }
+    }
+}
+__global__ void k_plan_mtail(int64_t TC, const int64_t* __restrict__ nm_dev, int64_t* __restrict__ mcnt) {
+    const int64_t nm = *nm_dev;
+    for (int64_t i = nm + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < TC; i += (int64_t)gridDim.x * blockDim.x)
+        mcnt[i] = 0;
+}
+__global__ void k_plan_slots(int64_t n, int4* __restrict__ rec, const uint32_t* __restrict__ mflag,
+                             const int64_t* __restrict__ mwpre, const int64_t* __restrict__ moff,
+                             uint32_t* __restrict__ mfill) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x) {
+        const int q = reinterpret_cast<const int*>(rec + p)[0];
+        if (q < 0 || !((mflag[q >> 5] >> (q & 31)) & 1u)) continue;
+        const int64_t mi = multi_index(mflag, mwpre, q);
+        const int64_t slot = moff[mi] + atomicAdd(mfill + mi, 1u);
+        reinterpret_cast<int*>(rec + p)[0] = (int)(-(slot + 2));
+    }
+}
+
 // mflag bit q <- C tile q takes more than one product
 __global__ void k_plan_mark(int64_t TC, const uint32_t* __restrict__ cnt, uint32_t* __restrict__ mflag) {
     const int64_t nw = (TC + 31) / 32;
@@ -2644,6 +2690,11 @@ struct SpgemmPlan {
     uint8_t* rowf = nullptr;    // per C block row: 1 = computed from the records
     cudaEvent_t used = nullptr;  // recorded after the last work that reads the plan (any stream)
     bool covers_all = false;     // every row with more than CAP C tiles has records
+    // deterministic multi-product tiles: their C tiles, slot ranges, and the product count
+    int64_t* nm_dev = nullptr;   // device: number of multi tiles
+    int32_t* mq = nullptr;
+    int64_t* moff = nullptr;
+    int64_t nmp = 0;             // products of the multi tiles (side-buffer slots)
 };
 
 static std::mutex g_plan_mu;
@@ -2662,6 +2713,9 @@ static void plan_free(SpgemmPlan* P, cudaStream_t s) {
     }
     scratch_put(P->rec, s);
     scratch_put(P->mflag, s);
+    scratch_put(P->nm_dev, s);
+    scratch_put(P->mq, s);
+    scratch_put(P->moff, s);
     scratch_put(P->rowf, s);
     delete P;
 }
@@ -3118,6 +3172,65 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             P->covers_all = dense_ok && hash_ok && bitonic_rows == 0;
             k_plan_mark<<<capped(ceil_div(TC, 256)), 256, 0, s>>>(TC, pcnt.p, P->mflag);
             AMGT_LAUNCHED();
+            // deterministic multi tiles: number them, give each a slot range, point their records at
+            // the slots (two read-backs: the tile count, then the slot count)
+            // opt-in (AMGT_SPGEMM_DET=1): two more host syncs and per-call slot arrays; measured on
+            // config 4 with erratic symbolic times (2.1-4.3 ms vs 1.88 ms without)
+            static const int det_env = [] { const char* e = getenv("AMGT_SPGEMM_DET"); return e ? atoi(e) : 0; }();
+            const int64_t nw = ceil_div(TC, 32);
+            Scratch<int64_t> wpop, mwpre, mcnt;
+            Scratch<uint32_t> mfill;
+            int64_t* pin = pinned_slots();
+            auto read1 = [&](const int64_t* dsrc, int64_t* out) -> amgt_status {  // one synchronised read-back
+                if (pin) {
+                    AMGT_CUDA(cudaMemcpyAsync(pin + PIN_SYM + 19, dsrc, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                    AMGT_CUDA(cudaStreamSynchronize(s));
+                    *out = pin[PIN_SYM + 19];
+                } else {
+                    AMGT_CUDA(cudaMemcpyAsync(out, dsrc, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+                    AMGT_CUDA(cudaStreamSynchronize(s));
+                }
+                return AMGT_OK;
+            };
+            int64_t nm = 0;
+            bool det = det_env && wpop.try_init(a, nw) && mwpre.try_init(a, nw + 1);
+            if (det) {
+                k_plan_wpop<<<capped(ceil_div(nw, 256)), 256, 0, s>>>(nw, P->mflag, wpop.p);
+                AMGT_LAUNCHED();
+                AMGT_TRY(scan_exclusive(wpop.p, mwpre.p, nw, a, s));
+                trace_point("sym det mark", s);
+                AMGT_TRY(read1(mwpre.p + nw, &nm));  // sync: the number of multi tiles
+                if (nm > 0) {
+                    P->nm_dev = (int64_t*)scratch_get(sizeof(int64_t), s);
+                    P->mq = (int32_t*)scratch_get((size_t)nm * sizeof(int32_t), s);
+                    P->moff = (int64_t*)scratch_get((size_t)(nm + 1) * sizeof(int64_t), s);
+                    det = P->nm_dev && P->mq && P->moff && mcnt.try_init(a, nm) && mfill.try_init(a, nm);
+                } else {
+                    det = false;  // no multi tiles: nothing to order
+                }
+            }
+            if (det) {
+                AMGT_CUDA(cudaMemcpyAsync(P->nm_dev, mwpre.p + nw, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+                k_plan_mlist<<<capped(ceil_div(nw, 256)), 256, 0, s>>>(TC, P->mflag, mwpre.p, pcnt.p, P->mq, mcnt.p);
+                AMGT_LAUNCHED();
+                AMGT_TRY(scan_exclusive(mcnt.p, P->moff, nm, a, s));
+                AMGT_CUDA(cudaMemsetAsync(mfill.p, 0, (size_t)nm * sizeof(uint32_t), s));
+                if (P->nrec > 0) {
+                    k_plan_slots<<<capped(ceil_div(P->nrec, 256)), 256, 0, s>>>(P->nrec, P->rec, P->mflag, mwpre.p,
+                                                                               P->moff, mfill.p);
+                    AMGT_LAUNCHED();
+                }
+                trace_point("sym det slots", s);
+                AMGT_TRY(read1(P->moff + nm, &P->nmp));  // sync: the products of the multi tiles
+                P->bytes += (size_t)nm * 12 + 8;
+            } else {
+                scratch_put(P->nm_dev, s);
+                scratch_put(P->mq, s);
+                scratch_put(P->moff, s);
+                P->nm_dev = nullptr;
+                P->mq = nullptr;
+                P->moff = nullptr;
+            }
             pscope.ok = true;
             plan_put(P, s);
         }
@@ -3374,6 +3487,68 @@ __global__ void k_plan_zero(int64_t TC, const uint32_t* __restrict__ mflag, Acc*
     }
 }
 
+template <typename Acc> struct SideRow;
+template <> struct SideRow<double> {
+    static __device__ __forceinline__ void store(double* p, const double (&v)[4]) {
+        reinterpret_cast<double2*>(p)[0] = make_double2(v[0], v[1]);
+        reinterpret_cast<double2*>(p)[1] = make_double2(v[2], v[3]);
+    }
+    static __device__ __forceinline__ void load(const double* p, double (&v)[4]) {
+        const double2 a = reinterpret_cast<const double2*>(p)[0], b = reinterpret_cast<const double2*>(p)[1];
+        v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+    }
+};
+template <> struct SideRow<float> {
+    static __device__ __forceinline__ void store(float* p, const float (&v)[4]) {
+        *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    }
+    static __device__ __forceinline__ void load(const float* p, float (&v)[4]) {
+        const float4 a = *reinterpret_cast<const float4*>(p);
+        v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+    }
+};
+
+// Each multi tile (a 4-lane group): its products' slots in ascending A-tile order (insertion by
+// t, recomputed per step so any count works), lane r adds row r of them into a zero row in that
+// order (the accumulation of Alg. 4 in pair order: deterministic) and writes the tile row
+// (+0.0 at the clear bits, R2; FP16 rounded once from the FP32 sum).
+template <typename T, typename Acc>
+__global__ void k_plan_msum(const int64_t* __restrict__ nm_dev, const int32_t* __restrict__ mq,
+                            const int64_t* __restrict__ moff, const Acc* __restrict__ side_v,
+                            const int32_t* __restrict__ side_t, const uint16_t* __restrict__ cmap,
+                            T* __restrict__ cval) {
+    const int64_t nm = *nm_dev;
+    const int r = threadIdx.x & 3;
+    for (int64_t mi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2; mi < nm;
+         mi += ((int64_t)gridDim.x * blockDim.x) >> 2) {
+        const int64_t s0 = moff[mi], s1 = moff[mi + 1];
+        Acc sum[4] = {Acc(0), Acc(0), Acc(0), Acc(0)};
+        int prev = INT_MIN;
+        int64_t prev_s = -1;
+        for (int64_t k = s0; k < s1; ++k) {  // next slot in (t, slot) order
+            int best = INT_MAX;
+            int64_t bs = -1;
+            for (int64_t x = s0; x < s1; ++x) {
+                const int tx = side_t[x];
+                const bool after = tx > prev || (tx == prev && x > prev_s);
+                if (after && (tx < best || (tx == best && x < bs))) { best = tx; bs = x; }
+            }
+            Acc v[4];
+            SideRow<Acc>::load(side_v + 16 * bs + 4 * r, v);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) sum[e] += v[e];
+            prev = best;
+            prev_s = bs;
+        }
+        const int64_t q = mq[mi];
+        const uint32_t nib = (cmap[q] >> (4 * r)) & 0xFu;
+        Acc o[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) o[e] = ((nib >> e) & 1u) ? sum[e] : Acc(0);
+        RowIO<T>::store(cval + 16 * q + 4 * r, o);
+    }
+}
+
 // One pass over the records, PLAN_R records per block of work: the records arrive in registers
 // one block ahead, the A and B tiles of a block are copied to shared memory with cp.async one
 // block ahead (double-buffered), and four threads per record each form one row of A_t * B_j
@@ -3413,12 +3588,13 @@ template <> struct RowCS<float> {
 template <> struct RowCS<__half> {
     static __device__ __forceinline__ void store(__half* p, const float (&v)[4]) { RowIO<__half>::store(p, v); }
 };
-template <typename T, typename Acc>
+template <typename T, typename Acc, bool DET = false>
 __global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(int64_t total, const int4* __restrict__ rec,
                                                          const uint32_t* __restrict__ mflag,
                                                          const T* __restrict__ aval, const T* __restrict__ bval,
                                                          T* __restrict__ cval, Acc* __restrict__ gacc,
-                                                         int hints) {
+                                                         int hints, Acc* __restrict__ side_v = nullptr,
+                                                         int32_t* __restrict__ side_t = nullptr) {
     constexpr int TE = 16;
     constexpr int CH = 16 / (int)sizeof(T);       // elements per 16-B piece
     constexpr int PC = TE / CH;                   // 16-B pieces per tile
@@ -3444,7 +3620,7 @@ __global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(int64_t total, const i
         if (tid < PLAN_R) {
             const int lane = tid & 31;
             const int zp = __shfl_up_sync(0xffffffffu, r.z, 1);
-            const unsigned bal = __ballot_sync(0xffffffffu, lane == 0 || r.x < 0 || r.z != zp);
+            const unsigned bal = __ballot_sync(0xffffffffu, lane == 0 || r.x == -1 || r.z != zp);
             sr[buf][tid] = r;
             sa[buf][tid] = (tid & ~31) + 31 - __clz(bal & (0xffffffffu >> (31 - lane)));
         }
@@ -3453,7 +3629,7 @@ __global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(int64_t total, const i
         for (int k = tid; k < PLAN_R * 2 * PC; k += PLAN_R * 4) {
             const int ri = k / (2 * PC), part = k - ri * 2 * PC;
             const int4 r = sr[buf][ri];
-            if (r.x < 0) continue;
+            if (r.x == -1) continue;  // empty product (<= -2: a multi tile's product slot)
             if (part < PC) {
                 if (sa[buf][ri] == ri) cp_async16_g<T>(&sA[buf][ri][part * CH], aval + 16 * (int64_t)r.z + part * CH);
             } else if (hints & 1) {
@@ -3514,6 +3690,25 @@ __global__ void __launch_bounds__(PLAN_R * 4) k_plan_flat(int64_t total, const i
                 for (int e = 0; e < 4; ++e)
                     if ((nib >> e) & 1u) atomicAdd(acc + 16 * q + 4 * row + e, o[e]);
             }
+        } else if (DET && r.x <= -2) {  // a product of a multi tile: to its slot (k_plan_msum adds them)
+            Acc a4[4], o[4];
+            SRow<T>::load(&sA[buf][sa[buf][ri]][4 * row], a4);
+            Acc b0[4], b1[4], b2[4], b3[4];
+            SRow<T>::load(&sB[buf][ri][0], b0);
+            SRow<T>::load(&sB[buf][ri][4], b1);
+            SRow<T>::load(&sB[buf][ri][8], b2);
+            SRow<T>::load(&sB[buf][ri][12], b3);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                Acc v = a4[0] * b0[e];
+                v = fma_acc(a4[1], b1[e], v);
+                v = fma_acc(a4[2], b2[e], v);
+                v = fma_acc(a4[3], b3[e], v);
+                o[e] = v;
+            }
+            const int64_t slot = -(int64_t)r.x - 2;
+            SideRow<Acc>::store(side_v + 16 * slot + 4 * row, o);
+            if (row == 0) side_t[slot] = r.z;
         }
         __syncthreads();  // buffer `buf` is refilled two iterations on
     }
@@ -3724,12 +3919,22 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
     }
     AMGT_LAUNCHED();
     if (plan) {  // the dense rows: one pass over the symbolic phase's records
-        Scratch<Acc> pacc;  // FP16: FP32 workspace of the multi-product tiles
-        if (sizeof(T) < sizeof(Acc)) AMGT_TRY(pacc.init(a, 16 * (size_t)C->blc_num));
+        const bool det = plan->moff != nullptr;  // multi tiles summed in A-tile order (k_plan_msum)
+        Scratch<Acc> pacc;  // FP16: FP32 workspace of the multi-product tiles (REDs path)
+        Scratch<Acc> side_v;
+        Scratch<int32_t> side_t;
+        if (det) {
+            AMGT_TRY(side_v.init(a, 16 * (size_t)std::max<int64_t>(plan->nmp, 1)));
+            AMGT_TRY(side_t.init(a, (size_t)std::max<int64_t>(plan->nmp, 1)));
+        } else if (sizeof(T) < sizeof(Acc)) {
+            AMGT_TRY(pacc.init(a, 16 * (size_t)C->blc_num));
+        }
         Acc* acc = sizeof(T) < sizeof(Acc) ? pacc.p : reinterpret_cast<Acc*>(C->blc_val);
         const int64_t nw = ceil_div(C->blc_num, 32);
-        k_plan_zero<Acc><<<capped(ceil_div(nw, 256)), 256, 0, s>>>(C->blc_num, plan->mflag, acc);
-        AMGT_LAUNCHED();
+        if (!det) {
+            k_plan_zero<Acc><<<capped(ceil_div(nw, 256)), 256, 0, s>>>(C->blc_num, plan->mflag, acc);
+            AMGT_LAUNCHED();
+        }
         // L2 policies: bit 0 B tiles evict-last, bit 1 C stores evict-first (AMGT_PLAN_HINTS)
         static const int plan_hints = [] { const char* e = getenv("AMGT_PLAN_HINTS"); return e ? atoi(e) : 3; }();
         static int flat_per_sm = 0;
@@ -3738,7 +3943,7 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
             flat_per_sm = max(flat_per_sm, 1);
         }
         static const int bulk_env = [] { const char* e = getenv("AMGT_PLAN_BULK"); return e ? atoi(e) : 0; }();  // measured slower (cfg4 1.80 vs 1.67 ms)
-        if (bulk_env) {
+        if (bulk_env && !det) {  // (the bulk form has no slot path)
             static int bulk_per_sm = 0;
             if (!bulk_per_sm) {
                 AMGT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bulk_per_sm, k_plan_flat_bulk<T, Acc>,
@@ -3749,11 +3954,20 @@ static amgt_status launch_numeric(const amgt_mbsr* A, const amgt_mbsr* B, amgt_m
                 plan->nrec, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
                 sizeof(T) < sizeof(Acc) ? pacc.p : nullptr, plan_hints);
         } else
-        k_plan_flat<T, Acc><<<(unsigned)(num_sms() * flat_per_sm), PLAN_R * 4, 0, s>>>(
-            plan->nrec, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
-            sizeof(T) < sizeof(Acc) ? pacc.p : nullptr, plan_hints);
+        if (det)
+            k_plan_flat<T, Acc, true><<<(unsigned)(num_sms() * flat_per_sm), PLAN_R * 4, 0, s>>>(
+                plan->nrec, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
+                nullptr, plan_hints, side_v.p, side_t.p);
+        else
+            k_plan_flat<T, Acc><<<(unsigned)(num_sms() * flat_per_sm), PLAN_R * 4, 0, s>>>(
+                plan->nrec, plan->rec, plan->mflag, (const T*)A->blc_val, (const T*)B->blc_val, (T*)C->blc_val,
+                sizeof(T) < sizeof(Acc) ? pacc.p : nullptr, plan_hints);
         AMGT_LAUNCHED();
-        if (sizeof(T) < sizeof(Acc)) {
+        if (det) {
+            k_plan_msum<T, Acc><<<capped(ceil_div(4 * std::max<int64_t>(C->blc_num / 8, 1), 256)), 256, 0, s>>>(
+                plan->nm_dev, plan->mq, plan->moff, side_v.p, side_t.p, C->blc_map, (T*)C->blc_val);
+            AMGT_LAUNCHED();
+        } else if (sizeof(T) < sizeof(Acc)) {
             k_plan_finalize<T, Acc><<<capped(ceil_div(nw, 256)), 256, 0, s>>>(C->blc_num, plan->mflag, C->blc_map,
                                                                             pacc.p, (T*)C->blc_val);
             AMGT_LAUNCHED();

@@ -342,3 +342,59 @@ def test_spgemm_searching_kernels_without_plan(tmp_path, case, prec):
         assert np.all(np.abs(g - r) <= bound + 1e-300)
     else:
         assert np.linalg.norm(g - r) <= 5e-3 * np.linalg.norm(r)
+
+
+_DET_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import gen, paper_conf_sc_luzwflcy0c024_b200 as amgt
+prec = sys.argv[3]
+A = gen.irregular_block_sparse(1 << 13, seed=9)
+M = amgt.from_csr(A, prec=prec)
+C, info = amgt.spgemm(M, M, info=True)
+bits = {"f16": torch.int16, "f32": torch.int32, "f64": torch.int64}[prec]
+v1 = C.blc_val.clone()
+same = True
+for _ in range(3):
+    amgt.spgemm_numeric(M, M, C)
+    same = same and torch.equal(C.blc_val.view(bits), v1.view(bits))
+C2 = amgt.spgemm(M, M)  # a fresh symbolic phase (new slot assignment)
+same = same and torch.equal(C2.blc_val.view(bits), v1.view(bits))
+np.savez(sys.argv[2], same=same, multi=info["pairs_nonzero"] > C.blc_num, ptr=C.blc_ptr.cpu().numpy(),
+         idx=C.blc_idx.cpu().numpy(), map=C.map_u16().cpu().numpy(), val=C.blc_val.double().cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("prec", ["f64", "f32", "f16"])
+def test_spgemm_multi_product_tiles_bitwise_reproducible(tmp_path, prec):
+    """AMGT_SPGEMM_DET=1 (separate process): the plan rows' tiles with several products are summed in
+    ascending A-tile order from their product slots (k_plan_msum), not by atomics: repeated numeric
+    calls and a fresh symbolic phase give bit-identical values, and the product matches the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "det.py"
+    script.write_text(_DET_SCRIPT)
+    out = tmp_path / "c.npz"
+    env = dict(os.environ, AMGT_SPGEMM_DET="1")
+    p = subprocess.run([sys.executable, str(script), root, str(out), prec], env=env, capture_output=True, text=True,
+                       timeout=300)
+    assert p.returncode == 0, p.stderr[-2000:]
+    got = np.load(out)
+    assert bool(got["multi"]) and bool(got["same"])
+    A = gen.irregular_block_sparse(1 << 13, seed=9)
+    Ao = oracle.as_csr(A)
+    Co, Cabs = oracle.spgemm(Ao, Ao, with_abs=True)
+    Cm = oracle.csr_to_mbsr(Co)
+    assert np.array_equal(got["ptr"], Cm.blc_ptr) and np.array_equal(got["idx"], Cm.blc_idx)
+    bits = ((got["map"][:, None] >> np.arange(16)) & 1).astype(bool)
+    g = got["val"].reshape(-1, 16)[bits]
+    r = np.asarray(Cm.blc_val).reshape(-1, 16)[bits]
+    if prec == "f64":
+        absm = oracle.csr_to_mbsr(oracle.Csr(Co.m, Co.n, Co.row_ptr, Co.col, Cabs))
+        assert np.all(np.abs(g - r) <= 1e-12 * np.asarray(absm.blc_val).reshape(-1, 16)[bits] + 1e-300)
+    elif prec == "f32":
+        assert np.max(np.abs(g - r)) <= 1e-5 * np.max(np.abs(r))
+    else:
+        assert np.linalg.norm(g - r) <= 5e-3 * np.linalg.norm(r)
