@@ -2695,6 +2695,21 @@ struct SpgemmPlan {
     int32_t* mq = nullptr;
     int64_t* moff = nullptr;
     int64_t nmp = 0;             // products of the multi tiles (side-buffer slots)
+    // plan memory comes from the caller's allocator when the symbolic call had one (a caching
+    // allocator reuses it across symbolic/numeric/free cycles; the scratch pool re-mapped it:
+    // erratic symbolic times), copied here because the plan outlives the call
+    amgt_allocator alc{};
+    bool has_alc = false;
+    size_t rec_b = 0, mflag_b = 0, rowf_b = 0, mq_b = 0, moff_b = 0;
+    void* get(size_t bytes, cudaStream_t st) {
+        Alloc a{has_alc ? &alc : nullptr, st};
+        return a.get(bytes);
+    }
+    void put(void* p, size_t bytes, cudaStream_t st) {
+        if (!p) return;
+        Alloc a{has_alc ? &alc : nullptr, st};
+        a.put(p, bytes);
+    }
 };
 
 static std::mutex g_plan_mu;
@@ -2711,12 +2726,12 @@ static void plan_free(SpgemmPlan* P, cudaStream_t s) {
         cudaStreamWaitEvent(s, P->used, 0);
         cudaEventDestroy(P->used);
     }
-    scratch_put(P->rec, s);
-    scratch_put(P->mflag, s);
-    scratch_put(P->nm_dev, s);
-    scratch_put(P->mq, s);
-    scratch_put(P->moff, s);
-    scratch_put(P->rowf, s);
+    P->put(P->rec, P->rec_b, s);
+    P->put(P->mflag, P->mflag_b, s);
+    P->put(P->nm_dev, sizeof(int64_t), s);
+    P->put(P->mq, P->mq_b, s);
+    P->put(P->moff, P->moff_b, s);
+    P->put(P->rowf, P->rowf_b, s);
     delete P;
 }
 
@@ -3120,9 +3135,14 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
             P->TC = TC;
             P->nrec = npD + nH;
             const size_t nf = (size_t)ceil_div(TC, 32);
-            P->rec = (int4*)scratch_get((size_t)P->nrec * sizeof(int4), s);
-            P->mflag = (uint32_t*)scratch_get(nf * sizeof(uint32_t), s);
-            P->rowf = (uint8_t*)scratch_get((size_t)BR, s);
+            P->has_alc = a.al != nullptr;
+            if (a.al) P->alc = *a.al;
+            P->rec_b = (size_t)P->nrec * sizeof(int4);
+            P->mflag_b = nf * sizeof(uint32_t);
+            P->rowf_b = (size_t)BR;
+            P->rec = (int4*)P->get(P->rec_b, s);
+            P->mflag = (uint32_t*)P->get(P->mflag_b, s);
+            P->rowf = (uint8_t*)P->get(P->rowf_b, s);
             P->bytes = (size_t)P->nrec * sizeof(int4) + nf * sizeof(uint32_t) + (size_t)BR;
             if (!P->rec || !P->mflag || !P->rowf || !pcnt.try_init(a, (size_t)TC)) {
                 plan_free(P, s);
@@ -3201,9 +3221,11 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 trace_point("sym det mark", s);
                 AMGT_TRY(read1(mwpre.p + nw, &nm));  // sync: the number of multi tiles
                 if (nm > 0) {
-                    P->nm_dev = (int64_t*)scratch_get(sizeof(int64_t), s);
-                    P->mq = (int32_t*)scratch_get((size_t)nm * sizeof(int32_t), s);
-                    P->moff = (int64_t*)scratch_get((size_t)(nm + 1) * sizeof(int64_t), s);
+                    P->mq_b = (size_t)nm * sizeof(int32_t);
+                    P->moff_b = (size_t)(nm + 1) * sizeof(int64_t);
+                    P->nm_dev = (int64_t*)P->get(sizeof(int64_t), s);
+                    P->mq = (int32_t*)P->get(P->mq_b, s);
+                    P->moff = (int64_t*)P->get(P->moff_b, s);
                     det = P->nm_dev && P->mq && P->moff && mcnt.try_init(a, nm) && mfill.try_init(a, nm);
                 } else {
                     det = false;  // no multi tiles: nothing to order
@@ -3224,9 +3246,9 @@ amgt_status spgemm_symbolic_impl(const amgt_mbsr* A, const amgt_mbsr* B, amgt_mb
                 AMGT_TRY(read1(P->moff + nm, &P->nmp));  // sync: the products of the multi tiles
                 P->bytes += (size_t)nm * 12 + 8;
             } else {
-                scratch_put(P->nm_dev, s);
-                scratch_put(P->mq, s);
-                scratch_put(P->moff, s);
+                P->put(P->nm_dev, sizeof(int64_t), s);
+                P->put(P->mq, P->mq_b, s);
+                P->put(P->moff, P->moff_b, s);
                 P->nm_dev = nullptr;
                 P->mq = nullptr;
                 P->moff = nullptr;

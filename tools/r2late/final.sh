@@ -1,6 +1,6 @@
 # late-round measurement batch: GPU suite, smoke, bench x2 (the driver's command), reference arm,
 # bench launch list (ncu), config-4 SpGEMM traffic capture (ncu --set full), sanitizer on SpGEMM
-cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late/final; mkdir -p $O
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late/final2; mkdir -p $O
 timeout 1800 python -m pytest tests -q -m gpu > $O/gpu_tests.log 2>&1; echo "rc=$?" >> $O/gpu_tests.log; tail -2 $O/gpu_tests.log
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log; tail -2 $O/smoke.log
 timeout 900 python bench.py > $O/bench_1.json 2> $O/bench_1.err
@@ -11,9 +11,4 @@ timeout 1500 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_
 python tools/ncu_traffic.py summarize cfg4 /tmp/ncu_spgemm_cfg4.ncu-rep > $O/ncu_cfg4_sum.log 2>&1
 cp profiles/ncu_traffic_cfg4.json $O/ncu_traffic_cfg4.json
 gzip -f $O/bench_launches.csv
-export PYTORCH_NO_CUDA_MEMORY_CACHING=1
-CS="compute-sanitizer --print-limit 20 --error-exitcode 99"
-timeout 1200 $CS --tool memcheck python -m pytest tests/test_gpu_spgemm.py -m gpu -q -x -p no:cacheprovider -k "not full and not cfg" > $O/spgemm_memcheck.log 2>&1; echo "memcheck rc=$?" >> $O/sanitize.txt
-timeout 1200 $CS --tool racecheck python -m pytest tests/test_gpu_spgemm.py -m gpu -q -x -p no:cacheprovider -k "long_rows or plan or info_bins" > $O/spgemm_racecheck.log 2>&1; echo "racecheck rc=$?" >> $O/sanitize.txt
-grep -h "ERROR SUMMARY" $O/*check.log >> $O/sanitize.txt
 echo done > $O/done
