@@ -11,15 +11,19 @@
 //   step 2        insert again, OR the bitmaps (R15), compress, sort ascending (Alg. 3 lines
 //                 13-14) -> blc_idxC, blc_mapC: k_sym_flat<2> + the per-bin kernels.
 //   numeric       rows by C-row length (<= 8 C tiles: staged 4-lane-group kernel; 9-32: warp
-//                 per row; 33-512; > 512: two passes).  A tiles with POPCOUNT >= threshold go
-//                 to the tensor-core route (DMMA m8n8k4: fragA = [A;A], fragB = [Bj|Bj'],
-//                 keep the two diagonal quadrants, L157-171); the others to CUDA cores
-//                 (L173).  Deterministic for rows with <= 32 C tiles.
+//                 per row; longer rows: one streaming pass over the records step 2 left —
+//                 the numeric plan, DESIGN R34 — or, without records, 33-512 warp / > 512
+//                 two-pass kernels).  A tiles with POPCOUNT >= threshold go to the tensor-core
+//                 route (DMMA m8n8k4: fragA = [A;A], fragB = [Bj|Bj'], keep the two diagonal
+//                 quadrants, L157-171); the others to CUDA cores (L173).  Deterministic for rows
+//                 with <= 32 C tiles (all rows with AMGT_SPGEMM_DET=1).
 //
 // Hash tables (R8): power-of-two, >= 2x the bin's Cub upper bound, multiplicative hash,
-// linear probing.  Bins 0-1: one warp per row, table per warp; bins 2-6: one block per
-// row, table per block; bin 7 (Cub >= 8192): dense bitmap over B's tile columns
-// (shared memory when it fits, else a per-block global slice) — sorted by construction.
+// linear probing.  Bins 0-1: one warp per row, table per warp; bins 2-4: one block per row,
+// table per block, block radix sort; from the bin whose lower edge reaches W/8 words (W = B's
+// column words): dense bitmaps over B's tile columns — per row in global memory, the row spread
+// over (row, 256-tile) work items (k_gdense_*; or k_sym_dense, one CTA per row) — sorted by
+// construction.
 #include <algorithm>
 #include <cmath>
 #include <climits>
@@ -360,14 +364,6 @@ struct HRec {
     uint32_t* cnt;
     uint8_t* rowf;
 };
-__device__ __forceinline__ int lower_pos(const int* keys, int n, int J) {  // keys ascending, J present
-    int lo = 0, hi = n - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (keys[mid] < J) lo = mid + 1; else hi = mid;
-    }
-    return lo;
-}
 
 // ---------------------------------------------------------------- step kernels: warp bins
 // LOGS = log2(table slots per warp).  STEP 1: count -> nnz_row[I].  STEP 2: write sorted
@@ -1052,11 +1048,6 @@ __global__ void k_plan_mlist(int64_t TC, const uint32_t* __restrict__ mflag, con
         }
     }
 }
-__global__ void k_plan_mtail(int64_t TC, const int64_t* __restrict__ nm_dev, int64_t* __restrict__ mcnt) {
-    const int64_t nm = *nm_dev;
-    for (int64_t i = nm + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < TC; i += (int64_t)gridDim.x * blockDim.x)
-        mcnt[i] = 0;
-}
 __global__ void k_plan_slots(int64_t n, int4* __restrict__ rec, const uint32_t* __restrict__ mflag,
                              const int64_t* __restrict__ mwpre, const int64_t* __restrict__ moff,
                              uint32_t* __restrict__ mfill) {
@@ -1085,7 +1076,6 @@ __global__ void __launch_bounds__(GD_CH) k_gdense_pairs(const int64_t* __restric
                                                       const int32_t* __restrict__ item_row,
                                                       const int64_t* __restrict__ ioff, const int32_t* __restrict__ rows,
                                                       SymCtx c, int64_t W, uint32_t* __restrict__ gbm,
-                                                      uint32_t* __restrict__ gbm2,
                                                       const uint32_t* __restrict__ gpre, const int64_t* __restrict__ cptr,
                                                       uint32_t* __restrict__ cmap32, PlanRec pr,
                                                       unsigned long long* __restrict__ npairs) {
@@ -2857,8 +2847,7 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
         k_gdense_item_rows<<<capped(nd), 256, 0, s>>>(nd, g.ioff.p, g.item_row.p);
         AMGT_LAUNCHED();
         k_gdense_pairs<1><<<pgrid, GD_CH, 0, s>>>(g.ioff.p + nd, g.item_row.p, g.ioff.p, rows, c, W, g.bm.p,
-                                                nullptr, nullptr, nullptr, nullptr, pr,
-                                                g.plan ? g.npairs_dev : nullptr);
+                                                nullptr, nullptr, nullptr, pr, g.plan ? g.npairs_dev : nullptr);
         AMGT_LAUNCHED();
         k_gdense_count<<<capped(nd), GD_CNT_THREADS, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, nnz_row);
         AMGT_LAUNCHED();
@@ -2903,7 +2892,7 @@ static amgt_status launch_gdense(int64_t nd, const int32_t* rows, const SymCtx& 
     k_gdense_out<<<capped(ceil_div(nd * W, 1024)), 256, 0, s>>>(nd, rows, W, g.bm.p, g.pre.p, cptr, cidx);
     AMGT_LAUNCHED();
     k_gdense_pairs<2><<<pgrid, GD_CH, 0, s>>>(g.ioff.p + nd, g.item_row.p, g.ioff.p, rows, c, W, g.bm.p,
-                                            nullptr, g.pre.p, cptr, reinterpret_cast<uint32_t*>(cmap), pr, nullptr);
+                                            g.pre.p, cptr, reinterpret_cast<uint32_t*>(cmap), pr, nullptr);
     AMGT_LAUNCHED();
     return AMGT_OK;
 }

@@ -1,6 +1,6 @@
 # late-round measurement batch: GPU suite, smoke, bench x2 (the driver's command), reference arm,
 # bench launch list (ncu), config-4 SpGEMM traffic capture (ncu --set full), sanitizer on SpGEMM
-cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late/final2; mkdir -p $O
+cd $GRAFT_REPO_ROOT; O=gpurun_out/r2late/final3; mkdir -p $O
 timeout 1800 python -m pytest tests -q -m gpu > $O/gpu_tests.log 2>&1; echo "rc=$?" >> $O/gpu_tests.log; tail -2 $O/gpu_tests.log
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log; tail -2 $O/smoke.log
 timeout 900 python bench.py > $O/bench_1.json 2> $O/bench_1.err
